@@ -1,0 +1,157 @@
+/*
+ * blas3.h -- C ABI of the B200-native (sm_100a) single-precision Level-3 BLAS
+ * derived from one tuned GEMM, after Cui, Wang, Xue, Yang, Feng, "Automatic
+ * Library Generation for BLAS3 on GPUs", IPDPS 2011
+ * (/root/reference/PAPER.md, cited P:<line>).
+ *
+ * The paper generates GEMM, SYMM, TRMM and TRSM variants from the GEMM-NN
+ * optimisation scheme (Fig. 3) by adaptors for Transpose,
+ * Symmetry, Triangular and Solver structure and states that
+ * matrices are column-major "to be consistent with BLAS3".
+ * The argument conventions below are therefore the reference-BLAS ones.
+ *
+ * Common rules for every entry point
+ * ----------------------------------
+ *  Layout     All matrices are fp32, column-major: X(i,j) = X[i + j*ldx].
+ *  Memory     A, B, C are DEVICE pointers (e.g. torch.Tensor.data_ptr() of a
+ *             tensor with strides (1, ld)) on the current CUDA device.
+ *             alpha/beta are host floats.  The caller owns every buffer; the
+ *             library keeps only caches (tensor-map descriptors) and uses
+ *             stream-ordered scratch (cudaMallocAsync) where a routine needs
+ *             it (STRMM, STRSM).
+ *  Streams    Work is enqueued on `stream` (NULL = legacy default stream) and
+ *             is asynchronous: no entry point synchronises the host.
+ *  Aliasing   C must not alias A or B (as in BLAS); B is overwritten in place
+ *             by STRMM/STRSM.
+ *  Sizes      int64_t (N = 32768 needs byte offsets beyond 2^32); otherwise
+ *             identical to the BLAS INTEGER arguments.
+ *  Characters case-insensitive; trans 'C' == 'T' for real data.
+ *  Return     0 on success.
+ *             > 0 : 1-based position of the first invalid argument in
+ *                   reference-BLAS XERBLA order, checked before anything is
+ *                   launched; nothing is modified.  (A NULL matrix pointer
+ *                   that would be referenced is reported by its position.)
+ *             < 0 : runtime failure: BLAS3_ERR_CUDA (a CUDA launch/runtime
+ *                   error), BLAS3_ERR_ARCH (current device is not sm_100),
+ *                   BLAS3_ERR_ALLOC (scratch allocation failed),
+ *                   BLAS3_ERR_TMA (tensor-map encoding failed).
+ *             The ABI never aborts and never throws.
+ *  Special    beta == 0: C is not read (NaN/Inf in C do not propagate).
+ *  values     alpha == 0: A and B are not read (C <- beta*C; B <- 0 for
+ *             STRMM/STRSM).  Entries outside the referenced triangle of a
+ *             symmetric/triangular A, and its diagonal when diag = 'U', are
+ *             never read (readings Q7, Q8, Q11, Q12).
+ *  Math       BLAS3_MATH_3XTF32 (default): tcgen05 tensor cores with a
+ *             3xTF32 split (hi*hi + hi*lo + lo*hi) and fp32 accumulation in
+ *             TMEM.  BLAS3_MATH_SIMT_FP32: exact-fp32 FFMA kernels.
+ *             Arguments that violate TMA's 16-byte rules (pointer not
+ *             16-byte aligned or ld % 4 != 0) run on the SIMT kernels in
+ *             either mode.
+ */
+#ifndef BLAS3_B200_H
+#define BLAS3_B200_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st *blas3_stream_t; /* identical to cudaStream_t */
+
+enum {
+    BLAS3_OK = 0,
+    BLAS3_ERR_CUDA = -1,
+    BLAS3_ERR_ARCH = -2,
+    BLAS3_ERR_ALLOC = -3,
+    BLAS3_ERR_TMA = -4
+};
+
+enum { BLAS3_MATH_3XTF32 = 0, BLAS3_MATH_SIMT_FP32 = 1 };
+
+/* SGEMM: C <- alpha*op(A)*op(B) + beta*C, op(X) = X or X^T.
+ * op(A) is m x k, op(B) is k x n, C is m x n.  Paper: GEMM-NN/-TN loop nests
+ * (P:77), Adaptor_Transpose.
+ * XERBLA: 1 transa, 2 transb, 3 m<0, 4 n<0, 5 k<0,
+ *         8 lda < max(1, transa=N ? m : k), 10 ldb < max(1, transb=N ? k : n),
+ *         13 ldc < max(1, m). */
+int blas3_sgemm(char transa, char transb, int64_t m, int64_t n, int64_t k,
+                float alpha, const float *A, int64_t lda, const float *B, int64_t ldb,
+                float beta, float *C, int64_t ldc, blas3_stream_t stream);
+
+/* SSYMM: side=L: C <- alpha*A*B + beta*C (A m x m);
+ *        side=R: C <- alpha*B*A + beta*C (A n x n).
+ * A symmetric; only its `uplo` triangle ("real area") is read, the "shadow
+ * area" is derived from it (Adaptor_Symmetry).  C, B are m x n.
+ * XERBLA: 1 side, 2 uplo, 3 m<0, 4 n<0, 7 lda < max(1, side=L ? m : n),
+ *         9 ldb < max(1, m), 12 ldc < max(1, m). */
+int blas3_ssymm(char side, char uplo, int64_t m, int64_t n, float alpha,
+                const float *A, int64_t lda, const float *B, int64_t ldb,
+                float beta, float *C, int64_t ldc, blas3_stream_t stream);
+
+/* SSYRK: trans=N: C <- alpha*A*A^T + beta*C (A n x k);
+ *        trans=T: C <- alpha*A^T*A + beta*C (A k x n).
+ * Only the `uplo` triangle of the n x n C is read and written; the other
+ * triangle is left bit-identical.  (Not evaluated in the paper; required by
+ * BASELINE.json's north star.)
+ * XERBLA: 1 uplo, 2 trans, 3 n<0, 4 k<0, 7 lda < max(1, trans=N ? n : k),
+ *         10 ldc < max(1, n). */
+int blas3_ssyrk(char uplo, char trans, int64_t n, int64_t k, float alpha,
+                const float *A, int64_t lda, float beta, float *C, int64_t ldc,
+                blas3_stream_t stream);
+
+/* SSYR2K: trans=N: C <- alpha*(A*B^T + B*A^T) + beta*C (A, B n x k);
+ *         trans=T: C <- alpha*(A^T*B + B^T*A) + beta*C (A, B k x n).
+ * Only the `uplo` triangle of C is read and written.
+ * XERBLA: 1 uplo, 2 trans, 3 n<0, 4 k<0, 7 lda < max(1, trans=N ? n : k),
+ *         9 ldb < max(1, trans=N ? n : k), 12 ldc < max(1, n). */
+int blas3_ssyr2k(char uplo, char trans, int64_t n, int64_t k, float alpha,
+                 const float *A, int64_t lda, const float *B, int64_t ldb,
+                 float beta, float *C, int64_t ldc, blas3_stream_t stream);
+
+/* STRMM: side=L: B <- alpha*op(A)*B (A m x m); side=R: B <- alpha*B*op(A)
+ * (A n x n).  A triangular (`uplo`), unit diagonal when diag='U'; the blank
+ * triangle is never read (Adaptor_Triangular; TRMM-LL-N P:395-398).
+ * B (m x n) is overwritten in place without clobbering rows still to be read.
+ * XERBLA: 1 side, 2 uplo, 3 transa, 4 diag, 5 m<0, 6 n<0,
+ *         9 lda < max(1, side=L ? m : n), 11 ldb < max(1, m). */
+int blas3_strmm(char side, char uplo, char transa, char diag, int64_t m, int64_t n,
+                float alpha, const float *A, int64_t lda, float *B, int64_t ldb,
+                blas3_stream_t stream);
+
+/* STRSM: side=L: solve op(A)*X = alpha*B; side=R: solve X*op(A) = alpha*B.
+ * X overwrites B (m x n).  Blocked: diagonal blocks inverted with warp-level
+ * primitives, then block sweep with tensor-core GEMM updates (Adaptor_Solver,
+ * P:225-244, TRSM-LL-N P:397-398).  A must be non-singular (diag='N'); no
+ * pivoting or singularity check, as in BLAS.
+ * XERBLA: as STRMM. */
+int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t n,
+                float alpha, const float *A, int64_t lda, float *B, int64_t ldb,
+                blas3_stream_t stream);
+
+/* Process-wide math mode (BLAS3_MATH_3XTF32 default; the environment
+ * variable BLAS3_MATH=simt|3xtf32 overrides the default at load).
+ * Returns 0, or 1 if `mode` is not a valid mode (nothing changed). */
+int blas3_set_math_mode(int mode);
+int blas3_get_math_mode(void);
+
+/* Optional caller-owned device scratch used before falling back to
+ * cudaMallocAsync.  The buffer must stay valid while calls that may use it
+ * are in flight.  (ptr=NULL, bytes=0 removes it.)  Returns 0. */
+int blas3_set_workspace(void *dptr, size_t bytes);
+
+/* Number of kernels the library launched since load (host-side counter;
+ * the bench uses it to report gpu_launches). */
+int64_t blas3_launch_count(void);
+
+/* Static string for a return code. */
+const char *blas3_error_string(int code);
+
+/* ABI version (major*100 + minor). */
+int blas3_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BLAS3_B200_H */

@@ -1,0 +1,188 @@
+"""B200-native (sm_100a) fp32 Level-3 BLAS derived from one tuned GEMM.
+
+Thin Python binding over the C ABI in ``include/blas3.h`` (``libblas3.so``,
+built in-tree by ``build.py``).  This module only marshals arguments: every
+step of every routine runs in the library's CUDA kernels.  There is no CPU
+fallback: importing the package fails loudly if the library is missing, and
+every routine raises on a non-zero return code.
+
+Two layers, same names as the C ABI:
+  * ``blas3_sgemm(...)`` etc. -- the raw C entry points (ctypes), BLAS
+    argument order, device pointers as ints, stream as int (0 = default).
+  * ``sgemm(transa, transb, alpha, A, B, beta, C)`` etc. -- the same call on
+    column-major CUDA ``torch.Tensor`` views (stride(0) == 1, ld = stride(1)),
+    issued on torch's current stream.  PyTorch provides memory and streams
+    only.
+Matrices are column-major as in BLAS3.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libblas3.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(
+        f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'` "
+        "(there is deliberately no CPU fallback)")
+
+_lib = ctypes.CDLL(LIB_PATH)
+
+_i64, _f, _p, _c, _i = ctypes.c_int64, ctypes.c_float, ctypes.c_void_p, ctypes.c_char, ctypes.c_int
+
+_SIGS = {
+    "blas3_sgemm": [_c, _c, _i64, _i64, _i64, _f, _p, _i64, _p, _i64, _f, _p, _i64, _p],
+    "blas3_ssymm": [_c, _c, _i64, _i64, _f, _p, _i64, _p, _i64, _f, _p, _i64, _p],
+    "blas3_ssyrk": [_c, _c, _i64, _i64, _f, _p, _i64, _f, _p, _i64, _p],
+    "blas3_ssyr2k": [_c, _c, _i64, _i64, _f, _p, _i64, _p, _i64, _f, _p, _i64, _p],
+    "blas3_strmm": [_c, _c, _c, _c, _i64, _i64, _f, _p, _i64, _p, _i64, _p],
+    "blas3_strsm": [_c, _c, _c, _c, _i64, _i64, _f, _p, _i64, _p, _i64, _p],
+    "blas3_set_math_mode": [_i],
+    "blas3_get_math_mode": [],
+    "blas3_set_workspace": [_p, ctypes.c_size_t],
+    "blas3_launch_count": [],
+    "blas3_error_string": [_i],
+    "blas3_version": [],
+}
+_RES = {"blas3_launch_count": _i64, "blas3_error_string": ctypes.c_char_p}
+
+for _name, _args in _SIGS.items():
+    _fn = getattr(_lib, _name)
+    _fn.argtypes = _args
+    _fn.restype = _RES.get(_name, _i)
+    globals()[_name] = _fn
+
+EXPORTED = tuple(_SIGS)
+MATH_3XTF32, MATH_SIMT_FP32 = 0, 1
+
+
+class Blas3Error(RuntimeError):
+    def __init__(self, routine, code):
+        self.code = code
+        msg = blas3_error_string(code).decode()  # noqa: F821
+        super().__init__(f"{routine} returned {code}: {msg}")
+
+
+def _chk(name, rc):
+    if rc != 0:
+        raise Blas3Error(name, rc)
+
+
+def _ch(x):
+    return x.encode() if isinstance(x, str) else x
+
+
+# ----------------------------------------------------------------- tensor helpers
+def _mat(X, name):
+    """(pointer, rows, cols, ld) of a column-major fp32 CUDA tensor view."""
+    import torch
+    if not isinstance(X, torch.Tensor):
+        raise TypeError(f"{name} must be a torch.Tensor")
+    if X.dtype != torch.float32 or not X.is_cuda or X.dim() != 2:
+        raise TypeError(f"{name} must be a 2-D float32 CUDA tensor")
+    m, n = X.shape
+    if m > 1 and X.stride(0) != 1:
+        raise ValueError(f"{name} must be column-major (stride(0) == 1)")
+    ld = X.stride(1) if n > 1 else max(1, m)
+    return X.data_ptr(), m, n, max(ld, 1)
+
+
+def _stream():
+    import torch
+    return torch.cuda.current_stream().cuda_stream
+
+
+def colmajor(m, n, ld=None, device="cuda", fill=None):
+    """Allocate an m x n column-major fp32 tensor (strides (1, ld))."""
+    import torch
+    ld = max(1, m) if ld is None else ld
+    buf = torch.empty((n, ld), dtype=torch.float32, device=device)
+    if fill is not None:
+        buf.fill_(fill)
+    return buf.t()[:m]
+
+
+def from_fortran(arr, device="cuda"):
+    """Copy a numpy Fortran-ordered (ld x n) buffer to a column-major device
+    tensor with the same ld; returns the full (ld x n) view."""
+    import numpy as np
+    import torch
+    a = np.asfortranarray(arr, dtype=np.float32)
+    t = torch.from_numpy(a.T.copy()).to(device)     # (n, ld) row-major == (ld, n) col-major
+    return t.t()
+
+
+# ----------------------------------------------------------------- routines
+def sgemm(transa, transb, alpha, A, B, beta, C):
+    """C <- alpha*op(A)*op(B) + beta*C (GEMM-NN/-TN)."""
+    pc, m, n, ldc = _mat(C, "C")
+    pa, ar, ac, lda = _mat(A, "A")
+    pb, br, bc, ldb = _mat(B, "B")
+    k = ac if transa.upper() == "N" else ar
+    _chk("blas3_sgemm", blas3_sgemm(_ch(transa), _ch(transb), m, n, k, alpha, pa, lda, pb, ldb,  # noqa: F821
+                                    beta, pc, ldc, _stream()))
+
+
+def ssymm(side, uplo, alpha, A, B, beta, C):
+    """side=L: C <- alpha*A*B + beta*C; side=R: C <- alpha*B*A + beta*C."""
+    pc, m, n, ldc = _mat(C, "C")
+    pa, _, _, lda = _mat(A, "A")
+    pb, _, _, ldb = _mat(B, "B")
+    _chk("blas3_ssymm", blas3_ssymm(_ch(side), _ch(uplo), m, n, alpha, pa, lda, pb, ldb,  # noqa: F821
+                                    beta, pc, ldc, _stream()))
+
+
+def ssyrk(uplo, trans, alpha, A, beta, C):
+    """C <- alpha*op(A)*op(A)^T + beta*C on the uplo triangle."""
+    pc, n, _, ldc = _mat(C, "C")
+    pa, ar, ac, lda = _mat(A, "A")
+    k = ac if trans.upper() == "N" else ar
+    _chk("blas3_ssyrk", blas3_ssyrk(_ch(uplo), _ch(trans), n, k, alpha, pa, lda, beta, pc, ldc,  # noqa: F821
+                                    _stream()))
+
+
+def ssyr2k(uplo, trans, alpha, A, B, beta, C):
+    """C <- alpha*(op(A)op(B)^T + op(B)op(A)^T) + beta*C on the uplo triangle."""
+    pc, n, _, ldc = _mat(C, "C")
+    pa, ar, ac, lda = _mat(A, "A")
+    pb, _, _, ldb = _mat(B, "B")
+    k = ac if trans.upper() == "N" else ar
+    _chk("blas3_ssyr2k", blas3_ssyr2k(_ch(uplo), _ch(trans), n, k, alpha, pa, lda, pb, ldb,  # noqa: F821
+                                      beta, pc, ldc, _stream()))
+
+
+def strmm(side, uplo, transa, diag, alpha, A, B):
+    """B <- alpha*op(A)*B (L) or alpha*B*op(A) (R), in place."""
+    pb, m, n, ldb = _mat(B, "B")
+    pa, _, _, lda = _mat(A, "A")
+    _chk("blas3_strmm", blas3_strmm(_ch(side), _ch(uplo), _ch(transa), _ch(diag), m, n, alpha,  # noqa: F821
+                                    pa, lda, pb, ldb, _stream()))
+
+
+def strsm(side, uplo, transa, diag, alpha, A, B):
+    """Solve op(A)X = alpha*B (L) or X op(A) = alpha*B (R); X overwrites B."""
+    pb, m, n, ldb = _mat(B, "B")
+    pa, _, _, lda = _mat(A, "A")
+    _chk("blas3_strsm", blas3_strsm(_ch(side), _ch(uplo), _ch(transa), _ch(diag), m, n, alpha,  # noqa: F821
+                                    pa, lda, pb, ldb, _stream()))
+
+
+def set_math_mode(mode):
+    if isinstance(mode, str):
+        mode = {"3xtf32": MATH_3XTF32, "simt": MATH_SIMT_FP32}[mode.lower()]
+    _chk("blas3_set_math_mode", blas3_set_math_mode(mode))  # noqa: F821
+
+
+def get_math_mode():
+    return blas3_get_math_mode()  # noqa: F821
+
+
+def launch_count():
+    return int(blas3_launch_count())  # noqa: F821
+
+
+__all__ = ["sgemm", "ssymm", "ssyrk", "ssyr2k", "strmm", "strsm", "set_math_mode",
+           "get_math_mode", "launch_count", "colmajor", "from_fortran", "Blas3Error",
+           "MATH_3XTF32", "MATH_SIMT_FP32", *EXPORTED]

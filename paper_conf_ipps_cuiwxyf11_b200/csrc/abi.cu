@@ -1,0 +1,429 @@
+// abi.cu -- the extern "C" boundary (include/blas3.h) and the routine
+// drivers: argument validation in XERBLA order, quick returns and alpha/beta
+// special cases (row A1), canonicalisation of every variant into one
+// structured-GEMM Problem (row A2), the in-place STRMM (row A9) and the
+// blocked STRSM sweep (rows A7/A8).
+#include <cuda_runtime.h>
+#include <ctype.h>
+#include <stdlib.h>
+#include <string.h>
+#include <atomic>
+#include <mutex>
+
+#include "../../include/blas3.h"
+#include "kernels.h"
+
+namespace blas3 {
+
+static std::atomic<int64_t> g_launches{0};
+void note_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+
+static int g_math = -1;              // -1: not initialised
+static void *g_ws = nullptr;
+static size_t g_ws_bytes = 0;
+
+static int math_mode() {
+  if (g_math < 0) {
+    const char *e = getenv("BLAS3_MATH");
+    g_math = (e && (e[0] == 's' || e[0] == 'S')) ? BLAS3_MATH_SIMT_FP32 : BLAS3_MATH_3XTF32;
+  }
+  return g_math;
+}
+
+// per-device facts: SM count, sm_100 check
+struct DevInfo { int sms = 0; int ok = -1; };
+static DevInfo g_dev[64];
+static std::mutex g_dev_mu;
+
+static int device_check(int &sms) {
+  int d = 0;
+  if (cudaGetDevice(&d) != cudaSuccess || d < 0 || d >= 64) return BLAS3_ERR_CUDA;
+  std::lock_guard<std::mutex> lk(g_dev_mu);
+  DevInfo &di = g_dev[d];
+  if (di.ok < 0) {
+    cudaDeviceProp p;
+    if (cudaGetDeviceProperties(&p, d) != cudaSuccess) return BLAS3_ERR_CUDA;
+    di.ok = (p.major == 10 && p.minor == 0) ? 1 : 0;
+    di.sms = p.multiProcessorCount;
+    // keep freed scratch cached in the pool (no host sync on reuse)
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, d) == cudaSuccess) {
+      uint64_t thr = UINT64_MAX;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
+  sms = di.sms;
+  return di.ok ? 0 : BLAS3_ERR_ARCH;
+}
+
+// stream-ordered scratch: caller-provided workspace first, else the pool
+struct Scratch {
+  float *p = nullptr;
+  bool owned = false;
+  cudaStream_t s = nullptr;
+  ~Scratch() { if (owned && p) cudaFreeAsync(p, s); }
+};
+static int get_scratch(Scratch &sc, size_t bytes, cudaStream_t s, size_t offset = 0) {
+  sc.s = s;
+  if (g_ws && offset + bytes <= g_ws_bytes) { sc.p = (float *)((char *)g_ws + offset); return 0; }
+  if (cudaMallocAsync((void **)&sc.p, bytes, s) != cudaSuccess) { cudaGetLastError(); return BLAS3_ERR_ALLOC; }
+  sc.owned = true;
+  return 0;
+}
+
+static int run_problem(const Problem &P, cudaStream_t s, int sms) {
+  if (P.M <= 0 || P.N <= 0) return 0;
+  if (math_mode() == BLAS3_MATH_3XTF32 && tc_eligible(P)) return launch_tc(P, s, sms);
+  int rc = launch_simt(P, s, sms);
+  return rc ? BLAS3_ERR_CUDA : 0;
+}
+
+static OpDesc dense(const float *p, int64_t ld, bool kr) {
+  OpDesc o; memset(&o, 0, sizeof(o));
+  o.ptr = p; o.ld = ld; o.kind = OP_DENSE; o.kr = kr; o.map_rk = o.map_kr = -1;
+  return o;
+}
+static OpDesc sym(const float *p, int64_t ld, bool lower) {
+  OpDesc o = dense(p, ld, false); o.kind = OP_SYM; o.lower = lower; return o;
+}
+static OpDesc tri(const float *p, int64_t ld, bool lower, bool swap, bool unit) {
+  OpDesc o = dense(p, ld, false); o.kind = OP_TRI; o.lower = lower; o.swap = swap; o.unit = unit;
+  return o;
+}
+static Problem problem(int64_t M, int64_t N, float alpha, float beta, const float *Cin,
+                       int64_t ldcin, float *Cout, int64_t ldcout) {
+  Problem P; memset(&P, 0, sizeof(P));
+  P.M = M; P.N = N; P.nseg = 1; P.alpha = alpha; P.beta = beta;
+  P.Cin = Cin; P.ldcin = ldcin; P.Cout = Cout; P.ldcout = ldcout;
+  return P;
+}
+
+// plain dense GEMM used by the TRSM sweep: C = alpha*Xa*Xb^T + beta*C
+static int gemm_dense(int64_t M, int64_t N, int64_t K, float alpha, const float *a, int64_t lda,
+                      bool a_kr, const float *b, int64_t ldb, bool b_kr, float beta, float *C,
+                      int64_t ldc, cudaStream_t s, int sms) {
+  if (M <= 0 || N <= 0) return 0;
+  Problem P = problem(M, N, alpha, beta, C, ldc, C, ldc);
+  P.seg[0].a = dense(a, lda, a_kr);
+  P.seg[0].b = dense(b, ldb, b_kr);
+  P.seg[0].K = K;
+  return run_problem(P, s, sms);
+}
+
+static inline int up(char c) { return toupper((unsigned char)c); }
+static inline bool is_trans(char c) { int u = up(c); return u == 'N' || u == 'T' || u == 'C'; }
+static inline bool is_side(char c) { int u = up(c); return u == 'L' || u == 'R'; }
+static inline bool is_uplo(char c) { int u = up(c); return u == 'L' || u == 'U'; }
+static inline bool is_diag(char c) { int u = up(c); return u == 'N' || u == 'U'; }
+static inline int64_t mx1(int64_t v) { return v > 1 ? v : 1; }
+
+static inline int finish(int rc) {
+  if (rc) return rc;
+  return cudaGetLastError() == cudaSuccess ? 0 : BLAS3_ERR_CUDA;
+}
+
+}  // namespace blas3
+
+using namespace blas3;
+
+extern "C" {
+
+int blas3_version(void) { return 100; }
+int64_t blas3_launch_count(void) { return g_launches.load(); }
+
+int blas3_set_math_mode(int mode) {
+  if (mode != BLAS3_MATH_3XTF32 && mode != BLAS3_MATH_SIMT_FP32) return 1;
+  g_math = mode;
+  return 0;
+}
+int blas3_get_math_mode(void) { return math_mode(); }
+
+int blas3_set_workspace(void *dptr, size_t bytes) {
+  g_ws = bytes ? dptr : nullptr;
+  g_ws_bytes = dptr ? bytes : 0;
+  return 0;
+}
+
+const char *blas3_error_string(int code) {
+  switch (code) {
+    case BLAS3_OK: return "success";
+    case BLAS3_ERR_CUDA: return "CUDA launch or runtime error";
+    case BLAS3_ERR_ARCH: return "current device is not sm_100 (B200)";
+    case BLAS3_ERR_ALLOC: return "scratch allocation failed";
+    case BLAS3_ERR_TMA: return "TMA tensor-map encoding failed";
+    default: return code > 0 ? "invalid argument (value = 1-based XERBLA position)" : "unknown error";
+  }
+}
+
+// ------------------------------------------------------------------- SGEMM
+int blas3_sgemm(char transa, char transb, int64_t m, int64_t n, int64_t k, float alpha,
+                const float *A, int64_t lda, const float *B, int64_t ldb, float beta, float *C,
+                int64_t ldc, blas3_stream_t stream) {
+  const bool ta = up(transa) != 'N', tb = up(transb) != 'N';
+  if (!is_trans(transa)) return 1;
+  if (!is_trans(transb)) return 2;
+  if (m < 0) return 3;
+  if (n < 0) return 4;
+  if (k < 0) return 5;
+  if (lda < mx1(ta ? k : m)) return 8;
+  if (ldb < mx1(tb ? n : k)) return 10;
+  if (ldc < mx1(m)) return 13;
+  if (m == 0 || n == 0 || ((alpha == 0.f || k == 0) && beta == 1.f)) return 0;
+  if (!C) return 12;
+  const bool reads_ab = alpha != 0.f && k > 0;
+  if (reads_ab && !A) return 7;
+  if (reads_ab && !B) return 9;
+  int sms, rc = device_check(sms);
+  if (rc) return rc;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!reads_ab) return finish(launch_scale(C, ldc, m, n, beta, 0, s) ? BLAS3_ERR_CUDA : 0);
+  Problem P = problem(m, n, alpha, beta, C, ldc, C, ldc);
+  P.seg[0].a = dense(A, lda, ta);       // op(A)(r,k) = A(k,r) when transposed -> "kr"
+  P.seg[0].b = dense(B, ldb, !tb);      // Xb(c,k) = op(B)(k,c)
+  P.seg[0].K = k;
+  return finish(run_problem(P, s, sms));
+}
+
+// ------------------------------------------------------------------- SSYMM
+int blas3_ssymm(char side, char uplo, int64_t m, int64_t n, float alpha, const float *A,
+                int64_t lda, const float *B, int64_t ldb, float beta, float *C, int64_t ldc,
+                blas3_stream_t stream) {
+  const bool left = up(side) == 'L', lower = up(uplo) == 'L';
+  if (!is_side(side)) return 1;
+  if (!is_uplo(uplo)) return 2;
+  if (m < 0) return 3;
+  if (n < 0) return 4;
+  if (lda < mx1(left ? m : n)) return 7;
+  if (ldb < mx1(m)) return 9;
+  if (ldc < mx1(m)) return 12;
+  if (m == 0 || n == 0 || (alpha == 0.f && beta == 1.f)) return 0;
+  if (!C) return 11;
+  if (alpha != 0.f && !A) return 6;
+  if (alpha != 0.f && !B) return 8;
+  int sms, rc = device_check(sms);
+  if (rc) return rc;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (alpha == 0.f) return finish(launch_scale(C, ldc, m, n, beta, 0, s) ? BLAS3_ERR_CUDA : 0);
+  Problem P = problem(m, n, alpha, beta, C, ldc, C, ldc);
+  if (left) {                       // C = Asym * B : Xa = Asym (m x m), Xb(c,k) = B(k,c)
+    P.seg[0].a = sym(A, lda, lower);
+    P.seg[0].b = dense(B, ldb, true);
+    P.seg[0].K = m;
+  } else {                          // C = B * Asym : Xa = B, Xb(c,k) = Asym(k,c) = Asym(c,k)
+    P.seg[0].a = dense(B, ldb, false);
+    P.seg[0].b = sym(A, lda, lower);
+    P.seg[0].K = n;
+  }
+  return finish(run_problem(P, s, sms));
+}
+
+// ------------------------------------------------------------------- SSYRK / SSYR2K
+static int syrk_common(bool two, char uplo, char trans, int64_t n, int64_t k, float alpha,
+                       const float *A, int64_t lda, const float *B, int64_t ldb, float beta,
+                       float *C, int64_t ldc, cudaStream_t s) {
+  const bool lower = up(uplo) == 'L', ta = up(trans) != 'N';
+  const int tri = lower ? 1 : 2;
+  if (n == 0 || ((alpha == 0.f || k == 0) && beta == 1.f)) return 0;
+  if (!C) return two ? 11 : 9;
+  const bool reads = alpha != 0.f && k > 0;
+  if (reads && !A) return 6;
+  if (two && reads && !B) return 8;
+  int sms, rc = device_check(sms);
+  if (rc) return rc;
+  if (!reads) return finish(launch_scale(C, ldc, n, n, beta, tri, s) ? BLAS3_ERR_CUDA : 0);
+  Problem P = problem(n, n, alpha, beta, C, ldc, C, ldc);
+  P.c_tri = tri;
+  // trans=N: op(A) = A (n x k) -> X(r,k) = A(r,k) "rk"; trans=T: X(r,k) = A(k,r) "kr"
+  P.seg[0].a = dense(A, lda, ta);
+  P.seg[0].b = dense(two ? B : A, two ? ldb : lda, ta);
+  P.seg[0].K = k;
+  if (two) {
+    P.nseg = 2;
+    P.seg[1].a = dense(B, ldb, ta);
+    P.seg[1].b = dense(A, lda, ta);
+    P.seg[1].K = k;
+  }
+  return finish(run_problem(P, s, sms));
+}
+
+int blas3_ssyrk(char uplo, char trans, int64_t n, int64_t k, float alpha, const float *A,
+                int64_t lda, float beta, float *C, int64_t ldc, blas3_stream_t stream) {
+  const bool ta = up(trans) != 'N';
+  if (!is_uplo(uplo)) return 1;
+  if (!is_trans(trans)) return 2;
+  if (n < 0) return 3;
+  if (k < 0) return 4;
+  if (lda < mx1(ta ? k : n)) return 7;
+  if (ldc < mx1(n)) return 10;
+  return syrk_common(false, uplo, trans, n, k, alpha, A, lda, nullptr, 0, beta, C, ldc,
+                     (cudaStream_t)stream);
+}
+
+int blas3_ssyr2k(char uplo, char trans, int64_t n, int64_t k, float alpha, const float *A,
+                 int64_t lda, const float *B, int64_t ldb, float beta, float *C, int64_t ldc,
+                 blas3_stream_t stream) {
+  const bool ta = up(trans) != 'N';
+  if (!is_uplo(uplo)) return 1;
+  if (!is_trans(trans)) return 2;
+  if (n < 0) return 3;
+  if (k < 0) return 4;
+  if (lda < mx1(ta ? k : n)) return 7;
+  if (ldb < mx1(ta ? k : n)) return 9;
+  if (ldc < mx1(n)) return 12;
+  return syrk_common(true, uplo, trans, n, k, alpha, A, lda, B, ldb, beta, C, ldc,
+                     (cudaStream_t)stream);
+}
+
+// ------------------------------------------------------------------- STRMM / STRSM validation
+static int tr_validate(char side, char uplo, char transa, char diag, int64_t m, int64_t n,
+                       int64_t lda, int64_t ldb) {
+  if (!is_side(side)) return 1;
+  if (!is_uplo(uplo)) return 2;
+  if (!is_trans(transa)) return 3;
+  if (!is_diag(diag)) return 4;
+  if (m < 0) return 5;
+  if (n < 0) return 6;
+  if (lda < mx1(up(side) == 'L' ? m : n)) return 9;
+  if (ldb < mx1(m)) return 11;
+  return 0;
+}
+
+// ------------------------------------------------------------------- STRMM (row A9)
+// B <- alpha*op(A)*B (L) or alpha*B*op(A) (R).  The tile-parallel product
+// reads rows (L) / columns (R) of B that other tiles overwrite, so the
+// product goes to stream-ordered scratch and is copied back (A9).
+int blas3_strmm(char side, char uplo, char transa, char diag, int64_t m, int64_t n, float alpha,
+                const float *A, int64_t lda, float *B, int64_t ldb, blas3_stream_t stream) {
+  int v = tr_validate(side, uplo, transa, diag, m, n, lda, ldb);
+  if (v) return v;
+  if (m == 0 || n == 0) return 0;
+  if (!B) return 10;
+  if (alpha != 0.f && !A) return 8;
+  int sms, rc = device_check(sms);
+  if (rc) return rc;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (alpha == 0.f) return finish(launch_scale(B, ldb, m, n, 0.f, 0, s) ? BLAS3_ERR_CUDA : 0);
+  const bool left = up(side) == 'L', lower = up(uplo) == 'L', ta = up(transa) != 'N',
+             unit = up(diag) == 'U';
+  Scratch W;
+  if ((rc = get_scratch(W, (size_t)m * n * sizeof(float), s))) return rc;
+  Problem P = problem(m, n, alpha, 0.f, nullptr, 0, W.p, m);
+  if (left) {     // Xa(r,k) = op(T)(r,k) -> swap = trans ; Xb(c,k) = B(k,c)
+    P.seg[0].a = tri(A, lda, lower, ta, unit);
+    P.seg[0].b = dense(B, ldb, true);
+    P.seg[0].K = m;
+    P.rev_m = tri_kle(P.seg[0].a);        // longest k-ranges first
+  } else {        // Xa = B ; Xb(c,k) = op(T)(k,c) -> swap = !trans
+    P.seg[0].a = dense(B, ldb, false);
+    P.seg[0].b = tri(A, lda, lower, !ta, unit);
+    P.seg[0].K = n;
+    P.rev_n = tri_kle(P.seg[0].b);
+  }
+  if ((rc = run_problem(P, s, sms))) return rc;
+  if (launch_copy(B, ldb, W.p, m, m, n, s)) return BLAS3_ERR_CUDA;
+  return finish(0);
+}
+
+// ------------------------------------------------------------------- STRSM (rows A7, A8)
+// Blocked sweep in dependency order: nb=128 diagonal blocks are
+// inverted up front (warp-level kernel), then per block X_b = inv(op(A)_bb)*B_b
+// followed by a GEMM update of the rows (L) / columns (R) still to be solved.
+// Updates are two-level: inside an outer panel of NBO rows only the panel is
+// updated; after the panel one large GEMM updates everything beyond it.
+// alpha is folded into the first operation touching each row/column.
+static const int NB = 128, NBO = 1024;
+
+int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t n, float alpha,
+                const float *A, int64_t lda, float *B, int64_t ldb, blas3_stream_t stream) {
+  int v = tr_validate(side, uplo, transa, diag, m, n, lda, ldb);
+  if (v) return v;
+  if (m == 0 || n == 0) return 0;
+  if (!B) return 10;
+  if (alpha != 0.f && !A) return 8;
+  int sms, rc = device_check(sms);
+  if (rc) return rc;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (alpha == 0.f) return finish(launch_scale(B, ldb, m, n, 0.f, 0, s) ? BLAS3_ERR_CUDA : 0);
+
+  const bool left = up(side) == 'L', lower = up(uplo) == 'L', ta = up(transa) != 'N',
+             unit = up(diag) == 'U';
+  const bool lower_op = lower != ta;               // op(A) lower-triangular
+  const int64_t nt = left ? m : n;                 // order of A
+  const int64_t nblk = cdiv(nt, NB);
+  const int64_t other = left ? n : m;              // RHS extent
+  const bool forward = left ? lower_op : !lower_op;
+
+  Scratch D, W;
+  if ((rc = get_scratch(D, (size_t)nblk * NB * NB * sizeof(float), s))) return rc;
+  if ((rc = get_scratch(W, (size_t)NB * other * sizeof(float), s,
+                        (size_t)nblk * NB * NB * sizeof(float)))) return rc;
+  if (launch_trsm_diag_inv(A, lda, nt, ta, lower_op, unit, NB, D.p, s)) return BLAS3_ERR_CUDA;
+
+  // op(A) sub-block as a GEMM operand with rows R (r0..) x k (k0..):
+  //   Xa(r,k) = op(A)(r0+r, k0+k) (left: rows of the update)
+  auto opA_rk = [&](int64_t r0, int64_t k0, const float *&p, bool &kr) {
+    if (!ta) { p = A + r0 + k0 * lda; kr = false; } else { p = A + k0 + r0 * lda; kr = true; }
+  };
+  const int64_t per_panel = NBO / NB;
+  const int64_t npanel = cdiv(nblk, per_panel);
+  for (int64_t pi = 0; pi < npanel; ++pi) {
+    // blocks of this panel in processing order
+    int64_t q0 = pi * per_panel, q1 = imin(nblk, q0 + per_panel);
+    for (int64_t q = q0; q < q1; ++q) {
+      const int64_t b = forward ? q : nblk - 1 - q;
+      const int64_t b0 = b * NB, nbr = imin(NB, nt - b0);
+      const bool pend = (pi == 0 && q == q0);      // rows of panel 0 still unscaled
+      const float a1 = pend ? alpha : 1.f;
+      // remaining blocks of the panel (in processing order) -> contiguous range
+      int64_t rq0 = q + 1, rq1 = q1;
+      int64_t r_lo, r_hi;                          // element range of those blocks
+      if (forward) { r_lo = (rq0 < rq1) ? rq0 * NB : 0; r_hi = (rq0 < rq1) ? imin(nt, rq1 * NB) : 0; }
+      else {
+        r_lo = (rq0 < rq1) ? (nblk - rq1) * NB : 0;
+        r_hi = (rq0 < rq1) ? imin(nt, (nblk - rq0) * NB) : 0;
+      }
+      const float *Db = D.p + b * NB * NB;
+      if (left) {
+        // W = a1 * Dinv_b * B_b   (nbr x n), then B_b <- W
+        if ((rc = gemm_dense(nbr, n, nbr, a1, Db, NB, false, B + b0, ldb, true, 0.f, W.p, NB, s, sms))) return rc;
+        if (launch_copy(B + b0, ldb, W.p, NB, nbr, n, s)) return BLAS3_ERR_CUDA;
+        if (r_hi > r_lo) {   // B_r <- a1*B_r - op(A)(r, b) * X_b
+          const float *pa; bool akr; opA_rk(r_lo, b0, pa, akr);
+          if ((rc = gemm_dense(r_hi - r_lo, n, nbr, -1.f, pa, lda, akr, W.p, NB, true, a1,
+                               B + r_lo, ldb, s, sms))) return rc;
+        }
+      } else {
+        // W = a1 * B_b * Dinv_b  (m x nbr), then B(:, b) <- W
+        if ((rc = gemm_dense(m, nbr, nbr, a1, B + b0 * ldb, ldb, false, Db, NB, true, 0.f, W.p, m, s, sms))) return rc;
+        if (launch_copy(B + b0 * ldb, ldb, W.p, m, m, nbr, s)) return BLAS3_ERR_CUDA;
+        if (r_hi > r_lo) {   // B(:,c) <- a1*B(:,c) - X_b * op(A)(b, c)
+          // Xb(c,k) = op(A)(b0+k, c0+c): !ta -> A[(b0+k) + (c0+c)*lda] (kr); ta -> A[(c0+c)+(b0+k)*lda]
+          const float *pb = ta ? A + r_lo + b0 * lda : A + b0 + r_lo * lda;
+          if ((rc = gemm_dense(m, r_hi - r_lo, nbr, -1.f, W.p, m, false, pb, lda, !ta, a1,
+                               B + r_lo * ldb, ldb, s, sms))) return rc;
+        }
+      }
+    }
+    // outer update of everything beyond the panel
+    int64_t pq0 = q0, pq1 = q1;                      // panel blocks (processing order)
+    int64_t p_lo = forward ? pq0 * NB : (nblk - pq1) * NB;
+    int64_t p_hi = forward ? imin(nt, pq1 * NB) : imin(nt, (nblk - pq0) * NB);
+    int64_t o_lo = forward ? p_hi : 0, o_hi = forward ? nt : p_lo;
+    if (o_hi > o_lo) {
+      const float a1 = (pi == 0) ? alpha : 1.f;
+      const int64_t kp = p_hi - p_lo;
+      if (left) {   // B_o <- a1*B_o - op(A)(o, panel) * X_panel (X_panel = B rows of the panel)
+        const float *pa; bool akr; opA_rk(o_lo, p_lo, pa, akr);
+        if ((rc = gemm_dense(o_hi - o_lo, n, kp, -1.f, pa, lda, akr, B + p_lo, ldb, true, a1,
+                             B + o_lo, ldb, s, sms))) return rc;
+      } else {      // B(:,o) <- a1*B(:,o) - X_panel * op(A)(panel, o)
+        const float *pb = ta ? A + o_lo + p_lo * lda : A + p_lo + o_lo * lda;
+        if ((rc = gemm_dense(m, o_hi - o_lo, kp, -1.f, B + p_lo * ldb, ldb, false, pb, lda, !ta, a1,
+                             B + o_lo * ldb, ldb, s, sms))) return rc;
+      }
+    }
+  }
+  return finish(0);
+}
+
+}  // extern "C"

@@ -1,0 +1,146 @@
+// simt_kernel.cu -- exact-FP32 SIMT variant of the structured GEMM (row A10).
+//
+// The paper's own kernel class: shared-memory tiles + register-blocked C
+// ("SM_alloc" P:93-99, "Reg_alloc(C)" P:101, Volkov-style scheme P:75) with
+// the structure of every routine applied while the tile is staged to shared
+// memory (mirror / zero-select / unit diagonal, via load_op) and the uplo
+// mask applied in the epilogue.  128x128 CTA tile, BK=16, 256 threads,
+// 8x8 outputs per thread, register-prefetched double buffer.
+#include <cuda_runtime.h>
+#include "problem.h"
+#include "kernels.h"
+
+namespace blas3 {
+
+namespace {
+constexpr int BM = 128, BN = 128, BK = 16, NT = 256, PADS = 4;
+
+struct Stage {
+  float a[BK][BM + PADS];
+  float b[BK][BN + PADS];
+};
+
+// r-contiguous ("rk") or k-contiguous ("kr") element mapping for coalescing
+__device__ __forceinline__ void elem_rk(int tid, int i, int &r, int &k) {
+  int e = tid + i * NT; r = e % BM; k = e / BM;
+}
+__device__ __forceinline__ void elem_kr(int tid, int i, int &r, int &k) {
+  int e = tid + i * NT; k = e % BK; r = e / BK;
+}
+__device__ __forceinline__ bool prefers_kr(const OpDesc &o) {
+  return o.kind == OP_DENSE ? o.kr != 0 : (o.kind == OP_TRI ? o.swap != 0 : false);
+}
+
+__device__ __forceinline__ void fetch(const OpDesc &o, bool kr, int64_t R, int64_t K,
+                                      int64_t r0, int64_t kb, float (&v)[8]) {
+  int tid = threadIdx.x;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    int r, k;
+    if (kr) elem_kr(tid, i, r, k); else elem_rk(tid, i, r, k);
+    v[i] = load_op(o, r0 + r, kb + k, R, K);
+  }
+}
+
+__device__ __forceinline__ void stash(float (*dst)[BM + PADS], bool kr, const float (&v)[8]) {
+  int tid = threadIdx.x;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    int r, k;
+    if (kr) elem_kr(tid, i, r, k); else elem_rk(tid, i, r, k);
+    dst[k][r] = v[i];
+  }
+}
+}  // namespace
+
+__global__ void __launch_bounds__(NT, 2)
+simt_structured_gemm(const Problem P) {
+  __shared__ __align__(16) Stage st[2];
+  const int tid = threadIdx.x, tx = tid % 16, ty = tid / 16;
+  const int64_t ntiles = Tiles<BM, BN>::count(P);
+
+  for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    int64_t mi, nj;
+    Tiles<BM, BN>::coords(P, t, mi, nj);
+    const int64_t m0 = mi * BM, n0 = nj * BN;
+    const int64_t m1 = imin(P.M, m0 + BM), n1 = imin(P.N, n0 + BN);
+
+    float acc[8][8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+#pragma unroll
+      for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+
+    for (int s = 0; s < P.nseg; ++s) {
+      const Segment &sg = P.seg[s];
+      int64_t k0, k1;
+      k_range(sg, m0, m1, n0, n1, k0, k1);
+      k0 = (k0 / BK) * BK;
+      if (k1 <= k0) continue;
+      const bool akr = prefers_kr(sg.a), bkr = prefers_kr(sg.b);
+      float va[8], vb[8];
+      fetch(sg.a, akr, P.M, sg.K, m0, k0, va);
+      fetch(sg.b, bkr, P.N, sg.K, n0, k0, vb);
+      int buf = 0;
+      __syncthreads();  // previous tile/segment finished reading smem
+      stash(st[0].a, akr, va);
+      stash(st[0].b, bkr, vb);
+      __syncthreads();
+      for (int64_t kb = k0; kb < k1; kb += BK) {
+        const bool more = kb + BK < k1;
+        if (more) {
+          fetch(sg.a, akr, P.M, sg.K, m0, kb + BK, va);
+          fetch(sg.b, bkr, P.N, sg.K, n0, kb + BK, vb);
+        }
+        const Stage &S = st[buf];
+#pragma unroll
+        for (int k = 0; k < BK; ++k) {
+          float4 a0 = *reinterpret_cast<const float4 *>(&S.a[k][tx * 4]);
+          float4 a1 = *reinterpret_cast<const float4 *>(&S.a[k][64 + tx * 4]);
+          float4 b0 = *reinterpret_cast<const float4 *>(&S.b[k][ty * 4]);
+          float4 b1 = *reinterpret_cast<const float4 *>(&S.b[k][64 + ty * 4]);
+          float a[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+          float b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+#pragma unroll
+            for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+        }
+        if (more) {
+          stash(st[buf ^ 1].a, akr, va);
+          stash(st[buf ^ 1].b, bkr, vb);
+          __syncthreads();
+          buf ^= 1;
+        }
+      }
+    }
+
+    // epilogue: D = alpha*acc + beta*C on the (masked) tile
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      int64_t c = n0 + (j < 4 ? ty * 4 + j : 64 + ty * 4 + (j - 4));
+      if (c >= P.N) continue;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        int64_t r = m0 + (i < 4 ? tx * 4 + i : 64 + tx * 4 + (i - 4));
+        if (r >= P.M) continue;
+        if (P.c_tri == 1 && r < c) continue;
+        if (P.c_tri == 2 && r > c) continue;
+        float v = P.alpha * acc[i][j];
+        if (P.beta != 0.f) v = fmaf(P.beta, P.Cin[r + c * P.ldcin], v);
+        P.Cout[r + c * P.ldcout] = v;
+      }
+    }
+  }
+}
+
+int launch_simt(const Problem &P, cudaStream_t stream, int num_sms) {
+  int64_t tiles = Tiles<BM, BN>::count(P);
+  if (tiles == 0) return 0;
+  int64_t grid = imin(tiles, (int64_t)num_sms * 2);
+  simt_structured_gemm<<<(unsigned)grid, NT, 0, stream>>>(P);
+  note_launch();
+  return cudaGetLastError() == cudaSuccess ? 0 : -1;
+}
+
+}  // namespace blas3

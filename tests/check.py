@@ -1,0 +1,64 @@
+"""Shared helpers for the GPU parity tests: run a routine through the public
+binding (-> C ABI -> CUDA kernels) on numpy inputs and compute the error
+metrics of DESIGN.md §Parity (north-star tolerances)."""
+import numpy as np
+
+F64 = np.float64
+
+
+def f64(x):
+    return np.asarray(x, dtype=F64)
+
+
+def to_dev(buf):
+    import paper_conf_ipps_cuiwxyf11_b200 as b3
+    return b3.from_fortran(buf)
+
+
+def to_host(t):
+    return np.asfortranarray(t.cpu().numpy())
+
+
+def bits_equal(a, b):
+    a = np.ascontiguousarray(np.asarray(a, dtype=np.float32))
+    b = np.ascontiguousarray(np.asarray(b, dtype=np.float32))
+    return a.shape == b.shape and np.array_equal(a.view(np.uint32), b.view(np.uint32))
+
+
+def op(X, t):
+    return X.T if t.upper() != "N" else X
+
+
+def sym_full(A, uplo, n):
+    A = np.nan_to_num(f64(A[:n, :n]))
+    if uplo.upper() == "L":
+        L = np.tril(A)
+        return L + np.tril(L, -1).T
+    U = np.triu(A)
+    return U + np.triu(U, 1).T
+
+
+def tri_full(A, uplo, diag, n):
+    A = np.nan_to_num(f64(A[:n, :n]))
+    T = np.tril(A) if uplo.upper() == "L" else np.triu(A)
+    if diag.upper() == "U":
+        np.fill_diagonal(T, 1.0)
+    return T
+
+
+def fro(x):
+    return float(np.linalg.norm(f64(x)))
+
+
+def e_nw(got, ref, scale):
+    """normwise ||C - C_ref||_F / scale (scale = |a| ||opA|| ||opB|| + |b| ||C||)."""
+    return fro(f64(got) - f64(ref)) / max(scale, 1e-300)
+
+
+def e_rel(got, ref):
+    return fro(f64(got) - f64(ref)) / max(fro(ref), 1e-300)
+
+
+# binding tolerance (north star) and the output-relative diagnostic
+TOL_NW = 1e-5
+TOL_REL = 5e-6
