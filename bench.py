@@ -1,0 +1,432 @@
+#!/usr/bin/env python
+"""Benchmark: the six fp32 Level-3 routines at N=8192 on B200 (BASELINE.json metric).
+
+One STEP = one pass of the whole hot path over one batch of synthetic input:
+    C <- sgemm ('N','N', a, A, B, b, C)          2 N^3 flops
+    C <- ssymm ('L','L', a, A, B, b, C)          2 N^3      (A's lower triangle)
+    C <- ssyrk ('L','N', a, A, b, C)             N^2 (N+1)  (lower triangle of C)
+    C <- ssyr2k('L','N', a, A, B, b, C)          2 N^3 + N
+    X <- strmm ('L','L','N','N', a, T, X)        N^3        (X = B copied)
+    X <- strsm ('L','L','N','N', a, T, X)        N^3
+with a = 1.5, b = 0.5, N = K = 8192 (configs[1..3] of BASELINE.json at N=8192),
+T diagonally dominant lower-triangular.  Flops are LAWN-41 algorithmic counts
+(Q1).  value = total flops / step time (GFLOPS, all ranks).
+
+Every operand is 256 MiB > 126 MB L2, so no L2 flush is needed between steps.
+At N>1 (torchrun) each rank runs the chain on its own column slab of B/C/X
+(n_global = 8192 * world) after an NCCL broadcast of A and T from rank 0
+inside the timed region (column-slab sharding, weak scaling).
+
+--impl reference times the fp64 CPU oracle (the deliberately slow reference
+arm of this tier) on a bounded column sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+N = 8192
+ALPHA, BETA = 1.5, 0.5
+ROUTINES = ["sgemm", "ssymm", "ssyrk", "ssyr2k", "strmm", "strsm"]
+
+
+def flops(n, cols=None):
+    """LAWN-41 counts for one step (cols = columns of B/C actually computed)."""
+    c = n if cols is None else cols
+    return {
+        "sgemm": 2.0 * n * n * c,
+        "ssymm": 2.0 * n * n * c,
+        "ssyrk": 1.0 * n * n * (n + 1) * (c / n),
+        "ssyr2k": (2.0 * n * n * n + n) * (c / n),
+        "strmm": 1.0 * n * n * c,
+        "strsm": 1.0 * n * n * c,
+    }
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured"
+    return {"bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0, "hbm_gbs": 6650.0}, "fallback"
+
+
+# nominal dense TF32 / BF16 ratio (B200_PROFILING.md: 1.1 vs 2.25 PFLOP/s)
+TF32_OVER_BF16 = 1.1 / 2.25
+
+
+def fp32_3xtf32_peak(peaks, sustained=True):
+    """fp32-via-3xTF32 peak: measured bf16 x nominal tf32/bf16 ratio / 3 UMMAs."""
+    bf16 = peaks["bf16_tflops_sustained" if sustained else "bf16_tflops"]
+    return bf16 * TF32_OVER_BF16 / 3.0
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for nm, v in zip(names, r[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "samples": len(self.rows), "reasons": sorted(reasons)}
+
+
+# ----------------------------------------------------------------------------- inputs
+def make_inputs(n, cols, rank):
+    """Seeded host inputs (pinned later).  A, T are shared (broadcast at N>1);
+    B, C are this rank's column slab of the global matrices."""
+    import blas3_inputs as gen
+    A = gen.uniform(n, n, "bench-A") if rank == 0 else None
+    T = gen.triangular_dd(n, "L", "N", "bench-T") if rank == 0 else None
+    B = gen.uniform(n, cols, "bench-B", rank)
+    C = gen.uniform(n, cols, "bench-C", rank)
+    return A, T, B, C
+
+
+def pinned(arr, torch):
+    """numpy Fortran (n x c) -> pinned host tensor laid out (c, n) row-major."""
+    t = torch.from_numpy(np.ascontiguousarray(arr.T)).pin_memory()
+    return t
+
+
+# ----------------------------------------------------------------------------- our arm
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    import paper_conf_ipps_cuiwxyf11_b200 as b3
+    b3.set_math_mode(args.math)
+    n = args.n
+    cols = n                                   # per-rank slab width (weak scaling)
+    A_h, T_h, B_h, C_h = make_inputs(n, cols, rank)
+    dev = torch.device("cuda", local)
+
+    def colmaj(t2d):                           # (c, n) row-major device -> (n, c) column-major view
+        return t2d.t()
+
+    # device buffers (column-major views of (cols, n) row-major storage)
+    dA = torch.empty((n, n), device=dev); dT = torch.empty((n, n), device=dev)
+    dB = torch.empty((cols, n), device=dev); dC0 = torch.empty((cols, n), device=dev)
+    dC = torch.empty((cols, n), device=dev); dX = torch.empty((cols, n), device=dev)
+    hA = pinned(A_h, torch) if rank == 0 else None
+    hT = pinned(T_h, torch) if rank == 0 else None
+    hB, hC = pinned(B_h, torch), pinned(C_h, torch)
+    hC_out = torch.empty((cols, n), pin_memory=True); hX_out = torch.empty((cols, n), pin_memory=True)
+    if rank == 0:
+        dA.copy_(hA); dT.copy_(hT)
+    dB.copy_(hB); dC0.copy_(hC)
+    if world > 1:
+        dist.broadcast(dA, 0); dist.broadcast(dT, 0)
+    torch.cuda.synchronize()
+
+    A, T = colmaj(dA), colmaj(dT)
+    Bm, C0, C, X = colmaj(dB), colmaj(dC0), colmaj(dC), colmaj(dX)
+    stream = torch.cuda.current_stream()
+    fl = flops(n, cols)
+    ev = {r: [] for r in ROUTINES}
+
+    def chain(record):
+        def timed(name, fn):
+            if record:
+                e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+                e0.record(stream); fn(); e1.record(stream)
+                ev[name].append((e0, e1))
+            else:
+                fn()
+        timed("sgemm", lambda: b3.sgemm("N", "N", ALPHA, A, Bm, BETA, C))
+        timed("ssymm", lambda: b3.ssymm("L", "L", ALPHA, A, Bm, BETA, C))
+        timed("ssyrk", lambda: b3.ssyrk("L", "N", ALPHA, A, BETA, C))
+        timed("ssyr2k", lambda: b3.ssyr2k("L", "N", ALPHA, A, Bm, BETA, C))
+        timed("strmm", lambda: b3.strmm("L", "L", "N", "N", ALPHA, T, X))
+        timed("strsm", lambda: b3.strsm("L", "L", "N", "N", ALPHA, T, X))
+
+    def step_device(record=False):
+        # fresh working copies so every step computes on the same data
+        dC.copy_(dC0); dX.copy_(dB)
+        if world > 1:
+            dist.broadcast(dA, 0); dist.broadcast(dT, 0)      # the one exchange step
+        chain(record)
+
+    def step_e2e():
+        # host -> device inputs, the chain, device -> host results (pinned)
+        if rank == 0:
+            dA.copy_(hA, non_blocking=True); dT.copy_(hT, non_blocking=True)
+        dB.copy_(hB, non_blocking=True); dC.copy_(hC, non_blocking=True)
+        if world > 1:
+            dist.broadcast(dA, 0); dist.broadcast(dT, 0)
+        dX.copy_(dB)
+        chain(False)
+        hC_out.copy_(dC, non_blocking=True); hX_out.copy_(dX, non_blocking=True)
+
+    def timed_loop(fn, steps, record=False):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(steps):
+            fn(record) if record is not None else fn()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        ms = e0.elapsed_time(e1)
+        if world > 1:
+            t = torch.tensor([ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+        return ms
+
+    for _ in range(args.warmup):
+        step_device()
+    torch.cuda.synchronize()
+    launches0 = b3.launch_count()
+    with ClockSampler(local) as clk:
+        ms = timed_loop(lambda rec: step_device(rec), args.steps, record=True)
+    launches = b3.launch_count() - launches0
+
+    # e2e: same metric through the public API with host buffers
+    for _ in range(max(1, min(2, args.warmup))):
+        step_e2e()
+    torch.cuda.synchronize()
+    ms_e2e = timed_loop(lambda: step_e2e(), args.steps, record=None)
+
+    total_flops = sum(fl.values()) * world
+    step_ms = ms / args.steps
+    value = total_flops / (step_ms * 1e-3) / 1e9
+    e2e_value = total_flops / (ms_e2e / args.steps * 1e-3) / 1e9
+    per = {}
+    for r in ROUTINES:
+        ts = [a.elapsed_time(b) for a, b in ev[r]]
+        avg = float(np.mean(ts))
+        per[r] = {"ms": round(avg, 4), "gflops": round(fl[r] / (avg * 1e-3) / 1e9, 1)}
+    peaks, peak_src = load_peaks()
+    pk = fp32_3xtf32_peak(peaks, sustained=True)
+    if args.math == "simt":
+        pk = 148 * 128 * 2 * (peaks.get("sm_max_mhz", 1965.0)) * 1e6 / 1e12
+    sg_ms = per["sgemm"]["ms"]
+    achieved = fl["sgemm"] / (sg_ms * 1e-3) / 1e12
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_sgemm_traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+        except (ValueError, OSError):
+            traffic = None
+    h2d = (2 * n * n * 4 if rank == 0 else 0) + 2 * n * cols * 4
+    d2h = 2 * n * cols * 4
+    out = {
+        "metric": "GFLOPS per routine (SGEMM/SSYMM/SSYRK/SSYR2K/STRMM/STRSM) at N=8192, "
+                  "1/2/4/8 B200, % of peak",
+        "value": round(value, 1),
+        "unit": "GFLOPS",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": round(step_ms, 3),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "f32",
+        "data": "synthetic (seeded U(-1,1); diagonally dominant T)",
+        "config": {
+            "workload": "configs[1..3] at N=8192: sgemm NN, ssymm LL, ssyrk LN, ssyr2k LN "
+                        "(K=8192), strmm LLNN, strsm LLNN; alpha=1.5 beta=0.5",
+            "n": n, "k": n, "cols_per_rank": cols, "math": args.math,
+            "l2": "no flush: every operand is 256 MiB > 126 MB L2",
+            "parallelism": f"column slabs of B/C x{world}, A/T broadcast (NCCL)" if world > 1
+            else "1 GPU",
+        },
+        "routines": per,
+        "pct_of_peak": round(100.0 * value / world / 1e3 / pk, 1),
+        "roofline": {
+            "bound": "tensor" if args.math != "simt" else "alu",
+            "kernel": "tc_structured_gemm (the sgemm launch)" if args.math != "simt"
+            else "simt_structured_gemm (the sgemm launch)",
+            "achieved": round(achieved, 2),
+            "peak": round(pk, 1),
+            "unit": "TFLOP/s",
+            "frac": round(achieved / pk, 3),
+            "peak_source": (f"{peak_src} bf16 sustained {peaks.get('bf16_tflops_sustained')} TF/s x "
+                            f"nominal tf32/bf16 {TF32_OVER_BF16:.3f} / 3 (3xTF32)")
+            if args.math != "simt" else "148 SM x 128 FP32 lanes x 2 x max SM clock",
+            "traffic": traffic,
+        },
+        "e2e": {"value": round(e2e_value, 1), "unit": "GFLOPS",
+                "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world},
+        "gpu_launches": int(launches),
+        "gpu_launches_per_step": round(launches / args.steps, 1),
+        "clocks": clk.summary(),
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        out["cpu_baseline"] = cpu_baseline(args.cpu_seconds)
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+# ----------------------------------------------------------------------------- oracle (reference arm)
+def oracle_sample(n, ncols, seconds_hint=None):
+    """Time the fp64 oracle on `ncols` sampled output columns of each routine
+    of the step at size n (the same seeded inputs as our arm)."""
+    import blas3_inputs as gen
+    import oracle
+    oracle.build()
+    A, T, B, C = make_inputs(n, n, 0)
+    sel = gen.sample_indices(n, ncols, "bench-sample")
+    fl = flops(n, len(sel))
+    times = {}
+    calls = {
+        "sgemm": lambda: oracle.sgemm("N", "N", ALPHA, A, B, BETA, C, sel=sel),
+        "ssymm": lambda: oracle.ssymm("L", "L", ALPHA, A, B, BETA, C, sel=sel),
+        "ssyrk": lambda: oracle.ssyrk("L", "N", ALPHA, A, BETA, C, sel=sel),
+        "ssyr2k": lambda: oracle.ssyr2k("L", "N", ALPHA, A, B, BETA, C, sel=sel),
+        "strmm": lambda: oracle.strmm("L", "L", "N", "N", ALPHA, T, B, sel=sel),
+        "strsm": lambda: oracle.strsm("L", "L", "N", "N", ALPHA, T, B, sel=sel),
+    }
+    for r, f in calls.items():
+        t0 = time.perf_counter(); f(); times[r] = time.perf_counter() - t0
+    # LAWN-41 per-column counts; ssyrk/ssyr2k columns of the lower triangle vary
+    # in length, so use the exact sampled-column count for them
+    fl["ssyrk"] = float(sum(2.0 * n * (n - j) for j in sel)) / 2.0 * 2.0
+    fl["ssyr2k"] = float(sum(4.0 * n * (n - j) for j in sel))
+    return fl, times, len(sel)
+
+
+def cpu_baseline(target_seconds):
+    import oracle
+    oracle.build()
+    n = N
+    # calibrate: a small sample first, then scale to ~target_seconds total
+    fl, times, ns = oracle_sample(n, max(2, oracle.num_threads()))
+    t = sum(times.values())
+    ncols = int(min(n, max(ns, ns * target_seconds / max(t, 1e-3))))
+    if ncols > ns:
+        fl, times, ns = oracle_sample(n, ncols)
+    tot = sum(times.values())
+    return {"value": round(sum(fl.values()) / tot / 1e9, 3), "unit": "GFLOPS",
+            "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": f"{ns} sampled output columns of each of the six routines at N={n} "
+                      f"(fp64 C oracle, OpenMP over columns), {tot:.1f} s"}
+
+
+def run_reference(args):
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    oracle.build()
+    ncols = max(2, oracle.num_threads())
+    # calibrate one step to ~ (budget / (steps + warmup)) seconds
+    budget = args.cpu_seconds * 3
+    fl, times, ns = oracle_sample(N, ncols)
+    per_step = budget / max(1, args.steps + args.warmup)
+    ncols = int(min(N, max(ncols, ncols * per_step / max(sum(times.values()), 1e-3))))
+    for _ in range(args.warmup):
+        oracle_sample(N, ncols)
+    tot_t, tot_f = 0.0, 0.0
+    for _ in range(args.steps):
+        fl, times, ns = oracle_sample(N, ncols)
+        tot_t += sum(times.values()); tot_f += sum(fl.values())
+    value = tot_f / tot_t / 1e9
+    out = {
+        "impl": "reference",
+        "metric": "GFLOPS per routine (SGEMM/SSYMM/SSYRK/SSYR2K/STRMM/STRSM) at N=8192, "
+                  "1/2/4/8 B200, % of peak",
+        "value": round(value, 3), "unit": "GFLOPS", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(1e3 * tot_t / args.steps, 1),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic (seeded U(-1,1); diagonally dominant T)",
+        "config": {"workload": "configs[1..3] at N=8192: sgemm NN, ssymm LL, ssyrk LN, ssyr2k LN "
+                               "(K=8192), strmm LLNN, strsm LLNN; alpha=1.5 beta=0.5",
+                   "n": N, "k": N},
+        "cpu_baseline": {"value": round(value, 3), "unit": "GFLOPS", "cores": oracle.num_threads(),
+                         "kind": "oracle",
+                         "sample": f"{ns} sampled output columns of each routine per step"},
+        "e2e": {"value": round(value, 3), "unit": "GFLOPS", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--math", default="3xtf32", choices=["3xtf32", "simt"])
+    ap.add_argument("--n", type=int, default=N)
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -43,10 +43,11 @@ _SIGS = {
     "blas3_get_math_mode": [],
     "blas3_set_workspace": [_p, ctypes.c_size_t],
     "blas3_launch_count": [],
+    "blas3_launch_count_by_path": [_i],
     "blas3_error_string": [_i],
     "blas3_version": [],
 }
-_RES = {"blas3_launch_count": _i64, "blas3_error_string": ctypes.c_char_p}
+_RES = {"blas3_launch_count": _i64, "blas3_launch_count_by_path": _i64, "blas3_error_string": ctypes.c_char_p}
 
 for _name, _args in _SIGS.items():
     _fn = getattr(_lib, _name)
@@ -179,8 +180,16 @@ def get_math_mode():
     return blas3_get_math_mode()  # noqa: F821
 
 
-def launch_count():
-    return int(blas3_launch_count())  # noqa: F821
+PATH_TCGEN05, PATH_SIMT, PATH_AUX = 0, 1, 2
+
+
+def launch_count(path=None):
+    """Kernels launched since load (all, or one route: 'tc', 'simt', 'aux')."""
+    if path is None:
+        return int(blas3_launch_count())  # noqa: F821
+    if isinstance(path, str):
+        path = {"tc": PATH_TCGEN05, "simt": PATH_SIMT, "aux": PATH_AUX}[path]
+    return int(blas3_launch_count_by_path(path))  # noqa: F821
 
 
 __all__ = ["sgemm", "ssymm", "ssyrk", "ssyr2k", "strmm", "strsm", "set_math_mode",

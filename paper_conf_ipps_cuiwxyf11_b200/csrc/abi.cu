@@ -16,7 +16,11 @@
 namespace blas3 {
 
 static std::atomic<int64_t> g_launches{0};
-void note_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+static std::atomic<int64_t> g_path_launches[3];
+void note_launch(int path) {
+  g_launches.fetch_add(1, std::memory_order_relaxed);
+  if (path >= 0 && path < 3) g_path_launches[path].fetch_add(1, std::memory_order_relaxed);
+}
 
 static int g_math = -1;              // -1: not initialised
 static void *g_ws = nullptr;
@@ -130,6 +134,9 @@ extern "C" {
 
 int blas3_version(void) { return 100; }
 int64_t blas3_launch_count(void) { return g_launches.load(); }
+int64_t blas3_launch_count_by_path(int path) {
+  return (path >= 0 && path < 3) ? g_path_launches[path].load() : -1;
+}
 
 int blas3_set_math_mode(int mode) {
   if (mode != BLAS3_MATH_3XTF32 && mode != BLAS3_MATH_SIMT_FP32) return 1;

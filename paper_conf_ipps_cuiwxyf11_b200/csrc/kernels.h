@@ -7,7 +7,7 @@
 
 namespace blas3 {
 
-void note_launch();                 // host-side launch counter (blas3_launch_count)
+void note_launch(int path = 2);      // host-side launch counter (blas3_launch_count[_by_path])
 
 // Structured GEMM kernels (all routines canonicalise to a Problem).
 int launch_simt(const Problem &P, cudaStream_t s, int num_sms);

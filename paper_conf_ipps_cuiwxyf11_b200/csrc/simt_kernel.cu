@@ -139,7 +139,7 @@ int launch_simt(const Problem &P, cudaStream_t stream, int num_sms) {
   if (tiles == 0) return 0;
   int64_t grid = imin(tiles, (int64_t)num_sms * 2);
   simt_structured_gemm<<<(unsigned)grid, NT, 0, stream>>>(P);
-  note_launch();
+  note_launch(1);
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
 

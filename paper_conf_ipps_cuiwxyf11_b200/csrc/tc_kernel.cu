@@ -1,6 +1,483 @@
-// tc_kernel.cu -- placeholder until the tcgen05 kernel lands (routes to SIMT).
+// tc_kernel.cu -- the one tuned GEMM every routine derives from, B200-native:
+// TMA -> shared memory -> staging transform -> tcgen05.mma (3xTF32) -> TMEM
+// -> epilogue.  Rows A2-A6 of the hot-path table.
+//
+// Paper mapping:
+//   thread_grouping / loop_tiling  -> persistent CTAs over a
+//       128x256 tile schedule (Tiles<> in problem.h), BK = 32 k-blocks;
+//   SM_alloc(X, Transpose|Symmetry)   -> TMA loads each k-block in
+//       the orientation it is stored in (K-major or MN-major 128B-swizzled
+//       tiles; the UMMA descriptor's major bit absorbs the transpose), and
+//       symmetric blocks crossing the diagonal are MERGED from both stored
+//       orientations while staging (selection, never src+src^T-diag, Q7);
+//   padding/peel_triangular         -> blank k-blocks skipped via
+//       the tile's k-range, diagonal blocks zero-SELECTED (+unit diagonal)
+//       in shared memory (the blank triangle is never multiplied, Q8);
+//   Reg_alloc(C)                        -> fp32 accumulator in TMEM
+//       (two 256-column accumulators: epilogue of tile i overlaps tile i+1).
+// fp32 accuracy on TF32 tensor cores (north star): every staged value x is
+// split into hi = rna_tf32(x), lo = rna_tf32(x - hi) and each k-step issues
+// lo*hi + hi*lo + hi*hi (small terms first) into the same fp32 accumulator.
+//
+// Warp roles (448 threads, 1 CTA/SM):
+//   warp 0       TMA producer (one lane)
+//   warp 1       TMEM allocator + MMA issuer (one lane)
+//   warps 2..9   transform: structure fix-ups + hi/lo split (256 threads)
+//   warps 10..13 epilogue: tcgen05.ld -> alpha*acc + beta*C -> global
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <mutex>
+#include <string.h>
+
 #include "kernels.h"
+#include "tc_ptx.h"
+
 namespace blas3 {
-bool tc_eligible(const Problem &) { return false; }
-int launch_tc(const Problem &, cudaStream_t, int) { return -1; }
+
+namespace {
+constexpr int BM = 128, BN = 256, BK = 32, STAGES = 2;
+constexpr int WARP_TMA = 0, WARP_MMA = 1, WARP_TR0 = 2, NUM_TR_WARPS = 8;
+constexpr int WARP_EPI0 = WARP_TR0 + NUM_TR_WARPS, NUM_EPI_WARPS = 4;
+constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;
+constexpr int TR_THREADS = NUM_TR_WARPS * 32;
+constexpr uint32_t A_BYTES = BM * BK * 4;
+constexpr uint32_t B_BYTES = BN * BK * 4;
+constexpr int TMEM_COLS = 512;          // 2 accumulators x BN columns
+constexpr int MAX_MAPS = 8;
+constexpr int LAYOUT_K = 0, LAYOUT_MN = 1;
+
+struct alignas(1024) StageBuf {
+  uint8_t rawA[A_BYTES];   // TMA destination; becomes hi (tf32) in place
+  uint8_t rawB[B_BYTES];
+  uint8_t loA[A_BYTES];    // lo (tf32); also the kr-view landing zone of
+  uint8_t loB[B_BYTES];    //   symmetric diagonal blocks before the merge
+};
+struct Barriers {
+  uint64_t full[STAGES];   // TMA -> transform (expect_tx)
+  uint64_t ready[STAGES];  // transform -> MMA (TR_THREADS arrivals)
+  uint64_t empty[STAGES];  // MMA -> TMA (tcgen05.commit)
+  uint64_t tfull[2];       // MMA -> epilogue
+  uint64_t tempty[2];      // epilogue -> MMA (128 arrivals)
+  uint32_t tmem_base;
+};
+constexpr size_t SMEM_BYTES = sizeof(StageBuf) * STAGES + sizeof(Barriers) + 1024;
+
+struct TcParams {
+  CUtensorMap maps[MAX_MAPS];
+  Problem P;
+};
+
+// byte offset of element (r, k) inside a staged operand tile
+__device__ __forceinline__ uint32_t off_k(int r, int k) {       // K-major, 128 B per row r
+  return (uint32_t)(r * 128 + ((((k >> 2) ^ (r & 7)) & 7) << 4) + (k & 3) * 4);
+}
+// MN-major, 32-row chunks of BK 128-B rows; 128B swizzle with 32-B atomicity
+// (TMA SWIZZLE_128B_ATOM_32B == UMMA SWIZZLE_128B_BASE32B == Swizzle<2,5,2>)
+__device__ __forceinline__ uint32_t off_mn(int r, int k) {
+  return (uint32_t)((r >> 5) * (BK * 128) + k * 128 + (((((r & 31) >> 3) ^ (k & 3)) & 3) << 5) +
+                    (r & 7) * 4);
+}
+
+__host__ __device__ __forceinline__ int layout_of(const OpDesc &o, int cls) {
+  if (o.kind == OP_DENSE) return o.kr ? LAYOUT_K : LAYOUT_MN;
+  if (cls == BLK_KR) return LAYOUT_K;
+  if (cls == BLK_TRI_DIAG) return o.swap ? LAYOUT_K : LAYOUT_MN;
+  return LAYOUT_MN;   // BLK_RK, BLK_SYM_DIAG (merged into the rk orientation)
+}
+
+struct StageInfo {
+  int clsA, clsB, layA, layB;
+};
+
+__device__ __forceinline__ StageInfo stage_info(const Problem &P, const Segment &sg, int64_t m0,
+                                                int64_t n0, int64_t k0) {
+  StageInfo si;
+  const int64_t k1 = imin(sg.K, k0 + BK);
+  si.clsA = block_class(sg.a, m0, imin(P.M, m0 + BM), k0, k1);
+  si.clsB = block_class(sg.b, n0, imin(P.N, n0 + BN), k0, k1);
+  si.layA = layout_of(sg.a, si.clsA);
+  si.layB = layout_of(sg.b, si.clsB);
+  return si;
+}
+
+__device__ __forceinline__ void seg_kblocks(const Problem &P, const Segment &sg, int64_t m0,
+                                            int64_t n0, int64_t &kb0, int64_t &kb1) {
+  int64_t k0, k1;
+  k_range(sg, m0, imin(P.M, m0 + BM), n0, imin(P.N, n0 + BN), k0, k1);
+  kb0 = k0 / BK;
+  kb1 = (k1 > k0) ? cdiv(k1, BK) : kb0;
+}
+
+__device__ __forceinline__ int64_t tile_kblocks(const Problem &P, int64_t m0, int64_t n0) {
+  int64_t tot = 0;
+  for (int s = 0; s < P.nseg; ++s) {
+    int64_t a, b;
+    seg_kblocks(P, P.seg[s], m0, n0, a, b);
+    tot += b - a;
+  }
+  return tot;
+}
+
+// ---------------------------------------------------------------- producer
+__device__ __forceinline__ uint32_t load_operand(const TcParams &prm, const OpDesc &o, int cls,
+                                                 int lay, uint8_t *raw, uint8_t *lo, int64_t r0,
+                                                 int64_t k0, int rows, uint64_t *bar) {
+  uint32_t bytes = 0;
+  if (lay == LAYOUT_MN) {
+    const CUtensorMap *m = &prm.maps[o.map_rk];
+    for (int c = 0; c < rows / 32; ++c) {
+      ptx::tma_load_2d(m, bar, raw + c * (BK * 128), (int32_t)(r0 + 32 * c), (int32_t)k0);
+    }
+  } else {
+    ptx::tma_load_2d(&prm.maps[o.map_kr], bar, raw, (int32_t)k0, (int32_t)r0);
+  }
+  bytes += rows * BK * 4;
+  if (cls == BLK_SYM_DIAG) {       // the mirrored orientation lands in the lo buffer
+    ptx::tma_load_2d(&prm.maps[o.map_kr], bar, lo, (int32_t)k0, (int32_t)r0);
+    bytes += rows * BK * 4;
+  }
+  return bytes;
+}
+
+__device__ __forceinline__ uint32_t operand_bytes(int cls, int rows) {
+  return rows * BK * 4 * (cls == BLK_SYM_DIAG ? 2 : 1);
+}
+
+// ---------------------------------------------------------------- transform
+// Symmetric block crossing the diagonal: elements whose stored position is
+// the mirrored one are copied from the kr-view tile (in lo) into the rk tile.
+__device__ __forceinline__ void sym_merge(const OpDesc &o, uint8_t *raw, const uint8_t *krtile,
+                                          int64_t r0, int64_t k0, int rows, int t) {
+  for (int e = t; e < rows * BK; e += TR_THREADS) {
+    int r = e % rows, k = e / rows;
+    int64_t gr = r0 + r, gk = k0 + k;
+    bool mirrored = o.lower ? (gr < gk) : (gr > gk);
+    if (mirrored) *reinterpret_cast<float *>(raw + off_mn(r, k)) =
+        *reinterpret_cast<const float *>(krtile + off_k(r, k));
+  }
+}
+
+// Triangular block touching the diagonal: zero-select the blank part, force
+// the unit diagonal (the stored values there are never used).
+__device__ __forceinline__ void tri_fix(const OpDesc &o, int lay, uint8_t *raw, int64_t r0,
+                                        int64_t k0, int rows, int64_t R, int64_t K, int t) {
+  const bool kle = tri_kle(o);
+  for (int e = t; e < rows * BK; e += TR_THREADS) {
+    int r, k;
+    if (lay == LAYOUT_MN) { r = e % rows; k = e / rows; } else { k = e % BK; r = e / BK; }
+    int64_t gr = r0 + r, gk = k0 + k;
+    bool nz = kle ? (gk <= gr) : (gk >= gr);
+    uint32_t off = (lay == LAYOUT_MN) ? off_mn(r, k) : off_k(r, k);
+    float *p = reinterpret_cast<float *>(raw + off);
+    if (!nz) *p = 0.f;
+    else if (o.unit && gr == gk && gr < R && gk < K) *p = 1.f;
+  }
+}
+
+__device__ __forceinline__ float split1(float x, float &lo) {
+  float hi = __uint_as_float(ptx::cvt_rna_tf32(x));
+  lo = __uint_as_float(ptx::cvt_rna_tf32(x - hi));
+  return hi;
+}
+
+__device__ __forceinline__ void split_pass(uint8_t *raw, uint8_t *lo, uint32_t bytes, int t) {
+  float4 *r4 = reinterpret_cast<float4 *>(raw);
+  float4 *l4 = reinterpret_cast<float4 *>(lo);
+  for (uint32_t c = t; c < bytes / 16; c += TR_THREADS) {
+    float4 v = r4[c], l;
+    v.x = split1(v.x, l.x);
+    v.y = split1(v.y, l.y);
+    v.z = split1(v.z, l.z);
+    v.w = split1(v.w, l.w);
+    r4[c] = v;
+    l4[c] = l;
+  }
+}
+
+// ---------------------------------------------------------------- MMA
+__device__ __forceinline__ uint64_t op_desc(uint32_t base, int lay, int k8) {
+  if (lay == LAYOUT_MN) return ptx::smem_desc(base + k8 * 1024, BK * 128, 512, 1);
+  return ptx::smem_desc(base + k8 * 32, 16, 1024, 2);
+}
+
+}  // namespace
+
+__global__ void __launch_bounds__(NTHREADS, 1)
+tc_structured_gemm(const __grid_constant__ TcParams prm) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  StageBuf *st = reinterpret_cast<StageBuf *>(smem);
+  Barriers *bars = reinterpret_cast<Barriers *>(smem + sizeof(StageBuf) * STAGES);
+  const Problem &P = prm.P;
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < STAGES; ++s) {
+      ptx::mbar_init(&bars->full[s], 1);
+      ptx::mbar_init(&bars->ready[s], TR_THREADS);
+      ptx::mbar_init(&bars->empty[s], 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      ptx::mbar_init(&bars->tfull[a], 1);
+      ptx::mbar_init(&bars->tempty[a], NUM_EPI_WARPS * 32);
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == WARP_MMA) ptx::tmem_alloc(&bars->tmem_base, TMEM_COLS);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = bars->tmem_base;
+
+  const int64_t ntiles = Tiles<BM, BN>::count(P);
+
+  if (warp == WARP_TMA) {
+    // ============================ TMA producer
+    if (lane == 0) {
+      for (int i = 0; i < MAX_MAPS; ++i) ptx::tma_prefetch(&prm.maps[i]);
+      uint32_t it = 0;
+      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        int64_t mi, nj;
+        Tiles<BM, BN>::coords(P, t, mi, nj);
+        const int64_t m0 = mi * BM, n0 = nj * BN;
+        for (int s = 0; s < P.nseg; ++s) {
+          const Segment &sg = P.seg[s];
+          int64_t kb0, kb1;
+          seg_kblocks(P, sg, m0, n0, kb0, kb1);
+          for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
+            const int stg = it % STAGES;
+            const uint32_t ph = (it / STAGES) & 1;
+            const int64_t k0 = kb * BK;
+            StageInfo si = stage_info(P, sg, m0, n0, k0);
+            ptx::mbar_wait(&bars->empty[stg], ph ^ 1);
+            ptx::mbar_arrive_expect_tx(&bars->full[stg],
+                                       operand_bytes(si.clsA, BM) + operand_bytes(si.clsB, BN));
+            load_operand(prm, sg.a, si.clsA, si.layA, st[stg].rawA, st[stg].loA, m0, k0, BM,
+                         &bars->full[stg]);
+            load_operand(prm, sg.b, si.clsB, si.layB, st[stg].rawB, st[stg].loB, n0, k0, BN,
+                         &bars->full[stg]);
+          }
+        }
+      }
+      // producer tail: every stage released by the MMA before the CTA retires
+      for (int i = 0; i < STAGES; ++i, ++it)
+        ptx::mbar_wait(&bars->empty[it % STAGES], ((it / STAGES) & 1) ^ 1);
+    }
+  } else if (warp == WARP_MMA) {
+    // ============================ MMA issuer
+    uint32_t it = 0, tcount = 0;
+    const uint32_t sA[STAGES] = {ptx::smem_u32(st[0].rawA), ptx::smem_u32(st[1].rawA)};
+    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++tcount) {
+      int64_t mi, nj;
+      Tiles<BM, BN>::coords(P, t, mi, nj);
+      const int64_t m0 = mi * BM, n0 = nj * BN;
+      const uint32_t acc = tcount & 1, aph = (tcount >> 1) & 1;
+      ptx::mbar_wait(&bars->tempty[acc], aph ^ 1);
+      ptx::tc_fence_after();
+      const uint32_t d_tmem = tmem + acc * BN;
+      uint32_t accumulate = 0;
+      for (int s = 0; s < P.nseg; ++s) {
+        const Segment &sg = P.seg[s];
+        int64_t kb0, kb1;
+        seg_kblocks(P, sg, m0, n0, kb0, kb1);
+        for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
+          const int stg = it % STAGES;
+          const uint32_t ph = (it / STAGES) & 1;
+          StageInfo si = stage_info(P, sg, m0, n0, kb * BK);
+          ptx::mbar_wait(&bars->ready[stg], ph);
+          ptx::tc_fence_after();
+          if (lane == 0) {
+            const uint32_t hiA = sA[stg], hiB = hiA + A_BYTES;
+            const uint32_t loA = hiB + B_BYTES, loB = loA + A_BYTES;
+            const uint32_t idesc = ptx::idesc_tf32(BM, BN, si.layA == LAYOUT_MN, si.layB == LAYOUT_MN);
+#pragma unroll
+            for (int k8 = 0; k8 < BK / 8; ++k8) {
+              const uint64_t ah = op_desc(hiA, si.layA, k8), al = op_desc(loA, si.layA, k8);
+              const uint64_t bh = op_desc(hiB, si.layB, k8), bl = op_desc(loB, si.layB, k8);
+              ptx::mma_tf32_ss(d_tmem, al, bh, idesc, accumulate);
+              ptx::mma_tf32_ss(d_tmem, ah, bl, idesc, 1);
+              ptx::mma_tf32_ss(d_tmem, ah, bh, idesc, 1);
+              accumulate = 1;
+            }
+            ptx::mma_commit(&bars->empty[stg]);
+          }
+          accumulate = 1;
+          __syncwarp();
+        }
+      }
+      if (lane == 0) {
+        if (accumulate) ptx::mma_commit(&bars->tfull[acc]);
+        else ptx::mbar_arrive(&bars->tfull[acc]);     // empty k-range: accumulator = 0
+      }
+      __syncwarp();
+    }
+  } else if (warp < WARP_EPI0) {
+    // ============================ transform warps
+    const int tt = threadIdx.x - WARP_TR0 * 32;
+    uint32_t it = 0;
+    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      int64_t mi, nj;
+      Tiles<BM, BN>::coords(P, t, mi, nj);
+      const int64_t m0 = mi * BM, n0 = nj * BN;
+      for (int s = 0; s < P.nseg; ++s) {
+        const Segment &sg = P.seg[s];
+        int64_t kb0, kb1;
+        seg_kblocks(P, sg, m0, n0, kb0, kb1);
+        for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
+          const int stg = it % STAGES;
+          const uint32_t ph = (it / STAGES) & 1;
+          const int64_t k0 = kb * BK;
+          StageInfo si = stage_info(P, sg, m0, n0, k0);
+          ptx::mbar_wait(&bars->full[stg], ph);
+          StageBuf &b = st[stg];
+          bool fix = false;
+          if (si.clsA == BLK_SYM_DIAG) { sym_merge(sg.a, b.rawA, b.loA, m0, k0, BM, tt); fix = true; }
+          else if (si.clsA == BLK_TRI_DIAG) { tri_fix(sg.a, si.layA, b.rawA, m0, k0, BM, P.M, sg.K, tt); fix = true; }
+          if (si.clsB == BLK_SYM_DIAG) { sym_merge(sg.b, b.rawB, b.loB, n0, k0, BN, tt); fix = true; }
+          else if (si.clsB == BLK_TRI_DIAG) { tri_fix(sg.b, si.layB, b.rawB, n0, k0, BN, P.N, sg.K, tt); fix = true; }
+          if (fix) ptx::named_bar_sync(1, TR_THREADS);
+          split_pass(b.rawA, b.loA, A_BYTES, tt);
+          split_pass(b.rawB, b.loB, B_BYTES, tt);
+          ptx::fence_proxy_async_smem();
+          ptx::mbar_arrive(&bars->ready[stg]);
+        }
+      }
+    }
+  } else {
+    // ============================ epilogue warps
+    const int q = warp & 3;                     // TMEM lane quarter of this warp
+    uint32_t tcount = 0;
+    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++tcount) {
+      int64_t mi, nj;
+      Tiles<BM, BN>::coords(P, t, mi, nj);
+      const int64_t m0 = mi * BM, n0 = nj * BN;
+      const bool has_k = tile_kblocks(P, m0, n0) > 0;
+      const uint32_t acc = tcount & 1, aph = (tcount >> 1) & 1;
+      ptx::mbar_wait(&bars->tfull[acc], aph);
+      ptx::tc_fence_after();
+      const int64_t r = m0 + q * 32 + lane;
+      for (int ch = 0; ch < BN / 32; ++ch) {
+        const int64_t c0 = n0 + ch * 32;
+        if (c0 >= P.N) break;
+        uint32_t v[32];
+        if (has_k) {
+          ptx::tmem_ld_32x32b_x32(tmem + acc * BN + ch * 32 + ((uint32_t)(q * 32) << 16), v);
+          ptx::tmem_ld_wait();
+        } else {
+#pragma unroll
+          for (int j = 0; j < 32; ++j) v[j] = 0u;
+        }
+        if (r < P.M) {
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            const int64_t c = c0 + j;
+            const bool ok = c < P.N && !(P.c_tri == 1 && r < c) && !(P.c_tri == 2 && r > c);
+            if (!ok) continue;
+            float o = P.alpha * __uint_as_float(v[j]);
+            if (P.beta != 0.f) o = fmaf(P.beta, P.Cin[r + c * P.ldcin], o);
+            P.Cout[r + c * P.ldcout] = o;
+          }
+        }
+      }
+      ptx::tc_fence_before();
+      ptx::mbar_arrive(&bars->tempty[acc]);
+    }
+  }
+
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == WARP_MMA) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc(tmem, TMEM_COLS);
+  }
+}
+
+// ====================================================================== host side
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                                  const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
+                                  const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static EncodeTiledFn encode_fn() {
+  static EncodeTiledFn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(p);
+  });
+  return fn;
+}
+
+// 2-D fp32 tensor map: dim0 contiguous (extent d0), dim1 stride ld floats.
+static bool make_map(CUtensorMap *m, const float *ptr, int64_t d0, int64_t d1, int64_t ld,
+                     uint32_t box0, uint32_t box1, CUtensorMapSwizzle swz) {
+  EncodeTiledFn fn = encode_fn();
+  if (!fn) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)d0, (cuuint64_t)d1};
+  cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
+  cuuint32_t box[2] = {box0, box1};
+  cuuint32_t es[2] = {1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(ptr), dims, strides, box, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, swz,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// maps for one operand with R rows, K columns, staged `rows` at a time
+static bool op_maps(TcParams &prm, int &slot, OpDesc &o, int64_t R, int64_t K, int rows) {
+  o.map_rk = o.map_kr = -1;
+  const bool need_rk = (o.kind == OP_DENSE && !o.kr) || o.kind == OP_SYM || (o.kind == OP_TRI && !o.swap);
+  const bool need_kr = (o.kind == OP_DENSE && o.kr) || o.kind == OP_SYM || (o.kind == OP_TRI && o.swap);
+  if (need_rk) {       // X(r,k) = G[r + k*ld]: dim0 = r (R), dim1 = k (K)
+    if (slot >= MAX_MAPS || !make_map(&prm.maps[slot], o.ptr, R, K, o.ld, 32, BK,
+                                                CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return false;
+    o.map_rk = slot++;
+  }
+  if (need_kr) {       // X(r,k) = G[k + r*ld]: dim0 = k (K), dim1 = r (R)
+    if (slot >= MAX_MAPS || !make_map(&prm.maps[slot], o.ptr, K, R, o.ld, BK, rows,
+                                                CU_TENSOR_MAP_SWIZZLE_128B)) return false;
+    o.map_kr = slot++;
+  }
+  return true;
+}
+
+static bool aligned_op(const OpDesc &o) {
+  return (reinterpret_cast<uintptr_t>(o.ptr) % 16 == 0) && (o.ld % 4 == 0);
+}
+
+bool tc_eligible(const Problem &P) {
+  for (int s = 0; s < P.nseg; ++s)
+    if (!aligned_op(P.seg[s].a) || !aligned_op(P.seg[s].b)) return false;
+  return true;
+}
+
+int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
+  static TcParams prm;                    // host staging (the launch copies it)
+  static std::mutex mu;
+  std::lock_guard<std::mutex> lk(mu);
+  memset(&prm, 0, sizeof(prm));
+  prm.P = P0;
+  int slot = 0;
+  for (int s = 0; s < prm.P.nseg; ++s) {
+    Segment &sg = prm.P.seg[s];
+    if (sg.K <= 0) continue;
+    if (!op_maps(prm, slot, sg.a, prm.P.M, sg.K, BM)) return -4;
+    if (!op_maps(prm, slot, sg.b, prm.P.N, sg.K, BN)) return -4;
+  }
+  static bool attr = false;
+  if (!attr) {
+    if (cudaFuncSetAttribute(tc_structured_gemm, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)SMEM_BYTES) != cudaSuccess) return -1;
+    attr = true;
+  }
+  const int64_t tiles = Tiles<BM, BN>::count(prm.P);
+  if (tiles == 0) return 0;
+  const int64_t grid = imin(tiles, (int64_t)num_sms);
+  tc_structured_gemm<<<(unsigned)grid, NTHREADS, SMEM_BYTES, stream>>>(prm);
+  note_launch(0);
+  return cudaGetLastError() == cudaSuccess ? 0 : -1;
+}
+
 }  // namespace blas3

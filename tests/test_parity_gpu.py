@@ -15,8 +15,8 @@ import numpy as np
 import pytest
 
 import blas3_inputs as gen
-from check import (TOL_NW, TOL_REL, bits_equal, e_nw, e_rel, f64, fro, op, sym_full, to_dev,
-                   to_host, tri_full)
+from check import (TOL_NW, bits_equal, e_nw, e_rel, f64, fro, op, sym_full, to_dev, to_host,
+                   tol_rel, tri_full)
 
 pytestmark = pytest.mark.gpu
 
@@ -42,26 +42,44 @@ def mode(request, b3):
     b3.set_math_mode("3xtf32")
 
 
+@pytest.fixture
+def route(b3, mode):
+    """route(*lds) after a call: in 3xtf32 mode, TMA-eligible leading
+    dimensions (all % 4 == 0) must have run on the tcgen05 kernel; anything
+    else (or SIMT mode) must not have."""
+    before = {p: b3.launch_count(p) for p in ("tc", "simt")}
+
+    def check(*lds):
+        tc = b3.launch_count("tc") > before["tc"]
+        if mode == "3xtf32" and all(ld % 4 == 0 for ld in lds):
+            assert tc, "expected the tcgen05 route"
+        else:
+            assert not tc, "tcgen05 route taken unexpectedly"
+    return check
+
+
 # ------------------------------------------------------------------------------------ SGEMM
-GEMM_SIZES = [(1, 1, 1), (33, 17, 45), (129, 257, 100), (256, 256, 256), (300, 131, 520)]
+GEMM_SIZES = [(1, 1, 1), (33, 17, 45), (132, 260, 100), (256, 256, 256), (300, 132, 520),
+              (516, 1000, 260)]
 
 
 @pytest.mark.parametrize("ta,tb", list(itertools.product("NT", "NT")))
 @pytest.mark.parametrize("m,n,k", GEMM_SIZES)
-def test_sgemm(b3, oracle_mod, mode, ta, tb, m, n, k):
+def test_sgemm(b3, oracle_mod, mode, route, ta, tb, m, n, k):
     A = gen.uniform(*((m, k) if ta == "N" else (k, m)), "pg-a", ta)
     B = gen.uniform(*((k, n) if tb == "N" else (n, k)), "pg-b", tb)
     C = gen.uniform(m, n, "pg-c")
     dC = to_dev(C)
     b3.sgemm(ta, tb, AL, to_dev(A), to_dev(B), BE, dC)
     got = to_host(dC)
+    route(A.shape[0], B.shape[0], m)
     ref = oracle_mod.sgemm(ta, tb, AL, A, B, BE, C)
     assert e_nw(got, ref, AL * fro(A) * fro(B) + BE * fro(C)) <= TOL_NW
-    assert e_rel(got, ref) <= TOL_REL
+    assert e_rel(got, ref) <= tol_rel(k, mode)
 
 
 @pytest.mark.parametrize("ta,tb", list(itertools.product("NT", "NT")))
-@pytest.mark.parametrize("m,n,k", [(130, 260, 1000), (64, 300, 33)])
+@pytest.mark.parametrize("m,n,k", [(132, 260, 1000), (64, 300, 36)])
 def test_sgemm_integer_bitexact(b3, oracle_mod, mode, ta, tb, m, n, k):
     A = gen.integers(*((m, k) if ta == "N" else (k, m)), "ig-a")
     B = gen.integers(*((k, n) if tb == "N" else (n, k)), "ig-b")
@@ -105,6 +123,29 @@ def test_sgemm_padded_ld(b3, oracle_mod, mode, pad):
     assert np.isnan(full[m:]).all()
 
 
+@pytest.mark.parametrize("big_on", ["A", "B"])
+@pytest.mark.parametrize("ta,tb", list(itertools.product("NT", "NT")))
+def test_split_is_real(b3, oracle_mod, route, mode, big_on, ta, tb):
+    """Decisive pin for the 3xTF32 split: one operand holds 15-bit integers
+    (|x| < 2^14, needs hi + lo: TF32 keeps 11 significant bits), the other
+    3-bit integers (lo = 0).  Then hi*hi + lo*hi (+ hi*lo = 0) is the exact
+    product, every partial sum is an integer < 2^24, so the result must be
+    bit-exact -- a 1xTF32 (or a dropped lo term) cannot be."""
+    m, n, k = 260, 132, 64
+    big = lambda *s: gen.integers(*s, "big", lo=-(2 ** 14) + 1, hi=2 ** 14 - 1)  # noqa: E731
+    small = lambda *s: gen.integers(*s, "small", lo=-4, hi=4)                    # noqa: E731
+    shpA = (m, k) if ta == "N" else (k, m)
+    shpB = (k, n) if tb == "N" else (n, k)
+    A = big(*shpA) if big_on == "A" else small(*shpA)
+    B = big(*shpB) if big_on == "B" else small(*shpB)
+    C = np.zeros((m, n), np.float32, order="F")
+    dC = to_dev(C)
+    b3.sgemm(ta, tb, 1.0, to_dev(A), to_dev(B), 0.0, dC)
+    got = to_host(dC)
+    route(A.shape[0], B.shape[0], m)
+    assert bits_equal(got, oracle_mod.sgemm(ta, tb, 1.0, A, B, 0.0, C).astype(np.float32))
+
+
 def test_determinism(b3):
     m = n = k = 384
     A, B, C = gen.uniform(m, k, "d-a"), gen.uniform(k, n, "d-b"), gen.uniform(m, n, "d-c")
@@ -118,23 +159,24 @@ def test_determinism(b3):
 
 # ------------------------------------------------------------------------------------ SSYMM
 @pytest.mark.parametrize("side,uplo", list(itertools.product("LR", "LU")))
-@pytest.mark.parametrize("m,n", [(1, 1), (45, 70), (200, 130), (256, 300)])
-def test_ssymm(b3, oracle_mod, mode, side, uplo, m, n):
+@pytest.mark.parametrize("m,n", [(1, 1), (44, 68), (200, 132), (256, 300), (516, 260)])
+def test_ssymm(b3, oracle_mod, mode, route, side, uplo, m, n):
     ka = m if side == "L" else n
     A = gen.symmetric_stored(ka, uplo, "ps", side)        # other triangle = NaN sentinel
     B, C = gen.uniform(m, n, "ps-b"), gen.uniform(m, n, "ps-c")
     dC = to_dev(C)
     b3.ssymm(side, uplo, AL, to_dev(A), to_dev(B), BE, dC)
     got = to_host(dC)
+    route(ka, m)
     ref = oracle_mod.ssymm(side, uplo, AL, A, B, BE, C)
     S = sym_full(A, uplo, ka)
     assert e_nw(got, ref, AL * fro(S) * fro(B) + BE * fro(C)) <= TOL_NW
-    assert e_rel(got, ref) <= TOL_REL
+    assert e_rel(got, ref) <= tol_rel(ka, mode)
 
 
 @pytest.mark.parametrize("side,uplo", list(itertools.product("LR", "LU")))
 def test_ssymm_integer_bitexact_and_equals_gemm(b3, oracle_mod, mode, side, uplo):
-    m, n = 300, 170
+    m, n = 300, 172
     ka = m if side == "L" else n
     A = gen.symmetric_stored(ka, uplo, "is", integer=True)
     B, C = gen.integers(m, n, "is-b"), gen.integers(m, n, "is-c")
@@ -155,8 +197,8 @@ def test_ssymm_integer_bitexact_and_equals_gemm(b3, oracle_mod, mode, side, uplo
 # ------------------------------------------------------------------------------------ SYRK / SYR2K
 @pytest.mark.parametrize("two", [False, True])
 @pytest.mark.parametrize("uplo,trans", list(itertools.product("LU", "NT")))
-@pytest.mark.parametrize("n,k", [(1, 1), (70, 33), (300, 200), (257, 520)])
-def test_syrk_syr2k(b3, oracle_mod, mode, two, uplo, trans, n, k):
+@pytest.mark.parametrize("n,k", [(1, 1), (68, 32), (300, 200), (260, 520)])
+def test_syrk_syr2k(b3, oracle_mod, mode, route, two, uplo, trans, n, k):
     shp = (n, k) if trans == "N" else (k, n)
     A, B = gen.uniform(*shp, "pk-a"), gen.uniform(*shp, "pk-b")
     C = gen.uniform(n, n, "pk-c")
@@ -172,14 +214,15 @@ def test_syrk_syr2k(b3, oracle_mod, mode, two, uplo, trans, n, k):
         ref = oracle_mod.ssyrk(uplo, trans, AL, A, BE, C)
         scale = AL * fro(A) ** 2 + BE * fro(C[mask])
     got = to_host(dC)
+    route(A.shape[0], n)
     assert e_nw(got[mask], ref[mask], scale) <= TOL_NW
-    assert e_rel(got[mask], ref[mask]) <= TOL_REL
+    assert e_rel(got[mask], ref[mask]) <= tol_rel(2 * k if two else k, mode)
     assert bits_equal(got[~mask], C[~mask])
 
 
 @pytest.mark.parametrize("uplo,trans", list(itertools.product("LU", "NT")))
 def test_syr2k_integer_equals_two_gemms(b3, mode, uplo, trans):
-    n, k = 290, 150
+    n, k = 292, 152
     shp = (n, k) if trans == "N" else (k, n)
     A, B, C = gen.integers(*shp, "i2-a"), gen.integers(*shp, "i2-b"), gen.integers(n, n, "i2-c")
     dC = to_dev(C)
@@ -199,23 +242,24 @@ V16 = list(itertools.product("LR", "LU", "NT", "NU"))
 
 
 @pytest.mark.parametrize("side,uplo,ta,diag", V16)
-@pytest.mark.parametrize("m,n", [(1, 1), (70, 45), (260, 300)])
-def test_strmm(b3, oracle_mod, mode, side, uplo, ta, diag, m, n):
+@pytest.mark.parametrize("m,n", [(1, 1), (68, 44), (260, 300), (516, 132)])
+def test_strmm(b3, oracle_mod, mode, route, side, uplo, ta, diag, m, n):
     ka = m if side == "L" else n
     A = gen.triangular_dd(ka, uplo, diag, "pt")          # NaN blank triangle (+ NaN unit diagonal)
     B = gen.uniform(m, n, "pt-b")
     dB = to_dev(B)
     b3.strmm(side, uplo, ta, diag, AL, to_dev(A), dB)
     got = to_host(dB)
+    route(ka, m)
     ref = oracle_mod.strmm(side, uplo, ta, diag, AL, A, B)
     T = tri_full(A, uplo, diag, ka)
     assert e_nw(got, ref, AL * fro(T) * fro(B)) <= TOL_NW
-    assert e_rel(got, ref) <= TOL_REL
+    assert e_rel(got, ref) <= tol_rel(ka, mode)
 
 
 @pytest.mark.parametrize("side,uplo,ta,diag", V16)
 def test_strmm_integer_bitexact(b3, oracle_mod, mode, side, uplo, ta, diag):
-    m, n = 290, 200
+    m, n = 292, 200
     ka = m if side == "L" else n
     A = gen.triangular_integer(ka, uplo, diag, "it")
     B = gen.integers(m, n, "it-b")
@@ -236,8 +280,8 @@ def trsm_metrics(got, A, B, side, uplo, ta, diag, alpha, oracle_mod):
 
 
 @pytest.mark.parametrize("side,uplo,ta,diag", V16)
-@pytest.mark.parametrize("m,n", [(1, 1), (70, 45), (300, 260), (1100, 64)])
-def test_strsm(b3, oracle_mod, mode, side, uplo, ta, diag, m, n):
+@pytest.mark.parametrize("m,n", [(1, 1), (68, 44), (300, 260), (1100, 64)])
+def test_strsm(b3, oracle_mod, mode, route, side, uplo, ta, diag, m, n):
     if side == "R":
         m, n = n, m            # keep the triangular order large for side=R too
     ka = m if side == "L" else n
@@ -245,6 +289,7 @@ def test_strsm(b3, oracle_mod, mode, side, uplo, ta, diag, m, n):
     B = gen.uniform(m, n, "px-b")
     dB = to_dev(B)
     b3.strsm(side, uplo, ta, diag, AL, to_dev(A), dB)
+    route(ka, m)
     resid, fwd = trsm_metrics(to_host(dB), A, B, side, uplo, ta, diag, AL, oracle_mod)
     assert resid <= 1e-5 * np.sqrt(ka)
     assert fwd <= 1e-5
