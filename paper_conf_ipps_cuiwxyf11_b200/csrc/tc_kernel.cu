@@ -16,14 +16,16 @@
 //   Reg_alloc(C)                        -> fp32 accumulator in TMEM
 //       (two 256-column accumulators: epilogue of tile i overlaps tile i+1).
 // fp32 accuracy on TF32 tensor cores (north star): every staged value x is
-// split into hi = rna_tf32(x), lo = rna_tf32(x - hi) and each k-step issues
-// lo*hi + hi*lo + hi*hi (small terms first) into the same fp32 accumulator.
+// split into hi = trunc_tf32(x) (what the tensor core reads from the raw
+// word) and lo = rna_tf32(x - hi), and each k-step issues lo*hi + hi*lo +
+// hi*hi (small terms first) into the same fp32 accumulator.
 //
-// Warp roles (448 threads, 1 CTA/SM):
+// Warp roles (576 threads, 1 CTA/SM):
 //   warp 0       TMA producer (one lane)
 //   warp 1       TMEM allocator + MMA issuer (one lane)
 //   warps 2..9   transform: structure fix-ups + hi/lo split (256 threads)
-//   warps 10..13 epilogue: tcgen05.ld -> alpha*acc + beta*C -> global
+//   warps 10..17 epilogue: tcgen05.ld -> alpha*acc + beta*C -> global
+//                (two warps per TMEM lane quarter, 128 columns each)
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <mutex>
@@ -37,7 +39,7 @@ namespace blas3 {
 namespace {
 constexpr int BM = 128, BN = 256, BK = 32, STAGES = 2;
 constexpr int WARP_TMA = 0, WARP_MMA = 1, WARP_TR0 = 2, NUM_TR_WARPS = 8;
-constexpr int WARP_EPI0 = WARP_TR0 + NUM_TR_WARPS, NUM_EPI_WARPS = 4;
+constexpr int WARP_EPI0 = WARP_TR0 + NUM_TR_WARPS, NUM_EPI_WARPS = 8;
 constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;
 constexpr int TR_THREADS = NUM_TR_WARPS * 32;
 constexpr uint32_t A_BYTES = BM * BK * 4;
@@ -47,7 +49,7 @@ constexpr int MAX_MAPS = 8;
 constexpr int LAYOUT_K = 0, LAYOUT_MN = 1;
 
 struct alignas(1024) StageBuf {
-  uint8_t rawA[A_BYTES];   // TMA destination; becomes hi (tf32) in place
+  uint8_t rawA[A_BYTES];   // TMA destination; read by UMMA as hi (low 13 bits ignored)
   uint8_t rawB[B_BYTES];
   uint8_t loA[A_BYTES];    // lo (tf32); also the kr-view landing zone of
   uint8_t loB[B_BYTES];    //   symmetric diagonal blocks before the merge
@@ -57,7 +59,7 @@ struct Barriers {
   uint64_t ready[STAGES];  // transform -> MMA (TR_THREADS arrivals)
   uint64_t empty[STAGES];  // MMA -> TMA (tcgen05.commit)
   uint64_t tfull[2];       // MMA -> epilogue
-  uint64_t tempty[2];      // epilogue -> MMA (128 arrivals)
+  uint64_t tempty[2];      // epilogue -> MMA (256 arrivals)
   uint32_t tmem_base;
 };
 constexpr size_t SMEM_BYTES = sizeof(StageBuf) * STAGES + sizeof(Barriers) + 1024;
@@ -174,22 +176,29 @@ __device__ __forceinline__ void tri_fix(const OpDesc &o, int lay, uint8_t *raw, 
   }
 }
 
-__device__ __forceinline__ float split1(float x, float &lo) {
-  float hi = __uint_as_float(ptx::cvt_rna_tf32(x));
-  lo = __uint_as_float(ptx::cvt_rna_tf32(x - hi));
-  return hi;
+// 3xTF32 split without rewriting hi: kind::tf32 UMMA reads the raw fp32
+// word and ignores its low 13 mantissa bits, i.e. it consumes
+// hi = trunc_tf32(x) directly from the TMA-staged tile (pinned by
+// tests/test_parity_gpu.py::test_split_is_real).  Only lo = x - hi (exact in
+// fp32) is produced, rounded to nearest tf32 (ties away) with integer ops so
+// the transform stays on the ALU/FMA pipes and writes half the bytes.
+__device__ __forceinline__ float split_lo(float x) {
+  const float hi = __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
+  const float l = x - hi;
+  return __uint_as_float((__float_as_uint(l) + 0x1000u) & 0xFFFFE000u);
 }
 
-__device__ __forceinline__ void split_pass(uint8_t *raw, uint8_t *lo, uint32_t bytes, int t) {
-  float4 *r4 = reinterpret_cast<float4 *>(raw);
+__device__ __forceinline__ void split_pass(const uint8_t *raw, uint8_t *lo, uint32_t bytes, int t) {
+  const float4 *r4 = reinterpret_cast<const float4 *>(raw);
   float4 *l4 = reinterpret_cast<float4 *>(lo);
+#pragma unroll 4
   for (uint32_t c = t; c < bytes / 16; c += TR_THREADS) {
-    float4 v = r4[c], l;
-    v.x = split1(v.x, l.x);
-    v.y = split1(v.y, l.y);
-    v.z = split1(v.z, l.z);
-    v.w = split1(v.w, l.w);
-    r4[c] = v;
+    const float4 v = r4[c];
+    float4 l;
+    l.x = split_lo(v.x);
+    l.y = split_lo(v.y);
+    l.z = split_lo(v.z);
+    l.w = split_lo(v.w);
     l4[c] = l;
   }
 }
@@ -346,6 +355,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
   } else {
     // ============================ epilogue warps
     const int q = warp & 3;                     // TMEM lane quarter of this warp
+    const int half = (warp - WARP_EPI0) >> 2;   // which 128 of the 256 columns
     uint32_t tcount = 0;
     for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++tcount) {
       int64_t mi, nj;
@@ -356,27 +366,35 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
       ptx::mbar_wait(&bars->tfull[acc], aph);
       ptx::tc_fence_after();
       const int64_t r = m0 + q * 32 + lane;
-      for (int ch = 0; ch < BN / 32; ++ch) {
-        const int64_t c0 = n0 + ch * 32;
+      const bool row_ok = r < P.M;
+      const float *cin = P.Cin + r;
+      float *cout = P.Cout + r;
+      constexpr int EC = 16;                    // epilogue chunk: 16 columns
+      for (int ch = half * (BN / EC / 2); ch < (half + 1) * (BN / EC / 2); ++ch) {
+        const int64_t c0 = n0 + ch * EC;
         if (c0 >= P.N) break;
-        uint32_t v[32];
-        if (has_k) {
-          ptx::tmem_ld_32x32b_x32(tmem + acc * BN + ch * 32 + ((uint32_t)(q * 32) << 16), v);
-          ptx::tmem_ld_wait();
-        } else {
+        uint32_t v[EC];
+        if (has_k) ptx::tmem_ld_32x32b_x16(tmem + acc * BN + ch * EC + ((uint32_t)(q * 32) << 16), v);
+        // C(r, c0..c0+15): all loads issued before any store (Cin may
+        // alias Cout, so interleaving would serialise every load behind the
+        // previous store); each is a coalesced 128-B warp access per column.
+        float cv[EC];
 #pragma unroll
-          for (int j = 0; j < 32; ++j) v[j] = 0u;
+        for (int j = 0; j < EC; ++j) {
+          const int64_t c = c0 + j;
+          const bool ok = row_ok && c < P.N && !(P.c_tri == 1 && r < c) && !(P.c_tri == 2 && r > c);
+          cv[j] = (ok && P.beta != 0.f) ? cin[c * P.ldcin] : 0.f;
         }
-        if (r < P.M) {
+        if (has_k) ptx::tmem_ld_wait();
+        else {
 #pragma unroll
-          for (int j = 0; j < 32; ++j) {
-            const int64_t c = c0 + j;
-            const bool ok = c < P.N && !(P.c_tri == 1 && r < c) && !(P.c_tri == 2 && r > c);
-            if (!ok) continue;
-            float o = P.alpha * __uint_as_float(v[j]);
-            if (P.beta != 0.f) o = fmaf(P.beta, P.Cin[r + c * P.ldcin], o);
-            P.Cout[r + c * P.ldcout] = o;
-          }
+          for (int j = 0; j < EC; ++j) v[j] = 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < EC; ++j) {
+          const int64_t c = c0 + j;
+          const bool ok = row_ok && c < P.N && !(P.c_tri == 1 && r < c) && !(P.c_tri == 2 && r > c);
+          if (ok) cout[c * P.ldcout] = fmaf(P.beta, cv[j], P.alpha * __uint_as_float(v[j]));
         }
       }
       ptx::tc_fence_before();
