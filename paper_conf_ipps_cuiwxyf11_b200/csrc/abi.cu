@@ -99,6 +99,7 @@ static Problem problem(int64_t M, int64_t N, float alpha, float beta, const floa
   Problem P; memset(&P, 0, sizeof(P));
   P.M = M; P.N = N; P.nseg = 1; P.alpha = alpha; P.beta = beta;
   P.Cin = Cin; P.ldcin = ldcin; P.Cout = Cout; P.ldcout = ldcout;
+  P.nbatch = 1; P.per = 1;
   return P;
 }
 
@@ -332,13 +333,64 @@ int blas3_strmm(char side, char uplo, char transa, char diag, int64_t m, int64_t
 }
 
 // ------------------------------------------------------------------- STRSM (rows A7, A8)
-// Blocked sweep in dependency order: nb=128 diagonal blocks are
-// inverted up front (warp-level kernel), then per block X_b = inv(op(A)_bb)*B_b
-// followed by a GEMM update of the rows (L) / columns (R) still to be solved.
-// Updates are two-level: inside an outer panel of NBO rows only the panel is
-// updated; after the panel one large GEMM updates everything beyond it.
-// alpha is folded into the first operation touching each row/column.
-static const int NB = 128, NBO = 1024;
+// Dependency order of the solver: X_i needs X_k, k < i.  The
+// paper binds the diagonal step to one thread; here it is taken off
+// the critical path.  With L = the stored triangle of A in lower form
+// (op(A) = L or L^T):
+//   1. every 128-block of L is inverted by the warp-level kernel (row A7);
+//   2. 128 -> 256 -> 512 -> NBO doubling builds inv(L_pp) of every NBO-wide
+//      diagonal panel: for each diagonal pair [[L11,0],[L21,L22]],
+//      X21 = -inv(L22) * (L21 * inv(L11)) as two batched GEMMs per level;
+//   3. the sweep (row A8) visits panels in dependency order:
+//        X_p = alpha_p * inv(op(A)_pp) * B_p        (TRI operand, GEMM)
+//        B_rest <- alpha_p * B_rest - op(A)(rest, p) * X_p   (GEMM, K = NBO)
+//      alpha is folded into the first operation that touches each row.
+// Every flop of steps 2-3 runs in the structured GEMM kernels.
+static const int64_t NBO = 1024;   // panel width (multiple of the 128 diagonal block)
+
+static int trsm_panel_inverses(const float *A, int64_t lda, int64_t nt, bool lower, bool unit,
+                               float *D, float *Tw, cudaStream_t s, int sms) {
+  int rc;
+  if (cudaMemsetAsync(D, 0, (size_t)cdiv(nt, NBO) * NBO * NBO * sizeof(float), s) != cudaSuccess)
+    return BLAS3_ERR_CUDA;
+  if (launch_trsm_diag_inv(A, lda, nt, lower, unit, D, NBO, s)) return BLAS3_ERR_CUDA;
+  for (int64_t sz = 128; sz < NBO; sz *= 2) {
+    // pair b covers rows/cols [o, o + 2 sz) of L, o = 2 sz b; L21 = L[o+sz.., o..]
+    const int64_t per = NBO / (2 * sz);
+    const int64_t full = nt / (2 * sz);                    // pairs entirely inside L
+    const int64_t rag_rows = nt - full * 2 * sz - sz;        // second half of a ragged pair
+    // L21 as an Xa operand: X(r,k) = L(o+sz+r, o+k) = lower ? A(o+sz+r, o+k) : A(o+k, o+sz+r)
+    auto l21 = [&](int64_t o) { return lower ? A + (o + sz) + o * lda : A + o + (o + sz) * lda; };
+    auto dblk = [&](int64_t o) { return D + (o / NBO) * NBO * NBO + (o % NBO) * (1 + NBO); };
+    for (int pass = 0; pass < 2; ++pass) {
+      const int64_t cnt = pass == 0 ? full : (rag_rows > 0 ? 1 : 0);
+      if (cnt == 0) continue;
+      const int64_t o = pass == 0 ? 0 : full * 2 * sz;
+      const int64_t m2 = pass == 0 ? sz : rag_rows;          // rows of L21 / order of L22
+      // T = L21 * inv(L11): Xa = L21 (m2 x sz), Xb(c,k) = inv(L11)(k,c) (lower -> TRI swap)
+      Problem P1 = problem(m2, sz, 1.f, 0.f, nullptr, 0, Tw, m2);
+      P1.seg[0].a = dense(l21(o), lda, !lower);
+      P1.seg[0].b = tri(dblk(o), NBO, true, true, false);
+      P1.seg[0].K = sz;
+      P1.nbatch = cnt; P1.per = per;
+      P1.bs_a = {per * 2 * sz * (1 + lda), 2 * sz * (1 + lda)};
+      P1.bs_b = {NBO * NBO, 2 * sz * (1 + NBO)};
+      P1.bs_c = {per * sz * sz, sz * sz};
+      if ((rc = run_problem(P1, s, sms))) return rc;
+      // X21 = -inv(L22) * T: Xa = inv(L22) (lower TRI), Xb(c,k) = T(k,c) (kr)
+      Problem P2 = problem(m2, sz, -1.f, 0.f, nullptr, 0, dblk(o) + sz, NBO);
+      P2.seg[0].a = tri(dblk(o) + sz * (1 + NBO), NBO, true, false, false);
+      P2.seg[0].b = dense(Tw, m2, true);
+      P2.seg[0].K = m2;
+      P2.nbatch = cnt; P2.per = per;
+      P2.bs_a = {NBO * NBO, 2 * sz * (1 + NBO)};
+      P2.bs_b = {per * sz * sz, sz * sz};
+      P2.bs_c = {NBO * NBO, 2 * sz * (1 + NBO)};
+      if ((rc = run_problem(P2, s, sms))) return rc;
+    }
+  }
+  return 0;
+}
 
 int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t n, float alpha,
                 const float *A, int64_t lda, float *B, int64_t ldb, blas3_stream_t stream) {
@@ -354,78 +406,56 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
 
   const bool left = up(side) == 'L', lower = up(uplo) == 'L', ta = up(transa) != 'N',
              unit = up(diag) == 'U';
-  const bool lower_op = lower != ta;               // op(A) lower-triangular
+  const bool lower_op = lower != ta;               // op(A) = L (true) or L^T (false)
   const int64_t nt = left ? m : n;                 // order of A
-  const int64_t nblk = cdiv(nt, NB);
+  const int64_t npanel = cdiv(nt, NBO);
   const int64_t other = left ? n : m;              // RHS extent
   const bool forward = left ? lower_op : !lower_op;
 
-  Scratch D, W;
-  if ((rc = get_scratch(D, (size_t)nblk * NB * NB * sizeof(float), s))) return rc;
-  if ((rc = get_scratch(W, (size_t)NB * other * sizeof(float), s,
-                        (size_t)nblk * NB * NB * sizeof(float)))) return rc;
-  if (launch_trsm_diag_inv(A, lda, nt, ta, lower_op, unit, NB, D.p, s)) return BLAS3_ERR_CUDA;
+  const size_t d_bytes = (size_t)npanel * NBO * NBO * sizeof(float);
+  // doubling scratch: (nt / 2sz) pairs x sz^2 floats at the widest level (sz = NBO/2)
+  const size_t t_bytes = ((size_t)nt * (NBO / 4) + (size_t)NBO * NBO / 4) * sizeof(float);
+  const size_t w_bytes = (size_t)NBO * other * sizeof(float);        // one solved panel
+  Scratch D, Tw, W;
+  if ((rc = get_scratch(D, d_bytes, s))) return rc;
+  if ((rc = get_scratch(Tw, t_bytes, s, d_bytes))) return rc;
+  if ((rc = get_scratch(W, w_bytes, s, d_bytes + t_bytes))) return rc;
+  if ((rc = trsm_panel_inverses(A, lda, nt, lower, unit, D.p, Tw.p, s, sms))) return rc;
 
-  // op(A) sub-block as a GEMM operand with rows R (r0..) x k (k0..):
-  //   Xa(r,k) = op(A)(r0+r, k0+k) (left: rows of the update)
-  auto opA_rk = [&](int64_t r0, int64_t k0, const float *&p, bool &kr) {
-    if (!ta) { p = A + r0 + k0 * lda; kr = false; } else { p = A + k0 + r0 * lda; kr = true; }
-  };
-  const int64_t per_panel = NBO / NB;
-  const int64_t npanel = cdiv(nblk, per_panel);
-  for (int64_t pi = 0; pi < npanel; ++pi) {
-    // blocks of this panel in processing order
-    int64_t q0 = pi * per_panel, q1 = imin(nblk, q0 + per_panel);
-    for (int64_t q = q0; q < q1; ++q) {
-      const int64_t b = forward ? q : nblk - 1 - q;
-      const int64_t b0 = b * NB, nbr = imin(NB, nt - b0);
-      const bool pend = (pi == 0 && q == q0);      // rows of panel 0 still unscaled
-      const float a1 = pend ? alpha : 1.f;
-      // remaining blocks of the panel (in processing order) -> contiguous range
-      int64_t rq0 = q + 1, rq1 = q1;
-      int64_t r_lo, r_hi;                          // element range of those blocks
-      if (forward) { r_lo = (rq0 < rq1) ? rq0 * NB : 0; r_hi = (rq0 < rq1) ? imin(nt, rq1 * NB) : 0; }
-      else {
-        r_lo = (rq0 < rq1) ? (nblk - rq1) * NB : 0;
-        r_hi = (rq0 < rq1) ? imin(nt, (nblk - rq0) * NB) : 0;
-      }
-      const float *Db = D.p + b * NB * NB;
-      if (left) {
-        // W = a1 * Dinv_b * B_b   (nbr x n), then B_b <- W
-        if ((rc = gemm_dense(nbr, n, nbr, a1, Db, NB, false, B + b0, ldb, true, 0.f, W.p, NB, s, sms))) return rc;
-        if (launch_copy(B + b0, ldb, W.p, NB, nbr, n, s)) return BLAS3_ERR_CUDA;
-        if (r_hi > r_lo) {   // B_r <- a1*B_r - op(A)(r, b) * X_b
-          const float *pa; bool akr; opA_rk(r_lo, b0, pa, akr);
-          if ((rc = gemm_dense(r_hi - r_lo, n, nbr, -1.f, pa, lda, akr, W.p, NB, true, a1,
-                               B + r_lo, ldb, s, sms))) return rc;
-        }
-      } else {
-        // W = a1 * B_b * Dinv_b  (m x nbr), then B(:, b) <- W
-        if ((rc = gemm_dense(m, nbr, nbr, a1, B + b0 * ldb, ldb, false, Db, NB, true, 0.f, W.p, m, s, sms))) return rc;
-        if (launch_copy(B + b0 * ldb, ldb, W.p, m, m, nbr, s)) return BLAS3_ERR_CUDA;
-        if (r_hi > r_lo) {   // B(:,c) <- a1*B(:,c) - X_b * op(A)(b, c)
-          // Xb(c,k) = op(A)(b0+k, c0+c): !ta -> A[(b0+k) + (c0+c)*lda] (kr); ta -> A[(c0+c)+(b0+k)*lda]
-          const float *pb = ta ? A + r_lo + b0 * lda : A + b0 + r_lo * lda;
-          if ((rc = gemm_dense(m, r_hi - r_lo, nbr, -1.f, W.p, m, false, pb, lda, !ta, a1,
-                               B + r_lo * ldb, ldb, s, sms))) return rc;
-        }
-      }
-    }
-    // outer update of everything beyond the panel
-    int64_t pq0 = q0, pq1 = q1;                      // panel blocks (processing order)
-    int64_t p_lo = forward ? pq0 * NB : (nblk - pq1) * NB;
-    int64_t p_hi = forward ? imin(nt, pq1 * NB) : imin(nt, (nblk - pq0) * NB);
-    int64_t o_lo = forward ? p_hi : 0, o_hi = forward ? nt : p_lo;
-    if (o_hi > o_lo) {
-      const float a1 = (pi == 0) ? alpha : 1.f;
-      const int64_t kp = p_hi - p_lo;
-      if (left) {   // B_o <- a1*B_o - op(A)(o, panel) * X_panel (X_panel = B rows of the panel)
-        const float *pa; bool akr; opA_rk(o_lo, p_lo, pa, akr);
-        if ((rc = gemm_dense(o_hi - o_lo, n, kp, -1.f, pa, lda, akr, B + p_lo, ldb, true, a1,
+  for (int64_t q = 0; q < npanel; ++q) {
+    const int64_t p = forward ? q : npanel - 1 - q;
+    const int64_t p0 = p * NBO, pr = imin(NBO, nt - p0);
+    const float a1 = (q == 0) ? alpha : 1.f;       // first touch of every row/column
+    const float *Dp = D.p + p * NBO * NBO;
+    const int64_t o_lo = forward ? p0 + pr : 0, o_hi = forward ? nt : p0;
+    if (left) {
+      // X_p = a1 * inv(op(A)_pp) * B_p: Xa(r,k) = Dop(r,k), Dop = lower_op ? D : D^T
+      Problem P = problem(pr, n, a1, 0.f, nullptr, 0, W.p, pr);
+      P.seg[0].a = tri(Dp, NBO, true, !lower_op, false);
+      P.seg[0].b = dense(B + p0, ldb, true);
+      P.seg[0].K = pr;
+      P.rev_m = tri_kle(P.seg[0].a);
+      if ((rc = run_problem(P, s, sms))) return rc;
+      if (launch_copy(B + p0, ldb, W.p, pr, pr, n, s)) return BLAS3_ERR_CUDA;
+      if (o_hi > o_lo) {   // B_o <- a1*B_o - op(A)(o, p) * X_p
+        // Xa(r,k) = op(A)(o_lo+r, p0+k): !ta -> A(o_lo+r, p0+k) rk; ta -> A(p0+k, o_lo+r) kr
+        const float *pa = ta ? A + p0 + o_lo * lda : A + o_lo + p0 * lda;
+        if ((rc = gemm_dense(o_hi - o_lo, n, pr, -1.f, pa, lda, ta, W.p, pr, true, a1,
                              B + o_lo, ldb, s, sms))) return rc;
-      } else {      // B(:,o) <- a1*B(:,o) - X_panel * op(A)(panel, o)
-        const float *pb = ta ? A + o_lo + p_lo * lda : A + p_lo + o_lo * lda;
-        if ((rc = gemm_dense(m, o_hi - o_lo, kp, -1.f, B + p_lo * ldb, ldb, false, pb, lda, !ta, a1,
+      }
+    } else {
+      // X_p = a1 * B_p * inv(op(A)_pp): Xb(c,k) = Dop(k,c) -> TRI swap = lower_op
+      Problem P = problem(m, pr, a1, 0.f, nullptr, 0, W.p, m);
+      P.seg[0].a = dense(B + p0 * ldb, ldb, false);
+      P.seg[0].b = tri(Dp, NBO, true, lower_op, false);
+      P.seg[0].K = pr;
+      P.rev_n = tri_kle(P.seg[0].b);
+      if ((rc = run_problem(P, s, sms))) return rc;
+      if (launch_copy(B + p0 * ldb, ldb, W.p, m, m, pr, s)) return BLAS3_ERR_CUDA;
+      if (o_hi > o_lo) {   // B(:,o) <- a1*B(:,o) - X_p * op(A)(p, o)
+        // Xb(c,k) = op(A)(p0+k, o_lo+c): !ta -> A(p0+k, o_lo+c) kr; ta -> A(o_lo+c, p0+k) rk
+        const float *pb = ta ? A + o_lo + p0 * lda : A + p0 + o_lo * lda;
+        if ((rc = gemm_dense(m, o_hi - o_lo, pr, -1.f, W.p, m, false, pb, lda, !ta, a1,
                              B + o_lo * ldb, ldb, s, sms))) return rc;
       }
     }

@@ -62,11 +62,11 @@ constexpr int DNB = 128;          // diagonal block size (4 warps x 32)
 constexpr int DLD = DNB + 1;      // padded smem row (bank-conflict free)
 }
 
-// One CTA (128 threads) per diagonal block.  L = the block of op(A) brought
-// to lower-triangular form (transposed when op(A) is upper); X = inv(L).
+// One CTA (128 threads) per 128-block of L (the stored triangle of A in
+// lower form); X = inv(L_bb) written into the panel-inverse workspace.
 __global__ void __launch_bounds__(128)
-trsm_diag_inv_kernel(const float *A, int64_t lda, int64_t n, int trans, int lower_op,
-                     int unit, float *Dinv) {
+trsm_diag_inv_kernel(const float *A, int64_t lda, int64_t n, int stored_lower, int unit,
+                     float *Dinv, int64_t ldD) {
   extern __shared__ float sm[];
   float *L = sm;                  // [DNB][DLD]
   float *X = sm + DNB * DLD;      // [DNB][DLD]
@@ -76,17 +76,11 @@ trsm_diag_inv_kernel(const float *A, int64_t lda, int64_t n, int trans, int lowe
 
   // stage L (lower) and clear X; the blank triangle of A is never read (Q8)
   for (int c = 0; c < DNB; ++c) {
-    int r = tid;
+    const int r = tid;
     float v = 0.f;
     if (r < nr && c < nr) {
-      if (r == c) {
-        if (unit) v = 1.f;
-        else v = trans ? A[(i0 + r) + (i0 + r) * lda] : A[(i0 + r) + (i0 + r) * lda];
-      } else if (r > c) {
-        // L(r,c) = op(A)(i0+r, i0+c) if op(A) lower, else op(A)(i0+c, i0+r)
-        int64_t a = lower_op ? r : c, b = lower_op ? c : r;        // op(A)(a,b)
-        v = trans ? A[(i0 + b) + (i0 + a) * lda] : A[(i0 + a) + (i0 + b) * lda];
-      }
+      if (r == c) v = unit ? 1.f : A[(i0 + r) + (i0 + r) * lda];
+      else if (r > c) v = stored_lower ? A[(i0 + r) + (i0 + c) * lda] : A[(i0 + c) + (i0 + r) * lda];
     } else if (r == c) {
       v = 1.f;                     // identity padding of a ragged last block
     }
@@ -141,19 +135,18 @@ trsm_diag_inv_kernel(const float *A, int64_t lda, int64_t n, int trans, int lowe
   }
   __syncthreads();
 
-  // write inv(op(A)_bb) column-major (ld DNB); padded rows/cols are zero
-  float *D = Dinv + (int64_t)blockIdx.x * DNB * DNB;
+  // write inv(L_bb) (lower, column-major) into its panel slot; padded rows/cols zero
+  const int64_t bpp = ldD / DNB;                     // 128-blocks per panel
+  float *D = Dinv + (blockIdx.x / bpp) * ldD * ldD + (blockIdx.x % bpp) * DNB * (1 + ldD);
   for (int c = 0; c < DNB; ++c) {
-    int r = tid;
-    float v = 0.f;
-    if (r < nr && c < nr) v = lower_op ? X[r * DLD + c] : X[c * DLD + r];
-    D[r + (int64_t)c * DNB] = v;
+    const int r = tid;
+    D[r + (int64_t)c * ldD] = (r < nr && c < nr) ? X[r * DLD + c] : 0.f;
   }
 }
 
-int launch_trsm_diag_inv(const float *A, int64_t lda, int64_t n, int trans, int lower_op,
-                         int unit, int nb, float *Dinv, cudaStream_t s) {
-  if (nb != DNB) return -1;
+int launch_trsm_diag_inv(const float *A, int64_t lda, int64_t n, int stored_lower, int unit,
+                         float *Dinv, int64_t ldD, cudaStream_t s) {
+  if (ldD % DNB) return -1;
   const size_t smem = 2 * DNB * DLD * sizeof(float);
   static bool attr = false;
   if (!attr) {
@@ -162,7 +155,7 @@ int launch_trsm_diag_inv(const float *A, int64_t lda, int64_t n, int trans, int 
     attr = true;
   }
   int64_t blocks = cdiv(n, DNB);
-  trsm_diag_inv_kernel<<<(unsigned)blocks, 128, smem, s>>>(A, lda, n, trans, lower_op, unit, Dinv);
+  trsm_diag_inv_kernel<<<(unsigned)blocks, 128, smem, s>>>(A, lda, n, stored_lower, unit, Dinv, ldD);
   note_launch();
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }

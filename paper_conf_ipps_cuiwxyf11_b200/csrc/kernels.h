@@ -22,10 +22,13 @@ int launch_scale(float *C, int64_t ldc, int64_t m, int64_t n, float beta, int tr
 int launch_copy(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t m, int64_t n,
                 cudaStream_t s);
 
-// TRSM diagonal blocks: Dinv[b] = inv(op(A)_bb) for every nb x nb diagonal
-// block b of op(A) (last block ragged, zero-padded to nb), column-major with
-// leading dimension nb, stored consecutively.  lower_op: op(A) is lower.
-int launch_trsm_diag_inv(const float *A, int64_t lda, int64_t n, int trans, int lower,
-                         int unit, int nb, float *Dinv, cudaStream_t s);
+// TRSM diagonal blocks: for every 128 x 128 diagonal block b of L, where L
+// is the stored triangle of A brought to lower form (L(i,j) = A(i,j) if A is
+// stored lower, A(j,i) if stored upper; unit -> L(i,i) = 1), writes inv(L_bb)
+// (lower) into the panel-inverse workspace: panel p = b / (panel/128) is an
+// ldD x ldD column-major block at Dinv + p*ldD*ldD, block b sits on its
+// diagonal.  The last block may be ragged (zero-padded).
+int launch_trsm_diag_inv(const float *A, int64_t lda, int64_t n, int stored_lower, int unit,
+                         float *Dinv, int64_t ldD, cudaStream_t s);
 
 }  // namespace blas3

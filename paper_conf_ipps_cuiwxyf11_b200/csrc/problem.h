@@ -45,6 +45,15 @@ struct Segment {
   int64_t K;
 };
 
+// Two-level batch stride: element offset of batch b is
+//   (b / per) * outer + (b % per) * inner
+// (used by the TRSM panel-inverse doubling, whose pairs sit at a uniform
+// stride along the diagonal of A but at a two-level stride in the compact
+// panel-inverse workspace).
+struct BatchStride {
+  int64_t outer, inner;
+};
+
 struct Problem {
   int64_t M, N;
   Segment seg[2];
@@ -55,7 +64,15 @@ struct Problem {
   float alpha, beta;
   const float *Cin; int64_t ldcin;   // read only when beta != 0
   float *Cout; int64_t ldcout;
+  // batched problems (SIMT route only): nbatch >= 1 independent problems of
+  // the same shape; seg[0] operands and C advance by the strides below.
+  int64_t nbatch, per;
+  BatchStride bs_a, bs_b, bs_c;
 };
+
+HD int64_t batch_off(const BatchStride &s, int64_t b, int64_t per) {
+  return (b / per) * s.outer + (b % per) * s.inner;
+}
 
 HD int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 HD int64_t imin(int64_t a, int64_t b) { return a < b ? a : b; }
@@ -69,7 +86,7 @@ HD bool tri_kle(const OpDesc &o) { return o.lower != o.swap; }
 // Triangular (SYRK/SYR2K): only tiles intersecting the referenced triangle.
 template <int BM, int BN>
 struct Tiles {
-  static constexpr int GM = 8;
+  static constexpr int GM = 16;   // ~sqrt(#SMs * |B panel| / |A panel|) for L2 reuse
 
   HD static int64_t tri_first_m(int64_t j) { return (j * BN) / BM; }          // lower
   HD static int64_t tri_end_m(int64_t j, int64_t mt) {                        // upper

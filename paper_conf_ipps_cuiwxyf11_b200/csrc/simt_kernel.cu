@@ -54,12 +54,24 @@ __device__ __forceinline__ void stash(float (*dst)[BM + PADS], bool kr, const fl
 }  // namespace
 
 __global__ void __launch_bounds__(NT, 2)
-simt_structured_gemm(const Problem P) {
+simt_structured_gemm(const Problem P0) {
   __shared__ __align__(16) Stage st[2];
   const int tid = threadIdx.x, tx = tid % 16, ty = tid / 16;
-  const int64_t ntiles = Tiles<BM, BN>::count(P);
+  const int64_t tiles_per = Tiles<BM, BN>::count(P0);
+  const int64_t nb = P0.nbatch > 0 ? P0.nbatch : 1;
+  const int64_t ntiles = tiles_per * nb;
 
-  for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+  for (int64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x) {
+    // batch member of this tile: offset seg[0] operands and C
+    const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
+    Problem P = P0;
+    if (nb > 1) {
+      P.seg[0].a.ptr += batch_off(P0.bs_a, b, P0.per);
+      P.seg[0].b.ptr += batch_off(P0.bs_b, b, P0.per);
+      const int64_t oc = batch_off(P0.bs_c, b, P0.per);
+      P.Cin += oc;
+      P.Cout += oc;
+    }
     int64_t mi, nj;
     Tiles<BM, BN>::coords(P, t, mi, nj);
     const int64_t m0 = mi * BM, n0 = nj * BN;
@@ -135,7 +147,7 @@ simt_structured_gemm(const Problem P) {
 }
 
 int launch_simt(const Problem &P, cudaStream_t stream, int num_sms) {
-  int64_t tiles = Tiles<BM, BN>::count(P);
+  int64_t tiles = Tiles<BM, BN>::count(P) * (P.nbatch > 0 ? P.nbatch : 1);
   if (tiles == 0) return 0;
   int64_t grid = imin(tiles, (int64_t)num_sms * 2);
   simt_structured_gemm<<<(unsigned)grid, NT, 0, stream>>>(P);

@@ -466,6 +466,7 @@ static bool aligned_op(const OpDesc &o) {
 }
 
 bool tc_eligible(const Problem &P) {
+  if (P.nbatch > 1) return false;        // batched problems run on the SIMT kernel
   for (int s = 0; s < P.nseg; ++s)
     if (!aligned_op(P.seg[s].a) || !aligned_op(P.seg[s].b)) return false;
   return true;
