@@ -121,21 +121,24 @@ __device__ __forceinline__ int64_t tile_kblocks(const Problem &P, int64_t m0, in
 }
 
 // ---------------------------------------------------------------- producer
+// Every operand map is 4-D: (element dims) x (batch-inner, batch-outer);
+// (bj, bg) select the batch member (0, 0 for an ordinary problem).
 __device__ __forceinline__ uint32_t load_operand(const TcParams &prm, const OpDesc &o, int cls,
                                                  int lay, uint8_t *raw, uint8_t *lo, int64_t r0,
-                                                 int64_t k0, int rows, uint64_t *bar) {
+                                                 int64_t k0, int rows, uint64_t *bar, int32_t bj,
+                                                 int32_t bg) {
   uint32_t bytes = 0;
   if (lay == LAYOUT_MN) {
     const CUtensorMap *m = &prm.maps[o.map_rk];
     for (int c = 0; c < rows / 32; ++c) {
-      ptx::tma_load_2d(m, bar, raw + c * (BK * 128), (int32_t)(r0 + 32 * c), (int32_t)k0);
+      ptx::tma_load_4d(m, bar, raw + c * (BK * 128), (int32_t)(r0 + 32 * c), (int32_t)k0, bj, bg);
     }
   } else {
-    ptx::tma_load_2d(&prm.maps[o.map_kr], bar, raw, (int32_t)k0, (int32_t)r0);
+    ptx::tma_load_4d(&prm.maps[o.map_kr], bar, raw, (int32_t)k0, (int32_t)r0, bj, bg);
   }
   bytes += rows * BK * 4;
   if (cls == BLK_SYM_DIAG) {       // the mirrored orientation lands in the lo buffer
-    ptx::tma_load_2d(&prm.maps[o.map_kr], bar, lo, (int32_t)k0, (int32_t)r0);
+    ptx::tma_load_4d(&prm.maps[o.map_kr], bar, lo, (int32_t)k0, (int32_t)r0, bj, bg);
     bytes += rows * BK * 4;
   }
   return bytes;
@@ -238,14 +241,19 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
   ptx::tc_fence_after();
   const uint32_t tmem = bars->tmem_base;
 
-  const int64_t ntiles = Tiles<BM, BN>::count(P);
+  // batched problems: tile tb -> batch member b = tb / tiles_per, tile t
+  const int64_t tiles_per = Tiles<BM, BN>::count(P);
+  const int64_t per = P.per > 0 ? P.per : 1;
+  const int64_t ntiles = tiles_per * (P.nbatch > 0 ? P.nbatch : 1);
 
   if (warp == WARP_TMA) {
     // ============================ TMA producer
     if (lane == 0) {
       for (int i = 0; i < MAX_MAPS; ++i) ptx::tma_prefetch(&prm.maps[i]);
       uint32_t it = 0;
-      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      for (int64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x) {
+        const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
+        const int32_t bj = (int32_t)(b % per), bg = (int32_t)(b / per);
         int64_t mi, nj;
         Tiles<BM, BN>::coords(P, t, mi, nj);
         const int64_t m0 = mi * BM, n0 = nj * BN;
@@ -262,9 +270,9 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
             ptx::mbar_arrive_expect_tx(&bars->full[stg],
                                        operand_bytes(si.clsA, BM) + operand_bytes(si.clsB, BN));
             load_operand(prm, sg.a, si.clsA, si.layA, st[stg].rawA, st[stg].loA, m0, k0, BM,
-                         &bars->full[stg]);
+                         &bars->full[stg], bj, bg);
             load_operand(prm, sg.b, si.clsB, si.layB, st[stg].rawB, st[stg].loB, n0, k0, BN,
-                         &bars->full[stg]);
+                         &bars->full[stg], bj, bg);
           }
         }
       }
@@ -276,7 +284,8 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     // ============================ MMA issuer
     uint32_t it = 0, tcount = 0;
     const uint32_t sA[STAGES] = {ptx::smem_u32(st[0].rawA), ptx::smem_u32(st[1].rawA)};
-    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++tcount) {
+    for (int64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x, ++tcount) {
+      const int64_t t = tb % tiles_per;
       int64_t mi, nj;
       Tiles<BM, BN>::coords(P, t, mi, nj);
       const int64_t m0 = mi * BM, n0 = nj * BN;
@@ -324,7 +333,8 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     // ============================ transform warps
     const int tt = threadIdx.x - WARP_TR0 * 32;
     uint32_t it = 0;
-    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    for (int64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x) {
+      const int64_t t = tb % tiles_per;
       int64_t mi, nj;
       Tiles<BM, BN>::coords(P, t, mi, nj);
       const int64_t m0 = mi * BM, n0 = nj * BN;
@@ -357,7 +367,9 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     const int q = warp & 3;                     // TMEM lane quarter of this warp
     const int half = (warp - WARP_EPI0) >> 2;   // which 128 of the 256 columns
     uint32_t tcount = 0;
-    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++tcount) {
+    for (int64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x, ++tcount) {
+      const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
+      const int64_t coff = (P.nbatch > 1) ? batch_off(P.bs_c, b, per) : 0;
       int64_t mi, nj;
       Tiles<BM, BN>::coords(P, t, mi, nj);
       const int64_t m0 = mi * BM, n0 = nj * BN;
@@ -367,8 +379,8 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
       ptx::tc_fence_after();
       const int64_t r = m0 + q * 32 + lane;
       const bool row_ok = r < P.M;
-      const float *cin = P.Cin + r;
-      float *cout = P.Cout + r;
+      const float *cin = P.Cin + coff + r;
+      float *cout = P.Cout + coff + r;
       constexpr int EC = 16;                    // epilogue chunk: 16 columns
       for (int ch = half * (BN / EC / 2); ch < (half + 1) * (BN / EC / 2); ++ch) {
         const int64_t c0 = n0 + ch * EC;
@@ -429,33 +441,40 @@ static EncodeTiledFn encode_fn() {
   return fn;
 }
 
-// 2-D fp32 tensor map: dim0 contiguous (extent d0), dim1 stride ld floats.
+// 4-D fp32 tensor map: dim0 contiguous (extent d0), dim1 stride ld floats,
+// dims 2/3 = batch (inner, outer) with element strides bs.inner / bs.outer.
+// Extents are the sub-problem's, so TMA zero-fills every out-of-range element
+// of a tile (including those of a batch member's neighbours).
 static bool make_map(CUtensorMap *m, const float *ptr, int64_t d0, int64_t d1, int64_t ld,
-                     uint32_t box0, uint32_t box1, CUtensorMapSwizzle swz) {
+                     uint32_t box0, uint32_t box1, CUtensorMapSwizzle swz, int64_t per,
+                     int64_t groups, BatchStride bs) {
   EncodeTiledFn fn = encode_fn();
   if (!fn) return false;
-  cuuint64_t dims[2] = {(cuuint64_t)d0, (cuuint64_t)d1};
-  cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
-  cuuint32_t box[2] = {box0, box1};
-  cuuint32_t es[2] = {1, 1};
-  return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(ptr), dims, strides, box, es,
+  const int64_t plain = ld * d1;               // stride for unit batch dims
+  cuuint64_t dims[4] = {(cuuint64_t)d0, (cuuint64_t)d1, (cuuint64_t)per, (cuuint64_t)groups};
+  cuuint64_t strides[3] = {(cuuint64_t)ld * 4, (cuuint64_t)(per > 1 ? bs.inner : plain) * 4,
+                           (cuuint64_t)(groups > 1 ? bs.outer : plain) * 4};
+  cuuint32_t box[4] = {box0, box1, 1, 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, const_cast<float *>(ptr), dims, strides, box, es,
             CU_TENSOR_MAP_INTERLEAVE_NONE, swz,
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 // maps for one operand with R rows, K columns, staged `rows` at a time
-static bool op_maps(TcParams &prm, int &slot, OpDesc &o, int64_t R, int64_t K, int rows) {
+static bool op_maps(TcParams &prm, int &slot, OpDesc &o, int64_t R, int64_t K, int rows,
+                    int64_t per, int64_t groups, BatchStride bs) {
   o.map_rk = o.map_kr = -1;
   const bool need_rk = (o.kind == OP_DENSE && !o.kr) || o.kind == OP_SYM || (o.kind == OP_TRI && !o.swap);
   const bool need_kr = (o.kind == OP_DENSE && o.kr) || o.kind == OP_SYM || (o.kind == OP_TRI && o.swap);
   if (need_rk) {       // X(r,k) = G[r + k*ld]: dim0 = r (R), dim1 = k (K)
     if (slot >= MAX_MAPS || !make_map(&prm.maps[slot], o.ptr, R, K, o.ld, 32, BK,
-                                                CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return false;
+                                                CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B, per, groups, bs)) return false;
     o.map_rk = slot++;
   }
   if (need_kr) {       // X(r,k) = G[k + r*ld]: dim0 = k (K), dim1 = r (R)
     if (slot >= MAX_MAPS || !make_map(&prm.maps[slot], o.ptr, K, R, o.ld, BK, rows,
-                                                CU_TENSOR_MAP_SWIZZLE_128B)) return false;
+                                                CU_TENSOR_MAP_SWIZZLE_128B, per, groups, bs)) return false;
     o.map_kr = slot++;
   }
   return true;
@@ -466,7 +485,11 @@ static bool aligned_op(const OpDesc &o) {
 }
 
 bool tc_eligible(const Problem &P) {
-  if (P.nbatch > 1) return false;        // batched problems run on the SIMT kernel
+  if (P.nbatch > 1) {                    // batch strides become TMA strides (16-B multiples)
+    if (P.nseg != 1 || P.per < 1) return false;
+    for (const BatchStride *b : {&P.bs_a, &P.bs_b})
+      if (b->inner % 4 || b->outer % 4) return false;
+  }
   for (int s = 0; s < P.nseg; ++s)
     if (!aligned_op(P.seg[s].a) || !aligned_op(P.seg[s].b)) return false;
   return true;
@@ -482,8 +505,10 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
   for (int s = 0; s < prm.P.nseg; ++s) {
     Segment &sg = prm.P.seg[s];
     if (sg.K <= 0) continue;
-    if (!op_maps(prm, slot, sg.a, prm.P.M, sg.K, BM)) return -4;
-    if (!op_maps(prm, slot, sg.b, prm.P.N, sg.K, BN)) return -4;
+    const int64_t nb = prm.P.nbatch > 1 ? prm.P.nbatch : 1;
+    const int64_t per = nb > 1 ? prm.P.per : 1, groups = cdiv(nb, per);
+    if (!op_maps(prm, slot, sg.a, prm.P.M, sg.K, BM, per, groups, prm.P.bs_a)) return -4;
+    if (!op_maps(prm, slot, sg.b, prm.P.N, sg.K, BN, per, groups, prm.P.bs_b)) return -4;
   }
   static bool attr = false;
   if (!attr) {
@@ -491,7 +516,7 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
                              (int)SMEM_BYTES) != cudaSuccess) return -1;
     attr = true;
   }
-  const int64_t tiles = Tiles<BM, BN>::count(prm.P);
+  const int64_t tiles = Tiles<BM, BN>::count(prm.P) * (prm.P.nbatch > 1 ? prm.P.nbatch : 1);
   if (tiles == 0) return 0;
   const int64_t grid = imin(tiles, (int64_t)num_sms);
   tc_structured_gemm<<<(unsigned)grid, NTHREADS, SMEM_BYTES, stream>>>(prm);
