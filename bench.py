@@ -148,9 +148,14 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = local % max(1, torch.cuda.device_count())   # (a 1-GPU logic check may share a device)
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("BLAS3_BENCH_BACKEND", "nccl")   # gloo: 1-GPU logic check only
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
 
     import paper_conf_ipps_cuiwxyf11_b200 as b3
     b3.set_math_mode(args.math)
@@ -183,6 +188,16 @@ def run_ours(args):
     fl = flops(n, cols)
     ev = {r: [] for r in ROUTINES}
 
+    if world > 1:
+        from paper_conf_ipps_cuiwxyf11_b200 import dist as d3
+        # SYRK/SYR2K at N>1: k-split weak scaling -- rank r's own k-slab A_r (= its B
+        # slab) and B_r (= its C0 slab), partials summed by one NCCL all-reduce; beta*C
+        # is applied on rank 0 only and the other ranks start from zeros, so the sum is
+        # exact on both triangles.
+        dCs = torch.empty((n, n), device=dev)
+        Cs = colmaj(dCs)
+        beta_r = BETA if rank == 0 else 0.0
+
     def chain(record):
         def timed(name, fn):
             if record:
@@ -193,8 +208,25 @@ def run_ours(args):
                 fn()
         timed("sgemm", lambda: b3.sgemm("N", "N", ALPHA, A, Bm, BETA, C))
         timed("ssymm", lambda: b3.ssymm("L", "L", ALPHA, A, Bm, BETA, C))
-        timed("ssyrk", lambda: b3.ssyrk("L", "N", ALPHA, A, BETA, C))
-        timed("ssyr2k", lambda: b3.ssyr2k("L", "N", ALPHA, A, Bm, BETA, C))
+        if world == 1:
+            timed("ssyrk", lambda: b3.ssyrk("L", "N", ALPHA, A, BETA, C))
+            timed("ssyr2k", lambda: b3.ssyr2k("L", "N", ALPHA, A, Bm, BETA, C))
+        else:
+            def syrk_k():
+                if rank == 0:
+                    dCs.copy_(dC0)
+                else:
+                    dCs.zero_()
+                b3.ssyrk("L", "N", ALPHA, Bm, beta_r, Cs)
+                d3.syrk_k_split(dCs)
+
+            def syr2k_k():
+                if rank != 0:
+                    dCs.zero_()
+                b3.ssyr2k("L", "N", ALPHA, Bm, C0, 1.0 if rank == 0 else 0.0, Cs)
+                d3.syrk_k_split(dCs)
+            timed("ssyrk", syrk_k)
+            timed("ssyr2k", syr2k_k)
         timed("strmm", lambda: b3.strmm("L", "L", "N", "N", ALPHA, T, X))
         timed("strsm", lambda: b3.strsm("L", "L", "N", "N", ALPHA, T, X))
 
@@ -295,8 +327,9 @@ def run_ours(args):
                         "(K=8192), strmm LLNN, strsm LLNN; alpha=1.5 beta=0.5",
             "n": n, "k": n, "cols_per_rank": cols, "math": args.math,
             "l2": "no flush: every operand is 256 MiB > 126 MB L2",
-            "parallelism": f"column slabs of B/C x{world}, A/T broadcast (NCCL)" if world > 1
-            else "1 GPU",
+            "parallelism": (f"dp{world}: column slabs of B/C/X per rank (8192 columns each), A and T "
+                            f"broadcast from rank 0 (NCCL); ssyrk/ssyr2k k-split, partials "
+                            f"all-reduced (NCCL)") if world > 1 else "1 GPU",
         },
         "routines": per,
         "pct_of_peak": round(100.0 * value / world / 1e3 / pk, 1),
