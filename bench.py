@@ -159,7 +159,7 @@ def run_ours(args):
 
     import paper_conf_ipps_cuiwxyf11_b200 as b3
     b3.set_math_mode(args.math)
-    n = args.n
+    n = args.size
     cols = n                                   # per-rank slab width (weak scaling)
     A_h, T_h, B_h, C_h = make_inputs(n, cols, rank)
     dev = torch.device("cuda", local)
@@ -301,7 +301,7 @@ def run_ours(args):
     achieved = fl["sgemm"] / (sg_ms * 1e-3) / 1e12
     traffic = None
     tp = os.path.join(ROOT, "profiles", "ncu_sgemm_traffic.json")
-    if os.path.exists(tp):
+    if os.path.exists(tp) and n == N and args.math != "simt":
         try:
             traffic = json.load(open(tp)).get("dram_bytes_per_launch")
         except (ValueError, OSError):
@@ -327,7 +327,7 @@ def run_ours(args):
                         "(K=8192), strmm LLNN, strsm LLNN; alpha=1.5 beta=0.5",
             "n": n, "k": n, "cols_per_rank": cols, "math": args.math,
             "l2": "no flush: every operand is 256 MiB > 126 MB L2",
-            "parallelism": (f"dp{world}: column slabs of B/C/X per rank (8192 columns each), A and T "
+            "parallelism": (f"dp{world}: column slabs of B/C/X per rank ({cols} columns each), A and T "
                             f"broadcast from rank 0 (NCCL); ssyrk/ssyr2k k-split, partials "
                             f"all-reduced (NCCL)") if world > 1 else "1 GPU",
         },
@@ -452,7 +452,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--math", default="3xtf32", choices=["3xtf32", "simt"])
-    ap.add_argument("--n", type=int, default=N)
+    ap.add_argument("--size", type=int, default=N, help="matrix order (default 8192)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the e2e leg (profiling runs)")

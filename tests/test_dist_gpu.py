@@ -74,7 +74,16 @@ def test_virtual_ranks_syrk_balanced(mods, two, uplo, trans):
     for r in range(world):
         d3._tri_slab_products(two, uplo, trans, 1.5, dA, dB if two else None, 0.5, dsl,
                               d3.balanced_tri_slabs(n, world, r))
-    assert np.array_equal(bits(to_host(dfull)), bits(to_host(dsl)))
+    full, sl = to_host(dfull), to_host(dsl)
+    if two:
+        # off-diagonal slabs = two SGEMMs (C rounded in between): same product,
+        # different rounding grouping -> compare with the north-star tolerance
+        mask = np.tril(np.ones((n, n), bool)) if uplo == "L" else np.triu(np.ones((n, n), bool))
+        scale = 1.5 * fro(A) * fro(B) + 0.5 * fro(C[mask])
+        assert e_nw(sl[mask], full[mask].astype(np.float64), scale) <= TOL_NW
+        assert np.array_equal(bits(sl[~mask]), bits(full[~mask]))
+    else:
+        assert np.array_equal(bits(full), bits(sl))
 
 
 def test_pipelined_sgemm_panels(mods, oracle_mod):
