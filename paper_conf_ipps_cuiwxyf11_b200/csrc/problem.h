@@ -68,6 +68,10 @@ struct Problem {
   // the same shape; seg[0] operands and C advance by the strides below.
   int64_t nbatch, per;
   BatchStride bs_a, bs_b, bs_c;
+  // performance-experiment knobs (env BLAS3_DEBUG_TC; results are WRONG when
+  // set, never used by tests or the bench): bit0 skip the split pass,
+  // bit1 issue only hi*hi (1xTF32), bit2 skip the epilogue stores
+  int32_t dbg;
 };
 
 HD int64_t batch_off(const BatchStride &s, int64_t b, int64_t per) {

@@ -3,8 +3,9 @@
 // -> epilogue.  Rows A2-A6 of the hot-path table.
 //
 // Paper mapping:
-//   thread_grouping / loop_tiling  -> persistent CTAs over a
-//       128x256 tile schedule (Tiles<> in problem.h), BK = 32 k-blocks;
+//   thread_grouping / loop_tiling  -> persistent CTAs (or CTA
+//       pairs, tcgen05 cta_group::2) over a 128x256 (256x256) tile schedule
+//       (Tiles<> in problem.h), BK = 32 k-blocks;
 //   SM_alloc(X, Transpose|Symmetry)   -> TMA loads each k-block in
 //       the orientation it is stored in (K-major or MN-major 128B-swizzled
 //       tiles; the UMMA descriptor's major bit absorbs the transpose), and
@@ -20,7 +21,8 @@
 // word) and lo = rna_tf32(x - hi), and each k-step issues lo*hi + hi*lo +
 // hi*hi (small terms first) into the same fp32 accumulator.
 //
-// Warp roles (576 threads, 1 CTA/SM):
+// Warp roles (576 threads, 1 CTA/SM; in a pair every CTA runs all roles on its
+// own halves except the MMA issuer, which only the leader CTA runs):
 //   warp 0       TMA producer (one lane)
 //   warp 1       TMEM allocator + MMA issuer (one lane)
 //   warps 2..9   transform: structure fix-ups + hi/lo split (256 threads)
@@ -29,6 +31,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <mutex>
+#include <stdlib.h>
 #include <string.h>
 
 #include "kernels.h"
@@ -37,32 +40,53 @@
 namespace blas3 {
 
 namespace {
-constexpr int BM = 128, BN = 256, BK = 32, STAGES = 2;
+// Tile geometry.  CG = CTA group: CG=1 -> one CTA computes a 128x256 tile;
+// CG=2 -> a CTA pair (cluster of 2, tcgen05 cta_group::2) computes a 256x256
+// tile, each CTA staging its 128 rows of A and 128 of the 256 B rows: per SM
+// the tensor core reads half as many B bytes per flop, and shared-memory
+// bandwidth is what bounds this kernel (profiles/r01_sgemm_ncu.md).
+constexpr int BK = 32;
+constexpr int HA = 128;                    // A rows staged per CTA
+constexpr int BN = 256;                    // tile columns (UMMA N)
 constexpr int WARP_TMA = 0, WARP_MMA = 1, WARP_TR0 = 2, NUM_TR_WARPS = 8;
 constexpr int WARP_EPI0 = WARP_TR0 + NUM_TR_WARPS, NUM_EPI_WARPS = 8;
 constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;
 constexpr int TR_THREADS = NUM_TR_WARPS * 32;
-constexpr uint32_t A_BYTES = BM * BK * 4;
-constexpr uint32_t B_BYTES = BN * BK * 4;
-constexpr int TMEM_COLS = 512;          // 2 accumulators x BN columns
+constexpr int EPI_THREADS = NUM_EPI_WARPS * 32;
+constexpr int TMEM_COLS = 512;             // 2 accumulators x BN columns
 constexpr int MAX_MAPS = 8;
 constexpr int LAYOUT_K = 0, LAYOUT_MN = 1;
 
-struct alignas(1024) StageBuf {
-  uint8_t rawA[A_BYTES];   // TMA destination; read by UMMA as hi (low 13 bits ignored)
-  uint8_t rawB[B_BYTES];
-  uint8_t loA[A_BYTES];    // lo (tf32); also the kr-view landing zone of
-  uint8_t loB[B_BYTES];    //   symmetric diagonal blocks before the merge
+// Two shared-memory rings: a deep RAW ring (TMA destination, read by UMMA as
+// hi) lets TMA run RS k-blocks ahead to hide load latency, and a shallow LO
+// ring (written by the transform) only has to cover transform/MMA overlap.
+template <int CG>
+struct Geo {
+  static constexpr int TM = HA * CG;                 // tile rows
+  static constexpr int HB = BN / CG;                 // B rows staged per CTA
+  static constexpr uint32_t A_BYTES = HA * BK * 4;
+  static constexpr uint32_t B_BYTES = HB * BK * 4;
+  static constexpr int RS = CG == 1 ? 2 : 4;         // raw stages
+  static constexpr int LS = 2;                       // lo stages
+  struct alignas(1024) RawBuf {
+    uint8_t A[A_BYTES];      // TMA destination; read by UMMA as hi (low 13 bits ignored)
+    uint8_t B[B_BYTES];
+  };
+  struct alignas(1024) LoBuf {
+    uint8_t A[A_BYTES];      // lo = rna_tf32(x - hi), written by the transform
+    uint8_t B[B_BYTES];
+  };
+  struct Barriers {
+    uint64_t full[RS];       // TMA -> transform (expect_tx), local
+    uint64_t empty[RS];      // MMA -> TMA: raw slot free (tcgen05.commit, multicast)
+    uint64_t ready[LS];      // transform -> MMA (one arrival per CTA of the pair, leader)
+    uint64_t lo_empty[LS];   // MMA -> transform: lo slot free (tcgen05.commit, multicast)
+    uint64_t tfull[2];       // MMA -> epilogue (multicast to the pair)
+    uint64_t tempty[2];      // epilogue -> MMA (one arrival per CTA of the pair, leader)
+    uint32_t tmem_base;
+  };
+  static constexpr size_t SMEM = sizeof(RawBuf) * RS + sizeof(LoBuf) * LS + sizeof(Barriers) + 1024;
 };
-struct Barriers {
-  uint64_t full[STAGES];   // TMA -> transform (expect_tx)
-  uint64_t ready[STAGES];  // transform -> MMA (TR_THREADS arrivals)
-  uint64_t empty[STAGES];  // MMA -> TMA (tcgen05.commit)
-  uint64_t tfull[2];       // MMA -> epilogue
-  uint64_t tempty[2];      // epilogue -> MMA (256 arrivals)
-  uint32_t tmem_base;
-};
-constexpr size_t SMEM_BYTES = sizeof(StageBuf) * STAGES + sizeof(Barriers) + 1024;
 
 struct TcParams {
   CUtensorMap maps[MAX_MAPS];
@@ -91,30 +115,36 @@ struct StageInfo {
   int clsA, clsB, layA, layB;
 };
 
+// Block classes are decided on the WHOLE tile (both CTAs of a pair), so the
+// UMMA major bits agree for the two halves; a half whose own block would be
+// plain real/shadow is then merged per element, which selects the same values.
+template <int CG>
 __device__ __forceinline__ StageInfo stage_info(const Problem &P, const Segment &sg, int64_t m0,
                                                 int64_t n0, int64_t k0) {
   StageInfo si;
   const int64_t k1 = imin(sg.K, k0 + BK);
-  si.clsA = block_class(sg.a, m0, imin(P.M, m0 + BM), k0, k1);
+  si.clsA = block_class(sg.a, m0, imin(P.M, m0 + Geo<CG>::TM), k0, k1);
   si.clsB = block_class(sg.b, n0, imin(P.N, n0 + BN), k0, k1);
   si.layA = layout_of(sg.a, si.clsA);
   si.layB = layout_of(sg.b, si.clsB);
   return si;
 }
 
+template <int CG>
 __device__ __forceinline__ void seg_kblocks(const Problem &P, const Segment &sg, int64_t m0,
                                             int64_t n0, int64_t &kb0, int64_t &kb1) {
   int64_t k0, k1;
-  k_range(sg, m0, imin(P.M, m0 + BM), n0, imin(P.N, n0 + BN), k0, k1);
+  k_range(sg, m0, imin(P.M, m0 + Geo<CG>::TM), n0, imin(P.N, n0 + BN), k0, k1);
   kb0 = k0 / BK;
   kb1 = (k1 > k0) ? cdiv(k1, BK) : kb0;
 }
 
+template <int CG>
 __device__ __forceinline__ int64_t tile_kblocks(const Problem &P, int64_t m0, int64_t n0) {
   int64_t tot = 0;
   for (int s = 0; s < P.nseg; ++s) {
     int64_t a, b;
-    seg_kblocks(P, P.seg[s], m0, n0, a, b);
+    seg_kblocks<CG>(P, P.seg[s], m0, n0, a, b);
     tot += b - a;
   }
   return tot;
@@ -123,11 +153,9 @@ __device__ __forceinline__ int64_t tile_kblocks(const Problem &P, int64_t m0, in
 // ---------------------------------------------------------------- producer
 // Every operand map is 4-D: (element dims) x (batch-inner, batch-outer);
 // (bj, bg) select the batch member (0, 0 for an ordinary problem).
-__device__ __forceinline__ uint32_t load_operand(const TcParams &prm, const OpDesc &o, int cls,
-                                                 int lay, uint8_t *raw, uint8_t *lo, int64_t r0,
-                                                 int64_t k0, int rows, uint64_t *bar, int32_t bj,
-                                                 int32_t bg) {
-  uint32_t bytes = 0;
+__device__ __forceinline__ void load_operand(const TcParams &prm, const OpDesc &o, int lay,
+                                             uint8_t *raw, int64_t r0, int64_t k0, int rows,
+                                             uint64_t *bar, int32_t bj, int32_t bg) {
   if (lay == LAYOUT_MN) {
     const CUtensorMap *m = &prm.maps[o.map_rk];
     for (int c = 0; c < rows / 32; ++c) {
@@ -136,29 +164,21 @@ __device__ __forceinline__ uint32_t load_operand(const TcParams &prm, const OpDe
   } else {
     ptx::tma_load_4d(&prm.maps[o.map_kr], bar, raw, (int32_t)k0, (int32_t)r0, bj, bg);
   }
-  bytes += rows * BK * 4;
-  if (cls == BLK_SYM_DIAG) {       // the mirrored orientation lands in the lo buffer
-    ptx::tma_load_4d(&prm.maps[o.map_kr], bar, lo, (int32_t)k0, (int32_t)r0, bj, bg);
-    bytes += rows * BK * 4;
-  }
-  return bytes;
-}
-
-__device__ __forceinline__ uint32_t operand_bytes(int cls, int rows) {
-  return rows * BK * 4 * (cls == BLK_SYM_DIAG ? 2 : 1);
 }
 
 // ---------------------------------------------------------------- transform
-// Symmetric block crossing the diagonal: elements whose stored position is
-// the mirrored one are copied from the kr-view tile (in lo) into the rk tile.
-__device__ __forceinline__ void sym_merge(const OpDesc &o, uint8_t *raw, const uint8_t *krtile,
-                                          int64_t r0, int64_t k0, int rows, int t) {
+// Symmetric block crossing the diagonal (staged from the rk view): elements
+// whose stored position is the mirrored one (the "shadow area")
+// are SELECTED from the stored triangle, S(r,k) := S(k,r), read straight from
+// global memory (rare blocks; keeps the raw ring free of a second view).
+__device__ __forceinline__ void sym_merge(const OpDesc &o, uint8_t *raw, int64_t r0, int64_t k0,
+                                          int rows, int64_t R, int64_t K, int t) {
   for (int e = t; e < rows * BK; e += TR_THREADS) {
     int r = e % rows, k = e / rows;
     int64_t gr = r0 + r, gk = k0 + k;
     bool mirrored = o.lower ? (gr < gk) : (gr > gk);
-    if (mirrored) *reinterpret_cast<float *>(raw + off_mn(r, k)) =
-        *reinterpret_cast<const float *>(krtile + off_k(r, k));
+    if (mirrored && gr < R && gk < K)
+      *reinterpret_cast<float *>(raw + off_mn(r, k)) = __ldg(o.ptr + gk + gr * o.ld);
   }
 }
 
@@ -212,172 +232,221 @@ __device__ __forceinline__ uint64_t op_desc(uint32_t base, int lay, int k8) {
   return ptx::smem_desc(base + k8 * 32, 16, 1024, 2);
 }
 
+// A role's warps (nthreads, named barrier `id`) have finished with a stage:
+// sync them CTA-locally, then ONE thread arrives on the barrier owned by the
+// pair's leader (a cluster-scope release per thread would cost a GPU-scope
+// membar + L1 invalidate each).
+template <int CG>
+__device__ __forceinline__ void arrive_leader(uint64_t *bar, uint32_t rank, uint32_t id,
+                                              uint32_t nthreads, bool first) {
+  ptx::named_bar_sync(id, nthreads);
+  if (first) {
+    if (CG == 1 || rank == 0) ptx::mbar_arrive(bar);
+    else ptx::mbar_arrive_cluster(bar, 0);
+  }
+}
+
 }  // namespace
 
+template <int CG>
 __global__ void __launch_bounds__(NTHREADS, 1)
 tc_structured_gemm(const __grid_constant__ TcParams prm) {
+  using G = Geo<CG>;
+  using RawBuf = typename G::RawBuf;
+  using LoBuf = typename G::LoBuf;
+  using Barriers = typename G::Barriers;
+  constexpr int RS = G::RS, LS = G::LS, TM = G::TM, HB = G::HB;
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  StageBuf *st = reinterpret_cast<StageBuf *>(smem);
-  Barriers *bars = reinterpret_cast<Barriers *>(smem + sizeof(StageBuf) * STAGES);
+  RawBuf *raw = reinterpret_cast<RawBuf *>(smem);
+  LoBuf *lo = reinterpret_cast<LoBuf *>(smem + sizeof(RawBuf) * RS);
+  Barriers *bars = reinterpret_cast<Barriers *>(smem + sizeof(RawBuf) * RS + sizeof(LoBuf) * LS);
   const Problem &P = prm.P;
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const uint32_t rank = (CG == 2) ? ptx::cluster_ctarank() : 0;
+  const int64_t cid = blockIdx.x / CG, ncl = gridDim.x / CG;
 
   if (threadIdx.x == 0) {
-    for (int s = 0; s < STAGES; ++s) {
+    for (int s = 0; s < RS; ++s) {
       ptx::mbar_init(&bars->full[s], 1);
-      ptx::mbar_init(&bars->ready[s], TR_THREADS);
       ptx::mbar_init(&bars->empty[s], 1);
+    }
+    for (int s = 0; s < LS; ++s) {
+      ptx::mbar_init(&bars->ready[s], CG);
+      ptx::mbar_init(&bars->lo_empty[s], 1);
     }
     for (int a = 0; a < 2; ++a) {
       ptx::mbar_init(&bars->tfull[a], 1);
-      ptx::mbar_init(&bars->tempty[a], NUM_EPI_WARPS * 32);
+      ptx::mbar_init(&bars->tempty[a], CG);
     }
     ptx::fence_mbar_init();
   }
-  if (warp == WARP_MMA) ptx::tmem_alloc(&bars->tmem_base, TMEM_COLS);
+  if (warp == WARP_MMA) ptx::tmem_alloc<CG>(&bars->tmem_base, TMEM_COLS);
   ptx::tc_fence_before();
-  __syncthreads();
+  if (CG == 2) ptx::cluster_sync(); else __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = bars->tmem_base;
 
   // batched problems: tile tb -> batch member b = tb / tiles_per, tile t
-  const int64_t tiles_per = Tiles<BM, BN>::count(P);
+  const int64_t tiles_per = Tiles<TM, BN>::count(P);
   const int64_t per = P.per > 0 ? P.per : 1;
   const int64_t ntiles = tiles_per * (P.nbatch > 0 ? P.nbatch : 1);
 
   if (warp == WARP_TMA) {
-    // ============================ TMA producer
+    // ============================ TMA producer (each CTA stages its own halves)
     if (lane == 0) {
       for (int i = 0; i < MAX_MAPS; ++i) ptx::tma_prefetch(&prm.maps[i]);
       uint32_t it = 0;
-      for (int64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x) {
+      for (int64_t tb = cid; tb < ntiles; tb += ncl) {
         const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
         const int32_t bj = (int32_t)(b % per), bg = (int32_t)(b / per);
         int64_t mi, nj;
-        Tiles<BM, BN>::coords(P, t, mi, nj);
-        const int64_t m0 = mi * BM, n0 = nj * BN;
+        Tiles<TM, BN>::coords(P, t, mi, nj);
+        const int64_t m0 = mi * TM, n0 = nj * BN;
+        const int64_t ma = m0 + HA * rank, nb = n0 + HB * rank;
         for (int s = 0; s < P.nseg; ++s) {
           const Segment &sg = P.seg[s];
           int64_t kb0, kb1;
-          seg_kblocks(P, sg, m0, n0, kb0, kb1);
+          seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
-            const int stg = it % STAGES;
-            const uint32_t ph = (it / STAGES) & 1;
+            const int rs = it % RS;
+            const uint32_t ph = (it / RS) & 1;
             const int64_t k0 = kb * BK;
-            StageInfo si = stage_info(P, sg, m0, n0, k0);
-            ptx::mbar_wait(&bars->empty[stg], ph ^ 1);
-            ptx::mbar_arrive_expect_tx(&bars->full[stg],
-                                       operand_bytes(si.clsA, BM) + operand_bytes(si.clsB, BN));
-            load_operand(prm, sg.a, si.clsA, si.layA, st[stg].rawA, st[stg].loA, m0, k0, BM,
-                         &bars->full[stg], bj, bg);
-            load_operand(prm, sg.b, si.clsB, si.layB, st[stg].rawB, st[stg].loB, n0, k0, BN,
-                         &bars->full[stg], bj, bg);
+            const StageInfo si = stage_info<CG>(P, sg, m0, n0, k0);
+            ptx::mbar_wait(&bars->empty[rs], ph ^ 1);
+            ptx::mbar_arrive_expect_tx(&bars->full[rs], (HA + HB) * BK * 4);
+            load_operand(prm, sg.a, si.layA, raw[rs].A, ma, k0, HA, &bars->full[rs], bj, bg);
+            load_operand(prm, sg.b, si.layB, raw[rs].B, nb, k0, HB, &bars->full[rs], bj, bg);
           }
         }
       }
-      // producer tail: every stage released by the MMA before the CTA retires
-      for (int i = 0; i < STAGES; ++i, ++it)
-        ptx::mbar_wait(&bars->empty[it % STAGES], ((it / STAGES) & 1) ^ 1);
+      // producer tail: every raw slot released by the MMA before the CTA retires
+      for (int i = 0; i < RS; ++i, ++it)
+        ptx::mbar_wait(&bars->empty[it % RS], ((it / RS) & 1) ^ 1);
     }
   } else if (warp == WARP_MMA) {
-    // ============================ MMA issuer
-    uint32_t it = 0, tcount = 0;
-    const uint32_t sA[STAGES] = {ptx::smem_u32(st[0].rawA), ptx::smem_u32(st[1].rawA)};
-    for (int64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x, ++tcount) {
-      const int64_t t = tb % tiles_per;
-      int64_t mi, nj;
-      Tiles<BM, BN>::coords(P, t, mi, nj);
-      const int64_t m0 = mi * BM, n0 = nj * BN;
-      const uint32_t acc = tcount & 1, aph = (tcount >> 1) & 1;
-      ptx::mbar_wait(&bars->tempty[acc], aph ^ 1);
-      ptx::tc_fence_after();
-      const uint32_t d_tmem = tmem + acc * BN;
-      uint32_t accumulate = 0;
-      for (int s = 0; s < P.nseg; ++s) {
-        const Segment &sg = P.seg[s];
-        int64_t kb0, kb1;
-        seg_kblocks(P, sg, m0, n0, kb0, kb1);
-        for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
-          const int stg = it % STAGES;
-          const uint32_t ph = (it / STAGES) & 1;
-          StageInfo si = stage_info(P, sg, m0, n0, kb * BK);
-          ptx::mbar_wait(&bars->ready[stg], ph);
-          ptx::tc_fence_after();
-          if (lane == 0) {
-            const uint32_t hiA = sA[stg], hiB = hiA + A_BYTES;
-            const uint32_t loA = hiB + B_BYTES, loB = loA + A_BYTES;
-            const uint32_t idesc = ptx::idesc_tf32(BM, BN, si.layA == LAYOUT_MN, si.layB == LAYOUT_MN);
+    // ============================ MMA issuer (leader CTA of the pair only)
+    if (rank == 0) {
+      uint32_t it = 0, tcount = 0;
+      for (int64_t tb = cid; tb < ntiles; tb += ncl, ++tcount) {
+        const int64_t t = tb % tiles_per;
+        int64_t mi, nj;
+        Tiles<TM, BN>::coords(P, t, mi, nj);
+        const int64_t m0 = mi * TM, n0 = nj * BN;
+        const uint32_t acc = tcount & 1, aph = (tcount >> 1) & 1;
+        if (CG == 2) ptx::mbar_wait_cluster(&bars->tempty[acc], aph ^ 1);
+        else ptx::mbar_wait(&bars->tempty[acc], aph ^ 1);
+        ptx::tc_fence_after();
+        const uint32_t d_tmem = tmem + acc * BN;
+        uint32_t accumulate = 0;
+        for (int s = 0; s < P.nseg; ++s) {
+          const Segment &sg = P.seg[s];
+          int64_t kb0, kb1;
+          seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
+          for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
+            const int rs = it % RS, ls = it % LS;
+            const uint32_t lph = (it / LS) & 1;
+            const StageInfo si = stage_info<CG>(P, sg, m0, n0, kb * BK);
+            if (CG == 2) ptx::mbar_wait_cluster(&bars->ready[ls], lph);
+            else ptx::mbar_wait(&bars->ready[ls], lph);
+            ptx::tc_fence_after();
+            if (lane == 0) {
+              const uint32_t hiA = ptx::smem_u32(raw[rs].A), hiB = ptx::smem_u32(raw[rs].B);
+              const uint32_t loA = ptx::smem_u32(lo[ls].A), loB = ptx::smem_u32(lo[ls].B);
+              const uint32_t idesc = ptx::idesc_tf32(TM, BN, si.layA == LAYOUT_MN, si.layB == LAYOUT_MN);
 #pragma unroll
-            for (int k8 = 0; k8 < BK / 8; ++k8) {
-              const uint64_t ah = op_desc(hiA, si.layA, k8), al = op_desc(loA, si.layA, k8);
-              const uint64_t bh = op_desc(hiB, si.layB, k8), bl = op_desc(loB, si.layB, k8);
-              ptx::mma_tf32_ss(d_tmem, al, bh, idesc, accumulate);
-              ptx::mma_tf32_ss(d_tmem, ah, bl, idesc, 1);
-              ptx::mma_tf32_ss(d_tmem, ah, bh, idesc, 1);
-              accumulate = 1;
+              for (int k8 = 0; k8 < BK / 8; ++k8) {
+                const uint64_t ah = op_desc(hiA, si.layA, k8), al = op_desc(loA, si.layA, k8);
+                const uint64_t bh = op_desc(hiB, si.layB, k8), bl = op_desc(loB, si.layB, k8);
+                const bool one = P.dbg & 2;
+                if constexpr (CG == 1) {
+                  if (!one) ptx::mma_tf32_ss(d_tmem, al, bh, idesc, accumulate);
+                  if (!one) ptx::mma_tf32_ss(d_tmem, ah, bl, idesc, 1);
+                  ptx::mma_tf32_ss(d_tmem, ah, bh, idesc, one ? accumulate : 1);
+                } else {
+                  if (!one) ptx::mma_tf32_ss_pair(d_tmem, al, bh, idesc, accumulate);
+                  if (!one) ptx::mma_tf32_ss_pair(d_tmem, ah, bl, idesc, 1);
+                  ptx::mma_tf32_ss_pair(d_tmem, ah, bh, idesc, one ? accumulate : 1);
+                }
+                accumulate = 1;
+              }
+              if constexpr (CG == 1) {
+                ptx::mma_commit(&bars->empty[rs]);
+                ptx::mma_commit(&bars->lo_empty[ls]);
+              } else {
+                ptx::mma_commit_pair(&bars->empty[rs], 0x3);
+                ptx::mma_commit_pair(&bars->lo_empty[ls], 0x3);
+              }
             }
-            ptx::mma_commit(&bars->empty[stg]);
+            accumulate = 1;
+            __syncwarp();
           }
-          accumulate = 1;
-          __syncwarp();
         }
+        if (lane == 0) {
+          if (accumulate) {
+            if constexpr (CG == 1) ptx::mma_commit(&bars->tfull[acc]);
+            else ptx::mma_commit_pair(&bars->tfull[acc], 0x3);
+          } else {                                   // empty k-range: accumulator = 0
+            ptx::mbar_arrive(&bars->tfull[acc]);
+            if (CG == 2) ptx::mbar_arrive_cluster(&bars->tfull[acc], 1);
+          }
+        }
+        __syncwarp();
       }
-      if (lane == 0) {
-        if (accumulate) ptx::mma_commit(&bars->tfull[acc]);
-        else ptx::mbar_arrive(&bars->tfull[acc]);     // empty k-range: accumulator = 0
-      }
-      __syncwarp();
     }
   } else if (warp < WARP_EPI0) {
-    // ============================ transform warps
+    // ============================ transform warps (own halves; arrive at the leader)
     const int tt = threadIdx.x - WARP_TR0 * 32;
     uint32_t it = 0;
-    for (int64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x) {
+    for (int64_t tb = cid; tb < ntiles; tb += ncl) {
       const int64_t t = tb % tiles_per;
       int64_t mi, nj;
-      Tiles<BM, BN>::coords(P, t, mi, nj);
-      const int64_t m0 = mi * BM, n0 = nj * BN;
+      Tiles<TM, BN>::coords(P, t, mi, nj);
+      const int64_t m0 = mi * TM, n0 = nj * BN;
+      const int64_t ma = m0 + HA * rank, nb = n0 + HB * rank;
       for (int s = 0; s < P.nseg; ++s) {
         const Segment &sg = P.seg[s];
         int64_t kb0, kb1;
-        seg_kblocks(P, sg, m0, n0, kb0, kb1);
+        seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
         for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
-          const int stg = it % STAGES;
-          const uint32_t ph = (it / STAGES) & 1;
+          const int rs = it % RS, ls = it % LS;
+          const uint32_t ph = (it / RS) & 1, lph = (it / LS) & 1;
           const int64_t k0 = kb * BK;
-          StageInfo si = stage_info(P, sg, m0, n0, k0);
-          ptx::mbar_wait(&bars->full[stg], ph);
-          StageBuf &b = st[stg];
+          const StageInfo si = stage_info<CG>(P, sg, m0, n0, k0);
+          ptx::mbar_wait(&bars->full[rs], ph);
+          RawBuf &rb = raw[rs];
           bool fix = false;
-          if (si.clsA == BLK_SYM_DIAG) { sym_merge(sg.a, b.rawA, b.loA, m0, k0, BM, tt); fix = true; }
-          else if (si.clsA == BLK_TRI_DIAG) { tri_fix(sg.a, si.layA, b.rawA, m0, k0, BM, P.M, sg.K, tt); fix = true; }
-          if (si.clsB == BLK_SYM_DIAG) { sym_merge(sg.b, b.rawB, b.loB, n0, k0, BN, tt); fix = true; }
-          else if (si.clsB == BLK_TRI_DIAG) { tri_fix(sg.b, si.layB, b.rawB, n0, k0, BN, P.N, sg.K, tt); fix = true; }
+          if (si.clsA == BLK_SYM_DIAG) { sym_merge(sg.a, rb.A, ma, k0, HA, P.M, sg.K, tt); fix = true; }
+          else if (si.clsA == BLK_TRI_DIAG) { tri_fix(sg.a, si.layA, rb.A, ma, k0, HA, P.M, sg.K, tt); fix = true; }
+          if (si.clsB == BLK_SYM_DIAG) { sym_merge(sg.b, rb.B, nb, k0, HB, P.N, sg.K, tt); fix = true; }
+          else if (si.clsB == BLK_TRI_DIAG) { tri_fix(sg.b, si.layB, rb.B, nb, k0, HB, P.N, sg.K, tt); fix = true; }
           if (fix) ptx::named_bar_sync(1, TR_THREADS);
-          split_pass(b.rawA, b.loA, A_BYTES, tt);
-          split_pass(b.rawB, b.loB, B_BYTES, tt);
+          ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
+          if (!(P.dbg & 1)) {
+            split_pass(rb.A, lo[ls].A, G::A_BYTES, tt);
+            split_pass(rb.B, lo[ls].B, G::B_BYTES, tt);
+          }
           ptx::fence_proxy_async_smem();
-          ptx::mbar_arrive(&bars->ready[stg]);
+          arrive_leader<CG>(&bars->ready[ls], rank, 2, TR_THREADS, tt == 0);
         }
       }
     }
   } else {
-    // ============================ epilogue warps
+    // ============================ epilogue warps (own 128 rows, all BN columns)
     const int q = warp & 3;                     // TMEM lane quarter of this warp
     const int half = (warp - WARP_EPI0) >> 2;   // which 128 of the 256 columns
     uint32_t tcount = 0;
-    for (int64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x, ++tcount) {
+    for (int64_t tb = cid; tb < ntiles; tb += ncl, ++tcount) {
       const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
       const int64_t coff = (P.nbatch > 1) ? batch_off(P.bs_c, b, per) : 0;
       int64_t mi, nj;
-      Tiles<BM, BN>::coords(P, t, mi, nj);
-      const int64_t m0 = mi * BM, n0 = nj * BN;
-      const bool has_k = tile_kblocks(P, m0, n0) > 0;
+      Tiles<TM, BN>::coords(P, t, mi, nj);
+      const int64_t m0 = mi * TM, n0 = nj * BN;
+      const bool has_k = tile_kblocks<CG>(P, m0, n0) > 0;
       const uint32_t acc = tcount & 1, aph = (tcount >> 1) & 1;
       ptx::mbar_wait(&bars->tfull[acc], aph);
       ptx::tc_fence_after();
-      const int64_t r = m0 + q * 32 + lane;
+      const int64_t r = m0 + HA * rank + q * 32 + lane;
       const bool row_ok = r < P.M;
       const float *cin = P.Cin + coff + r;
       float *cout = P.Cout + coff + r;
@@ -406,19 +475,19 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
         for (int j = 0; j < EC; ++j) {
           const int64_t c = c0 + j;
           const bool ok = row_ok && c < P.N && !(P.c_tri == 1 && r < c) && !(P.c_tri == 2 && r > c);
-          if (ok) cout[c * P.ldcout] = fmaf(P.beta, cv[j], P.alpha * __uint_as_float(v[j]));
+          if (ok && !(P.dbg & 4)) cout[c * P.ldcout] = fmaf(P.beta, cv[j], P.alpha * __uint_as_float(v[j]));
         }
       }
       ptx::tc_fence_before();
-      ptx::mbar_arrive(&bars->tempty[acc]);
+      arrive_leader<CG>(&bars->tempty[acc], rank, 3, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
     }
   }
 
   ptx::tc_fence_before();
-  __syncthreads();
+  if (CG == 2) ptx::cluster_sync(); else __syncthreads();
   if (warp == WARP_MMA) {
     ptx::tc_fence_after();
-    ptx::tmem_dealloc(tmem, TMEM_COLS);
+    ptx::tmem_dealloc<CG>(tmem, TMEM_COLS);
   }
 }
 
@@ -495,33 +564,71 @@ bool tc_eligible(const Problem &P) {
   return true;
 }
 
-int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
-  static TcParams prm;                    // host staging (the launch copies it)
-  static std::mutex mu;
-  std::lock_guard<std::mutex> lk(mu);
-  memset(&prm, 0, sizeof(prm));
-  prm.P = P0;
+// CTA-group choice.  The pair kernel (CG=2, 256x256 tiles, cta_group::2) is
+// parity-green but measured slower than CG=1 on B200 so far (DESIGN.md §7:
+// 159-197 vs 200 TF/s at 8192^3), so CG=1 is the default; BLAS3_TC_CTA=2
+// selects the pair kernel (tests run both).
+static int choose_cg(const Problem &P, int num_sms) {
+  static int forced = -1;
+  if (forced < 0) {
+    const char *e = getenv("BLAS3_TC_CTA");
+    forced = (e && e[0] == '2') ? 2 : 1;
+  }
+  (void)P; (void)num_sms;
+  return forced;
+}
+
+template <int CG>
+static int launch_cg(TcParams &prm, cudaStream_t stream, int num_sms) {
+  using G = Geo<CG>;
   int slot = 0;
   for (int s = 0; s < prm.P.nseg; ++s) {
     Segment &sg = prm.P.seg[s];
     if (sg.K <= 0) continue;
     const int64_t nb = prm.P.nbatch > 1 ? prm.P.nbatch : 1;
     const int64_t per = nb > 1 ? prm.P.per : 1, groups = cdiv(nb, per);
-    if (!op_maps(prm, slot, sg.a, prm.P.M, sg.K, BM, per, groups, prm.P.bs_a)) return -4;
-    if (!op_maps(prm, slot, sg.b, prm.P.N, sg.K, BN, per, groups, prm.P.bs_b)) return -4;
+    if (!op_maps(prm, slot, sg.a, prm.P.M, sg.K, HA, per, groups, prm.P.bs_a)) return -4;
+    if (!op_maps(prm, slot, sg.b, prm.P.N, sg.K, G::HB, per, groups, prm.P.bs_b)) return -4;
   }
   static bool attr = false;
   if (!attr) {
-    if (cudaFuncSetAttribute(tc_structured_gemm, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)SMEM_BYTES) != cudaSuccess) return -1;
+    if (cudaFuncSetAttribute(tc_structured_gemm<CG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)G::SMEM) != cudaSuccess) return -1;
     attr = true;
   }
-  const int64_t tiles = Tiles<BM, BN>::count(prm.P) * (prm.P.nbatch > 1 ? prm.P.nbatch : 1);
+  const int64_t tiles = Tiles<G::TM, BN>::count(prm.P) * (prm.P.nbatch > 1 ? prm.P.nbatch : 1);
   if (tiles == 0) return 0;
-  const int64_t grid = imin(tiles, (int64_t)num_sms);
-  tc_structured_gemm<<<(unsigned)grid, NTHREADS, SMEM_BYTES, stream>>>(prm);
+  const int64_t units = imin(tiles, (int64_t)(num_sms / CG));      // CTAs (CG=1) or pairs
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(units * CG));
+  cfg.blockDim = dim3(NTHREADS);
+  cfg.dynamicSmemBytes = G::SMEM;
+  cfg.stream = stream;
+  cudaLaunchAttribute attrs[1];
+  attrs[0].id = cudaLaunchAttributeClusterDimension;
+  attrs[0].val.clusterDim.x = CG;
+  attrs[0].val.clusterDim.y = 1;
+  attrs[0].val.clusterDim.z = 1;
+  cfg.attrs = attrs;
+  cfg.numAttrs = 1;
+  const cudaError_t e = cudaLaunchKernelEx(&cfg, tc_structured_gemm<CG>, prm);
   note_launch(0);
-  return cudaGetLastError() == cudaSuccess ? 0 : -1;
+  return (e == cudaSuccess && cudaGetLastError() == cudaSuccess) ? 0 : -1;
+}
+
+int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
+  static TcParams prm;                    // host staging (the launch copies it)
+  static std::mutex mu;
+  std::lock_guard<std::mutex> lk(mu);
+  memset(&prm, 0, sizeof(prm));
+  prm.P = P0;
+  {
+    static int dbg = -1;
+    if (dbg < 0) { const char *e = getenv("BLAS3_DEBUG_TC"); dbg = e ? atoi(e) : 0; }
+    prm.P.dbg = dbg;
+  }
+  return choose_cg(prm.P, num_sms) == 2 ? launch_cg<2>(prm, stream, num_sms)
+                                        : launch_cg<1>(prm, stream, num_sms);
 }
 
 }  // namespace blas3
