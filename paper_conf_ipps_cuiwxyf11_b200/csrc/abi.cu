@@ -8,6 +8,7 @@
 #include <stdlib.h>
 #include <string.h>
 #include <atomic>
+#include <functional>
 #include <mutex>
 
 #include "../../include/blas3.h"
@@ -341,9 +342,10 @@ int blas3_strmm(char side, char uplo, char transa, char diag, int64_t m, int64_t
 //   2. 128 -> 256 -> 512 -> NBO doubling builds inv(L_pp) of every NBO-wide
 //      diagonal panel: for each diagonal pair [[L11,0],[L21,L22]],
 //      X21 = -inv(L22) * (L21 * inv(L11)) as two batched GEMMs per level;
-//   3. the sweep (row A8) visits panels in dependency order:
-//        X_p = alpha_p * inv(op(A)_pp) * B_p        (TRI operand, GEMM)
-//        B_rest <- alpha_p * B_rest - op(A)(rest, p) * X_p   (GEMM, K = NBO)
+//   3. the sweep (row A8) visits panels in dependency order, recursively
+//      halving the panel range: solve the first half, one GEMM update of the
+//      second half by the first (K = nt/2, nt/4, ...), solve the second half;
+//      a single panel is X_p = alpha_p * inv(op(A)_pp) * B_p (TRI operand).
 //      alpha is folded into the first operation that touches each row.
 // Every flop of steps 2-3 runs in the structured GEMM kernels.
 static const int64_t NBO = 1024;   // panel width (multiple of the 128 diagonal block)
@@ -422,44 +424,65 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   if ((rc = get_scratch(W, w_bytes, s, d_bytes + t_bytes))) return rc;
   if ((rc = trsm_panel_inverses(A, lda, nt, lower, unit, D.p, Tw.p, s, sms))) return rc;
 
-  for (int64_t q = 0; q < npanel; ++q) {
-    const int64_t p = forward ? q : npanel - 1 - q;
-    const int64_t p0 = p * NBO, pr = imin(NBO, nt - p0);
-    const float a1 = (q == 0) ? alpha : 1.f;       // first touch of every row/column
-    const float *Dp = D.p + p * NBO * NBO;
-    const int64_t o_lo = forward ? p0 + pr : 0, o_hi = forward ? nt : p0;
-    if (left) {
-      // X_p = a1 * inv(op(A)_pp) * B_p: Xa(r,k) = Dop(r,k), Dop = lower_op ? D : D^T
-      Problem P = problem(pr, n, a1, 0.f, nullptr, 0, W.p, pr);
-      P.seg[0].a = tri(Dp, NBO, true, !lower_op, false);
-      P.seg[0].b = dense(B + p0, ldb, true);
-      P.seg[0].K = pr;
-      P.rev_m = tri_kle(P.seg[0].a);
-      if ((rc = run_problem(P, s, sms))) return rc;
-      if (launch_copy(B + p0, ldb, W.p, pr, pr, n, s)) return BLAS3_ERR_CUDA;
-      if (o_hi > o_lo) {   // B_o <- a1*B_o - op(A)(o, p) * X_p
-        // Xa(r,k) = op(A)(o_lo+r, p0+k): !ta -> A(o_lo+r, p0+k) rk; ta -> A(p0+k, o_lo+r) kr
-        const float *pa = ta ? A + p0 + o_lo * lda : A + o_lo + p0 * lda;
-        if ((rc = gemm_dense(o_hi - o_lo, n, pr, -1.f, pa, lda, ta, W.p, pr, true, a1,
-                             B + o_lo, ldb, s, sms))) return rc;
+  // Recursive sweep over panels in processing order (forward or backward):
+  //   solve(first half); B_rest <- a*B_rest - op(A)(rest, first) * X_first;
+  //   solve(second half).
+  // The updates are few large-K GEMMs (K = nt/2, nt/4, ...) instead of one
+  // K = NBO GEMM per panel.  `scaled` says whether alpha has already been
+  // applied to the rows of the range (alpha is folded into the first touch).
+  auto elem = [&](int64_t qa, int64_t qb, int64_t &lo, int64_t &hi) {  // processing -> elements
+    const int64_t pa = forward ? qa : npanel - qb, pb = forward ? qb : npanel - qa;
+    lo = pa * NBO;
+    hi = imin(nt, pb * NBO);
+  };
+  std::function<int(int64_t, int64_t, bool)> rec = [&](int64_t q0, int64_t q1, bool scaled) -> int {
+    int rc2;
+    if (q1 - q0 == 1) {
+      const int64_t p = forward ? q0 : npanel - 1 - q0;
+      const int64_t p0 = p * NBO, pr = imin(NBO, nt - p0);
+      const float a1 = scaled ? 1.f : alpha;
+      const float *Dp = D.p + p * NBO * NBO;
+      if (left) {
+        // X_p = a1 * inv(op(A)_pp) * B_p: Xa(r,k) = Dop(r,k), Dop = lower_op ? D : D^T
+        Problem P = problem(pr, n, a1, 0.f, nullptr, 0, W.p, pr);
+        P.seg[0].a = tri(Dp, NBO, true, !lower_op, false);
+        P.seg[0].b = dense(B + p0, ldb, true);
+        P.seg[0].K = pr;
+        P.rev_m = tri_kle(P.seg[0].a);
+        if ((rc2 = run_problem(P, s, sms))) return rc2;
+        if (launch_copy(B + p0, ldb, W.p, pr, pr, n, s)) return BLAS3_ERR_CUDA;
+      } else {
+        // X_p = a1 * B_p * inv(op(A)_pp): Xb(c,k) = Dop(k,c) -> TRI swap = lower_op
+        Problem P = problem(m, pr, a1, 0.f, nullptr, 0, W.p, m);
+        P.seg[0].a = dense(B + p0 * ldb, ldb, false);
+        P.seg[0].b = tri(Dp, NBO, true, lower_op, false);
+        P.seg[0].K = pr;
+        P.rev_n = tri_kle(P.seg[0].b);
+        if ((rc2 = run_problem(P, s, sms))) return rc2;
+        if (launch_copy(B + p0 * ldb, ldb, W.p, m, m, pr, s)) return BLAS3_ERR_CUDA;
       }
-    } else {
-      // X_p = a1 * B_p * inv(op(A)_pp): Xb(c,k) = Dop(k,c) -> TRI swap = lower_op
-      Problem P = problem(m, pr, a1, 0.f, nullptr, 0, W.p, m);
-      P.seg[0].a = dense(B + p0 * ldb, ldb, false);
-      P.seg[0].b = tri(Dp, NBO, true, lower_op, false);
-      P.seg[0].K = pr;
-      P.rev_n = tri_kle(P.seg[0].b);
-      if ((rc = run_problem(P, s, sms))) return rc;
-      if (launch_copy(B + p0 * ldb, ldb, W.p, m, m, pr, s)) return BLAS3_ERR_CUDA;
-      if (o_hi > o_lo) {   // B(:,o) <- a1*B(:,o) - X_p * op(A)(p, o)
-        // Xb(c,k) = op(A)(p0+k, o_lo+c): !ta -> A(p0+k, o_lo+c) kr; ta -> A(o_lo+c, p0+k) rk
-        const float *pb = ta ? A + o_lo + p0 * lda : A + p0 + o_lo * lda;
-        if ((rc = gemm_dense(m, o_hi - o_lo, pr, -1.f, W.p, m, false, pb, lda, !ta, a1,
-                             B + o_lo * ldb, ldb, s, sms))) return rc;
-      }
+      return 0;
     }
-  }
+    const int64_t mid = q0 + (q1 - q0) / 2;
+    if ((rc2 = rec(q0, mid, scaled))) return rc2;
+    int64_t k_lo, k_hi, o_lo, o_hi;
+    elem(q0, mid, k_lo, k_hi);                       // solved part
+    elem(mid, q1, o_lo, o_hi);                       // part to update
+    const float a1 = scaled ? 1.f : alpha;
+    if (left) {   // B_o <- a1*B_o - op(A)(o, k) * X_k (X_k = B rows k)
+      // Xa(r,kk) = op(A)(o_lo+r, k_lo+kk): !ta -> A(o_lo+r, k_lo+kk) rk; ta -> A(k_lo+kk, o_lo+r) kr
+      const float *pa = ta ? A + k_lo + o_lo * lda : A + o_lo + k_lo * lda;
+      if ((rc2 = gemm_dense(o_hi - o_lo, n, k_hi - k_lo, -1.f, pa, lda, ta, B + k_lo, ldb, true, a1,
+                            B + o_lo, ldb, s, sms))) return rc2;
+    } else {      // B(:,o) <- a1*B(:,o) - X_k * op(A)(k, o)
+      // Xb(c,kk) = op(A)(k_lo+kk, o_lo+c): !ta -> A(k_lo+kk, o_lo+c) kr; ta -> A(o_lo+c, k_lo+kk) rk
+      const float *pb = ta ? A + o_lo + k_lo * lda : A + k_lo + o_lo * lda;
+      if ((rc2 = gemm_dense(m, o_hi - o_lo, k_hi - k_lo, -1.f, B + k_lo * ldb, ldb, false, pb, lda,
+                            !ta, a1, B + o_lo * ldb, ldb, s, sms))) return rc2;
+    }
+    return rec(mid, q1, true);
+  };
+  if ((rc = rec(0, npanel, false))) return rc;
   return finish(0);
 }
 

@@ -451,21 +451,30 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
       const float *cin = P.Cin + coff + r;
       float *cout = P.Cout + coff + r;
       constexpr int EC = 16;                    // epilogue chunk: 16 columns
-      for (int ch = half * (BN / EC / 2); ch < (half + 1) * (BN / EC / 2); ++ch) {
+      const int ch0 = half * (BN / EC / 2), ch1 = (half + 1) * (BN / EC / 2);
+      // C(r, c0..c0+15) of the NEXT chunk is loaded while the current chunk is
+      // stored (loads are issued before the stores in program order because
+      // Cin may alias Cout); each access is a coalesced 128-B warp access.
+      auto load_c = [&](int ch, float (&cv)[EC]) {
         const int64_t c0 = n0 + ch * EC;
-        if (c0 >= P.N) break;
-        uint32_t v[EC];
-        if (has_k) ptx::tmem_ld_32x32b_x16(tmem + acc * BN + ch * EC + ((uint32_t)(q * 32) << 16), v);
-        // C(r, c0..c0+15): all loads issued before any store (Cin may
-        // alias Cout, so interleaving would serialise every load behind the
-        // previous store); each is a coalesced 128-B warp access per column.
-        float cv[EC];
 #pragma unroll
         for (int j = 0; j < EC; ++j) {
           const int64_t c = c0 + j;
           const bool ok = row_ok && c < P.N && !(P.c_tri == 1 && r < c) && !(P.c_tri == 2 && r > c);
           cv[j] = (ok && P.beta != 0.f) ? cin[c * P.ldcin] : 0.f;
         }
+      };
+      float cnext[EC];
+      if (n0 + ch0 * EC < P.N) load_c(ch0, cnext);
+      for (int ch = ch0; ch < ch1; ++ch) {
+        const int64_t c0 = n0 + ch * EC;
+        if (c0 >= P.N) break;
+        float cv[EC];
+#pragma unroll
+        for (int j = 0; j < EC; ++j) cv[j] = cnext[j];
+        uint32_t v[EC];
+        if (has_k) ptx::tmem_ld_32x32b_x16(tmem + acc * BN + ch * EC + ((uint32_t)(q * 32) << 16), v);
+        if (ch + 1 < ch1 && c0 + EC < P.N) load_c(ch + 1, cnext);
         if (has_k) ptx::tmem_ld_wait();
         else {
 #pragma unroll
