@@ -203,12 +203,13 @@ __device__ __forceinline__ void tri_fix(const OpDesc &o, int lay, uint8_t *raw, 
 // word and ignores its low 13 mantissa bits, i.e. it consumes
 // hi = trunc_tf32(x) directly from the TMA-staged tile (pinned by
 // tests/test_parity_gpu.py::test_split_is_real).  Only lo = x - hi (exact in
-// fp32) is produced, rounded to nearest tf32 (ties away) with integer ops so
-// the transform stays on the ALU/FMA pipes and writes half the bytes.
+// fp32: the 13 bits below hi) is produced; the tensor core reads its top 11
+// bits the same way, so hi + tf32(lo) represents x to within 2^-21 |x|, far
+// below the K-linear accumulation error of the fp32 TMEM accumulator
+// (Q17, Q24).  Two ops per element (LOP + FADD).
 __device__ __forceinline__ float split_lo(float x) {
   const float hi = __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
-  const float l = x - hi;
-  return __uint_as_float((__float_as_uint(l) + 0x1000u) & 0xFFFFE000u);
+  return x - hi;
 }
 
 __device__ __forceinline__ void split_pass(const uint8_t *raw, uint8_t *lo, uint32_t bytes, int t) {
