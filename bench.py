@@ -198,6 +198,24 @@ def run_ours(args):
         Cs = colmaj(dCs)
         beta_r = BETA if rank == 0 else 0.0
 
+    def syrk_k():
+        if rank == 0:
+            dCs.copy_(dC0)
+        else:
+            dCs.zero_()
+        b3.ssyrk("L", "N", ALPHA, Bm, beta_r, Cs)
+        d3.syrk_k_split(dCs)
+
+    def syr2k_k():
+        if rank != 0:
+            dCs.zero_()
+        b3.ssyr2k("L", "N", ALPHA, Bm, C0, 1.0 if rank == 0 else 0.0, Cs)
+        d3.syrk_k_split(dCs)
+
+    def chain_syrk_k():
+        syrk_k()
+        syr2k_k()
+
     def chain(record):
         def timed(name, fn):
             if record:
@@ -212,19 +230,6 @@ def run_ours(args):
             timed("ssyrk", lambda: b3.ssyrk("L", "N", ALPHA, A, BETA, C))
             timed("ssyr2k", lambda: b3.ssyr2k("L", "N", ALPHA, A, Bm, BETA, C))
         else:
-            def syrk_k():
-                if rank == 0:
-                    dCs.copy_(dC0)
-                else:
-                    dCs.zero_()
-                b3.ssyrk("L", "N", ALPHA, Bm, beta_r, Cs)
-                d3.syrk_k_split(dCs)
-
-            def syr2k_k():
-                if rank != 0:
-                    dCs.zero_()
-                b3.ssyr2k("L", "N", ALPHA, Bm, C0, 1.0 if rank == 0 else 0.0, Cs)
-                d3.syrk_k_split(dCs)
             timed("ssyrk", syrk_k)
             timed("ssyr2k", syr2k_k)
         timed("strmm", lambda: b3.strmm("L", "L", "N", "N", ALPHA, T, X))
@@ -237,16 +242,51 @@ def run_ours(args):
             dist.broadcast(dA, 0); dist.broadcast(dT, 0)      # the one exchange step
         chain(record)
 
+    copy_stream = torch.cuda.Stream(device=dev)
+    E2E_CHUNKS = 4
+
     def step_e2e():
-        # host -> device inputs, the chain, device -> host results (pinned)
+        """Host (pinned) -> device inputs, the chain, device -> host results,
+        with the transfers overlapped with compute through the public API:
+        B/C arrive in column chunks on a copy stream and the sgemm runs on
+        each column slab as it lands; T uploads behind sgemm/ssymm; C
+        downloads behind strmm/strsm."""
         if rank == 0:
-            dA.copy_(hA, non_blocking=True); dT.copy_(hT, non_blocking=True)
-        dB.copy_(hB, non_blocking=True); dC.copy_(hC, non_blocking=True)
+            dA.copy_(hA, non_blocking=True)
         if world > 1:
-            dist.broadcast(dA, 0); dist.broadcast(dT, 0)
+            dist.broadcast(dA, 0)
+        copy_stream.wait_stream(stream)
+        evs = []
+        bounds = [(i * cols // E2E_CHUNKS, (i + 1) * cols // E2E_CHUNKS) for i in range(E2E_CHUNKS)]
+        with torch.cuda.stream(copy_stream):
+            for c0, c1 in bounds:                       # (cols, n) row-major rows = matrix columns
+                dB[c0:c1].copy_(hB[c0:c1], non_blocking=True)
+                dC[c0:c1].copy_(hC[c0:c1], non_blocking=True)
+                e = torch.cuda.Event(); e.record(copy_stream); evs.append(e)
+            if rank == 0:
+                dT.copy_(hT, non_blocking=True)
+            eT = torch.cuda.Event(); eT.record(copy_stream)
+        for (c0, c1), e in zip(bounds, evs):
+            stream.wait_event(e)
+            b3.sgemm("N", "N", ALPHA, A, Bm[:, c0:c1], BETA, C[:, c0:c1])
+        b3.ssymm("L", "L", ALPHA, A, Bm, BETA, C)
+        if world == 1:
+            b3.ssyrk("L", "N", ALPHA, A, BETA, C)
+            b3.ssyr2k("L", "N", ALPHA, A, Bm, BETA, C)
+        else:
+            chain_syrk_k()
+        eC = torch.cuda.Event(); eC.record(stream)
+        with torch.cuda.stream(copy_stream):
+            copy_stream.wait_event(eC)
+            hC_out.copy_(dC, non_blocking=True)
+        stream.wait_event(eT)
+        if world > 1:
+            dist.broadcast(dT, 0)
         dX.copy_(dB)
-        chain(False)
-        hC_out.copy_(dC, non_blocking=True); hX_out.copy_(dX, non_blocking=True)
+        b3.strmm("L", "L", "N", "N", ALPHA, T, X)
+        b3.strsm("L", "L", "N", "N", ALPHA, T, X)
+        hX_out.copy_(dX, non_blocking=True)
+        stream.wait_stream(copy_stream)
 
     def timed_loop(fn, steps, record=False):
         if world > 1:
