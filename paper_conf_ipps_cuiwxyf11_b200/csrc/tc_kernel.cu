@@ -48,9 +48,20 @@ namespace {
 constexpr int BK = 32;
 constexpr int HA = 128;                    // A rows staged per CTA
 constexpr int BN = 256;                    // tile columns (UMMA N)
-constexpr int WARP_TMA = 0, WARP_MMA = 1, WARP_TR0 = 2, NUM_TR_WARPS = 8;
+// Roles are aligned to warpgroups so setmaxnreg can move registers to the
+// epilogue, which holds a 128-column fp32 running sum per thread.
+constexpr int WARP_TMA = 0, WARP_MMA = 1, WARP_TR0 = 4, NUM_TR_WARPS = 8;
 constexpr int WARP_EPI0 = WARP_TR0 + NUM_TR_WARPS, NUM_EPI_WARPS = 8;
-constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;
+constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;       // 640
+// setmaxnreg moves registers inside the CTA's own pool (the launch allocation,
+// 96 x 640 = 61440), so 256*EPI_REGS + 384*OTHER_REGS must not exceed it.
+constexpr int EPI_REGS = 144, OTHER_REGS = 64;   // 36864 + 24576 = 61440
+// Chunked accumulation: the tensor core's fp32 accumulator truncates on every
+// UMMA add (Q24), so a TMEM partial only ever sums KC k-blocks
+// (K = 256) before the epilogue folds it into a register running sum with
+// round-to-nearest adds; the two TMEM buffers ping-pong per chunk.
+constexpr int KC = 16;
+constexpr int EC = 16;                            // epilogue column group
 constexpr int TR_THREADS = NUM_TR_WARPS * 32;
 constexpr int EPI_THREADS = NUM_EPI_WARPS * 32;
 constexpr int TMEM_COLS = 512;             // 2 accumulators x BN columns
@@ -81,8 +92,8 @@ struct Geo {
     uint64_t empty[RS];      // MMA -> TMA: raw slot free (tcgen05.commit, multicast)
     uint64_t ready[LS];      // transform -> MMA (one arrival per CTA of the pair, leader)
     uint64_t lo_empty[LS];   // MMA -> transform: lo slot free (tcgen05.commit, multicast)
-    uint64_t tfull[2];       // MMA -> epilogue (multicast to the pair)
-    uint64_t tempty[2];      // epilogue -> MMA (one arrival per CTA of the pair, leader)
+    uint64_t tfull[2];       // MMA -> epilogue: TMEM partial ready (multicast to the pair)
+    uint64_t tempty[2];      // epilogue -> MMA: partial drained (one arrival per CTA, leader)
     uint32_t tmem_base;
   };
   static constexpr size_t SMEM = sizeof(RawBuf) * RS + sizeof(LoBuf) * LS + sizeof(Barriers) + 1024;
@@ -293,7 +304,14 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
   const int64_t per = P.per > 0 ? P.per : 1;
   const int64_t ntiles = tiles_per * (P.nbatch > 0 ? P.nbatch : 1);
 
-  if (warp == WARP_TMA) {
+  // register rebalancing per warpgroup role (setmaxnreg dominates each role's code)
+#define BLAS3_DEC_REGS() asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(OTHER_REGS))
+#define BLAS3_INC_REGS() asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(EPI_REGS))
+  if (warp < WARP_TR0) {
+    // first warpgroup: TMA producer (warp 0), MMA issuer (warp 1), 2 spares.
+    // setmaxnreg is warpgroup-collective: one instruction, one PC.
+    BLAS3_DEC_REGS();
+   if (warp == WARP_TMA) {
     // ============================ TMA producer (each CTA stages its own halves)
     if (lane == 0) {
       for (int i = 0; i < MAX_MAPS; ++i) ptx::tma_prefetch(&prm.maps[i]);
@@ -325,26 +343,47 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
       for (int i = 0; i < RS; ++i, ++it)
         ptx::mbar_wait(&bars->empty[it % RS], ((it / RS) & 1) ^ 1);
     }
-  } else if (warp == WARP_MMA) {
+   } else if (warp == WARP_MMA) {
     // ============================ MMA issuer (leader CTA of the pair only)
     if (rank == 0) {
-      uint32_t it = 0, tcount = 0;
-      for (int64_t tb = cid; tb < ntiles; tb += ncl, ++tcount) {
+      uint32_t it = 0, cc = 0;                  // k-block and TMEM-chunk counters
+      for (int64_t tb = cid; tb < ntiles; tb += ncl) {
         const int64_t t = tb % tiles_per;
         int64_t mi, nj;
         Tiles<TM, BN>::coords(P, t, mi, nj);
         const int64_t m0 = mi * TM, n0 = nj * BN;
-        const uint32_t acc = tcount & 1, aph = (tcount >> 1) & 1;
-        if (CG == 2) ptx::mbar_wait_cluster(&bars->tempty[acc], aph ^ 1);
-        else ptx::mbar_wait(&bars->tempty[acc], aph ^ 1);
-        ptx::tc_fence_after();
-        const uint32_t d_tmem = tmem + acc * BN;
-        uint32_t accumulate = 0;
+        const int64_t nkb = tile_kblocks<CG>(P, m0, n0);
+        int64_t done = 0;
+        uint32_t accumulate = 0, buf = 0;
+        auto open_chunk = [&]() {
+          buf = cc & 1;
+          const uint32_t aph = (cc >> 1) & 1;
+          if (CG == 2) ptx::mbar_wait_cluster(&bars->tempty[buf], aph ^ 1);
+          else ptx::mbar_wait(&bars->tempty[buf], aph ^ 1);
+          ptx::tc_fence_after();
+          accumulate = 0;
+        };
+        auto close_chunk = [&](bool issued) {
+          if (lane == 0) {
+            if (issued) {
+              if constexpr (CG == 1) ptx::mma_commit(&bars->tfull[buf]);
+              else ptx::mma_commit_pair(&bars->tfull[buf], 0x3);
+            } else {                                 // empty k-range: partial = 0
+              ptx::mbar_arrive(&bars->tfull[buf]);
+              if (CG == 2) ptx::mbar_arrive_cluster(&bars->tfull[buf], 1);
+            }
+          }
+          __syncwarp();
+          ++cc;
+        };
+        if (nkb == 0) { open_chunk(); close_chunk(false); continue; }
         for (int s = 0; s < P.nseg; ++s) {
           const Segment &sg = P.seg[s];
           int64_t kb0, kb1;
           seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
+            if (done % KC == 0) open_chunk();
+            const uint32_t d_tmem = tmem + buf * BN;
             const int rs = it % RS, ls = it % LS;
             const uint32_t lph = (it / LS) & 1;
             const StageInfo si = stage_info<CG>(P, sg, m0, n0, kb * BK);
@@ -381,22 +420,16 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
             }
             accumulate = 1;
             __syncwarp();
+            ++done;
+            if (done % KC == 0 || done == nkb) close_chunk(true);
           }
         }
-        if (lane == 0) {
-          if (accumulate) {
-            if constexpr (CG == 1) ptx::mma_commit(&bars->tfull[acc]);
-            else ptx::mma_commit_pair(&bars->tfull[acc], 0x3);
-          } else {                                   // empty k-range: accumulator = 0
-            ptx::mbar_arrive(&bars->tfull[acc]);
-            if (CG == 2) ptx::mbar_arrive_cluster(&bars->tfull[acc], 1);
-          }
-        }
-        __syncwarp();
       }
     }
+   }
   } else if (warp < WARP_EPI0) {
     // ============================ transform warps (own halves; arrive at the leader)
+    BLAS3_DEC_REGS();
     const int tt = threadIdx.x - WARP_TR0 * 32;
     uint32_t it = 0;
     for (int64_t tb = cid; tb < ntiles; tb += ncl) {
@@ -433,63 +466,68 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
       }
     }
   } else {
-    // ============================ epilogue warps (own 128 rows, all BN columns)
+    // ============================ epilogue warps (own 128 rows, 128 of the BN columns)
+    BLAS3_INC_REGS();
+    // Each thread owns one row r and 128 columns: S[] is the fp32 running sum
+    // of the KC-chunk partials (round-to-nearest adds), then
+    // D = alpha*S + beta*C is stored with coalesced 128-B warp accesses.
     const int q = warp & 3;                     // TMEM lane quarter of this warp
     const int half = (warp - WARP_EPI0) >> 2;   // which 128 of the 256 columns
-    uint32_t tcount = 0;
-    for (int64_t tb = cid; tb < ntiles; tb += ncl, ++tcount) {
+    constexpr int NG = BN / 2 / EC;             // column groups per thread (8)
+    uint32_t cc = 0;
+    for (int64_t tb = cid; tb < ntiles; tb += ncl) {
       const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
       const int64_t coff = (P.nbatch > 1) ? batch_off(P.bs_c, b, per) : 0;
       int64_t mi, nj;
       Tiles<TM, BN>::coords(P, t, mi, nj);
       const int64_t m0 = mi * TM, n0 = nj * BN;
-      const bool has_k = tile_kblocks<CG>(P, m0, n0) > 0;
-      const uint32_t acc = tcount & 1, aph = (tcount >> 1) & 1;
-      ptx::mbar_wait(&bars->tfull[acc], aph);
-      ptx::tc_fence_after();
+      const int64_t nkb = tile_kblocks<CG>(P, m0, n0);
+      const int64_t nchunks = nkb > 0 ? cdiv(nkb, KC) : 1;
+      float S[NG * EC];
+#pragma unroll
+      for (int i = 0; i < NG * EC; ++i) S[i] = 0.f;
+      for (int64_t c = 0; c < nchunks; ++c, ++cc) {
+        const uint32_t buf = cc & 1, ph = (cc >> 1) & 1;
+        ptx::mbar_wait(&bars->tfull[buf], ph);
+        ptx::tc_fence_after();
+        if (nkb > 0) {
+#pragma unroll
+          for (int g = 0; g < NG; ++g) {
+            uint32_t v[EC];
+            ptx::tmem_ld_32x32b_x16(tmem + buf * BN + half * (BN / 2) + g * EC +
+                                        ((uint32_t)(q * 32) << 16), v);
+            ptx::tmem_ld_wait();
+#pragma unroll
+            for (int j = 0; j < EC; ++j) S[g * EC + j] += __uint_as_float(v[j]);
+          }
+        }
+        ptx::tc_fence_before();
+        arrive_leader<CG>(&bars->tempty[buf], rank, 3, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
+      }
       const int64_t r = m0 + HA * rank + q * 32 + lane;
       const bool row_ok = r < P.M;
       const float *cin = P.Cin + coff + r;
       float *cout = P.Cout + coff + r;
-      constexpr int EC = 16;                    // epilogue chunk: 16 columns
-      const int ch0 = half * (BN / EC / 2), ch1 = (half + 1) * (BN / EC / 2);
-      // C(r, c0..c0+15) of the NEXT chunk is loaded while the current chunk is
-      // stored (loads are issued before the stores in program order because
-      // Cin may alias Cout); each access is a coalesced 128-B warp access.
-      auto load_c = [&](int ch, float (&cv)[EC]) {
-        const int64_t c0 = n0 + ch * EC;
-#pragma unroll
-        for (int j = 0; j < EC; ++j) {
-          const int64_t c = c0 + j;
-          const bool ok = row_ok && c < P.N && !(P.c_tri == 1 && r < c) && !(P.c_tri == 2 && r > c);
-          cv[j] = (ok && P.beta != 0.f) ? cin[c * P.ldcin] : 0.f;
-        }
+      const int64_t cbase = n0 + half * (BN / 2);
+      // per 8-column group: all C loads first, then the stores (Cin may alias
+      // Cout); each is a coalesced 128-B warp access.
+      auto ok_at = [&](int64_t c) {
+        return row_ok && c < P.N && !(P.c_tri == 1 && r < c) && !(P.c_tri == 2 && r > c);
       };
-      float cnext[EC];
-      if (n0 + ch0 * EC < P.N) load_c(ch0, cnext);
-      for (int ch = ch0; ch < ch1; ++ch) {
-        const int64_t c0 = n0 + ch * EC;
-        if (c0 >= P.N) break;
-        float cv[EC];
+      constexpr int SG = 8;
 #pragma unroll
-        for (int j = 0; j < EC; ++j) cv[j] = cnext[j];
-        uint32_t v[EC];
-        if (has_k) ptx::tmem_ld_32x32b_x16(tmem + acc * BN + ch * EC + ((uint32_t)(q * 32) << 16), v);
-        if (ch + 1 < ch1 && c0 + EC < P.N) load_c(ch + 1, cnext);
-        if (has_k) ptx::tmem_ld_wait();
-        else {
+      for (int g = 0; g < NG * EC / SG; ++g) {
+        const int64_t c0 = cbase + g * SG;
+        float cv[SG];
 #pragma unroll
-          for (int j = 0; j < EC; ++j) v[j] = 0u;
-        }
+        for (int j = 0; j < SG; ++j)
+          cv[j] = (P.beta != 0.f && ok_at(c0 + j)) ? cin[(c0 + j) * P.ldcin] : 0.f;
 #pragma unroll
-        for (int j = 0; j < EC; ++j) {
+        for (int j = 0; j < SG; ++j) {
           const int64_t c = c0 + j;
-          const bool ok = row_ok && c < P.N && !(P.c_tri == 1 && r < c) && !(P.c_tri == 2 && r > c);
-          if (ok && !(P.dbg & 4)) cout[c * P.ldcout] = fmaf(P.beta, cv[j], P.alpha * __uint_as_float(v[j]));
+          if (ok_at(c) && !(P.dbg & 4)) cout[c * P.ldcout] = fmaf(P.beta, cv[j], P.alpha * S[g * SG + j]);
         }
       }
-      ptx::tc_fence_before();
-      arrive_leader<CG>(&bars->tempty[acc], rank, 3, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
     }
   }
 
