@@ -62,6 +62,10 @@ constexpr int EPI_REGS = 144, OTHER_REGS = 64;   // 36864 + 24576 = 61440
 // round-to-nearest adds; the two TMEM buffers ping-pong per chunk.
 constexpr int KC = 16;
 constexpr int EC = 16;                            // epilogue column group
+// Tile queue: the producer warp claims tiles (atomic counter, or the static
+// round-robin sequence for CTA pairs) and hands them to the MMA, transform
+// and epilogue roles through a TQ-deep shared-memory queue.
+constexpr int TQ = 4;
 constexpr int TR_THREADS = NUM_TR_WARPS * 32;
 constexpr int EPI_THREADS = NUM_EPI_WARPS * 32;
 constexpr int TMEM_COLS = 512;             // 2 accumulators x BN columns
@@ -92,6 +96,9 @@ struct Geo {
     uint64_t empty[RS];      // MMA -> TMA: raw slot free (tcgen05.commit, multicast)
     uint64_t ready[LS];      // transform -> MMA (one arrival per CTA of the pair, leader)
     uint64_t lo_empty[LS];   // MMA -> transform: lo slot free (tcgen05.commit, multicast)
+    uint64_t tq_full[TQ];    // producer -> roles: tile index published
+    uint64_t tq_empty[TQ];   // roles -> producer: slot read (3 arrivals: MMA, transform, epilogue)
+    int64_t tq[TQ];
     uint64_t tfull[2];       // MMA -> epilogue: TMEM partial ready (multicast to the pair)
     uint64_t tempty[2];      // epilogue -> MMA: partial drained (one arrival per CTA, leader)
     uint32_t tmem_base;
@@ -102,7 +109,9 @@ struct Geo {
 struct TcParams {
   CUtensorMap maps[MAX_MAPS];
   Problem P;
+  uint32_t *tile_ctr;      // dynamic tile scheduler counter (zeroed per launch), or null
 };
+
 
 // byte offset of element (r, k) inside a staged operand tile
 __device__ __forceinline__ uint32_t off_k(int r, int k) {       // K-major, 128 B per row r
@@ -287,6 +296,10 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
       ptx::mbar_init(&bars->ready[s], CG);
       ptx::mbar_init(&bars->lo_empty[s], 1);
     }
+    for (int q = 0; q < TQ; ++q) {
+      ptx::mbar_init(&bars->tq_full[q], 1);
+      ptx::mbar_init(&bars->tq_empty[q], 3);
+    }
     for (int a = 0; a < 2; ++a) {
       ptx::mbar_init(&bars->tfull[a], 1);
       ptx::mbar_init(&bars->tempty[a], CG);
@@ -303,6 +316,17 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
   const int64_t tiles_per = Tiles<TM, BN>::count(P);
   const int64_t per = P.per > 0 ? P.per : 1;
   const int64_t ntiles = tiles_per * (P.nbatch > 0 ? P.nbatch : 1);
+  // consumer side of the tile queue: returns the next tile (or -1 = done);
+  // every thread of the role reads the slot, then one thread releases it.
+  auto next_tile = [&](uint32_t &qi, uint32_t bar_id, uint32_t nthreads, bool first) -> int64_t {
+    const int slot = qi % TQ;
+    ptx::mbar_wait(&bars->tq_full[slot], (qi / TQ) & 1);
+    const int64_t tb = *reinterpret_cast<volatile int64_t *>(&bars->tq[slot]);
+    if (nthreads > 32) ptx::named_bar_sync(bar_id, nthreads); else __syncwarp();
+    if (first) ptx::mbar_arrive(&bars->tq_empty[slot]);
+    ++qi;
+    return tb;
+  };
 
   // register rebalancing per warpgroup role (setmaxnreg dominates each role's code)
 #define BLAS3_DEC_REGS() asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(OTHER_REGS))
@@ -316,7 +340,14 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     if (lane == 0) {
       for (int i = 0; i < MAX_MAPS; ++i) ptx::tma_prefetch(&prm.maps[i]);
       uint32_t it = 0;
-      for (int64_t tb = cid; tb < ntiles; tb += ncl) {
+      for (uint32_t qi = 0;; ++qi) {
+        int64_t tb = prm.tile_ctr ? (int64_t)atomicAdd(prm.tile_ctr, 1u) : cid + (int64_t)qi * ncl;
+        if (tb >= ntiles) tb = -1;
+        const int slot = qi % TQ;
+        ptx::mbar_wait(&bars->tq_empty[slot], ((qi / TQ) & 1) ^ 1);
+        *reinterpret_cast<volatile int64_t *>(&bars->tq[slot]) = tb;
+        ptx::mbar_arrive(&bars->tq_full[slot]);
+        if (tb < 0) break;
         const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
         const int32_t bj = (int32_t)(b % per), bg = (int32_t)(b / per);
         int64_t mi, nj;
@@ -345,9 +376,14 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     }
    } else if (warp == WARP_MMA) {
     // ============================ MMA issuer (leader CTA of the pair only)
-    if (rank == 0) {
-      uint32_t it = 0, cc = 0;                  // k-block and TMEM-chunk counters
-      for (int64_t tb = cid; tb < ntiles; tb += ncl) {
+    if (rank != 0) {                          // peer CTA: only drain the tile queue
+      uint32_t qi = 0;
+      while (next_tile(qi, 0, 32, lane == 0) >= 0) {}
+    } else {
+      uint32_t it = 0, cc = 0, qi = 0;          // k-block, TMEM-chunk, tile-queue counters
+      for (;;) {
+        const int64_t tb = next_tile(qi, 0, 32, lane == 0);
+        if (tb < 0) break;
         const int64_t t = tb % tiles_per;
         int64_t mi, nj;
         Tiles<TM, BN>::coords(P, t, mi, nj);
@@ -431,8 +467,10 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     // ============================ transform warps (own halves; arrive at the leader)
     BLAS3_DEC_REGS();
     const int tt = threadIdx.x - WARP_TR0 * 32;
-    uint32_t it = 0;
-    for (int64_t tb = cid; tb < ntiles; tb += ncl) {
+    uint32_t it = 0, qi = 0;
+    for (;;) {
+      const int64_t tb = next_tile(qi, 4, TR_THREADS, tt == 0);
+      if (tb < 0) break;
       const int64_t t = tb % tiles_per;
       int64_t mi, nj;
       Tiles<TM, BN>::coords(P, t, mi, nj);
@@ -474,8 +512,10 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     const int q = warp & 3;                     // TMEM lane quarter of this warp
     const int half = (warp - WARP_EPI0) >> 2;   // which 128 of the 256 columns
     constexpr int NG = BN / 2 / EC;             // column groups per thread (8)
-    uint32_t cc = 0;
-    for (int64_t tb = cid; tb < ntiles; tb += ncl) {
+    uint32_t cc = 0, qi = 0;
+    for (;;) {
+      const int64_t tb = next_tile(qi, 5, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
+      if (tb < 0) break;
       const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
       const int64_t coff = (P.nbatch > 1) ? batch_off(P.bs_c, b, per) : 0;
       int64_t mi, nj;
@@ -664,6 +704,24 @@ static int launch_cg(TcParams &prm, cudaStream_t stream, int num_sms) {
   return (e == cudaSuccess && cudaGetLastError() == cudaSuccess) ? 0 : -1;
 }
 
+// Dynamic tile scheduling counters: a ring of per-launch slots per device,
+// each zeroed by a stream-ordered memset right before its launch.
+static uint32_t *tile_counter(cudaStream_t stream) {
+  constexpr int SLOTS = 256;
+  static uint32_t *ring[64] = {};
+  static uint32_t next[64] = {};
+  int d = 0;
+  if (cudaGetDevice(&d) != cudaSuccess || d < 0 || d >= 64) return nullptr;
+  if (!ring[d] && cudaMalloc(&ring[d], SLOTS * 32 * sizeof(uint32_t)) != cudaSuccess) {
+    cudaGetLastError();
+    ring[d] = nullptr;
+    return nullptr;
+  }
+  uint32_t *c = ring[d] + (next[d]++ % SLOTS) * 32;     // 128-B apart
+  if (cudaMemsetAsync(c, 0, sizeof(uint32_t), stream) != cudaSuccess) return nullptr;
+  return c;
+}
+
 int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
   static TcParams prm;                    // host staging (the launch copies it)
   static std::mutex mu;
@@ -675,8 +733,14 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
     if (dbg < 0) { const char *e = getenv("BLAS3_DEBUG_TC"); dbg = e ? atoi(e) : 0; }
     prm.P.dbg = dbg;
   }
-  return choose_cg(prm.P, num_sms) == 2 ? launch_cg<2>(prm, stream, num_sms)
-                                        : launch_cg<1>(prm, stream, num_sms);
+  const int cg = choose_cg(prm.P, num_sms);
+  // CTA pairs must walk the same tile sequence: static round-robin for CG=2
+  if (cg == 1) {
+    static int dyn = -1;
+    if (dyn < 0) { const char *e = getenv("BLAS3_TC_STATIC"); dyn = (e && e[0] == '1') ? 0 : 1; }
+    if (dyn && !(prm.tile_ctr = tile_counter(stream))) return -1;
+  }
+  return cg == 2 ? launch_cg<2>(prm, stream, num_sms) : launch_cg<1>(prm, stream, num_sms);
 }
 
 }  // namespace blas3
