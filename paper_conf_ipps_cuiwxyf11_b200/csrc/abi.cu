@@ -435,7 +435,11 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
     lo = pa * NBO;
     hi = imin(nt, pb * NBO);
   };
-  std::function<int(int64_t, int64_t, bool)> rec = [&](int64_t q0, int64_t q1, bool scaled) -> int {
+  // in_w: the rows (L) / columns (R) of a single-panel range were left in W
+  // (already updated) by the preceding update, so the solve reads W and writes
+  // B directly -- no copy-back.
+  std::function<int(int64_t, int64_t, bool, bool)> rec = [&](int64_t q0, int64_t q1, bool scaled,
+                                                             bool in_w) -> int {
     int rc2;
     if (q1 - q0 == 1) {
       const int64_t p = forward ? q0 : npanel - 1 - q0;
@@ -444,45 +448,56 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
       const float *Dp = D.p + p * NBO * NBO;
       if (left) {
         // X_p = a1 * inv(op(A)_pp) * B_p: Xa(r,k) = Dop(r,k), Dop = lower_op ? D : D^T
-        Problem P = problem(pr, n, a1, 0.f, nullptr, 0, W.p, pr);
+        Problem P = in_w ? problem(pr, n, a1, 0.f, nullptr, 0, B + p0, ldb)
+                         : problem(pr, n, a1, 0.f, nullptr, 0, W.p, pr);
         P.seg[0].a = tri(Dp, NBO, true, !lower_op, false);
-        P.seg[0].b = dense(B + p0, ldb, true);
+        P.seg[0].b = in_w ? dense(W.p, pr, true) : dense(B + p0, ldb, true);
         P.seg[0].K = pr;
         P.rev_m = tri_kle(P.seg[0].a);
         if ((rc2 = run_problem(P, s, sms))) return rc2;
-        if (launch_copy(B + p0, ldb, W.p, pr, pr, n, s)) return BLAS3_ERR_CUDA;
+        if (!in_w && launch_copy(B + p0, ldb, W.p, pr, pr, n, s)) return BLAS3_ERR_CUDA;
       } else {
         // X_p = a1 * B_p * inv(op(A)_pp): Xb(c,k) = Dop(k,c) -> TRI swap = lower_op
-        Problem P = problem(m, pr, a1, 0.f, nullptr, 0, W.p, m);
-        P.seg[0].a = dense(B + p0 * ldb, ldb, false);
+        Problem P = in_w ? problem(m, pr, a1, 0.f, nullptr, 0, B + p0 * ldb, ldb)
+                         : problem(m, pr, a1, 0.f, nullptr, 0, W.p, m);
+        P.seg[0].a = in_w ? dense(W.p, m, false) : dense(B + p0 * ldb, ldb, false);
         P.seg[0].b = tri(Dp, NBO, true, lower_op, false);
         P.seg[0].K = pr;
         P.rev_n = tri_kle(P.seg[0].b);
         if ((rc2 = run_problem(P, s, sms))) return rc2;
-        if (launch_copy(B + p0 * ldb, ldb, W.p, m, m, pr, s)) return BLAS3_ERR_CUDA;
+        if (!in_w && launch_copy(B + p0 * ldb, ldb, W.p, m, m, pr, s)) return BLAS3_ERR_CUDA;
       }
       return 0;
     }
     const int64_t mid = q0 + (q1 - q0) / 2;
-    if ((rc2 = rec(q0, mid, scaled))) return rc2;
+    if ((rc2 = rec(q0, mid, scaled, in_w && false))) return rc2;
     int64_t k_lo, k_hi, o_lo, o_hi;
     elem(q0, mid, k_lo, k_hi);                       // solved part
     elem(mid, q1, o_lo, o_hi);                       // part to update
     const float a1 = scaled ? 1.f : alpha;
+    const bool to_w = (q1 - mid == 1);               // updated panel goes straight to W
     if (left) {   // B_o <- a1*B_o - op(A)(o, k) * X_k (X_k = B rows k)
       // Xa(r,kk) = op(A)(o_lo+r, k_lo+kk): !ta -> A(o_lo+r, k_lo+kk) rk; ta -> A(k_lo+kk, o_lo+r) kr
       const float *pa = ta ? A + k_lo + o_lo * lda : A + o_lo + k_lo * lda;
-      if ((rc2 = gemm_dense(o_hi - o_lo, n, k_hi - k_lo, -1.f, pa, lda, ta, B + k_lo, ldb, true, a1,
-                            B + o_lo, ldb, s, sms))) return rc2;
+      Problem P = to_w ? problem(o_hi - o_lo, n, -1.f, a1, B + o_lo, ldb, W.p, o_hi - o_lo)
+                       : problem(o_hi - o_lo, n, -1.f, a1, B + o_lo, ldb, B + o_lo, ldb);
+      P.seg[0].a = dense(pa, lda, ta);
+      P.seg[0].b = dense(B + k_lo, ldb, true);
+      P.seg[0].K = k_hi - k_lo;
+      if ((rc2 = run_problem(P, s, sms))) return rc2;
     } else {      // B(:,o) <- a1*B(:,o) - X_k * op(A)(k, o)
       // Xb(c,kk) = op(A)(k_lo+kk, o_lo+c): !ta -> A(k_lo+kk, o_lo+c) kr; ta -> A(o_lo+c, k_lo+kk) rk
       const float *pb = ta ? A + o_lo + k_lo * lda : A + k_lo + o_lo * lda;
-      if ((rc2 = gemm_dense(m, o_hi - o_lo, k_hi - k_lo, -1.f, B + k_lo * ldb, ldb, false, pb, lda,
-                            !ta, a1, B + o_lo * ldb, ldb, s, sms))) return rc2;
+      Problem P = to_w ? problem(m, o_hi - o_lo, -1.f, a1, B + o_lo * ldb, ldb, W.p, m)
+                       : problem(m, o_hi - o_lo, -1.f, a1, B + o_lo * ldb, ldb, B + o_lo * ldb, ldb);
+      P.seg[0].a = dense(B + k_lo * ldb, ldb, false);
+      P.seg[0].b = dense(pb, lda, !ta);
+      P.seg[0].K = k_hi - k_lo;
+      if ((rc2 = run_problem(P, s, sms))) return rc2;
     }
-    return rec(mid, q1, true);
+    return rec(mid, q1, true, to_w);
   };
-  if ((rc = rec(0, npanel, false))) return rc;
+  if ((rc = rec(0, npanel, false, false))) return rc;
   return finish(0);
 }
 
