@@ -1,0 +1,28 @@
+"""The opt-in kernel variants selected by environment variables at library
+load (they are cached once per process, hence subprocesses): the CTA-pair
+tcgen05 kernel (BLAS3_TC_CTA=2, cta_group::2) and the static tile schedule
+(BLAS3_TC_STATIC=1).  Each child process runs a representative subset of the
+parity suite (every routine family, both transposes/sides) on that variant."""
+import os
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.mark.parametrize("env", [{"BLAS3_TC_CTA": "2"}, {"BLAS3_TC_STATIC": "1"}],
+                         ids=["cta_pair", "static_schedule"])
+def test_variant_subset(env):
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    sel = "3xtf32 and (sgemm or ssymm or syrk or strmm or strsm or split_is_real)"
+    cmd = [sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k", sel,
+           os.path.join(ROOT, "tests", "test_parity_gpu.py")]
+    r = subprocess.run(cmd, env={**os.environ, **env}, cwd=ROOT, capture_output=True, text=True,
+                       timeout=900)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
+    assert " passed" in r.stdout
