@@ -652,18 +652,20 @@ bool tc_eligible(const Problem &P) {
   return true;
 }
 
-// CTA-group choice.  The pair kernel (CG=2, 256x256 tiles, cta_group::2) is
-// parity-green but measured slower than CG=1 on B200 so far (DESIGN.md §7:
-// 159-197 vs 200 TF/s at 8192^3), so CG=1 is the default; BLAS3_TC_CTA=2
-// selects the pair kernel (tests run both).
+// CTA-group choice.  The pair kernel (CG=2: 256x256 tiles, tcgen05
+// cta_group::2, each CTA staging half of B) needs half the per-SM operand
+// traffic and a 4-deep raw ring; it is used whenever it still gives every CTA
+// pair at least one tile, else the single-CTA kernel (more, smaller tiles,
+// dynamic scheduling).  BLAS3_TC_CTA=1|2 forces one (tests).
 static int choose_cg(const Problem &P, int num_sms) {
   static int forced = -1;
   if (forced < 0) {
     const char *e = getenv("BLAS3_TC_CTA");
-    forced = (e && e[0] == '2') ? 2 : 1;
+    forced = (e && e[0] == '1') ? 1 : (e && e[0] == '2') ? 2 : 0;
   }
-  (void)P; (void)num_sms;
-  return forced;
+  if (forced) return forced;
+  const int64_t nb = P.nbatch > 1 ? P.nbatch : 1;
+  return Tiles<Geo<2>::TM, BN>::count(P) * nb >= num_sms / 2 ? 2 : 1;
 }
 
 template <int CG>

@@ -1,7 +1,8 @@
 """The opt-in kernel variants selected by environment variables at library
 load (they are cached once per process, hence subprocesses): the CTA-pair
 tcgen05 kernel (BLAS3_TC_CTA=2, cta_group::2) and the static tile schedule
-(BLAS3_TC_STATIC=1).  Each child process runs a representative subset of the
+(BLAS3_TC_STATIC=1), and the single-CTA kernel (BLAS3_TC_CTA=1; the default
+picks the pair kernel for large problems).  Each child process runs a representative subset of the
 parity suite (every routine family, both transposes/sides) on that variant."""
 import os
 import subprocess
@@ -13,8 +14,8 @@ pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-@pytest.mark.parametrize("env", [{"BLAS3_TC_CTA": "2"}, {"BLAS3_TC_STATIC": "1"}],
-                         ids=["cta_pair", "static_schedule"])
+@pytest.mark.parametrize("env", [{"BLAS3_TC_CTA": "1"}, {"BLAS3_TC_CTA": "2"}, {"BLAS3_TC_STATIC": "1"}],
+                         ids=["single_cta", "cta_pair", "static_schedule"])
 def test_variant_subset(env):
     import torch
     if not torch.cuda.is_available():
