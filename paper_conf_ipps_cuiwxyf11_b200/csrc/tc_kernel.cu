@@ -97,7 +97,7 @@ struct Geo {
     uint64_t ready[LS];      // transform -> MMA (one arrival per CTA of the pair, leader)
     uint64_t lo_empty[LS];   // MMA -> transform: lo slot free (tcgen05.commit, multicast)
     uint64_t tq_full[TQ];    // producer -> roles: tile index published
-    uint64_t tq_empty[TQ];   // roles -> producer: slot read (3 arrivals: MMA, transform, epilogue)
+    uint64_t tq_empty[TQ];   // roles -> leader producer: slot read (3 per CTA; +1 peer producer)
     int64_t tq[TQ];
     uint64_t tfull[2];       // MMA -> epilogue: TMEM partial ready (multicast to the pair)
     uint64_t tempty[2];      // epilogue -> MMA: partial drained (one arrival per CTA, leader)
@@ -193,8 +193,10 @@ __device__ __forceinline__ void load_operand(const TcParams &prm, const OpDesc &
 // global memory (rare blocks; keeps the raw ring free of a second view).
 __device__ __forceinline__ void sym_merge(const OpDesc &o, uint8_t *raw, int64_t r0, int64_t k0,
                                           int rows, int64_t R, int64_t K, int t) {
+  // k fastest across a warp: the stored elements S(k, r) of one r are
+  // contiguous in memory, so each warp load is one coalesced 128-B access
   for (int e = t; e < rows * BK; e += TR_THREADS) {
-    int r = e % rows, k = e / rows;
+    int k = e % BK, r = e / BK;
     int64_t gr = r0 + r, gk = k0 + k;
     bool mirrored = o.lower ? (gr < gk) : (gr > gk);
     if (mirrored && gr < R && gk < K)
@@ -298,7 +300,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     }
     for (int q = 0; q < TQ; ++q) {
       ptx::mbar_init(&bars->tq_full[q], 1);
-      ptx::mbar_init(&bars->tq_empty[q], 3);
+      ptx::mbar_init(&bars->tq_empty[q], CG == 1 ? 3 : 7);
     }
     for (int a = 0; a < 2; ++a) {
       ptx::mbar_init(&bars->tfull[a], 1);
@@ -318,12 +320,19 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
   const int64_t ntiles = tiles_per * (P.nbatch > 0 ? P.nbatch : 1);
   // consumer side of the tile queue: returns the next tile (or -1 = done);
   // every thread of the role reads the slot, then one thread releases it.
+  // (for a CTA pair the leader's producer fills both CTAs' queues, and every
+  // role of both CTAs releases the slot at the leader)
   auto next_tile = [&](uint32_t &qi, uint32_t bar_id, uint32_t nthreads, bool first) -> int64_t {
     const int slot = qi % TQ;
-    ptx::mbar_wait(&bars->tq_full[slot], (qi / TQ) & 1);
+    if (CG == 2) ptx::mbar_wait_cluster(&bars->tq_full[slot], (qi / TQ) & 1);
+    else ptx::mbar_wait(&bars->tq_full[slot], (qi / TQ) & 1);
     const int64_t tb = *reinterpret_cast<volatile int64_t *>(&bars->tq[slot]);
-    if (nthreads > 32) ptx::named_bar_sync(bar_id, nthreads); else __syncwarp();
-    if (first) ptx::mbar_arrive(&bars->tq_empty[slot]);
+    if (nthreads > 32) ptx::named_bar_sync(bar_id, nthreads);
+    else if (nthreads == 32) __syncwarp();
+    if (first) {
+      if (CG == 1 || rank == 0) ptx::mbar_arrive(&bars->tq_empty[slot]);
+      else ptx::mbar_arrive_cluster(&bars->tq_empty[slot], 0);
+    }
     ++qi;
     return tb;
   };
@@ -340,13 +349,22 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     if (lane == 0) {
       for (int i = 0; i < MAX_MAPS; ++i) ptx::tma_prefetch(&prm.maps[i]);
       uint32_t it = 0;
-      for (uint32_t qi = 0;; ++qi) {
-        int64_t tb = prm.tile_ctr ? (int64_t)atomicAdd(prm.tile_ctr, 1u) : cid + (int64_t)qi * ncl;
-        if (tb >= ntiles) tb = -1;
-        const int slot = qi % TQ;
-        ptx::mbar_wait(&bars->tq_empty[slot], ((qi / TQ) & 1) ^ 1);
-        *reinterpret_cast<volatile int64_t *>(&bars->tq[slot]) = tb;
-        ptx::mbar_arrive(&bars->tq_full[slot]);
+      for (uint32_t qi = 0;;) {
+        int64_t tb;
+        if (CG == 1 || rank == 0) {
+          // claim a tile (dynamic) or take the static round-robin one
+          tb = prm.tile_ctr ? (int64_t)atomicAdd(prm.tile_ctr, 1u) : cid + (int64_t)qi * ncl;
+          if (tb >= ntiles) tb = -1;
+          const int slot = qi % TQ;
+          if (CG == 2) ptx::mbar_wait_cluster(&bars->tq_empty[slot], ((qi / TQ) & 1) ^ 1);
+          else ptx::mbar_wait(&bars->tq_empty[slot], ((qi / TQ) & 1) ^ 1);
+          *reinterpret_cast<volatile int64_t *>(&bars->tq[slot]) = tb;
+          if (CG == 2) ptx::st_remote_and_arrive(&bars->tq[slot], tb, &bars->tq_full[slot], 1);
+          ptx::mbar_arrive(&bars->tq_full[slot]);
+          ++qi;
+        } else {
+          tb = next_tile(qi, 0, 1, true);             // the pair's peer follows the leader
+        }
         if (tb < 0) break;
         const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
         const int32_t bj = (int32_t)(b % per), bg = (int32_t)(b / per);
@@ -736,12 +754,9 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
     prm.P.dbg = dbg;
   }
   const int cg = choose_cg(prm.P, num_sms);
-  // CTA pairs must walk the same tile sequence: static round-robin for CG=2
-  if (cg == 1) {
-    static int dyn = -1;
-    if (dyn < 0) { const char *e = getenv("BLAS3_TC_STATIC"); dyn = (e && e[0] == '1') ? 0 : 1; }
-    if (dyn && !(prm.tile_ctr = tile_counter(stream))) return -1;
-  }
+  static int dyn = -1;
+  if (dyn < 0) { const char *e = getenv("BLAS3_TC_STATIC"); dyn = (e && e[0] == '1') ? 0 : 1; }
+  if (dyn && !(prm.tile_ctr = tile_counter(stream))) return -1;
   return cg == 2 ? launch_cg<2>(prm, stream, num_sms) : launch_cg<1>(prm, stream, num_sms);
 }
 
