@@ -348,7 +348,7 @@ int blas3_strmm(char side, char uplo, char transa, char diag, int64_t m, int64_t
 //      a single panel is X_p = alpha_p * inv(op(A)_pp) * B_p (TRI operand).
 //      alpha is folded into the first operation that touches each row.
 // Every flop of steps 2-3 runs in the structured GEMM kernels.
-static const int64_t NBO = 1024;   // panel width (multiple of the 128 diagonal block)
+static const int64_t NBO = 2048;   // panel width (multiple of the 128 diagonal block)
 
 static int trsm_panel_inverses(const float *A, int64_t lda, int64_t nt, bool lower, bool unit,
                                float *D, float *Tw, cudaStream_t s, int sms) {
