@@ -4,8 +4,14 @@
 // ("SM_alloc" P:93-99, "Reg_alloc(C)" P:101, Volkov-style scheme P:75) with
 // the structure of every routine applied while the tile is staged to shared
 // memory (mirror / zero-select / unit diagonal, via load_op) and the uplo
-// mask applied in the epilogue.  128x128 CTA tile, BK=16, 256 threads,
-// 8x8 outputs per thread, register-prefetched double buffer.
+// mask applied in the epilogue.  128x128 CTA tile, BK=8, 256 threads, 8x8
+// outputs per thread, register-prefetched double buffer.  It is the route for
+// arguments TMA cannot address (unaligned pointers, ld % 4 != 0) and the FP32
+// comparison point for the 3xTF32 path.
+//
+// The Problem stays in kernel-parameter space (dynamic segment indexing
+// becomes constant-bank loads); only the current segment's operand
+// descriptors are copied to registers.
 #include <cuda_runtime.h>
 #include "problem.h"
 #include "kernels.h"
@@ -13,7 +19,8 @@
 namespace blas3 {
 
 namespace {
-constexpr int BM = 128, BN = 128, BK = 16, NT = 256, PADS = 4;
+constexpr int BM = 128, BN = 128, BK = 8, NT = 256, PADS = 4;
+constexpr int EPT = BM * BK / NT;         // elements of each operand fetched per thread (4)
 
 struct Stage {
   float a[BK][BM + PADS];
@@ -21,57 +28,44 @@ struct Stage {
 };
 
 // r-contiguous ("rk") or k-contiguous ("kr") element mapping for coalescing
-__device__ __forceinline__ void elem_rk(int tid, int i, int &r, int &k) {
-  int e = tid + i * NT; r = e % BM; k = e / BM;
-}
-__device__ __forceinline__ void elem_kr(int tid, int i, int &r, int &k) {
-  int e = tid + i * NT; k = e % BK; r = e / BK;
+__device__ __forceinline__ void elem_map(bool kr, int tid, int i, int &r, int &k) {
+  const int e = tid + i * NT;
+  if (kr) { k = e % BK; r = e / BK; } else { r = e % BM; k = e / BM; }
 }
 __device__ __forceinline__ bool prefers_kr(const OpDesc &o) {
   return o.kind == OP_DENSE ? o.kr != 0 : (o.kind == OP_TRI ? o.swap != 0 : false);
 }
 
-__device__ __forceinline__ void fetch(const OpDesc &o, bool kr, int64_t R, int64_t K,
-                                      int64_t r0, int64_t kb, float (&v)[8]) {
-  int tid = threadIdx.x;
+__device__ __forceinline__ void fetch(const OpDesc &o, bool kr, int64_t R, int64_t K, int64_t r0,
+                                      int64_t kb, float (&v)[EPT]) {
 #pragma unroll
-  for (int i = 0; i < 8; ++i) {
+  for (int i = 0; i < EPT; ++i) {
     int r, k;
-    if (kr) elem_kr(tid, i, r, k); else elem_rk(tid, i, r, k);
+    elem_map(kr, threadIdx.x, i, r, k);
     v[i] = load_op(o, r0 + r, kb + k, R, K);
   }
 }
 
-__device__ __forceinline__ void stash(float (*dst)[BM + PADS], bool kr, const float (&v)[8]) {
-  int tid = threadIdx.x;
+__device__ __forceinline__ void stash(float (*dst)[BM + PADS], bool kr, const float (&v)[EPT]) {
 #pragma unroll
-  for (int i = 0; i < 8; ++i) {
+  for (int i = 0; i < EPT; ++i) {
     int r, k;
-    if (kr) elem_kr(tid, i, r, k); else elem_rk(tid, i, r, k);
+    elem_map(kr, threadIdx.x, i, r, k);
     dst[k][r] = v[i];
   }
 }
 }  // namespace
 
 __global__ void __launch_bounds__(NT, 2)
-simt_structured_gemm(const Problem P0) {
+simt_structured_gemm(const Problem P) {
   __shared__ __align__(16) Stage st[2];
   const int tid = threadIdx.x, tx = tid % 16, ty = tid / 16;
-  const int64_t tiles_per = Tiles<BM, BN>::count(P0);
-  const int64_t nb = P0.nbatch > 0 ? P0.nbatch : 1;
+  const int64_t tiles_per = Tiles<BM, BN>::count(P);
+  const int64_t nb = P.nbatch > 0 ? P.nbatch : 1;
   const int64_t ntiles = tiles_per * nb;
 
   for (int64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x) {
-    // batch member of this tile: offset seg[0] operands and C
     const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
-    Problem P = P0;
-    if (nb > 1) {
-      P.seg[0].a.ptr += batch_off(P0.bs_a, b, P0.per);
-      P.seg[0].b.ptr += batch_off(P0.bs_b, b, P0.per);
-      const int64_t oc = batch_off(P0.bs_c, b, P0.per);
-      P.Cin += oc;
-      P.Cout += oc;
-    }
     int64_t mi, nj;
     Tiles<BM, BN>::coords(P, t, mi, nj);
     const int64_t m0 = mi * BM, n0 = nj * BN;
@@ -84,15 +78,21 @@ simt_structured_gemm(const Problem P0) {
       for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
 
     for (int s = 0; s < P.nseg; ++s) {
-      const Segment &sg = P.seg[s];
+      OpDesc oa = P.seg[s].a, ob = P.seg[s].b;     // registers from here on
+      const int64_t K = P.seg[s].K;
+      if (nb > 1) {
+        oa.ptr += batch_off(P.bs_a, b, P.per);
+        ob.ptr += batch_off(P.bs_b, b, P.per);
+      }
+      Segment sg; sg.a = oa; sg.b = ob; sg.K = K;
       int64_t k0, k1;
       k_range(sg, m0, m1, n0, n1, k0, k1);
       k0 = (k0 / BK) * BK;
       if (k1 <= k0) continue;
-      const bool akr = prefers_kr(sg.a), bkr = prefers_kr(sg.b);
-      float va[8], vb[8];
-      fetch(sg.a, akr, P.M, sg.K, m0, k0, va);
-      fetch(sg.b, bkr, P.N, sg.K, n0, k0, vb);
+      const bool akr = prefers_kr(oa), bkr = prefers_kr(ob);
+      float va[EPT], vb[EPT];
+      fetch(oa, akr, P.M, K, m0, k0, va);
+      fetch(ob, bkr, P.N, K, n0, k0, vb);
       int buf = 0;
       __syncthreads();  // previous tile/segment finished reading smem
       stash(st[0].a, akr, va);
@@ -101,22 +101,22 @@ simt_structured_gemm(const Problem P0) {
       for (int64_t kb = k0; kb < k1; kb += BK) {
         const bool more = kb + BK < k1;
         if (more) {
-          fetch(sg.a, akr, P.M, sg.K, m0, kb + BK, va);
-          fetch(sg.b, bkr, P.N, sg.K, n0, kb + BK, vb);
+          fetch(oa, akr, P.M, K, m0, kb + BK, va);
+          fetch(ob, bkr, P.N, K, n0, kb + BK, vb);
         }
         const Stage &S = st[buf];
 #pragma unroll
         for (int k = 0; k < BK; ++k) {
-          float4 a0 = *reinterpret_cast<const float4 *>(&S.a[k][tx * 4]);
-          float4 a1 = *reinterpret_cast<const float4 *>(&S.a[k][64 + tx * 4]);
-          float4 b0 = *reinterpret_cast<const float4 *>(&S.b[k][ty * 4]);
-          float4 b1 = *reinterpret_cast<const float4 *>(&S.b[k][64 + ty * 4]);
-          float a[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-          float b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+          const float4 a0 = *reinterpret_cast<const float4 *>(&S.a[k][tx * 4]);
+          const float4 a1 = *reinterpret_cast<const float4 *>(&S.a[k][64 + tx * 4]);
+          const float4 b0 = *reinterpret_cast<const float4 *>(&S.b[k][ty * 4]);
+          const float4 b1 = *reinterpret_cast<const float4 *>(&S.b[k][64 + ty * 4]);
+          const float a[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+          const float bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
 #pragma unroll
           for (int i = 0; i < 8; ++i)
 #pragma unroll
-            for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+            for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], bb[j], acc[i][j]);
         }
         if (more) {
           stash(st[buf ^ 1].a, akr, va);
@@ -128,19 +128,22 @@ simt_structured_gemm(const Problem P0) {
     }
 
     // epilogue: D = alpha*acc + beta*C on the (masked) tile
+    const int64_t coff = (nb > 1) ? batch_off(P.bs_c, b, P.per) : 0;
+    const float *cin = P.Cin + coff;
+    float *cout = P.Cout + coff;
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
-      int64_t c = n0 + (j < 4 ? ty * 4 + j : 64 + ty * 4 + (j - 4));
+      const int64_t c = n0 + (j < 4 ? ty * 4 + j : 64 + ty * 4 + (j - 4));
       if (c >= P.N) continue;
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
-        int64_t r = m0 + (i < 4 ? tx * 4 + i : 64 + tx * 4 + (i - 4));
+        const int64_t r = m0 + (i < 4 ? tx * 4 + i : 64 + tx * 4 + (i - 4));
         if (r >= P.M) continue;
         if (P.c_tri == 1 && r < c) continue;
         if (P.c_tri == 2 && r > c) continue;
         float v = P.alpha * acc[i][j];
-        if (P.beta != 0.f) v = fmaf(P.beta, P.Cin[r + c * P.ldcin], v);
-        P.Cout[r + c * P.ldcout] = v;
+        if (P.beta != 0.f) v = fmaf(P.beta, cin[r + c * P.ldcin], v);
+        cout[r + c * P.ldcout] = v;
       }
     }
   }
