@@ -221,6 +221,11 @@ __device__ __forceinline__ void tri_fix(const OpDesc &o, int lay, uint8_t *raw, 
   }
 }
 
+__device__ __forceinline__ void zero_fill(uint8_t *buf, uint32_t bytes, int t) {
+  float4 *b4 = reinterpret_cast<float4 *>(buf);
+  for (uint32_t c = t; c < bytes / 16; c += TR_THREADS) b4[c] = make_float4(0.f, 0.f, 0.f, 0.f);
+}
+
 // 3xTF32 split without rewriting hi: kind::tf32 UMMA reads the raw fp32
 // word and ignores its low 13 mantissa bits, i.e. it consumes
 // hi = trunc_tf32(x) directly from the TMA-staged tile (pinned by
@@ -506,10 +511,22 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           ptx::mbar_wait(&bars->full[rs], ph);
           RawBuf &rb = raw[rs];
           bool fix = false;
+          // fix-ups are decided on this CTA's own half: a half that is entirely
+          // in the nonzero region needs none, an entirely blank half is a
+          // vectorised zero-fill, only halves touching the diagonal go per element
+          const int64_t k1 = imin(sg.K, k0 + BK);
           if (si.clsA == BLK_SYM_DIAG) { sym_merge(sg.a, rb.A, ma, k0, HA, P.M, sg.K, tt); fix = true; }
-          else if (si.clsA == BLK_TRI_DIAG) { tri_fix(sg.a, si.layA, rb.A, ma, k0, HA, P.M, sg.K, tt); fix = true; }
+          else if (si.clsA == BLK_TRI_DIAG) {
+            const int own = block_class(sg.a, ma, imin(P.M, ma + HA), k0, k1);
+            if (own == BLK_ZERO) { zero_fill(rb.A, G::A_BYTES, tt); fix = true; }
+            else if (own == BLK_TRI_DIAG) { tri_fix(sg.a, si.layA, rb.A, ma, k0, HA, P.M, sg.K, tt); fix = true; }
+          }
           if (si.clsB == BLK_SYM_DIAG) { sym_merge(sg.b, rb.B, nb, k0, HB, P.N, sg.K, tt); fix = true; }
-          else if (si.clsB == BLK_TRI_DIAG) { tri_fix(sg.b, si.layB, rb.B, nb, k0, HB, P.N, sg.K, tt); fix = true; }
+          else if (si.clsB == BLK_TRI_DIAG) {
+            const int own = block_class(sg.b, nb, imin(P.N, nb + HB), k0, k1);
+            if (own == BLK_ZERO) { zero_fill(rb.B, G::B_BYTES, tt); fix = true; }
+            else if (own == BLK_TRI_DIAG) { tri_fix(sg.b, si.layB, rb.B, nb, k0, HB, P.N, sg.K, tt); fix = true; }
+          }
           if (fix) ptx::named_bar_sync(1, TR_THREADS);
           ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
           if (!(P.dbg & 1)) {
