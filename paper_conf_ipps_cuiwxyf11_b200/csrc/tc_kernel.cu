@@ -584,8 +584,48 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
       const float *cin = P.Cin + coff + r;
       float *cout = P.Cout + coff + r;
       const int64_t cbase = n0 + half * (BN / 2);
-      // per 8-column group: all C loads first, then the stores (Cin may alias
-      // Cout); each is a coalesced 128-B warp access.
+      // Fast path: this warp group's 128 x 128 block lies inside the matrix and
+      // entirely inside the referenced triangle -> no per-element predicates,
+      // strength-reduced column pointers (the epilogue shares issue slots with
+      // the transform warps, so its instruction count matters).
+      const int64_t rlo = m0 + HA * rank, chi = cbase + BN / 2 - 1;
+      const bool interior = rlo + HA <= P.M && chi < P.N &&
+                            (P.c_tri == 0 || (P.c_tri == 1 && rlo >= chi) ||
+                             (P.c_tri == 2 && rlo + HA - 1 <= cbase));
+      if (interior) {
+        const int64_t ldi = P.ldcin, ldo = P.ldcout;
+        const float *cp = cin + cbase * ldi;
+        float *op = cout + cbase * ldo;
+        const float al = P.alpha, be = P.beta;
+        const bool nostore = (P.dbg & 4) != 0;
+        if (be != 0.f) {
+          // D = alpha*S + beta*C: group g+1's C loads are issued before group
+          // g's stores (different columns; in-place D reuses S's registers).
+          constexpr int SG = 8;
+          float cv[SG];
+#pragma unroll
+          for (int j = 0; j < SG; ++j) cv[j] = __ldcs(cp + j * ldi);
+#pragma unroll
+          for (int g = 0; g < NG * EC / SG; ++g) {
+#pragma unroll
+            for (int j = 0; j < SG; ++j) S[g * SG + j] = fmaf(be, cv[j], al * S[g * SG + j]);
+            if (g + 1 < NG * EC / SG) {
+#pragma unroll
+              for (int j = 0; j < SG; ++j) cv[j] = __ldcs(cp + ((g + 1) * SG + j) * ldi);
+            }
+            if (!nostore) {
+#pragma unroll
+              for (int j = 0; j < SG; ++j) __stcs(op + (g * SG + j) * ldo, S[g * SG + j]);
+            }
+          }
+        } else if (!nostore) {
+#pragma unroll
+          for (int i = 0; i < NG * EC; ++i) __stcs(op + i * ldo, al * S[i]);
+        }
+        continue;
+      }
+      // general path (edge / diagonal tiles): per 8-column group all C loads
+      // first, then the stores (Cin may alias Cout); coalesced 128-B accesses.
       auto ok_at = [&](int64_t c) {
         return row_ok && c < P.N && !(P.c_tri == 1 && r < c) && !(P.c_tri == 2 && r > c);
       };
