@@ -68,17 +68,14 @@ __device__ __forceinline__ void st_remote_and_arrive(int64_t *slot, int64_t v, u
   asm volatile("st.shared::cluster.b64 [%0], %1;" ::"r"(rs), "l"(v) : "memory");
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(rb) : "memory");
 }
-__device__ __forceinline__ bool mbar_try_wait_cluster(uint64_t *bar, uint32_t parity) {
-  uint32_t ok;
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n\t"
-      "selp.u32 %0, 1, 0, p;\n\t}"
-      : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
-  return ok != 0;
-}
+// Wait on a barrier that peer CTAs of the cluster arrive on.  The poll is a
+// CTA-scope acquire: what it guards is shared memory written through DSMEM
+// before a release.cluster arrive, and smem / TMEM reuse by the async proxy --
+// none of it lives in L1.  (An .acquire.cluster poll compiles to CCTL.IVALL,
+// an L1 invalidate on every iteration, which the profile showed as the top
+// stall of the pair kernel.)
 __device__ __forceinline__ void mbar_wait_cluster(uint64_t *bar, uint32_t parity) {
-  while (!mbar_try_wait_cluster(bar, parity)) {}
+  while (!mbar_try_wait(bar, parity)) {}
 }
 
 // ------------------------------------------------------------------ fences / barriers
