@@ -454,6 +454,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
         P.seg[0].b = in_w ? dense(W.p, pr, true) : dense(B + p0, ldb, true);
         P.seg[0].K = pr;
         P.rev_m = tri_kle(P.seg[0].a);
+        P.outer = 1;                     // all longest m-rows first (LPT)
         if ((rc2 = run_problem(P, s, sms))) return rc2;
         if (!in_w && launch_copy(B + p0, ldb, W.p, pr, pr, n, s)) return BLAS3_ERR_CUDA;
       } else {
@@ -464,6 +465,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
         P.seg[0].b = tri(Dp, NBO, true, lower_op, false);
         P.seg[0].K = pr;
         P.rev_n = tri_kle(P.seg[0].b);
+        P.outer = 2;
         if ((rc2 = run_problem(P, s, sms))) return rc2;
         if (!in_w && launch_copy(B + p0 * ldb, ldb, W.p, m, m, pr, s)) return BLAS3_ERR_CUDA;
       }

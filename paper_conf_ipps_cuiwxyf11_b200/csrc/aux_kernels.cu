@@ -17,81 +17,153 @@
 namespace blas3 {
 
 // ---------------------------------------------------------------- scale / copy
-__global__ void scale_kernel(float *C, int64_t ldc, int64_t m, int64_t n, float beta, int tri) {
-  int64_t total = m * n;
-  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total;
-       e += (int64_t)gridDim.x * blockDim.x) {
-    int64_t r = e % m, c = e / m;
-    if (tri == 1 && r < c) continue;
-    if (tri == 2 && r > c) continue;
-    float *p = C + r + c * ldc;
-    *p = (beta == 0.f) ? 0.f : beta * *p;     // beta = 0: C not read (Q11)
+// Column-major 2-D grids: blockIdx.x covers rows (4 per thread when the
+// columns are 16-byte aligned), blockIdx.y strides over columns, CU unrolled
+// so each thread keeps several independent accesses in flight.  HBM-bound:
+// 4 (scale, beta != 0: 8) bytes per element.
+namespace {
+constexpr int AUX_T = 256, CU = 4;
+inline dim3 aux_grid(int64_t m, int64_t n, bool vec) {
+  const int64_t rows_per_cta = AUX_T * (vec ? 4 : 1);
+  const int64_t gx = cdiv(m, rows_per_cta);
+  const int64_t gy = imin(cdiv(n, CU), imax(1, (148 * 32) / imax(1, gx)));
+  return dim3((unsigned)gx, (unsigned)imin(gy, 65535));
+}
+inline bool aligned16(const void *p, int64_t ld, int64_t m) {
+  return ((uintptr_t)p % 16 == 0) && ld % 4 == 0 && m % 4 == 0;
+}
+}  // namespace
+
+template <bool VEC>
+__global__ void __launch_bounds__(AUX_T)
+scale_kernel(float *C, int64_t ldc, int64_t m, int64_t n, float beta, int tri) {
+  const int64_t r = ((int64_t)blockIdx.x * AUX_T + threadIdx.x) * (VEC ? 4 : 1);
+  if (r >= m) return;
+  for (int64_t c0 = (int64_t)blockIdx.y * CU; c0 < n; c0 += (int64_t)gridDim.y * CU) {
+#pragma unroll
+    for (int u = 0; u < CU; ++u) {
+      const int64_t c = c0 + u;
+      if (c >= n) break;
+      float *p = C + r + c * ldc;
+      if (VEC && tri == 0) {
+        float4 v = beta == 0.f ? make_float4(0.f, 0.f, 0.f, 0.f) : *reinterpret_cast<float4 *>(p);
+        if (beta != 0.f) { v.x *= beta; v.y *= beta; v.z *= beta; v.w *= beta; }
+        *reinterpret_cast<float4 *>(p) = v;
+      } else {
+#pragma unroll
+        for (int e = 0; e < (VEC ? 4 : 1); ++e) {
+          const int64_t rr = r + e;
+          if (rr >= m || (tri == 1 && rr < c) || (tri == 2 && rr > c)) continue;
+          p[e] = (beta == 0.f) ? 0.f : beta * p[e];     // beta = 0: C not read (Q11)
+        }
+      }
+    }
   }
 }
 
 int launch_scale(float *C, int64_t ldc, int64_t m, int64_t n, float beta, int tri, cudaStream_t s) {
   if (m <= 0 || n <= 0) return 0;
-  int64_t total = m * n;
-  int64_t blocks = imin(cdiv(total, 256), 148 * 16);
-  scale_kernel<<<(unsigned)blocks, 256, 0, s>>>(C, ldc, m, n, beta, tri);
+  const bool vec = aligned16(C, ldc, m);
+  const dim3 g = aux_grid(m, n, vec);
+  if (vec) scale_kernel<true><<<g, AUX_T, 0, s>>>(C, ldc, m, n, beta, tri);
+  else scale_kernel<false><<<g, AUX_T, 0, s>>>(C, ldc, m, n, beta, tri);
   note_launch();
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
 
-__global__ void copy_kernel(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t m, int64_t n) {
-  int64_t total = m * n;
-  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total;
-       e += (int64_t)gridDim.x * blockDim.x) {
-    int64_t r = e % m, c = e / m;
-    dst[r + c * ldd] = src[r + c * lds];
+template <bool VEC>
+__global__ void __launch_bounds__(AUX_T)
+copy_kernel(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t m, int64_t n) {
+  const int64_t r = ((int64_t)blockIdx.x * AUX_T + threadIdx.x) * (VEC ? 4 : 1);
+  if (r >= m) return;
+  for (int64_t c0 = (int64_t)blockIdx.y * CU; c0 < n; c0 += (int64_t)gridDim.y * CU) {
+    if (VEC) {
+      float4 v[CU];
+#pragma unroll
+      for (int u = 0; u < CU; ++u)
+        if (c0 + u < n) v[u] = __ldcs(reinterpret_cast<const float4 *>(src + r + (c0 + u) * lds));
+#pragma unroll
+      for (int u = 0; u < CU; ++u)
+        if (c0 + u < n) __stcs(reinterpret_cast<float4 *>(dst + r + (c0 + u) * ldd), v[u]);
+    } else {
+#pragma unroll
+      for (int u = 0; u < CU; ++u)
+        if (c0 + u < n) dst[r + (c0 + u) * ldd] = src[r + (c0 + u) * lds];
+    }
   }
 }
 
 int launch_copy(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t m, int64_t n,
                 cudaStream_t s) {
   if (m <= 0 || n <= 0) return 0;
-  int64_t blocks = imin(cdiv(m * n, 256), 148 * 16);
-  copy_kernel<<<(unsigned)blocks, 256, 0, s>>>(dst, ldd, src, lds, m, n);
+  const bool vec = aligned16(dst, ldd, m) && aligned16(src, lds, m);
+  const dim3 g = aux_grid(m, n, vec);
+  if (vec) copy_kernel<true><<<g, AUX_T, 0, s>>>(dst, ldd, src, lds, m, n);
+  else copy_kernel<false><<<g, AUX_T, 0, s>>>(dst, ldd, src, lds, m, n);
   note_launch();
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
 
 // ---------------------------------------------------------------- TRSM diag inverse
 namespace {
-constexpr int DNB = 128;          // diagonal block size (4 warps x 32)
-constexpr int DLD = DNB + 1;      // padded smem row (bank-conflict free)
+constexpr int DNB = 128;          // diagonal block size (4 x 32)
+constexpr int DLD = DNB + 4;      // padded smem row (16-B aligned rows for float4 broadcasts)
+constexpr int DT = 256;           // threads: 8 warps
 }
 
-// One CTA (128 threads) per 128-block of L (the stored triangle of A in
-// lower form); X = inv(L_bb) written into the panel-inverse workspace.
-__global__ void __launch_bounds__(128)
+// One CTA per 128-block of L (the stored triangle of A in lower form);
+// X = inv(L_bb) is written into the panel-inverse workspace.
+//   staging : the raw 128 x 128 block of A, loaded column by column (coalesced,
+//             16 loads in flight per thread), then L built in shared memory
+//             (transposed when the stored triangle is the upper one; the blank
+//             triangle of A is never read, Q8)
+//   phase 1 : warp w < 4 inverts L_ww (32 x 32) by forward substitution --
+//             lane j solves column j, the rows of L broadcast by shuffles
+//   phase 2 : block forward substitution X(I,J) = -inv(L_II) sum_{K=J}^{I-1}
+//             L(I,K) X(K,J); block column J is a chain over I, its 32 rows of
+//             the running sum are split between two warps (8 warps, 4 columns)
+__global__ void __launch_bounds__(DT)
 trsm_diag_inv_kernel(const float *A, int64_t lda, int64_t n, int stored_lower, int unit,
                      float *Dinv, int64_t ldD) {
-  extern __shared__ float sm[];
-  float *L = sm;                  // [DNB][DLD]
-  float *X = sm + DNB * DLD;      // [DNB][DLD]
+  extern __shared__ __align__(16) float sm[];
+  float *L = sm;                  // [DNB][DLD]  row-major L
+  float *X = sm + DNB * DLD;      // [DNB][DLD]  row-major inverse (staging first)
+  float *T = X + DNB * DLD;       // [4][32][33] partial sums of phase 2
   const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
   const int64_t i0 = (int64_t)blockIdx.x * DNB;
   const int nr = (int)imin(DNB, n - i0);
 
-  // stage L (lower) and clear X; the blank triangle of A is never read (Q8)
-  for (int c = 0; c < DNB; ++c) {
-    const int r = tid;
-    float v = 0.f;
-    if (r < nr && c < nr) {
-      if (r == c) v = unit ? 1.f : A[(i0 + r) + (i0 + r) * lda];
-      else if (r > c) v = stored_lower ? A[(i0 + r) + (i0 + c) * lda] : A[(i0 + c) + (i0 + r) * lda];
-    } else if (r == c) {
-      v = 1.f;                     // identity padding of a ragged last block
+  // staging: thread (r = tid % 128) loads columns c = tid/128 + 2u of the raw
+  // block (only the stored triangle), 16 independent loads at a time
+  {
+    const int r = tid % DNB, c0 = tid / DNB;
+    const float *col = A + i0 + r + i0 * lda;
+    for (int u0 = 0; u0 < DNB / 2; u0 += 16) {
+      float v[16];
+#pragma unroll
+      for (int u = 0; u < 16; ++u) {
+        const int c = c0 + 2 * (u0 + u);
+        const bool stored = stored_lower ? (r >= c) : (r <= c);
+        v[u] = (r < nr && c < nr && stored) ? __ldg(col + (int64_t)c * lda) : 0.f;
+      }
+#pragma unroll
+      for (int u = 0; u < 16; ++u) X[r * DLD + c0 + 2 * (u0 + u)] = v[u];
     }
-    L[r * DLD + c] = v;
-    X[r * DLD + c] = 0.f;
   }
   __syncthreads();
+  for (int e = tid; e < DNB * DNB; e += DT) {
+    const int r = e / DNB, c = e % DNB;
+    float v = 0.f;
+    if (r == c) v = (unit || r >= nr) ? 1.f : X[r * DLD + r];     // identity padding when ragged
+    else if (r > c) v = stored_lower ? X[r * DLD + c] : X[c * DLD + r];
+    L[r * DLD + c] = v;
+  }
+  __syncthreads();
+  for (int e = tid; e < DNB * DNB; e += DT) X[(e / DNB) * DLD + e % DNB] = 0.f;
+  __syncthreads();
 
-  // phase 1: warp w inverts L_ww (32x32) -- lane i holds row i of L_ww,
-  // lane j solves for column j of the inverse; rows broadcast by shuffles.
-  {
+  // phase 1
+  if (warp < 4) {
     const int b = warp * 32;
     float lrow[32], x[32];
 #pragma unroll
@@ -108,29 +180,55 @@ trsm_diag_inv_kernel(const float *A, int64_t lda, int64_t n, int stored_lower, i
   }
   __syncthreads();
 
-  // phase 2: block forward substitution, warp J owns block column J:
-  //   X(I,J) = -inv(L_II) * sum_{K=J}^{I-1} L(I,K) X(K,J)
+  // phase 2: warps (2J, 2J+1) own block column J < 3; each sums 16 of the 32
+  // rows of t = sum_K L(I,K) X(K,J) (L rows as float4 broadcasts, X(K,J)
+  // column in registers), then both apply -inv(L_II) to 16 rows each.
   {
-    const int J = warp, c = J * 32 + lane;
-    for (int I = J + 1; I < 4; ++I) {
-      float t[32];
+    const int J = warp / 2, h = warp % 2, c = J * 32 + lane;
+    float *Tj = T + J * 32 * 33;
+    const uint32_t bar = 1 + J;                    // named barrier per column pair
+    for (int I = J + 1; I < 4 && J < 3; ++I) {
+      float t[16];
 #pragma unroll
-      for (int ii = 0; ii < 32; ++ii) t[ii] = 0.f;
+      for (int ii = 0; ii < 16; ++ii) t[ii] = 0.f;
       for (int K = J; K < I; ++K) {
-        for (int kk = 0; kk < 32; ++kk) {
-          float xk = X[(K * 32 + kk) * DLD + c];
+        float xk[32];
 #pragma unroll
-          for (int ii = 0; ii < 32; ++ii) t[ii] = fmaf(L[(I * 32 + ii) * DLD + K * 32 + kk], xk, t[ii]);
+        for (int kk = 0; kk < 32; ++kk) xk[kk] = X[(K * 32 + kk) * DLD + c];
+#pragma unroll
+        for (int ii = 0; ii < 16; ++ii) {
+          const float4 *lr = reinterpret_cast<const float4 *>(&L[(I * 32 + h * 16 + ii) * DLD + K * 32]);
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            const float4 l4 = lr[q];
+            t[ii] = fmaf(l4.x, xk[4 * q], t[ii]);
+            t[ii] = fmaf(l4.y, xk[4 * q + 1], t[ii]);
+            t[ii] = fmaf(l4.z, xk[4 * q + 2], t[ii]);
+            t[ii] = fmaf(l4.w, xk[4 * q + 3], t[ii]);
+          }
         }
       }
-#pragma unroll 4
-      for (int ii = 0; ii < 32; ++ii) {
+#pragma unroll
+      for (int ii = 0; ii < 16; ++ii) Tj[(h * 16 + ii) * 33 + lane] = t[ii];
+      asm volatile("bar.sync %0, 64;" ::"r"(bar) : "memory");
+      float tt[32];
+#pragma unroll
+      for (int q = 0; q < 32; ++q) tt[q] = Tj[q * 33 + lane];
+#pragma unroll
+      for (int ii = 0; ii < 16; ++ii) {
+        const float4 *xr = reinterpret_cast<const float4 *>(&X[(I * 32 + h * 16 + ii) * DLD + I * 32]);
         float v = 0.f;
 #pragma unroll
-        for (int q = 0; q < 32; ++q) v = fmaf(X[(I * 32 + ii) * DLD + I * 32 + q], t[q], v);
-        X[(I * 32 + ii) * DLD + c] = -v;
+        for (int q = 0; q < 8; ++q) {
+          const float4 x4 = xr[q];
+          v = fmaf(x4.x, tt[4 * q], v);
+          v = fmaf(x4.y, tt[4 * q + 1], v);
+          v = fmaf(x4.z, tt[4 * q + 2], v);
+          v = fmaf(x4.w, tt[4 * q + 3], v);
+        }
+        X[(I * 32 + h * 16 + ii) * DLD + c] = -v;
       }
-      __syncwarp();
+      asm volatile("bar.sync %0, 64;" ::"r"(bar) : "memory");
     }
   }
   __syncthreads();
@@ -138,16 +236,18 @@ trsm_diag_inv_kernel(const float *A, int64_t lda, int64_t n, int stored_lower, i
   // write inv(L_bb) (lower, column-major) into its panel slot; padded rows/cols zero
   const int64_t bpp = ldD / DNB;                     // 128-blocks per panel
   float *D = Dinv + (blockIdx.x / bpp) * ldD * ldD + (blockIdx.x % bpp) * DNB * (1 + ldD);
-  for (int c = 0; c < DNB; ++c) {
-    const int r = tid;
-    D[r + (int64_t)c * ldD] = (r < nr && c < nr) ? X[r * DLD + c] : 0.f;
+  {
+    const int r = tid % DNB, c0 = tid / DNB;
+#pragma unroll 8
+    for (int c = c0; c < DNB; c += 2)
+      D[r + (int64_t)c * ldD] = (r < nr && c < nr && r >= c) ? X[r * DLD + c] : 0.f;
   }
 }
 
 int launch_trsm_diag_inv(const float *A, int64_t lda, int64_t n, int stored_lower, int unit,
                          float *Dinv, int64_t ldD, cudaStream_t s) {
   if (ldD % DNB) return -1;
-  const size_t smem = 2 * DNB * DLD * sizeof(float);
+  const size_t smem = (2 * DNB * DLD + 4 * 32 * 33) * sizeof(float);
   static bool attr = false;
   if (!attr) {
     if (cudaFuncSetAttribute(trsm_diag_inv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -155,7 +255,7 @@ int launch_trsm_diag_inv(const float *A, int64_t lda, int64_t n, int stored_lowe
     attr = true;
   }
   int64_t blocks = cdiv(n, DNB);
-  trsm_diag_inv_kernel<<<(unsigned)blocks, 128, smem, s>>>(A, lda, n, stored_lower, unit, Dinv, ldD);
+  trsm_diag_inv_kernel<<<(unsigned)blocks, DT, smem, s>>>(A, lda, n, stored_lower, unit, Dinv, ldD);
   note_launch();
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }

@@ -61,6 +61,7 @@ struct Problem {
   int32_t c_tri;    // 0: full C; 1: lower triangle only; 2: upper only
   int32_t rev_m;    // schedule m-tiles in reverse (longest K first)
   int32_t rev_n;
+  int32_t outer;    // full grid order: 0 grouped raster, 1 m-tiles outer, 2 n-tiles outer
   float alpha, beta;
   const float *Cin; int64_t ldcin;   // read only when beta != 0
   float *Cout; int64_t ldcout;
@@ -109,7 +110,11 @@ struct Tiles {
   // tile index -> (m-tile, n-tile)
   HD static void coords(const Problem &P, int64_t t, int64_t &mi, int64_t &nj) {
     int64_t mt = cdiv(P.M, BM), nt = cdiv(P.N, BN);
-    if (P.c_tri == 0) {
+    if (P.c_tri == 0 && P.outer == 1) {          // whole m-rows in turn (with rev_m:
+      mi = t / nt; nj = t - mi * nt;             // longest-processing-time first)
+    } else if (P.c_tri == 0 && P.outer == 2) {
+      nj = t / mt; mi = t - nj * mt;
+    } else if (P.c_tri == 0) {
       int64_t per_group = (int64_t)GM * nt;
       int64_t g = t / per_group, local = t - g * per_group;
       int64_t gm = imin(GM, mt - g * GM);

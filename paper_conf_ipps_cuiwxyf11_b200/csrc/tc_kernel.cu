@@ -31,6 +31,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <mutex>
+#include <cstdio>
 #include <stdlib.h>
 #include <string.h>
 
@@ -109,8 +110,20 @@ struct Geo {
 struct TcParams {
   CUtensorMap maps[MAX_MAPS];
   Problem P;
-  uint32_t *tile_ctr;      // dynamic tile scheduler counter (zeroed per launch), or null
+  uint32_t *tile_ctr;      // dynamic tile scheduler counter, or null (static schedule)
+  uint32_t tile_base;      // its value when this launch starts
+  unsigned long long *trace;   // phase timestamps of CTA 0 (env BLAS3_TRACE), or null
 };
+
+// %globaltimer (ns) of the first occurrence of a phase in CTA 0 (diagnostics)
+#define BLAS3_TRACE(i)                                                              \
+  do {                                                                              \
+    if (prm.trace != nullptr && blockIdx.x == 0 && prm.trace[i] == 0ull) {          \
+      unsigned long long t_;                                                        \
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                        \
+      prm.trace[i] = t_;                                                            \
+    }                                                                               \
+  } while (0)
 
 
 // byte offset of element (r, k) inside a staged operand tile
@@ -295,6 +308,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
   const int64_t cid = blockIdx.x / CG, ncl = gridDim.x / CG;
 
   if (threadIdx.x == 0) {
+    BLAS3_TRACE(0);
     for (int s = 0; s < RS; ++s) {
       ptx::mbar_init(&bars->full[s], 1);
       ptx::mbar_init(&bars->empty[s], 1);
@@ -318,6 +332,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
   if (CG == 2) ptx::cluster_sync(); else __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = bars->tmem_base;
+  if (threadIdx.x == 0) BLAS3_TRACE(1);
 
   // batched problems: tile tb -> batch member b = tb / tiles_per, tile t
   const int64_t tiles_per = Tiles<TM, BN>::count(P);
@@ -358,8 +373,12 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
         int64_t tb;
         if (CG == 1 || rank == 0) {
           // claim a tile (dynamic) or take the static round-robin one
-          tb = prm.tile_ctr ? (int64_t)atomicAdd(prm.tile_ctr, 1u) : cid + (int64_t)qi * ncl;
+          // (the first tile of every producer is its own id: no claim round trip)
+          tb = (prm.tile_ctr == nullptr || qi == 0)
+                   ? cid + (int64_t)qi * ncl
+                   : ncl + (int64_t)(uint32_t)(atomicAdd(prm.tile_ctr, 1u) - prm.tile_base);
           if (tb >= ntiles) tb = -1;
+          BLAS3_TRACE(2);
           const int slot = qi % TQ;
           if (CG == 2) ptx::mbar_wait_cluster(&bars->tq_empty[slot], ((qi / TQ) & 1) ^ 1);
           else ptx::mbar_wait(&bars->tq_empty[slot], ((qi / TQ) & 1) ^ 1);
@@ -390,6 +409,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
             ptx::mbar_arrive_expect_tx(&bars->full[rs], (HA + HB) * BK * 4);
             load_operand(prm, sg.a, si.layA, raw[rs].A, ma, k0, HA, &bars->full[rs], bj, bg);
             load_operand(prm, sg.b, si.layB, raw[rs].B, nb, k0, HB, &bars->full[rs], bj, bg);
+            BLAS3_TRACE(3);
           }
         }
       }
@@ -469,6 +489,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
                 }
                 accumulate = 1;
               }
+              BLAS3_TRACE(6);
               if constexpr (CG == 1) {
                 ptx::mma_commit(&bars->empty[rs]);
                 ptx::mma_commit(&bars->lo_empty[ls]);
@@ -509,6 +530,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           const int64_t k0 = kb * BK;
           const StageInfo si = stage_info<CG>(P, sg, m0, n0, k0);
           ptx::mbar_wait(&bars->full[rs], ph);
+          if (tt == 0) BLAS3_TRACE(4);
           RawBuf &rb = raw[rs];
           bool fix = false;
           // fix-ups are decided on this CTA's own half: a half that is entirely
@@ -535,6 +557,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           }
           ptx::fence_proxy_async_smem();
           arrive_leader<CG>(&bars->ready[ls], rank, 2, TR_THREADS, tt == 0);
+          if (tt == 0) BLAS3_TRACE(5);
         }
       }
     }
@@ -565,6 +588,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
         const uint32_t buf = cc & 1, ph = (cc >> 1) & 1;
         ptx::mbar_wait(&bars->tfull[buf], ph);
         ptx::tc_fence_after();
+        if (threadIdx.x == WARP_EPI0 * 32) BLAS3_TRACE(7);
         if (nkb > 0) {
 #pragma unroll
           for (int g = 0; g < NG; ++g) {
@@ -579,78 +603,82 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
         ptx::tc_fence_before();
         arrive_leader<CG>(&bars->tempty[buf], rank, 3, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
       }
+      // ---- store phase: D = alpha*S + beta*C for row r, columns cbase + [0,128).
+      // The valid columns of the row form one range [jlo, jhi) (column bound
+      // N, uplo mask c_tri); each warp access is a coalesced 128-B line.
+      // Column pointers advance by ld (no per-element index math) and edge
+      // elements use single predicated ld/st instructions: the epilogue shares
+      // issue slots (and the instruction cache) with the transform warps.
       const int64_t r = m0 + HA * rank + q * 32 + lane;
-      const bool row_ok = r < P.M;
-      const float *cin = P.Cin + coff + r;
-      float *cout = P.Cout + coff + r;
       const int64_t cbase = n0 + half * (BN / 2);
-      // Fast path: this warp group's 128 x 128 block lies inside the matrix and
-      // entirely inside the referenced triangle -> no per-element predicates,
-      // strength-reduced column pointers (the epilogue shares issue slots with
-      // the transform warps, so its instruction count matters).
-      const int64_t rlo = m0 + HA * rank, chi = cbase + BN / 2 - 1;
-      const bool interior = rlo + HA <= P.M && chi < P.N &&
-                            (P.c_tri == 0 || (P.c_tri == 1 && rlo >= chi) ||
-                             (P.c_tri == 2 && rlo + HA - 1 <= cbase));
-      if (interior) {
-        const int64_t ldi = P.ldcin, ldo = P.ldcout;
-        const float *cp = cin + cbase * ldi;
-        float *op = cout + cbase * ldo;
-        const float al = P.alpha, be = P.beta;
-        const bool nostore = (P.dbg & 4) != 0;
-        if (be != 0.f) {
-          // D = alpha*S + beta*C: group g+1's C loads are issued before group
-          // g's stores (different columns; in-place D reuses S's registers).
-          constexpr int SG = 8;
-          float cv[SG];
-#pragma unroll
-          for (int j = 0; j < SG; ++j) cv[j] = __ldcs(cp + j * ldi);
-#pragma unroll
-          for (int g = 0; g < NG * EC / SG; ++g) {
-#pragma unroll
-            for (int j = 0; j < SG; ++j) S[g * SG + j] = fmaf(be, cv[j], al * S[g * SG + j]);
-            if (g + 1 < NG * EC / SG) {
-#pragma unroll
-              for (int j = 0; j < SG; ++j) cv[j] = __ldcs(cp + ((g + 1) * SG + j) * ldi);
-            }
-            if (!nostore) {
-#pragma unroll
-              for (int j = 0; j < SG; ++j) __stcs(op + (g * SG + j) * ldo, S[g * SG + j]);
-            }
-          }
-        } else if (!nostore) {
-#pragma unroll
-          for (int i = 0; i < NG * EC; ++i) __stcs(op + i * ldo, al * S[i]);
-        }
-        continue;
-      }
-      // general path (edge / diagonal tiles): per 8-column group all C loads
-      // first, then the stores (Cin may alias Cout); coalesced 128-B accesses.
-      auto ok_at = [&](int64_t c) {
-        return row_ok && c < P.N && !(P.c_tri == 1 && r < c) && !(P.c_tri == 2 && r > c);
-      };
+      const int64_t ldi = P.ldcin, ldo = P.ldcout;
+      const float *cp = P.Cin + coff + r + cbase * ldi;
+      float *op = P.Cout + coff + r + cbase * ldo;
+      const float al = P.alpha, be = P.beta;
+      const bool st_on = !(P.dbg & 4);
+      int jlo = 0, jhi = r < P.M ? (int)imin(BN / 2, P.N - cbase) : 0;
+      if (P.c_tri == 1) jhi = (int)imin(jhi, imax(0, r - cbase + 1));   // lower: c <= r
+      if (P.c_tri == 2) jlo = (int)imin(BN / 2, imax(0, r - cbase));    // upper: c >= r
+      const uint32_t jn = jhi > jlo ? (uint32_t)(jhi - jlo) : 0u;
+      const bool full = __all_sync(0xffffffffu, jlo == 0 && jhi == BN / 2);
+      const bool none = __all_sync(0xffffffffu, jn == 0u);
       constexpr int SG = 8;
+      if (none) {
+        // nothing of this warp's 32 x 128 block is referenced (ragged edge)
+      } else if (full && be == 0.f) {
+        if (st_on) {
 #pragma unroll
-      for (int g = 0; g < NG * EC / SG; ++g) {
-        const int64_t c0 = cbase + g * SG;
+          for (int i = 0; i < NG * EC; ++i) { ptx::st_cs(op, al * S[i]); op += ldo; }
+        }
+      } else if (full) {
+        // group g+1's C loads are issued before group g's stores (different
+        // columns; D is formed in place in S's registers)
         float cv[SG];
 #pragma unroll
-        for (int j = 0; j < SG; ++j)
-          cv[j] = (P.beta != 0.f && ok_at(c0 + j)) ? cin[(c0 + j) * P.ldcin] : 0.f;
+        for (int j = 0; j < SG; ++j) { cv[j] = ptx::ld_cs(cp); cp += ldi; }
 #pragma unroll
-        for (int j = 0; j < SG; ++j) {
-          const int64_t c = c0 + j;
-          if (ok_at(c) && !(P.dbg & 4)) cout[c * P.ldcout] = fmaf(P.beta, cv[j], P.alpha * S[g * SG + j]);
+        for (int g = 0; g < NG * EC / SG; ++g) {
+#pragma unroll
+          for (int j = 0; j < SG; ++j) S[g * SG + j] = fmaf(be, cv[j], al * S[g * SG + j]);
+          if (g + 1 < NG * EC / SG) {
+#pragma unroll
+            for (int j = 0; j < SG; ++j) { cv[j] = ptx::ld_cs(cp); cp += ldi; }
+          }
+          if (st_on) {
+#pragma unroll
+            for (int j = 0; j < SG; ++j) { ptx::st_cs(op, S[g * SG + j]); op += ldo; }
+          }
+        }
+      } else {
+        const bool ld_on = be != 0.f;
+#pragma unroll
+        for (int g = 0; g < NG * EC / SG; ++g) {
+          float cv[SG];
+#pragma unroll
+          for (int j = 0; j < SG; ++j) {
+            cv[j] = ptx::ld_cs_pred(cp, ld_on && (uint32_t)(g * SG + j - jlo) < jn);
+            cp += ldi;
+          }
+#pragma unroll
+          for (int j = 0; j < SG; ++j) {
+            ptx::st_cs_pred(op, fmaf(be, cv[j], al * S[g * SG + j]),
+                            st_on && (uint32_t)(g * SG + j - jlo) < jn);
+            op += ldo;
+          }
         }
       }
+      if (threadIdx.x == WARP_EPI0 * 32) BLAS3_TRACE(8);
     }
+    if (threadIdx.x == WARP_EPI0 * 32) BLAS3_TRACE(9);
   }
 
   ptx::tc_fence_before();
   if (CG == 2) ptx::cluster_sync(); else __syncthreads();
+  if (threadIdx.x == 0) BLAS3_TRACE(10);
   if (warp == WARP_MMA) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc<CG>(tmem, TMEM_COLS);
+    if (lane == 0) BLAS3_TRACE(11);
   }
 }
 
@@ -781,22 +809,33 @@ static int launch_cg(TcParams &prm, cudaStream_t stream, int num_sms) {
   return (e == cudaSuccess && cudaGetLastError() == cudaSuccess) ? 0 : -1;
 }
 
-// Dynamic tile scheduling counters: a ring of per-launch slots per device,
-// each zeroed by a stream-ordered memset right before its launch.
-static uint32_t *tile_counter(cudaStream_t stream) {
+// Dynamic tile scheduling counters: a ring of per-launch slots per device.
+// A launch makes exactly ntiles + producers claims on its slot (every tile
+// once, then one failing claim per producer), so the host knows the slot's
+// value when the launch is over and passes it as the base of the next launch
+// on that slot -- no memset node per launch.  (A slot is reused only 256
+// launches later, long after its previous launch has drained.)
+struct TileCounter { uint32_t *ctr; uint32_t base; };
+static bool tile_counter(TileCounter &tc, uint32_t claims) {
   constexpr int SLOTS = 256;
   static uint32_t *ring[64] = {};
   static uint32_t next[64] = {};
+  static uint32_t value[64][SLOTS] = {};
   int d = 0;
-  if (cudaGetDevice(&d) != cudaSuccess || d < 0 || d >= 64) return nullptr;
-  if (!ring[d] && cudaMalloc(&ring[d], SLOTS * 32 * sizeof(uint32_t)) != cudaSuccess) {
-    cudaGetLastError();
-    ring[d] = nullptr;
-    return nullptr;
+  if (cudaGetDevice(&d) != cudaSuccess || d < 0 || d >= 64) return false;
+  if (!ring[d]) {
+    if (cudaMalloc(&ring[d], SLOTS * 32 * sizeof(uint32_t)) != cudaSuccess ||
+        cudaMemset(ring[d], 0, SLOTS * 32 * sizeof(uint32_t)) != cudaSuccess) {
+      cudaGetLastError();
+      ring[d] = nullptr;
+      return false;
+    }
   }
-  uint32_t *c = ring[d] + (next[d]++ % SLOTS) * 32;     // 128-B apart
-  if (cudaMemsetAsync(c, 0, sizeof(uint32_t), stream) != cudaSuccess) return nullptr;
-  return c;
+  const uint32_t slot = next[d]++ % SLOTS;
+  tc.ctr = ring[d] + slot * 32;                     // 128-B apart
+  tc.base = value[d][slot];
+  value[d][slot] += claims;                         // wraps mod 2^32 consistently
+  return true;
 }
 
 int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
@@ -813,8 +852,41 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
   const int cg = choose_cg(prm.P, num_sms);
   static int dyn = -1;
   if (dyn < 0) { const char *e = getenv("BLAS3_TC_STATIC"); dyn = (e && e[0] == '1') ? 0 : 1; }
-  if (dyn && !(prm.tile_ctr = tile_counter(stream))) return -1;
-  return cg == 2 ? launch_cg<2>(prm, stream, num_sms) : launch_cg<1>(prm, stream, num_sms);
+  if (dyn) {
+    using G2 = Geo<2>;
+    const int64_t nb = prm.P.nbatch > 1 ? prm.P.nbatch : 1;
+    const int64_t tiles = (cg == 2 ? Tiles<G2::TM, BN>::count(prm.P) : Tiles<Geo<1>::TM, BN>::count(prm.P)) * nb;
+    TileCounter tc;
+    // claims: (tiles - producers) beyond the first wave + one failing claim per producer
+    if (tiles > 0) {
+      if (!tile_counter(tc, (uint32_t)tiles)) return -1;
+      prm.tile_ctr = tc.ctr;
+      prm.tile_base = tc.base;
+    }
+  }
+  // diagnostics: BLAS3_TRACE=1 prints CTA 0's phase timeline (synchronises)
+  static int trace = -1;
+  static unsigned long long *tbuf = nullptr;
+  if (trace < 0) { const char *e = getenv("BLAS3_TRACE"); trace = (e && e[0] == '1') ? 1 : 0; }
+  if (trace) {
+    if (!tbuf && cudaMalloc(&tbuf, 16 * sizeof(unsigned long long)) != cudaSuccess) return -1;
+    cudaMemsetAsync(tbuf, 0, 16 * sizeof(unsigned long long), stream);
+    prm.trace = tbuf;
+  }
+  const int rc = cg == 2 ? launch_cg<2>(prm, stream, num_sms) : launch_cg<1>(prm, stream, num_sms);
+  if (trace && rc == 0) {
+    unsigned long long h[16];
+    cudaStreamSynchronize(stream);
+    cudaMemcpy(h, tbuf, sizeof(h), cudaMemcpyDeviceToHost);
+    static const char *names[12] = {"entry", "prologue", "claim", "tma", "full", "ready",
+                                    "mma", "tfull", "stored", "epi_exit", "final_sync", "dealloc"};
+    fprintf(stderr, "[blas3 trace] cg=%d M=%lld N=%lld K=%lld:", cg, (long long)P0.M,
+            (long long)P0.N, (long long)P0.seg[0].K);
+    for (int i = 1; i < 12; ++i)
+      fprintf(stderr, " %s=%.2f", names[i], h[i] ? (double)(h[i] - h[0]) / 1e3 : -1.0);
+    fprintf(stderr, " us\n");
+  }
+  return rc;
 }
 
 }  // namespace blas3

@@ -78,6 +78,31 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t *bar, uint32_t parity
   while (!mbar_try_wait(bar, parity)) {}
 }
 
+// ------------------------------------------------------------------ epilogue global access
+// Streaming (evict-first) fp32 load/store; the _pred forms are ONE predicated
+// instruction each (no branch / convergence barrier per element).
+__device__ __forceinline__ float ld_cs(const float *p) {
+  float v;
+  asm volatile("ld.global.cs.f32 %0, [%1];" : "=f"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void st_cs(float *p, float v) {
+  asm volatile("st.global.cs.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+}
+__device__ __forceinline__ float ld_cs_pred(const float *p, bool pr) {
+  float v;
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\tmov.b32 %0, 0;\n\t"
+      "@q ld.global.cs.f32 %0, [%1];\n\t}"
+      : "=f"(v) : "l"(p), "r"((int)pr));
+  return v;
+}
+__device__ __forceinline__ void st_cs_pred(float *p, float v, bool pr) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q st.global.cs.f32 [%0], %1;\n\t}"
+      ::"l"(p), "f"(v), "r"((int)pr) : "memory");
+}
+
 // ------------------------------------------------------------------ fences / barriers
 __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
