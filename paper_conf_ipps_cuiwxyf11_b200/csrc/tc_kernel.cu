@@ -73,6 +73,13 @@ constexpr int TMEM_COLS = 512;             // 2 accumulators x BN columns
 constexpr int MAX_MAPS = 8;
 constexpr int LAYOUT_K = 0, LAYOUT_MN = 1;
 
+// A work item: the tile (batch member b, tile t at m0, n0) and the range
+// [g0, g1) of its k-blocks, counted over the concatenated segments.
+struct Work {
+  int64_t tb, b, t, m0, n0, g0, g1;
+  int32_t slice;          // k-slice of a split tile, or -1 for a whole tile
+};
+
 // Two shared-memory rings: a deep RAW ring (TMA destination, read by UMMA as
 // hi) lets TMA run RS k-blocks ahead to hide load latency, and a shallow LO
 // ring (written by the transform) only has to cover transform/MMA overlap.
@@ -97,12 +104,15 @@ struct Geo {
     uint64_t empty[RS];      // MMA -> TMA: raw slot free (tcgen05.commit, multicast)
     uint64_t ready[LS];      // transform -> MMA (one arrival per CTA of the pair, leader)
     uint64_t lo_empty[LS];   // MMA -> transform: lo slot free (tcgen05.commit, multicast)
-    uint64_t tq_full[TQ];    // producer -> roles: tile index published
+    uint64_t tq_full[TQ];    // leader producer -> peer producer: item index published
     uint64_t tq_empty[TQ];   // roles -> leader producer: slot read (3 per CTA; +1 peer producer)
     int64_t tq[TQ];
+    uint64_t wk_full[TQ];    // local producer -> local roles: decoded work item published
+    Work wk[TQ];
     uint64_t tfull[2];       // MMA -> epilogue: TMEM partial ready (multicast to the pair)
     uint64_t tempty[2];      // epilogue -> MMA: partial drained (one arrival per CTA, leader)
     uint32_t tmem_base;
+    uint32_t split_last;     // epilogue: this CTA's slice of a split tile is the last one
   };
   static constexpr size_t SMEM = sizeof(RawBuf) * RS + sizeof(LoBuf) * LS + sizeof(Barriers) + 1024;
 };
@@ -112,6 +122,16 @@ struct TcParams {
   Problem P;
   uint32_t *tile_ctr;      // dynamic tile scheduler counter, or null (static schedule)
   uint32_t tile_base;      // its value when this launch starts
+  // Split tail (wave quantisation): work items [0, khead) are whole tiles; the
+  // last (ntiles - khead) tiles are cut into ksplit k-slices each, item
+  // khead + j -> tile khead + j / ksplit, slice j % ksplit.  Slices write
+  // fp32 partials to ws; the last arriving slice (ws_cnt) reduces them in
+  // slice order and runs the epilogue.
+  int64_t tiles_per;       // tiles of one batch member (Tiles<TM,BN>::count)
+  int64_t nitems, khead;
+  int32_t ksplit;
+  float *ws;
+  uint32_t *ws_cnt;
   unsigned long long *trace;   // phase timestamps of CTA 0 (env BLAS3_TRACE), or null
 };
 
@@ -164,7 +184,7 @@ __device__ __forceinline__ StageInfo stage_info(const Problem &P, const Segment 
 }
 
 template <int CG>
-__device__ __forceinline__ void seg_kblocks(const Problem &P, const Segment &sg, int64_t m0,
+HD void seg_kblocks(const Problem &P, const Segment &sg, int64_t m0,
                                             int64_t n0, int64_t &kb0, int64_t &kb1) {
   int64_t k0, k1;
   k_range(sg, m0, imin(P.M, m0 + Geo<CG>::TM), n0, imin(P.N, n0 + BN), k0, k1);
@@ -173,7 +193,7 @@ __device__ __forceinline__ void seg_kblocks(const Problem &P, const Segment &sg,
 }
 
 template <int CG>
-__device__ __forceinline__ int64_t tile_kblocks(const Problem &P, int64_t m0, int64_t n0) {
+HD int64_t tile_kblocks(const Problem &P, int64_t m0, int64_t n0) {
   int64_t tot = 0;
   for (int s = 0; s < P.nseg; ++s) {
     int64_t a, b;
@@ -181,6 +201,42 @@ __device__ __forceinline__ int64_t tile_kblocks(const Problem &P, int64_t m0, in
     tot += b - a;
   }
   return tot;
+}
+
+template <int CG>
+__device__ __forceinline__ Work work_of(const TcParams &prm, int64_t item, int64_t tiles_per) {
+  const Problem &P = prm.P;
+  Work w;
+  w.slice = -1;
+  w.tb = item;
+  if (item >= prm.khead && prm.ksplit > 1) {
+    const int64_t j = item - prm.khead;
+    w.tb = prm.khead + j / prm.ksplit;
+    w.slice = (int32_t)(j % prm.ksplit);
+  }
+  w.b = w.tb / tiles_per;
+  w.t = w.tb - w.b * tiles_per;
+  int64_t mi, nj;
+  Tiles<Geo<CG>::TM, BN>::coords(P, w.t, mi, nj);
+  w.m0 = mi * Geo<CG>::TM;
+  w.n0 = nj * BN;
+  const int64_t nkb = tile_kblocks<CG>(P, w.m0, w.n0);
+  w.g0 = 0;
+  w.g1 = nkb;
+  if (w.slice >= 0) {
+    w.g0 = nkb * w.slice / prm.ksplit;
+    w.g1 = nkb * (w.slice + 1) / prm.ksplit;
+  }
+  return w;
+}
+// clip a segment's k-blocks [kb0, kb1) to the item's range; gi counts the
+// k-blocks of the earlier segments
+__device__ __forceinline__ void clip_kblocks(const Work &w, int64_t &gi, int64_t &kb0, int64_t &kb1) {
+  const int64_t n = kb1 - kb0;
+  const int64_t lo = imax(0, w.g0 - gi), hi = imin(n, w.g1 - gi);
+  gi += n;
+  kb1 = kb0 + imax(lo, hi);
+  kb0 = kb0 + lo;
 }
 
 // ---------------------------------------------------------------- producer
@@ -318,6 +374,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
       ptx::mbar_init(&bars->lo_empty[s], 1);
     }
     for (int q = 0; q < TQ; ++q) {
+      ptx::mbar_init(&bars->wk_full[q], 1);
       ptx::mbar_init(&bars->tq_full[q], 1);
       ptx::mbar_init(&bars->tq_empty[q], CG == 1 ? 3 : 7);
     }
@@ -335,18 +392,17 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
   if (threadIdx.x == 0) BLAS3_TRACE(1);
 
   // batched problems: tile tb -> batch member b = tb / tiles_per, tile t
-  const int64_t tiles_per = Tiles<TM, BN>::count(P);
+  const int64_t tiles_per = prm.tiles_per;
   const int64_t per = P.per > 0 ? P.per : 1;
-  const int64_t ntiles = tiles_per * (P.nbatch > 0 ? P.nbatch : 1);
-  // consumer side of the tile queue: returns the next tile (or -1 = done);
-  // every thread of the role reads the slot, then one thread releases it.
-  // (for a CTA pair the leader's producer fills both CTAs' queues, and every
-  // role of both CTAs releases the slot at the leader)
-  auto next_tile = [&](uint32_t &qi, uint32_t bar_id, uint32_t nthreads, bool first) -> int64_t {
+  // Tile queue.  The (leader) producer claims work items and publishes them
+  // (to the peer producer too, for a CTA pair); every CTA's producer decodes
+  // its item once (work_of) into wk[slot] for the local roles.  Consumer
+  // side: every thread of a role reads the slot, then one thread releases it
+  // at the leader (all roles of both CTAs, plus the peer producer).
+  auto next_work = [&](uint32_t &qi, uint32_t bar_id, uint32_t nthreads, bool first) -> Work {
     const int slot = qi % TQ;
-    if (CG == 2) ptx::mbar_wait_cluster(&bars->tq_full[slot], (qi / TQ) & 1);
-    else ptx::mbar_wait(&bars->tq_full[slot], (qi / TQ) & 1);
-    const int64_t tb = *reinterpret_cast<volatile int64_t *>(&bars->tq[slot]);
+    ptx::mbar_wait(&bars->wk_full[slot], (qi / TQ) & 1);
+    const Work w = *const_cast<const Work *>(&bars->wk[slot]);
     if (nthreads > 32) ptx::named_bar_sync(bar_id, nthreads);
     else if (nthreads == 32) __syncwarp();
     if (first) {
@@ -354,7 +410,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
       else ptx::mbar_arrive_cluster(&bars->tq_empty[slot], 0);
     }
     ++qi;
-    return tb;
+    return w;
   };
 
   // register rebalancing per warpgroup role (setmaxnreg dominates each role's code)
@@ -371,35 +427,39 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
       uint32_t it = 0;
       for (uint32_t qi = 0;;) {
         int64_t tb;
+        const int slot = qi % TQ;
+        const uint32_t par = (qi / TQ) & 1;
         if (CG == 1 || rank == 0) {
-          // claim a tile (dynamic) or take the static round-robin one
-          // (the first tile of every producer is its own id: no claim round trip)
+          // claim an item (dynamic) or take the static round-robin one
+          // (the first item of every producer is its own id: no claim round trip)
           tb = (prm.tile_ctr == nullptr || qi == 0)
                    ? cid + (int64_t)qi * ncl
                    : ncl + (int64_t)(uint32_t)(atomicAdd(prm.tile_ctr, 1u) - prm.tile_base);
-          if (tb >= ntiles) tb = -1;
+          if (tb >= prm.nitems) tb = -1;
           BLAS3_TRACE(2);
-          const int slot = qi % TQ;
-          if (CG == 2) ptx::mbar_wait_cluster(&bars->tq_empty[slot], ((qi / TQ) & 1) ^ 1);
-          else ptx::mbar_wait(&bars->tq_empty[slot], ((qi / TQ) & 1) ^ 1);
-          *reinterpret_cast<volatile int64_t *>(&bars->tq[slot]) = tb;
+          ptx::mbar_wait(&bars->tq_empty[slot], par ^ 1);
           if (CG == 2) ptx::st_remote_and_arrive(&bars->tq[slot], tb, &bars->tq_full[slot], 1);
-          ptx::mbar_arrive(&bars->tq_full[slot]);
-          ++qi;
-        } else {
-          tb = next_tile(qi, 0, 1, true);             // the pair's peer follows the leader
+        } else {                                      // the pair's peer follows the leader
+          ptx::mbar_wait(&bars->tq_full[slot], par);
+          tb = *reinterpret_cast<volatile int64_t *>(&bars->tq[slot]);
+          ptx::mbar_arrive_cluster(&bars->tq_empty[slot], 0);
         }
+        Work w;
+        if (tb >= 0) w = work_of<CG>(prm, tb, tiles_per);
+        else w.tb = -1;
+        bars->wk[slot] = w;
+        ptx::mbar_arrive(&bars->wk_full[slot]);       // release: local roles see wk[slot]
+        ++qi;
         if (tb < 0) break;
-        const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
-        const int32_t bj = (int32_t)(b % per), bg = (int32_t)(b / per);
-        int64_t mi, nj;
-        Tiles<TM, BN>::coords(P, t, mi, nj);
-        const int64_t m0 = mi * TM, n0 = nj * BN;
+        const int32_t bj = (int32_t)(w.b % per), bg = (int32_t)(w.b / per);
+        const int64_t m0 = w.m0, n0 = w.n0;
         const int64_t ma = m0 + HA * rank, nb = n0 + HB * rank;
+        int64_t gi = 0;
         for (int s = 0; s < P.nseg; ++s) {
           const Segment &sg = P.seg[s];
           int64_t kb0, kb1;
           seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
+          clip_kblocks(w, gi, kb0, kb1);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
             const int rs = it % RS;
             const uint32_t ph = (it / RS) & 1;
@@ -421,17 +481,14 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     // ============================ MMA issuer (leader CTA of the pair only)
     if (rank != 0) {                          // peer CTA: only drain the tile queue
       uint32_t qi = 0;
-      while (next_tile(qi, 0, 32, lane == 0) >= 0) {}
+      while (next_work(qi, 0, 32, lane == 0).tb >= 0) {}
     } else {
       uint32_t it = 0, cc = 0, qi = 0;          // k-block, TMEM-chunk, tile-queue counters
       for (;;) {
-        const int64_t tb = next_tile(qi, 0, 32, lane == 0);
-        if (tb < 0) break;
-        const int64_t t = tb % tiles_per;
-        int64_t mi, nj;
-        Tiles<TM, BN>::coords(P, t, mi, nj);
-        const int64_t m0 = mi * TM, n0 = nj * BN;
-        const int64_t nkb = tile_kblocks<CG>(P, m0, n0);
+        const Work w = next_work(qi, 0, 32, lane == 0);
+        if (w.tb < 0) break;
+        const int64_t m0 = w.m0, n0 = w.n0;
+        const int64_t nkb = w.g1 - w.g0;
         int64_t done = 0;
         uint32_t accumulate = 0, buf = 0;
         auto open_chunk = [&]() {
@@ -456,10 +513,12 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           ++cc;
         };
         if (nkb == 0) { open_chunk(); close_chunk(false); continue; }
+        int64_t gi = 0;
         for (int s = 0; s < P.nseg; ++s) {
           const Segment &sg = P.seg[s];
           int64_t kb0, kb1;
           seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
+          clip_kblocks(w, gi, kb0, kb1);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
             if (done % KC == 0) open_chunk();
             const uint32_t d_tmem = tmem + buf * BN;
@@ -513,17 +572,16 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     const int tt = threadIdx.x - WARP_TR0 * 32;
     uint32_t it = 0, qi = 0;
     for (;;) {
-      const int64_t tb = next_tile(qi, 4, TR_THREADS, tt == 0);
-      if (tb < 0) break;
-      const int64_t t = tb % tiles_per;
-      int64_t mi, nj;
-      Tiles<TM, BN>::coords(P, t, mi, nj);
-      const int64_t m0 = mi * TM, n0 = nj * BN;
+      const Work w = next_work(qi, 4, TR_THREADS, tt == 0);
+      if (w.tb < 0) break;
+      const int64_t m0 = w.m0, n0 = w.n0;
       const int64_t ma = m0 + HA * rank, nb = n0 + HB * rank;
+      int64_t gi = 0;
       for (int s = 0; s < P.nseg; ++s) {
         const Segment &sg = P.seg[s];
         int64_t kb0, kb1;
         seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
+        clip_kblocks(w, gi, kb0, kb1);
         for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
           const int rs = it % RS, ls = it % LS;
           const uint32_t ph = (it / RS) & 1, lph = (it / LS) & 1;
@@ -572,14 +630,11 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     constexpr int NG = BN / 2 / EC;             // column groups per thread (8)
     uint32_t cc = 0, qi = 0;
     for (;;) {
-      const int64_t tb = next_tile(qi, 5, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
-      if (tb < 0) break;
-      const int64_t b = tb / tiles_per, t = tb - b * tiles_per;
-      const int64_t coff = (P.nbatch > 1) ? batch_off(P.bs_c, b, per) : 0;
-      int64_t mi, nj;
-      Tiles<TM, BN>::coords(P, t, mi, nj);
-      const int64_t m0 = mi * TM, n0 = nj * BN;
-      const int64_t nkb = tile_kblocks<CG>(P, m0, n0);
+      const Work w = next_work(qi, 5, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
+      if (w.tb < 0) break;
+      const int64_t coff = (P.nbatch > 1) ? batch_off(P.bs_c, w.b, per) : 0;
+      const int64_t m0 = w.m0, n0 = w.n0;
+      const int64_t nkb = w.g1 - w.g0;
       const int64_t nchunks = nkb > 0 ? cdiv(nkb, KC) : 1;
       float S[NG * EC];
 #pragma unroll
@@ -602,6 +657,37 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
         }
         ptx::tc_fence_before();
         arrive_leader<CG>(&bars->tempty[buf], rank, 3, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
+      }
+      if (w.slice >= 0) {
+        // k-slice of a split tile: publish the partial (this CTA's 128 rows,
+        // column-major, coalesced), count the arrival; the last slice sums all
+        // partials in slice order (deterministic) and continues to the stores
+        const int64_t tt = w.tb - prm.khead;
+        const int64_t slab = (int64_t)HA * BN;                       // floats per CTA slice
+        const int64_t row = q * 32 + lane, col0 = half * (BN / 2);
+        float *mine = prm.ws + ((tt * prm.ksplit + w.slice) * CG + rank) * slab + col0 * HA + row;
+#pragma unroll
+        for (int i = 0; i < NG * EC; ++i) __stcg(mine + i * HA, S[i]);
+        __threadfence();
+        ptx::named_bar_sync(5, EPI_THREADS);
+        if (threadIdx.x == WARP_EPI0 * 32) {
+          uint32_t *cnt = prm.ws_cnt + tt * CG + rank;
+          const uint32_t old = atomicAdd(cnt, 1u);
+          const uint32_t last = (old == (uint32_t)prm.ksplit - 1) ? 1u : 0u;
+          if (last) *cnt = 0u;                                     // self-cleaning for the next launch
+          bars->split_last = last;
+        }
+        ptx::named_bar_sync(5, EPI_THREADS);
+        if (!bars->split_last) continue;
+        __threadfence();
+        const float *part = prm.ws + (tt * prm.ksplit * CG + rank) * slab + col0 * HA + row;
+#pragma unroll
+        for (int i = 0; i < NG * EC; ++i) S[i] = 0.f;
+        for (int sl = 0; sl < prm.ksplit; ++sl) {
+          const float *ps = part + (int64_t)sl * CG * slab;
+#pragma unroll
+          for (int i = 0; i < NG * EC; ++i) S[i] += __ldcg(ps + i * HA);
+        }
       }
       // ---- store phase: D = alpha*S + beta*C for row r, columns cbase + [0,128).
       // The valid columns of the row form one range [jlo, jhi) (column bound
@@ -789,9 +875,9 @@ static int launch_cg(TcParams &prm, cudaStream_t stream, int num_sms) {
                              (int)G::SMEM) != cudaSuccess) return -1;
     attr = true;
   }
-  const int64_t tiles = Tiles<G::TM, BN>::count(prm.P) * (prm.P.nbatch > 1 ? prm.P.nbatch : 1);
-  if (tiles == 0) return 0;
-  const int64_t units = imin(tiles, (int64_t)(num_sms / CG));      // CTAs (CG=1) or pairs
+  const int64_t items = prm.nitems;        // tiles, or tiles + split-tail slices
+  if (items == 0) return 0;
+  const int64_t units = imin(items, (int64_t)(num_sms / CG));      // CTAs (CG=1) or pairs
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)(units * CG));
   cfg.blockDim = dim3(NTHREADS);
@@ -838,6 +924,66 @@ static bool tile_counter(TileCounter &tc, uint32_t claims) {
   return true;
 }
 
+// Split-tail workspace, one per (device, stream): the slices of one launch's
+// tail never exceed one wave (num_sms CTAs x 128 x BN floats), counters are
+// left at zero by the last slice of every tile.
+static bool split_workspace(cudaStream_t stream, int num_sms, float **ws, uint32_t **cnt) {
+  struct Entry { int dev; cudaStream_t st; float *ws; uint32_t *cnt; };
+  static Entry tab[16];
+  static int n = 0;
+  int d = 0;
+  if (cudaGetDevice(&d) != cudaSuccess) return false;
+  for (int i = 0; i < n; ++i)
+    if (tab[i].dev == d && tab[i].st == stream) { *ws = tab[i].ws; *cnt = tab[i].cnt; return true; }
+  if (n == 16) return false;
+  Entry e{d, stream, nullptr, nullptr};
+  const size_t wsb = (size_t)num_sms * HA * BN * sizeof(float), cb = 1024 * sizeof(uint32_t);
+  if (cudaMalloc(&e.ws, wsb) != cudaSuccess) { cudaGetLastError(); return false; }
+  if (cudaMalloc(&e.cnt, cb) != cudaSuccess || cudaMemset(e.cnt, 0, cb) != cudaSuccess) {
+    cudaGetLastError(); cudaFree(e.ws); return false;
+  }
+  tab[n++] = e;
+  *ws = e.ws; *cnt = e.cnt;
+  return true;
+}
+
+// Wave quantisation: with T tiles on U producers the last wave holds
+// R = T mod U tiles (all T when T < U) and leaves U - R producers idle.
+// Those R tiles are cut into S = U / R k-slices.  Only worth it while the
+// tail is a sizeable share of the launch (fewer than 8 waves) and each slice
+// keeps >= 8 k-blocks (its partial write-back costs about what ~3 k-blocks
+// of MMA do).
+template <int CG>
+static void plan_split(TcParams &prm, int num_sms, cudaStream_t stream) {
+  const Problem &P = prm.P;
+  const int64_t nb = P.nbatch > 1 ? P.nbatch : 1;
+  const int64_t tiles_per = Tiles<Geo<CG>::TM, BN>::count(P), T = tiles_per * nb;
+  prm.tiles_per = tiles_per;
+  prm.nitems = T; prm.khead = T; prm.ksplit = 1;
+  static int enabled = -1;
+  if (enabled < 0) { const char *e = getenv("BLAS3_TC_SPLIT"); enabled = (e && e[0] == '0') ? 0 : 1; }
+  if (!enabled || T == 0) return;
+  const int64_t U = imin(T, (int64_t)(num_sms / CG));
+  const int64_t R = T < (int64_t)(num_sms / CG) ? T : T % U;
+  if (R == 0 || T >= 8 * U) return;
+  int64_t S = imin((int64_t)(num_sms / CG) / R, 16);
+  if (S < 2) return;
+  const int64_t head = T - R;
+  int64_t min_kb = INT64_MAX;
+  for (int64_t tb = head; tb < T; ++tb) {
+    const int64_t t = tb % tiles_per;
+    int64_t mi, nj;
+    Tiles<Geo<CG>::TM, BN>::coords(P, t, mi, nj);
+    min_kb = imin(min_kb, tile_kblocks<CG>(P, mi * Geo<CG>::TM, nj * BN));
+  }
+  S = imin(S, min_kb / 8);
+  if (S < 2) return;
+  if (!split_workspace(stream, num_sms, &prm.ws, &prm.ws_cnt)) return;
+  prm.khead = head;
+  prm.ksplit = (int32_t)S;
+  prm.nitems = head + R * S;
+}
+
 int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
   static TcParams prm;                    // host staging (the launch copies it)
   static std::mutex mu;
@@ -852,12 +998,11 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
   const int cg = choose_cg(prm.P, num_sms);
   static int dyn = -1;
   if (dyn < 0) { const char *e = getenv("BLAS3_TC_STATIC"); dyn = (e && e[0] == '1') ? 0 : 1; }
+  if (cg == 2) plan_split<2>(prm, num_sms, stream); else plan_split<1>(prm, num_sms, stream);
   if (dyn) {
-    using G2 = Geo<2>;
-    const int64_t nb = prm.P.nbatch > 1 ? prm.P.nbatch : 1;
-    const int64_t tiles = (cg == 2 ? Tiles<G2::TM, BN>::count(prm.P) : Tiles<Geo<1>::TM, BN>::count(prm.P)) * nb;
+    const int64_t tiles = prm.nitems;
     TileCounter tc;
-    // claims: (tiles - producers) beyond the first wave + one failing claim per producer
+    // claims: (items - producers) beyond the first wave + one failing claim per producer
     if (tiles > 0) {
       if (!tile_counter(tc, (uint32_t)tiles)) return -1;
       prm.tile_ctr = tc.ctr;

@@ -1,8 +1,9 @@
 """The opt-in kernel variants selected by environment variables at library
 load (they are cached once per process, hence subprocesses): the CTA-pair
 tcgen05 kernel (BLAS3_TC_CTA=2, cta_group::2) and the static tile schedule
-(BLAS3_TC_STATIC=1), and the single-CTA kernel (BLAS3_TC_CTA=1; the default
-picks the pair kernel for large problems).  Each child process runs a representative subset of the
+(BLAS3_TC_STATIC=1), the single-CTA kernel (BLAS3_TC_CTA=1; the default
+picks the pair kernel for large problems), and whole tiles only
+(BLAS3_TC_SPLIT=0: no k-sliced tail).  Each child process runs a representative subset of the
 parity suite (every routine family, both transposes/sides) on that variant."""
 import os
 import subprocess
@@ -14,8 +15,9 @@ pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-@pytest.mark.parametrize("env", [{"BLAS3_TC_CTA": "1"}, {"BLAS3_TC_CTA": "2"}, {"BLAS3_TC_STATIC": "1"}],
-                         ids=["single_cta", "cta_pair", "static_schedule"])
+@pytest.mark.parametrize("env", [{"BLAS3_TC_CTA": "1"}, {"BLAS3_TC_CTA": "2"}, {"BLAS3_TC_STATIC": "1"},
+                                 {"BLAS3_TC_SPLIT": "0"}, {"BLAS3_TC_CTA": "1", "BLAS3_TC_SPLIT": "0"}],
+                         ids=["single_cta", "cta_pair", "static_schedule", "no_split", "single_cta_no_split"])
 def test_variant_subset(env):
     import torch
     if not torch.cuda.is_available():
