@@ -71,7 +71,8 @@ struct Problem {
   BatchStride bs_a, bs_b, bs_c;
   // performance-experiment knobs (env BLAS3_DEBUG_TC; results are WRONG when
   // set, never used by tests or the bench): bit0 skip the split pass,
-  // bit1 issue only hi*hi (1xTF32), bit2 skip the epilogue stores
+  // bit1 issue only hi*hi (1xTF32), bit2 skip the epilogue stores,
+  // bit3 issue no MMAs (commits only), bit4 issue no TMA loads
   int32_t dbg;
 };
 

@@ -183,6 +183,15 @@ __device__ __forceinline__ StageInfo stage_info(const Problem &P, const Segment 
   return si;
 }
 
+// StageInfo of a segment whose operands are both dense is the same for every
+// k-block (classes RK/KR fixed by the views): computed once per segment.
+template <int CG>
+__device__ __forceinline__ StageInfo stage_info_at(const Problem &P, const Segment &sg, int64_t m0,
+                                                   int64_t n0, int64_t k0, bool dense,
+                                                   const StageInfo &si0) {
+  return dense ? si0 : stage_info<CG>(P, sg, m0, n0, k0);
+}
+
 template <int CG>
 HD void seg_kblocks(const Problem &P, const Segment &sg, int64_t m0,
                                             int64_t n0, int64_t &kb0, int64_t &kb1) {
@@ -460,12 +469,16 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           int64_t kb0, kb1;
           seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
           clip_kblocks(w, gi, kb0, kb1);
+          const bool dense = sg.a.kind == OP_DENSE && sg.b.kind == OP_DENSE;
+          StageInfo si0{};
+          if (dense) si0 = stage_info<CG>(P, sg, m0, n0, 0);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
             const int rs = it % RS;
             const uint32_t ph = (it / RS) & 1;
             const int64_t k0 = kb * BK;
-            const StageInfo si = stage_info<CG>(P, sg, m0, n0, k0);
+            const StageInfo si = stage_info_at<CG>(P, sg, m0, n0, k0, dense, si0);
             ptx::mbar_wait(&bars->empty[rs], ph ^ 1);
+            if (P.dbg & 16) { ptx::mbar_arrive(&bars->full[rs]); continue; }   // diag: no loads
             ptx::mbar_arrive_expect_tx(&bars->full[rs], (HA + HB) * BK * 4);
             load_operand(prm, sg.a, si.layA, raw[rs].A, ma, k0, HA, &bars->full[rs], bj, bg);
             load_operand(prm, sg.b, si.layB, raw[rs].B, nb, k0, HB, &bars->full[rs], bj, bg);
@@ -519,12 +532,15 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           int64_t kb0, kb1;
           seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
           clip_kblocks(w, gi, kb0, kb1);
+          const bool dense = sg.a.kind == OP_DENSE && sg.b.kind == OP_DENSE;
+          StageInfo si0{};
+          if (dense) si0 = stage_info<CG>(P, sg, m0, n0, 0);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
             if (done % KC == 0) open_chunk();
             const uint32_t d_tmem = tmem + buf * BN;
             const int rs = it % RS, ls = it % LS;
             const uint32_t lph = (it / LS) & 1;
-            const StageInfo si = stage_info<CG>(P, sg, m0, n0, kb * BK);
+            const StageInfo si = stage_info_at<CG>(P, sg, m0, n0, kb * BK, dense, si0);
             if (CG == 2) ptx::mbar_wait_cluster(&bars->ready[ls], lph);
             else ptx::mbar_wait(&bars->ready[ls], lph);
             ptx::tc_fence_after();
@@ -537,6 +553,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
                 const uint64_t ah = op_desc(hiA, si.layA, k8), al = op_desc(loA, si.layA, k8);
                 const uint64_t bh = op_desc(hiB, si.layB, k8), bl = op_desc(loB, si.layB, k8);
                 const bool one = P.dbg & 2;
+                if (P.dbg & 8) continue;                       // diag: no MMAs
                 if constexpr (CG == 1) {
                   if (!one) ptx::mma_tf32_ss(d_tmem, al, bh, idesc, accumulate);
                   if (!one) ptx::mma_tf32_ss(d_tmem, ah, bl, idesc, 1);
@@ -582,11 +599,14 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
         int64_t kb0, kb1;
         seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
         clip_kblocks(w, gi, kb0, kb1);
+        const bool dense = sg.a.kind == OP_DENSE && sg.b.kind == OP_DENSE;
+        StageInfo si0{};
+        if (dense) si0 = stage_info<CG>(P, sg, m0, n0, 0);
         for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
           const int rs = it % RS, ls = it % LS;
           const uint32_t ph = (it / RS) & 1, lph = (it / LS) & 1;
           const int64_t k0 = kb * BK;
-          const StageInfo si = stage_info<CG>(P, sg, m0, n0, k0);
+          const StageInfo si = stage_info_at<CG>(P, sg, m0, n0, k0, dense, si0);
           ptx::mbar_wait(&bars->full[rs], ph);
           if (tt == 0) BLAS3_TRACE(4);
           RawBuf &rb = raw[rs];

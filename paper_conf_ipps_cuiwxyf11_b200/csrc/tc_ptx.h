@@ -38,8 +38,16 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t *bar, uint32_t parity) {
       : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
   return ok != 0;
 }
+// The whole poll loop is one PTX block (labels are scoped to it), so no
+// spill/reload code can be scheduled inside it: idle roles spin on the
+// try_wait alone (which suspends the warp for a while per attempt).
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
-  while (!mbar_try_wait(bar, parity)) {}
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "BLAS3_WAIT:\n\t"
+      "mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra BLAS3_WAIT;\n\t}"
+      ::"r"(smem_u32(bar)), "r"(parity) : "memory");
 }
 
 // ------------------------------------------------------------------ clusters (CTA pairs)
