@@ -183,13 +183,41 @@ __device__ __forceinline__ StageInfo stage_info(const Problem &P, const Segment 
   return si;
 }
 
-// StageInfo of a segment whose operands are both dense is the same for every
-// k-block (classes RK/KR fixed by the views): computed once per segment.
+// An operand's block class can only change on the k-blocks that intersect
+// its rows [r0, r1) (the diagonal band); below and above the band it is
+// constant (SYM: rk / kr view; TRI: nonzero / blank).  So per segment the
+// band (hull over both operands) and the two outer StageInfos are computed
+// once, and stage_info runs per k-block only inside the band (dense
+// operands have no band at all).
+struct StageBand {
+  int64_t b0, b1;
+  StageInfo lo, hi;
+};
 template <int CG>
-__device__ __forceinline__ StageInfo stage_info_at(const Problem &P, const Segment &sg, int64_t m0,
-                                                   int64_t n0, int64_t k0, bool dense,
-                                                   const StageInfo &si0) {
-  return dense ? si0 : stage_info<CG>(P, sg, m0, n0, k0);
+__device__ __forceinline__ StageBand make_band(const Problem &P, const Segment &sg, int64_t m0,
+                                               int64_t n0) {
+  StageBand bd;
+  bd.b0 = INT64_MAX;
+  bd.b1 = INT64_MIN;
+  if (sg.a.kind != OP_DENSE) {
+    bd.b0 = imin(bd.b0, m0 / BK);
+    bd.b1 = imax(bd.b1, cdiv(imin(P.M, m0 + Geo<CG>::TM), BK));
+  }
+  if (sg.b.kind != OP_DENSE) {
+    bd.b0 = imin(bd.b0, n0 / BK);
+    bd.b1 = imax(bd.b1, cdiv(imin(P.N, n0 + BN), BK));
+  }
+  if (bd.b1 < bd.b0) bd.b0 = bd.b1 = 0;           // both dense: one class everywhere
+  bd.lo = stage_info<CG>(P, sg, m0, n0, imax(0, bd.b0 - 1) * BK);
+  bd.hi = stage_info<CG>(P, sg, m0, n0, imin(imax(0, cdiv(sg.K, BK) - 1), bd.b1) * BK);
+  return bd;
+}
+template <int CG>
+__device__ __forceinline__ StageInfo stage_at(const StageBand &bd, const Problem &P, const Segment &sg,
+                                              int64_t m0, int64_t n0, int64_t kb) {
+  if (kb < bd.b0) return bd.lo;
+  if (kb >= bd.b1) return bd.hi;
+  return stage_info<CG>(P, sg, m0, n0, kb * BK);
 }
 
 template <int CG>
@@ -469,14 +497,12 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           int64_t kb0, kb1;
           seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
           clip_kblocks(w, gi, kb0, kb1);
-          const bool dense = sg.a.kind == OP_DENSE && sg.b.kind == OP_DENSE;
-          StageInfo si0{};
-          if (dense) si0 = stage_info<CG>(P, sg, m0, n0, 0);
+          const StageBand bd = make_band<CG>(P, sg, m0, n0);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
             const int rs = it % RS;
             const uint32_t ph = (it / RS) & 1;
             const int64_t k0 = kb * BK;
-            const StageInfo si = stage_info_at<CG>(P, sg, m0, n0, k0, dense, si0);
+            const StageInfo si = stage_at<CG>(bd, P, sg, m0, n0, kb);
             ptx::mbar_wait(&bars->empty[rs], ph ^ 1);
             if (P.dbg & 16) { ptx::mbar_arrive(&bars->full[rs]); continue; }   // diag: no loads
             ptx::mbar_arrive_expect_tx(&bars->full[rs], (HA + HB) * BK * 4);
@@ -532,15 +558,13 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           int64_t kb0, kb1;
           seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
           clip_kblocks(w, gi, kb0, kb1);
-          const bool dense = sg.a.kind == OP_DENSE && sg.b.kind == OP_DENSE;
-          StageInfo si0{};
-          if (dense) si0 = stage_info<CG>(P, sg, m0, n0, 0);
+          const StageBand bd = make_band<CG>(P, sg, m0, n0);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
             if (done % KC == 0) open_chunk();
             const uint32_t d_tmem = tmem + buf * BN;
             const int rs = it % RS, ls = it % LS;
             const uint32_t lph = (it / LS) & 1;
-            const StageInfo si = stage_info_at<CG>(P, sg, m0, n0, kb * BK, dense, si0);
+            const StageInfo si = stage_at<CG>(bd, P, sg, m0, n0, kb);
             if (CG == 2) ptx::mbar_wait_cluster(&bars->ready[ls], lph);
             else ptx::mbar_wait(&bars->ready[ls], lph);
             ptx::tc_fence_after();
@@ -599,14 +623,12 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
         int64_t kb0, kb1;
         seg_kblocks<CG>(P, sg, m0, n0, kb0, kb1);
         clip_kblocks(w, gi, kb0, kb1);
-        const bool dense = sg.a.kind == OP_DENSE && sg.b.kind == OP_DENSE;
-        StageInfo si0{};
-        if (dense) si0 = stage_info<CG>(P, sg, m0, n0, 0);
+        const StageBand bd = make_band<CG>(P, sg, m0, n0);
         for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
           const int rs = it % RS, ls = it % LS;
           const uint32_t ph = (it / RS) & 1, lph = (it / LS) & 1;
           const int64_t k0 = kb * BK;
-          const StageInfo si = stage_info_at<CG>(P, sg, m0, n0, k0, dense, si0);
+          const StageInfo si = stage_at<CG>(bd, P, sg, m0, n0, kb);
           ptx::mbar_wait(&bars->full[rs], ph);
           if (tt == 0) BLAS3_TRACE(4);
           RawBuf &rb = raw[rs];
