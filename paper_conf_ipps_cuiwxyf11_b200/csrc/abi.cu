@@ -95,6 +95,10 @@ static OpDesc tri(const float *p, int64_t ld, bool lower, bool swap, bool unit) 
   OpDesc o = dense(p, ld, false); o.kind = OP_TRI; o.lower = lower; o.swap = swap; o.unit = unit;
   return o;
 }
+// a TRI operand in library workspace whose blank triangle holds zeros
+static OpDesc tri_zeroed(const float *p, int64_t ld, bool lower, bool swap) {
+  OpDesc o = tri(p, ld, lower, swap, false); o.zero_blank = 1; return o;
+}
 static Problem problem(int64_t M, int64_t N, float alpha, float beta, const float *Cin,
                        int64_t ldcin, float *Cout, int64_t ldcout) {
   Problem P; memset(&P, 0, sizeof(P));
@@ -372,7 +376,7 @@ static int trsm_panel_inverses(const float *A, int64_t lda, int64_t nt, bool low
       // T = L21 * inv(L11): Xa = L21 (m2 x sz), Xb(c,k) = inv(L11)(k,c) (lower -> TRI swap)
       Problem P1 = problem(m2, sz, 1.f, 0.f, nullptr, 0, Tw, m2);
       P1.seg[0].a = dense(l21(o), lda, !lower);
-      P1.seg[0].b = tri(dblk(o), NBO, true, true, false);
+      P1.seg[0].b = tri_zeroed(dblk(o), NBO, true, true);
       P1.seg[0].K = sz;
       P1.nbatch = cnt; P1.per = per;
       P1.bs_a = {per * 2 * sz * (1 + lda), 2 * sz * (1 + lda)};
@@ -381,7 +385,7 @@ static int trsm_panel_inverses(const float *A, int64_t lda, int64_t nt, bool low
       if ((rc = run_problem(P1, s, sms))) return rc;
       // X21 = -inv(L22) * T: Xa = inv(L22) (lower TRI), Xb(c,k) = T(k,c) (kr)
       Problem P2 = problem(m2, sz, -1.f, 0.f, nullptr, 0, dblk(o) + sz, NBO);
-      P2.seg[0].a = tri(dblk(o) + sz * (1 + NBO), NBO, true, false, false);
+      P2.seg[0].a = tri_zeroed(dblk(o) + sz * (1 + NBO), NBO, true, false);
       P2.seg[0].b = dense(Tw, m2, true);
       P2.seg[0].K = m2;
       P2.nbatch = cnt; P2.per = per;
@@ -450,7 +454,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
         // X_p = a1 * inv(op(A)_pp) * B_p: Xa(r,k) = Dop(r,k), Dop = lower_op ? D : D^T
         Problem P = in_w ? problem(pr, n, a1, 0.f, nullptr, 0, B + p0, ldb)
                          : problem(pr, n, a1, 0.f, nullptr, 0, W.p, pr);
-        P.seg[0].a = tri(Dp, NBO, true, !lower_op, false);
+        P.seg[0].a = tri_zeroed(Dp, NBO, true, !lower_op);
         P.seg[0].b = in_w ? dense(W.p, pr, true) : dense(B + p0, ldb, true);
         P.seg[0].K = pr;
         P.rev_m = tri_kle(P.seg[0].a);
@@ -462,7 +466,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
         Problem P = in_w ? problem(m, pr, a1, 0.f, nullptr, 0, B + p0 * ldb, ldb)
                          : problem(m, pr, a1, 0.f, nullptr, 0, W.p, m);
         P.seg[0].a = in_w ? dense(W.p, m, false) : dense(B + p0 * ldb, ldb, false);
-        P.seg[0].b = tri(Dp, NBO, true, lower_op, false);
+        P.seg[0].b = tri_zeroed(Dp, NBO, true, lower_op);
         P.seg[0].K = pr;
         P.rev_n = tri_kle(P.seg[0].b);
         P.outer = 2;

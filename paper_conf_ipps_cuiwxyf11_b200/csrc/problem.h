@@ -36,7 +36,9 @@ struct OpDesc {
   int32_t unit;    // TRI: unit diagonal (stored diagonal not read)
   int32_t map_rk;  // tcgen05 path: tensor-map slot of the rk view (-1: none)
   int32_t map_kr;  // tcgen05 path: tensor-map slot of the kr view (-1: none)
-  int32_t pad_;
+  int32_t zero_blank;  // TRI (not unit): the blank triangle is stored as zeros (library
+                       // workspace, e.g. the TRSM inverse panels) -> the k-range is still
+                       // clipped, but diagonal blocks load as plain blocks (no zero-select)
 };
 
 struct Segment {
@@ -185,7 +187,7 @@ HD int32_t block_class(const OpDesc &o, int64_t r0, int64_t r1, int64_t k0, int6
   bool full = kle ? (k1 - 1 < r0) : (k0 > r1 - 1);
   bool blank = kle ? (k0 > r1 - 1) : (k1 - 1 < r0);
   if (blank) return BLK_ZERO;
-  if (full) return o.swap ? BLK_KR : BLK_RK;
+  if (full || (o.zero_blank && !o.unit)) return o.swap ? BLK_KR : BLK_RK;
   return BLK_TRI_DIAG;
 }
 
