@@ -78,6 +78,7 @@ static int get_scratch(Scratch &sc, size_t bytes, cudaStream_t s, size_t offset 
 
 static int run_problem(const Problem &P, cudaStream_t s, int sms) {
   if (P.M <= 0 || P.N <= 0) return 0;
+  if (P.max_sms > 0 && P.max_sms < sms) sms = P.max_sms;
   if (math_mode() == BLAS3_MATH_3XTF32 && tc_eligible(P)) return launch_tc(P, s, sms);
   int rc = launch_simt(P, s, sms);
   return rc ? BLAS3_ERR_CUDA : 0;
@@ -325,12 +326,14 @@ int blas3_strmm(char side, char uplo, char transa, char diag, int64_t m, int64_t
     P.seg[0].a = tri(A, lda, lower, ta, unit);
     P.seg[0].b = dense(B, ldb, true);
     P.seg[0].K = m;
-    P.rev_m = tri_kle(P.seg[0].a);        // longest k-ranges first
+    P.rev_m = tri_kle(P.seg[0].a);        // longest k-ranges first:
+    P.outer = 1;                          // whole m-rows in turn (LPT)
   } else {        // Xa = B ; Xb(c,k) = op(T)(k,c) -> swap = !trans
     P.seg[0].a = dense(B, ldb, false);
     P.seg[0].b = tri(A, lda, lower, !ta, unit);
     P.seg[0].K = n;
     P.rev_n = tri_kle(P.seg[0].b);
+    P.outer = 2;
   }
   if ((rc = run_problem(P, s, sms))) return rc;
   if (launch_copy(B, ldb, W.p, m, m, n, s)) return BLAS3_ERR_CUDA;
@@ -352,15 +355,30 @@ int blas3_strmm(char side, char uplo, char transa, char diag, int64_t m, int64_t
 //      a single panel is X_p = alpha_p * inv(op(A)_pp) * B_p (TRI operand).
 //      alpha is folded into the first operation that touches each row.
 // Every flop of steps 2-3 runs in the structured GEMM kernels.
-static const int64_t NBO = 2048;   // panel width (multiple of the 128 diagonal block)
+// panel width (a power of two >= 128, the diagonal block); env BLAS3_TRSM_NB
+// overrides it for experiments (tests/bench use the default)
+static int64_t trsm_nbo() {
+  static int64_t nb = -1;
+  if (nb < 0) {
+    const char *e = getenv("BLAS3_TRSM_NB");
+    const int64_t v = e ? atoll(e) : 0;
+    nb = (v >= 128 && v <= 8192 && (v & (v - 1)) == 0) ? v : 2048;
+  }
+  return nb;
+}
 
-static int trsm_panel_inverses(const float *A, int64_t lda, int64_t nt, bool lower, bool unit,
-                               float *D, float *Tw, cudaStream_t s, int sms) {
+// Doubling levels 128 -> NBO for the panels of the order-nt triangle whose
+// top-left corner is A (and whose panel inverses start at D); the 128-block
+// inverses are already on D's diagonal.  Tw: (nt / 2sz) x sz^2 floats.
+static int trsm_panel_doubling(const float *A, int64_t lda, int64_t nt, bool lower, float *D,
+                               float *Tw, cudaStream_t s, int sms, cudaEvent_t *ev_lvl) {
+  const int64_t NBO = trsm_nbo();
   int rc;
-  if (cudaMemsetAsync(D, 0, (size_t)cdiv(nt, NBO) * NBO * NBO * sizeof(float), s) != cudaSuccess)
-    return BLAS3_ERR_CUDA;
-  if (launch_trsm_diag_inv(A, lda, nt, lower, unit, D, NBO, s)) return BLAS3_ERR_CUDA;
-  for (int64_t sz = 128; sz < NBO; sz *= 2) {
+  for (int64_t sz = 128, lvl = 0; sz < NBO; sz *= 2, ++lvl) {
+    if (sz >= nt) {                    // no pair reaches this level: nothing left to do
+      if (cudaEventRecord(ev_lvl[lvl], s) != cudaSuccess) return BLAS3_ERR_CUDA;
+      continue;
+    }
     // pair b covers rows/cols [o, o + 2 sz) of L, o = 2 sz b; L21 = L[o+sz.., o..]
     const int64_t per = NBO / (2 * sz);
     const int64_t full = nt / (2 * sz);                    // pairs entirely inside L
@@ -394,8 +412,84 @@ static int trsm_panel_inverses(const float *A, int64_t lda, int64_t nt, bool low
       P2.bs_c = {NBO * NBO, 2 * sz * (1 + NBO)};
       if ((rc = run_problem(P2, s, sms))) return rc;
     }
+    // inverses of every aligned 2sz-block are complete
+    if (cudaEventRecord(ev_lvl[lvl], s) != cudaSuccess) return BLAS3_ERR_CUDA;
   }
   return 0;
+}
+
+// Side streams of the STRSM driver, per device, created once: one for the
+// panel-inverse doubling of all but the first panel, and up to MAX_SLABS for
+// the per-slab sweeps.  Fork/join is event-based, so the call stays
+// asynchronous (and graph-capturable) on the caller's stream.
+constexpr int MAX_SLABS = 4, MAX_LEVELS = 8;
+struct TrsmStreams {
+  cudaStream_t side, side2, slab[MAX_SLABS];
+  cudaEvent_t ev_fork, ev_lvl[MAX_LEVELS], ev_lvl2[MAX_LEVELS], ev_join[MAX_SLABS];
+};
+static std::mutex g_trsm_mu;
+static TrsmStreams *trsm_streams() {
+  static TrsmStreams tab[64];
+  static bool made[64] = {};
+  int d = 0;
+  if (cudaGetDevice(&d) != cudaSuccess || d < 0 || d >= 64) return nullptr;
+  TrsmStreams &t = tab[d];
+  if (!made[d]) {
+    const unsigned fl = cudaEventDisableTiming;
+    // the doubling chain is latency-bound and on the critical path: its
+    // kernels get SMs before the sweep's (highest stream priority)
+    int lo_pri = 0, hi_pri = 0;
+    if (cudaDeviceGetStreamPriorityRange(&lo_pri, &hi_pri) != cudaSuccess) return nullptr;
+    if (cudaStreamCreateWithPriority(&t.side, cudaStreamNonBlocking, hi_pri) != cudaSuccess) return nullptr;
+    if (cudaStreamCreateWithPriority(&t.side2, cudaStreamNonBlocking, lo_pri) != cudaSuccess) return nullptr;
+    for (int i = 0; i < MAX_LEVELS; ++i)
+      if (cudaEventCreateWithFlags(&t.ev_lvl[i], fl) != cudaSuccess ||
+          cudaEventCreateWithFlags(&t.ev_lvl2[i], fl) != cudaSuccess) return nullptr;
+    for (int i = 0; i < MAX_SLABS; ++i) {
+      if (cudaStreamCreateWithFlags(&t.slab[i], cudaStreamNonBlocking) != cudaSuccess ||
+          cudaEventCreateWithFlags(&t.ev_join[i], fl) != cudaSuccess) return nullptr;
+    }
+    if (cudaEventCreateWithFlags(&t.ev_fork, fl) != cudaSuccess) return nullptr;
+    made[d] = true;
+  }
+  return &t;
+}
+// number of right-hand-side slabs: slabs of >= 2048 columns (rows), at most
+// 2; env BLAS3_TRSM_SLABS / BLAS3_TRSM_SLAB_MIN override the maximum (<= 4)
+// and the minimum width (tests reach the multi-slab sweep at small sizes)
+static int64_t trsm_slabs(int64_t other) {
+  static int64_t mx = -1, mn = -1;
+  if (mx < 0) {
+    const char *e = getenv("BLAS3_TRSM_SLABS");
+    const int64_t v = e ? atoll(e) : 0;
+    mx = (v >= 1 && v <= MAX_SLABS) ? v : 2;
+    const char *f = getenv("BLAS3_TRSM_SLAB_MIN");
+    const int64_t w = f ? atoll(f) : 0;
+    mn = (w >= 256) ? w / 256 * 256 : 2048;
+  }
+  return imax(1, imin(mx, other / mn));
+}
+static inline int64_t align_down(int64_t v, int64_t a) { return v / a * a; }
+// SMs the first panel's sweep kernels leave free for its doubling chain;
+// env BLAS3_TRSM_RESERVE overrides it (experiments)
+static int64_t trsm_reserve() {
+  static int64_t r = -1;
+  if (r < 0) {
+    const char *e = getenv("BLAS3_TRSM_RESERVE");
+    r = e ? imax(0, atoll(e)) : 32;
+  }
+  return r;
+}
+// width below which the first panel's geometric halving stops (a power of
+// two in [128, NBO]); env BLAS3_TRSM_GEO_LEAF overrides it (experiments)
+static int64_t trsm_geo_leaf() {
+  static int64_t w = -1;
+  if (w < 0) {
+    const char *e = getenv("BLAS3_TRSM_GEO_LEAF");
+    const int64_t v = e ? atoll(e) : 0;
+    w = (v >= 128 && (v & (v - 1)) == 0) ? v : 256;
+  }
+  return w;
 }
 
 int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t n, float alpha,
@@ -414,96 +508,192 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
              unit = up(diag) == 'U';
   const bool lower_op = lower != ta;               // op(A) = L (true) or L^T (false)
   const int64_t nt = left ? m : n;                 // order of A
+  const int64_t NBO = trsm_nbo();
   const int64_t npanel = cdiv(nt, NBO);
   const int64_t other = left ? n : m;              // RHS extent
   const bool forward = left ? lower_op : !lower_op;
 
   const size_t d_bytes = (size_t)npanel * NBO * NBO * sizeof(float);
-  // doubling scratch: (nt / 2sz) pairs x sz^2 floats at the widest level (sz = NBO/2)
-  const size_t t_bytes = ((size_t)nt * (NBO / 4) + (size_t)NBO * NBO / 4) * sizeof(float);
+  // doubling scratch: nt/2sz pairs x sz^2 floats at the widest level
+  const size_t t_rest = (size_t)nt * (NBO / 4), t_first = (size_t)NBO * NBO / 4;
+  const size_t t_bytes = (t_rest + t_first) * sizeof(float);
   const size_t w_bytes = (size_t)NBO * other * sizeof(float);        // one solved panel
   Scratch D, Tw, W;
   if ((rc = get_scratch(D, d_bytes, s))) return rc;
   if ((rc = get_scratch(Tw, t_bytes, s, d_bytes))) return rc;
   if ((rc = get_scratch(W, w_bytes, s, d_bytes + t_bytes))) return rc;
-  if ((rc = trsm_panel_inverses(A, lda, nt, lower, unit, D.p, Tw.p, s, sms))) return rc;
 
-  // Recursive sweep over panels in processing order (forward or backward):
-  //   solve(first half); B_rest <- a*B_rest - op(A)(rest, first) * X_first;
-  //   solve(second half).
-  // The updates are few large-K GEMMs (K = nt/2, nt/4, ...) instead of one
-  // K = NBO GEMM per panel.  `scaled` says whether alpha has already been
-  // applied to the rows of the range (alpha is folded into the first touch).
-  auto elem = [&](int64_t qa, int64_t qb, int64_t &lo, int64_t &hi) {  // processing -> elements
-    const int64_t pa = forward ? qa : npanel - qb, pb = forward ? qb : npanel - qa;
-    lo = pa * NBO;
-    hi = imin(nt, pb * NBO);
-  };
-  // in_w: the rows (L) / columns (R) of a single-panel range were left in W
-  // (already updated) by the preceding update, so the solve reads W and writes
-  // B directly -- no copy-back.
-  std::function<int(int64_t, int64_t, bool, bool)> rec = [&](int64_t q0, int64_t q1, bool scaled,
-                                                             bool in_w) -> int {
-    int rc2;
-    if (q1 - q0 == 1) {
-      const int64_t p = forward ? q0 : npanel - 1 - q0;
-      const int64_t p0 = p * NBO, pr = imin(NBO, nt - p0);
+  std::lock_guard<std::mutex> lk(g_trsm_mu);          // the per-device side streams
+  TrsmStreams *ts = trsm_streams();
+  if (!ts) return BLAS3_ERR_CUDA;
+  // 1. every 128-block inverse on the caller's stream; then the doubling
+  //    levels of all panels on the high-priority side stream, one event per
+  //    level, while the sweep starts on blocks whose inverse already exists.
+  if (launch_trsm_diag_inv(A, lda, nt, lower, unit, D.p, NBO, s)) return BLAS3_ERR_CUDA;
+  if (cudaEventRecord(ts->ev_fork, s) != cudaSuccess ||
+      cudaStreamWaitEvent(ts->side, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+  int nlvl = 0;
+  for (int64_t sz = 128; sz < NBO; sz *= 2) ++nlvl;
+  // the first processed panel's levels (on the sweep's critical path) alone on
+  // the high-priority stream; the other panels' levels (needed one panel
+  // sweep later) on a second side stream
+  const int64_t pfirst = forward ? 0 : npanel - 1;
+  {
+    const int64_t o = pfirst * NBO;
+    if ((rc = trsm_panel_doubling(A + o * (1 + lda), lda, imin(NBO, nt - o), lower,
+                                  D.p + pfirst * NBO * NBO, Tw.p + t_rest, ts->side, sms, ts->ev_lvl)))
+      return rc;
+  }
+  if (npanel > 1) {
+    const int64_t prest = forward ? 1 : 0, o = prest * NBO;
+    if (cudaStreamWaitEvent(ts->side2, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+    if ((rc = trsm_panel_doubling(A + o * (1 + lda), lda, imin(nt, (prest + npanel - 1) * NBO) - o, lower,
+                                  D.p + prest * NBO * NBO, Tw.p, ts->side2, sms, ts->ev_lvl2)))
+      return rc;
+  }
+
+  // 2. the sweep, independently per slab of the right-hand side (columns of B
+  //    for side=L, rows for side=R), each slab on its own stream.
+  //    Panels (NBO wide) are visited in dependency order by recursive halving
+  //    of the panel range: solve the first half; ONE GEMM update of the second
+  //    half by the first (K = nt/2, nt/4, ...); solve the second half.  The
+  //    FIRST processed panel is itself halved geometrically down to 256-wide
+  //    blocks (its first blocks only need the first doubling levels), so the
+  //    sweep starts ~one level after the 128-block inverses instead of after
+  //    the whole doubling chain.  A leaf [e0, e0+cnt) -- an aligned block of
+  //    width wblk, clipped to the matrix -- is X = a1 * inv(op(A)_blk) * B_blk
+  //    with the inverse read from D (the diagonal blocks of a panel inverse
+  //    are the inverses of the aligned sub-blocks).  alpha is folded into the
+  //    first operation that touches each row (`scaled`).
+  const int64_t nslab = trsm_slabs(other);
+  for (int64_t q = 0; q < nslab; ++q) {
+    const int64_t c0 = align_down(other * q / nslab, 256), c1 = q + 1 == nslab ? other : align_down(other * (q + 1) / nslab, 256);
+    cudaStream_t st = nslab == 1 ? s : ts->slab[q];
+    if (st != s && cudaStreamWaitEvent(st, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+    float *Bq = left ? B + c0 * ldb : B + c0;
+    float *Wq = left ? W.p + c0 * NBO : W.p + c0;
+    const int64_t mq = left ? m : c1 - c0, nq = left ? c1 - c0 : n;
+    int waited = -1;                                  // highest first-panel level waited on
+    bool waited_rest = false;                         // the other panels' inverses waited on
+
+    // leaf: rows (L) / columns (R) [e0, e0 + cnt) of X, aligned block width wblk
+    // kernels of the first panel leave SMs to the latency-bound doubling
+    // chain of that panel (high-priority side stream)
+    const int32_t first_sms = (int32_t)imax(sms / 2, sms - trsm_reserve());
+    auto leaf = [&](int64_t e0, int64_t cnt, int64_t wblk, bool scaled, bool in_w) -> int {
+      int rc2;
+      int lv = -1;                                    // doubling level that built inv(block)
+      for (int64_t w2 = 256; w2 <= wblk; w2 *= 2) ++lv;
+      if (e0 / NBO == pfirst) {
+        if (lv > waited) {
+          if (cudaStreamWaitEvent(st, ts->ev_lvl[lv], 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+          waited = lv;
+        }
+      } else if (lv >= 0 && !waited_rest) {            // full panels: the last level of the rest
+        if (cudaStreamWaitEvent(st, ts->ev_lvl2[nlvl - 1], 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+        waited_rest = true;
+      }
       const float a1 = scaled ? 1.f : alpha;
-      const float *Dp = D.p + p * NBO * NBO;
+      const float *Dp = D.p + (e0 / NBO) * NBO * NBO + (e0 % NBO) * (1 + NBO);
       if (left) {
-        // X_p = a1 * inv(op(A)_pp) * B_p: Xa(r,k) = Dop(r,k), Dop = lower_op ? D : D^T
-        Problem P = in_w ? problem(pr, n, a1, 0.f, nullptr, 0, B + p0, ldb)
-                         : problem(pr, n, a1, 0.f, nullptr, 0, W.p, pr);
+        // X = a1 * inv(op(A)_bb) * B_b: Xa(r,k) = Dop(r,k), Dop = lower_op ? D : D^T
+        Problem P = in_w ? problem(cnt, nq, a1, 0.f, nullptr, 0, Bq + e0, ldb)
+                         : problem(cnt, nq, a1, 0.f, nullptr, 0, Wq, cnt);
         P.seg[0].a = tri_zeroed(Dp, NBO, true, !lower_op);
-        P.seg[0].b = in_w ? dense(W.p, pr, true) : dense(B + p0, ldb, true);
-        P.seg[0].K = pr;
+        P.seg[0].b = in_w ? dense(Wq, cnt, true) : dense(Bq + e0, ldb, true);
+        P.seg[0].K = cnt;
         P.rev_m = tri_kle(P.seg[0].a);
         P.outer = 1;                     // all longest m-rows first (LPT)
-        if ((rc2 = run_problem(P, s, sms))) return rc2;
-        if (!in_w && launch_copy(B + p0, ldb, W.p, pr, pr, n, s)) return BLAS3_ERR_CUDA;
+        if (e0 / NBO == pfirst) P.max_sms = first_sms;
+        if ((rc2 = run_problem(P, st, sms))) return rc2;
+        if (!in_w && launch_copy(Bq + e0, ldb, Wq, cnt, cnt, nq, st)) return BLAS3_ERR_CUDA;
       } else {
-        // X_p = a1 * B_p * inv(op(A)_pp): Xb(c,k) = Dop(k,c) -> TRI swap = lower_op
-        Problem P = in_w ? problem(m, pr, a1, 0.f, nullptr, 0, B + p0 * ldb, ldb)
-                         : problem(m, pr, a1, 0.f, nullptr, 0, W.p, m);
-        P.seg[0].a = in_w ? dense(W.p, m, false) : dense(B + p0 * ldb, ldb, false);
+        // X = a1 * B_b * inv(op(A)_bb): Xb(c,k) = Dop(k,c) -> TRI swap = lower_op
+        Problem P = in_w ? problem(mq, cnt, a1, 0.f, nullptr, 0, Bq + e0 * ldb, ldb)
+                         : problem(mq, cnt, a1, 0.f, nullptr, 0, Wq, m);
+        P.seg[0].a = in_w ? dense(Wq, m, false) : dense(Bq + e0 * ldb, ldb, false);
         P.seg[0].b = tri_zeroed(Dp, NBO, true, lower_op);
-        P.seg[0].K = pr;
+        P.seg[0].K = cnt;
         P.rev_n = tri_kle(P.seg[0].b);
         P.outer = 2;
-        if ((rc2 = run_problem(P, s, sms))) return rc2;
-        if (!in_w && launch_copy(B + p0 * ldb, ldb, W.p, m, m, pr, s)) return BLAS3_ERR_CUDA;
+        if (e0 / NBO == pfirst) P.max_sms = first_sms;
+        if ((rc2 = run_problem(P, st, sms))) return rc2;
+        if (!in_w && launch_copy(Bq + e0 * ldb, ldb, Wq, m, mq, cnt, st)) return BLAS3_ERR_CUDA;
       }
       return 0;
-    }
-    const int64_t mid = q0 + (q1 - q0) / 2;
-    if ((rc2 = rec(q0, mid, scaled, in_w && false))) return rc2;
-    int64_t k_lo, k_hi, o_lo, o_hi;
-    elem(q0, mid, k_lo, k_hi);                       // solved part
-    elem(mid, q1, o_lo, o_hi);                       // part to update
-    const float a1 = scaled ? 1.f : alpha;
-    const bool to_w = (q1 - mid == 1);               // updated panel goes straight to W
-    if (left) {   // B_o <- a1*B_o - op(A)(o, k) * X_k (X_k = B rows k)
-      // Xa(r,kk) = op(A)(o_lo+r, k_lo+kk): !ta -> A(o_lo+r, k_lo+kk) rk; ta -> A(k_lo+kk, o_lo+r) kr
-      const float *pa = ta ? A + k_lo + o_lo * lda : A + o_lo + k_lo * lda;
-      Problem P = to_w ? problem(o_hi - o_lo, n, -1.f, a1, B + o_lo, ldb, W.p, o_hi - o_lo)
-                       : problem(o_hi - o_lo, n, -1.f, a1, B + o_lo, ldb, B + o_lo, ldb);
-      P.seg[0].a = dense(pa, lda, ta);
-      P.seg[0].b = dense(B + k_lo, ldb, true);
-      P.seg[0].K = k_hi - k_lo;
-      if ((rc2 = run_problem(P, s, sms))) return rc2;
-    } else {      // B(:,o) <- a1*B(:,o) - X_k * op(A)(k, o)
+    };
+    // update: rows (L) / columns (R) [o_lo, o_hi) <- a1 * B_o - op(A)(o, k) X_k, k in [k_lo, k_hi);
+    // to_w: the result goes to W (the next operation is the leaf solve of o)
+    auto update = [&](int64_t k_lo, int64_t k_hi, int64_t o_lo, int64_t o_hi, float a1, bool to_w) -> int {
+      if (left) {   // Xa(r,kk) = op(A)(o_lo+r, k_lo+kk): !ta -> A(o_lo+r, k_lo+kk) rk; ta -> A(k_lo+kk, o_lo+r) kr
+        const float *pa = ta ? A + k_lo + o_lo * lda : A + o_lo + k_lo * lda;
+        Problem P = to_w ? problem(o_hi - o_lo, nq, -1.f, a1, Bq + o_lo, ldb, Wq, o_hi - o_lo)
+                         : problem(o_hi - o_lo, nq, -1.f, a1, Bq + o_lo, ldb, Bq + o_lo, ldb);
+        P.seg[0].a = dense(pa, lda, ta);
+        P.seg[0].b = dense(Bq + k_lo, ldb, true);
+        P.seg[0].K = k_hi - k_lo;
+        if (o_lo / NBO == pfirst) P.max_sms = first_sms;
+        return run_problem(P, st, sms);
+      }
+      // B(:,o) <- a1*B(:,o) - X_k * op(A)(k, o):
       // Xb(c,kk) = op(A)(k_lo+kk, o_lo+c): !ta -> A(k_lo+kk, o_lo+c) kr; ta -> A(o_lo+c, k_lo+kk) rk
       const float *pb = ta ? A + o_lo + k_lo * lda : A + k_lo + o_lo * lda;
-      Problem P = to_w ? problem(m, o_hi - o_lo, -1.f, a1, B + o_lo * ldb, ldb, W.p, m)
-                       : problem(m, o_hi - o_lo, -1.f, a1, B + o_lo * ldb, ldb, B + o_lo * ldb, ldb);
-      P.seg[0].a = dense(B + k_lo * ldb, ldb, false);
+      Problem P = to_w ? problem(mq, o_hi - o_lo, -1.f, a1, Bq + o_lo * ldb, ldb, Wq, m)
+                       : problem(mq, o_hi - o_lo, -1.f, a1, Bq + o_lo * ldb, ldb, Bq + o_lo * ldb, ldb);
+      P.seg[0].a = dense(Bq + k_lo * ldb, ldb, false);
       P.seg[0].b = dense(pb, lda, !ta);
       P.seg[0].K = k_hi - k_lo;
-      if ((rc2 = run_problem(P, s, sms))) return rc2;
-    }
-    return rec(mid, q1, true, to_w);
-  };
-  if ((rc = rec(0, npanel, false, false))) return rc;
+      if (o_lo / NBO == pfirst) P.max_sms = first_sms;
+      return run_problem(P, st, sms);
+    };
+    // geometric solve of the aligned block [lo, lo + w) (clipped to nt): the
+    // first half (in processing order) recursively, the second as one leaf
+    std::function<int(int64_t, int64_t, bool)> geo = [&](int64_t lo, int64_t w, bool scaled) -> int {
+      int rc2;
+      const int64_t e1 = imin(nt, lo + w);
+      if (w <= trsm_geo_leaf()) return leaf(lo, e1 - lo, w, scaled, false);
+      const int64_t h = w / 2, mid = lo + h;
+      if (mid >= e1) return geo(lo, h, scaled);          // upper half empty (ragged end)
+      const int64_t f_lo = forward ? lo : mid, f_hi = forward ? mid : e1;   // first half
+      const int64_t s_lo = forward ? mid : lo, s_hi = forward ? e1 : mid;   // second half
+      if ((rc2 = geo(f_lo, h, scaled))) return rc2;
+      if ((rc2 = update(f_lo, f_hi, s_lo, s_hi, scaled ? 1.f : alpha, true))) return rc2;
+      return leaf(s_lo, s_hi - s_lo, h, true, true);
+    };
+    auto elem = [&](int64_t qa, int64_t qb, int64_t &lo, int64_t &hi) {  // processing -> elements
+      const int64_t pa = forward ? qa : npanel - qb, pb = forward ? qb : npanel - qa;
+      lo = pa * NBO;
+      hi = imin(nt, pb * NBO);
+    };
+    // in_w: the rows (L) / columns (R) of a single-panel range were left in W
+    // (already updated) by the preceding update, so the solve reads W and writes
+    // B directly -- no copy-back.
+    std::function<int(int64_t, int64_t, bool, bool)> rec = [&](int64_t q0, int64_t q1, bool scaled,
+                                                               bool in_w) -> int {
+      int rc2;
+      if (q1 - q0 == 1) {
+        const int64_t p = forward ? q0 : npanel - 1 - q0;
+        const int64_t p0 = p * NBO, pr = imin(NBO, nt - p0);
+        if (q0 == 0) return geo(p0, NBO, scaled);       // the first processed panel (p == pfirst)
+        return leaf(p0, pr, NBO, scaled, in_w);
+      }
+      const int64_t mid = q0 + (q1 - q0) / 2;
+      if ((rc2 = rec(q0, mid, scaled, false))) return rc2;
+      int64_t k_lo, k_hi, o_lo, o_hi;
+      elem(q0, mid, k_lo, k_hi);                       // solved part
+      elem(mid, q1, o_lo, o_hi);                       // part to update
+      const bool to_w = (q1 - mid == 1);               // updated panel goes straight to W
+      if ((rc2 = update(k_lo, k_hi, o_lo, o_hi, scaled ? 1.f : alpha, to_w))) return rc2;
+      return rec(mid, q1, true, to_w);
+    };
+    if ((rc = rec(0, npanel, false, false))) return rc;
+    if (st != s && (cudaEventRecord(ts->ev_join[q], st) != cudaSuccess ||
+                    cudaStreamWaitEvent(s, ts->ev_join[q], 0) != cudaSuccess)) return BLAS3_ERR_CUDA;
+  }
+  // the side streams' last levels are part of this call (scratch is freed on s)
+  if (nlvl > 0 && cudaStreamWaitEvent(s, ts->ev_lvl[nlvl - 1], 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+  if (nlvl > 0 && npanel > 1 && cudaStreamWaitEvent(s, ts->ev_lvl2[nlvl - 1], 0) != cudaSuccess)
+    return BLAS3_ERR_CUDA;
   return finish(0);
 }
 

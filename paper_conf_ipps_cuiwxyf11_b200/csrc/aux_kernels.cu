@@ -241,6 +241,16 @@ trsm_diag_inv_kernel(const float *A, int64_t lda, int64_t n, int stored_lower, i
 #pragma unroll 8
     for (int c = c0; c < DNB; c += 2)
       D[r + (int64_t)c * ldD] = (r < nr && c < nr && r >= c) ? X[r * DLD + c] : 0.f;
+    // the blank (upper) triangle of the panel inverse is read as zeros by the
+    // structured GEMMs, but only within 256 of the diagonal (tile height): zero
+    // the two 128-blocks to the right of this diagonal block (inside the panel)
+    // so the workspace needs no memset
+    const int64_t bi = blockIdx.x % bpp;
+    for (int j = 1; j <= 2 && bi + j < bpp; ++j) {
+      float *U = D + (int64_t)j * DNB * ldD;
+#pragma unroll 8
+      for (int c = c0; c < DNB; c += 2) U[r + (int64_t)c * ldD] = 0.f;
+    }
   }
 }
 

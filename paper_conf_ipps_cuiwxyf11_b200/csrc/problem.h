@@ -74,8 +74,12 @@ struct Problem {
   // performance-experiment knobs (env BLAS3_DEBUG_TC; results are WRONG when
   // set, never used by tests or the bench): bit0 skip the split pass,
   // bit1 issue only hi*hi (1xTF32), bit2 skip the epilogue stores,
-  // bit3 issue no MMAs (commits only), bit4 issue no TMA loads
+  // bit3 issue no MMAs (commits only), bit4 issue no TMA loads,
+  // bit5 skip the triangular zero-select/unit-diagonal fix-up
   int32_t dbg;
+  // launch at most this many SMs' worth of CTAs (0: all).  The STRSM driver
+  // leaves SMs free for its latency-bound side-stream kernels this way.
+  int32_t max_sms;
 };
 
 HD int64_t batch_off(const BatchStride &s, int64_t b, int64_t per) {

@@ -312,18 +312,38 @@ __device__ __forceinline__ void sym_merge(const OpDesc &o, uint8_t *raw, int64_t
 
 // Triangular block touching the diagonal: zero-select the blank part, force
 // the unit diagonal (the stored values there are never used).
+// Vectorised: both staged layouts keep 4 consecutive elements along the
+// contiguous dimension (r for MN-major, k for K-major) in one 16-B word, so
+// each thread handles float4s and rewrites one only when it crosses the
+// blank triangle or the diagonal.
 __device__ __forceinline__ void tri_fix(const OpDesc &o, int lay, uint8_t *raw, int64_t r0,
                                         int64_t k0, int rows, int64_t R, int64_t K, int t) {
   const bool kle = tri_kle(o);
-  for (int e = t; e < rows * BK; e += TR_THREADS) {
-    int r, k;
-    if (lay == LAYOUT_MN) { r = e % rows; k = e / rows; } else { k = e % BK; r = e / BK; }
-    int64_t gr = r0 + r, gk = k0 + k;
-    bool nz = kle ? (gk <= gr) : (gk >= gr);
-    uint32_t off = (lay == LAYOUT_MN) ? off_mn(r, k) : off_k(r, k);
-    float *p = reinterpret_cast<float *>(raw + off);
-    if (!nz) *p = 0.f;
-    else if (o.unit && gr == gk && gr < R && gk < K) *p = 1.f;
+  const bool unit = o.unit;
+  const int nvec = rows * BK / 4;
+  for (int e = t; e < nvec; e += TR_THREADS) {
+    int r, k, dr, dk;          // first element and the step between the 4 lanes
+    uint32_t off;
+    if (lay == LAYOUT_MN) { r = (e % (rows / 4)) * 4; k = e / (rows / 4); dr = 1; dk = 0; off = off_mn(r, k); }
+    else                  { k = (e % (BK / 4)) * 4; r = e / (BK / 4); dr = 0; dk = 1; off = off_k(r, k); }
+    const int64_t d0 = (r0 + r) - (k0 + k);          // gr - gk of lane 0; lane j: d0 + j*(dr - dk)
+    const int64_t d3 = d0 + 3 * (dr - dk);
+    const int64_t dmin = d0 < d3 ? d0 : d3, dmax = d0 < d3 ? d3 : d0;
+    // nonzero iff gr - gk >= 0 (kle) or <= 0; untouched if all 4 lanes are
+    // strictly inside the nonzero region (no diagonal element either)
+    if (kle ? dmin > 0 : dmax < 0) continue;
+    float4 *p = reinterpret_cast<float4 *>(raw + off);
+    if (kle ? dmax < 0 : dmin > 0) { *p = make_float4(0.f, 0.f, 0.f, 0.f); continue; }
+    float v[4];
+    *reinterpret_cast<float4 *>(v) = *p;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int64_t d = d0 + j * (dr - dk);
+      const int64_t gr = r0 + r + j * dr, gk = k0 + k + j * dk;
+      if (kle ? d < 0 : d > 0) v[j] = 0.f;
+      else if (unit && d == 0 && gr < R && gk < K) v[j] = 1.f;
+    }
+    *p = *reinterpret_cast<float4 *>(v);
   }
 }
 
@@ -426,6 +446,10 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
   if (CG == 2) ptx::cluster_sync(); else __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = bars->tmem_base;
+  // Everything above (barrier init, TMEM allocation, tensor-map prefetch)
+  // overlaps the tail of the previous kernel of the stream when launched with
+  // PDL; no global memory is touched before the previous grid is complete.
+  ptx::griddep_wait();
   if (threadIdx.x == 0) BLAS3_TRACE(1);
 
   // batched problems: tile tb -> batch member b = tb / tiles_per, tile t
@@ -487,7 +511,12 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
         bars->wk[slot] = w;
         ptx::mbar_arrive(&bars->wk_full[slot]);       // release: local roles see wk[slot]
         ++qi;
-        if (tb < 0) break;
+        if (tb < 0) {
+          // this CTA has claimed its last tile: the next kernel of the stream
+          // may be scheduled onto SMs as they drain (PDL)
+          ptx::griddep_launch_dependents();
+          break;
+        }
         const int32_t bj = (int32_t)(w.b % per), bg = (int32_t)(w.b / per);
         const int64_t m0 = w.m0, n0 = w.n0;
         const int64_t ma = m0 + HA * rank, nb = n0 + HB * rank;
@@ -641,13 +670,13 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           else if (si.clsA == BLK_TRI_DIAG) {
             const int own = block_class(sg.a, ma, imin(P.M, ma + HA), k0, k1);
             if (own == BLK_ZERO) { zero_fill(rb.A, G::A_BYTES, tt); fix = true; }
-            else if (own == BLK_TRI_DIAG) { tri_fix(sg.a, si.layA, rb.A, ma, k0, HA, P.M, sg.K, tt); fix = true; }
+            else if (own == BLK_TRI_DIAG && !(P.dbg & 32)) { tri_fix(sg.a, si.layA, rb.A, ma, k0, HA, P.M, sg.K, tt); fix = true; }
           }
           if (si.clsB == BLK_SYM_DIAG) { sym_merge(sg.b, rb.B, nb, k0, HB, P.N, sg.K, tt); fix = true; }
           else if (si.clsB == BLK_TRI_DIAG) {
             const int own = block_class(sg.b, nb, imin(P.N, nb + HB), k0, k1);
             if (own == BLK_ZERO) { zero_fill(rb.B, G::B_BYTES, tt); fix = true; }
-            else if (own == BLK_TRI_DIAG) { tri_fix(sg.b, si.layB, rb.B, nb, k0, HB, P.N, sg.K, tt); fix = true; }
+            else if (own == BLK_TRI_DIAG && !(P.dbg & 32)) { tri_fix(sg.b, si.layB, rb.B, nb, k0, HB, P.N, sg.K, tt); fix = true; }
           }
           if (fix) ptx::named_bar_sync(1, TR_THREADS);
           ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
@@ -925,13 +954,20 @@ static int launch_cg(TcParams &prm, cudaStream_t stream, int num_sms) {
   cfg.blockDim = dim3(NTHREADS);
   cfg.dynamicSmemBytes = G::SMEM;
   cfg.stream = stream;
-  cudaLaunchAttribute attrs[1];
+  cudaLaunchAttribute attrs[2];
   attrs[0].id = cudaLaunchAttributeClusterDimension;
   attrs[0].val.clusterDim.x = CG;
   attrs[0].val.clusterDim.y = 1;
   attrs[0].val.clusterDim.z = 1;
+  // programmatic dependent launch: this grid's prologue may overlap the tail
+  // of the previous kernel on the stream (the kernel waits before touching
+  // global memory).  BLAS3_PDL=0 disables it (experiments).
+  static int pdl = -1;
+  if (pdl < 0) { const char *e = getenv("BLAS3_PDL"); pdl = (e && e[0] == '0') ? 0 : 1; }
+  attrs[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attrs[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attrs;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = pdl ? 2 : 1;
   const cudaError_t e = cudaLaunchKernelEx(&cfg, tc_structured_gemm<CG>, prm);
   note_launch(0);
   return (e == cudaSuccess && cudaGetLastError() == cudaSuccess) ? 0 : -1;
@@ -979,7 +1015,11 @@ static bool split_workspace(cudaStream_t stream, int num_sms, float **ws, uint32
     if (tab[i].dev == d && tab[i].st == stream) { *ws = tab[i].ws; *cnt = tab[i].cnt; return true; }
   if (n == 16) return false;
   Entry e{d, stream, nullptr, nullptr};
-  const size_t wsb = (size_t)num_sms * HA * BN * sizeof(float), cb = 1024 * sizeof(uint32_t);
+  // sized for the whole device: launches may use fewer SMs (Problem::max_sms)
+  int dev_sms = num_sms;
+  if (cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, d) != cudaSuccess) return false;
+  dev_sms = dev_sms > num_sms ? dev_sms : num_sms;
+  const size_t wsb = (size_t)dev_sms * HA * BN * sizeof(float), cb = 1024 * sizeof(uint32_t);
   if (cudaMalloc(&e.ws, wsb) != cudaSuccess) { cudaGetLastError(); return false; }
   if (cudaMalloc(&e.cnt, cb) != cudaSuccess || cudaMemset(e.cnt, 0, cb) != cudaSuccess) {
     cudaGetLastError(); cudaFree(e.ws); return false;

@@ -1,0 +1,75 @@
+"""STRSM sweep structure (rows A7/A8): several diagonal panels, the side-stream
+doubling of all but the first processed panel, and the per-slab sweeps on
+their own streams.
+
+* in process, at the default panel width (2048): ragged orders > 2048 with
+  >= 4096 right-hand sides (two slabs, a ragged last slab and panel), every
+  side/uplo/trans/diag variant, residual and forward error on sampled
+  columns (side=L) / rows (side=R) against the fp64 oracle;
+* in a subprocess with a 256-wide panel, up to 4 slabs and a 256-wide slab
+  minimum (env knobs read once per process), the whole small-size STRSM
+  parity suite -- many panels, forward and backward orders, several slabs.
+"""
+import itertools
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+import blas3_inputs as gen
+from check import f64, fro, op, to_dev, to_host, tri_full
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+AL = 1.5
+V16 = list(itertools.product("LR", "LU", "NT", "NU"))
+
+
+@pytest.fixture(scope="module")
+def b3():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_cuiwxyf11_b200 as m
+    m.set_math_mode("3xtf32")
+    return m
+
+
+@pytest.mark.parametrize("side,uplo,ta,diag", V16)
+def test_strsm_multi_panel_multi_slab(b3, oracle_mod, side, uplo, ta, diag):
+    ka, other = 2600, 4500                 # 2 panels (ragged), 2 slabs (ragged last)
+    m, n = (ka, other) if side == "L" else (other, ka)
+    A = gen.triangular_dd(ka, uplo, diag, "sweep-a")
+    B = gen.uniform(m, n, "sweep-b")
+    dB = to_dev(B)
+    b3.strsm(side, uplo, ta, diag, AL, to_dev(A), dB)
+    X = f64(to_host(dB))
+    T = op(tri_full(A, uplo, diag, ka), ta)
+    # samples straddle the slab boundary (2048 + 256 k) and the ragged tail
+    sel = np.unique(np.concatenate([gen.sample_indices(other, 20, "sweep-sel"),
+                                    [0, 2047, 2048, 2303, 2304, other - 1]]))
+    if side == "L":
+        Xs, Bs = X[:, sel], f64(B[:, sel])
+        resid = fro(T @ Xs - AL * Bs) / (fro(T) * fro(Xs))
+    else:
+        Xs, Bs = X[sel, :], f64(B[sel, :])
+        resid = fro(Xs @ T - AL * Bs) / (fro(T) * fro(Xs))
+    assert resid <= 1e-5 * np.sqrt(ka)
+    ref = oracle_mod.strsm(side, uplo, ta, diag, AL, A, B, sel=sel)
+    assert fro(Xs - ref) / fro(ref) <= 1e-5
+
+
+def test_strsm_small_panels_many_slabs():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    env = {**os.environ, "BLAS3_TRSM_NB": "256", "BLAS3_TRSM_SLABS": "4", "BLAS3_TRSM_SLAB_MIN": "256"}
+    cmd = [sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k", "strsm",
+           os.path.join(ROOT, "tests", "test_parity_gpu.py")]
+    r = subprocess.run(cmd, env=env, cwd=ROOT, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
+    assert " passed" in r.stdout
