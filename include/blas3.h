@@ -44,6 +44,9 @@
  *  Math       BLAS3_MATH_3XTF32 (default): tcgen05 tensor cores with a
  *             3xTF32 split (hi*hi + hi*lo + lo*hi) and fp32 accumulation in
  *             TMEM.  BLAS3_MATH_SIMT_FP32: exact-fp32 FFMA kernels.
+ *             BLAS3_MATH_1XTF32: opt-in fast mode, one TF32 pass
+ *             (inputs truncated to TF32, 10-bit mantissa; normwise error
+ *             ~1e-3, NOT the fp32 accuracy of the other two modes).
  *             Arguments that violate TMA's 16-byte rules (pointer not
  *             16-byte aligned or ld % 4 != 0) run on the SIMT kernels in
  *             either mode.
@@ -68,7 +71,7 @@ enum {
     BLAS3_ERR_TMA = -4
 };
 
-enum { BLAS3_MATH_3XTF32 = 0, BLAS3_MATH_SIMT_FP32 = 1 };
+enum { BLAS3_MATH_3XTF32 = 0, BLAS3_MATH_SIMT_FP32 = 1, BLAS3_MATH_1XTF32 = 2 };
 
 /* SGEMM: C <- alpha*op(A)*op(B) + beta*C, op(X) = X or X^T.
  * op(A) is m x k, op(B) is k x n, C is m x n.  Paper: GEMM-NN/-TN loop nests
@@ -131,10 +134,50 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
                 blas3_stream_t stream);
 
 /* Process-wide math mode (BLAS3_MATH_3XTF32 default; the environment
- * variable BLAS3_MATH=simt|3xtf32 overrides the default at load).
+ * variable BLAS3_MATH=simt|3xtf32|1xtf32 overrides the default at load).
  * Returns 0, or 1 if `mode` is not a valid mode (nothing changed). */
 int blas3_set_math_mode(int mode);
 int blas3_get_math_mode(void);
+
+/* Tuning options: the variant choice of the paper's generator (its search
+ * over optimisation schemes) as process-wide
+ * integer knobs read by every later call.  Every value selects among
+ * implementations that compute the same result (each is parity-tested).
+ * Each option starts from its environment variable (named in brackets, read
+ * once at the first call) or its default.
+ *   BLAS3_OPT_GM_MAP       [BLAS3_GM_MAP]   GM_map adaptor: rewrite a
+ *                          transposed / symmetric / triangular operand in global
+ *                          memory first.  -1 auto (default: per-routine size
+ *                          thresholds below), 0 never, 1 always
+ *   BLAS3_OPT_GM_MIN_GEMM  SGEMM transa!='N': auto threshold on n (default 1<<30 = off)
+ *   BLAS3_OPT_GM_MIN_SYMM  SSYMM: auto threshold on the non-symmetric extent (2048)
+ *   BLAS3_OPT_GM_MIN_TRMM  STRMM: auto threshold on the right-hand-side extent (1<<30)
+ *   BLAS3_OPT_GM_MIN_TRSM  STRSM transa!='N': auto threshold on the RHS extent (1<<30)
+ *                          (auto also requires the structured order >= 2048)
+ *   BLAS3_OPT_TC_CTA       [BLAS3_TC_CTA]   0 auto (default), 1 single-CTA 128x256
+ *                          tiles, 2 CTA-pair 256x256 tiles (cta_group::2)
+ *   BLAS3_OPT_TC_SPLIT     [BLAS3_TC_SPLIT] 1 split the tail wave along K (default), 0 off
+ *   BLAS3_OPT_TC_STATIC    [BLAS3_TC_STATIC] 0 dynamic tile scheduler (default), 1 static
+ *   BLAS3_OPT_PDL          [BLAS3_PDL]      1 programmatic dependent launch (default), 0 off
+ *   BLAS3_OPT_TRSM_NB      [BLAS3_TRSM_NB]  STRSM panel width: power of 2 in [128, 8192] (2048)
+ *   BLAS3_OPT_TRSM_SLABS   [BLAS3_TRSM_SLABS] right-hand-side slabs on own streams, 1..4 (2)
+ *   BLAS3_OPT_TRSM_SLAB_MIN [BLAS3_TRSM_SLAB_MIN] minimum slab width, >= 256 (2048)
+ *   BLAS3_OPT_TRSM_RESERVE [BLAS3_TRSM_RESERVE] SMs the first panel's sweep leaves to
+ *                          the panel-inverse doubling chain, 0..#SMs/2 (32)
+ *   BLAS3_OPT_TRSM_GEO_LEAF [BLAS3_TRSM_GEO_LEAF] the first panel is halved down to
+ *                          this width: power of 2 in [128, 8192] (256)
+ * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
+ * (nothing changed).  blas3_get_option returns the current value, or
+ * INT64_MIN for an unknown key. */
+enum {
+    BLAS3_OPT_GM_MAP = 0, BLAS3_OPT_GM_MIN_GEMM = 1, BLAS3_OPT_GM_MIN_SYMM = 2,
+    BLAS3_OPT_GM_MIN_TRMM = 3, BLAS3_OPT_GM_MIN_TRSM = 4, BLAS3_OPT_TC_CTA = 5,
+    BLAS3_OPT_TC_SPLIT = 6, BLAS3_OPT_TC_STATIC = 7, BLAS3_OPT_PDL = 8,
+    BLAS3_OPT_TRSM_NB = 9, BLAS3_OPT_TRSM_SLABS = 10, BLAS3_OPT_TRSM_SLAB_MIN = 11,
+    BLAS3_OPT_TRSM_RESERVE = 12, BLAS3_OPT_TRSM_GEO_LEAF = 13, BLAS3_OPT_COUNT = 14
+};
+int blas3_set_option(int key, int64_t value);
+int64_t blas3_get_option(int key);
 
 /* Optional caller-owned device scratch used before falling back to
  * cudaMallocAsync.  The buffer must stay valid while calls that may use it

@@ -42,12 +42,14 @@ _SIGS = {
     "blas3_set_math_mode": [_i],
     "blas3_get_math_mode": [],
     "blas3_set_workspace": [_p, ctypes.c_size_t],
+    "blas3_set_option": [_i, _i64],
+    "blas3_get_option": [_i],
     "blas3_launch_count": [],
     "blas3_launch_count_by_path": [_i],
     "blas3_error_string": [_i],
     "blas3_version": [],
 }
-_RES = {"blas3_launch_count": _i64, "blas3_launch_count_by_path": _i64, "blas3_error_string": ctypes.c_char_p}
+_RES = {"blas3_get_option": _i64, "blas3_launch_count": _i64, "blas3_launch_count_by_path": _i64, "blas3_error_string": ctypes.c_char_p}
 
 for _name, _args in _SIGS.items():
     _fn = getattr(_lib, _name)
@@ -56,7 +58,7 @@ for _name, _args in _SIGS.items():
     globals()[_name] = _fn
 
 EXPORTED = tuple(_SIGS)
-MATH_3XTF32, MATH_SIMT_FP32 = 0, 1
+MATH_3XTF32, MATH_SIMT_FP32, MATH_1XTF32 = 0, 1, 2
 
 
 class Blas3Error(RuntimeError):
@@ -172,7 +174,7 @@ def strsm(side, uplo, transa, diag, alpha, A, B):
 
 def set_math_mode(mode):
     if isinstance(mode, str):
-        mode = {"3xtf32": MATH_3XTF32, "simt": MATH_SIMT_FP32}[mode.lower()]
+        mode = {"3xtf32": MATH_3XTF32, "simt": MATH_SIMT_FP32, "1xtf32": MATH_1XTF32}[mode.lower()]
     _chk("blas3_set_math_mode", blas3_set_math_mode(mode))  # noqa: F821
 
 
@@ -181,6 +183,41 @@ def get_math_mode():
 
 
 PATH_TCGEN05, PATH_SIMT, PATH_AUX = 0, 1, 2
+
+# tuning options (include/blas3.h BLAS3_OPT_*): name -> key
+OPTIONS = {"gm_map": 0, "gm_min_gemm": 1, "gm_min_symm": 2, "gm_min_trmm": 3, "gm_min_trsm": 4,
+           "tc_cta": 5, "tc_split": 6, "tc_static": 7, "pdl": 8, "trsm_nb": 9, "trsm_slabs": 10,
+           "trsm_slab_min": 11, "trsm_reserve": 12, "trsm_geo_leaf": 13}
+
+
+def set_option(name, value):
+    """Set a tuning option (see include/blas3.h); raises on an invalid name/value."""
+    key = OPTIONS[name] if isinstance(name, str) else int(name)
+    if blas3_set_option(key, int(value)) != 0:  # noqa: F821
+        raise ValueError(f"invalid option {name}={value}")
+
+
+def get_option(name):
+    key = OPTIONS[name] if isinstance(name, str) else int(name)
+    return int(blas3_get_option(key))  # noqa: F821
+
+
+class options:
+    """Context manager: temporarily set tuning options, restore on exit."""
+
+    def __init__(self, **kv):
+        self.kv = kv
+        self.old = {}
+
+    def __enter__(self):
+        for k, v in self.kv.items():
+            self.old[k] = get_option(k)
+            set_option(k, v)
+        return self
+
+    def __exit__(self, *a):
+        for k, v in self.old.items():
+            set_option(k, v)
 
 
 def launch_count(path=None):

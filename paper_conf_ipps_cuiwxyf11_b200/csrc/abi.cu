@@ -23,6 +23,50 @@ void note_launch(int path) {
   if (path >= 0 && path < 3) g_path_launches[path].fetch_add(1, std::memory_order_relaxed);
 }
 
+// ---- tuning options (include/blas3.h): defaults, environment names, ranges
+struct OptSpec { const char *env; int64_t def, lo, hi; bool pow2; };
+static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
+    {"BLAS3_GM_MAP", -1, -1, 1, false},
+    {"BLAS3_GM_MIN_GEMM", int64_t(1) << 30, 0, int64_t(1) << 40, false},
+    {"BLAS3_GM_MIN_SYMM", 2048, 0, int64_t(1) << 40, false},
+    {"BLAS3_GM_MIN_TRMM", int64_t(1) << 30, 0, int64_t(1) << 40, false},
+    {"BLAS3_GM_MIN_TRSM", int64_t(1) << 30, 0, int64_t(1) << 40, false},
+    {"BLAS3_TC_CTA", 0, 0, 2, false},
+    {"BLAS3_TC_SPLIT", 1, 0, 1, false},
+    {"BLAS3_TC_STATIC", 0, 0, 1, false},
+    {"BLAS3_PDL", 1, 0, 1, false},
+    {"BLAS3_TRSM_NB", 2048, 128, 8192, true},
+    {"BLAS3_TRSM_SLABS", 2, 1, 4, false},
+    {"BLAS3_TRSM_SLAB_MIN", 2048, 256, int64_t(1) << 40, false},
+    {"BLAS3_TRSM_RESERVE", 32, 0, 74, false},
+    {"BLAS3_TRSM_GEO_LEAF", 256, 128, 8192, true},
+};
+static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
+static std::once_flag g_opt_once;
+static bool opt_valid(int key, int64_t v) {
+  const OptSpec &o = kOpt[key];
+  if (v < o.lo || v > o.hi) return false;
+  if (o.pow2 && (v & (v - 1))) return false;
+  return true;
+}
+static void opt_init() {
+  std::call_once(g_opt_once, [] {
+    for (int k = 0; k < BLAS3_OPT_COUNT; ++k) {
+      int64_t v = kOpt[k].def;
+      const char *e = getenv(kOpt[k].env);
+      if (e && *e) {
+        const int64_t x = atoll(e);
+        if (opt_valid(k, x)) v = x;
+      }
+      g_opt[k].store(v);
+    }
+  });
+}
+int64_t opt(int key) {
+  opt_init();
+  return (key >= 0 && key < BLAS3_OPT_COUNT) ? g_opt[key].load(std::memory_order_relaxed) : 0;
+}
+
 static int g_math = -1;              // -1: not initialised
 static void *g_ws = nullptr;
 static size_t g_ws_bytes = 0;
@@ -30,10 +74,12 @@ static size_t g_ws_bytes = 0;
 static int math_mode() {
   if (g_math < 0) {
     const char *e = getenv("BLAS3_MATH");
-    g_math = (e && (e[0] == 's' || e[0] == 'S')) ? BLAS3_MATH_SIMT_FP32 : BLAS3_MATH_3XTF32;
+    g_math = (e && (e[0] == 's' || e[0] == 'S')) ? BLAS3_MATH_SIMT_FP32
+             : (e && e[0] == '1') ? BLAS3_MATH_1XTF32 : BLAS3_MATH_3XTF32;
   }
   return g_math;
 }
+static bool tensor_mode() { return math_mode() != BLAS3_MATH_SIMT_FP32; }
 
 // per-device facts: SM count, sm_100 check
 struct DevInfo { int sms = 0; int ok = -1; };
@@ -79,7 +125,11 @@ static int get_scratch(Scratch &sc, size_t bytes, cudaStream_t s, size_t offset 
 static int run_problem(const Problem &P, cudaStream_t s, int sms) {
   if (P.M <= 0 || P.N <= 0) return 0;
   if (P.max_sms > 0 && P.max_sms < sms) sms = P.max_sms;
-  if (math_mode() == BLAS3_MATH_3XTF32 && tc_eligible(P)) return launch_tc(P, s, sms);
+  if (tensor_mode() && tc_eligible(P)) {
+    Problem Q = P;
+    Q.passes = math_mode() == BLAS3_MATH_1XTF32 ? 1 : 3;
+    return launch_tc(Q, s, sms);
+  }
   int rc = launch_simt(P, s, sms);
   return rc ? BLAS3_ERR_CUDA : 0;
 }
@@ -133,6 +183,19 @@ static inline int finish(int rc) {
   return cudaGetLastError() == cudaSuccess ? 0 : BLAS3_ERR_CUDA;
 }
 
+// GM_map policy (paper Adaptor rule 2): rewrite the
+// structured / transposed operand once in global memory (O(n^2) traffic) when
+// the O(n^2 * other) product is large enough to amortise it; the GEMM kernel
+// then stages a plain MN-major operand.  `order` = order of the rewritten
+// operand, `other` = the remaining product dimension.  Env BLAS3_GM_MAP:
+// 0 = never, 1 = always (tests), unset = by size.
+static bool use_gm_map(int64_t order, int64_t other, int min_key) {
+  const int64_t e = opt(BLAS3_OPT_GM_MAP);
+  if (e >= 0) return e == 1;
+  return order >= 2048 && other >= opt(min_key);
+}
+static inline int64_t ld4(int64_t rows) { return (imax(rows, 1) + 3) / 4 * 4; }
+
 }  // namespace blas3
 
 using namespace blas3;
@@ -145,8 +208,20 @@ int64_t blas3_launch_count_by_path(int path) {
   return (path >= 0 && path < 3) ? g_path_launches[path].load() : -1;
 }
 
+int blas3_set_option(int key, int64_t value) {
+  if (key < 0 || key >= BLAS3_OPT_COUNT) return 1;
+  opt_init();
+  if (!opt_valid(key, value)) return 1;
+  g_opt[key].store(value);
+  return 0;
+}
+int64_t blas3_get_option(int key) {
+  if (key < 0 || key >= BLAS3_OPT_COUNT) return INT64_MIN;
+  return opt(key);
+}
+
 int blas3_set_math_mode(int mode) {
-  if (mode != BLAS3_MATH_3XTF32 && mode != BLAS3_MATH_SIMT_FP32) return 1;
+  if (mode != BLAS3_MATH_3XTF32 && mode != BLAS3_MATH_SIMT_FP32 && mode != BLAS3_MATH_1XTF32) return 1;
   g_math = mode;
   return 0;
 }
@@ -195,6 +270,15 @@ int blas3_sgemm(char transa, char transb, int64_t m, int64_t n, int64_t k, float
   P.seg[0].a = dense(A, lda, ta);       // op(A)(r,k) = A(k,r) when transposed -> "kr"
   P.seg[0].b = dense(B, ldb, !tb);      // Xb(c,k) = op(B)(k,c)
   P.seg[0].K = k;
+  Scratch Wm;
+  if (ta && tensor_mode() && use_gm_map(imax(m, k), n, BLAS3_OPT_GM_MIN_GEMM)) {
+    // GM_map: op(A) = A^T materialised m x k (the K-major A operand stages
+    // slower than the MN-major one)
+    const int64_t ldw = ld4(m);
+    if ((rc = get_scratch(Wm, (size_t)ldw * k * sizeof(float), s))) return rc;
+    if (launch_materialize(Wm.p, ldw, A, lda, m, k, MAT_TRANS, 0, 0, 0, s)) return BLAS3_ERR_CUDA;
+    P.seg[0].a = dense(Wm.p, ldw, false);
+  }
   return finish(run_problem(P, s, sms));
 }
 
@@ -219,6 +303,17 @@ int blas3_ssymm(char side, char uplo, int64_t m, int64_t n, float alpha, const f
   cudaStream_t s = (cudaStream_t)stream;
   if (alpha == 0.f) return finish(launch_scale(C, ldc, m, n, beta, 0, s) ? BLAS3_ERR_CUDA : 0);
   Problem P = problem(m, n, alpha, beta, C, ldc, C, ldc);
+  const int64_t ka = left ? m : n;
+  if (tensor_mode() && use_gm_map(ka, left ? n : m, BLAS3_OPT_GM_MIN_SYMM)) {
+    // GM_map: sym(A) materialised as a full ka x ka matrix, then a plain GEMM
+    Scratch Wm;
+    const int64_t ldw = ld4(ka);
+    if ((rc = get_scratch(Wm, (size_t)ldw * ka * sizeof(float), s))) return rc;
+    if (launch_materialize(Wm.p, ldw, A, lda, ka, ka, MAT_SYM, lower, 0, 0, s)) return BLAS3_ERR_CUDA;
+    if (left) { P.seg[0].a = dense(Wm.p, ldw, false); P.seg[0].b = dense(B, ldb, true); P.seg[0].K = m; }
+    else      { P.seg[0].a = dense(B, ldb, false); P.seg[0].b = dense(Wm.p, ldw, false); P.seg[0].K = n; }
+    return finish(run_problem(P, s, sms));
+  }
   if (left) {                       // C = Asym * B : Xa = Asym (m x m), Xb(c,k) = B(k,c)
     P.seg[0].a = sym(A, lda, lower);
     P.seg[0].b = dense(B, ldb, true);
@@ -303,6 +398,7 @@ static int tr_validate(char side, char uplo, char transa, char diag, int64_t m, 
 }
 
 // ------------------------------------------------------------------- STRMM (row A9)
+
 // B <- alpha*op(A)*B (L) or alpha*B*op(A) (R).  The tile-parallel product
 // reads rows (L) / columns (R) of B that other tiles overwrite, so the
 // product goes to stream-ordered scratch and is copied back (A9).
@@ -319,9 +415,36 @@ int blas3_strmm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   if (alpha == 0.f) return finish(launch_scale(B, ldb, m, n, 0.f, 0, s) ? BLAS3_ERR_CUDA : 0);
   const bool left = up(side) == 'L', lower = up(uplo) == 'L', ta = up(transa) != 'N',
              unit = up(diag) == 'U';
-  Scratch W;
+  Scratch W, Wm;
   if ((rc = get_scratch(W, (size_t)m * n * sizeof(float), s))) return rc;
   Problem P = problem(m, n, alpha, 0.f, nullptr, 0, W.p, m);
+  const int64_t ka = left ? m : n;
+  if (tensor_mode() && use_gm_map(ka, left ? n : m, BLAS3_OPT_GM_MIN_TRMM)) {
+    // GM_map: op(T) materialised MN-major with zeros in the blank triangle and
+    // the unit diagonal written: the kernel clips k-ranges but loads every
+    // block as a plain block (no zero-select / transpose)
+    const int64_t ldw = ld4(ka);
+    const bool lop = lower != ta;                  // op(T) is lower
+    if ((rc = get_scratch(Wm, (size_t)ldw * ka * sizeof(float), s, (size_t)m * n * sizeof(float))))
+      return rc;
+    if (launch_materialize(Wm.p, ldw, A, lda, ka, ka, MAT_TRI, lower, ta, unit, s)) return BLAS3_ERR_CUDA;
+    if (left) {   // Xa(r,k) = Wop(r,k)
+      P.seg[0].a = tri_zeroed(Wm.p, ldw, lop, false);
+      P.seg[0].b = dense(B, ldb, true);
+      P.seg[0].K = m;
+      P.rev_m = tri_kle(P.seg[0].a);
+      P.outer = 1;
+    } else {      // Xb(c,k) = Wop(k,c)
+      P.seg[0].a = dense(B, ldb, false);
+      P.seg[0].b = tri_zeroed(Wm.p, ldw, lop, true);
+      P.seg[0].K = n;
+      P.rev_n = tri_kle(P.seg[0].b);
+      P.outer = 2;
+    }
+    if ((rc = run_problem(P, s, sms))) return rc;
+    if (launch_copy(B, ldb, W.p, m, m, n, s)) return BLAS3_ERR_CUDA;
+    return finish(0);
+  }
   if (left) {     // Xa(r,k) = op(T)(r,k) -> swap = trans ; Xb(c,k) = B(k,c)
     P.seg[0].a = tri(A, lda, lower, ta, unit);
     P.seg[0].b = dense(B, ldb, true);
@@ -355,17 +478,8 @@ int blas3_strmm(char side, char uplo, char transa, char diag, int64_t m, int64_t
 //      a single panel is X_p = alpha_p * inv(op(A)_pp) * B_p (TRI operand).
 //      alpha is folded into the first operation that touches each row.
 // Every flop of steps 2-3 runs in the structured GEMM kernels.
-// panel width (a power of two >= 128, the diagonal block); env BLAS3_TRSM_NB
-// overrides it for experiments (tests/bench use the default)
-static int64_t trsm_nbo() {
-  static int64_t nb = -1;
-  if (nb < 0) {
-    const char *e = getenv("BLAS3_TRSM_NB");
-    const int64_t v = e ? atoll(e) : 0;
-    nb = (v >= 128 && v <= 8192 && (v & (v - 1)) == 0) ? v : 2048;
-  }
-  return nb;
-}
+// panel width (a power of two >= 128, the diagonal block; BLAS3_OPT_TRSM_NB)
+static int64_t trsm_nbo() { return opt(BLAS3_OPT_TRSM_NB); }
 
 // Doubling levels 128 -> NBO for the panels of the order-nt triangle whose
 // top-left corner is A (and whose panel inverses start at D); the 128-block
@@ -454,43 +568,17 @@ static TrsmStreams *trsm_streams() {
   }
   return &t;
 }
-// number of right-hand-side slabs: slabs of >= 2048 columns (rows), at most
-// 2; env BLAS3_TRSM_SLABS / BLAS3_TRSM_SLAB_MIN override the maximum (<= 4)
-// and the minimum width (tests reach the multi-slab sweep at small sizes)
+// number of right-hand-side slabs (BLAS3_OPT_TRSM_SLABS at most, each at least
+// BLAS3_OPT_TRSM_SLAB_MIN columns (rows) wide)
 static int64_t trsm_slabs(int64_t other) {
-  static int64_t mx = -1, mn = -1;
-  if (mx < 0) {
-    const char *e = getenv("BLAS3_TRSM_SLABS");
-    const int64_t v = e ? atoll(e) : 0;
-    mx = (v >= 1 && v <= MAX_SLABS) ? v : 2;
-    const char *f = getenv("BLAS3_TRSM_SLAB_MIN");
-    const int64_t w = f ? atoll(f) : 0;
-    mn = (w >= 256) ? w / 256 * 256 : 2048;
-  }
-  return imax(1, imin(mx, other / mn));
+  const int64_t mn = opt(BLAS3_OPT_TRSM_SLAB_MIN) / 256 * 256;
+  return imax(1, imin(opt(BLAS3_OPT_TRSM_SLABS), other / mn));
 }
 static inline int64_t align_down(int64_t v, int64_t a) { return v / a * a; }
-// SMs the first panel's sweep kernels leave free for its doubling chain;
-// env BLAS3_TRSM_RESERVE overrides it (experiments)
-static int64_t trsm_reserve() {
-  static int64_t r = -1;
-  if (r < 0) {
-    const char *e = getenv("BLAS3_TRSM_RESERVE");
-    r = e ? imax(0, atoll(e)) : 32;
-  }
-  return r;
-}
-// width below which the first panel's geometric halving stops (a power of
-// two in [128, NBO]); env BLAS3_TRSM_GEO_LEAF overrides it (experiments)
-static int64_t trsm_geo_leaf() {
-  static int64_t w = -1;
-  if (w < 0) {
-    const char *e = getenv("BLAS3_TRSM_GEO_LEAF");
-    const int64_t v = e ? atoll(e) : 0;
-    w = (v >= 128 && (v & (v - 1)) == 0) ? v : 256;
-  }
-  return w;
-}
+// SMs the first panel's sweep kernels leave free for its doubling chain
+static int64_t trsm_reserve() { return opt(BLAS3_OPT_TRSM_RESERVE); }
+// width below which the first panel's geometric halving stops (power of 2)
+static int64_t trsm_geo_leaf() { return opt(BLAS3_OPT_TRSM_GEO_LEAF); }
 
 int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t n, float alpha,
                 const float *A, int64_t lda, float *B, int64_t ldb, blas3_stream_t stream) {
@@ -504,8 +592,8 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   cudaStream_t s = (cudaStream_t)stream;
   if (alpha == 0.f) return finish(launch_scale(B, ldb, m, n, 0.f, 0, s) ? BLAS3_ERR_CUDA : 0);
 
-  const bool left = up(side) == 'L', lower = up(uplo) == 'L', ta = up(transa) != 'N',
-             unit = up(diag) == 'U';
+  const bool left = up(side) == 'L';
+  bool lower = up(uplo) == 'L', ta = up(transa) != 'N', unit = up(diag) == 'U';
   const bool lower_op = lower != ta;               // op(A) = L (true) or L^T (false)
   const int64_t nt = left ? m : n;                 // order of A
   const int64_t NBO = trsm_nbo();
@@ -513,15 +601,29 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   const int64_t other = left ? n : m;              // RHS extent
   const bool forward = left ? lower_op : !lower_op;
 
+  // GM_map canonicalisation for transposed variants: op(A) is materialised
+  // (MN-major, zeros in the blank triangle, unit diagonal written), and the
+  // solve runs on it as a non-transposed triangle with the same op(A) -- the
+  // sweep's update GEMMs then stage op(A) blocks in the MN-major orientation.
+  Scratch Aop;
+  size_t aop_bytes = 0;
+  if (ta && tensor_mode() && use_gm_map(nt, other, BLAS3_OPT_GM_MIN_TRSM)) {
+    const int64_t ldw = ld4(nt);
+    aop_bytes = (size_t)ldw * nt * sizeof(float);
+    if ((rc = get_scratch(Aop, aop_bytes, s))) return rc;
+    if (launch_materialize(Aop.p, ldw, A, lda, nt, nt, MAT_TRI, lower, ta, unit, s)) return BLAS3_ERR_CUDA;
+    A = Aop.p; lda = ldw; lower = lower_op; ta = false; unit = false;
+  }
+
   const size_t d_bytes = (size_t)npanel * NBO * NBO * sizeof(float);
   // doubling scratch: nt/2sz pairs x sz^2 floats at the widest level
   const size_t t_rest = (size_t)nt * (NBO / 4), t_first = (size_t)NBO * NBO / 4;
   const size_t t_bytes = (t_rest + t_first) * sizeof(float);
   const size_t w_bytes = (size_t)NBO * other * sizeof(float);        // one solved panel
   Scratch D, Tw, W;
-  if ((rc = get_scratch(D, d_bytes, s))) return rc;
-  if ((rc = get_scratch(Tw, t_bytes, s, d_bytes))) return rc;
-  if ((rc = get_scratch(W, w_bytes, s, d_bytes + t_bytes))) return rc;
+  if ((rc = get_scratch(D, d_bytes, s, aop_bytes))) return rc;
+  if ((rc = get_scratch(Tw, t_bytes, s, aop_bytes + d_bytes))) return rc;
+  if ((rc = get_scratch(W, w_bytes, s, aop_bytes + d_bytes + t_bytes))) return rc;
 
   std::lock_guard<std::mutex> lk(g_trsm_mu);          // the per-device side streams
   TrsmStreams *ts = trsm_streams();

@@ -104,6 +104,88 @@ int launch_copy(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t 
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
 
+// ---------------------------------------------------------------- GM_map materialisation
+// The paper's Adaptor rule 2 ("GM_map"): the structured operand is
+// rewritten once in global memory in the orientation the GEMM kernel stages
+// best (MN-major, i.e. plain column-major), so the hot kernel runs its dense
+// / zero-blank path.  dst(r, c), 0 <= r < rows, 0 <= c < cols, is
+//   MAT_TRANS : src(c, r)
+//   MAT_SYM   : the stored triangle (lower: r >= c) selected, else its mirror
+//               (selection, never src + src^T - diag, reading Q7)
+//   MAT_TRI   : op(T)(r, c) with T the stored triangle, 0 in the blank part,
+//               1 on the diagonal when unit (the stored diagonal is not read)
+// 32 x 32 output tiles through shared memory: the direct and the mirrored
+// source tiles are each read with coalesced column accesses, and only the
+// one(s) the tile needs (both only on diagonal tiles).  HBM-bound: <= 4 B
+// read + 4 B written per element.
+namespace {
+constexpr int MT = 32, MR = 8;     // tile, rows of threads (256 threads)
+}
+__global__ void __launch_bounds__(MT * MR)
+materialize_kernel(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t rows,
+                   int64_t cols, int mode, int lower, int trans, int unit) {
+  __shared__ float dir[MT][MT + 1], mir[MT][MT + 1];
+  const int64_t r0 = (int64_t)blockIdx.x * MT, c0 = (int64_t)blockIdx.y * MT;
+  const int tx = threadIdx.x % MT, ty = threadIdx.x / MT;
+  // which source tiles are referenced: element (r, c) reads src(i, j) with
+  // (i, j) = (r, c) ("direct") or (c, r) ("mirrored")
+  bool need_dir, need_mir;
+  if (mode == MAT_TRANS) { need_dir = false; need_mir = true; }
+  else {
+    // the stored triangle decides per element; a tile strictly below (r > c
+    // everywhere) or above the diagonal needs one side only
+    const bool below = r0 >= c0 + MT, above = c0 >= r0 + MT;
+    const bool stored_below = mode == MAT_SYM ? lower : (lower != trans);   // TRI: op(T) nonzero side
+    if (mode == MAT_SYM) {
+      need_dir = !(below ? !lower : above ? lower : false);
+      need_mir = !(below ? lower : above ? !lower : false);
+    } else {
+      // op(T)(r,c) = trans ? T(c,r) : T(r,c); nonzero iff (r >= c) == stored_below
+      const bool blank = stored_below ? above : below;
+      need_dir = !trans && !blank;
+      need_mir = trans && !blank;
+    }
+  }
+  if (need_dir) {
+    for (int rr = ty; rr < MT; rr += MR) {        // warp = 32 consecutive rows of one column
+      const int64_t c = c0 + rr, r = r0 + tx;
+      dir[rr][tx] = (r < rows && c < cols) ? __ldg(src + r + c * lds) : 0.f;
+    }
+  }
+  if (need_mir) {
+    for (int rr = ty; rr < MT; rr += MR) {        // src(c, r) for r = r0 + rr: column r0+rr of src
+      const int64_t i = c0 + tx, j = r0 + rr;
+      mir[tx][rr] = (j < rows && i < cols) ? __ldg(src + i + j * lds) : 0.f;   // mir[c][r] = src(c, r)
+    }
+  }
+  __syncthreads();
+  for (int cc = ty; cc < MT; cc += MR) {
+    const int64_t r = r0 + tx, c = c0 + cc;
+    if (r >= rows || c >= cols) continue;
+    float v;
+    if (mode == MAT_TRANS) v = mir[cc][tx];
+    else if (mode == MAT_SYM) {
+      const bool direct = lower ? (r >= c) : (r <= c);
+      v = direct ? dir[cc][tx] : mir[cc][tx];
+    } else {
+      const int64_t i = trans ? c : r, j = trans ? r : c;        // T(i, j)
+      const bool nz = lower ? (i >= j) : (i <= j);
+      v = !nz ? 0.f : (unit && i == j) ? 1.f : (trans ? mir[cc][tx] : dir[cc][tx]);
+    }
+    dst[r + c * ldd] = v;
+  }
+}
+
+int launch_materialize(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t rows,
+                       int64_t cols, int mode, int lower, int trans, int unit, cudaStream_t s) {
+  if (rows <= 0 || cols <= 0) return 0;
+  const dim3 g((unsigned)cdiv(rows, MT), (unsigned)cdiv(cols, MT));
+  if (g.y > 65535) return -1;
+  materialize_kernel<<<g, MT * MR, 0, s>>>(dst, ldd, src, lds, rows, cols, mode, lower, trans, unit);
+  note_launch();
+  return cudaGetLastError() == cudaSuccess ? 0 : -1;
+}
+
 // ---------------------------------------------------------------- TRSM diag inverse
 namespace {
 constexpr int DNB = 128;          // diagonal block size (4 x 32)

@@ -8,6 +8,7 @@
 namespace blas3 {
 
 void note_launch(int path = 2);      // host-side launch counter (blas3_launch_count[_by_path])
+int64_t opt(int key);                // tuning option (blas3_set_option / environment)
 
 // Structured GEMM kernels (all routines canonicalise to a Problem).
 int launch_simt(const Problem &P, cudaStream_t s, int num_sms);
@@ -21,6 +22,10 @@ int launch_scale(float *C, int64_t ldc, int64_t m, int64_t n, float beta, int tr
                  cudaStream_t s);                       // C <- beta*C (beta=0 -> 0), tri: 0/1 lower/2 upper
 int launch_copy(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t m, int64_t n,
                 cudaStream_t s);
+// GM_map (paper Adaptor rule 2): dst (rows x cols, column-major) <- op(src)
+enum MatMode : int { MAT_TRANS = 0, MAT_SYM = 1, MAT_TRI = 2 };
+int launch_materialize(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t rows,
+                       int64_t cols, int mode, int lower, int trans, int unit, cudaStream_t s);
 
 // TRSM diagonal blocks: for every 128 x 128 diagonal block b of L, where L
 // is the stored triangle of A brought to lower form (L(i,j) = A(i,j) if A is

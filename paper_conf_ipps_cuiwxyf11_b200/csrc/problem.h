@@ -80,6 +80,9 @@ struct Problem {
   // launch at most this many SMs' worth of CTAs (0: all).  The STRSM driver
   // leaves SMs free for its latency-bound side-stream kernels this way.
   int32_t max_sms;
+  // tcgen05 path: 3 = 3xTF32 (lo*hi + hi*lo + hi*hi, fp32-accurate, default),
+  // 1 = 1xTF32 (hi*hi only: the BLAS3_MATH_1XTF32 fast mode, TF32 accuracy)
+  int32_t passes;
 };
 
 HD int64_t batch_off(const BatchStride &s, int64_t b, int64_t per) {

@@ -35,6 +35,7 @@
 #include <stdlib.h>
 #include <string.h>
 
+#include "../../include/blas3.h"
 #include "kernels.h"
 #include "tc_ptx.h"
 
@@ -605,7 +606,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
               for (int k8 = 0; k8 < BK / 8; ++k8) {
                 const uint64_t ah = op_desc(hiA, si.layA, k8), al = op_desc(loA, si.layA, k8);
                 const uint64_t bh = op_desc(hiB, si.layB, k8), bl = op_desc(loB, si.layB, k8);
-                const bool one = P.dbg & 2;
+                const bool one = (P.dbg & 2) || P.passes == 1;
                 if (P.dbg & 8) continue;                       // diag: no MMAs
                 if constexpr (CG == 1) {
                   if (!one) ptx::mma_tf32_ss(d_tmem, al, bh, idesc, accumulate);
@@ -680,7 +681,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           }
           if (fix) ptx::named_bar_sync(1, TR_THREADS);
           ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
-          if (!(P.dbg & 1)) {
+          if (!(P.dbg & 1) && P.passes != 1) {
             split_pass(rb.A, lo[ls].A, G::A_BYTES, tt);
             split_pass(rb.B, lo[ls].B, G::B_BYTES, tt);
           }
@@ -918,11 +919,7 @@ bool tc_eligible(const Problem &P) {
 // pair at least one tile, else the single-CTA kernel (more, smaller tiles,
 // dynamic scheduling).  BLAS3_TC_CTA=1|2 forces one (tests).
 static int choose_cg(const Problem &P, int num_sms) {
-  static int forced = -1;
-  if (forced < 0) {
-    const char *e = getenv("BLAS3_TC_CTA");
-    forced = (e && e[0] == '1') ? 1 : (e && e[0] == '2') ? 2 : 0;
-  }
+  const int forced = (int)opt(BLAS3_OPT_TC_CTA);
   if (forced) return forced;
   const int64_t nb = P.nbatch > 1 ? P.nbatch : 1;
   return Tiles<Geo<2>::TM, BN>::count(P) * nb >= num_sms / 2 ? 2 : 1;
@@ -962,8 +959,7 @@ static int launch_cg(TcParams &prm, cudaStream_t stream, int num_sms) {
   // programmatic dependent launch: this grid's prologue may overlap the tail
   // of the previous kernel on the stream (the kernel waits before touching
   // global memory).  BLAS3_PDL=0 disables it (experiments).
-  static int pdl = -1;
-  if (pdl < 0) { const char *e = getenv("BLAS3_PDL"); pdl = (e && e[0] == '0') ? 0 : 1; }
+  const bool pdl = opt(BLAS3_OPT_PDL) != 0;
   attrs[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attrs[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attrs;
@@ -1042,9 +1038,7 @@ static void plan_split(TcParams &prm, int num_sms, cudaStream_t stream) {
   const int64_t tiles_per = Tiles<Geo<CG>::TM, BN>::count(P), T = tiles_per * nb;
   prm.tiles_per = tiles_per;
   prm.nitems = T; prm.khead = T; prm.ksplit = 1;
-  static int enabled = -1;
-  if (enabled < 0) { const char *e = getenv("BLAS3_TC_SPLIT"); enabled = (e && e[0] == '0') ? 0 : 1; }
-  if (!enabled || T == 0) return;
+  if (!opt(BLAS3_OPT_TC_SPLIT) || T == 0) return;
   const int64_t U = imin(T, (int64_t)(num_sms / CG));
   const int64_t R = T < (int64_t)(num_sms / CG) ? T : T % U;
   if (R == 0 || T >= 8 * U) return;
@@ -1078,8 +1072,7 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
     prm.P.dbg = dbg;
   }
   const int cg = choose_cg(prm.P, num_sms);
-  static int dyn = -1;
-  if (dyn < 0) { const char *e = getenv("BLAS3_TC_STATIC"); dyn = (e && e[0] == '1') ? 0 : 1; }
+  const bool dyn = opt(BLAS3_OPT_TC_STATIC) == 0;
   if (cg == 2) plan_split<2>(prm, num_sms, stream); else plan_split<1>(prm, num_sms, stream);
   if (dyn) {
     const int64_t tiles = prm.nitems;

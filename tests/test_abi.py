@@ -163,3 +163,22 @@ def test_math_mode_and_misc(lib):
     assert lib.blas3_error_string(-2).decode().startswith("current device")
     assert lib.blas3_error_string(5).decode().startswith("invalid argument")
     assert lib.launch_count() >= 0
+
+
+def test_options_roundtrip_and_validation(lib):
+    """Tuning options (blas3_set_option): defaults, valid updates, rejected
+    values leave the option unchanged, unknown keys report INT64_MIN / 1."""
+    assert lib.get_option("trsm_nb") in (128, 256, 512, 1024, 2048, 4096, 8192)
+    with lib.options(trsm_nb=1024, gm_map=1, tc_cta=2):
+        assert lib.get_option("trsm_nb") == 1024
+        assert lib.get_option("gm_map") == 1
+        assert lib.get_option("tc_cta") == 2
+    assert lib.get_option("gm_map") in (-1, 0, 1)
+    old = lib.get_option("trsm_nb")
+    for bad in (100, 3000, 16384, -1):            # not a power of two in [128, 8192]
+        assert lib.blas3_set_option(lib.OPTIONS["trsm_nb"], bad) == 1
+    assert lib.get_option("trsm_nb") == old
+    assert lib.blas3_set_option(lib.OPTIONS["tc_cta"], 3) == 1
+    assert lib.blas3_set_option(99, 0) == 1
+    assert lib.blas3_get_option(99) == -(2 ** 63)
+    assert len(lib.OPTIONS) == 14

@@ -2,8 +2,10 @@
 load (they are cached once per process, hence subprocesses): the CTA-pair
 tcgen05 kernel (BLAS3_TC_CTA=2, cta_group::2) and the static tile schedule
 (BLAS3_TC_STATIC=1), the single-CTA kernel (BLAS3_TC_CTA=1; the default
-picks the pair kernel for large problems), and whole tiles only
-(BLAS3_TC_SPLIT=0: no k-sliced tail).  Each child process runs a representative subset of the
+picks the pair kernel for large problems), whole tiles only
+(BLAS3_TC_SPLIT=0: no k-sliced tail), and the GM_map adaptor forced on at
+every size (BLAS3_GM_MAP=1: transposed / symmetric / triangular operands
+materialised in global memory first, the default only for large problems).  Each child process runs a representative subset of the
 parity suite (every routine family, both transposes/sides) on that variant."""
 import os
 import subprocess
@@ -16,8 +18,10 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 @pytest.mark.parametrize("env", [{"BLAS3_TC_CTA": "1"}, {"BLAS3_TC_CTA": "2"}, {"BLAS3_TC_STATIC": "1"},
-                                 {"BLAS3_TC_SPLIT": "0"}, {"BLAS3_TC_CTA": "1", "BLAS3_TC_SPLIT": "0"}],
-                         ids=["single_cta", "cta_pair", "static_schedule", "no_split", "single_cta_no_split"])
+                                 {"BLAS3_TC_SPLIT": "0"}, {"BLAS3_TC_CTA": "1", "BLAS3_TC_SPLIT": "0"},
+                                 {"BLAS3_GM_MAP": "1"}],
+                         ids=["single_cta", "cta_pair", "static_schedule", "no_split", "single_cta_no_split",
+                              "gm_map"])
 def test_variant_subset(env):
     import torch
     if not torch.cuda.is_available():
