@@ -114,65 +114,104 @@ int launch_copy(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t 
 //               (selection, never src + src^T - diag, reading Q7)
 //   MAT_TRI   : op(T)(r, c) with T the stored triangle, 0 in the blank part,
 //               1 on the diagonal when unit (the stored diagonal is not read)
-// 32 x 32 output tiles through shared memory: the direct and the mirrored
-// source tiles are each read with coalesced column accesses, and only the
-// one(s) the tile needs (both only on diagonal tiles).  HBM-bound: <= 4 B
-// read + 4 B written per element.
+// 64 x 64 output tiles through shared memory: the direct and the mirrored
+// source tiles are each read with coalesced column accesses (16-byte vectors
+// when the source allows), and only the one(s) the tile needs (both only on
+// diagonal tiles); 16 loads per thread are in flight before the exchange.
+// HBM-bound: <= 4 B read + 4 B written per element.
 namespace {
-constexpr int MT = 32, MR = 8;     // tile, rows of threads (256 threads)
+constexpr int MT = 64, MTH = 256, MPAD = MT + 4, MPADM = MT + 1;   // float4 rows / conflict-free transpose
 }
-__global__ void __launch_bounds__(MT * MR)
+template <bool VEC>
+__global__ void __launch_bounds__(MTH)
 materialize_kernel(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t rows,
                    int64_t cols, int mode, int lower, int trans, int unit) {
-  __shared__ float dir[MT][MT + 1], mir[MT][MT + 1];
+  __shared__ __align__(16) float dir[MT][MPAD];   // dir[c][r] = src(r0 + r, c0 + c)
+  __shared__ float mir[MT][MPADM];                // mir[c][r] = src(c0 + c, r0 + r)
   const int64_t r0 = (int64_t)blockIdx.x * MT, c0 = (int64_t)blockIdx.y * MT;
-  const int tx = threadIdx.x % MT, ty = threadIdx.x / MT;
-  // which source tiles are referenced: element (r, c) reads src(i, j) with
-  // (i, j) = (r, c) ("direct") or (c, r) ("mirrored")
+  const int t = threadIdx.x;
   bool need_dir, need_mir;
   if (mode == MAT_TRANS) { need_dir = false; need_mir = true; }
   else {
-    // the stored triangle decides per element; a tile strictly below (r > c
-    // everywhere) or above the diagonal needs one side only
+    // a tile strictly below (r > c everywhere) or above the diagonal needs one side only
     const bool below = r0 >= c0 + MT, above = c0 >= r0 + MT;
-    const bool stored_below = mode == MAT_SYM ? lower : (lower != trans);   // TRI: op(T) nonzero side
     if (mode == MAT_SYM) {
       need_dir = !(below ? !lower : above ? lower : false);
       need_mir = !(below ? lower : above ? !lower : false);
     } else {
-      // op(T)(r,c) = trans ? T(c,r) : T(r,c); nonzero iff (r >= c) == stored_below
-      const bool blank = stored_below ? above : below;
+      // op(T)(r,c) = trans ? T(c,r) : T(r,c), nonzero iff (r >= c) == (lower != trans)
+      const bool blank = (lower != trans) ? above : below;
       need_dir = !trans && !blank;
       need_mir = trans && !blank;
     }
   }
+  // thread t covers 4 consecutive elements (e4 .. e4+3) of "line" ln, 4 times
   if (need_dir) {
-    for (int rr = ty; rr < MT; rr += MR) {        // warp = 32 consecutive rows of one column
-      const int64_t c = c0 + rr, r = r0 + tx;
-      dir[rr][tx] = (r < rows && c < cols) ? __ldg(src + r + c * lds) : 0.f;
+#pragma unroll
+    for (int it = 0; it < 4; ++it) {
+      const int idx = t + it * MTH, ln = idx / 16, e4 = (idx % 16) * 4;   // column c0+ln, rows r0+e4..
+      const int64_t r = r0 + e4, c = c0 + ln;
+      float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (c < cols) {
+        const float *p = src + r + c * lds;
+        if (VEC && r + 3 < rows) v = __ldg(reinterpret_cast<const float4 *>(p));
+        else {
+          if (r < rows) v.x = __ldg(p);
+          if (r + 1 < rows) v.y = __ldg(p + 1);
+          if (r + 2 < rows) v.z = __ldg(p + 2);
+          if (r + 3 < rows) v.w = __ldg(p + 3);
+        }
+      }
+      *reinterpret_cast<float4 *>(&dir[ln][e4]) = v;
     }
   }
   if (need_mir) {
-    for (int rr = ty; rr < MT; rr += MR) {        // src(c, r) for r = r0 + rr: column r0+rr of src
-      const int64_t i = c0 + tx, j = r0 + rr;
-      mir[tx][rr] = (j < rows && i < cols) ? __ldg(src + i + j * lds) : 0.f;   // mir[c][r] = src(c, r)
+#pragma unroll
+    for (int it = 0; it < 4; ++it) {
+      const int idx = t + it * MTH, ln = idx / 16, e4 = (idx % 16) * 4;   // src column r0+ln, rows c0+e4..
+      const int64_t j = r0 + ln, i = c0 + e4;
+      float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (j < rows) {
+        const float *p = src + i + j * lds;
+        if (VEC && i + 3 < cols) v = __ldg(reinterpret_cast<const float4 *>(p));
+        else {
+          if (i < cols) v.x = __ldg(p);
+          if (i + 1 < cols) v.y = __ldg(p + 1);
+          if (i + 2 < cols) v.z = __ldg(p + 2);
+          if (i + 3 < cols) v.w = __ldg(p + 3);
+        }
+      }
+      mir[e4][ln] = v.x; mir[e4 + 1][ln] = v.y; mir[e4 + 2][ln] = v.z; mir[e4 + 3][ln] = v.w;
     }
   }
   __syncthreads();
-  for (int cc = ty; cc < MT; cc += MR) {
-    const int64_t r = r0 + tx, c = c0 + cc;
-    if (r >= rows || c >= cols) continue;
-    float v;
-    if (mode == MAT_TRANS) v = mir[cc][tx];
-    else if (mode == MAT_SYM) {
-      const bool direct = lower ? (r >= c) : (r <= c);
-      v = direct ? dir[cc][tx] : mir[cc][tx];
-    } else {
-      const int64_t i = trans ? c : r, j = trans ? r : c;        // T(i, j)
-      const bool nz = lower ? (i >= j) : (i <= j);
-      v = !nz ? 0.f : (unit && i == j) ? 1.f : (trans ? mir[cc][tx] : dir[cc][tx]);
+#pragma unroll
+  for (int it = 0; it < 4; ++it) {
+    const int idx = t + it * MTH, ln = idx / 16, e4 = (idx % 16) * 4;       // column c0+ln, rows r0+e4..
+    const int64_t c = c0 + ln;
+    if (c >= cols) continue;
+    float v[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int64_t r = r0 + e4 + q;
+      if (mode == MAT_TRANS) v[q] = mir[ln][e4 + q];
+      else if (mode == MAT_SYM) {
+        const bool direct = lower ? (r >= c) : (r <= c);
+        v[q] = direct ? dir[ln][e4 + q] : mir[ln][e4 + q];
+      } else {
+        const int64_t ti = trans ? c : r, tj = trans ? r : c;     // T(ti, tj)
+        const bool nz = lower ? (ti >= tj) : (ti <= tj);
+        v[q] = !nz ? 0.f : (unit && ti == tj) ? 1.f : (trans ? mir[ln][e4 + q] : dir[ln][e4 + q]);
+      }
     }
-    dst[r + c * ldd] = v;
+    const int64_t r = r0 + e4;
+    float *p = dst + r + c * ldd;
+    if (VEC && r + 3 < rows) *reinterpret_cast<float4 *>(p) = make_float4(v[0], v[1], v[2], v[3]);
+    else {
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        if (r + q < rows) p[q] = v[q];
+    }
   }
 }
 
@@ -181,7 +220,9 @@ int launch_materialize(float *dst, int64_t ldd, const float *src, int64_t lds, i
   if (rows <= 0 || cols <= 0) return 0;
   const dim3 g((unsigned)cdiv(rows, MT), (unsigned)cdiv(cols, MT));
   if (g.y > 65535) return -1;
-  materialize_kernel<<<g, MT * MR, 0, s>>>(dst, ldd, src, lds, rows, cols, mode, lower, trans, unit);
+  const bool vec = ((uintptr_t)dst % 16 == 0) && ((uintptr_t)src % 16 == 0) && ldd % 4 == 0 && lds % 4 == 0;
+  if (vec) materialize_kernel<true><<<g, MTH, 0, s>>>(dst, ldd, src, lds, rows, cols, mode, lower, trans, unit);
+  else materialize_kernel<false><<<g, MTH, 0, s>>>(dst, ldd, src, lds, rows, cols, mode, lower, trans, unit);
   note_launch();
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
