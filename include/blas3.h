@@ -166,6 +166,11 @@ int blas3_get_math_mode(void);
  *                          the panel-inverse doubling chain, 0..#SMs/2 (32)
  *   BLAS3_OPT_TRSM_GEO_LEAF [BLAS3_TRSM_GEO_LEAF] the first panel is halved down to
  *                          this width: power of 2 in [128, 8192] (256)
+ *   BLAS3_OPT_TRSM_FUSED   [BLAS3_TRSM_FUSED] 1: the whole STRSM (panel-inverse
+ *                          doubling + sweep) as one persistent dependency-driven
+ *                          launch when it fits; 0 (default): one launch per step
+ *                          on the caller's and the side streams (measured equal
+ *                          or faster on B200 at N = 8192)
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */
@@ -174,7 +179,8 @@ enum {
     BLAS3_OPT_GM_MIN_TRMM = 3, BLAS3_OPT_GM_MIN_TRSM = 4, BLAS3_OPT_TC_CTA = 5,
     BLAS3_OPT_TC_SPLIT = 6, BLAS3_OPT_TC_STATIC = 7, BLAS3_OPT_PDL = 8,
     BLAS3_OPT_TRSM_NB = 9, BLAS3_OPT_TRSM_SLABS = 10, BLAS3_OPT_TRSM_SLAB_MIN = 11,
-    BLAS3_OPT_TRSM_RESERVE = 12, BLAS3_OPT_TRSM_GEO_LEAF = 13, BLAS3_OPT_COUNT = 14
+    BLAS3_OPT_TRSM_RESERVE = 12, BLAS3_OPT_TRSM_GEO_LEAF = 13, BLAS3_OPT_TRSM_FUSED = 14,
+    BLAS3_OPT_COUNT = 15
 };
 int blas3_set_option(int key, int64_t value);
 int64_t blas3_get_option(int key);

@@ -10,6 +10,7 @@
 #include <atomic>
 #include <functional>
 #include <mutex>
+#include <vector>
 
 #include "../../include/blas3.h"
 #include "kernels.h"
@@ -40,6 +41,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TRSM_SLAB_MIN", 2048, 256, int64_t(1) << 40, false},
     {"BLAS3_TRSM_RESERVE", 32, 0, 74, false},
     {"BLAS3_TRSM_GEO_LEAF", 256, 128, 8192, true},
+    {"BLAS3_TRSM_FUSED", 0, 0, 1, false},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;
@@ -483,16 +485,15 @@ static int64_t trsm_nbo() { return opt(BLAS3_OPT_TRSM_NB); }
 
 // Doubling levels 128 -> NBO for the panels of the order-nt triangle whose
 // top-left corner is A (and whose panel inverses start at D); the 128-block
-// inverses are already on D's diagonal.  Tw: (nt / 2sz) x sz^2 floats.
-static int trsm_panel_doubling(const float *A, int64_t lda, int64_t nt, bool lower, float *D,
-                               float *Tw, cudaStream_t s, int sms, cudaEvent_t *ev_lvl) {
+// inverses are already on D's diagonal.  Tw: (nt / 2sz) x sz^2 + sz^2 floats.
+// Builds the problems in order: per level, T = L21 inv(L11) (step 1) then
+// X21 = -inv(L22) T (step 2), for the full pairs and a ragged last pair.
+struct LevelProblem { int lvl, step; Problem P; };
+static void trsm_doubling_problems(const float *A, int64_t lda, int64_t nt, bool lower, float *D,
+                                   float *Tw, std::vector<LevelProblem> &out) {
   const int64_t NBO = trsm_nbo();
-  int rc;
   for (int64_t sz = 128, lvl = 0; sz < NBO; sz *= 2, ++lvl) {
-    if (sz >= nt) {                    // no pair reaches this level: nothing left to do
-      if (cudaEventRecord(ev_lvl[lvl], s) != cudaSuccess) return BLAS3_ERR_CUDA;
-      continue;
-    }
+    if (sz >= nt) continue;            // no pair reaches this level
     // pair b covers rows/cols [o, o + 2 sz) of L, o = 2 sz b; L21 = L[o+sz.., o..]
     const int64_t per = NBO / (2 * sz);
     const int64_t full = nt / (2 * sz);                    // pairs entirely inside L
@@ -505,8 +506,9 @@ static int trsm_panel_doubling(const float *A, int64_t lda, int64_t nt, bool low
       if (cnt == 0) continue;
       const int64_t o = pass == 0 ? 0 : full * 2 * sz;
       const int64_t m2 = pass == 0 ? sz : rag_rows;          // rows of L21 / order of L22
+      float *T = Tw + (pass == 0 ? 0 : full * sz * sz);       // the ragged pair's own slot
       // T = L21 * inv(L11): Xa = L21 (m2 x sz), Xb(c,k) = inv(L11)(k,c) (lower -> TRI swap)
-      Problem P1 = problem(m2, sz, 1.f, 0.f, nullptr, 0, Tw, m2);
+      Problem P1 = problem(m2, sz, 1.f, 0.f, nullptr, 0, T, m2);
       P1.seg[0].a = dense(l21(o), lda, !lower);
       P1.seg[0].b = tri_zeroed(dblk(o), NBO, true, true);
       P1.seg[0].K = sz;
@@ -514,19 +516,31 @@ static int trsm_panel_doubling(const float *A, int64_t lda, int64_t nt, bool low
       P1.bs_a = {per * 2 * sz * (1 + lda), 2 * sz * (1 + lda)};
       P1.bs_b = {NBO * NBO, 2 * sz * (1 + NBO)};
       P1.bs_c = {per * sz * sz, sz * sz};
-      if ((rc = run_problem(P1, s, sms))) return rc;
+      out.push_back({(int)lvl, 1, P1});
       // X21 = -inv(L22) * T: Xa = inv(L22) (lower TRI), Xb(c,k) = T(k,c) (kr)
       Problem P2 = problem(m2, sz, -1.f, 0.f, nullptr, 0, dblk(o) + sz, NBO);
       P2.seg[0].a = tri_zeroed(dblk(o) + sz * (1 + NBO), NBO, true, false);
-      P2.seg[0].b = dense(Tw, m2, true);
+      P2.seg[0].b = dense(T, m2, true);
       P2.seg[0].K = m2;
       P2.nbatch = cnt; P2.per = per;
       P2.bs_a = {NBO * NBO, 2 * sz * (1 + NBO)};
       P2.bs_b = {per * sz * sz, sz * sz};
       P2.bs_c = {NBO * NBO, 2 * sz * (1 + NBO)};
-      if ((rc = run_problem(P2, s, sms))) return rc;
+      out.push_back({(int)lvl, 2, P2});
     }
-    // inverses of every aligned 2sz-block are complete
+  }
+}
+// Runs the doubling on stream s, recording ev_lvl[l] once the inverses of
+// every aligned 2^(l+8)-block are complete.
+static int trsm_panel_doubling(const float *A, int64_t lda, int64_t nt, bool lower, float *D,
+                               float *Tw, cudaStream_t s, int sms, cudaEvent_t *ev_lvl) {
+  std::vector<LevelProblem> probs;
+  trsm_doubling_problems(A, lda, nt, lower, D, Tw, probs);
+  size_t i = 0;
+  int rc;
+  for (int64_t sz = 128, lvl = 0; sz < trsm_nbo(); sz *= 2, ++lvl) {
+    for (; i < probs.size() && probs[i].lvl == lvl; ++i)
+      if ((rc = run_problem(probs[i].P, s, sms))) return rc;
     if (cudaEventRecord(ev_lvl[lvl], s) != cudaSuccess) return BLAS3_ERR_CUDA;
   }
   return 0;
@@ -580,6 +594,203 @@ static int64_t trsm_reserve() { return opt(BLAS3_OPT_TRSM_RESERVE); }
 // width below which the first panel's geometric halving stops (power of 2)
 static int64_t trsm_geo_leaf() { return opt(BLAS3_OPT_TRSM_GEO_LEAF); }
 
+// ---- fused STRSM: the whole solve as ONE persistent launch (after the
+// 128-block inverses).  The doubling levels and the sweep are phases of one
+// grid; a sweep tile waits only for the previous sweep phase ON ITS OWN SLAB
+// (256 right-hand-side columns for side=L, rows for side=R) and a leaf for the
+// doubling level that built its inverse, so the solve runs as a wavefront
+// over the independent right-hand sides: no kernel boundaries, no launch
+// tails, and the latency-bound first panel overlaps the doubling.  Every
+// update writes the first panel of its output range to W (fixed leading
+// dimension), every later leaf reads W and writes B, and the first leaf (at
+// most one 256-row tile per slab) runs in place -- no copy-backs.
+// Returns 1 (not fusable: the caller runs the multi-launch path) before
+// anything is enqueued, 0 on success, < 0 on a CUDA error.
+struct TrsmGeom {
+  bool left, lower, ta, unit, lower_op, forward;
+  int64_t m, n, nt, NBO, npanel, other;
+  float alpha;
+  const float *A; int64_t lda;
+  float *B; int64_t ldb;
+  float *D, *Tw, *W;
+};
+static int strsm_fused(const TrsmGeom &g, cudaStream_t s, int sms) {
+  const int64_t NBO = g.NBO, nt = g.nt;
+  const int64_t ldw = g.left ? NBO : g.m;              // W(r, c) = W[r + c * ldw]
+  std::vector<LevelProblem> lv;
+  trsm_doubling_problems(g.A, g.lda, nt, g.lower, g.D, g.Tw, lv);
+  int nlvl = 0;
+  for (int64_t sz = 128; sz < NBO; sz *= 2) ++nlvl;
+
+  std::vector<FusedPhase> ph;
+  bool ok = true;
+  uint32_t lvl_mask[MAX_LEVELS] = {};                  // phases (step 2) completing level l
+  int emitted_lvl = -1;
+  // Exact slab dependencies from each sweep phase's accesses: rows (L) /
+  // columns (R) of B read and written, and whether it reads / writes W.  A
+  // phase waits (on its slab) for every earlier sweep phase it conflicts with
+  // (read-after-write, write-after-read, write-after-write).
+  struct Acc { int idx; int64_t r_lo[2], r_hi[2], w_lo, w_hi; bool rw, ww; };
+  std::vector<Acc> acc;
+  auto overlap = [](int64_t a0, int64_t a1, int64_t b0, int64_t b1) { return a0 < b1 && b0 < a1; };
+  auto add = [&](const Problem &P, uint32_t full, uint32_t slab) -> int {
+    if ((int)ph.size() >= MAX_FUSED_PHASES) { ok = false; return 0; }
+    FusedPhase f;
+    f.P = P; f.dep_full = (int32_t)full; f.dep_slab = (int32_t)slab; f.slab_m = g.left ? 0 : 1;
+    ph.push_back(f);
+    return (int)ph.size() - 1;
+  };
+  auto emit_level = [&](int l) {                        // step 1 after level l-1, step 2 after step 1
+    uint32_t step1 = 0;
+    for (const LevelProblem &q : lv)
+      if (q.lvl == l && q.step == 1) step1 |= 1u << add(q.P, l > 0 ? lvl_mask[l - 1] : 0u, 0u);
+    for (const LevelProblem &q : lv)
+      if (q.lvl == l && q.step == 2) lvl_mask[l] |= 1u << add(q.P, step1, 0u);
+  };
+  auto levels_upto = [&](int l) {
+    for (; emitted_lvl < l && emitted_lvl + 1 < nlvl; ) emit_level(++emitted_lvl);
+  };
+  auto sweep = [&](const Problem &P, int need, Acc a) {
+    levels_upto(need);
+    const uint32_t full = need >= 0 ? lvl_mask[need] : 0u;
+    uint32_t slab = 0;
+    for (const Acc &q : acc) {
+      bool c = (q.ww && a.rw) || (q.rw && a.ww) || (q.ww && a.ww);
+      for (int i = 0; i < 2 && !c; ++i) {
+        c = overlap(q.w_lo, q.w_hi, a.r_lo[i], a.r_hi[i]) || overlap(q.r_lo[i], q.r_hi[i], a.w_lo, a.w_hi);
+      }
+      c = c || overlap(q.w_lo, q.w_hi, a.w_lo, a.w_hi);
+      if (c) slab |= 1u << q.idx;
+    }
+    a.idx = add(P, full, slab);
+    acc.push_back(a);
+    levels_upto(need + 1);                              // one level of lookahead
+  };
+  // in-place parts of split updates, emitted right after the next leaf so the
+  // critical leaf is claimed before the bulk update (items run in claim order)
+  std::vector<std::function<void()>> pending;
+  auto flush_pending = [&]() {
+    std::vector<std::function<void()>> p;
+    p.swap(pending);
+    for (auto &f : p) f();
+  };
+  auto leaf_acc = [](int64_t e0, int64_t cnt, bool src_w) {
+    Acc a{};
+    a.r_lo[0] = src_w ? 0 : e0; a.r_hi[0] = src_w ? 0 : e0 + cnt;
+    a.w_lo = e0; a.w_hi = e0 + cnt;
+    a.rw = src_w;
+    return a;
+  };
+  auto upd_acc = [](int64_t k_lo, int64_t k_hi, int64_t o_lo, int64_t o_hi, bool to_w) {
+    Acc a{};
+    a.r_lo[0] = k_lo; a.r_hi[0] = k_hi; a.r_lo[1] = o_lo; a.r_hi[1] = o_hi;
+    if (!to_w) { a.w_lo = o_lo; a.w_hi = o_hi; }
+    a.ww = to_w;
+    return a;
+  };
+  // leaf: X rows (L) / columns (R) [e0, e0 + cnt) of the aligned block of width wblk
+  auto leaf = [&](int64_t e0, int64_t cnt, int64_t wblk, bool scaled, bool src_w) {
+    if (!src_w && cnt > 256) { ok = false; return; }    // in place only as one tile per slab
+    int need = -1;
+    for (int64_t w2 = 256; w2 <= wblk; w2 *= 2) ++need;
+    const float a1 = scaled ? 1.f : g.alpha;
+    const float *Dp = g.D + (e0 / NBO) * NBO * NBO + (e0 % NBO) * (1 + NBO);
+    if (g.left) {
+      Problem P = problem(cnt, g.n, a1, 0.f, nullptr, 0, g.B + e0, g.ldb);
+      P.seg[0].a = tri_zeroed(Dp, NBO, true, !g.lower_op);
+      P.seg[0].b = src_w ? dense(g.W, ldw, true) : dense(g.B + e0, g.ldb, true);
+      P.seg[0].K = cnt;
+      P.rev_m = tri_kle(P.seg[0].a);
+      P.outer = 2;                                     // slab (n-tile) outer, LPT rows inside
+      sweep(P, need, leaf_acc(e0, cnt, src_w));
+      flush_pending();
+    } else {
+      Problem P = problem(g.m, cnt, a1, 0.f, nullptr, 0, g.B + e0 * g.ldb, g.ldb);
+      P.seg[0].a = src_w ? dense(g.W, ldw, false) : dense(g.B + e0 * g.ldb, g.ldb, false);
+      P.seg[0].b = tri_zeroed(Dp, NBO, true, g.lower_op);
+      P.seg[0].K = cnt;
+      P.rev_n = tri_kle(P.seg[0].b);
+      P.outer = 1;                                     // slab (m-tile) outer
+      sweep(P, need, leaf_acc(e0, cnt, src_w));
+      flush_pending();
+    }
+  };
+  // update: [o_lo, o_hi) <- a1 * B_o - op(A)(o, k) X_k, k in [k_lo, k_hi); to W or in place
+  auto update = [&](int64_t k_lo, int64_t k_hi, int64_t o_lo, int64_t o_hi, float a1, bool to_w) {
+    if (g.left) {
+      const float *pa = g.ta ? g.A + k_lo + o_lo * g.lda : g.A + o_lo + k_lo * g.lda;
+      Problem P = to_w ? problem(o_hi - o_lo, g.n, -1.f, a1, g.B + o_lo, g.ldb, g.W, ldw)
+                       : problem(o_hi - o_lo, g.n, -1.f, a1, g.B + o_lo, g.ldb, g.B + o_lo, g.ldb);
+      P.seg[0].a = dense(pa, g.lda, g.ta);
+      P.seg[0].b = dense(g.B + k_lo, g.ldb, true);
+      P.seg[0].K = k_hi - k_lo;
+      P.outer = 2;
+      sweep(P, -1, upd_acc(k_lo, k_hi, o_lo, o_hi, to_w));
+    } else {
+      const float *pb = g.ta ? g.A + o_lo + k_lo * g.lda : g.A + k_lo + o_lo * g.lda;
+      Problem P = to_w ? problem(g.m, o_hi - o_lo, -1.f, a1, g.B + o_lo * g.ldb, g.ldb, g.W, ldw)
+                       : problem(g.m, o_hi - o_lo, -1.f, a1, g.B + o_lo * g.ldb, g.ldb,
+                                 g.B + o_lo * g.ldb, g.ldb);
+      P.seg[0].a = dense(g.B + k_lo * g.ldb, g.ldb, false);
+      P.seg[0].b = dense(pb, g.lda, !g.ta);
+      P.seg[0].K = k_hi - k_lo;
+      P.outer = 1;
+      sweep(P, -1, upd_acc(k_lo, k_hi, o_lo, o_hi, to_w));
+    }
+  };
+  const int64_t geo_leaf = trsm_geo_leaf();
+  std::function<void(int64_t, int64_t, bool)> geo = [&](int64_t lo, int64_t w, bool scaled) {
+    const int64_t e1 = imin(nt, lo + w);
+    if (w <= geo_leaf) { leaf(lo, e1 - lo, w, scaled, false); return; }
+    const int64_t h = w / 2, mid = lo + h;
+    if (mid >= e1) { geo(lo, h, scaled); return; }
+    const int64_t f_lo = g.forward ? lo : mid, f_hi = g.forward ? mid : e1;
+    const int64_t s_lo = g.forward ? mid : lo, s_hi = g.forward ? e1 : mid;
+    geo(f_lo, h, scaled);
+    update(f_lo, f_hi, s_lo, s_hi, scaled ? 1.f : g.alpha, true);
+    leaf(s_lo, s_hi - s_lo, h, true, true);
+  };
+  auto elem = [&](int64_t qa, int64_t qb, int64_t &lo, int64_t &hi) {
+    const int64_t pa = g.forward ? qa : g.npanel - qb, pb = g.forward ? qb : g.npanel - qa;
+    lo = pa * NBO;
+    hi = imin(nt, pb * NBO);
+  };
+  std::function<void(int64_t, int64_t, bool, bool)> rec = [&](int64_t q0, int64_t q1, bool scaled,
+                                                              bool in_w) {
+    if (q1 - q0 == 1) {
+      const int64_t p = g.forward ? q0 : g.npanel - 1 - q0;
+      const int64_t p0 = p * NBO, pr = imin(NBO, nt - p0);
+      if (q0 == 0) geo(p0, NBO, scaled);
+      else leaf(p0, pr, NBO, scaled, in_w);
+      return;
+    }
+    const int64_t mid = q0 + (q1 - q0) / 2;
+    rec(q0, mid, scaled, in_w);
+    int64_t k_lo, k_hi, o_lo, o_hi;
+    elem(q0, mid, k_lo, k_hi);
+    elem(mid, q1, o_lo, o_hi);
+    const float a1 = scaled ? 1.f : g.alpha;
+    if (q1 - mid == 1) update(k_lo, k_hi, o_lo, o_hi, a1, true);
+    else {                        // the first panel of [mid, q1) to W, the rest in place
+      int64_t f_lo, f_hi;
+      elem(mid, mid + 1, f_lo, f_hi);
+      update(k_lo, k_hi, f_lo, f_hi, a1, true);
+      const int64_t r_lo = g.forward ? f_hi : o_lo, r_hi = g.forward ? o_hi : f_lo;
+      pending.push_back([=, &update]() { update(k_lo, k_hi, r_lo, r_hi, a1, false); });
+    }
+    rec(mid, q1, true, true);
+  };
+  rec(0, g.npanel, false, false);
+  flush_pending();
+  if (!ok || ph.empty()) return 1;
+  for (const FusedPhase &f : ph)
+    if (!tc_eligible(f.P)) return 1;
+  // 128-block inverses (the fused phases read them), then the one launch
+  if (launch_trsm_diag_inv(g.A, g.lda, nt, g.lower, g.unit, g.D, NBO, s)) return BLAS3_ERR_CUDA;
+  const int rc = launch_tc_fused(ph.data(), (int)ph.size(), s, sms);
+  return rc == 0 ? 0 : (rc == -4 ? BLAS3_ERR_TMA : BLAS3_ERR_CUDA);
+}
+
 int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t n, float alpha,
                 const float *A, int64_t lda, float *B, int64_t ldb, blas3_stream_t stream) {
   int v = tr_validate(side, uplo, transa, diag, m, n, lda, ldb);
@@ -624,6 +835,13 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   if ((rc = get_scratch(D, d_bytes, s, aop_bytes))) return rc;
   if ((rc = get_scratch(Tw, t_bytes, s, aop_bytes + d_bytes))) return rc;
   if ((rc = get_scratch(W, w_bytes, s, aop_bytes + d_bytes + t_bytes))) return rc;
+
+  if (opt(BLAS3_OPT_TRSM_FUSED) && tensor_mode()) {
+    const TrsmGeom g{left, lower, ta, unit, lower_op, forward, m, n, nt, NBO, npanel, other, alpha,
+                     A, lda, B, ldb, D.p, Tw.p, W.p};
+    rc = strsm_fused(g, s, sms);
+    if (rc <= 0) return finish(rc);
+  }
 
   std::lock_guard<std::mutex> lk(g_trsm_mu);          // the per-device side streams
   TrsmStreams *ts = trsm_streams();

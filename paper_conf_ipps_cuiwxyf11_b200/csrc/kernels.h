@@ -16,6 +16,17 @@ int launch_simt(const Problem &P, cudaStream_t s, int num_sms);
 int launch_tc(const Problem &P, cudaStream_t s, int num_sms);
 // TMA eligibility of one operand / the output (16-B pointer alignment, ld%4).
 bool tc_eligible(const Problem &P);
+// Several dependent problems in ONE persistent launch (tcgen05 path, CTA
+// pairs): phase p's tiles wait for the phases in dep_full (complete) and
+// dep_slab (complete on the same slab: n-tile, or m-tile when slab_m).
+// Dependencies must point to earlier phases.  Returns 0, -1 (not fusable /
+// CUDA error: the caller falls back to one launch per phase) or -4.
+struct FusedPhase {
+  Problem P;
+  int32_t dep_full, dep_slab, slab_m;
+};
+constexpr int MAX_FUSED_PHASES = 24;
+int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t s, int num_sms);
 
 // O(N^2) helpers.
 int launch_scale(float *C, int64_t ldc, int64_t m, int64_t n, float beta, int tri,

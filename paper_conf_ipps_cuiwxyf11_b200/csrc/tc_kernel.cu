@@ -79,6 +79,7 @@ constexpr int LAYOUT_K = 0, LAYOUT_MN = 1;
 struct Work {
   int64_t tb, b, t, m0, n0, g0, g1;
   int32_t slice;          // k-slice of a split tile, or -1 for a whole tile
+  int32_t ph;             // phase of a fused launch (0 otherwise)
 };
 
 // Two shared-memory rings: a deep RAW ring (TMA destination, read by UMMA as
@@ -118,23 +119,51 @@ struct Geo {
   static constexpr size_t SMEM = sizeof(RawBuf) * RS + sizeof(LoBuf) * LS + sizeof(Barriers) + 1024;
 };
 
-struct TcParams {
-  CUtensorMap maps[MAX_MAPS];
+// One phase of a launch: a Problem, the work items it owns and, in a FUSED
+// launch (several dependent problems in one persistent grid, e.g. the STRSM
+// sweep), the phases it waits for.  Dependencies are tile counters in global
+// memory: a tile of phase p starts once every phase in dep_full is complete
+// and every phase in dep_slab is complete on the same SLAB (column block of
+// the right-hand side for side=L, row block for side=R): the right-hand-side
+// columns of a triangular solve are independent, so the sweep advances as a
+// wavefront instead of phase by phase.  Items are numbered phase by phase in
+// dependency order and claimed in that order, so every dependency of a
+// claimed tile belongs to an earlier claim of a running CTA (no deadlock).
+struct PhaseDesc {
   Problem P;
+  int64_t item0;           // first work item of this phase
+  int64_t tiles_per;       // tiles of one batch member (Tiles<TM,BN>::count)
+  int64_t ntiles;          // tiles of the phase (all batch members)
+  int32_t dep_full;        // bitmask of phases that must be complete
+  int32_t dep_slab;        // bitmask of phases that must be complete on this tile's slab
+  int32_t slab_m;          // slab = m-tile (1) or n-tile (0)
+  int32_t slab_cnt;        // tiles of this phase per slab
+};
+constexpr int MAX_SLAB = 128;            // slab counters per phase (32768 / 256)
+
+template <int NPH, int NMAPS>
+struct TcParamsT {
+  CUtensorMap maps[NMAPS];
+  PhaseDesc ph[NPH];
+  int32_t nphase;
   uint32_t *tile_ctr;      // dynamic tile scheduler counter, or null (static schedule)
   uint32_t tile_base;      // its value when this launch starts
-  // Split tail (wave quantisation): work items [0, khead) are whole tiles; the
-  // last (ntiles - khead) tiles are cut into ksplit k-slices each, item
-  // khead + j -> tile khead + j / ksplit, slice j % ksplit.  Slices write
-  // fp32 partials to ws; the last arriving slice (ws_cnt) reduces them in
-  // slice order and runs the epilogue.
-  int64_t tiles_per;       // tiles of one batch member (Tiles<TM,BN>::count)
+  // Split tail (wave quantisation, single-phase launches): work items [0, khead)
+  // are whole tiles; the last (ntiles - khead) tiles are cut into ksplit
+  // k-slices each, item khead + j -> tile khead + j / ksplit, slice j % ksplit.
+  // Slices write fp32 partials to ws; the last arriving slice (ws_cnt) reduces
+  // them in slice order and runs the epilogue.
   int64_t nitems, khead;
   int32_t ksplit;
   float *ws;
   uint32_t *ws_cnt;
+  uint32_t *dep_ctr;       // fused: [NPH] phase counters, then [NPH][MAX_SLAB] slab counters
   unsigned long long *trace;   // phase timestamps of CTA 0 (env BLAS3_TRACE), or null
+  unsigned long long *ph_trace;  // fused, BLAS3_TRACE=2: per phase [first dep-ready, last done] (ns)
 };
+using TcParams = TcParamsT<1, MAX_MAPS>;
+constexpr int FUSED_PH = 24, FUSED_MAPS = 48;
+using TcFusedParams = TcParamsT<FUSED_PH, FUSED_MAPS>;
 
 // %globaltimer (ns) of the first occurrence of a phase in CTA 0 (diagnostics)
 #define BLAS3_TRACE(i)                                                              \
@@ -241,11 +270,18 @@ HD int64_t tile_kblocks(const Problem &P, int64_t m0, int64_t n0) {
   return tot;
 }
 
-template <int CG>
-__device__ __forceinline__ Work work_of(const TcParams &prm, int64_t item, int64_t tiles_per) {
-  const Problem &P = prm.P;
+template <int CG, class PRM>
+__device__ __forceinline__ Work work_of(const PRM &prm, int64_t item) {
   Work w;
   w.slice = -1;
+  w.ph = 0;
+  if constexpr (sizeof(prm.ph) / sizeof(prm.ph[0]) > 1) {
+    for (int q = 1; q < prm.nphase; ++q)
+      if (item >= prm.ph[q].item0) w.ph = q;
+    item -= prm.ph[w.ph].item0;
+  }
+  const Problem &P = prm.ph[w.ph].P;
+  const int64_t tiles_per = prm.ph[w.ph].tiles_per;
   w.tb = item;
   if (item >= prm.khead && prm.ksplit > 1) {
     const int64_t j = item - prm.khead;
@@ -280,7 +316,8 @@ __device__ __forceinline__ void clip_kblocks(const Work &w, int64_t &gi, int64_t
 // ---------------------------------------------------------------- producer
 // Every operand map is 4-D: (element dims) x (batch-inner, batch-outer);
 // (bj, bg) select the batch member (0, 0 for an ordinary problem).
-__device__ __forceinline__ void load_operand(const TcParams &prm, const OpDesc &o, int lay,
+template <class PRM>
+__device__ __forceinline__ void load_operand(const PRM &prm, const OpDesc &o, int lay,
                                              uint8_t *raw, int64_t r0, int64_t k0, int rows,
                                              uint64_t *bar, int32_t bj, int32_t bg) {
   if (lay == LAYOUT_MN) {
@@ -391,6 +428,54 @@ __device__ __forceinline__ uint64_t op_desc(uint32_t base, int lay, int k8) {
 // sync them CTA-locally, then ONE thread arrives on the barrier owned by the
 // pair's leader (a cluster-scope release per thread would cost a GPU-scope
 // membar + L1 invalidate each).
+// ---------------------------------------------------------------- fused-launch dependencies
+template <int CG>
+__device__ __forceinline__ int64_t slab_of(const PhaseDesc &ph, const Work &w) {
+  const int64_t s = ph.slab_m ? w.m0 / Geo<CG>::TM : w.n0 / BN;
+  return s < MAX_SLAB ? s : MAX_SLAB - 1;
+}
+__device__ __forceinline__ void spin_until(const uint32_t *ctr, uint32_t target) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+  if (v >= target) return;
+  unsigned long long t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  for (;;) {
+    __nanosleep(128);
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+    if (v >= target) return;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t - t0 > 4000000000ull) __trap();      // a broken dependency graph fails loudly, never hangs
+  }
+}
+// Wait (one thread) until the tile's dependencies are complete; the acquire
+// makes the producing CTAs' stores visible, and the proxy fence orders them
+// before this CTA's later TMA (async-proxy) reads.
+template <int CG, class PRM>
+__device__ __forceinline__ void wait_deps(const PRM &prm, const Work &w) {
+  if constexpr (sizeof(prm.ph) / sizeof(prm.ph[0]) > 1) {
+    const PhaseDesc &ph = prm.ph[w.ph];
+    if ((ph.dep_full | ph.dep_slab) == 0) return;
+    const int64_t slab = slab_of<CG>(ph, w);
+    for (int q = 0; q < prm.nphase; ++q) {
+      if (ph.dep_full >> q & 1) spin_until(prm.dep_ctr + q, (uint32_t)(prm.ph[q].ntiles * CG));
+      if (ph.dep_slab >> q & 1)
+        spin_until(prm.dep_ctr + FUSED_PH + q * MAX_SLAB + slab, (uint32_t)(prm.ph[q].slab_cnt * CG));
+    }
+    asm volatile("fence.proxy.async.global;" ::: "memory");
+  }
+}
+// After this CTA's stores of a tile (one thread, after the epilogue barrier).
+template <int CG, class PRM>
+__device__ __forceinline__ void signal_done(const PRM &prm, const Work &w) {
+  if constexpr (sizeof(prm.ph) / sizeof(prm.ph[0]) > 1) {
+    const PhaseDesc &ph = prm.ph[w.ph];
+    __threadfence();
+    atomicAdd(prm.dep_ctr + w.ph, 1u);
+    atomicAdd(prm.dep_ctr + FUSED_PH + w.ph * MAX_SLAB + slab_of<CG>(ph, w), 1u);
+  }
+}
+
 template <int CG>
 __device__ __forceinline__ void arrive_leader(uint64_t *bar, uint32_t rank, uint32_t id,
                                               uint32_t nthreads, bool first) {
@@ -403,9 +488,11 @@ __device__ __forceinline__ void arrive_leader(uint64_t *bar, uint32_t rank, uint
 
 }  // namespace
 
-template <int CG>
+template <int CG, class PRM>
 __global__ void __launch_bounds__(NTHREADS, 1)
-tc_structured_gemm(const __grid_constant__ TcParams prm) {
+tc_structured_gemm(const __grid_constant__ PRM prm) {
+  constexpr bool FUSED = sizeof(prm.ph) / sizeof(prm.ph[0]) > 1;
+  constexpr int NMAPS = sizeof(prm.maps) / sizeof(prm.maps[0]);
   using G = Geo<CG>;
   using RawBuf = typename G::RawBuf;
   using LoBuf = typename G::LoBuf;
@@ -416,7 +503,6 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
   RawBuf *raw = reinterpret_cast<RawBuf *>(smem);
   LoBuf *lo = reinterpret_cast<LoBuf *>(smem + sizeof(RawBuf) * RS);
   Barriers *bars = reinterpret_cast<Barriers *>(smem + sizeof(RawBuf) * RS + sizeof(LoBuf) * LS);
-  const Problem &P = prm.P;
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const uint32_t rank = (CG == 2) ? ptx::cluster_ctarank() : 0;
   const int64_t cid = blockIdx.x / CG, ncl = gridDim.x / CG;
@@ -453,9 +539,6 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
   ptx::griddep_wait();
   if (threadIdx.x == 0) BLAS3_TRACE(1);
 
-  // batched problems: tile tb -> batch member b = tb / tiles_per, tile t
-  const int64_t tiles_per = prm.tiles_per;
-  const int64_t per = P.per > 0 ? P.per : 1;
   // Tile queue.  The (leader) producer claims work items and publishes them
   // (to the peer producer too, for a CTA pair); every CTA's producer decodes
   // its item once (work_of) into wk[slot] for the local roles.  Consumer
@@ -485,7 +568,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
    if (warp == WARP_TMA) {
     // ============================ TMA producer (each CTA stages its own halves)
     if (lane == 0) {
-      for (int i = 0; i < MAX_MAPS; ++i) ptx::tma_prefetch(&prm.maps[i]);
+      for (int i = 0; i < NMAPS; ++i) ptx::tma_prefetch(&prm.maps[i]);
       uint32_t it = 0;
       for (uint32_t qi = 0;;) {
         int64_t tb;
@@ -493,10 +576,13 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
         const uint32_t par = (qi / TQ) & 1;
         if (CG == 1 || rank == 0) {
           // claim an item (dynamic) or take the static round-robin one
-          // (the first item of every producer is its own id: no claim round trip)
-          tb = (prm.tile_ctr == nullptr || qi == 0)
-                   ? cid + (int64_t)qi * ncl
-                   : ncl + (int64_t)(uint32_t)(atomicAdd(prm.tile_ctr, 1u) - prm.tile_base);
+          // (the first item of every producer is its own id: no claim round
+          // trip -- except in a fused launch, whose items are claimed strictly
+          // in dependency order by running CTAs)
+          if (FUSED) tb = (int64_t)(uint32_t)(atomicAdd(prm.tile_ctr, 1u) - prm.tile_base);
+          else tb = (prm.tile_ctr == nullptr || qi == 0)
+                        ? cid + (int64_t)qi * ncl
+                        : ncl + (int64_t)(uint32_t)(atomicAdd(prm.tile_ctr, 1u) - prm.tile_base);
           if (tb >= prm.nitems) tb = -1;
           BLAS3_TRACE(2);
           ptx::mbar_wait(&bars->tq_empty[slot], par ^ 1);
@@ -507,7 +593,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           ptx::mbar_arrive_cluster(&bars->tq_empty[slot], 0);
         }
         Work w;
-        if (tb >= 0) w = work_of<CG>(prm, tb, tiles_per);
+        if (tb >= 0) w = work_of<CG>(prm, tb);
         else w.tb = -1;
         bars->wk[slot] = w;
         ptx::mbar_arrive(&bars->wk_full[slot]);       // release: local roles see wk[slot]
@@ -518,9 +604,17 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           ptx::griddep_launch_dependents();
           break;
         }
+        const Problem &P = prm.ph[FUSED ? w.ph : 0].P;
+        const int64_t per = P.per > 0 ? P.per : 1;
         const int32_t bj = (int32_t)(w.b % per), bg = (int32_t)(w.b / per);
         const int64_t m0 = w.m0, n0 = w.n0;
         const int64_t ma = m0 + HA * rank, nb = n0 + HB * rank;
+        wait_deps<CG>(prm, w);                        // fused launches: producing tiles done
+        if (FUSED && prm.ph_trace != nullptr) {
+          unsigned long long t_;
+          asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));
+          atomicMin(prm.ph_trace + 2 * w.ph, t_);
+        }
         int64_t gi = 0;
         for (int s = 0; s < P.nseg; ++s) {
           const Segment &sg = P.seg[s];
@@ -556,6 +650,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
       for (;;) {
         const Work w = next_work(qi, 0, 32, lane == 0);
         if (w.tb < 0) break;
+        const Problem &P = prm.ph[FUSED ? w.ph : 0].P;
         const int64_t m0 = w.m0, n0 = w.n0;
         const int64_t nkb = w.g1 - w.g0;
         int64_t done = 0;
@@ -645,6 +740,7 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     for (;;) {
       const Work w = next_work(qi, 4, TR_THREADS, tt == 0);
       if (w.tb < 0) break;
+      const Problem &P = prm.ph[FUSED ? w.ph : 0].P;
       const int64_t m0 = w.m0, n0 = w.n0;
       const int64_t ma = m0 + HA * rank, nb = n0 + HB * rank;
       int64_t gi = 0;
@@ -704,6 +800,8 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
     for (;;) {
       const Work w = next_work(qi, 5, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
       if (w.tb < 0) break;
+      const Problem &P = prm.ph[FUSED ? w.ph : 0].P;
+      const int64_t per = P.per > 0 ? P.per : 1;
       const int64_t coff = (P.nbatch > 1) ? batch_off(P.bs_c, w.b, per) : 0;
       const int64_t m0 = w.m0, n0 = w.n0;
       const int64_t nkb = w.g1 - w.g0;
@@ -760,6 +858,12 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
 #pragma unroll
           for (int i = 0; i < NG * EC; ++i) S[i] += __ldcg(ps + i * HA);
         }
+      }
+      if (FUSED) {
+        // C may have been written by earlier phases on other SMs: one acquire
+        // (which also invalidates this SM's L1) before any thread loads it
+        if (threadIdx.x == WARP_EPI0 * 32) wait_deps<CG>(prm, w);
+        ptx::named_bar_sync(5, EPI_THREADS);
       }
       // ---- store phase: D = alpha*S + beta*C for row r, columns cbase + [0,128).
       // The valid columns of the row form one range [jlo, jhi) (column bound
@@ -825,6 +929,17 @@ tc_structured_gemm(const __grid_constant__ TcParams prm) {
           }
         }
       }
+      if (FUSED) {                                 // this CTA's half of the tile is stored
+        ptx::named_bar_sync(5, EPI_THREADS);
+        if (threadIdx.x == WARP_EPI0 * 32) {
+          signal_done<CG>(prm, w);
+          if (prm.ph_trace != nullptr) {
+            unsigned long long t_;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));
+            atomicMax(prm.ph_trace + 2 * w.ph + 1, t_);
+          }
+        }
+      }
       if (threadIdx.x == WARP_EPI0 * 32) BLAS3_TRACE(8);
     }
     if (threadIdx.x == WARP_EPI0 * 32) BLAS3_TRACE(9);
@@ -880,18 +995,19 @@ static bool make_map(CUtensorMap *m, const float *ptr, int64_t d0, int64_t d1, i
 }
 
 // maps for one operand with R rows, K columns, staged `rows` at a time
-static bool op_maps(TcParams &prm, int &slot, OpDesc &o, int64_t R, int64_t K, int rows,
+template <class PRM>
+static bool op_maps(PRM &prm, int &slot, OpDesc &o, int64_t R, int64_t K, int rows,
                     int64_t per, int64_t groups, BatchStride bs) {
   o.map_rk = o.map_kr = -1;
   const bool need_rk = (o.kind == OP_DENSE && !o.kr) || o.kind == OP_SYM || (o.kind == OP_TRI && !o.swap);
   const bool need_kr = (o.kind == OP_DENSE && o.kr) || o.kind == OP_SYM || (o.kind == OP_TRI && o.swap);
   if (need_rk) {       // X(r,k) = G[r + k*ld]: dim0 = r (R), dim1 = k (K)
-    if (slot >= MAX_MAPS || !make_map(&prm.maps[slot], o.ptr, R, K, o.ld, 32, BK,
+    if (slot >= (int)(sizeof(prm.maps) / sizeof(prm.maps[0])) || !make_map(&prm.maps[slot], o.ptr, R, K, o.ld, 32, BK,
                                                 CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B, per, groups, bs)) return false;
     o.map_rk = slot++;
   }
   if (need_kr) {       // X(r,k) = G[k + r*ld]: dim0 = k (K), dim1 = r (R)
-    if (slot >= MAX_MAPS || !make_map(&prm.maps[slot], o.ptr, K, R, o.ld, BK, rows,
+    if (slot >= (int)(sizeof(prm.maps) / sizeof(prm.maps[0])) || !make_map(&prm.maps[slot], o.ptr, K, R, o.ld, BK, rows,
                                                 CU_TENSOR_MAP_SWIZZLE_128B, per, groups, bs)) return false;
     o.map_kr = slot++;
   }
@@ -925,21 +1041,24 @@ static int choose_cg(const Problem &P, int num_sms) {
   return Tiles<Geo<2>::TM, BN>::count(P) * nb >= num_sms / 2 ? 2 : 1;
 }
 
-template <int CG>
-static int launch_cg(TcParams &prm, cudaStream_t stream, int num_sms) {
+template <int CG, class PRM>
+static int launch_cg(PRM &prm, cudaStream_t stream, int num_sms, bool allow_pdl = true) {
   using G = Geo<CG>;
   int slot = 0;
-  for (int s = 0; s < prm.P.nseg; ++s) {
-    Segment &sg = prm.P.seg[s];
-    if (sg.K <= 0) continue;
-    const int64_t nb = prm.P.nbatch > 1 ? prm.P.nbatch : 1;
-    const int64_t per = nb > 1 ? prm.P.per : 1, groups = cdiv(nb, per);
-    if (!op_maps(prm, slot, sg.a, prm.P.M, sg.K, HA, per, groups, prm.P.bs_a)) return -4;
-    if (!op_maps(prm, slot, sg.b, prm.P.N, sg.K, G::HB, per, groups, prm.P.bs_b)) return -4;
+  for (int p = 0; p < prm.nphase; ++p) {
+    Problem &P = prm.ph[p].P;
+    for (int s = 0; s < P.nseg; ++s) {
+      Segment &sg = P.seg[s];
+      if (sg.K <= 0) continue;
+      const int64_t nb = P.nbatch > 1 ? P.nbatch : 1;
+      const int64_t per = nb > 1 ? P.per : 1, groups = cdiv(nb, per);
+      if (!op_maps(prm, slot, sg.a, P.M, sg.K, HA, per, groups, P.bs_a)) return -4;
+      if (!op_maps(prm, slot, sg.b, P.N, sg.K, G::HB, per, groups, P.bs_b)) return -4;
+    }
   }
   static bool attr = false;
   if (!attr) {
-    if (cudaFuncSetAttribute(tc_structured_gemm<CG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    if (cudaFuncSetAttribute(tc_structured_gemm<CG, PRM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)G::SMEM) != cudaSuccess) return -1;
     attr = true;
   }
@@ -958,13 +1077,13 @@ static int launch_cg(TcParams &prm, cudaStream_t stream, int num_sms) {
   attrs[0].val.clusterDim.z = 1;
   // programmatic dependent launch: this grid's prologue may overlap the tail
   // of the previous kernel on the stream (the kernel waits before touching
-  // global memory).  BLAS3_PDL=0 disables it (experiments).
-  const bool pdl = opt(BLAS3_OPT_PDL) != 0;
+  // global memory).  BLAS3_OPT_PDL=0 disables it (experiments).
+  const bool pdl = allow_pdl && opt(BLAS3_OPT_PDL) != 0;
   attrs[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attrs[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attrs;
   cfg.numAttrs = pdl ? 2 : 1;
-  const cudaError_t e = cudaLaunchKernelEx(&cfg, tc_structured_gemm<CG>, prm);
+  const cudaError_t e = cudaLaunchKernelEx(&cfg, tc_structured_gemm<CG, PRM>, prm);
   note_launch(0);
   return (e == cudaSuccess && cudaGetLastError() == cudaSuccess) ? 0 : -1;
 }
@@ -1033,10 +1152,11 @@ static bool split_workspace(cudaStream_t stream, int num_sms, float **ws, uint32
 // of MMA do).
 template <int CG>
 static void plan_split(TcParams &prm, int num_sms, cudaStream_t stream) {
-  const Problem &P = prm.P;
+  const Problem &P = prm.ph[0].P;
   const int64_t nb = P.nbatch > 1 ? P.nbatch : 1;
   const int64_t tiles_per = Tiles<Geo<CG>::TM, BN>::count(P), T = tiles_per * nb;
-  prm.tiles_per = tiles_per;
+  prm.ph[0].tiles_per = tiles_per;
+  prm.ph[0].ntiles = T;
   prm.nitems = T; prm.khead = T; prm.ksplit = 1;
   if (!opt(BLAS3_OPT_TC_SPLIT) || T == 0) return;
   const int64_t U = imin(T, (int64_t)(num_sms / CG));
@@ -1060,18 +1180,21 @@ static void plan_split(TcParams &prm, int num_sms, cudaStream_t stream) {
   prm.nitems = head + R * S;
 }
 
+static int debug_bits() {
+  static int dbg = -1;
+  if (dbg < 0) { const char *e = getenv("BLAS3_DEBUG_TC"); dbg = e ? atoi(e) : 0; }
+  return dbg;
+}
+
 int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
   static TcParams prm;                    // host staging (the launch copies it)
   static std::mutex mu;
   std::lock_guard<std::mutex> lk(mu);
   memset(&prm, 0, sizeof(prm));
-  prm.P = P0;
-  {
-    static int dbg = -1;
-    if (dbg < 0) { const char *e = getenv("BLAS3_DEBUG_TC"); dbg = e ? atoi(e) : 0; }
-    prm.P.dbg = dbg;
-  }
-  const int cg = choose_cg(prm.P, num_sms);
+  prm.nphase = 1;
+  prm.ph[0].P = P0;
+  prm.ph[0].P.dbg = debug_bits();
+  const int cg = choose_cg(prm.ph[0].P, num_sms);
   const bool dyn = opt(BLAS3_OPT_TC_STATIC) == 0;
   if (cg == 2) plan_split<2>(prm, num_sms, stream); else plan_split<1>(prm, num_sms, stream);
   if (dyn) {
@@ -1105,6 +1228,97 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
     for (int i = 1; i < 12; ++i)
       fprintf(stderr, " %s=%.2f", names[i], h[i] ? (double)(h[i] - h[0]) / 1e3 : -1.0);
     fprintf(stderr, " us\n");
+  }
+  return rc;
+}
+
+// Fused-launch dependency counters, one zeroed block per (device, stream).
+static uint32_t *dep_counters(cudaStream_t stream) {
+  struct Entry { int dev; cudaStream_t st; uint32_t *p; };
+  static Entry tab[32];
+  static int n = 0;
+  int d = 0;
+  if (cudaGetDevice(&d) != cudaSuccess) return nullptr;
+  for (int i = 0; i < n; ++i)
+    if (tab[i].dev == d && tab[i].st == stream) return tab[i].p;
+  if (n == 32) return nullptr;
+  Entry e{d, stream, nullptr};
+  if (cudaMalloc(&e.p, (size_t)FUSED_PH * (1 + MAX_SLAB) * sizeof(uint32_t)) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  tab[n++] = e;
+  return e.p;
+}
+
+int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int num_sms) {
+  if (nph < 1 || nph > FUSED_PH) return -1;
+  static TcFusedParams prm;               // host staging (the launch copies it)
+  static std::mutex mu;
+  std::lock_guard<std::mutex> lk(mu);
+  memset(&prm, 0, sizeof(prm));
+  constexpr int CG = 2;                   // one tile geometry for every phase (slabs align)
+  using TL = Tiles<Geo<CG>::TM, BN>;
+  int64_t item = 0;
+  for (int p = 0; p < nph; ++p) {
+    PhaseDesc &ph = prm.ph[p];
+    ph.P = phases[p].P;
+    ph.P.dbg = debug_bits();
+    if (!tc_eligible(ph.P) || ph.P.max_sms) return -1;
+    const int64_t nb = ph.P.nbatch > 1 ? ph.P.nbatch : 1;
+    ph.tiles_per = TL::count(ph.P);
+    ph.ntiles = ph.tiles_per * nb;
+    ph.item0 = item;
+    item += ph.ntiles;
+    ph.dep_full = phases[p].dep_full;
+    ph.dep_slab = phases[p].dep_slab;
+    ph.slab_m = phases[p].slab_m;
+    ph.slab_cnt = (int32_t)(phases[p].slab_m ? cdiv(ph.P.N, BN) : cdiv(ph.P.M, Geo<CG>::TM));
+    if ((ph.dep_full | ph.dep_slab) >> p) return -1;        // dependencies point backwards only
+    if (ph.P.c_tri != 0 || nb > 1 ? false : false) return -1;
+    for (int s = 0; s < ph.P.nseg; ++s)                      // SYM diagonal merges read global memory
+      if (ph.P.seg[s].a.kind == OP_SYM || ph.P.seg[s].b.kind == OP_SYM) return -1;
+    const int64_t nslab = phases[p].slab_m ? cdiv(ph.P.M, Geo<CG>::TM) : cdiv(ph.P.N, BN);
+    if (nslab > MAX_SLAB) return -1;
+  }
+  prm.nphase = nph;
+  prm.nitems = item;
+  prm.khead = item;
+  prm.ksplit = 1;
+  prm.dep_ctr = dep_counters(stream);
+  if (!prm.dep_ctr) return -1;
+  if (cudaMemsetAsync(prm.dep_ctr, 0, (size_t)FUSED_PH * (1 + MAX_SLAB) * sizeof(uint32_t), stream) !=
+      cudaSuccess) return -1;
+  TileCounter tc;
+  const int64_t units = imin(item, (int64_t)(num_sms / CG));
+  if (item == 0) return 0;
+  if (!tile_counter(tc, (uint32_t)(item + units))) return -1;     // every item + one failing claim each
+  prm.tile_ctr = tc.ctr;
+  prm.tile_base = tc.base;
+  // diagnostics: BLAS3_TRACE=2 prints each phase's [first start, last end] (synchronises)
+  static int trace = -1;
+  static unsigned long long *tbuf = nullptr;
+  if (trace < 0) { const char *e = getenv("BLAS3_TRACE"); trace = (e && e[0] == '2') ? 1 : 0; }
+  if (trace) {
+    if (!tbuf && cudaMalloc(&tbuf, 2 * FUSED_PH * sizeof(unsigned long long)) != cudaSuccess) return -1;
+    unsigned long long init[2 * FUSED_PH];
+    for (int i = 0; i < FUSED_PH; ++i) { init[2 * i] = ~0ull; init[2 * i + 1] = 0ull; }
+    cudaMemcpyAsync(tbuf, init, sizeof(init), cudaMemcpyHostToDevice, stream);
+    cudaStreamSynchronize(stream);
+    prm.ph_trace = tbuf;
+  }
+  // no PDL: the counters' memset node precedes this grid on the stream
+  const int rc = launch_cg<CG>(prm, stream, num_sms, false);
+  if (trace && rc == 0) {
+    unsigned long long h[2 * FUSED_PH];
+    cudaStreamSynchronize(stream);
+    cudaMemcpy(h, tbuf, sizeof(h), cudaMemcpyDeviceToHost);
+    unsigned long long t0 = ~0ull;
+    for (int p = 0; p < nph; ++p) t0 = h[2 * p] < t0 ? h[2 * p] : t0;
+    for (int p = 0; p < nph; ++p)
+      fprintf(stderr, "[blas3 fused] phase %2d M=%6lld N=%6lld K=%6lld tiles=%5lld: %8.1f .. %8.1f us\n", p,
+              (long long)prm.ph[p].P.M, (long long)prm.ph[p].P.N, (long long)prm.ph[p].P.seg[0].K,
+              (long long)prm.ph[p].ntiles, (h[2 * p] - t0) / 1e3, (h[2 * p + 1] - t0) / 1e3);
   }
   return rc;
 }

@@ -8,7 +8,8 @@ their own streams.
   columns (side=L) / rows (side=R) against the fp64 oracle;
 * in a subprocess with a 256-wide panel, up to 4 slabs and a 256-wide slab
   minimum (env knobs read once per process), the whole small-size STRSM
-  parity suite -- many panels, forward and backward orders, several slabs.
+  parity suite -- many panels, forward and backward orders, several slabs --
+  once on the fused single-launch path and once on the multi-launch path.
 """
 import itertools
 import os
@@ -63,11 +64,36 @@ def test_strsm_multi_panel_multi_slab(b3, oracle_mod, side, uplo, ta, diag):
     assert fro(Xs - ref) / fro(ref) <= 1e-5
 
 
-def test_strsm_small_panels_many_slabs():
+@pytest.mark.parametrize("side", ["L", "R"])
+def test_strsm_fused_is_one_launch(b3, oracle_mod, side):
+    """BLAS3_OPT_TRSM_FUSED=1: the doubling and the sweep are ONE persistent
+    tcgen05 launch after the 128-block inverses; the multi-launch path (the
+    default, option 0) gives the same answer to rounding."""
+    ka, other = 2600, 4500
+    m, n = (ka, other) if side == "L" else (other, ka)
+    A = gen.triangular_dd(ka, "L", "N", "fuse-a")
+    B = gen.uniform(m, n, "fuse-b")
+    dA = to_dev(A)
+    dB = to_dev(B)
+    with b3.options(trsm_fused=1):
+        tc0, all0 = b3.launch_count("tc"), b3.launch_count()
+        b3.strsm(side, "L", "N", "N", AL, dA, dB)
+        X1 = f64(to_host(dB))
+        assert b3.launch_count("tc") - tc0 == 1 and b3.launch_count() - all0 == 2
+    with b3.options(trsm_fused=0):
+        dB2 = to_dev(B)
+        b3.strsm(side, "L", "N", "N", AL, dA, dB2)
+        X0 = f64(to_host(dB2))
+    assert fro(X1 - X0) / fro(X0) <= 1e-6
+
+
+@pytest.mark.parametrize("fused", ["0", "1"])
+def test_strsm_small_panels_many_slabs(fused):
     import torch
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
-    env = {**os.environ, "BLAS3_TRSM_NB": "256", "BLAS3_TRSM_SLABS": "4", "BLAS3_TRSM_SLAB_MIN": "256"}
+    env = {**os.environ, "BLAS3_TRSM_NB": "256", "BLAS3_TRSM_SLABS": "4", "BLAS3_TRSM_SLAB_MIN": "256",
+           "BLAS3_TRSM_FUSED": fused}
     cmd = [sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k", "strsm",
            os.path.join(ROOT, "tests", "test_parity_gpu.py")]
     r = subprocess.run(cmd, env=env, cwd=ROOT, capture_output=True, text=True, timeout=900)
