@@ -499,7 +499,10 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
   using Barriers = typename G::Barriers;
   constexpr int RS = G::RS, LS = G::LS, TM = G::TM, HB = G::HB;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-B aligned base by pointer arithmetic on the __shared__ array (not via
+  // an integer round trip), so the compiler keeps the shared address space and
+  // emits LDS/STS instead of generic loads/stores in the transform
+  uint8_t *smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   RawBuf *raw = reinterpret_cast<RawBuf *>(smem);
   LoBuf *lo = reinterpret_cast<LoBuf *>(smem + sizeof(RawBuf) * RS);
   Barriers *bars = reinterpret_cast<Barriers *>(smem + sizeof(RawBuf) * RS + sizeof(LoBuf) * LS);
