@@ -163,7 +163,7 @@ int blas3_get_math_mode(void);
  *   BLAS3_OPT_TRSM_SLABS   [BLAS3_TRSM_SLABS] right-hand-side slabs on own streams, 1..4 (2)
  *   BLAS3_OPT_TRSM_SLAB_MIN [BLAS3_TRSM_SLAB_MIN] minimum slab width, >= 256 (2048)
  *   BLAS3_OPT_TRSM_RESERVE [BLAS3_TRSM_RESERVE] SMs the first panel's sweep leaves to
- *                          the panel-inverse doubling chain, 0..#SMs/2 (32)
+ *                          the panel-inverse doubling chain, 0..74 (48)
  *   BLAS3_OPT_TRSM_GEO_LEAF [BLAS3_TRSM_GEO_LEAF] the first panel is halved down to
  *                          this width: power of 2 in [128, 8192] (256)
  *   BLAS3_OPT_TRSM_FUSED   [BLAS3_TRSM_FUSED] 1: the whole STRSM (panel-inverse
@@ -171,6 +171,13 @@ int blas3_get_math_mode(void);
  *                          launch when it fits; 0 (default): one launch per step
  *                          on the caller's and the side streams (measured equal
  *                          or faster on B200 at N = 8192)
+ *   BLAS3_OPT_TRSM_FIRST_YM [BLAS3_TRSM_FIRST_YM] 1 (default): the first panel's
+ *                          blocks are solved as X_s = Y_s - M X_f with Y, M
+ *                          precomputed off the critical path; 0: update + solve
+ *   BLAS3_OPT_TRSM_FIRST_FUSED [BLAS3_TRSM_FIRST_FUSED] 1 (default): the first
+ *                          panel (its doubling, Y, M and the X chain) as ONE
+ *                          persistent dependency-driven launch; 0: separate
+ *                          launches on side streams
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */
@@ -180,7 +187,7 @@ enum {
     BLAS3_OPT_TC_SPLIT = 6, BLAS3_OPT_TC_STATIC = 7, BLAS3_OPT_PDL = 8,
     BLAS3_OPT_TRSM_NB = 9, BLAS3_OPT_TRSM_SLABS = 10, BLAS3_OPT_TRSM_SLAB_MIN = 11,
     BLAS3_OPT_TRSM_RESERVE = 12, BLAS3_OPT_TRSM_GEO_LEAF = 13, BLAS3_OPT_TRSM_FUSED = 14,
-    BLAS3_OPT_COUNT = 15
+    BLAS3_OPT_TRSM_FIRST_YM = 15, BLAS3_OPT_TRSM_FIRST_FUSED = 16, BLAS3_OPT_COUNT = 17
 };
 int blas3_set_option(int key, int64_t value);
 int64_t blas3_get_option(int key);

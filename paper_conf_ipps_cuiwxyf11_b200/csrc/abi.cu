@@ -39,9 +39,11 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TRSM_NB", 2048, 128, 8192, true},
     {"BLAS3_TRSM_SLABS", 2, 1, 4, false},
     {"BLAS3_TRSM_SLAB_MIN", 2048, 256, int64_t(1) << 40, false},
-    {"BLAS3_TRSM_RESERVE", 32, 0, 74, false},
+    {"BLAS3_TRSM_RESERVE", 48, 0, 74, false},
     {"BLAS3_TRSM_GEO_LEAF", 256, 128, 8192, true},
     {"BLAS3_TRSM_FUSED", 0, 0, 1, false},
+    {"BLAS3_TRSM_FIRST_YM", 1, 0, 1, false},
+    {"BLAS3_TRSM_FIRST_FUSED", 1, 0, 1, false},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;
@@ -552,8 +554,9 @@ static int trsm_panel_doubling(const float *A, int64_t lda, int64_t nt, bool low
 // asynchronous (and graph-capturable) on the caller's stream.
 constexpr int MAX_SLABS = 4, MAX_LEVELS = 8;
 struct TrsmStreams {
-  cudaStream_t side, side2, slab[MAX_SLABS];
-  cudaEvent_t ev_fork, ev_lvl[MAX_LEVELS], ev_lvl2[MAX_LEVELS], ev_join[MAX_SLABS];
+  cudaStream_t side, side2, side3, slab[MAX_SLABS];
+  cudaEvent_t ev_fork, ev_fork2, ev_lvl[MAX_LEVELS], ev_lvl2[MAX_LEVELS], ev_ym[MAX_LEVELS],
+      ev_join[MAX_SLABS];
 };
 static std::mutex g_trsm_mu;
 static TrsmStreams *trsm_streams() {
@@ -570,14 +573,17 @@ static TrsmStreams *trsm_streams() {
     if (cudaDeviceGetStreamPriorityRange(&lo_pri, &hi_pri) != cudaSuccess) return nullptr;
     if (cudaStreamCreateWithPriority(&t.side, cudaStreamNonBlocking, hi_pri) != cudaSuccess) return nullptr;
     if (cudaStreamCreateWithPriority(&t.side2, cudaStreamNonBlocking, lo_pri) != cudaSuccess) return nullptr;
+    if (cudaStreamCreateWithPriority(&t.side3, cudaStreamNonBlocking, hi_pri) != cudaSuccess) return nullptr;
     for (int i = 0; i < MAX_LEVELS; ++i)
       if (cudaEventCreateWithFlags(&t.ev_lvl[i], fl) != cudaSuccess ||
-          cudaEventCreateWithFlags(&t.ev_lvl2[i], fl) != cudaSuccess) return nullptr;
+          cudaEventCreateWithFlags(&t.ev_lvl2[i], fl) != cudaSuccess ||
+          cudaEventCreateWithFlags(&t.ev_ym[i], fl) != cudaSuccess) return nullptr;
     for (int i = 0; i < MAX_SLABS; ++i) {
       if (cudaStreamCreateWithFlags(&t.slab[i], cudaStreamNonBlocking) != cudaSuccess ||
           cudaEventCreateWithFlags(&t.ev_join[i], fl) != cudaSuccess) return nullptr;
     }
-    if (cudaEventCreateWithFlags(&t.ev_fork, fl) != cudaSuccess) return nullptr;
+    if (cudaEventCreateWithFlags(&t.ev_fork, fl) != cudaSuccess ||
+        cudaEventCreateWithFlags(&t.ev_fork2, fl) != cudaSuccess) return nullptr;
     made[d] = true;
   }
   return &t;
@@ -606,6 +612,10 @@ static int64_t trsm_geo_leaf() { return opt(BLAS3_OPT_TRSM_GEO_LEAF); }
 // most one 256-row tile per slab) runs in place -- no copy-backs.
 // Returns 1 (not fusable: the caller runs the multi-launch path) before
 // anything is enqueued, 0 on success, < 0 on a CUDA error.
+// A geometric pair of the first panel: first half f (solved before), second
+// half s (aligned block of width h), with the precomputed Y_s and M buffers.
+struct GeoPair { int64_t f_lo, f_hi, s_lo, s_hi, h; float *Y, *M; int64_t ldy, ldm; };
+
 struct TrsmGeom {
   bool left, lower, ta, unit, lower_op, forward;
   int64_t m, n, nt, NBO, npanel, other;
@@ -791,6 +801,119 @@ static int strsm_fused(const TrsmGeom &g, cudaStream_t s, int sms) {
   return rc == 0 ? 0 : (rc == -4 ? BLAS3_ERR_TMA : BLAS3_ERR_CUDA);
 }
 
+// The first processed panel as ONE fused launch (BLAS3_OPT_TRSM_FIRST_FUSED).
+// Phases, in claim order: the panel's doubling levels (each step waits for
+// the previous one), the first leaf (in place: one 256-row tile per slab),
+// then per geometric pair j: M_j and Y_j (wait for the level that built
+// inv(op(A)_ss)) and X_j = Y_j - M_j X_f (waits for M_j, and on its slab for
+// Y_j and every earlier chain phase).  Returns 1 if not fusable (nothing
+// enqueued), 0 on success, < 0 on a CUDA error.  The 128-block inverses must
+// already be on the stream.
+static int strsm_first_fused(const TrsmGeom &g, const std::vector<GeoPair> &gp, int64_t pfirst,
+                             cudaStream_t s, int sms) {
+  const int64_t NBO = g.NBO, nt = g.nt;
+  const int64_t o = pfirst * NBO;
+  std::vector<LevelProblem> lv;
+  trsm_doubling_problems(g.A + o * (1 + g.lda), g.lda, imin(NBO, nt - o), g.lower, g.D + pfirst * NBO * NBO,
+                         g.Tw, lv);
+  auto level_of = [](int64_t w) { int l = -1; for (int64_t w2 = 256; w2 <= w; w2 *= 2) ++l; return l; };
+  int need = 0;                                         // levels used: inv of every s block
+  for (const GeoPair &p : gp) need = imax(need, level_of(p.h) + 1);
+  std::vector<FusedPhase> ph;
+  auto add = [&](const Problem &P, uint32_t full, uint32_t slab) -> int {
+    FusedPhase f;
+    f.P = P; f.dep_full = (int32_t)full; f.dep_slab = (int32_t)slab; f.slab_m = g.left ? 0 : 1;
+    ph.push_back(f);
+    return (int)ph.size() - 1;
+  };
+  uint32_t lvl_mask[MAX_LEVELS] = {};
+  for (int l = 0; l < need; ++l) {
+    uint32_t step1 = 0;
+    for (const LevelProblem &q : lv)
+      if (q.lvl == l && q.step == 1) step1 |= 1u << add(q.P, l > 0 ? lvl_mask[l - 1] : 0u, 0u);
+    for (const LevelProblem &q : lv)
+      if (q.lvl == l && q.step == 2) lvl_mask[l] |= 1u << add(q.P, step1, 0u);
+  }
+  // first leaf: the block solved before every pair's f
+  const int64_t l_lo = gp[0].f_lo, l_cnt = gp[0].f_hi - gp[0].f_lo;
+  if (l_cnt > 256) return 1;
+  const int l_lv = level_of(gp[0].h);
+  const float *Dl = g.D + (l_lo / NBO) * NBO * NBO + (l_lo % NBO) * (1 + NBO);
+  uint32_t chain = 0;
+  {
+    Problem P;
+    if (g.left) {
+      P = problem(l_cnt, g.n, g.alpha, 0.f, nullptr, 0, g.B + l_lo, g.ldb);
+      P.seg[0].a = tri_zeroed(Dl, NBO, true, !g.lower_op);
+      P.seg[0].b = dense(g.B + l_lo, g.ldb, true);
+      P.rev_m = tri_kle(P.seg[0].a);
+      P.outer = 2;
+    } else {
+      P = problem(g.m, l_cnt, g.alpha, 0.f, nullptr, 0, g.B + l_lo * g.ldb, g.ldb);
+      P.seg[0].a = dense(g.B + l_lo * g.ldb, g.ldb, false);
+      P.seg[0].b = tri_zeroed(Dl, NBO, true, g.lower_op);
+      P.rev_n = tri_kle(P.seg[0].b);
+      P.outer = 1;
+    }
+    P.seg[0].K = l_cnt;
+    chain |= 1u << add(P, l_lv >= 0 ? lvl_mask[l_lv] : 0u, 0u);
+  }
+  for (const GeoPair &p : gp) {
+    const int64_t ns = p.s_hi - p.s_lo, nf = p.f_hi - p.f_lo;
+    const int lvp = level_of(p.h);
+    const uint32_t lmask = lvp >= 0 ? lvl_mask[lvp] : 0u;
+    const float *Ds = g.D + (p.s_lo / NBO) * NBO * NBO + (p.s_lo % NBO) * (1 + NBO);
+    Problem PM, PY, PX;
+    if (g.left) {
+      PM = problem(ns, nf, 1.f, 0.f, nullptr, 0, p.M, p.ldm);
+      PM.seg[0].a = tri_zeroed(Ds, NBO, true, !g.lower_op);
+      PM.seg[0].b = g.ta ? dense(g.A + p.f_lo + p.s_lo * g.lda, g.lda, false)
+                         : dense(g.A + p.s_lo + p.f_lo * g.lda, g.lda, true);
+      PM.seg[0].K = ns;
+      PM.rev_m = tri_kle(PM.seg[0].a);
+      PY = problem(ns, g.n, g.alpha, 0.f, nullptr, 0, p.Y, p.ldy);
+      PY.seg[0].a = tri_zeroed(Ds, NBO, true, !g.lower_op);
+      PY.seg[0].b = dense(g.B + p.s_lo, g.ldb, true);
+      PY.seg[0].K = ns;
+      PY.rev_m = tri_kle(PY.seg[0].a);
+      PY.outer = 2;
+      PX = problem(ns, g.n, -1.f, 1.f, p.Y, p.ldy, g.B + p.s_lo, g.ldb);
+      PX.seg[0].a = dense(p.M, p.ldm, false);
+      PX.seg[0].b = dense(g.B + p.f_lo, g.ldb, true);
+      PX.seg[0].K = nf;
+      PX.outer = 2;
+    } else {
+      PM = problem(nf, ns, 1.f, 0.f, nullptr, 0, p.M, p.ldm);
+      PM.seg[0].a = g.ta ? dense(g.A + p.s_lo + p.f_lo * g.lda, g.lda, true)
+                         : dense(g.A + p.f_lo + p.s_lo * g.lda, g.lda, false);
+      PM.seg[0].b = tri_zeroed(Ds, NBO, true, g.lower_op);
+      PM.seg[0].K = ns;
+      PM.rev_n = tri_kle(PM.seg[0].b);
+      PY = problem(g.m, ns, g.alpha, 0.f, nullptr, 0, p.Y, p.ldy);
+      PY.seg[0].a = dense(g.B + p.s_lo * g.ldb, g.ldb, false);
+      PY.seg[0].b = tri_zeroed(Ds, NBO, true, g.lower_op);
+      PY.seg[0].K = ns;
+      PY.rev_n = tri_kle(PY.seg[0].b);
+      PY.outer = 1;
+      PX = problem(g.m, ns, -1.f, 1.f, p.Y, p.ldy, g.B + p.s_lo * g.ldb, g.ldb);
+      PX.seg[0].a = dense(g.B + p.f_lo * g.ldb, g.ldb, false);
+      PX.seg[0].b = dense(p.M, p.ldm, true);
+      PX.seg[0].K = nf;
+      PX.outer = 1;
+    }
+    const int im = add(PM, lmask, 0u);
+    const int iy = add(PY, lmask, 0u);
+    chain |= 1u << add(PX, 1u << im, chain | (1u << iy));
+  }
+  if ((int)ph.size() > MAX_FUSED_PHASES) return 1;
+  for (const FusedPhase &f : ph)
+    if (!tc_eligible(f.P)) return 1;
+  // the chain is latency-bound: leave SMs to the other panels' doubling,
+  // which runs concurrently on a side stream
+  const int rc = launch_tc_fused(ph.data(), (int)ph.size(), s, (int)imax(sms / 2, sms - trsm_reserve()));
+  return rc == 0 ? 0 : (rc == -4 ? BLAS3_ERR_TMA : BLAS3_ERR_CUDA);
+}
+
 int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t n, float alpha,
                 const float *A, int64_t lda, float *B, int64_t ldb, blas3_stream_t stream) {
   int v = tr_validate(side, uplo, transa, diag, m, n, lda, ldb);
@@ -846,24 +969,59 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   std::lock_guard<std::mutex> lk(g_trsm_mu);          // the per-device side streams
   TrsmStreams *ts = trsm_streams();
   if (!ts) return BLAS3_ERR_CUDA;
+  // First-panel precompute (BLAS3_OPT_TRSM_FIRST_YM): each geometric pair
+  // (first half f solved, second half s) would be "update s by f, then solve
+  // s" on the critical path.  Instead, with Y_s = a * inv(op(A)_ss) B_s and
+  // M_sf = inv(op(A)_ss) op(A)_sf -- neither needs X -- a third high-priority
+  // stream computes Y and M as soon as inv(op(A)_ss) exists, and the chain is
+  // left with ONE GEMM per pair, X_s = Y_s - M_sf X_f (K = |f|): the first
+  // panel's sequential k-blocks halve.  (side=R: X_s = Y_s - X_f M_fs with
+  // Y_s = a B_s inv(op(A)_ss), M_fs = op(A)_fs inv(op(A)_ss).)
+  const int64_t pfirst = forward ? 0 : npanel - 1;
+  int nlvl = 0;
+  for (int64_t sz = 128; sz < NBO; sz *= 2) ++nlvl;
+  std::vector<GeoPair> gp;
+  Scratch YM;
+  const bool use_ym = opt(BLAS3_OPT_TRSM_FIRST_YM) != 0 || opt(BLAS3_OPT_TRSM_FIRST_FUSED) != 0;
+  if (use_ym) {
+    std::function<void(int64_t, int64_t)> pairs = [&](int64_t lo, int64_t w) {
+      const int64_t e1 = imin(nt, lo + w);
+      if (w <= trsm_geo_leaf()) return;
+      const int64_t h = w / 2, mid = lo + h;
+      if (mid >= e1) { pairs(lo, h); return; }
+      const int64_t f_lo = forward ? lo : mid, f_hi = forward ? mid : e1;
+      const int64_t s_lo = forward ? mid : lo, s_hi = forward ? e1 : mid;
+      pairs(f_lo, h);
+      gp.push_back({f_lo, f_hi, s_lo, s_hi, h, nullptr, nullptr, 0, 0});
+    };
+    pairs(pfirst * NBO, NBO);
+    if ((int)gp.size() > MAX_LEVELS) gp.clear();
+    size_t fl = 0;
+    for (GeoPair &p : gp) {
+      const int64_t ns = p.s_hi - p.s_lo, nf = p.f_hi - p.f_lo;
+      p.ldy = left ? ld4(ns) : ld4(m);
+      p.ldm = left ? ld4(ns) : ld4(nf);
+      fl += (size_t)p.ldy * (left ? n : ns) + (size_t)p.ldm * (left ? nf : ns);
+    }
+    if (!gp.empty()) {
+      if ((rc = get_scratch(YM, fl * sizeof(float), s, aop_bytes + d_bytes + t_bytes + w_bytes))) return rc;
+      float *cur = YM.p;
+      for (GeoPair &p : gp) {
+        const int64_t ns = p.s_hi - p.s_lo, nf = p.f_hi - p.f_lo;
+        p.Y = cur; cur += (size_t)p.ldy * (left ? n : ns);
+        p.M = cur; cur += (size_t)p.ldm * (left ? nf : ns);
+      }
+    }
+  }
+
   // 1. every 128-block inverse on the caller's stream; then the doubling
   //    levels of all panels on the high-priority side stream, one event per
   //    level, while the sweep starts on blocks whose inverse already exists.
   if (launch_trsm_diag_inv(A, lda, nt, lower, unit, D.p, NBO, s)) return BLAS3_ERR_CUDA;
   if (cudaEventRecord(ts->ev_fork, s) != cudaSuccess ||
       cudaStreamWaitEvent(ts->side, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
-  int nlvl = 0;
-  for (int64_t sz = 128; sz < NBO; sz *= 2) ++nlvl;
-  // the first processed panel's levels (on the sweep's critical path) alone on
-  // the high-priority stream; the other panels' levels (needed one panel
-  // sweep later) on a second side stream
-  const int64_t pfirst = forward ? 0 : npanel - 1;
-  {
-    const int64_t o = pfirst * NBO;
-    if ((rc = trsm_panel_doubling(A + o * (1 + lda), lda, imin(NBO, nt - o), lower,
-                                  D.p + pfirst * NBO * NBO, Tw.p + t_rest, ts->side, sms, ts->ev_lvl)))
-      return rc;
-  }
+  // the other panels' levels (needed one panel sweep later) on a second side
+  // stream, from the start
   if (npanel > 1) {
     const int64_t prest = forward ? 1 : 0, o = prest * NBO;
     if (cudaStreamWaitEvent(ts->side2, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
@@ -871,6 +1029,75 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
                                   D.p + prest * NBO * NBO, Tw.p, ts->side2, sms, ts->ev_lvl2)))
       return rc;
   }
+  // the first processed panel: ONE fused persistent launch (its doubling
+  // levels, the precomputed Y and M of every geometric pair, and the chain
+  // leaf -> X_1 -> X_2 -> ... with per-slab tile-counter dependencies) on the
+  // caller's stream; else its levels on the high-priority side stream and
+  // the Y/M precompute on a third stream, the chain on the slab streams.
+  bool first_done = false, ym_ready = false;
+  if (opt(BLAS3_OPT_TRSM_FIRST_FUSED) && tensor_mode() && !gp.empty()) {
+    const TrsmGeom g{left, lower, ta, unit, lower_op, forward, m, n, nt, NBO, npanel, other, alpha,
+                     A, lda, B, ldb, D.p, Tw.p + t_rest, W.p};
+    rc = strsm_first_fused(g, gp, pfirst, s, sms);
+    if (rc < 0) return rc;
+    first_done = rc == 0;
+  }
+  if (!first_done) {
+    const int64_t o = pfirst * NBO;
+    if ((rc = trsm_panel_doubling(A + o * (1 + lda), lda, imin(NBO, nt - o), lower,
+                                  D.p + pfirst * NBO * NBO, Tw.p + t_rest, ts->side, sms, ts->ev_lvl)))
+      return rc;
+  }
+  if (cudaEventRecord(ts->ev_fork2, s) != cudaSuccess) return BLAS3_ERR_CUDA;
+  if (!gp.empty() && !first_done && opt(BLAS3_OPT_TRSM_FIRST_YM)) {
+    ym_ready = true;
+    {
+      if (cudaStreamWaitEvent(ts->side3, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+      for (size_t j = 0; j < gp.size(); ++j) {
+        const GeoPair &p = gp[j];
+        const int64_t ns = p.s_hi - p.s_lo, nf = p.f_hi - p.f_lo;
+        int lv = -1;                                    // level that built inv(op(A)_ss)
+        for (int64_t w2 = 256; w2 <= p.h; w2 *= 2) ++lv;
+        if (lv >= 0 && cudaStreamWaitEvent(ts->side3, ts->ev_lvl[lv], 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+        const float *Ds = D.p + (p.s_lo / NBO) * NBO * NBO + (p.s_lo % NBO) * (1 + NBO);
+        if (left) {
+          // M = inv(op(A)_ss) op(A)_sf : Xb(c,k) = op(A)(s_lo+k, f_lo+c)
+          Problem PM = problem(ns, nf, 1.f, 0.f, nullptr, 0, p.M, p.ldm);
+          PM.seg[0].a = tri_zeroed(Ds, NBO, true, !lower_op);
+          PM.seg[0].b = ta ? dense(A + p.f_lo + p.s_lo * lda, lda, false)
+                           : dense(A + p.s_lo + p.f_lo * lda, lda, true);
+          PM.seg[0].K = ns;
+          PM.rev_m = tri_kle(PM.seg[0].a);
+          // Y = alpha inv(op(A)_ss) B_s
+          Problem PY = problem(ns, n, alpha, 0.f, nullptr, 0, p.Y, p.ldy);
+          PY.seg[0].a = tri_zeroed(Ds, NBO, true, !lower_op);
+          PY.seg[0].b = dense(B + p.s_lo, ldb, true);
+          PY.seg[0].K = ns;
+          PY.rev_m = tri_kle(PY.seg[0].a);
+          PY.outer = 1;
+          if ((rc = run_problem(PM, ts->side3, sms)) || (rc = run_problem(PY, ts->side3, sms))) return rc;
+        } else {
+          // M = op(A)_fs inv(op(A)_ss) : Xa(r,k) = op(A)(f_lo+r, s_lo+k), Xb(c,k) = inv(k,c)
+          Problem PM = problem(nf, ns, 1.f, 0.f, nullptr, 0, p.M, p.ldm);
+          PM.seg[0].a = ta ? dense(A + p.s_lo + p.f_lo * lda, lda, true)
+                           : dense(A + p.f_lo + p.s_lo * lda, lda, false);
+          PM.seg[0].b = tri_zeroed(Ds, NBO, true, lower_op);
+          PM.seg[0].K = ns;
+          PM.rev_n = tri_kle(PM.seg[0].b);
+          // Y = alpha B_s inv(op(A)_ss)
+          Problem PY = problem(m, ns, alpha, 0.f, nullptr, 0, p.Y, p.ldy);
+          PY.seg[0].a = dense(B + p.s_lo * ldb, ldb, false);
+          PY.seg[0].b = tri_zeroed(Ds, NBO, true, lower_op);
+          PY.seg[0].K = ns;
+          PY.rev_n = tri_kle(PY.seg[0].b);
+          PY.outer = 2;
+          if ((rc = run_problem(PM, ts->side3, sms)) || (rc = run_problem(PY, ts->side3, sms))) return rc;
+        }
+        if (cudaEventRecord(ts->ev_ym[j], ts->side3) != cudaSuccess) return BLAS3_ERR_CUDA;
+      }
+    }
+  }
+
 
   // 2. the sweep, independently per slab of the right-hand side (columns of B
   //    for side=L, rows for side=R), each slab on its own stream.
@@ -889,7 +1116,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   for (int64_t q = 0; q < nslab; ++q) {
     const int64_t c0 = align_down(other * q / nslab, 256), c1 = q + 1 == nslab ? other : align_down(other * (q + 1) / nslab, 256);
     cudaStream_t st = nslab == 1 ? s : ts->slab[q];
-    if (st != s && cudaStreamWaitEvent(st, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+    if (st != s && cudaStreamWaitEvent(st, ts->ev_fork2, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
     float *Bq = left ? B + c0 * ldb : B + c0;
     float *Wq = left ? W.p + c0 * NBO : W.p + c0;
     const int64_t mq = left ? m : c1 - c0, nq = left ? c1 - c0 : n;
@@ -968,6 +1195,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
     };
     // geometric solve of the aligned block [lo, lo + w) (clipped to nt): the
     // first half (in processing order) recursively, the second as one leaf
+    size_t gj = 0;                                    // next geometric pair (processing order)
     std::function<int(int64_t, int64_t, bool)> geo = [&](int64_t lo, int64_t w, bool scaled) -> int {
       int rc2;
       const int64_t e1 = imin(nt, lo + w);
@@ -977,6 +1205,27 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
       const int64_t f_lo = forward ? lo : mid, f_hi = forward ? mid : e1;   // first half
       const int64_t s_lo = forward ? mid : lo, s_hi = forward ? e1 : mid;   // second half
       if ((rc2 = geo(f_lo, h, scaled))) return rc2;
+      if (ym_ready && gj < gp.size() && gp[gj].s_lo == s_lo && gp[gj].f_lo == f_lo && !scaled) {
+        // X_s = Y_s - M_sf X_f (Y, M precomputed on the third stream)
+        const GeoPair &p = gp[gj];
+        if (cudaStreamWaitEvent(st, ts->ev_ym[gj], 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+        ++gj;
+        const int64_t ns = s_hi - s_lo, nf = f_hi - f_lo;
+        if (left) {
+          Problem P = problem(ns, nq, -1.f, 1.f, p.Y + c0 * p.ldy, p.ldy, Bq + s_lo, ldb);
+          P.seg[0].a = dense(p.M, p.ldm, false);
+          P.seg[0].b = dense(Bq + f_lo, ldb, true);
+          P.seg[0].K = nf;
+          P.max_sms = first_sms;
+          return run_problem(P, st, sms);
+        }
+        Problem P = problem(mq, ns, -1.f, 1.f, p.Y + c0, p.ldy, Bq + s_lo * ldb, ldb);
+        P.seg[0].a = dense(Bq + f_lo * ldb, ldb, false);
+        P.seg[0].b = dense(p.M, p.ldm, true);
+        P.seg[0].K = nf;
+        P.max_sms = first_sms;
+        return run_problem(P, st, sms);
+      }
       if ((rc2 = update(f_lo, f_hi, s_lo, s_hi, scaled ? 1.f : alpha, true))) return rc2;
       return leaf(s_lo, s_hi - s_lo, h, true, true);
     };
@@ -994,7 +1243,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
       if (q1 - q0 == 1) {
         const int64_t p = forward ? q0 : npanel - 1 - q0;
         const int64_t p0 = p * NBO, pr = imin(NBO, nt - p0);
-        if (q0 == 0) return geo(p0, NBO, scaled);       // the first processed panel (p == pfirst)
+        if (q0 == 0) return first_done ? 0 : geo(p0, NBO, scaled);   // the first processed panel
         return leaf(p0, pr, NBO, scaled, in_w);
       }
       const int64_t mid = q0 + (q1 - q0) / 2;
@@ -1010,8 +1259,11 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
     if (st != s && (cudaEventRecord(ts->ev_join[q], st) != cudaSuccess ||
                     cudaStreamWaitEvent(s, ts->ev_join[q], 0) != cudaSuccess)) return BLAS3_ERR_CUDA;
   }
+  if (ym_ready && cudaStreamWaitEvent(s, ts->ev_ym[gp.size() - 1], 0) != cudaSuccess)
+    return BLAS3_ERR_CUDA;
   // the side streams' last levels are part of this call (scratch is freed on s)
-  if (nlvl > 0 && cudaStreamWaitEvent(s, ts->ev_lvl[nlvl - 1], 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+  if (!first_done && nlvl > 0 && cudaStreamWaitEvent(s, ts->ev_lvl[nlvl - 1], 0) != cudaSuccess)
+    return BLAS3_ERR_CUDA;
   if (nlvl > 0 && npanel > 1 && cudaStreamWaitEvent(s, ts->ev_lvl2[nlvl - 1], 0) != cudaSuccess)
     return BLAS3_ERR_CUDA;
   return finish(0);

@@ -5,7 +5,9 @@ tcgen05 kernel (BLAS3_TC_CTA=2, cta_group::2) and the static tile schedule
 picks the pair kernel for large problems), whole tiles only
 (BLAS3_TC_SPLIT=0: no k-sliced tail), and the GM_map adaptor forced on at
 every size (BLAS3_GM_MAP=1: transposed / symmetric / triangular operands
-materialised in global memory first, the default only for large problems).  Each child process runs a representative subset of the
+materialised in global memory first, the default only for large problems), and
+STRSM's first panel by update + solve instead of the precomputed Y - M X form
+(BLAS3_TRSM_FIRST_YM=0).  Each child process runs a representative subset of the
 parity suite (every routine family, both transposes/sides) on that variant."""
 import os
 import subprocess
@@ -19,9 +21,9 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 @pytest.mark.parametrize("env", [{"BLAS3_TC_CTA": "1"}, {"BLAS3_TC_CTA": "2"}, {"BLAS3_TC_STATIC": "1"},
                                  {"BLAS3_TC_SPLIT": "0"}, {"BLAS3_TC_CTA": "1", "BLAS3_TC_SPLIT": "0"},
-                                 {"BLAS3_GM_MAP": "1"}],
+                                 {"BLAS3_GM_MAP": "1"}, {"BLAS3_TRSM_FIRST_YM": "0"}],
                          ids=["single_cta", "cta_pair", "static_schedule", "no_split", "single_cta_no_split",
-                              "gm_map"])
+                              "gm_map", "trsm_no_first_ym"])
 def test_variant_subset(env):
     import torch
     if not torch.cuda.is_available():
