@@ -5,7 +5,10 @@
 // the structure of every routine applied while the tile is staged to shared
 // memory (mirror / zero-select / unit diagonal, via load_op) and the uplo
 // mask applied in the epilogue.  128x128 CTA tile, BK=8, 256 threads, 8x8
-// outputs per thread, register-prefetched double buffer.  It is the route for
+// outputs per thread, register-prefetched double buffer, one CTA per SM
+// (251 registers: the 64 accumulators and both operand prefetches stay in
+// registers, no spills).  Dense operands of interior tiles are fetched by
+// per-thread pointers advanced by a constant stride per k-block.  It is the route for
 // arguments TMA cannot address (unaligned pointers, ld % 4 != 0) and the FP32
 // comparison point for the 3xTF32 path.
 //
@@ -56,7 +59,7 @@ __device__ __forceinline__ void stash(float (*dst)[BM + PADS], bool kr, const fl
 }
 }  // namespace
 
-__global__ void __launch_bounds__(NT, 2)
+__global__ void __launch_bounds__(NT, 1)
 simt_structured_gemm(const Problem P) {
   __shared__ __align__(16) Stage st[2];
   const int tid = threadIdx.x, tx = tid % 16, ty = tid / 16;
@@ -90,9 +93,36 @@ simt_structured_gemm(const Problem P) {
       k0 = (k0 / BK) * BK;
       if (k1 <= k0) continue;
       const bool akr = prefers_kr(oa), bkr = prefers_kr(ob);
+      // dense operands of interior tiles: per-thread element pointers, advanced
+      // by a constant stride per k-block (no per-element structure or bounds
+      // logic); the k-tail and structured / edge operands take fetch()
+      const bool fa = oa.kind == OP_DENSE && m0 + BM <= P.M;
+      const bool fb = ob.kind == OP_DENSE && n0 + BN <= P.N;
+      const float *pa[EPT], *pb[EPT];
+      const int64_t sa = akr ? BK : BK * oa.ld, sb = bkr ? BK : BK * ob.ld;
+#pragma unroll
+      for (int i = 0; i < EPT; ++i) {
+        int r, k;
+        elem_map(akr, tid, i, r, k);
+        pa[i] = akr ? oa.ptr + (k0 + k) + (m0 + r) * oa.ld : oa.ptr + (m0 + r) + (k0 + k) * oa.ld;
+        elem_map(bkr, tid, i, r, k);
+        pb[i] = bkr ? ob.ptr + (k0 + k) + (n0 + r) * ob.ld : ob.ptr + (n0 + r) + (k0 + k) * ob.ld;
+      }
+      auto fetch_a = [&](int64_t kb, float (&v)[EPT]) {
+        if (fa && kb + BK <= K) {
+#pragma unroll
+          for (int i = 0; i < EPT; ++i) v[i] = __ldg(pa[i] + ((kb - k0) / BK) * sa);
+        } else fetch(oa, akr, P.M, K, m0, kb, v);
+      };
+      auto fetch_b = [&](int64_t kb, float (&v)[EPT]) {
+        if (fb && kb + BK <= K) {
+#pragma unroll
+          for (int i = 0; i < EPT; ++i) v[i] = __ldg(pb[i] + ((kb - k0) / BK) * sb);
+        } else fetch(ob, bkr, P.N, K, n0, kb, v);
+      };
       float va[EPT], vb[EPT];
-      fetch(oa, akr, P.M, K, m0, k0, va);
-      fetch(ob, bkr, P.N, K, n0, k0, vb);
+      fetch_a(k0, va);
+      fetch_b(k0, vb);
       int buf = 0;
       __syncthreads();  // previous tile/segment finished reading smem
       stash(st[0].a, akr, va);
@@ -101,8 +131,8 @@ simt_structured_gemm(const Problem P) {
       for (int64_t kb = k0; kb < k1; kb += BK) {
         const bool more = kb + BK < k1;
         if (more) {
-          fetch(oa, akr, P.M, K, m0, kb + BK, va);
-          fetch(ob, bkr, P.N, K, n0, kb + BK, vb);
+          fetch_a(kb + BK, va);
+          fetch_b(kb + BK, vb);
         }
         const Stage &S = st[buf];
 #pragma unroll
@@ -152,7 +182,13 @@ simt_structured_gemm(const Problem P) {
 int launch_simt(const Problem &P, cudaStream_t stream, int num_sms) {
   int64_t tiles = Tiles<BM, BN>::count(P) * (P.nbatch > 0 ? P.nbatch : 1);
   if (tiles == 0) return 0;
-  int64_t grid = imin(tiles, (int64_t)num_sms * 2);
+  static int occ = 0;
+  if (occ == 0 && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, simt_structured_gemm, NT, 0) !=
+                   cudaSuccess || occ < 1)) {
+    cudaGetLastError();
+    occ = 1;
+  }
+  int64_t grid = imin(tiles, (int64_t)num_sms * occ);
   simt_structured_gemm<<<(unsigned)grid, NT, 0, stream>>>(P);
   note_launch(1);
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
