@@ -178,6 +178,15 @@ int blas3_get_math_mode(void);
  *                          panel (its doubling, Y, M and the X chain) as ONE
  *                          persistent dependency-driven launch; 0: separate
  *                          launches on side streams
+ *   BLAS3_OPT_TRSM_FIRST_SPLIT [BLAS3_TRSM_FIRST_SPLIT] F (power of 2): only
+ *                          the first F rows (L) / columns (R) of the first
+ *                          panel (processing order) run as the fused chain;
+ *                          the rest of the panel is swept right-looking in
+ *                          blocks of F, F, 2F, 4F, ...: the block solved last
+ *                          updates EVERY later row of the matrix in one bulk
+ *                          GEMM, then the next block is one leaf solve (its
+ *                          inverse doubled up front on a side stream).
+ *                          0 (default): the whole first panel in the chain
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */
@@ -187,7 +196,8 @@ enum {
     BLAS3_OPT_TC_SPLIT = 6, BLAS3_OPT_TC_STATIC = 7, BLAS3_OPT_PDL = 8,
     BLAS3_OPT_TRSM_NB = 9, BLAS3_OPT_TRSM_SLABS = 10, BLAS3_OPT_TRSM_SLAB_MIN = 11,
     BLAS3_OPT_TRSM_RESERVE = 12, BLAS3_OPT_TRSM_GEO_LEAF = 13, BLAS3_OPT_TRSM_FUSED = 14,
-    BLAS3_OPT_TRSM_FIRST_YM = 15, BLAS3_OPT_TRSM_FIRST_FUSED = 16, BLAS3_OPT_COUNT = 17
+    BLAS3_OPT_TRSM_FIRST_YM = 15, BLAS3_OPT_TRSM_FIRST_FUSED = 16, BLAS3_OPT_TRSM_FIRST_SPLIT = 17,
+    BLAS3_OPT_COUNT = 18
 };
 int blas3_set_option(int key, int64_t value);
 int64_t blas3_get_option(int key);

@@ -44,6 +44,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TRSM_FUSED", 0, 0, 1, false},
     {"BLAS3_TRSM_FIRST_YM", 1, 0, 1, false},
     {"BLAS3_TRSM_FIRST_FUSED", 1, 0, 1, false},
+    {"BLAS3_TRSM_FIRST_SPLIT", 0, 0, 8192, true},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;
@@ -808,14 +809,15 @@ static int strsm_fused(const TrsmGeom &g, cudaStream_t s, int sms) {
 // inv(op(A)_ss)) and X_j = Y_j - M_j X_f (waits for M_j, and on its slab for
 // Y_j and every earlier chain phase).  Returns 1 if not fusable (nothing
 // enqueued), 0 on success, < 0 on a CUDA error.  The 128-block inverses must
-// already be on the stream.
+// already be on the stream.  [r_lo, r_hi): the aligned block whose doubling
+// levels the launch builds (default: the whole panel).
 static int strsm_first_fused(const TrsmGeom &g, const std::vector<GeoPair> &gp, int64_t pfirst,
-                             cudaStream_t s, int sms) {
+                             cudaStream_t s, int sms, int64_t r_lo = -1, int64_t r_hi = -1) {
   const int64_t NBO = g.NBO, nt = g.nt;
-  const int64_t o = pfirst * NBO;
+  if (r_lo < 0) { r_lo = pfirst * NBO; r_hi = imin(nt, r_lo + NBO); }   // doubling range: the panel
   std::vector<LevelProblem> lv;
-  trsm_doubling_problems(g.A + o * (1 + g.lda), g.lda, imin(NBO, nt - o), g.lower, g.D + pfirst * NBO * NBO,
-                         g.Tw, lv);
+  trsm_doubling_problems(g.A + r_lo * (1 + g.lda), g.lda, r_hi - r_lo, g.lower,
+                         g.D + pfirst * NBO * NBO + (r_lo - pfirst * NBO) * (1 + NBO), g.Tw, lv);
   auto level_of = [](int64_t w) { int l = -1; for (int64_t w2 = 256; w2 <= w; w2 *= 2) ++l; return l; };
   int need = 0;                                         // levels used: inv of every s block
   for (const GeoPair &p : gp) need = imax(need, level_of(p.h) + 1);
@@ -827,13 +829,14 @@ static int strsm_first_fused(const TrsmGeom &g, const std::vector<GeoPair> &gp, 
     return (int)ph.size() - 1;
   };
   uint32_t lvl_mask[MAX_LEVELS] = {};
-  for (int l = 0; l < need; ++l) {
+  auto emit_level = [&](int l) {
     uint32_t step1 = 0;
     for (const LevelProblem &q : lv)
       if (q.lvl == l && q.step == 1) step1 |= 1u << add(q.P, l > 0 ? lvl_mask[l - 1] : 0u, 0u);
     for (const LevelProblem &q : lv)
       if (q.lvl == l && q.step == 2) lvl_mask[l] |= 1u << add(q.P, step1, 0u);
-  }
+  };
+  for (int l = 0; l < need; ++l) emit_level(l);
   // first leaf: the block solved before every pair's f
   const int64_t l_lo = gp[0].f_lo, l_cnt = gp[0].f_hi - gp[0].f_lo;
   if (l_cnt > 256) return 1;
@@ -952,7 +955,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   const size_t d_bytes = (size_t)npanel * NBO * NBO * sizeof(float);
   // doubling scratch: nt/2sz pairs x sz^2 floats at the widest level
   const size_t t_rest = (size_t)nt * (NBO / 4), t_first = (size_t)NBO * NBO / 4;
-  const size_t t_bytes = (t_rest + t_first) * sizeof(float);
+  const size_t t_bytes = (t_rest + 2 * t_first) * sizeof(float);   // + first-split s blocks
   const size_t w_bytes = (size_t)NBO * other * sizeof(float);        // one solved panel
   Scratch D, Tw, W;
   if ((rc = get_scratch(D, d_bytes, s, aop_bytes))) return rc;
@@ -1035,13 +1038,43 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // caller's stream; else its levels on the high-priority side stream and
   // the Y/M precompute on a third stream, the chain on the slab streams.
   bool first_done = false, ym_ready = false;
+  // BLAS3_OPT_TRSM_FIRST_SPLIT = F: only the first F rows (L) / columns (R)
+  // of the first panel (processing order) run as the latency-bound fused
+  // chain.  The outer geometric pairs (s blocks of width F, 2F, ...) leave it:
+  // after the chain, the block solved last updates EVERY later row of the
+  // matrix in one bulk GEMM (full machine), then the next s block is one
+  // leaf solve -- a right-looking sweep with geometrically growing blocks.
+  // The s blocks' inverses are doubled up front on the high-priority side
+  // stream, concurrently with the chain (they do not depend on X).
+  std::vector<GeoPair> outer;                         // popped pairs, inner -> outer
+  const int64_t fsplit = opt(BLAS3_OPT_TRSM_FIRST_SPLIT);
   if (opt(BLAS3_OPT_TRSM_FIRST_FUSED) && tensor_mode() && !gp.empty()) {
+    if (fsplit > 0)
+      while (gp.size() >= 2 && gp.back().h >= fsplit && outer.size() < (size_t)MAX_LEVELS) { outer.insert(outer.begin(), gp.back()); gp.pop_back(); }
+    const int64_t c_lo = outer.empty() ? -1 : outer[0].f_lo, c_hi = outer.empty() ? -1 : outer[0].f_hi;
     const TrsmGeom g{left, lower, ta, unit, lower_op, forward, m, n, nt, NBO, npanel, other, alpha,
                      A, lda, B, ldb, D.p, Tw.p + t_rest, W.p};
-    rc = strsm_first_fused(g, gp, pfirst, s, sms);
+    rc = strsm_first_fused(g, gp, pfirst, s, sms, c_lo, c_hi);
     if (rc < 0) return rc;
     first_done = rc == 0;
+    if (!first_done) {                                // not fusable: no split either
+      for (const GeoPair &p : outer) gp.push_back(p);
+      outer.clear();
+    }
+    if (!outer.empty()) {
+      // s-block inverses: sub-panel doubling per popped pair on the side stream
+      if (cudaStreamWaitEvent(ts->side, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+      for (size_t j = 0; j < outer.size(); ++j) {
+        const GeoPair &p = outer[j];
+        if ((rc = trsm_panel_doubling(A + p.s_lo * (1 + lda), lda, p.s_hi - p.s_lo, lower,
+                                      D.p + pfirst * NBO * NBO + (p.s_lo - pfirst * NBO) * (1 + NBO),
+                                      Tw.p + t_rest + t_first, ts->side, sms, ts->ev_ym)))
+          return rc;
+        if (cudaEventRecord(ts->ev_lvl[j], ts->side) != cudaSuccess) return BLAS3_ERR_CUDA;
+      }
+    }
   }
+  const bool split = !outer.empty();
   if (!first_done) {
     const int64_t o = pfirst * NBO;
     if ((rc = trsm_panel_doubling(A + o * (1 + lda), lda, imin(NBO, nt - o), lower,
@@ -1120,14 +1153,16 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
     float *Bq = left ? B + c0 * ldb : B + c0;
     float *Wq = left ? W.p + c0 * NBO : W.p + c0;
     const int64_t mq = left ? m : c1 - c0, nq = left ? c1 - c0 : n;
-    int waited = -1;                                  // highest first-panel level waited on
+    int waited = first_done ? nlvl : -1;              // highest first-panel level waited on
+                                                      // (the fused launch built them all)
     bool waited_rest = false;                         // the other panels' inverses waited on
 
     // leaf: rows (L) / columns (R) [e0, e0 + cnt) of X, aligned block width wblk
     // kernels of the first panel leave SMs to the latency-bound doubling
     // chain of that panel (high-priority side stream)
     const int32_t first_sms = (int32_t)imax(sms / 2, sms - trsm_reserve());
-    auto leaf = [&](int64_t e0, int64_t cnt, int64_t wblk, bool scaled, bool in_w) -> int {
+    int64_t app_lo = 0, app_hi = 0;                   // split sweep: updates already applied
+    auto leaf = [&](int64_t e0, int64_t cnt, int64_t wblk, bool scaled, bool in_w, bool restrict_sms = true) -> int {
       int rc2;
       int lv = -1;                                    // doubling level that built inv(block)
       for (int64_t w2 = 256; w2 <= wblk; w2 *= 2) ++lv;
@@ -1151,7 +1186,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
         P.seg[0].K = cnt;
         P.rev_m = tri_kle(P.seg[0].a);
         P.outer = 1;                     // all longest m-rows first (LPT)
-        if (e0 / NBO == pfirst) P.max_sms = first_sms;
+        if (e0 / NBO == pfirst && restrict_sms) P.max_sms = first_sms;
         if ((rc2 = run_problem(P, st, sms))) return rc2;
         if (!in_w && launch_copy(Bq + e0, ldb, Wq, cnt, cnt, nq, st)) return BLAS3_ERR_CUDA;
       } else {
@@ -1163,7 +1198,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
         P.seg[0].K = cnt;
         P.rev_n = tri_kle(P.seg[0].b);
         P.outer = 2;
-        if (e0 / NBO == pfirst) P.max_sms = first_sms;
+        if (e0 / NBO == pfirst && restrict_sms) P.max_sms = first_sms;
         if ((rc2 = run_problem(P, st, sms))) return rc2;
         if (!in_w && launch_copy(Bq + e0 * ldb, ldb, Wq, m, mq, cnt, st)) return BLAS3_ERR_CUDA;
       }
@@ -1171,7 +1206,9 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
     };
     // update: rows (L) / columns (R) [o_lo, o_hi) <- a1 * B_o - op(A)(o, k) X_k, k in [k_lo, k_hi);
     // to_w: the result goes to W (the next operation is the leaf solve of o)
-    auto update = [&](int64_t k_lo, int64_t k_hi, int64_t o_lo, int64_t o_hi, float a1, bool to_w) -> int {
+    auto update = [&](int64_t k_lo, int64_t k_hi, int64_t o_lo, int64_t o_hi, float a1, bool to_w,
+                      bool restrict_sms = true) -> int {
+      const bool rs = restrict_sms && o_lo / NBO == pfirst && (o_hi - 1) / NBO == pfirst;
       if (left) {   // Xa(r,kk) = op(A)(o_lo+r, k_lo+kk): !ta -> A(o_lo+r, k_lo+kk) rk; ta -> A(k_lo+kk, o_lo+r) kr
         const float *pa = ta ? A + k_lo + o_lo * lda : A + o_lo + k_lo * lda;
         Problem P = to_w ? problem(o_hi - o_lo, nq, -1.f, a1, Bq + o_lo, ldb, Wq, o_hi - o_lo)
@@ -1179,7 +1216,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
         P.seg[0].a = dense(pa, lda, ta);
         P.seg[0].b = dense(Bq + k_lo, ldb, true);
         P.seg[0].K = k_hi - k_lo;
-        if (o_lo / NBO == pfirst) P.max_sms = first_sms;
+        if (rs) P.max_sms = first_sms;
         return run_problem(P, st, sms);
       }
       // B(:,o) <- a1*B(:,o) - X_k * op(A)(k, o):
@@ -1190,7 +1227,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
       P.seg[0].a = dense(Bq + k_lo * ldb, ldb, false);
       P.seg[0].b = dense(pb, lda, !ta);
       P.seg[0].K = k_hi - k_lo;
-      if (o_lo / NBO == pfirst) P.max_sms = first_sms;
+      if (rs) P.max_sms = first_sms;
       return run_problem(P, st, sms);
     };
     // geometric solve of the aligned block [lo, lo + w) (clipped to nt): the
@@ -1251,15 +1288,39 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
       int64_t k_lo, k_hi, o_lo, o_hi;
       elem(q0, mid, k_lo, k_hi);                       // solved part
       elem(mid, q1, o_lo, o_hi);                       // part to update
+      if (split) {                                     // updates applied by the split sweep
+        if (forward && k_lo < app_hi) k_lo = imax(k_lo, app_hi);
+        if (!forward && k_hi > app_lo) k_hi = imin(k_hi, app_lo);
+      }
       const bool to_w = (q1 - mid == 1);               // updated panel goes straight to W
       if ((rc2 = update(k_lo, k_hi, o_lo, o_hi, scaled ? 1.f : alpha, to_w))) return rc2;
       return rec(mid, q1, true, to_w);
     };
-    if ((rc = rec(0, npanel, false, false))) return rc;
+    if (split) {
+      // right-looking over the popped pairs: the block solved last [a_lo, a_hi)
+      // updates every later row (L) / column (R) in one bulk GEMM, then the
+      // next s block is one leaf (its inverse from the side stream)
+      int64_t a_lo = outer[0].f_lo, a_hi = outer[0].f_hi;
+      for (size_t j = 0; j < outer.size(); ++j) {
+        const GeoPair &p = outer[j];
+        const int64_t r_lo = forward ? a_hi : 0, r_hi = forward ? nt : a_lo;
+        // when s is all that is left, the update goes to W and the leaf reads W
+        const bool last = r_lo == p.s_lo && r_hi == p.s_hi;
+        if ((rc = update(a_lo, a_hi, r_lo, r_hi, j == 0 ? alpha : 1.f, last, false))) return rc;
+        if (cudaStreamWaitEvent(st, ts->ev_lvl[j], 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+        if ((rc = leaf(p.s_lo, p.s_hi - p.s_lo, p.h, true, last, false))) return rc;
+        a_lo = p.s_lo; a_hi = p.s_hi;
+      }
+      app_lo = forward ? 0 : a_hi;                    // k ranges whose update is applied
+      app_hi = forward ? a_lo : nt;
+    }
+    if ((rc = rec(0, npanel, split, false))) return rc;
     if (st != s && (cudaEventRecord(ts->ev_join[q], st) != cudaSuccess ||
                     cudaStreamWaitEvent(s, ts->ev_join[q], 0) != cudaSuccess)) return BLAS3_ERR_CUDA;
   }
   if (ym_ready && cudaStreamWaitEvent(s, ts->ev_ym[gp.size() - 1], 0) != cudaSuccess)
+    return BLAS3_ERR_CUDA;
+  if (split && cudaStreamWaitEvent(s, ts->ev_lvl[outer.size() - 1], 0) != cudaSuccess)
     return BLAS3_ERR_CUDA;
   // the side streams' last levels are part of this call (scratch is freed on s)
   if (!first_done && nlvl > 0 && cudaStreamWaitEvent(s, ts->ev_lvl[nlvl - 1], 0) != cudaSuccess)

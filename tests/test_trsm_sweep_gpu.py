@@ -40,14 +40,18 @@ def b3():
     return m
 
 
+@pytest.mark.parametrize("split", [0, 512, 1024], ids=["chain", "first_split512", "first_split1024"])
 @pytest.mark.parametrize("side,uplo,ta,diag", V16)
-def test_strsm_multi_panel_multi_slab(b3, oracle_mod, side, uplo, ta, diag):
+def test_strsm_multi_panel_multi_slab(b3, oracle_mod, side, uplo, ta, diag, split):
+    """split=1: BLAS3_OPT_TRSM_FIRST_SPLIT (first panel's second half by a bulk
+    update + one leaf instead of the chain)."""
     ka, other = 2600, 4500                 # 2 panels (ragged), 2 slabs (ragged last)
     m, n = (ka, other) if side == "L" else (other, ka)
     A = gen.triangular_dd(ka, uplo, diag, "sweep-a")
     B = gen.uniform(m, n, "sweep-b")
     dB = to_dev(B)
-    b3.strsm(side, uplo, ta, diag, AL, to_dev(A), dB)
+    with b3.options(trsm_first_split=split):
+        b3.strsm(side, uplo, ta, diag, AL, to_dev(A), dB)
     X = f64(to_host(dB))
     T = op(tri_full(A, uplo, diag, ka), ta)
     # samples straddle the slab boundary (2048 + 256 k) and the ragged tail
@@ -87,13 +91,15 @@ def test_strsm_fused_is_one_launch(b3, oracle_mod, side):
     assert fro(X1 - X0) / fro(X0) <= 1e-6
 
 
-@pytest.mark.parametrize("fused", ["0", "1"])
-def test_strsm_small_panels_many_slabs(fused):
+@pytest.mark.parametrize("nb,fused,split", [("256", "0", "0"), ("256", "1", "0"), ("1024", "0", "512"),
+                                            ("8192", "0", "512")],
+                         ids=["multi_launch", "fused", "nb1024_first_split", "one_panel_first_split"])
+def test_strsm_small_panels_many_slabs(nb, fused, split):
     import torch
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
-    env = {**os.environ, "BLAS3_TRSM_NB": "256", "BLAS3_TRSM_SLABS": "4", "BLAS3_TRSM_SLAB_MIN": "256",
-           "BLAS3_TRSM_FUSED": fused}
+    env = {**os.environ, "BLAS3_TRSM_NB": nb, "BLAS3_TRSM_SLABS": "4", "BLAS3_TRSM_SLAB_MIN": "256",
+           "BLAS3_TRSM_FUSED": fused, "BLAS3_TRSM_FIRST_SPLIT": split}
     cmd = [sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k", "strsm",
            os.path.join(ROOT, "tests", "test_parity_gpu.py")]
     r = subprocess.run(cmd, env=env, cwd=ROOT, capture_output=True, text=True, timeout=900)

@@ -38,6 +38,8 @@ def chain():
 
 calls["chain"] = chain
 fn = calls[which]
+for k, v in json.loads(os.environ.get("TL_OPTS", "{}")).items():   # tuning options
+    b3.set_option(k, v)
 for _ in range(3):
     fn()
 torch.cuda.synchronize()
