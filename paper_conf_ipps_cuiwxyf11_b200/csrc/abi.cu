@@ -309,7 +309,10 @@ int blas3_ssymm(char side, char uplo, int64_t m, int64_t n, float alpha, const f
   if (alpha == 0.f) return finish(launch_scale(C, ldc, m, n, beta, 0, s) ? BLAS3_ERR_CUDA : 0);
   Problem P = problem(m, n, alpha, beta, C, ldc, C, ldc);
   const int64_t ka = left ? m : n;
-  if (tensor_mode() && use_gm_map(ka, left ? n : m, BLAS3_OPT_GM_MIN_SYMM)) {
+  // (SIMT mode: always from order 512 -- the materialisation is ~0.5% of the
+  // FFMA GEMM, and the shadow area would otherwise be read uncoalesced)
+  if (tensor_mode() ? use_gm_map(ka, left ? n : m, BLAS3_OPT_GM_MIN_SYMM)
+                    : (opt(BLAS3_OPT_GM_MAP) != 0 && (opt(BLAS3_OPT_GM_MAP) == 1 || ka >= 512))) {
     // GM_map: sym(A) materialised as a full ka x ka matrix, then a plain GEMM
     Scratch Wm;
     const int64_t ldw = ld4(ka);

@@ -7,8 +7,9 @@
 // mask applied in the epilogue.  128x128 CTA tile, BK=8, 256 threads, 8x8
 // outputs per thread, register-prefetched double buffer, one CTA per SM
 // (251 registers: the 64 accumulators and both operand prefetches stay in
-// registers, no spills).  Dense operands of interior tiles are fetched by
-// per-thread pointers advanced by a constant stride per k-block.  It is the route for
+// registers, no spills).  Dense operands of interior tiles -- and the blocks
+// of structured operands that lie entirely inside one stored orientation --
+// are fetched by per-thread pointers advanced by a constant stride per k-block.  It is the route for
 // arguments TMA cannot address (unaligned pointers, ld % 4 != 0) and the FP32
 // comparison point for the 3xTF32 path.
 //
@@ -37,6 +38,19 @@ __device__ __forceinline__ void elem_map(bool kr, int tid, int i, int &r, int &k
 }
 __device__ __forceinline__ bool prefers_kr(const OpDesc &o) {
   return o.kind == OP_DENSE ? o.kr != 0 : (o.kind == OP_TRI ? o.swap != 0 : false);
+}
+
+// A BM x BK block of a structured operand that the strided-pointer fetch may
+// read as stored: TRI blocks strictly inside the nonzero triangle (or any
+// block of a zero-filled, non-unit TRI workspace), SYM blocks entirely in the
+// stored (rk) triangle.  Diagonal-touching / shadow blocks take fetch().
+__device__ __forceinline__ bool plain_block(const OpDesc &o, int64_t r0, int64_t kb) {
+  if (o.kind == OP_DENSE) return true;
+  if (o.kind == OP_TRI) {
+    if (o.zero_blank && !o.unit) return true;
+    return tri_kle(o) ? (kb + BK <= r0) : (kb >= r0 + BM);
+  }
+  return o.lower ? (kb + BK - 1 <= r0) : (kb >= r0 + BM - 1);
 }
 
 __device__ __forceinline__ void fetch(const OpDesc &o, bool kr, int64_t R, int64_t K, int64_t r0,
@@ -96,8 +110,7 @@ simt_structured_gemm(const Problem P) {
       // dense operands of interior tiles: per-thread element pointers, advanced
       // by a constant stride per k-block (no per-element structure or bounds
       // logic); the k-tail and structured / edge operands take fetch()
-      const bool fa = oa.kind == OP_DENSE && m0 + BM <= P.M;
-      const bool fb = ob.kind == OP_DENSE && n0 + BN <= P.N;
+      const bool fa = m0 + BM <= P.M, fb = n0 + BN <= P.N;
       const float *pa[EPT], *pb[EPT];
       const int64_t sa = akr ? BK : BK * oa.ld, sb = bkr ? BK : BK * ob.ld;
 #pragma unroll
@@ -109,13 +122,13 @@ simt_structured_gemm(const Problem P) {
         pb[i] = bkr ? ob.ptr + (k0 + k) + (n0 + r) * ob.ld : ob.ptr + (n0 + r) + (k0 + k) * ob.ld;
       }
       auto fetch_a = [&](int64_t kb, float (&v)[EPT]) {
-        if (fa && kb + BK <= K) {
+        if (fa && kb + BK <= K && plain_block(oa, m0, kb)) {
 #pragma unroll
           for (int i = 0; i < EPT; ++i) v[i] = __ldg(pa[i] + ((kb - k0) / BK) * sa);
         } else fetch(oa, akr, P.M, K, m0, kb, v);
       };
       auto fetch_b = [&](int64_t kb, float (&v)[EPT]) {
-        if (fb && kb + BK <= K) {
+        if (fb && kb + BK <= K && plain_block(ob, n0, kb)) {
 #pragma unroll
           for (int i = 0; i < EPT; ++i) v[i] = __ldg(pb[i] + ((kb - k0) / BK) * sb);
         } else fetch(ob, bkr, P.N, K, n0, kb, v);
