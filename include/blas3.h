@@ -20,7 +20,11 @@
  *             stream-ordered scratch (cudaMallocAsync) where a routine needs
  *             it (STRMM, STRSM).
  *  Streams    Work is enqueued on `stream` (NULL = legacy default stream) and
- *             is asynchronous: no entry point synchronises the host.
+ *             is asynchronous: no entry point synchronises the host.  Calls
+ *             can be captured into a CUDA graph (stream capture) and
+ *             replayed; the first call on a given stream allocates that
+ *             stream's library state (tile-scheduler and split-tail
+ *             buffers), so make one eager call on the capture stream first.
  *  Aliasing   C must not alias A or B (as in BLAS); B is overwritten in place
  *             by STRMM/STRSM.
  *  Sizes      int64_t (N = 32768 needs byte offsets beyond 2^32); otherwise

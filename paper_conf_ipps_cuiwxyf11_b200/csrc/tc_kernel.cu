@@ -146,8 +146,9 @@ struct TcParamsT {
   CUtensorMap maps[NMAPS];
   PhaseDesc ph[NPH];
   int32_t nphase;
-  uint32_t *tile_ctr;      // dynamic tile scheduler counter, or null (static schedule)
-  uint32_t tile_base;      // its value when this launch starts
+  uint32_t *tile_ctr;      // dynamic tile scheduler counter, or null (static schedule);
+                           // 0 when the launch starts and left at 0 by its last claim
+  uint32_t tile_claims;    // atomic claims this launch makes in total
   // Split tail (wave quantisation, single-phase launches): work items [0, khead)
   // are whole tiles; the last (ntiles - khead) tiles are cut into ksplit
   // k-slices each, item khead + j -> tile khead + j / ksplit, slice j % ksplit.
@@ -582,10 +583,17 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           // (the first item of every producer is its own id: no claim round
           // trip -- except in a fused launch, whose items are claimed strictly
           // in dependency order by running CTAs)
-          if (FUSED) tb = (int64_t)(uint32_t)(atomicAdd(prm.tile_ctr, 1u) - prm.tile_base);
-          else tb = (prm.tile_ctr == nullptr || qi == 0)
-                        ? cid + (int64_t)qi * ncl
-                        : ncl + (int64_t)(uint32_t)(atomicAdd(prm.tile_ctr, 1u) - prm.tile_base);
+          if ((FUSED || qi > 0) && prm.tile_ctr != nullptr) {
+            const uint32_t v = atomicAdd(prm.tile_ctr, 1u);
+            // the launch's last claim (claims are totally ordered, and no
+            // producer claims again after a failing one) resets the counter,
+            // so every launch -- and every replay of a captured CUDA graph --
+            // starts from 0
+            if (v == prm.tile_claims - 1) atomicExch(prm.tile_ctr, 0u);
+            tb = FUSED ? (int64_t)v : ncl + (int64_t)v;
+          } else {
+            tb = cid + (int64_t)qi * ncl;
+          }
           if (tb >= prm.nitems) tb = -1;
           BLAS3_TRACE(2);
           ptx::mbar_wait(&bars->tq_empty[slot], par ^ 1);
@@ -1091,18 +1099,16 @@ static int launch_cg(PRM &prm, cudaStream_t stream, int num_sms, bool allow_pdl 
   return (e == cudaSuccess && cudaGetLastError() == cudaSuccess) ? 0 : -1;
 }
 
-// Dynamic tile scheduling counters: a ring of per-launch slots per device.
-// A launch makes exactly ntiles + producers claims on its slot (every tile
-// once, then one failing claim per producer), so the host knows the slot's
-// value when the launch is over and passes it as the base of the next launch
-// on that slot -- no memset node per launch.  (A slot is reused only 256
-// launches later, long after its previous launch has drained.)
-struct TileCounter { uint32_t *ctr; uint32_t base; };
-static bool tile_counter(TileCounter &tc, uint32_t claims) {
+// Dynamic tile scheduling counters: a ring of per-launch slots per device
+// (concurrent launches on different streams never share one).  Every slot is
+// 0 between launches: the launch's last claim resets it on the device
+// (tc_structured_gemm), so a captured CUDA graph replays correctly and no
+// memset node is needed.
+struct TileCounter { uint32_t *ctr; };
+static bool tile_counter(TileCounter &tc) {
   constexpr int SLOTS = 256;
   static uint32_t *ring[64] = {};
   static uint32_t next[64] = {};
-  static uint32_t value[64][SLOTS] = {};
   int d = 0;
   if (cudaGetDevice(&d) != cudaSuccess || d < 0 || d >= 64) return false;
   if (!ring[d]) {
@@ -1115,8 +1121,6 @@ static bool tile_counter(TileCounter &tc, uint32_t claims) {
   }
   const uint32_t slot = next[d]++ % SLOTS;
   tc.ctr = ring[d] + slot * 32;                     // 128-B apart
-  tc.base = value[d][slot];
-  value[d][slot] += claims;                         // wraps mod 2^32 consistently
   return true;
 }
 
@@ -1205,9 +1209,9 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
     TileCounter tc;
     // claims: (items - producers) beyond the first wave + one failing claim per producer
     if (tiles > 0) {
-      if (!tile_counter(tc, (uint32_t)tiles)) return -1;
+      if (!tile_counter(tc)) return -1;
       prm.tile_ctr = tc.ctr;
-      prm.tile_base = tc.base;
+      prm.tile_claims = (uint32_t)tiles;
     }
   }
   // diagnostics: BLAS3_TRACE=1 prints CTA 0's phase timeline (synchronises)
@@ -1295,9 +1299,9 @@ int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int 
   TileCounter tc;
   const int64_t units = imin(item, (int64_t)(num_sms / CG));
   if (item == 0) return 0;
-  if (!tile_counter(tc, (uint32_t)(item + units))) return -1;     // every item + one failing claim each
+  if (!tile_counter(tc)) return -1;
   prm.tile_ctr = tc.ctr;
-  prm.tile_base = tc.base;
+  prm.tile_claims = (uint32_t)(item + units);
   // diagnostics: BLAS3_TRACE=2 prints each phase's [first start, last end] (synchronises)
   static int trace = -1;
   static unsigned long long *tbuf = nullptr;

@@ -1,0 +1,101 @@
+"""CUDA-graph capture of the hot path.
+
+Every entry point is stream-ordered and host-sync-free (include/blas3.h
+"Streams"), so a caller can capture a whole chain of calls -- including
+STRSM's fork/join over side streams and its stream-ordered scratch -- into a
+CUDA graph and replay it.  The dynamic tile scheduler's claim counters are
+reset on the device by each launch's last claim, so replays start from the
+same state as eager launches.  Replays must reproduce the eager results bit
+for bit (the tile -> value computation does not depend on which CTA claims
+the tile, and split-k tails reduce their slices in a fixed order), on fresh
+inputs copied into the captured buffers, and again on a second replay.
+"""
+import numpy as np
+import pytest
+
+import blas3_inputs as gen
+from check import bits_equal, to_dev, to_host
+
+pytestmark = pytest.mark.gpu
+AL, BE = 1.5, 0.5
+
+
+@pytest.fixture(scope="module")
+def b3():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_cuiwxyf11_b200 as m
+    return m
+
+
+def _chain(b3, A, T, B, C, X):
+    b3.sgemm("N", "T", AL, A, B, BE, C)
+    b3.ssymm("L", "U", AL, A, B, BE, C)
+    b3.ssyrk("L", "N", AL, A, BE, C)
+    b3.ssyr2k("U", "T", AL, A, B, BE, C)
+    b3.strmm("L", "L", "N", "N", AL, T, X)
+    b3.strsm("L", "L", "N", "N", AL, T, X)
+    b3.strsm("R", "U", "T", "N", AL, T, X)
+
+
+@pytest.mark.parametrize("mode", ["3xtf32", "simt"])
+def test_chain_graph_replay_bit_identical(b3, mode):
+    import torch
+    b3.set_math_mode(mode)
+    n = 2304                               # several tiles, 2 STRSM panels (ragged)
+    inputs = []
+    for s in range(2):                     # two input sets: capture on one, replay both
+        inputs.append(dict(A=gen.uniform(n, n, f"g-a{s}"), T=gen.triangular_dd(n, "L", "N", f"g-t{s}"),
+                           B=gen.uniform(n, n, f"g-b{s}"), C=gen.uniform(n, n, f"g-c{s}")))
+    # eager reference results
+    eager = []
+    for inp in inputs:
+        A, T, B, C = (to_dev(inp[k]) for k in "ATBC")
+        X = B.clone()
+        _chain(b3, A, T, B, C, X)
+        torch.cuda.synchronize()
+        eager.append((to_host(C), to_host(X)))
+    # static buffers; warm up eagerly ON THE CAPTURE STREAM (per-stream library
+    # state is allocated on first use, which a capture does not allow)
+    sA, sT, sB, sC = (to_dev(inputs[0][k]) for k in "ATBC")
+    sX = sB.clone()
+    cs = torch.cuda.Stream()
+    cs.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(cs):
+        _chain(b3, sA, sT, sB, sC, sX)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=cs):
+        _chain(b3, sA, sT, sB, sC, sX)
+    for rep in range(2):
+        for s, inp in enumerate(inputs):
+            for k, buf in zip("ATBC", (sA, sT, sB, sC)):
+                buf.copy_(to_dev(inp[k]))
+            sX.copy_(sB)
+            g.replay()
+            torch.cuda.synchronize()
+            assert bits_equal(to_host(sC), eager[s][0]), f"C differs (set {s}, replay {rep})"
+            assert bits_equal(to_host(sX), eager[s][1]), f"X differs (set {s}, replay {rep})"
+    b3.set_math_mode("3xtf32")
+
+
+def test_tile_counters_survive_many_launches(b3):
+    """More launches than the scheduler's 256 counter slots, on sizes whose
+    claim counts differ per launch: every result still matches the first."""
+    import torch
+    b3.set_math_mode("3xtf32")
+    ref = None
+    for i in range(300):
+        m = 640 + 128 * (i % 5)            # 1-3 waves, with and without a split tail
+        A = gen.uniform(m, 512, "cnt-a")
+        B = gen.uniform(512, 384, "cnt-b")
+        dC = torch.zeros((384, m), device="cuda").t()
+        b3.sgemm("N", "N", 1.0, to_dev(A), to_dev(B), 0.0, dC)
+        if i % 5 == 0:
+            out = to_host(dC)
+            if ref is None:
+                ref = out
+            assert np.array_equal(out.view(np.uint32), ref.view(np.uint32))
