@@ -191,6 +191,11 @@ int blas3_get_math_mode(void);
  *                          GEMM, then the next block is one leaf solve (its
  *                          inverse doubled up front on a side stream).
  *                          0 (default): the whole first panel in the chain
+ *   BLAS3_OPT_TRSM_FIRST_ALL [BLAS3_TRSM_FIRST_ALL] 1: every panel's inverse
+ *                          doubling runs inside the first panel's fused
+ *                          launch (the levels its chain needs first, the
+ *                          rest after the chain) on all SMs; 0 (default): the
+ *                          other panels' doubling on a side stream beside it
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */
@@ -201,7 +206,7 @@ enum {
     BLAS3_OPT_TRSM_NB = 9, BLAS3_OPT_TRSM_SLABS = 10, BLAS3_OPT_TRSM_SLAB_MIN = 11,
     BLAS3_OPT_TRSM_RESERVE = 12, BLAS3_OPT_TRSM_GEO_LEAF = 13, BLAS3_OPT_TRSM_FUSED = 14,
     BLAS3_OPT_TRSM_FIRST_YM = 15, BLAS3_OPT_TRSM_FIRST_FUSED = 16, BLAS3_OPT_TRSM_FIRST_SPLIT = 17,
-    BLAS3_OPT_COUNT = 18
+    BLAS3_OPT_TRSM_FIRST_ALL = 18, BLAS3_OPT_COUNT = 19
 };
 int blas3_set_option(int key, int64_t value);
 int64_t blas3_get_option(int key);

@@ -45,6 +45,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TRSM_FIRST_YM", 1, 0, 1, false},
     {"BLAS3_TRSM_FIRST_FUSED", 1, 0, 1, false},
     {"BLAS3_TRSM_FIRST_SPLIT", 0, 0, 8192, true},
+    {"BLAS3_TRSM_FIRST_ALL", 0, 0, 1, false},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;
@@ -815,9 +816,11 @@ static int strsm_fused(const TrsmGeom &g, cudaStream_t s, int sms) {
 // already be on the stream.  [r_lo, r_hi): the aligned block whose doubling
 // levels the launch builds (default: the whole panel).
 static int strsm_first_fused(const TrsmGeom &g, const std::vector<GeoPair> &gp, int64_t pfirst,
-                             cudaStream_t s, int sms, int64_t r_lo = -1, int64_t r_hi = -1) {
+                             cudaStream_t s, int sms, int64_t r_lo = -1, int64_t r_hi = -1,
+                             bool all = false) {
   const int64_t NBO = g.NBO, nt = g.nt;
-  if (r_lo < 0) { r_lo = pfirst * NBO; r_hi = imin(nt, r_lo + NBO); }   // doubling range: the panel
+  if (all) { r_lo = 0; r_hi = nt; pfirst = 0; }        // every panel's doubling, whole grid
+  else if (r_lo < 0) { r_lo = pfirst * NBO; r_hi = imin(nt, r_lo + NBO); }   // doubling range: the panel
   std::vector<LevelProblem> lv;
   trsm_doubling_problems(g.A + r_lo * (1 + g.lda), g.lda, r_hi - r_lo, g.lower,
                          g.D + pfirst * NBO * NBO + (r_lo - pfirst * NBO) * (1 + NBO), g.Tw, lv);
@@ -911,12 +914,18 @@ static int strsm_first_fused(const TrsmGeom &g, const std::vector<GeoPair> &gp, 
     const int iy = add(PY, lmask, 0u);
     chain |= 1u << add(PX, 1u << im, chain | (1u << iy));
   }
+  if (all) {                                            // the other panels' last levels, claimed last
+    int nl = 0;
+    for (int64_t sz = 128; sz < NBO; sz *= 2) ++nl;
+    for (int l = need; l < nl; ++l) emit_level(l);
+  }
   if ((int)ph.size() > MAX_FUSED_PHASES) return 1;
   for (const FusedPhase &f : ph)
     if (!tc_eligible(f.P)) return 1;
   // the chain is latency-bound: leave SMs to the other panels' doubling,
   // which runs concurrently on a side stream
-  const int rc = launch_tc_fused(ph.data(), (int)ph.size(), s, (int)imax(sms / 2, sms - trsm_reserve()));
+  const int rc = launch_tc_fused(ph.data(), (int)ph.size(), s,
+                                 all ? sms : (int)imax(sms / 2, sms - trsm_reserve()));
   return rc == 0 ? 0 : (rc == -4 ? BLAS3_ERR_TMA : BLAS3_ERR_CUDA);
 }
 
@@ -1026,9 +1035,21 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   if (launch_trsm_diag_inv(A, lda, nt, lower, unit, D.p, NBO, s)) return BLAS3_ERR_CUDA;
   if (cudaEventRecord(ts->ev_fork, s) != cudaSuccess ||
       cudaStreamWaitEvent(ts->side, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+  // BLAS3_OPT_TRSM_FIRST_ALL: every panel's doubling inside the first panel's
+  // fused launch (levels the chain needs first, the rest claimed after the
+  // chain), on the whole grid -- no side stream competes for SMs
+  bool all_done = false;
+  if (opt(BLAS3_OPT_TRSM_FIRST_ALL) && opt(BLAS3_OPT_TRSM_FIRST_FUSED) && opt(BLAS3_OPT_TRSM_FIRST_SPLIT) == 0 &&
+      tensor_mode() && !gp.empty()) {
+    const TrsmGeom g{left, lower, ta, unit, lower_op, forward, m, n, nt, NBO, npanel, other, alpha,
+                     A, lda, B, ldb, D.p, Tw.p, W.p};
+    rc = strsm_first_fused(g, gp, pfirst, s, sms, -1, -1, true);
+    if (rc < 0) return rc;
+    all_done = rc == 0;
+  }
   // the other panels' levels (needed one panel sweep later) on a second side
   // stream, from the start
-  if (npanel > 1) {
+  if (npanel > 1 && !all_done) {
     const int64_t prest = forward ? 1 : 0, o = prest * NBO;
     if (cudaStreamWaitEvent(ts->side2, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
     if ((rc = trsm_panel_doubling(A + o * (1 + lda), lda, imin(nt, (prest + npanel - 1) * NBO) - o, lower,
@@ -1051,7 +1072,8 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // stream, concurrently with the chain (they do not depend on X).
   std::vector<GeoPair> outer;                         // popped pairs, inner -> outer
   const int64_t fsplit = opt(BLAS3_OPT_TRSM_FIRST_SPLIT);
-  if (opt(BLAS3_OPT_TRSM_FIRST_FUSED) && tensor_mode() && !gp.empty()) {
+  first_done = all_done;
+  if (!all_done && opt(BLAS3_OPT_TRSM_FIRST_FUSED) && tensor_mode() && !gp.empty()) {
     if (fsplit > 0)
       while (gp.size() >= 2 && gp.back().h >= fsplit && outer.size() < (size_t)MAX_LEVELS) { outer.insert(outer.begin(), gp.back()); gp.pop_back(); }
     const int64_t c_lo = outer.empty() ? -1 : outer[0].f_lo, c_hi = outer.empty() ? -1 : outer[0].f_hi;
@@ -1158,7 +1180,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
     const int64_t mq = left ? m : c1 - c0, nq = left ? c1 - c0 : n;
     int waited = first_done ? nlvl : -1;              // highest first-panel level waited on
                                                       // (the fused launch built them all)
-    bool waited_rest = false;                         // the other panels' inverses waited on
+    bool waited_rest = all_done;                      // the other panels' inverses waited on
 
     // leaf: rows (L) / columns (R) [e0, e0 + cnt) of X, aligned block width wblk
     // kernels of the first panel leave SMs to the latency-bound doubling
@@ -1328,7 +1350,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // the side streams' last levels are part of this call (scratch is freed on s)
   if (!first_done && nlvl > 0 && cudaStreamWaitEvent(s, ts->ev_lvl[nlvl - 1], 0) != cudaSuccess)
     return BLAS3_ERR_CUDA;
-  if (nlvl > 0 && npanel > 1 && cudaStreamWaitEvent(s, ts->ev_lvl2[nlvl - 1], 0) != cudaSuccess)
+  if (nlvl > 0 && npanel > 1 && !all_done && cudaStreamWaitEvent(s, ts->ev_lvl2[nlvl - 1], 0) != cudaSuccess)
     return BLAS3_ERR_CUDA;
   return finish(0);
 }

@@ -40,7 +40,8 @@ def b3():
     return m
 
 
-@pytest.mark.parametrize("split", [0, 512, 1024], ids=["chain", "first_split512", "first_split1024"])
+@pytest.mark.parametrize("split", [0, 512, 1024, "all"], ids=["chain", "first_split512", "first_split1024",
+                                                              "first_all"])
 @pytest.mark.parametrize("side,uplo,ta,diag", V16)
 def test_strsm_multi_panel_multi_slab(b3, oracle_mod, side, uplo, ta, diag, split):
     """split=1: BLAS3_OPT_TRSM_FIRST_SPLIT (first panel's second half by a bulk
@@ -50,7 +51,8 @@ def test_strsm_multi_panel_multi_slab(b3, oracle_mod, side, uplo, ta, diag, spli
     A = gen.triangular_dd(ka, uplo, diag, "sweep-a")
     B = gen.uniform(m, n, "sweep-b")
     dB = to_dev(B)
-    with b3.options(trsm_first_split=split):
+    opts = dict(trsm_first_all=1) if split == "all" else dict(trsm_first_split=split)
+    with b3.options(**opts):
         b3.strsm(side, uplo, ta, diag, AL, to_dev(A), dB)
     X = f64(to_host(dB))
     T = op(tri_full(A, uplo, diag, ka), ta)
