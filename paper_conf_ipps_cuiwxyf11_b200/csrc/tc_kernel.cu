@@ -161,6 +161,8 @@ struct TcParamsT {
   uint32_t *dep_ctr;       // fused: [NPH] phase counters, then [NPH][MAX_SLAB] slab counters
   unsigned long long *trace;   // phase timestamps of CTA 0 (env BLAS3_TRACE), or null
   unsigned long long *ph_trace;  // fused, BLAS3_TRACE=2: per phase [first dep-ready, last done] (ns)
+  unsigned long long *st_trace;  // fused, BLAS3_TRACE_PH=p: per stage [min, max] over phase p's tiles
+  int32_t st_phase;
 };
 using TcParams = TcParamsT<1, MAX_MAPS>;
 constexpr int FUSED_PH = 24, FUSED_MAPS = 48;
@@ -176,6 +178,18 @@ using TcFusedParams = TcParamsT<FUSED_PH, FUSED_MAPS>;
     }                                                                               \
   } while (0)
 
+
+// fused launches, BLAS3_TRACE_PH=p: earliest and latest %globaltimer at which
+// any CTA reached stage i for a tile of phase p (diagnostics)
+#define BLAS3_STRACE(i, ph_)                                                        \
+  do {                                                                              \
+    if (FUSED && prm.st_trace != nullptr && (ph_) == prm.st_phase) {               \
+      unsigned long long t_;                                                        \
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                        \
+      atomicMin(prm.st_trace + 2 * (i), t_);                                        \
+      atomicMax(prm.st_trace + 2 * (i) + 1, t_);                                    \
+    }                                                                               \
+  } while (0)
 
 // byte offset of element (r, k) inside a staged operand tile
 __device__ __forceinline__ uint32_t off_k(int r, int k) {       // K-major, 128 B per row r
@@ -453,7 +467,7 @@ __device__ __forceinline__ void spin_until(const uint32_t *ctr, uint32_t target)
 // makes the producing CTAs' stores visible, and the proxy fence orders them
 // before this CTA's later TMA (async-proxy) reads.
 template <int CG, class PRM>
-__device__ __forceinline__ void wait_deps(const PRM &prm, const Work &w) {
+__device__ __forceinline__ void wait_deps(const PRM &prm, const Work &w, bool async_proxy = true) {
   if constexpr (sizeof(prm.ph) / sizeof(prm.ph[0]) > 1) {
     const PhaseDesc &ph = prm.ph[w.ph];
     if ((ph.dep_full | ph.dep_slab) == 0) return;
@@ -463,7 +477,15 @@ __device__ __forceinline__ void wait_deps(const PRM &prm, const Work &w) {
       if (ph.dep_slab >> q & 1)
         spin_until(prm.dep_ctr + FUSED_PH + q * MAX_SLAB + slab, (uint32_t)(prm.ph[q].slab_cnt * CG));
     }
-    asm volatile("fence.proxy.async.global;" ::: "memory");
+    if (prm.st_trace != nullptr && w.ph == prm.st_phase && async_proxy) {
+      unsigned long long t_;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));
+      atomicMin(prm.st_trace + 2 * 10, t_);
+      atomicMax(prm.st_trace + 2 * 10 + 1, t_);
+    }
+    // the producer's TMA (async proxy) reads what other CTAs stored through
+    // the generic proxy; the epilogue's plain loads need only the acquire
+    if (async_proxy) asm volatile("fence.proxy.async.global;" ::: "memory");
   }
 }
 // After this CTA's stores of a tile (one thread, after the epilogue barrier).
@@ -621,6 +643,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
         const int64_t m0 = w.m0, n0 = w.n0;
         const int64_t ma = m0 + HA * rank, nb = n0 + HB * rank;
         wait_deps<CG>(prm, w);                        // fused launches: producing tiles done
+        BLAS3_STRACE(0, w.ph);
         if (FUSED && prm.ph_trace != nullptr) {
           unsigned long long t_;
           asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));
@@ -644,6 +667,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
             load_operand(prm, sg.a, si.layA, raw[rs].A, ma, k0, HA, &bars->full[rs], bj, bg);
             load_operand(prm, sg.b, si.layB, raw[rs].B, nb, k0, HB, &bars->full[rs], bj, bg);
             BLAS3_TRACE(3);
+            if (kb == kb0) BLAS3_STRACE(1, w.ph);
           }
         }
       }
@@ -704,6 +728,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
             if (CG == 2) ptx::mbar_wait_cluster(&bars->ready[ls], lph);
             else ptx::mbar_wait(&bars->ready[ls], lph);
             ptx::tc_fence_after();
+            if (lane == 0 && kb == kb0) BLAS3_STRACE(4, w.ph);
             if (lane == 0) {
               const uint32_t hiA = ptx::smem_u32(raw[rs].A), hiB = ptx::smem_u32(raw[rs].B);
               const uint32_t loA = ptx::smem_u32(lo[ls].A), loB = ptx::smem_u32(lo[ls].B);
@@ -737,6 +762,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
             accumulate = 1;
             __syncwarp();
             ++done;
+            if (lane == 0 && done == nkb) BLAS3_STRACE(5, w.ph);
             if (done % KC == 0 || done == nkb) close_chunk(true);
           }
         }
@@ -768,6 +794,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           const StageInfo si = stage_at<CG>(bd, P, sg, m0, n0, kb);
           ptx::mbar_wait(&bars->full[rs], ph);
           if (tt == 0) BLAS3_TRACE(4);
+          if (tt == 0 && kb == kb0) BLAS3_STRACE(2, w.ph);
           RawBuf &rb = raw[rs];
           bool fix = false;
           // fix-ups are decided on this CTA's own half: a half that is entirely
@@ -795,6 +822,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           ptx::fence_proxy_async_smem();
           arrive_leader<CG>(&bars->ready[ls], rank, 2, TR_THREADS, tt == 0);
           if (tt == 0) BLAS3_TRACE(5);
+          if (tt == 0 && kb == kb0) BLAS3_STRACE(3, w.ph);
         }
       }
     }
@@ -825,6 +853,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
         ptx::mbar_wait(&bars->tfull[buf], ph);
         ptx::tc_fence_after();
         if (threadIdx.x == WARP_EPI0 * 32) BLAS3_TRACE(7);
+        if (threadIdx.x == WARP_EPI0 * 32 && c == nchunks - 1) BLAS3_STRACE(6, w.ph);
         if (nkb > 0) {
 #pragma unroll
           for (int g = 0; g < NG; ++g) {
@@ -873,8 +902,10 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
       if (FUSED) {
         // C may have been written by earlier phases on other SMs: one acquire
         // (which also invalidates this SM's L1) before any thread loads it
-        if (threadIdx.x == WARP_EPI0 * 32) wait_deps<CG>(prm, w);
+        if (threadIdx.x == WARP_EPI0 * 32) BLAS3_STRACE(11, w.ph);
+        if (threadIdx.x == WARP_EPI0 * 32) wait_deps<CG>(prm, w, false);
         ptx::named_bar_sync(5, EPI_THREADS);
+        if (threadIdx.x == WARP_EPI0 * 32) BLAS3_STRACE(7, w.ph);
       }
       // ---- store phase: D = alpha*S + beta*C for row r, columns cbase + [0,128).
       // The valid columns of the row form one range [jlo, jhi) (column bound
@@ -943,7 +974,9 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
       if (FUSED) {                                 // this CTA's half of the tile is stored
         ptx::named_bar_sync(5, EPI_THREADS);
         if (threadIdx.x == WARP_EPI0 * 32) {
+          BLAS3_STRACE(8, w.ph);
           signal_done<CG>(prm, w);
+          BLAS3_STRACE(9, w.ph);
           if (prm.ph_trace != nullptr) {
             unsigned long long t_;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));
@@ -1314,6 +1347,20 @@ int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int 
     cudaStreamSynchronize(stream);
     prm.ph_trace = tbuf;
   }
+  // BLAS3_TRACE_PH=p: per-stage [earliest, latest] over the tiles of phase p
+  static int st_phase = -2;
+  static unsigned long long *sbuf = nullptr;
+  constexpr int NST = 12;
+  if (st_phase == -2) { const char *e = getenv("BLAS3_TRACE_PH"); st_phase = e ? atoi(e) : -1; }
+  if (st_phase >= 0 && st_phase < nph) {
+    if (!sbuf && cudaMalloc(&sbuf, 2 * NST * sizeof(unsigned long long)) != cudaSuccess) return -1;
+    unsigned long long init[2 * NST];
+    for (int i = 0; i < NST; ++i) { init[2 * i] = ~0ull; init[2 * i + 1] = 0ull; }
+    cudaMemcpyAsync(sbuf, init, sizeof(init), cudaMemcpyHostToDevice, stream);
+    cudaStreamSynchronize(stream);
+    prm.st_trace = sbuf;
+    prm.st_phase = st_phase;
+  }
   // no PDL: the counters' memset node precedes this grid on the stream
   const int rc = launch_cg<CG>(prm, stream, num_sms, false);
   if (trace && rc == 0) {
@@ -1326,6 +1373,19 @@ int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int 
       fprintf(stderr, "[blas3 fused] phase %2d M=%6lld N=%6lld K=%6lld tiles=%5lld: %8.1f .. %8.1f us\n", p,
               (long long)prm.ph[p].P.M, (long long)prm.ph[p].P.N, (long long)prm.ph[p].P.seg[0].K,
               (long long)prm.ph[p].ntiles, (h[2 * p] - t0) / 1e3, (h[2 * p + 1] - t0) / 1e3);
+  }
+  if (prm.st_trace && rc == 0) {
+    static const char *names[NST] = {"deps_ready", "tma_issued", "raw_full", "split_done", "mma_start",
+                                     "mma_last_issued", "tmem_full", "epi_deps", "stored", "signaled",
+                                     "prod_acquired", "tmem_drained"};
+    unsigned long long h[2 * NST];
+    cudaStreamSynchronize(stream);
+    cudaMemcpy(h, sbuf, sizeof(h), cudaMemcpyDeviceToHost);
+    const unsigned long long t0 = h[0];
+    fprintf(stderr, "[blas3 stages] phase %d (%lld tiles):", st_phase, (long long)prm.ph[st_phase].ntiles);
+    for (int i = 0; i < NST; ++i)
+      if (h[2 * i + 1]) fprintf(stderr, " %s=%.2f/%.2f", names[i], (h[2 * i] - t0) / 1e3, (h[2 * i + 1] - t0) / 1e3);
+    fprintf(stderr, " us (earliest/latest tile)\n");
   }
   return rc;
 }
