@@ -45,7 +45,10 @@ def uniform(m: int, n: int, *tags, ld: int | None = None, lo=-1.0, hi=1.0) -> np
     """U(lo, hi) fp32, column-major.  Returns the (ld x n) buffer; rows >= m are NaN."""
     buf = _fortran(m, n, ld)
     g = rng("uniform", m, n, *tags)
-    buf[:m, :] = (g.random((n, m), dtype=np.float32) * np.float32(hi - lo) + np.float32(lo)).T
+    Y = g.random((n, m), dtype=np.float32)
+    Y *= np.float32(hi - lo)                # in place: the same fp32 ops, no 2nd temporary
+    Y += np.float32(lo)
+    buf[:m, :] = Y.T
     return buf
 
 
@@ -61,12 +64,13 @@ def nan_outside(X: np.ndarray, uplo: str, keep_diag: bool = True) -> np.ndarray:
     """Fill the strict triangle NOT named by uplo (and optionally the
     diagonal) of the leading square block with NaN sentinels, in place."""
     n = min(X.shape[0], X.shape[1])
-    i, j = np.indices((n, n))
-    blank = (i < j) if uplo.upper() == "L" else (i > j)
-    if not keep_diag:
-        blank |= i == j
-    sub = X[:n, :n]
-    sub[blank] = np.nan
+    lower = uplo.upper() == "L"
+    d = 0 if keep_diag else 1
+    for j in range(n):                      # column by column: no n x n index temporaries
+        if lower:
+            X[:j + d, j] = np.nan           # rows above the diagonal (and it, if not kept)
+        else:
+            X[j + 1 - d:n, j] = np.nan      # rows below the diagonal (and it, if not kept)
     return X
 
 
@@ -82,14 +86,26 @@ def triangular_dd(n: int, uplo: str, diag: str, *tags, ld: int | None = None) ->
     X = uniform(n, n, "tri", uplo, diag, *tags, ld=ld)
     sub = X[:n, :n]
     lower = uplo.upper() == "L"
-    tri = np.tril(sub, -1) if lower else np.triu(sub, 1)
+    # strict triangle kept, the rest (diagonal included) set below; the
+    # absolute row / column sums of the strict triangle are accumulated in
+    # fp64 over column chunks (no n x n fp64 temporaries at large n)
+    ch = 1024
+    colsum = np.zeros(n)
+    rowsum = np.zeros(n)
+    for c0 in range(0, n, ch):
+        blk = sub[:, c0:c0 + ch]
+        strict = np.tril(blk, -1 - c0) if lower else np.triu(blk, 1 - c0)
+        if diag.upper() == "U":
+            blk[:, :] = strict / np.float32(max(n, 1))
+        else:
+            a = np.abs(strict.astype(np.float64))
+            colsum[c0:c0 + ch] = a.sum(axis=0)
+            rowsum += a.sum(axis=1)
+            blk[:, :] = strict
     if diag.upper() == "U":
-        sub[:, :] = tri / np.float32(max(n, 1))
         nan_outside(X, uplo, keep_diag=False)
     else:
-        a = np.abs(tri.astype(np.float64))
-        dom = 1.0 + np.maximum(a.sum(axis=0), a.sum(axis=1))
-        sub[:, :] = tri
+        dom = 1.0 + np.maximum(colsum, rowsum)
         np.fill_diagonal(sub, dom.astype(np.float32))
         nan_outside(X, uplo, keep_diag=True)
     return X
