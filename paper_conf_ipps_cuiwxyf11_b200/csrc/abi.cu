@@ -46,6 +46,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TRSM_FIRST_FUSED", 1, 0, 1, false},
     {"BLAS3_TRSM_FIRST_SPLIT", 0, 0, 8192, true},
     {"BLAS3_TRSM_FIRST_ALL", 0, 0, 1, false},
+    {"BLAS3_TC_RASTER", 0, 0, 64, false},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;
@@ -162,6 +163,7 @@ static Problem problem(int64_t M, int64_t N, float alpha, float beta, const floa
   P.M = M; P.N = N; P.nseg = 1; P.alpha = alpha; P.beta = beta;
   P.Cin = Cin; P.ldcin = ldcin; P.Cout = Cout; P.ldcout = ldcout;
   P.nbatch = 1; P.per = 1;
+  P.raster_gm = (int32_t)opt(BLAS3_OPT_TC_RASTER);
   return P;
 }
 

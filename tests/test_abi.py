@@ -181,4 +181,4 @@ def test_options_roundtrip_and_validation(lib):
     assert lib.blas3_set_option(lib.OPTIONS["tc_cta"], 3) == 1
     assert lib.blas3_set_option(99, 0) == 1
     assert lib.blas3_get_option(99) == -(2 ** 63)
-    assert len(lib.OPTIONS) == 19
+    assert len(lib.OPTIONS) == 20
