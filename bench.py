@@ -524,7 +524,9 @@ def run_reference(args):
         "data": "synthetic (seeded U(-1,1); diagonally dominant T)",
         "config": {"workload": "configs[1..3] at N=8192: sgemm NN, ssymm LL, ssyrk LN, ssyr2k LN "
                                "(K=8192), strmm LLNN, strsm LLNN; alpha=1.5 beta=0.5",
-                   "n": N, "k": N},
+                   "n": N, "k": N, "cols_per_rank": N, "math": "fp64 oracle (plain C)",
+                   "l2": "n/a (host CPU)",
+                   "parallelism": f"host CPU, {oracle.num_threads()} OpenMP threads over output columns"},
         "cpu_baseline": {"value": round(value, 3), "unit": "GFLOPS", "cores": oracle.num_threads(),
                          "kind": "oracle",
                          "sample": f"{ns} sampled output columns of each routine per step"},
