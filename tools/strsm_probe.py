@@ -49,7 +49,7 @@ flop = float(n) ** 3
 _, tg = tune.search(gemm_only, [{}], reps=3, rounds=3)
 g_ms = tg[0][1]
 for name, fn, base in (("isolated", iso, 0.0), ("after_gemm", after_gemm, g_ms)):
-    _, table = tune.search(fn, cands, reps=3, rounds=3)
+    _, table = tune.search(fn, cands, reps=3, rounds=int(os.environ.get("PROBE_ROUNDS", "3")))
     for c, ms in table:
         t = ms - base
         print(json.dumps({"mode": name, "opts": c, "ms": round(t, 4), "tflops": round(flop / t / 1e9, 1)}))
