@@ -216,7 +216,11 @@ int64_t blas3_get_option(int key);
 
 /* Optional caller-owned device scratch used before falling back to
  * cudaMallocAsync.  The buffer must stay valid while calls that may use it
- * are in flight.  (ptr=NULL, bytes=0 removes it.)  Returns 0. */
+ * are in flight, and it is process-wide: calls that use it must not run
+ * concurrently on different streams (as with one cuBLAS workspace); without
+ * it every call takes its own stream-ordered scratch, and calls on different
+ * streams / host threads are independent.  (ptr=NULL, bytes=0 removes it.)
+ * Returns 0. */
 int blas3_set_workspace(void *dptr, size_t bytes);
 
 /* Number of kernels the library launched since load (host-side counter;

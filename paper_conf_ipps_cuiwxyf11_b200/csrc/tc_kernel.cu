@@ -30,6 +30,7 @@
 //                (two warps per TMEM lane quarter, 128 columns each)
 #include <cuda.h>
 #include <cuda_runtime.h>
+#include <atomic>
 #include <mutex>
 #include <cstdio>
 #include <stdlib.h>
@@ -1141,9 +1142,11 @@ struct TileCounter { uint32_t *ctr; };
 static bool tile_counter(TileCounter &tc) {
   constexpr int SLOTS = 256;
   static uint32_t *ring[64] = {};
-  static uint32_t next[64] = {};
+  static std::atomic<uint32_t> next[64];      // regular and fused launches hold different locks
+  static std::mutex alloc_mu;
   int d = 0;
   if (cudaGetDevice(&d) != cudaSuccess || d < 0 || d >= 64) return false;
+  std::lock_guard<std::mutex> lk(alloc_mu);
   if (!ring[d]) {
     if (cudaMalloc(&ring[d], SLOTS * 32 * sizeof(uint32_t)) != cudaSuccess ||
         cudaMemset(ring[d], 0, SLOTS * 32 * sizeof(uint32_t)) != cudaSuccess) {
@@ -1152,7 +1155,7 @@ static bool tile_counter(TileCounter &tc) {
       return false;
     }
   }
-  const uint32_t slot = next[d]++ % SLOTS;
+  const uint32_t slot = next[d].fetch_add(1u) % SLOTS;
   tc.ctr = ring[d] + slot * 32;                     // 128-B apart
   return true;
 }
