@@ -48,6 +48,10 @@
  *  Math       BLAS3_MATH_3XTF32 (default): tcgen05 tensor cores with a
  *             3xTF32 split (hi*hi + hi*lo + lo*hi) and fp32 accumulation in
  *             TMEM.  BLAS3_MATH_SIMT_FP32: exact-fp32 FFMA kernels.
+ *             BLAS3_MATH_TF32_BF16X: opt-in: hi*hi as one TF32 UMMA and
+ *             the two cross terms lo*hi + hi*lo packed into ONE BF16 UMMA (K = 16,
+ *             hi and lo rounded to bf16): 2 UMMAs per k-step instead of 3,
+ *             output-relative error ~1e-6 above the 3XTF32 split (DESIGN Q28).
  *             BLAS3_MATH_1XTF32: opt-in fast mode, one TF32 pass
  *             (inputs truncated to TF32, 10-bit mantissa; normwise error
  *             ~1e-3, NOT the fp32 accuracy of the other two modes).
@@ -75,7 +79,7 @@ enum {
     BLAS3_ERR_TMA = -4
 };
 
-enum { BLAS3_MATH_3XTF32 = 0, BLAS3_MATH_SIMT_FP32 = 1, BLAS3_MATH_1XTF32 = 2 };
+enum { BLAS3_MATH_3XTF32 = 0, BLAS3_MATH_SIMT_FP32 = 1, BLAS3_MATH_1XTF32 = 2, BLAS3_MATH_TF32_BF16X = 3 };
 
 /* SGEMM: C <- alpha*op(A)*op(B) + beta*C, op(X) = X or X^T.
  * op(A) is m x k, op(B) is k x n, C is m x n.  Paper: GEMM-NN/-TN loop nests
@@ -138,7 +142,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
                 blas3_stream_t stream);
 
 /* Process-wide math mode (BLAS3_MATH_3XTF32 default; the environment
- * variable BLAS3_MATH=simt|3xtf32|1xtf32 overrides the default at load).
+ * variable BLAS3_MATH=simt|3xtf32|1xtf32|bf16x overrides the default at load).
  * Returns 0, or 1 if `mode` is not a valid mode (nothing changed). */
 int blas3_set_math_mode(int mode);
 int blas3_get_math_mode(void);

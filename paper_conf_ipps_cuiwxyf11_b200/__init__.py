@@ -58,7 +58,7 @@ for _name, _args in _SIGS.items():
     globals()[_name] = _fn
 
 EXPORTED = tuple(_SIGS)
-MATH_3XTF32, MATH_SIMT_FP32, MATH_1XTF32 = 0, 1, 2
+MATH_3XTF32, MATH_SIMT_FP32, MATH_1XTF32, MATH_TF32_BF16X = 0, 1, 2, 3
 
 
 class Blas3Error(RuntimeError):
@@ -174,7 +174,8 @@ def strsm(side, uplo, transa, diag, alpha, A, B):
 
 def set_math_mode(mode):
     if isinstance(mode, str):
-        mode = {"3xtf32": MATH_3XTF32, "simt": MATH_SIMT_FP32, "1xtf32": MATH_1XTF32}[mode.lower()]
+        mode = {"3xtf32": MATH_3XTF32, "simt": MATH_SIMT_FP32, "1xtf32": MATH_1XTF32,
+                "tf32_bf16x": MATH_TF32_BF16X}[mode.lower()]
     _chk("blas3_set_math_mode", blas3_set_math_mode(mode))  # noqa: F821
 
 

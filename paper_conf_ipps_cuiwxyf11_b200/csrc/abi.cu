@@ -82,7 +82,8 @@ static int math_mode() {
   if (g_math < 0) {
     const char *e = getenv("BLAS3_MATH");
     g_math = (e && (e[0] == 's' || e[0] == 'S')) ? BLAS3_MATH_SIMT_FP32
-             : (e && e[0] == '1') ? BLAS3_MATH_1XTF32 : BLAS3_MATH_3XTF32;
+             : (e && e[0] == '1') ? BLAS3_MATH_1XTF32
+             : (e && (e[0] == 'b' || e[0] == 'B')) ? BLAS3_MATH_TF32_BF16X : BLAS3_MATH_3XTF32;
   }
   return g_math;
 }
@@ -134,7 +135,7 @@ static int run_problem(const Problem &P, cudaStream_t s, int sms) {
   if (P.max_sms > 0 && P.max_sms < sms) sms = P.max_sms;
   if (tensor_mode() && tc_eligible(P)) {
     Problem Q = P;
-    Q.passes = math_mode() == BLAS3_MATH_1XTF32 ? 1 : 3;
+    Q.passes = math_mode() == BLAS3_MATH_1XTF32 ? 1 : math_mode() == BLAS3_MATH_TF32_BF16X ? 2 : 3;
     return launch_tc(Q, s, sms);
   }
   int rc = launch_simt(P, s, sms);
@@ -229,7 +230,8 @@ int64_t blas3_get_option(int key) {
 }
 
 int blas3_set_math_mode(int mode) {
-  if (mode != BLAS3_MATH_3XTF32 && mode != BLAS3_MATH_SIMT_FP32 && mode != BLAS3_MATH_1XTF32) return 1;
+  if (mode != BLAS3_MATH_3XTF32 && mode != BLAS3_MATH_SIMT_FP32 && mode != BLAS3_MATH_1XTF32 &&
+      mode != BLAS3_MATH_TF32_BF16X) return 1;
   g_math = mode;
   return 0;
 }

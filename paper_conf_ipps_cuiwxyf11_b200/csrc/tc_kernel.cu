@@ -39,6 +39,7 @@
 #include "../../include/blas3.h"
 #include "kernels.h"
 #include "tc_ptx.h"
+#include <cuda_bf16.h>
 
 namespace blas3 {
 
@@ -419,6 +420,45 @@ __device__ __forceinline__ float split_lo(float x) {
   return x - hi;
 }
 
+// BLAS3_MATH_TF32_BF16X: the two cross terms of the split packed into ONE bf16
+// operand pair per k8 step.  For a staged tile (raw, either layout) with
+// x = hi + lo (hi = trunc_tf32(x)), the K-major bf16 tile `dst` holds, per
+// row and k8 chunk c, two 16-B chunks: A side [lo(8c..8c+7) | hi(8c..8c+7)],
+// B side [hi | lo], so one K = 16 bf16 UMMA sums lo_A*hi_B + hi_A*lo_B.
+// 128-B rows, SWIZZLE_128B (16-B chunk j of row r at (j ^ (r & 7)) << 4).
+__device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
+  const __nv_bfloat162 v = __floats2bfloat162_rn(a, b);     // a -> low half (lower address)
+  return *reinterpret_cast<const uint32_t *>(&v);
+}
+__device__ __forceinline__ void pack_cross(const uint8_t *raw, int lay, uint8_t *dst, int rows, int t,
+                                           bool a_side) {
+  for (int u = t; u < rows * 4; u += TR_THREADS) {
+    const int r = u % rows, c = u / rows;
+    float x[8];
+    if (lay == LAYOUT_K) {
+      const float4 v0 = *reinterpret_cast<const float4 *>(raw + off_k(r, 8 * c));
+      const float4 v1 = *reinterpret_cast<const float4 *>(raw + off_k(r, 8 * c + 4));
+      x[0] = v0.x; x[1] = v0.y; x[2] = v0.z; x[3] = v0.w;
+      x[4] = v1.x; x[5] = v1.y; x[6] = v1.z; x[7] = v1.w;
+    } else {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) x[i] = *reinterpret_cast<const float *>(raw + off_mn(r, 8 * c + i));
+    }
+    uint4 hi, lo;
+    uint32_t *hp = &hi.x, *lp = &lo.x;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float h0 = __uint_as_float(__float_as_uint(x[2 * i]) & 0xFFFFE000u);
+      const float h1 = __uint_as_float(__float_as_uint(x[2 * i + 1]) & 0xFFFFE000u);
+      hp[i] = pack_bf16x2(h0, h1);
+      lp[i] = pack_bf16x2(x[2 * i] - h0, x[2 * i + 1] - h1);
+    }
+    uint8_t *row = dst + r * 128;
+    *reinterpret_cast<uint4 *>(row + (((2 * c) ^ (r & 7)) << 4)) = a_side ? lo : hi;
+    *reinterpret_cast<uint4 *>(row + (((2 * c + 1) ^ (r & 7)) << 4)) = a_side ? hi : lo;
+  }
+}
+
 __device__ __forceinline__ void split_pass(const uint8_t *raw, uint8_t *lo, uint32_t bytes, int t) {
   const float4 *r4 = reinterpret_cast<const float4 *>(raw);
   float4 *l4 = reinterpret_cast<float4 *>(lo);
@@ -740,6 +780,21 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
                 const uint64_t bh = op_desc(hiB, si.layB, k8), bl = op_desc(loB, si.layB, k8);
                 const bool one = (P.dbg & 2) || P.passes == 1;
                 if (P.dbg & 8) continue;                       // diag: no MMAs
+                if (P.passes == 2) {
+                  // packed cross terms (one bf16 UMMA, K = 16, K-major) + hi*hi (tf32)
+                  const uint64_t ax = ptx::smem_desc(loA + k8 * 32, 16, 1024, 2);
+                  const uint64_t bx = ptx::smem_desc(loB + k8 * 32, 16, 1024, 2);
+                  constexpr uint32_t idx = ptx::idesc_bf16(TM, BN, 0, 0);
+                  if constexpr (CG == 1) {
+                    ptx::mma_bf16_ss(d_tmem, ax, bx, idx, accumulate);
+                    ptx::mma_tf32_ss(d_tmem, ah, bh, idesc, 1);
+                  } else {
+                    ptx::mma_bf16_ss_pair(d_tmem, ax, bx, idx, accumulate);
+                    ptx::mma_tf32_ss_pair(d_tmem, ah, bh, idesc, 1);
+                  }
+                  accumulate = 1;
+                  continue;
+                }
                 if constexpr (CG == 1) {
                   if (!one) ptx::mma_tf32_ss(d_tmem, al, bh, idesc, accumulate);
                   if (!one) ptx::mma_tf32_ss(d_tmem, ah, bl, idesc, 1);
@@ -816,7 +871,10 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           }
           if (fix) ptx::named_bar_sync(1, TR_THREADS);
           ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
-          if (!(P.dbg & 1) && P.passes != 1) {
+          if (P.passes == 2) {                              // packed bf16 cross terms
+            pack_cross(rb.A, si.layA, lo[ls].A, HA, tt, true);
+            pack_cross(rb.B, si.layB, lo[ls].B, HB, tt, false);
+          } else if (!(P.dbg & 1) && P.passes != 1) {
             split_pass(rb.A, lo[ls].A, G::A_BYTES, tt);
             split_pass(rb.B, lo[ls].B, G::B_BYTES, tt);
           }

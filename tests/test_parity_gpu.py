@@ -7,7 +7,8 @@ diagonally dominant A.  Because 1xTF32 would also pass those at N >= 1024
 <= 5e-6 and STRSM's forward error <= 1e-5.
 Integer-valued inputs must reproduce the oracle bit for bit (one correct
 answer, Q18).  Sizes span several tiles and ragged tails.
-Both math modes (3xTF32 tcgen05 and FP32 SIMT) are exercised.
+All three fp32-accurate math modes (3xTF32 and TF32+BF16X on tcgen05, FP32
+SIMT) are exercised.
 """
 import itertools
 
@@ -20,7 +21,7 @@ from check import (TOL_NW, bits_equal, e_nw, e_rel, f64, fro, op, sym_full, to_d
 
 pytestmark = pytest.mark.gpu
 
-MODES = ["3xtf32", "simt"]
+MODES = ["3xtf32", "simt", "tf32_bf16x"]
 AL, BE = 1.5, 0.5
 
 
@@ -51,7 +52,7 @@ def route(b3, mode):
 
     def check(*lds):
         tc = b3.launch_count("tc") > before["tc"]
-        if mode == "3xtf32" and all(ld % 4 == 0 for ld in lds):
+        if mode != "simt" and all(ld % 4 == 0 for ld in lds):
             assert tc, "expected the tcgen05 route"
         else:
             assert not tc, "tcgen05 route taken unexpectedly"

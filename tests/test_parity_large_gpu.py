@@ -122,3 +122,20 @@ def test_strsm_8192(env, ta):
     assert resid <= 1e-5 * np.sqrt(N)
     ref = oracle.strsm("L", "L", ta, "N", AL, T, B, sel=sel)
     assert fro(X - ref) / fro(ref) <= 1e-5
+
+
+@pytest.mark.parametrize("ta,tb", [("N", "N"), ("T", "N")])
+def test_sgemm_8192_tf32_bf16x(env, ta, tb):
+    """The opt-in TF32+BF16X mode (packed bf16 cross terms) at the bench size."""
+    b3, oracle, A, T, B, C, sel, d = env
+    b3.set_math_mode("tf32_bf16x")
+    try:
+        dC = to_dev(C)
+        b3.sgemm(ta, tb, AL, d["A"], d["B"], BE, dC)
+        got = to_host(dC)[:, sel]
+    finally:
+        b3.set_math_mode("3xtf32")
+    ref = oracle.sgemm(ta, tb, AL, A, B, BE, C, sel=sel)
+    scale = AL * fro(A) * fro(B[:, sel]) + BE * fro(C[:, sel])
+    assert e_nw(got, ref, scale) <= TOL_NW
+    assert fro(f64(got) - ref) / fro(ref) <= tol_rel(N, "tf32_bf16x")
