@@ -552,7 +552,9 @@ __device__ __forceinline__ void arrive_leader(uint64_t *bar, uint32_t rank, uint
 
 }  // namespace
 
-template <int CG, class PRM>
+// BX: the BLAS3_MATH_TF32_BF16X instantiation (packed bf16 cross terms); a
+// compile-time switch so the default 3xTF32 kernel carries none of its code.
+template <int CG, class PRM, bool BX = false>
 __global__ void __launch_bounds__(NTHREADS, 1)
 tc_structured_gemm(const __grid_constant__ PRM prm) {
   constexpr bool FUSED = sizeof(prm.ph) / sizeof(prm.ph[0]) > 1;
@@ -780,7 +782,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
                 const uint64_t bh = op_desc(hiB, si.layB, k8), bl = op_desc(loB, si.layB, k8);
                 const bool one = (P.dbg & 2) || P.passes == 1;
                 if (P.dbg & 8) continue;                       // diag: no MMAs
-                if (P.passes == 2) {
+                if constexpr (BX) {
                   // packed cross terms (one bf16 UMMA, K = 16, K-major) + hi*hi (tf32)
                   const uint64_t ax = ptx::smem_desc(loA + k8 * 32, 16, 1024, 2);
                   const uint64_t bx = ptx::smem_desc(loB + k8 * 32, 16, 1024, 2);
@@ -871,7 +873,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           }
           if (fix) ptx::named_bar_sync(1, TR_THREADS);
           ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
-          if (P.passes == 2) {                              // packed bf16 cross terms
+          if constexpr (BX) {                               // packed bf16 cross terms
             pack_cross(rb.A, si.layA, lo[ls].A, HA, tt, true);
             pack_cross(rb.B, si.layB, lo[ls].B, HB, tt, false);
           } else if (!(P.dbg & 1) && P.passes != 1) {
@@ -1159,11 +1161,17 @@ static int launch_cg(PRM &prm, cudaStream_t stream, int num_sms, bool allow_pdl 
       if (!op_maps(prm, slot, sg.b, P.N, sg.K, G::HB, per, groups, P.bs_b)) return -4;
     }
   }
-  static bool attr = false;
-  if (!attr) {
-    if (cudaFuncSetAttribute(tc_structured_gemm<CG, PRM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)G::SMEM) != cudaSuccess) return -1;
-    attr = true;
+  // the TF32+BF16X instantiation for single-phase launches in that mode
+  constexpr bool SINGLE = sizeof(prm.ph) / sizeof(prm.ph[0]) == 1;
+  const bool bx = SINGLE && prm.ph[0].P.passes == 2;
+  void (*kfn)(PRM) = tc_structured_gemm<CG, PRM, false>;
+  if constexpr (SINGLE)
+    if (bx) kfn = tc_structured_gemm<CG, PRM, true>;
+  static bool attr[2] = {false, false};
+  if (!attr[bx]) {
+    if (cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)G::SMEM) != cudaSuccess)
+      return -1;
+    attr[bx] = true;
   }
   const int64_t items = prm.nitems;        // tiles, or tiles + split-tail slices
   if (items == 0) return 0;
@@ -1186,7 +1194,7 @@ static int launch_cg(PRM &prm, cudaStream_t stream, int num_sms, bool allow_pdl 
   attrs[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attrs;
   cfg.numAttrs = pdl ? 2 : 1;
-  const cudaError_t e = cudaLaunchKernelEx(&cfg, tc_structured_gemm<CG, PRM>, prm);
+  const cudaError_t e = cudaLaunchKernelEx(&cfg, kfn, prm);
   note_launch(0);
   return (e == cudaSuccess && cudaGetLastError() == cudaSuccess) ? 0 : -1;
 }
