@@ -430,32 +430,43 @@ __device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
   const __nv_bfloat162 v = __floats2bfloat162_rn(a, b);     // a -> low half (lower address)
   return *reinterpret_cast<const uint32_t *>(&v);
 }
+__device__ __forceinline__ void pack8(const float (&x)[8], uint8_t *row, int r, int c, bool a_side) {
+  uint4 hi, lo;
+  uint32_t *hp = &hi.x, *lp = &lo.x;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const float h0 = __uint_as_float(__float_as_uint(x[2 * i]) & 0xFFFFE000u);
+    const float h1 = __uint_as_float(__float_as_uint(x[2 * i + 1]) & 0xFFFFE000u);
+    hp[i] = pack_bf16x2(h0, h1);
+    lp[i] = pack_bf16x2(x[2 * i] - h0, x[2 * i + 1] - h1);
+  }
+  *reinterpret_cast<uint4 *>(row + (((2 * c) ^ (r & 7)) << 4)) = a_side ? lo : hi;
+  *reinterpret_cast<uint4 *>(row + (((2 * c + 1) ^ (r & 7)) << 4)) = a_side ? hi : lo;
+}
+__device__ __forceinline__ void load8(const uint8_t *raw, int lay, int r, int c, float (&x)[8]) {
+  if (lay == LAYOUT_K) {            // a row's 8 k-values: two swizzled 16-B chunks
+    const float4 v0 = *reinterpret_cast<const float4 *>(raw + off_k(r, 8 * c));
+    const float4 v1 = *reinterpret_cast<const float4 *>(raw + off_k(r, 8 * c + 4));
+    x[0] = v0.x; x[1] = v0.y; x[2] = v0.z; x[3] = v0.w;
+    x[4] = v1.x; x[5] = v1.y; x[6] = v1.z; x[7] = v1.w;
+  } else {                          // MN-major: a warp's rows are contiguous per k
+#pragma unroll
+    for (int i = 0; i < 8; ++i) x[i] = *reinterpret_cast<const float *>(raw + off_mn(r, 8 * c + i));
+  }
+}
 __device__ __forceinline__ void pack_cross(const uint8_t *raw, int lay, uint8_t *dst, int rows, int t,
                                            bool a_side) {
-  for (int u = t; u < rows * 4; u += TR_THREADS) {
-    const int r = u % rows, c = u / rows;
-    float x[8];
-    if (lay == LAYOUT_K) {
-      const float4 v0 = *reinterpret_cast<const float4 *>(raw + off_k(r, 8 * c));
-      const float4 v1 = *reinterpret_cast<const float4 *>(raw + off_k(r, 8 * c + 4));
-      x[0] = v0.x; x[1] = v0.y; x[2] = v0.z; x[3] = v0.w;
-      x[4] = v1.x; x[5] = v1.y; x[6] = v1.z; x[7] = v1.w;
-    } else {
-#pragma unroll
-      for (int i = 0; i < 8; ++i) x[i] = *reinterpret_cast<const float *>(raw + off_mn(r, 8 * c + i));
-    }
-    uint4 hi, lo;
-    uint32_t *hp = &hi.x, *lp = &lo.x;
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const float h0 = __uint_as_float(__float_as_uint(x[2 * i]) & 0xFFFFE000u);
-      const float h1 = __uint_as_float(__float_as_uint(x[2 * i + 1]) & 0xFFFFE000u);
-      hp[i] = pack_bf16x2(h0, h1);
-      lp[i] = pack_bf16x2(x[2 * i] - h0, x[2 * i + 1] - h1);
-    }
-    uint8_t *row = dst + r * 128;
-    *reinterpret_cast<uint4 *>(row + (((2 * c) ^ (r & 7)) << 4)) = a_side ? lo : hi;
-    *reinterpret_cast<uint4 *>(row + (((2 * c + 1) ^ (r & 7)) << 4)) = a_side ? hi : lo;
+  // units (row r, k8 chunk c); two per thread at a time, loads issued first (ILP)
+  const int units = rows * 4;
+  for (int u = t; u < units; u += 2 * TR_THREADS) {
+    const int u2 = u + TR_THREADS;
+    const int r0 = u % rows, c0 = u / rows;
+    const int r1 = u2 % rows, c1 = u2 / rows;
+    float x0[8], x1[8];
+    load8(raw, lay, r0, c0, x0);
+    if (u2 < units) load8(raw, lay, r1, c1, x1);
+    pack8(x0, dst + r0 * 128, r0, c0, a_side);
+    if (u2 < units) pack8(x1, dst + r1 * 128, r1, c1, a_side);
   }
 }
 
