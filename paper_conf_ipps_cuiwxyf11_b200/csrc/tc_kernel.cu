@@ -885,8 +885,23 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           if (fix) ptx::named_bar_sync(1, TR_THREADS);
           ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
           if constexpr (BX) {                               // packed bf16 cross terms
-            pack_cross(rb.A, si.layA, lo[ls].A, HA, tt, true);
-            pack_cross(rb.B, si.layB, lo[ls].B, HB, tt, false);
+            if (HA == HB && !(P.dbg & 4096)) {
+              // pair tiles: A and B have 128 rows = 2 units per thread each --
+              // all four units' loads first, then the packing (ILP)
+              const int ua = tt, ub = tt + TR_THREADS;
+              float xa0[8], xa1[8], xb0[8], xb1[8];
+              load8(rb.A, si.layA, ua % HA, ua / HA, xa0);
+              load8(rb.A, si.layA, ub % HA, ub / HA, xa1);
+              load8(rb.B, si.layB, ua % HB, ua / HB, xb0);
+              load8(rb.B, si.layB, ub % HB, ub / HB, xb1);
+              pack8(xa0, lo[ls].A + (ua % HA) * 128, ua % HA, ua / HA, true);
+              pack8(xa1, lo[ls].A + (ub % HA) * 128, ub % HA, ub / HA, true);
+              pack8(xb0, lo[ls].B + (ua % HB) * 128, ua % HB, ua / HB, false);
+              pack8(xb1, lo[ls].B + (ub % HB) * 128, ub % HB, ub / HB, false);
+            } else {
+              pack_cross(rb.A, si.layA, lo[ls].A, HA, tt, true);
+              pack_cross(rb.B, si.layB, lo[ls].B, HB, tt, false);
+            }
           } else if (!(P.dbg & 1) && P.passes != 1) {
             split_pass(rb.A, lo[ls].A, G::A_BYTES, tt);
             split_pass(rb.B, lo[ls].B, G::B_BYTES, tt);
