@@ -656,6 +656,7 @@ static int strsm_fused(const TrsmGeom &g, cudaStream_t s, int sms) {
     if ((int)ph.size() >= MAX_FUSED_PHASES) { ok = false; return 0; }
     FusedPhase f;
     f.P = P; f.dep_full = (int32_t)full; f.dep_slab = (int32_t)slab; f.slab_m = g.left ? 0 : 1;
+    if (math_mode() == BLAS3_MATH_TF32_BF16X) f.P.passes = 2;   // (1xTF32: fused stays 3xTF32)
     ph.push_back(f);
     return (int)ph.size() - 1;
   };
@@ -835,6 +836,7 @@ static int strsm_first_fused(const TrsmGeom &g, const std::vector<GeoPair> &gp, 
   auto add = [&](const Problem &P, uint32_t full, uint32_t slab) -> int {
     FusedPhase f;
     f.P = P; f.dep_full = (int32_t)full; f.dep_slab = (int32_t)slab; f.slab_m = g.left ? 0 : 1;
+    if (math_mode() == BLAS3_MATH_TF32_BF16X) f.P.passes = 2;   // (1xTF32: fused stays 3xTF32)
     ph.push_back(f);
     return (int)ph.size() - 1;
   };

@@ -1187,12 +1187,10 @@ static int launch_cg(PRM &prm, cudaStream_t stream, int num_sms, bool allow_pdl 
       if (!op_maps(prm, slot, sg.b, P.N, sg.K, G::HB, per, groups, P.bs_b)) return -4;
     }
   }
-  // the TF32+BF16X instantiation for single-phase launches in that mode
-  constexpr bool SINGLE = sizeof(prm.ph) / sizeof(prm.ph[0]) == 1;
-  const bool bx = SINGLE && prm.ph[0].P.passes == 2;
-  void (*kfn)(PRM) = tc_structured_gemm<CG, PRM, false>;
-  if constexpr (SINGLE)
-    if (bx) kfn = tc_structured_gemm<CG, PRM, true>;
+  // the TF32+BF16X instantiation in that mode (every phase of a fused launch
+  // carries the same mode)
+  const bool bx = prm.ph[0].P.passes == 2;
+  void (*kfn)(PRM) = bx ? tc_structured_gemm<CG, PRM, true> : tc_structured_gemm<CG, PRM, false>;
   static bool attr[2] = {false, false};
   if (!attr[bx]) {
     if (cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)G::SMEM) != cudaSuccess)

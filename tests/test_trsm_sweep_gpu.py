@@ -107,3 +107,27 @@ def test_strsm_small_panels_many_slabs(nb, fused, split):
     r = subprocess.run(cmd, env=env, cwd=ROOT, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
     assert " passed" in r.stdout
+
+
+@pytest.mark.parametrize("side,uplo,ta", [("L", "L", "N"), ("R", "U", "T"), ("L", "U", "T")])
+def test_strsm_multi_panel_tf32_bf16x(b3, oracle_mod, side, uplo, ta):
+    """The TF32+BF16X mode on the multi-panel path, whose fused first-panel
+    launch then runs the BX kernel instantiation too."""
+    ka, other = 2600, 4500
+    m, n = (ka, other) if side == "L" else (other, ka)
+    A = gen.triangular_dd(ka, uplo, "N", "bx-a")
+    B = gen.uniform(m, n, "bx-b")
+    dB = to_dev(B)
+    b3.set_math_mode("tf32_bf16x")
+    try:
+        b3.strsm(side, uplo, ta, "N", AL, to_dev(A), dB)
+    finally:
+        b3.set_math_mode("3xtf32")
+    X = f64(to_host(dB))
+    T = op(tri_full(A, uplo, "N", ka), ta)
+    sel = gen.sample_indices(other, 16, "bx-sel")
+    Xs, Bs = (X[:, sel], f64(B[:, sel])) if side == "L" else (X[sel, :], f64(B[sel, :]))
+    resid = (T @ Xs - AL * Bs) if side == "L" else (Xs @ T - AL * Bs)
+    assert fro(resid) / (fro(T) * fro(Xs)) <= 1e-5 * np.sqrt(ka)
+    ref = oracle_mod.strsm(side, uplo, ta, "N", AL, A, B, sel=sel)
+    assert fro(Xs - ref) / fro(ref) <= 1e-5
