@@ -231,8 +231,8 @@ int blas3_set_workspace(void *dptr, size_t bytes);
  * the bench uses it to report gpu_launches). */
 int64_t blas3_launch_count(void);
 
-/* Same counter split by route: BLAS3_PATH_TCGEN05 (3xTF32 tensor-core
- * structured GEMM), BLAS3_PATH_SIMT (FP32 SIMT structured GEMM),
+/* Same counter split by route: BLAS3_PATH_TCGEN05 (tcgen05 tensor-core
+ * structured GEMM, any tensor math mode), BLAS3_PATH_SIMT (FP32 SIMT structured GEMM),
  * BLAS3_PATH_AUX (scale / copy / TRSM diagonal-inverse kernels).  Returns -1
  * for an unknown path.  Lets tests assert which route a call took. */
 enum { BLAS3_PATH_TCGEN05 = 0, BLAS3_PATH_SIMT = 1, BLAS3_PATH_AUX = 2 };
