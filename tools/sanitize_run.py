@@ -20,7 +20,7 @@ def rnd(m, n):
 
 
 calls = 0
-for mode in ("3xtf32", "simt"):
+for mode in ("3xtf32", "simt", "tf32_bf16x"):
     b3.set_math_mode(mode)
     m, n, k = 300, 260, 270
     A, B, C = rnd(m, k), rnd(k, n), rnd(m, n)
