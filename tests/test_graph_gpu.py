@@ -41,7 +41,7 @@ def _chain(b3, A, T, B, C, X):
     b3.strsm("R", "U", "T", "N", AL, T, X)
 
 
-@pytest.mark.parametrize("mode", ["3xtf32", "simt"])
+@pytest.mark.parametrize("mode", ["3xtf32", "simt", "tf32_bf16x"])
 def test_chain_graph_replay_bit_identical(b3, mode):
     import torch
     b3.set_math_mode(mode)

@@ -25,16 +25,17 @@ def ld_for(rows, kind, off):
     return ld + 1 if kind == "ld_odd" else ld
 
 
-@pytest.fixture(scope="module")
-def b3():
+@pytest.fixture(scope="module", params=["3xtf32", "tf32_bf16x"])
+def b3(request):
     import torch
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     import __graft_entry__
     __graft_entry__.build()
     import paper_conf_ipps_cuiwxyf11_b200 as m
+    m.set_math_mode(request.param)
+    yield m
     m.set_math_mode("3xtf32")
-    return m
 
 
 def embed(X, kind, off, tag):
