@@ -19,7 +19,8 @@ inside the timed region (column-slab sharding, weak scaling).
 
 After the headline (default 3xTF32) run, a short device-only pass of the same
 chain in the opt-in TF32+BF16X mode is reported under "alt_mode" (never as
-the headline; --no-alt-mode skips it).
+the headline; --no-alt-mode skips it), and the box's cuBLAS SGEMM (fp32 and
+1-pass TF32, torch.matmul) under "context" (--no-context skips it).
 
 --impl reference times the fp64 CPU oracle (the deliberately slow reference
 arm of this tier) on a bounded column sample of the same workload.
@@ -397,6 +398,33 @@ def run_ours(args):
             for r in ROUTINES:
                 ev[r][:] = per_default[r]
 
+    # context (north star: "reports the box's cuBLAS SGEMM as context"): torch's
+    # cuBLAS fp32 SGEMM (TF32 off) and its 1-pass TF32 mode on the same A, B
+    context = None
+    if world == 1 and n == N and not args.no_context:
+        def cublas_rate(tf32):
+            prev = torch.backends.cuda.matmul.allow_tf32
+            torch.backends.cuda.matmul.allow_tf32 = tf32
+            try:
+                out = torch.empty((n, n), device=dev)
+                for _ in range(2):
+                    torch.matmul(A, Bm, out=out)
+                torch.cuda.synchronize()
+                c0 = torch.cuda.Event(enable_timing=True); c1 = torch.cuda.Event(enable_timing=True)
+                reps = 3
+                c0.record(stream)
+                for _ in range(reps):
+                    torch.matmul(A, Bm, out=out)
+                c1.record(stream)
+                torch.cuda.synchronize()
+                return round(2.0 * n ** 3 / (c0.elapsed_time(c1) / reps * 1e-3) / 1e9, 1)
+            finally:
+                torch.backends.cuda.matmul.allow_tf32 = prev
+        context = {"cublas_sgemm_fp32_gflops": cublas_rate(False),
+                   "cublas_sgemm_tf32_1pass_gflops": cublas_rate(True),
+                   "note": "torch.matmul (cuBLAS) N=8192 NN on the bench's A, B; fp32 = TF32 off "
+                           "(the fp32-accurate comparator); tf32 = 1 pass, ~1e-3 accuracy"}
+
     total_flops = sum(fl.values()) * world
     step_ms = ms / args.steps
     value = total_flops / (step_ms * 1e-3) / 1e9
@@ -467,6 +495,7 @@ def run_ours(args):
                 "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world},
         "gpu_launches": int(launches),
         "alt_mode": alt,
+        "context": context,
         "gpu_launches_per_step": round(launches / args.steps, 1),
         "clocks": clk.summary(),
     }
@@ -583,6 +612,7 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the e2e leg (profiling runs)")
+    ap.add_argument("--no-context", action="store_true", help="skip the cuBLAS context timing")
     ap.add_argument("--no-alt-mode", action="store_true",
                     help="skip the extra device-only pass in the opt-in TF32+BF16X mode")
     args = ap.parse_args()
