@@ -423,7 +423,13 @@ def run_ours(args):
         context = {"cublas_sgemm_fp32_gflops": cublas_rate(False),
                    "cublas_sgemm_tf32_1pass_gflops": cublas_rate(True),
                    "note": "torch.matmul (cuBLAS) N=8192 NN on the bench's A, B; fp32 = TF32 off "
-                           "(the fp32-accurate comparator); tf32 = 1 pass, ~1e-3 accuracy"}
+                           "(the fp32-accurate comparator); tf32 = 1 pass, ~1e-3 accuracy",
+                   # the paper's own numbers with their hardware (quoted, not measured here;
+                   # PAPER.md P:15)
+                   "paper": {"max_speedup_over_cublas3.2": {"GeForce 9800": 5.4, "GTX285": 2.8,
+                                                             "Tesla C2050": 3.4},
+                             "gtx285_cublas3.2_sgemm_gflops": 420, "gtx285_cublas3.2_ssymm_gflops": 155,
+                             "gtx285_oa_ssymm_gflops": 403, "problem": "fp32, N=4096"}}
 
     total_flops = sum(fl.values()) * world
     step_ms = ms / args.steps
@@ -451,6 +457,9 @@ def run_ours(args):
             traffic = None
     h2d = (2 * n * n * 4 if rank == 0 else 0) + 2 * n * cols * 4
     d2h = 2 * n * cols * 4
+    if context is not None:
+        context["sgemm_speedup_over_cublas_fp32"] = round(
+            per["sgemm"]["gflops"] / context["cublas_sgemm_fp32_gflops"], 2)
     out = {
         "metric": "GFLOPS per routine (SGEMM/SSYMM/SSYRK/SSYR2K/STRMM/STRSM) at N=8192, "
                   "1/2/4/8 B200, % of peak",
