@@ -169,7 +169,9 @@ int blas3_get_math_mode(void);
  *   BLAS3_OPT_PDL          [BLAS3_PDL]      1 programmatic dependent launch (default), 0 off
  *   BLAS3_OPT_TRSM_NB      [BLAS3_TRSM_NB]  STRSM panel width: power of 2 in [128, 8192] (2048)
  *   BLAS3_OPT_TRSM_SLABS   [BLAS3_TRSM_SLABS] right-hand-side slabs on own streams, 1..4 (2)
- *   BLAS3_OPT_TRSM_SLAB_MIN [BLAS3_TRSM_SLAB_MIN] minimum slab width, >= 256 (2048)
+ *   BLAS3_OPT_TRSM_SLAB_MIN [BLAS3_TRSM_SLAB_MIN] minimum slab width, >= 256 (4096:
+ *                          one slab below 8192 right-hand sides -- measured 12%
+ *                          faster at 4096 -- two from 8192)
  *   BLAS3_OPT_TRSM_RESERVE [BLAS3_TRSM_RESERVE] SMs the first panel's sweep leaves to
  *                          the panel-inverse doubling chain, 0..74 (48)
  *   BLAS3_OPT_TRSM_GEO_LEAF [BLAS3_TRSM_GEO_LEAF] the first panel is halved down to

@@ -52,6 +52,7 @@ def test_strsm_multi_panel_multi_slab(b3, oracle_mod, side, uplo, ta, diag, spli
     B = gen.uniform(m, n, "sweep-b")
     dB = to_dev(B)
     opts = dict(trsm_first_all=1) if split == "all" else dict(trsm_first_split=split)
+    opts["trsm_slab_min"] = 2048          # two RHS slabs at 4500 (the default minimum is 4096)
     with b3.options(**opts):
         b3.strsm(side, uplo, ta, diag, AL, to_dev(A), dB)
     X = f64(to_host(dB))
