@@ -10,9 +10,9 @@ fastest.  Host-side orchestration only: every candidate runs through the same
 C-ABI entry points and CUDA kernels.
 
 Timing: CUDA events on the current stream; candidates are INTERLEAVED over
-``rounds`` rounds (1 warm-up + ``reps`` calls each) and compared by their
-median, so slow drifts of the clock under the power cap hit all candidates
-alike.
+``rounds`` rounds (1 warm-up + ``reps`` calls each, the visiting order rotated
+every round) and compared by their median, so slow drifts of the clock under
+the power cap and position effects hit all candidates alike.
 """
 from __future__ import annotations
 
@@ -39,9 +39,13 @@ def search(fn, candidates, reps=3, rounds=3):
     """Time `fn` under every option setting in `candidates` (dicts of option
     name -> value), interleaved.  Returns (best setting, [(setting, median ms)])."""
     samples = [[] for _ in candidates]
-    for _ in range(rounds):
-        for i, cand in enumerate(candidates):
-            with b3.options(**cand):
+    nc = len(candidates)
+    for r in range(rounds):
+        # rotate the visiting order every round, so position effects (clock /
+        # thermal state left by the previous candidate) do not favour any one
+        for j in range(nc):
+            i = (r + j) % nc
+            with b3.options(**candidates[i]):
                 samples[i].append(_time(fn, reps))
     table = [(c, statistics.median(s)) for c, s in zip(candidates, samples)]
     best = min(table, key=lambda t: t[1])[0]
