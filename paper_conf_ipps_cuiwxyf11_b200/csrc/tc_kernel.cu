@@ -443,6 +443,25 @@ __device__ __forceinline__ void pack8(const float (&x)[8], uint8_t *row, int r, 
   *reinterpret_cast<uint4 *>(row + (((2 * c) ^ (r & 7)) << 4)) = a_side ? lo : hi;
   *reinterpret_cast<uint4 *>(row + (((2 * c + 1) ^ (r & 7)) << 4)) = a_side ? hi : lo;
 }
+// pack8 in two halves: the packed 16-B chunks into registers (no shared-memory
+// writes), and their stores -- so the packing can run before the lo stage is free
+struct Packed { uint4 first, second; };
+__device__ __forceinline__ Packed pack8_regs(const float (&x)[8], bool a_side) {
+  uint4 hi, lo;
+  uint32_t *hp = &hi.x, *lp = &lo.x;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const float h0 = __uint_as_float(__float_as_uint(x[2 * i]) & 0xFFFFE000u);
+    const float h1 = __uint_as_float(__float_as_uint(x[2 * i + 1]) & 0xFFFFE000u);
+    hp[i] = pack_bf16x2(h0, h1);
+    lp[i] = pack_bf16x2(x[2 * i] - h0, x[2 * i + 1] - h1);
+  }
+  return Packed{a_side ? lo : hi, a_side ? hi : lo};
+}
+__device__ __forceinline__ void store_packed(const Packed &v, uint8_t *row, int r, int c) {
+  *reinterpret_cast<uint4 *>(row + (((2 * c) ^ (r & 7)) << 4)) = v.first;
+  *reinterpret_cast<uint4 *>(row + (((2 * c + 1) ^ (r & 7)) << 4)) = v.second;
+}
 __device__ __forceinline__ void load8(const uint8_t *raw, int lay, int r, int c, float (&x)[8]) {
   if (lay == LAYOUT_K) {            // a row's 8 k-values: two swizzled 16-B chunks
     const float4 v0 = *reinterpret_cast<const float4 *>(raw + off_k(r, 8 * c));
@@ -883,28 +902,35 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
             else if (own == BLK_TRI_DIAG && !(P.dbg & 32)) { tri_fix(sg.b, si.layB, rb.B, nb, k0, HB, P.N, sg.K, tt); fix = true; }
           }
           if (fix) ptx::named_bar_sync(1, TR_THREADS);
-          ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
           if constexpr (BX) {                               // packed bf16 cross terms
             if (HA == HB && !(P.dbg & 4096)) {
               // pair tiles: A and B have 128 rows = 2 units per thread each --
-              // all four units' loads first, then the packing (ILP)
+              // all four units loaded and packed into registers BEFORE waiting
+              // for the lo stage (overlaps the MMA still reading it), then stored
               const int ua = tt, ub = tt + TR_THREADS;
               float xa0[8], xa1[8], xb0[8], xb1[8];
               load8(rb.A, si.layA, ua % HA, ua / HA, xa0);
               load8(rb.A, si.layA, ub % HA, ub / HA, xa1);
               load8(rb.B, si.layB, ua % HB, ua / HB, xb0);
               load8(rb.B, si.layB, ub % HB, ub / HB, xb1);
-              pack8(xa0, lo[ls].A + (ua % HA) * 128, ua % HA, ua / HA, true);
-              pack8(xa1, lo[ls].A + (ub % HA) * 128, ub % HA, ub / HA, true);
-              pack8(xb0, lo[ls].B + (ua % HB) * 128, ua % HB, ua / HB, false);
-              pack8(xb1, lo[ls].B + (ub % HB) * 128, ub % HB, ub / HB, false);
+              const Packed pa0 = pack8_regs(xa0, true), pa1 = pack8_regs(xa1, true);
+              const Packed pb0 = pack8_regs(xb0, false), pb1 = pack8_regs(xb1, false);
+              ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
+              store_packed(pa0, lo[ls].A + (ua % HA) * 128, ua % HA, ua / HA);
+              store_packed(pa1, lo[ls].A + (ub % HA) * 128, ub % HA, ub / HA);
+              store_packed(pb0, lo[ls].B + (ua % HB) * 128, ua % HB, ua / HB);
+              store_packed(pb1, lo[ls].B + (ub % HB) * 128, ub % HB, ub / HB);
             } else {
+              ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
               pack_cross(rb.A, si.layA, lo[ls].A, HA, tt, true);
               pack_cross(rb.B, si.layB, lo[ls].B, HB, tt, false);
             }
-          } else if (!(P.dbg & 1) && P.passes != 1) {
-            split_pass(rb.A, lo[ls].A, G::A_BYTES, tt);
-            split_pass(rb.B, lo[ls].B, G::B_BYTES, tt);
+          } else {
+            ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
+            if (!(P.dbg & 1) && P.passes != 1) {
+              split_pass(rb.A, lo[ls].A, G::A_BYTES, tt);
+              split_pass(rb.B, lo[ls].B, G::B_BYTES, tt);
+            }
           }
           ptx::fence_proxy_async_smem();
           arrive_leader<CG>(&bars->ready[ls], rank, 2, TR_THREADS, tt == 0);
