@@ -205,6 +205,13 @@ int blas3_get_math_mode(void);
  *   BLAS3_OPT_TC_RASTER    [BLAS3_TC_RASTER] tile rows per group of the grouped
  *                          raster order of full grids (L2 reuse), 0..64; 0 =
  *                          the built-in default (8)
+ *   BLAS3_OPT_TC_KC        [BLAS3_TC_KC]    tcgen05 path: k-blocks (32 deep) summed in
+ *                          one TMEM partial before it is folded into the
+ *                          round-to-nearest register sum (Q24): power
+ *                          of 2 in [1, 64], default 4 (K = 128).  The tensor
+ *                          core's accumulator truncates on every UMMA add, so
+ *                          the output-relative error grows with this value
+ *                          (measured: 16 -> 3.9e-6, 4 -> fp32 class)
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */
@@ -215,7 +222,8 @@ enum {
     BLAS3_OPT_TRSM_NB = 9, BLAS3_OPT_TRSM_SLABS = 10, BLAS3_OPT_TRSM_SLAB_MIN = 11,
     BLAS3_OPT_TRSM_RESERVE = 12, BLAS3_OPT_TRSM_GEO_LEAF = 13, BLAS3_OPT_TRSM_FUSED = 14,
     BLAS3_OPT_TRSM_FIRST_YM = 15, BLAS3_OPT_TRSM_FIRST_FUSED = 16, BLAS3_OPT_TRSM_FIRST_SPLIT = 17,
-    BLAS3_OPT_TRSM_FIRST_ALL = 18, BLAS3_OPT_TC_RASTER = 19, BLAS3_OPT_COUNT = 20
+    BLAS3_OPT_TRSM_FIRST_ALL = 18, BLAS3_OPT_TC_RASTER = 19, BLAS3_OPT_TC_KC = 20,
+    BLAS3_OPT_COUNT = 21
 };
 int blas3_set_option(int key, int64_t value);
 int64_t blas3_get_option(int key);

@@ -19,6 +19,7 @@ Parity status: all six functions are pinned (tests/test_oracle.py); none is
 from __future__ import annotations
 
 import ctypes
+import hashlib
 import os
 import subprocess
 
@@ -35,13 +36,22 @@ _ptr = ctypes.c_void_p
 _chr = ctypes.c_char
 
 
+_CMD = ["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-std=c99", "-Wall"]
+
+
 def build(force: bool = False) -> str:
-    """Compile oracle.c into liboracle.so (gcc -O2 -fopenmp)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+    """Compile oracle.c into liboracle.so (gcc -O2 -fopenmp); rebuilt when the
+    SHA-256 of the source and command (stored in liboracle.so.sha256) changes."""
+    with open(_SRC, "rb") as f:
+        digest = hashlib.sha256(f.read() + repr(_CMD).encode()).hexdigest()
+    stamp = _LIB + ".sha256"
+    fresh = os.path.exists(_LIB) and os.path.exists(stamp) and open(stamp).read().strip() == digest
+    if force or not fresh:
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-std=c99",
-                               "-Wall", "-o", tmp, _SRC])
+        subprocess.check_call([*_CMD, "-o", tmp, _SRC])
         os.replace(tmp, _LIB)
+        with open(stamp, "w") as f:
+            f.write(digest + "\n")
     return _LIB
 
 

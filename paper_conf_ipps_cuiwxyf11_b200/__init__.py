@@ -118,12 +118,28 @@ def from_fortran(arr, device="cuda"):
 
 
 # ----------------------------------------------------------------- routines
+# Shape checks: the C ABI only sees pointers and leading dimensions, so a
+# tensor smaller than the problem needs would be read (or written) past its
+# allocation.  Each wrapper derives the problem size from C (or B) and op(A)
+# as in BLAS and requires every operand to hold at least the leading block
+# the routine reads (extra rows / columns are ignored, as with BLAS's ld).
+def _need(name, X, rows, cols):
+    if X.shape[0] < rows or X.shape[1] < cols:
+        raise ValueError(f"{name} is {tuple(X.shape)}, the call needs at least {rows} x {cols}")
+
+
+def _t(c):
+    return c.upper() != "N" if isinstance(c, str) else c.upper() != b"N"
+
+
 def sgemm(transa, transb, alpha, A, B, beta, C):
     """C <- alpha*op(A)*op(B) + beta*C (GEMM-NN/-TN, P:77, P:392)."""
     pc, m, n, ldc = _mat(C, "C")
     pa, ar, ac, lda = _mat(A, "A")
     pb, br, bc, ldb = _mat(B, "B")
-    k = ac if transa.upper() == "N" else ar
+    k = ac if not _t(transa) else ar
+    _need("A", A, *((k, m) if _t(transa) else (m, k)))
+    _need("B", B, *((n, k) if _t(transb) else (k, n)))
     _chk("blas3_sgemm", blas3_sgemm(_ch(transa), _ch(transb), m, n, k, alpha, pa, lda, pb, ldb,  # noqa: F821
                                     beta, pc, ldc, _stream()))
 
@@ -133,6 +149,9 @@ def ssymm(side, uplo, alpha, A, B, beta, C):
     pc, m, n, ldc = _mat(C, "C")
     pa, _, _, lda = _mat(A, "A")
     pb, _, _, ldb = _mat(B, "B")
+    ka = m if (side.upper() if isinstance(side, str) else side.decode().upper()) == "L" else n
+    _need("A", A, ka, ka)
+    _need("B", B, m, n)
     _chk("blas3_ssymm", blas3_ssymm(_ch(side), _ch(uplo), m, n, alpha, pa, lda, pb, ldb,  # noqa: F821
                                     beta, pc, ldc, _stream()))
 
@@ -141,7 +160,9 @@ def ssyrk(uplo, trans, alpha, A, beta, C):
     """C <- alpha*op(A)*op(A)^T + beta*C on the uplo triangle."""
     pc, n, _, ldc = _mat(C, "C")
     pa, ar, ac, lda = _mat(A, "A")
-    k = ac if trans.upper() == "N" else ar
+    k = ac if not _t(trans) else ar
+    _need("C", C, n, n)
+    _need("A", A, *((k, n) if _t(trans) else (n, k)))
     _chk("blas3_ssyrk", blas3_ssyrk(_ch(uplo), _ch(trans), n, k, alpha, pa, lda, beta, pc, ldc,  # noqa: F821
                                     _stream()))
 
@@ -151,15 +172,24 @@ def ssyr2k(uplo, trans, alpha, A, B, beta, C):
     pc, n, _, ldc = _mat(C, "C")
     pa, ar, ac, lda = _mat(A, "A")
     pb, _, _, ldb = _mat(B, "B")
-    k = ac if trans.upper() == "N" else ar
+    k = ac if not _t(trans) else ar
+    _need("C", C, n, n)
+    _need("A", A, *((k, n) if _t(trans) else (n, k)))
+    _need("B", B, *((k, n) if _t(trans) else (n, k)))
     _chk("blas3_ssyr2k", blas3_ssyr2k(_ch(uplo), _ch(trans), n, k, alpha, pa, lda, pb, ldb,  # noqa: F821
                                       beta, pc, ldc, _stream()))
+
+
+def _order(side, m, n):
+    return m if (side.upper() if isinstance(side, str) else side.decode().upper()) == "L" else n
 
 
 def strmm(side, uplo, transa, diag, alpha, A, B):
     """B <- alpha*op(A)*B (L) or alpha*B*op(A) (R), in place."""
     pb, m, n, ldb = _mat(B, "B")
     pa, _, _, lda = _mat(A, "A")
+    ka = _order(side, m, n)
+    _need("A", A, ka, ka)
     _chk("blas3_strmm", blas3_strmm(_ch(side), _ch(uplo), _ch(transa), _ch(diag), m, n, alpha,  # noqa: F821
                                     pa, lda, pb, ldb, _stream()))
 
@@ -168,6 +198,8 @@ def strsm(side, uplo, transa, diag, alpha, A, B):
     """Solve op(A)X = alpha*B (L) or X op(A) = alpha*B (R); X overwrites B."""
     pb, m, n, ldb = _mat(B, "B")
     pa, _, _, lda = _mat(A, "A")
+    ka = _order(side, m, n)
+    _need("A", A, ka, ka)
     _chk("blas3_strsm", blas3_strsm(_ch(side), _ch(uplo), _ch(transa), _ch(diag), m, n, alpha,  # noqa: F821
                                     pa, lda, pb, ldb, _stream()))
 
@@ -189,7 +221,8 @@ PATH_TCGEN05, PATH_SIMT, PATH_AUX = 0, 1, 2
 OPTIONS = {"gm_map": 0, "gm_min_gemm": 1, "gm_min_symm": 2, "gm_min_trmm": 3, "gm_min_trsm": 4,
            "tc_cta": 5, "tc_split": 6, "tc_static": 7, "pdl": 8, "trsm_nb": 9, "trsm_slabs": 10,
            "trsm_slab_min": 11, "trsm_reserve": 12, "trsm_geo_leaf": 13, "trsm_fused": 14,
-           "trsm_first_ym": 15, "trsm_first_fused": 16, "trsm_first_split": 17, "trsm_first_all": 18, "tc_raster": 19}
+           "trsm_first_ym": 15, "trsm_first_fused": 16, "trsm_first_split": 17, "trsm_first_all": 18, "tc_raster": 19,
+           "tc_kc": 20}
 
 
 def set_option(name, value):

@@ -1,12 +1,15 @@
 """Build libblas3.so (the C-ABI library) in-tree for sm_100a.
 
 nvcc -gencode arch=compute_100a,code=sm_100a -lineinfo, cudart linked
-statically, one object per .cu compiled in parallel, then linked.  The .so
+statically, one object per .cu compiled in parallel, then linked.  Every
+step is keyed by a SHA-256 of its inputs (sources, headers, flags), stored
+beside the output as <file>.sha256.  The .so
 lives next to this file so it travels with the repo snapshot to the GPU box.
 """
 from __future__ import annotations
 
 import concurrent.futures as cf
+import hashlib
 import os
 import subprocess
 import sys
@@ -25,17 +28,43 @@ def sources():
     return sorted(os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith(".cu"))
 
 
-def _headers_mtime():
-    hs = [os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith(".h")]
+def _headers():
+    hs = sorted(os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith(".h"))
     hs.append(os.path.join(os.path.dirname(HERE), "include", "blas3.h"))
-    return max(os.path.getmtime(h) for h in hs)
+    return hs
+
+
+def _digest(paths, extra):
+    """Content hash of the inputs of one build step (sources, every header,
+    compiler and flags): rebuilds follow content, never file times, so a
+    stale object or library shipped with a snapshot is never reused."""
+    h = hashlib.sha256()
+    for p in paths:
+        h.update(p.encode())
+        with open(p, "rb") as f:
+            h.update(f.read())
+    h.update(repr(extra).encode())
+    return h.hexdigest()
+
+
+def _stamp_ok(out, digest):
+    try:
+        with open(out + ".sha256") as f:
+            return os.path.exists(out) and f.read().strip() == digest
+    except OSError:
+        return False
+
+
+def _write_stamp(out, digest):
+    with open(out + ".sha256", "w") as f:
+        f.write(digest + "\n")
 
 
 def _compile(src, verbose):
     obj = os.path.join(BUILD, os.path.basename(src) + ".o")
-    if (os.path.exists(obj) and os.path.getmtime(obj) >= os.path.getmtime(src)
-            and os.path.getmtime(obj) >= _headers_mtime()):
-        return obj
+    digest = _digest([src, *_headers()], (NVCC, ARCH, FLAGS))
+    if _stamp_ok(obj, digest):
+        return obj, digest
     cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
@@ -44,7 +73,8 @@ def _compile(src, verbose):
         raise RuntimeError(f"nvcc failed on {src}:\n{r.stdout}\n{r.stderr}")
     if verbose and r.stderr:
         print(r.stderr, file=sys.stderr)
-    return obj
+    _write_stamp(obj, digest)
+    return obj, digest
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
@@ -52,15 +82,20 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if force:
         for f in os.listdir(BUILD):
             os.remove(os.path.join(BUILD, f))
+        if os.path.exists(OUT + ".sha256"):
+            os.remove(OUT + ".sha256")
     with cf.ThreadPoolExecutor(max_workers=os.cpu_count() or 4) as ex:
-        objs = list(ex.map(lambda s: _compile(s, verbose), sources()))
-    if not os.path.exists(OUT) or any(os.path.getmtime(o) > os.path.getmtime(OUT) for o in objs):
+        res = list(ex.map(lambda s: _compile(s, verbose), sources()))
+    objs = [o for o, _ in res]
+    link_digest = hashlib.sha256("".join(d for _, d in res).encode()).hexdigest()
+    if not _stamp_ok(OUT, link_digest):
         tmp = OUT + f".tmp{os.getpid()}"
         cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
         os.replace(tmp, OUT)
+        _write_stamp(OUT, link_digest)
     return OUT
 
 

@@ -47,6 +47,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TRSM_FIRST_SPLIT", 0, 0, 8192, true},
     {"BLAS3_TRSM_FIRST_ALL", 0, 0, 1, false},
     {"BLAS3_TC_RASTER", 0, 0, 64, false},
+    {"BLAS3_TC_KC", 4, 1, 64, true},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;
@@ -69,24 +70,48 @@ static void opt_init() {
     }
   });
 }
-int64_t opt(int key) {
-  opt_init();
-  return (key >= 0 && key < BLAS3_OPT_COUNT) ? g_opt[key].load(std::memory_order_relaxed) : 0;
-}
-
-static int g_math = -1;              // -1: not initialised
+static std::atomic<int> g_math{-1};   // -1: not initialised
 static void *g_ws = nullptr;
 static size_t g_ws_bytes = 0;
 
-static int math_mode() {
-  if (g_math < 0) {
+static int global_math_mode() {
+  int m = g_math.load(std::memory_order_acquire);
+  if (m < 0) {
     const char *e = getenv("BLAS3_MATH");
-    g_math = (e && (e[0] == 's' || e[0] == 'S')) ? BLAS3_MATH_SIMT_FP32
-             : (e && e[0] == '1') ? BLAS3_MATH_1XTF32
-             : (e && (e[0] == 'b' || e[0] == 'B')) ? BLAS3_MATH_TF32_BF16X : BLAS3_MATH_3XTF32;
+    const int env = (e && (e[0] == 's' || e[0] == 'S')) ? BLAS3_MATH_SIMT_FP32
+                    : (e && e[0] == '1') ? BLAS3_MATH_1XTF32
+                    : (e && (e[0] == 'b' || e[0] == 'B')) ? BLAS3_MATH_TF32_BF16X : BLAS3_MATH_3XTF32;
+    int expect = -1;
+    g_math.compare_exchange_strong(expect, env);
+    m = g_math.load(std::memory_order_acquire);
   }
-  return g_math;
+  return m;
 }
+
+// Per-call snapshot of the process-wide options and math mode: every entry
+// point takes one (CallOpts) before it reads any, so a blas3_set_option /
+// blas3_set_math_mode from another thread mid-call can never give one call
+// two different panel widths, tile shapes or modes.
+struct OptSnap { int64_t v[BLAS3_OPT_COUNT]; int math; };
+static thread_local const OptSnap *t_snap = nullptr;
+struct CallOpts {
+  OptSnap snap;
+  const OptSnap *prev;
+  CallOpts() : prev(t_snap) {
+    opt_init();
+    for (int k = 0; k < BLAS3_OPT_COUNT; ++k) snap.v[k] = g_opt[k].load(std::memory_order_relaxed);
+    snap.math = global_math_mode();
+    t_snap = &snap;
+  }
+  ~CallOpts() { t_snap = prev; }
+};
+int64_t opt(int key) {
+  if (key < 0 || key >= BLAS3_OPT_COUNT) return 0;
+  if (t_snap) return t_snap->v[key];
+  opt_init();
+  return g_opt[key].load(std::memory_order_relaxed);
+}
+static int math_mode() { return t_snap ? t_snap->math : global_math_mode(); }
 static bool tensor_mode() { return math_mode() != BLAS3_MATH_SIMT_FP32; }
 
 // per-device facts: SM count, sm_100 check
@@ -165,6 +190,7 @@ static Problem problem(int64_t M, int64_t N, float alpha, float beta, const floa
   P.Cin = Cin; P.ldcin = ldcin; P.Cout = Cout; P.ldcout = ldcout;
   P.nbatch = 1; P.per = 1;
   P.raster_gm = (int32_t)opt(BLAS3_OPT_TC_RASTER);
+  P.kc = (int32_t)opt(BLAS3_OPT_TC_KC);
   return P;
 }
 
@@ -232,10 +258,10 @@ int64_t blas3_get_option(int key) {
 int blas3_set_math_mode(int mode) {
   if (mode != BLAS3_MATH_3XTF32 && mode != BLAS3_MATH_SIMT_FP32 && mode != BLAS3_MATH_1XTF32 &&
       mode != BLAS3_MATH_TF32_BF16X) return 1;
-  g_math = mode;
+  g_math.store(mode, std::memory_order_release);
   return 0;
 }
-int blas3_get_math_mode(void) { return math_mode(); }
+int blas3_get_math_mode(void) { return global_math_mode(); }
 
 int blas3_set_workspace(void *dptr, size_t bytes) {
   g_ws = bytes ? dptr : nullptr;
@@ -258,6 +284,7 @@ const char *blas3_error_string(int code) {
 int blas3_sgemm(char transa, char transb, int64_t m, int64_t n, int64_t k, float alpha,
                 const float *A, int64_t lda, const float *B, int64_t ldb, float beta, float *C,
                 int64_t ldc, blas3_stream_t stream) {
+  CallOpts call_opts;
   const bool ta = up(transa) != 'N', tb = up(transb) != 'N';
   if (!is_trans(transa)) return 1;
   if (!is_trans(transb)) return 2;
@@ -296,6 +323,7 @@ int blas3_sgemm(char transa, char transb, int64_t m, int64_t n, int64_t k, float
 int blas3_ssymm(char side, char uplo, int64_t m, int64_t n, float alpha, const float *A,
                 int64_t lda, const float *B, int64_t ldb, float beta, float *C, int64_t ldc,
                 blas3_stream_t stream) {
+  CallOpts call_opts;
   const bool left = up(side) == 'L', lower = up(uplo) == 'L';
   if (!is_side(side)) return 1;
   if (!is_uplo(uplo)) return 2;
@@ -343,6 +371,7 @@ int blas3_ssymm(char side, char uplo, int64_t m, int64_t n, float alpha, const f
 static int syrk_common(bool two, char uplo, char trans, int64_t n, int64_t k, float alpha,
                        const float *A, int64_t lda, const float *B, int64_t ldb, float beta,
                        float *C, int64_t ldc, cudaStream_t s) {
+  CallOpts call_opts;
   const bool lower = up(uplo) == 'L', ta = up(trans) != 'N';
   const int tri = lower ? 1 : 2;
   if (n == 0 || ((alpha == 0.f || k == 0) && beta == 1.f)) return 0;
@@ -417,6 +446,7 @@ static int tr_validate(char side, char uplo, char transa, char diag, int64_t m, 
 // product goes to stream-ordered scratch and is copied back (A9).
 int blas3_strmm(char side, char uplo, char transa, char diag, int64_t m, int64_t n, float alpha,
                 const float *A, int64_t lda, float *B, int64_t ldb, blas3_stream_t stream) {
+  CallOpts call_opts;
   int v = tr_validate(side, uplo, transa, diag, m, n, lda, ldb);
   if (v) return v;
   if (m == 0 || n == 0) return 0;
@@ -937,6 +967,7 @@ static int strsm_first_fused(const TrsmGeom &g, const std::vector<GeoPair> &gp, 
 
 int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t n, float alpha,
                 const float *A, int64_t lda, float *B, int64_t ldb, blas3_stream_t stream) {
+  CallOpts call_opts;
   int v = tr_validate(side, uplo, transa, diag, m, n, lda, ldb);
   if (v) return v;
   if (m == 0 || n == 0) return 0;

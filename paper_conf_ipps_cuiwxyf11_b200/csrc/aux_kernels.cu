@@ -12,6 +12,7 @@
 // and broadcast by __shfl_sync, then the off-diagonal 32x32 blocks follow by
 // block forward substitution, one warp per block column.
 #include <cuda_runtime.h>
+#include <atomic>
 #include "kernels.h"
 
 namespace blas3 {
@@ -381,11 +382,13 @@ int launch_trsm_diag_inv(const float *A, int64_t lda, int64_t n, int stored_lowe
                          float *Dinv, int64_t ldD, cudaStream_t s) {
   if (ldD % DNB) return -1;
   const size_t smem = (2 * DNB * DLD + 4 * 32 * 33) * sizeof(float);
-  static bool attr = false;
-  if (!attr) {
+  static std::atomic<bool> attr[64];              // per device context
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return -1;
+  if (!attr[dev].load(std::memory_order_acquire)) {
     if (cudaFuncSetAttribute(trsm_diag_inv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)smem) != cudaSuccess) return -1;
-    attr = true;
+    attr[dev].store(true, std::memory_order_release);
   }
   int64_t blocks = cdiv(n, DNB);
   trsm_diag_inv_kernel<<<(unsigned)blocks, DT, smem, s>>>(A, lda, n, stored_lower, unit, Dinv, ldD);

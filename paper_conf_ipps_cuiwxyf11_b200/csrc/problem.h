@@ -85,6 +85,8 @@ struct Problem {
   int32_t passes;
   // full-grid raster: m-tiles per group (0: Tiles::GM); BLAS3_OPT_TC_RASTER
   int32_t raster_gm;
+  // tcgen05 path: k-blocks per TMEM partial (power of 2; BLAS3_OPT_TC_KC)
+  int32_t kc;
 };
 
 HD int64_t batch_off(const BatchStride &s, int64_t b, int64_t per) {

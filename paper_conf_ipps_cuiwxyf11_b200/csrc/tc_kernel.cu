@@ -17,21 +17,26 @@
 //   Reg_alloc(C)                        -> fp32 accumulator in TMEM
 //       (two 256-column accumulators: epilogue of tile i overlaps tile i+1).
 // fp32 accuracy on TF32 tensor cores (north star): every staged value x is
-// split into hi = trunc_tf32(x) (what the tensor core reads from the raw
-// word) and lo = rna_tf32(x - hi), and each k-step issues lo*hi + hi*lo +
-// hi*hi (small terms first) into the same fp32 accumulator.
+// split into hi = trunc_tf32(x) -- what the tensor core reads from the raw
+// TMA-staged word (kind::tf32 ignores the low 13 mantissa bits, DESIGN.md
+// Q23) -- and lo = x - hi (exact in fp32, written by the transform warps);
+// each k8-step issues lo*hi + hi*lo + hi*hi (small terms first) into one fp32
+// TMEM partial that is restarted every Problem::kc k-blocks (Q24).
 //
-// Warp roles (576 threads, 1 CTA/SM; in a pair every CTA runs all roles on its
-// own halves except the MMA issuer, which only the leader CTA runs):
-//   warp 0       TMA producer (one lane)
-//   warp 1       TMEM allocator + MMA issuer (one lane)
-//   warps 2..9   transform: structure fix-ups + hi/lo split (256 threads)
-//   warps 10..17 epilogue: tcgen05.ld -> alpha*acc + beta*C -> global
-//                (two warps per TMEM lane quarter, 128 columns each)
+// Warp roles (640 threads, 1 CTA/SM, aligned to warpgroups for setmaxnreg;
+// in a pair every CTA runs all roles on its own halves except the MMA issuer,
+// which only the leader CTA runs):
+//   warp 0        TMA producer (one lane)
+//   warp 1        TMEM allocator + MMA issuer (one lane)
+//   warps 2..3    idle (pad the first warpgroup)
+//   warps 4..11   transform: structure fix-ups + lo split (256 threads)
+//   warps 12..19  epilogue: tcgen05.ld -> running sum -> alpha*S + beta*C ->
+//                 global (two warps per TMEM lane quarter, 128 columns each)
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <atomic>
 #include <mutex>
+#include <vector>
 #include <cstdio>
 #include <stdlib.h>
 #include <string.h>
@@ -61,10 +66,10 @@ constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;       // 640
 // 96 x 640 = 61440), so 256*EPI_REGS + 384*OTHER_REGS must not exceed it.
 constexpr int EPI_REGS = 144, OTHER_REGS = 64;   // 36864 + 24576 = 61440
 // Chunked accumulation: the tensor core's fp32 accumulator truncates on every
-// UMMA add (Q24), so a TMEM partial only ever sums KC k-blocks
-// (K = 256) before the epilogue folds it into a register running sum with
-// round-to-nearest adds; the two TMEM buffers ping-pong per chunk.
-constexpr int KC = 16;
+// UMMA add (Q24), so a TMEM partial only ever sums Problem::kc
+// k-blocks (BLAS3_OPT_TC_KC, default 4: K = 128) before the epilogue folds it
+// into a register running sum with round-to-nearest adds; the two TMEM
+// buffers ping-pong per chunk.
 constexpr int EC = 16;                            // epilogue column group
 // Tile queue: the producer warp claims tiles (atomic counter, or the static
 // round-robin sequence for CTA pairs) and hands them to the MMA, transform
@@ -762,6 +767,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
         const int64_t m0 = w.m0, n0 = w.n0;
         const int64_t nkb = w.g1 - w.g0;
         int64_t done = 0;
+        const int64_t kc = P.kc;
         uint32_t accumulate = 0, buf = 0;
         auto open_chunk = [&]() {
           buf = cc & 1;
@@ -793,7 +799,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           clip_kblocks(w, gi, kb0, kb1);
           const StageBand bd = make_band<CG>(P, sg, m0, n0);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
-            if (done % KC == 0) open_chunk();
+            if (done % kc == 0) open_chunk();
             const uint32_t d_tmem = tmem + buf * BN;
             const int rs = it % RS, ls = it % LS;
             const uint32_t lph = (it / LS) & 1;
@@ -851,7 +857,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
             __syncwarp();
             ++done;
             if (lane == 0 && done == nkb) BLAS3_STRACE(5, w.ph);
-            if (done % KC == 0 || done == nkb) close_chunk(true);
+            if (done % kc == 0 || done == nkb) close_chunk(true);
           }
         }
       }
@@ -943,7 +949,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
     // ============================ epilogue warps (own 128 rows, 128 of the BN columns)
     BLAS3_INC_REGS();
     // Each thread owns one row r and 128 columns: S[] is the fp32 running sum
-    // of the KC-chunk partials (round-to-nearest adds), then
+    // of the kc-chunk partials (round-to-nearest adds), then
     // D = alpha*S + beta*C is stored with coalesced 128-B warp accesses.
     const int q = warp & 3;                     // TMEM lane quarter of this warp
     const int half = (warp - WARP_EPI0) >> 2;   // which 128 of the 256 columns
@@ -957,7 +963,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
       const int64_t coff = (P.nbatch > 1) ? batch_off(P.bs_c, w.b, per) : 0;
       const int64_t m0 = w.m0, n0 = w.n0;
       const int64_t nkb = w.g1 - w.g0;
-      const int64_t nchunks = nkb > 0 ? cdiv(nkb, KC) : 1;
+      const int64_t nchunks = nkb > 0 ? cdiv(nkb, P.kc) : 1;
       float S[NG * EC];
 #pragma unroll
       for (int i = 0; i < NG * EC; ++i) S[i] = 0.f;
@@ -1217,11 +1223,14 @@ static int launch_cg(PRM &prm, cudaStream_t stream, int num_sms, bool allow_pdl 
   // carries the same mode)
   const bool bx = prm.ph[0].P.passes == 2;
   void (*kfn)(PRM) = bx ? tc_structured_gemm<CG, PRM, true> : tc_structured_gemm<CG, PRM, false>;
-  static bool attr[2] = {false, false};
-  if (!attr[bx]) {
+  // the attribute is per device context: remembered per (device, instantiation)
+  static std::atomic<bool> attr[64][2];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return -1;
+  if (!attr[dev][bx].load(std::memory_order_acquire)) {
     if (cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)G::SMEM) != cudaSuccess)
       return -1;
-    attr[bx] = true;
+    attr[dev][bx].store(true, std::memory_order_release);
   }
   const int64_t items = prm.nitems;        // tiles, or tiles + split-tail slices
   if (items == 0) return 0;
@@ -1249,58 +1258,92 @@ static int launch_cg(PRM &prm, cudaStream_t stream, int num_sms, bool allow_pdl 
   return (e == cudaSuccess && cudaGetLastError() == cudaSuccess) ? 0 : -1;
 }
 
-// Dynamic tile scheduling counters: a ring of per-launch slots per device
-// (concurrent launches on different streams never share one).  Every slot is
-// 0 between launches: the launch's last claim resets it on the device
-// (tc_structured_gemm), so a captured CUDA graph replays correctly and no
-// memset node is needed.
-struct TileCounter { uint32_t *ctr; };
-static bool tile_counter(TileCounter &tc) {
-  constexpr int SLOTS = 256;
-  static uint32_t *ring[64] = {};
-  static std::atomic<uint32_t> next[64];      // regular and fused launches hold different locks
-  static std::mutex alloc_mu;
-  int d = 0;
-  if (cudaGetDevice(&d) != cudaSuccess || d < 0 || d >= 64) return false;
-  std::lock_guard<std::mutex> lk(alloc_mu);
-  if (!ring[d]) {
-    if (cudaMalloc(&ring[d], SLOTS * 32 * sizeof(uint32_t)) != cudaSuccess ||
-        cudaMemset(ring[d], 0, SLOTS * 32 * sizeof(uint32_t)) != cudaSuccess) {
-      cudaGetLastError();
-      ring[d] = nullptr;
-      return false;
-    }
-  }
-  const uint32_t slot = next[d].fetch_add(1u) % SLOTS;
-  tc.ctr = ring[d] + slot * 32;                     // 128-B apart
-  return true;
+// Per-launch device state: the dynamic scheduler's claim counter, the split
+// tail's partial workspace and arrival counters, and a fused launch's
+// dependency counters.
+//  * Eager launches: one block per (device, stream).  Launches on one stream
+//    never overlap in global memory (each grid waits for the previous one
+//    before its first global access, PDL included) and every launch leaves
+//    the counters at zero (the last claim resets the claim counter, the last
+//    slice of a split tile its arrival counter; fused counters are zeroed by a
+//    memset before the launch), so the next launch on the stream starts clean.
+//    Launches on different streams never share a block.
+//  * Launches captured into a CUDA graph (cudaStreamIsCapturing): a private
+//    block allocated, zeroed and freed INSIDE the graph (stream-ordered
+//    alloc / memset / free nodes), so every replay of the graph -- on any
+//    stream, beside eager calls or other graphs -- owns its counters.
+// (the earlier device-wide ring could hand one slot to two
+// concurrent launches, and graphs kept per-capture-stream slots.)
+struct LaunchState {
+  uint32_t *ctr = nullptr;      // claim counter (128 B)
+  uint32_t *dep = nullptr;      // fused: [FUSED_PH] phase + [FUSED_PH][MAX_SLAB] slab counters
+  float *ws = nullptr;          // split tail partials: dev_sms x HA x BN floats
+  uint32_t *ws_cnt = nullptr;   // split tail arrival counters (1024)
+  void *graph_block = nullptr;  // captured launch: the private block to free after the kernel
+};
+constexpr size_t CTR_BYTES = 128, DEP_BYTES = (size_t)FUSED_PH * (1 + MAX_SLAB) * sizeof(uint32_t),
+                 WSCNT_BYTES = 1024 * sizeof(uint32_t);
+static size_t ws_bytes_for(int dev) {
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  return (size_t)sms * HA * BN * sizeof(float);
 }
-
-// Split-tail workspace, one per (device, stream): the slices of one launch's
-// tail never exceed one wave (num_sms CTAs x 128 x BN floats), counters are
-// left at zero by the last slice of every tile.
-static bool split_workspace(cudaStream_t stream, int num_sms, float **ws, uint32_t **cnt) {
-  struct Entry { int dev; cudaStream_t st; float *ws; uint32_t *cnt; };
-  static Entry tab[16];
-  static int n = 0;
+static bool capturing(cudaStream_t s) {
+  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(s, &st) != cudaSuccess) { cudaGetLastError(); return false; }
+  return st == cudaStreamCaptureStatusActive;
+}
+// need_ws: the launch splits its tail; need_dep: a fused launch.  Returns false
+// on an allocation failure (nothing enqueued).
+static bool launch_state(cudaStream_t stream, bool need_ws, bool need_dep, LaunchState &ls) {
   int d = 0;
   if (cudaGetDevice(&d) != cudaSuccess) return false;
-  for (int i = 0; i < n; ++i)
-    if (tab[i].dev == d && tab[i].st == stream) { *ws = tab[i].ws; *cnt = tab[i].cnt; return true; }
-  if (n == 16) return false;
-  Entry e{d, stream, nullptr, nullptr};
-  // sized for the whole device: launches may use fewer SMs (Problem::max_sms)
-  int dev_sms = num_sms;
-  if (cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, d) != cudaSuccess) return false;
-  dev_sms = dev_sms > num_sms ? dev_sms : num_sms;
-  const size_t wsb = (size_t)dev_sms * HA * BN * sizeof(float), cb = 1024 * sizeof(uint32_t);
-  if (cudaMalloc(&e.ws, wsb) != cudaSuccess) { cudaGetLastError(); return false; }
-  if (cudaMalloc(&e.cnt, cb) != cudaSuccess || cudaMemset(e.cnt, 0, cb) != cudaSuccess) {
-    cudaGetLastError(); cudaFree(e.ws); return false;
+  if (capturing(stream)) {
+    const size_t wsb = need_ws ? ws_bytes_for(d) : 0;
+    const size_t bytes = CTR_BYTES + DEP_BYTES + WSCNT_BYTES + wsb;
+    void *blk = nullptr;
+    if (cudaMallocAsync(&blk, bytes, stream) != cudaSuccess) { cudaGetLastError(); return false; }
+    // (the partials need no zeroing: every slice writes its own before the count)
+    if (cudaMemsetAsync(blk, 0, CTR_BYTES + DEP_BYTES + WSCNT_BYTES, stream) != cudaSuccess) {
+      cudaGetLastError(); cudaFreeAsync(blk, stream); return false;
+    }
+    uint8_t *p = static_cast<uint8_t *>(blk);
+    ls.ctr = reinterpret_cast<uint32_t *>(p);
+    ls.dep = reinterpret_cast<uint32_t *>(p + CTR_BYTES);
+    ls.ws_cnt = reinterpret_cast<uint32_t *>(p + CTR_BYTES + DEP_BYTES);
+    ls.ws = need_ws ? reinterpret_cast<float *>(p + CTR_BYTES + DEP_BYTES + WSCNT_BYTES) : nullptr;
+    ls.graph_block = blk;
+    return true;
   }
-  tab[n++] = e;
-  *ws = e.ws; *cnt = e.cnt;
+  struct Key { int dev; cudaStream_t st; };
+  struct Entry { Key k; LaunchState s; };
+  static std::vector<Entry> tab;
+  static std::mutex mu;
+  std::lock_guard<std::mutex> lk(mu);
+  Entry *e = nullptr;
+  for (Entry &x : tab)
+    if (x.k.dev == d && x.k.st == stream) { e = &x; break; }
+  if (!e) { tab.push_back(Entry{Key{d, stream}, LaunchState{}}); e = &tab.back(); }
+  LaunchState &st = e->s;
+  auto zalloc = [](void **p, size_t bytes, bool zero) {
+    if (cudaMalloc(p, bytes) != cudaSuccess) { cudaGetLastError(); *p = nullptr; return false; }
+    if (zero && cudaMemset(*p, 0, bytes) != cudaSuccess) { cudaGetLastError(); cudaFree(*p); *p = nullptr; return false; }
+    return true;
+  };
+  if (!st.ctr && !zalloc(reinterpret_cast<void **>(&st.ctr), CTR_BYTES, true)) return false;
+  if (need_dep && !st.dep && !zalloc(reinterpret_cast<void **>(&st.dep), DEP_BYTES, true)) return false;
+  if (need_ws && !st.ws) {
+    if (!zalloc(reinterpret_cast<void **>(&st.ws_cnt), WSCNT_BYTES, true)) return false;
+    if (!zalloc(reinterpret_cast<void **>(&st.ws), ws_bytes_for(d), false)) {
+      cudaFree(st.ws_cnt); st.ws_cnt = nullptr; return false;
+    }
+  }
+  ls = st;
+  ls.graph_block = nullptr;
   return true;
+}
+static void release_state(cudaStream_t stream, const LaunchState &ls) {
+  if (ls.graph_block) cudaFreeAsync(ls.graph_block, stream);
 }
 
 // Wave quantisation: with T tiles on U producers the last wave holds
@@ -1310,7 +1353,7 @@ static bool split_workspace(cudaStream_t stream, int num_sms, float **ws, uint32
 // keeps >= 8 k-blocks (its partial write-back costs about what ~3 k-blocks
 // of MMA do).
 template <int CG>
-static void plan_split(TcParams &prm, int num_sms, cudaStream_t stream) {
+static void plan_split(TcParams &prm, int num_sms) {
   const Problem &P = prm.ph[0].P;
   const int64_t nb = P.nbatch > 1 ? P.nbatch : 1;
   const int64_t tiles_per = Tiles<Geo<CG>::TM, BN>::count(P), T = tiles_per * nb;
@@ -1333,7 +1376,6 @@ static void plan_split(TcParams &prm, int num_sms, cudaStream_t stream) {
   }
   S = imin(S, min_kb / 8);
   if (S < 2) return;
-  if (!split_workspace(stream, num_sms, &prm.ws, &prm.ws_cnt)) return;
   prm.khead = head;
   prm.ksplit = (int32_t)S;
   prm.nitems = head + R * S;
@@ -1353,18 +1395,21 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
   prm.nphase = 1;
   prm.ph[0].P = P0;
   prm.ph[0].P.dbg = debug_bits();
+  if (prm.ph[0].P.kc <= 0) prm.ph[0].P.kc = 4;
   const int cg = choose_cg(prm.ph[0].P, num_sms);
   const bool dyn = opt(BLAS3_OPT_TC_STATIC) == 0;
-  if (cg == 2) plan_split<2>(prm, num_sms, stream); else plan_split<1>(prm, num_sms, stream);
-  if (dyn) {
-    const int64_t tiles = prm.nitems;
-    TileCounter tc;
-    // claims: (items - producers) beyond the first wave + one failing claim per producer
-    if (tiles > 0) {
-      if (!tile_counter(tc)) return -1;
-      prm.tile_ctr = tc.ctr;
-      prm.tile_claims = (uint32_t)tiles;
+  if (cg == 2) plan_split<2>(prm, num_sms); else plan_split<1>(prm, num_sms);
+  const bool split = prm.ksplit > 1;
+  LaunchState ls;
+  if ((dyn || split) && prm.nitems > 0) {
+    if (!launch_state(stream, split, false, ls)) {
+      if (!split) return -1;
+      prm.nitems = prm.khead = prm.ph[0].ntiles; prm.ksplit = 1;      // no workspace: no split
+      if (dyn && !launch_state(stream, false, false, ls)) return -1;
     }
+    if (prm.ksplit > 1) { prm.ws = ls.ws; prm.ws_cnt = ls.ws_cnt; }
+    // claims: (items - producers) beyond the first wave + one failing claim per producer
+    if (dyn) { prm.tile_ctr = ls.ctr; prm.tile_claims = (uint32_t)prm.nitems; }
   }
   // diagnostics: BLAS3_TRACE=1 prints CTA 0's phase timeline (synchronises)
   static int trace = -1;
@@ -1375,7 +1420,9 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
     cudaMemsetAsync(tbuf, 0, 16 * sizeof(unsigned long long), stream);
     prm.trace = tbuf;
   }
-  const int rc = cg == 2 ? launch_cg<2>(prm, stream, num_sms) : launch_cg<1>(prm, stream, num_sms);
+  const int rc = cg == 2 ? launch_cg<2>(prm, stream, num_sms, ls.graph_block == nullptr)
+                         : launch_cg<1>(prm, stream, num_sms, ls.graph_block == nullptr);
+  release_state(stream, ls);
   if (trace && rc == 0) {
     unsigned long long h[16];
     cudaStreamSynchronize(stream);
@@ -1391,25 +1438,6 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
   return rc;
 }
 
-// Fused-launch dependency counters, one zeroed block per (device, stream).
-static uint32_t *dep_counters(cudaStream_t stream) {
-  struct Entry { int dev; cudaStream_t st; uint32_t *p; };
-  static Entry tab[32];
-  static int n = 0;
-  int d = 0;
-  if (cudaGetDevice(&d) != cudaSuccess) return nullptr;
-  for (int i = 0; i < n; ++i)
-    if (tab[i].dev == d && tab[i].st == stream) return tab[i].p;
-  if (n == 32) return nullptr;
-  Entry e{d, stream, nullptr};
-  if (cudaMalloc(&e.p, (size_t)FUSED_PH * (1 + MAX_SLAB) * sizeof(uint32_t)) != cudaSuccess) {
-    cudaGetLastError();
-    return nullptr;
-  }
-  tab[n++] = e;
-  return e.p;
-}
-
 int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int num_sms) {
   if (nph < 1 || nph > FUSED_PH) return -1;
   static TcFusedParams prm;               // host staging (the launch copies it)
@@ -1423,6 +1451,7 @@ int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int 
     PhaseDesc &ph = prm.ph[p];
     ph.P = phases[p].P;
     ph.P.dbg = debug_bits();
+    if (ph.P.kc <= 0) ph.P.kc = 4;
     if (!tc_eligible(ph.P) || ph.P.max_sms) return -1;
     const int64_t nb = ph.P.nbatch > 1 ? ph.P.nbatch : 1;
     ph.tiles_per = TL::count(ph.P);
@@ -1434,7 +1463,6 @@ int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int 
     ph.slab_m = phases[p].slab_m;
     ph.slab_cnt = (int32_t)(phases[p].slab_m ? cdiv(ph.P.N, BN) : cdiv(ph.P.M, Geo<CG>::TM));
     if ((ph.dep_full | ph.dep_slab) >> p) return -1;        // dependencies point backwards only
-    if (ph.P.c_tri != 0 || nb > 1 ? false : false) return -1;
     for (int s = 0; s < ph.P.nseg; ++s)                      // SYM diagonal merges read global memory
       if (ph.P.seg[s].a.kind == OP_SYM || ph.P.seg[s].b.kind == OP_SYM) return -1;
     const int64_t nslab = phases[p].slab_m ? cdiv(ph.P.M, Geo<CG>::TM) : cdiv(ph.P.N, BN);
@@ -1444,15 +1472,13 @@ int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int 
   prm.nitems = item;
   prm.khead = item;
   prm.ksplit = 1;
-  prm.dep_ctr = dep_counters(stream);
-  if (!prm.dep_ctr) return -1;
-  if (cudaMemsetAsync(prm.dep_ctr, 0, (size_t)FUSED_PH * (1 + MAX_SLAB) * sizeof(uint32_t), stream) !=
-      cudaSuccess) return -1;
-  TileCounter tc;
-  const int64_t units = imin(item, (int64_t)(num_sms / CG));
   if (item == 0) return 0;
-  if (!tile_counter(tc)) return -1;
-  prm.tile_ctr = tc.ctr;
+  LaunchState ls;
+  if (!launch_state(stream, false, true, ls)) return -1;
+  prm.dep_ctr = ls.dep;
+  if (cudaMemsetAsync(prm.dep_ctr, 0, DEP_BYTES, stream) != cudaSuccess) { release_state(stream, ls); return -1; }
+  const int64_t units = imin(item, (int64_t)(num_sms / CG));
+  prm.tile_ctr = ls.ctr;
   prm.tile_claims = (uint32_t)(item + units);
   // diagnostics: BLAS3_TRACE=2 prints each phase's [first start, last end] (synchronises)
   static int trace = -1;
@@ -1482,6 +1508,7 @@ int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int 
   }
   // no PDL: the counters' memset node precedes this grid on the stream
   const int rc = launch_cg<CG>(prm, stream, num_sms, false);
+  release_state(stream, ls);
   if (trace && rc == 0) {
     unsigned long long h[2 * FUSED_PH];
     cudaStreamSynchronize(stream);

@@ -14,7 +14,8 @@ import numpy as np
 import pytest
 
 import blas3_inputs as gen
-from check import TOL_NW, e_nw, f64, fro, to_dev, to_host, tol_rel, tri_full
+from check import (TOL_NW, e_nw, e_rel, f64, fro, rel_bound, sel_f32, sym_f32, to_dev, to_host,
+                   tri_f32, tri_full)
 
 pytestmark = pytest.mark.gpu
 AL, BE = 1.5, 0.5
@@ -45,7 +46,8 @@ def test_cfg2_sgemm_ssymm_sweep(b3, oracle_mod, n):
         ref = oracle_mod.sgemm(ta, tb, AL, A, B, BE, C, sel=sel)
         opB_S = B[:, sel] if tb == "N" else B[sel, :]
         assert e_nw(got, ref, AL * fro(A) * fro(opB_S) + BE * fro(C[:, sel])) <= TOL_NW, (ta, tb)
-        assert fro(f64(got) - ref) / fro(ref) <= tol_rel(n, "3xtf32"), (ta, tb)
+        f32 = sel_f32("sgemm", (ta, tb, AL, A, B, BE, C), sel)
+        assert e_rel(got, ref) <= rel_bound(f32, ref), (ta, tb)
     Af = f64(A)
     for side, uplo in itertools.product("LR", "LU"):
         dC = to_dev(C)
@@ -56,6 +58,8 @@ def test_cfg2_sgemm_ssymm_sweep(b3, oracle_mod, n):
         scale = (AL * fro(S) * fro(B[:, sel]) if side == "L" else AL * fro(B) * fro(S[:, sel])) \
             + BE * fro(C[:, sel])
         assert e_nw(got, ref, scale) <= TOL_NW, (side, uplo)
+        f32 = sel_f32("ssymm", (side, uplo, AL, A, B, BE, C, sym_f32(A, uplo)), sel)
+        assert e_rel(got, ref) <= rel_bound(f32, ref), (side, uplo)
 
 
 @pytest.fixture(scope="module")
@@ -81,6 +85,8 @@ def test_cfg3_strmm_strsm_4096(b3, oracle_mod, cfg3, side, uplo, ta, diag):
     ref = oracle_mod.strmm(side, uplo, ta, diag, AL, A, B, sel=sel)
     scale = AL * fro(opT) * fro(B[:, sel]) if side == "L" else AL * fro(B) * fro(opT[:, sel])
     assert e_nw(got, ref, scale) <= TOL_NW
+    f32 = sel_f32("strmm", (side, ta, AL, tri_f32(A, uplo, diag), B), sel)
+    assert e_rel(got, ref) <= rel_bound(f32, ref)
     # STRSM: residual + forward error on the sample (rows for side=R)
     dX = to_dev(B)
     b3.strsm(side, uplo, ta, diag, AL, dA, dX)
@@ -129,4 +135,6 @@ def test_cfg4_tall_skinny_syrk_syr2k(b3, oracle_mod, cfg4, two, uplo, trans):
     scale = (AL * (fro(A) * fro(opB_S) + fro(B) * fro(opA_S)) if two else AL * fro(A) * fro(opA_S)) \
         + BE * fro(C[:, sel][mask])
     assert e_nw(got[mask], ref[mask], scale) <= TOL_NW
+    f32 = sel_f32("ssyr2k" if two else "ssyrk", (uplo, trans, AL, A, B if two else None, BE, C), sel)
+    assert e_rel(got[mask], ref[mask]) <= rel_bound(f32[mask], ref[mask])
     assert np.array_equal(got[~mask].view(np.uint32), C[:, sel][~mask].view(np.uint32))

@@ -1,21 +1,30 @@
 """Parity at BASELINE.json's full size, in the configuration bench.py times.
 
-N = K = 8192, alpha = 1.5, beta = 0.5, the bench's seeded inputs and variants
-(sgemm NN, ssymm LL, ssyrk LN, ssyr2k LN, strmm LLNN, strsm LLNN, plus the
-transposed / right-side / upper variants below).  The fp64 oracle computes a
-sample of output columns exactly (columns are independent), and the metrics
-are restricted to that sample consistently.
+N = K = 8192, alpha = 1.5, beta = 0.5, the bench's seeded inputs, and EVERY
+variant of every routine at that size: SGEMM x 4 transa/transb, SSYMM x 4
+side/uplo (default route and the staged route with GM_map off), SSYRK and
+SSYR2K x 4 uplo/trans (configs[3] at N = K = 8192), STRMM and STRSM x 16
+side/uplo/trans/diag (configs[2] at 8192).  The fp64 oracle computes a sample
+of output columns exactly (columns are independent; rows for STRSM side=R),
+and the metrics are restricted to that sample consistently:
+normwise <= 1e-5 (north star), the output-relative diagnostic
+max(4 * e_rel(plain fp32), 2e-6) (check.rel_bound), STRSM
+residual <= 1e-5 sqrt(N) and forward error <= 1e-5.
 """
+import itertools
+
 import numpy as np
 import pytest
 
 import blas3_inputs as gen
-from check import TOL_NW, e_nw, f64, fro, to_dev, to_host, tol_rel
+from check import (TOL_NW, e_nw, e_rel, f64, fro, op, rel_bound, sel_f32, sym_f32, to_dev, to_host,
+                   tri_f32)
 
 pytestmark = pytest.mark.gpu
 
 N = 8192
 AL, BE = 1.5, 0.5
+NSEL = 24
 
 
 @pytest.fixture(scope="module")
@@ -30,112 +39,145 @@ def env():
     oracle.build()
     b3.set_math_mode("3xtf32")
     A = gen.uniform(N, N, "bench-A")
-    T = gen.triangular_dd(N, "L", "N", "bench-T")
     B = gen.uniform(N, N, "bench-B", 0)
     C = gen.uniform(N, N, "bench-C", 0)
-    sel = gen.sample_indices(N, 24, "large-parity")
-    return b3, oracle, A, T, B, C, sel, {k: to_dev(v) for k, v in dict(A=A, T=T, B=B).items()}
+    sel = gen.sample_indices(N, NSEL, "large-parity")
+    return dict(b3=b3, oracle=oracle, A=A, B=B, C=C, sel=sel, dA=to_dev(A), dB=to_dev(B))
+
+
+_TRI = {}
+
+
+def tri(uplo, diag):
+    """The bench's T (lower, diag N) and the other three stored forms."""
+    key = (uplo, diag)
+    if key not in _TRI:
+        _TRI.clear()                     # one 256 MiB triangle (+ device copy) at a time
+        T = gen.triangular_dd(N, "L", "N", "bench-T") if key == ("L", "N") else \
+            gen.triangular_dd(N, uplo, diag, "large-T")
+        _TRI[key] = (T, to_dev(T), tri_f32(T, uplo, diag))
+    return _TRI[key]
 
 
 def _tc_used(b3, before):
     assert b3.launch_count("tc") > before, "expected the tcgen05 route"
 
 
-@pytest.mark.parametrize("ta,tb", [("N", "N"), ("T", "N"), ("N", "T")])
-def test_sgemm_8192(env, ta, tb):
-    b3, oracle, A, T, B, C, sel, d = env
-    before = b3.launch_count("tc")
-    dC = to_dev(C)
-    b3.sgemm(ta, tb, AL, d["A"], d["B"], BE, dC)
-    got = to_host(dC)[:, sel]
-    _tc_used(b3, before)
-    ref = oracle.sgemm(ta, tb, AL, A, B, BE, C, sel=sel)
-    opB_S = B[:, sel] if tb == "N" else B[sel, :]
-    scale = AL * fro(A) * fro(opB_S) + BE * fro(C[:, sel])
-    assert e_nw(got, ref, scale) <= TOL_NW
-    assert fro(f64(got) - ref) / fro(ref) <= tol_rel(N, "3xtf32")
-
-
-@pytest.mark.parametrize("side,uplo", [("L", "L"), ("R", "U")])
-def test_ssymm_8192(env, side, uplo):
-    b3, oracle, A, T, B, C, sel, d = env
-    dC = to_dev(C)
-    b3.ssymm(side, uplo, AL, d["A"], d["B"], BE, dC)     # only A's uplo triangle is read
-    got = to_host(dC)[:, sel]
-    ref = oracle.ssymm(side, uplo, AL, A, B, BE, C, sel=sel)
-    Af = f64(A)
-    S = (np.tril(Af) + np.tril(Af, -1).T) if uplo == "L" else (np.triu(Af) + np.triu(Af, 1).T)
-    # side=L: column j of C uses B(:,j); side=R: column j uses Asym(:,j)
-    scale = (AL * fro(S) * fro(B[:, sel]) if side == "L" else AL * fro(B) * fro(S[:, sel])) \
-        + BE * fro(C[:, sel])
-    assert e_nw(got, ref, scale) <= TOL_NW
-
-
-@pytest.mark.parametrize("two", [False, True])
-@pytest.mark.parametrize("uplo,trans", [("L", "N"), ("U", "T")])
-def test_syrk_syr2k_8192(env, two, uplo, trans):
-    b3, oracle, A, T, B, C, sel, d = env
-    dC = to_dev(C)
-    if two:
-        b3.ssyr2k(uplo, trans, AL, d["A"], d["B"], BE, dC)
-        ref = oracle.ssyr2k(uplo, trans, AL, A, B, BE, C, sel=sel)
-    else:
-        b3.ssyrk(uplo, trans, AL, d["A"], BE, dC)
-        ref = oracle.ssyrk(uplo, trans, AL, A, BE, C, sel=sel)
-    got = to_host(dC)[:, sel]
+def _col_mask(sel, uplo):
     mask = np.zeros((N, len(sel)), bool)
     for t, j in enumerate(sel):
         if uplo == "L":
             mask[j:, t] = True
         else:
             mask[: j + 1, t] = True
+    return mask
+
+
+@pytest.mark.parametrize("ta,tb", list(itertools.product("NT", "NT")))
+def test_sgemm_8192(env, ta, tb):
+    b3, A, B, C, sel = env["b3"], env["A"], env["B"], env["C"], env["sel"]
+    before = b3.launch_count("tc")
+    dC = to_dev(C)
+    b3.sgemm(ta, tb, AL, env["dA"], env["dB"], BE, dC)
+    got = to_host(dC)[:, sel]
+    _tc_used(b3, before)
+    ref = env["oracle"].sgemm(ta, tb, AL, A, B, BE, C, sel=sel)
+    opB_S = B[:, sel] if tb == "N" else B[sel, :]
+    scale = AL * fro(A) * fro(opB_S) + BE * fro(C[:, sel])
+    assert e_nw(got, ref, scale) <= TOL_NW
+    assert e_rel(got, ref) <= rel_bound(sel_f32("sgemm", (ta, tb, AL, A, B, BE, C), sel), ref)
+
+
+@pytest.mark.parametrize("gm_map", [-1, 0])
+@pytest.mark.parametrize("side,uplo", list(itertools.product("LR", "LU")))
+def test_ssymm_8192(env, side, uplo, gm_map):
+    """gm_map=-1: the default route; 0: the staged route (sym(A) merged while
+    staging, never materialised)."""
+    b3, A, B, C, sel = env["b3"], env["A"], env["B"], env["C"], env["sel"]
+    dC = to_dev(C)
+    with b3.options(gm_map=gm_map):
+        b3.ssymm(side, uplo, AL, env["dA"], env["dB"], BE, dC)   # only A's uplo triangle is read
+    got = to_host(dC)[:, sel]
+    ref = env["oracle"].ssymm(side, uplo, AL, A, B, BE, C, sel=sel)
+    S = sym_f32(A, uplo)
+    # side=L: column j of C uses B(:,j); side=R: column j uses Asym(:,j)
+    scale = (AL * fro(S) * fro(B[:, sel]) if side == "L" else AL * fro(B) * fro(S[:, sel])) \
+        + BE * fro(C[:, sel])
+    assert e_nw(got, ref, scale) <= TOL_NW
+    assert e_rel(got, ref) <= rel_bound(sel_f32("ssymm", (side, uplo, AL, A, B, BE, C, S), sel), ref)
+
+
+@pytest.mark.parametrize("two", [False, True])
+@pytest.mark.parametrize("uplo,trans", list(itertools.product("LU", "NT")))
+def test_syrk_syr2k_8192(env, two, uplo, trans):
+    b3, A, B, C, sel = env["b3"], env["A"], env["B"], env["C"], env["sel"]
+    dC = to_dev(C)
+    if two:
+        b3.ssyr2k(uplo, trans, AL, env["dA"], env["dB"], BE, dC)
+        ref = env["oracle"].ssyr2k(uplo, trans, AL, A, B, BE, C, sel=sel)
+    else:
+        b3.ssyrk(uplo, trans, AL, env["dA"], BE, dC)
+        ref = env["oracle"].ssyrk(uplo, trans, AL, A, BE, C, sel=sel)
+    got = to_host(dC)[:, sel]
+    mask = _col_mask(sel, uplo)
     opA_S = A[sel, :] if trans == "N" else A[:, sel]
     opB_S = B[sel, :] if trans == "N" else B[:, sel]
     scale = (AL * (fro(A) * fro(opB_S) + fro(B) * fro(opA_S)) if two else AL * fro(A) * fro(opA_S)) \
         + BE * fro(C[:, sel][mask])
     assert e_nw(got[mask], ref[mask], scale) <= TOL_NW
+    f32 = sel_f32("ssyr2k" if two else "ssyrk", (uplo, trans, AL, A, B if two else None, BE, C), sel)
+    assert e_rel(got[mask], ref[mask]) <= rel_bound(f32[mask], ref[mask])
     assert np.array_equal(got[~mask].view(np.uint32), C[:, sel][~mask].view(np.uint32))
 
 
-@pytest.mark.parametrize("side,ta", [("L", "N"), ("R", "T")])
-def test_strmm_8192(env, side, ta):
-    b3, oracle, A, T, B, C, sel, d = env
+V16 = list(itertools.product("LU", "NU", "LR", "NT"))     # (uplo, diag) outer: one T at a time
+
+
+@pytest.mark.parametrize("uplo,diag,side,ta", V16)
+def test_strmm_8192(env, uplo, diag, side, ta):
+    b3, B, sel = env["b3"], env["B"], env["sel"]
+    T, dT, T32 = tri(uplo, diag)
     dX = to_dev(B)
-    b3.strmm(side, "L", ta, "N", AL, d["T"], dX)
+    b3.strmm(side, uplo, ta, diag, AL, dT, dX)
     got = to_host(dX)[:, sel]
-    ref = oracle.strmm(side, "L", ta, "N", AL, T, B, sel=sel)
-    Tf = np.tril(np.nan_to_num(f64(T)))
-    opT = Tf if ta == "N" else Tf.T
+    ref = env["oracle"].strmm(side, uplo, ta, diag, AL, T, B, sel=sel)
+    opT = op(T32, ta)
     scale = AL * fro(opT) * fro(B[:, sel]) if side == "L" else AL * fro(B) * fro(opT[:, sel])
     assert e_nw(got, ref, scale) <= TOL_NW
+    assert e_rel(got, ref) <= rel_bound(sel_f32("strmm", (side, ta, AL, T32, B), sel), ref)
 
 
-@pytest.mark.parametrize("ta", ["N", "T"])
-def test_strsm_8192(env, ta):
-    b3, oracle, A, T, B, C, sel, d = env
+@pytest.mark.parametrize("uplo,diag,side,ta", V16)
+def test_strsm_8192(env, uplo, diag, side, ta):
+    b3, B, sel = env["b3"], env["B"], env["sel"]
+    T, dT, T32 = tri(uplo, diag)
     dX = to_dev(B)
-    b3.strsm("L", "L", ta, "N", AL, d["T"], dX)
-    X = f64(to_host(dX)[:, sel])
-    Tf = np.tril(np.nan_to_num(f64(T)))
-    opT = Tf if ta == "N" else Tf.T
-    resid = fro(opT @ X - AL * f64(B[:, sel])) / (fro(opT) * fro(X))
+    b3.strsm(side, uplo, ta, diag, AL, dT, dX)
+    X = to_host(dX)
+    opT = f64(op(T32, ta))
+    if side == "L":
+        Xs = f64(X[:, sel])
+        resid = fro(opT @ Xs - AL * f64(B[:, sel])) / (fro(opT) * fro(Xs))
+    else:
+        Xs = f64(X[sel, :])
+        resid = fro(Xs @ opT - AL * f64(B[sel, :])) / (fro(opT) * fro(Xs))
     assert resid <= 1e-5 * np.sqrt(N)
-    ref = oracle.strsm("L", "L", ta, "N", AL, T, B, sel=sel)
-    assert fro(X - ref) / fro(ref) <= 1e-5
+    ref = env["oracle"].strsm(side, uplo, ta, diag, AL, T, B, sel=sel)
+    assert fro(Xs - ref) / fro(ref) <= 1e-5
 
 
 @pytest.mark.parametrize("ta,tb", [("N", "N"), ("T", "N")])
 def test_sgemm_8192_tf32_bf16x(env, ta, tb):
     """The opt-in TF32+BF16X mode (packed bf16 cross terms) at the bench size."""
-    b3, oracle, A, T, B, C, sel, d = env
+    b3, A, B, C, sel = env["b3"], env["A"], env["B"], env["C"], env["sel"]
     b3.set_math_mode("tf32_bf16x")
     try:
         dC = to_dev(C)
-        b3.sgemm(ta, tb, AL, d["A"], d["B"], BE, dC)
+        b3.sgemm(ta, tb, AL, env["dA"], env["dB"], BE, dC)
         got = to_host(dC)[:, sel]
     finally:
         b3.set_math_mode("3xtf32")
-    ref = oracle.sgemm(ta, tb, AL, A, B, BE, C, sel=sel)
+    ref = env["oracle"].sgemm(ta, tb, AL, A, B, BE, C, sel=sel)
     scale = AL * fro(A) * fro(B[:, sel]) + BE * fro(C[:, sel])
     assert e_nw(got, ref, scale) <= TOL_NW
-    assert fro(f64(got) - ref) / fro(ref) <= tol_rel(N, "tf32_bf16x")
+    assert e_rel(got, ref) <= rel_bound(sel_f32("sgemm", (ta, tb, AL, A, B, BE, C), sel), ref)
