@@ -208,10 +208,18 @@ int blas3_get_math_mode(void);
  *   BLAS3_OPT_TC_KC        [BLAS3_TC_KC]    tcgen05 path: k-blocks (32 deep) summed in
  *                          one TMEM partial before it is folded into the
  *                          round-to-nearest register sum (Q24): power
- *                          of 2 in [1, 64], default 4 (K = 128).  The tensor
+ *                          of 2 in [1, 64], default 2 (K = 64).  The tensor
  *                          core's accumulator truncates on every UMMA add, so
- *                          the output-relative error grows with this value
- *                          (measured: 16 -> 3.9e-6, 4 -> fp32 class)
+ *                          the output-relative error grows with this value:
+ *                          ~4e-8 per add, coherent on same-sign data (3 adds per
+ *                          8-deep k-step); measured e_rel on U(-1,1) SGEMM
+ *                          16 -> 3.9e-6, 4 -> 1.1e-6, 2 -> 6.8e-7, and 2.6e-6 at
+ *                          4 on an all-positive (SYRK diagonal) sum
+ *   BLAS3_OPT_TC_TMA_STORE [BLAS3_TC_TMA_STORE] tcgen05 epilogue: 1 (default) the
+ *                          output tile leaves through shared memory as TMA
+ *                          tensor stores (32-row x 8-column boxes, 128-B rows),
+ *                          when C is 16-B aligned with ldc % 4 == 0; 0 per-thread
+ *                          coalesced 4-B stores
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */
@@ -223,7 +231,7 @@ enum {
     BLAS3_OPT_TRSM_RESERVE = 12, BLAS3_OPT_TRSM_GEO_LEAF = 13, BLAS3_OPT_TRSM_FUSED = 14,
     BLAS3_OPT_TRSM_FIRST_YM = 15, BLAS3_OPT_TRSM_FIRST_FUSED = 16, BLAS3_OPT_TRSM_FIRST_SPLIT = 17,
     BLAS3_OPT_TRSM_FIRST_ALL = 18, BLAS3_OPT_TC_RASTER = 19, BLAS3_OPT_TC_KC = 20,
-    BLAS3_OPT_COUNT = 21
+    BLAS3_OPT_TC_TMA_STORE = 21, BLAS3_OPT_COUNT = 22
 };
 int blas3_set_option(int key, int64_t value);
 int64_t blas3_get_option(int key);

@@ -87,6 +87,9 @@ struct Problem {
   int32_t raster_gm;
   // tcgen05 path: k-blocks per TMEM partial (power of 2; BLAS3_OPT_TC_KC)
   int32_t kc;
+  // tcgen05 path: tensor-map slot of Cout for the bulk (TMA) epilogue
+  // stores, or -1 (scalar coalesced stores); set at launch
+  int32_t c_map;
 };
 
 HD int64_t batch_off(const BatchStride &s, int64_t b, int64_t per) {

@@ -67,7 +67,7 @@ constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;       // 640
 constexpr int EPI_REGS = 144, OTHER_REGS = 64;   // 36864 + 24576 = 61440
 // Chunked accumulation: the tensor core's fp32 accumulator truncates on every
 // UMMA add (Q24), so a TMEM partial only ever sums Problem::kc
-// k-blocks (BLAS3_OPT_TC_KC, default 4: K = 128) before the epilogue folds it
+// k-blocks (BLAS3_OPT_TC_KC, default 2: K = 64) before the epilogue folds it
 // into a register running sum with round-to-nearest adds; the two TMEM
 // buffers ping-pong per chunk.
 constexpr int EC = 16;                            // epilogue column group
@@ -78,7 +78,9 @@ constexpr int TQ = 4;
 constexpr int TR_THREADS = NUM_TR_WARPS * 32;
 constexpr int EPI_THREADS = NUM_EPI_WARPS * 32;
 constexpr int TMEM_COLS = 512;             // 2 accumulators x BN columns
-constexpr int MAX_MAPS = 8;
+constexpr int MAX_MAPS = 10;                 // 2 segments x 2 operands x 2 views + C
+// epilogue staging: per epilogue warp two 32-row x 8-column fp32 boxes (TMA store)
+constexpr int EPI_GW = 8, EPI_BOX = 32 * EPI_GW;
 constexpr int LAYOUT_K = 0, LAYOUT_MN = 1;
 
 // A work item: the tile (batch member b, tile t at m0, n0) and the range
@@ -123,7 +125,11 @@ struct Geo {
     uint32_t tmem_base;
     uint32_t split_last;     // epilogue: this CTA's slice of a split tile is the last one
   };
-  static constexpr size_t SMEM = sizeof(RawBuf) * RS + sizeof(LoBuf) * LS + sizeof(Barriers) + 1024;
+  struct alignas(1024) EpiStage {
+    float box[NUM_EPI_WARPS][2][EPI_BOX];   // D staging for the TMA tensor stores
+  };
+  static constexpr size_t SMEM =
+      sizeof(RawBuf) * RS + sizeof(LoBuf) * LS + sizeof(EpiStage) + sizeof(Barriers) + 1024;
 };
 
 // One phase of a launch: a Problem, the work items it owns and, in a FUSED
@@ -172,8 +178,9 @@ struct TcParamsT {
   int32_t st_phase;
 };
 using TcParams = TcParamsT<1, MAX_MAPS>;
-constexpr int FUSED_PH = 24, FUSED_MAPS = 48;
+constexpr int FUSED_PH = 24, FUSED_MAPS = 72;
 using TcFusedParams = TcParamsT<FUSED_PH, FUSED_MAPS>;
+static_assert(sizeof(TcFusedParams) <= 32764, "kernel parameter block exceeds 32764 bytes");
 
 // %globaltimer (ns) of the first occurrence of a phase in CTA 0 (diagnostics)
 #define BLAS3_TRACE(i)                                                              \
@@ -606,7 +613,9 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
   uint8_t *smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   RawBuf *raw = reinterpret_cast<RawBuf *>(smem);
   LoBuf *lo = reinterpret_cast<LoBuf *>(smem + sizeof(RawBuf) * RS);
-  Barriers *bars = reinterpret_cast<Barriers *>(smem + sizeof(RawBuf) * RS + sizeof(LoBuf) * LS);
+  float *epi_stage = reinterpret_cast<float *>(smem + sizeof(RawBuf) * RS + sizeof(LoBuf) * LS);
+  Barriers *bars = reinterpret_cast<Barriers *>(smem + sizeof(RawBuf) * RS + sizeof(LoBuf) * LS +
+                                                sizeof(typename G::EpiStage));
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const uint32_t rank = (CG == 2) ? ptx::cluster_ctarank() : 0;
   const int64_t cid = blockIdx.x / CG, ncl = gridDim.x / CG;
@@ -954,7 +963,8 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
     const int q = warp & 3;                     // TMEM lane quarter of this warp
     const int half = (warp - WARP_EPI0) >> 2;   // which 128 of the 256 columns
     constexpr int NG = BN / 2 / EC;             // column groups per thread (8)
-    uint32_t cc = 0, qi = 0;
+    uint32_t cc = 0, qi = 0, ebox = 0;
+    float *box0 = epi_stage + (warp - WARP_EPI0) * 2 * EPI_BOX;
     for (;;) {
       const Work w = next_work(qi, 5, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
       if (w.tb < 0) break;
@@ -1048,6 +1058,56 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
       constexpr int SG = 8;
       if (none) {
         // nothing of this warp's 32 x 128 block is referenced (ragged edge)
+      } else if (full && P.c_map >= 0) {
+        // ---- bulk stores (NS "coalesced 128-bit epilogue stores"; DESIGN A6):
+        // the warp's whole 32 x 128 block is valid (ragged-edge and
+        // uplo-cut warps take the predicated path below).  Per group of 8
+        // columns the warp forms D = alpha*S + beta*C for its 32 rows in a
+        // 1 KiB shared box (column-major: the thread's row is the lane, so the
+        // 8 shared stores are conflict-free) and ONE lane writes the box with
+        // a TMA tensor store (128-B rows).  Two boxes per warp alternate:
+        // forming the next group overlaps the previous store's read of shared
+        // memory.  C (beta != 0) is read one group ahead, coalesced.
+        const int32_t rw0 = (int32_t)(m0 + HA * rank + q * 32), cb = (int32_t)cbase;
+        const int32_t bj = (int32_t)(w.b % per), bg = (int32_t)(w.b / per);
+        const uint32_t box_s = ptx::smem_u32(box0) + lane * 4;
+        constexpr int NGW = BN / 2 / EPI_GW;
+        const bool l0 = lane == 0;
+        const CUtensorMap *cmap = &prm.maps[P.c_map];
+        // one group: box <- S[g*8 .. g*8+7] (alpha/beta already applied), TMA store
+        auto put = [&](int g) {
+          const uint32_t box = box_s + (ebox & 1) * (EPI_BOX * 4);
+          ptx::bulk_wait_group_read1_if(l0);         // the store that used this box has read it
+          __syncwarp();
+#pragma unroll
+          for (int j = 0; j < EPI_GW; ++j) ptx::st_shared_f32(box + j * 128, S[g * EPI_GW + j]);
+          ptx::fence_proxy_async_smem();
+          __syncwarp();
+          ptx::tma_store_4d_commit_if(l0, cmap, box - lane * 4, rw0, cb + g * EPI_GW, bj, bg);
+          ++ebox;
+        };
+        if (be != 0.f) {
+          float cv[EPI_GW];
+#pragma unroll
+          for (int j = 0; j < EPI_GW; ++j) { cv[j] = ptx::ld_cs(cp); cp += ldi; }
+#pragma unroll
+          for (int g = 0; g < NGW; ++g) {
+#pragma unroll
+            for (int j = 0; j < EPI_GW; ++j) S[g * EPI_GW + j] = fmaf(be, cv[j], al * S[g * EPI_GW + j]);
+            if (g + 1 < NGW) {
+#pragma unroll
+              for (int j = 0; j < EPI_GW; ++j) { cv[j] = ptx::ld_cs(cp); cp += ldi; }
+            }
+            if (st_on) put(g);
+          }
+        } else {
+#pragma unroll
+          for (int g = 0; g < NGW; ++g) {
+#pragma unroll
+            for (int j = 0; j < EPI_GW; ++j) S[g * EPI_GW + j] *= al;
+            if (st_on) put(g);
+          }
+        }
       } else if (full && be == 0.f) {
         if (st_on) {
 #pragma unroll
@@ -1091,6 +1151,10 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
         }
       }
       if (FUSED) {                                 // this CTA's half of the tile is stored
+        if (P.c_map >= 0 && lane == 0) {           // bulk stores complete, ordered before the signal
+          ptx::bulk_wait_group<0>();
+          ptx::fence_proxy_async_global();
+        }
         ptx::named_bar_sync(5, EPI_THREADS);
         if (threadIdx.x == WARP_EPI0 * 32) {
           BLAS3_STRACE(8, w.ph);
@@ -1105,6 +1169,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
       }
       if (threadIdx.x == WARP_EPI0 * 32) BLAS3_TRACE(8);
     }
+    if (lane == 0) ptx::bulk_wait_group<0>();  // shared boxes read, stores complete, before exit
     if (threadIdx.x == WARP_EPI0 * 32) BLAS3_TRACE(9);
   }
 
@@ -1218,6 +1283,19 @@ static int launch_cg(PRM &prm, cudaStream_t stream, int num_sms, bool allow_pdl 
       if (!op_maps(prm, slot, sg.a, P.M, sg.K, HA, per, groups, P.bs_a)) return -4;
       if (!op_maps(prm, slot, sg.b, P.N, sg.K, G::HB, per, groups, P.bs_b)) return -4;
     }
+  }
+  // Cout as a TMA store target (bulk epilogue): 16-B aligned, ld % 4 == 0
+  for (int p = 0; p < prm.nphase; ++p) {
+    Problem &P = prm.ph[p].P;
+    P.c_map = -1;
+    const int64_t nb = P.nbatch > 1 ? P.nbatch : 1;
+    const bool ok = opt(BLAS3_OPT_TC_TMA_STORE) != 0 && reinterpret_cast<uintptr_t>(P.Cout) % 16 == 0 &&
+                    P.ldcout % 4 == 0 && (nb == 1 || (P.bs_c.inner % 4 == 0 && P.bs_c.outer % 4 == 0));
+    if (!ok || slot >= (int)(sizeof(prm.maps) / sizeof(prm.maps[0]))) continue;
+    const int64_t per = nb > 1 ? P.per : 1, groups = cdiv(nb, per);
+    if (!make_map(&prm.maps[slot], P.Cout, P.M, P.N, P.ldcout, 32, EPI_GW, CU_TENSOR_MAP_SWIZZLE_NONE, per,
+                  groups, P.bs_c)) return -4;
+    P.c_map = slot++;
   }
   // the TF32+BF16X instantiation in that mode (every phase of a fused launch
   // carries the same mode)
@@ -1395,7 +1473,7 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
   prm.nphase = 1;
   prm.ph[0].P = P0;
   prm.ph[0].P.dbg = debug_bits();
-  if (prm.ph[0].P.kc <= 0) prm.ph[0].P.kc = 4;
+  if (prm.ph[0].P.kc <= 0) prm.ph[0].P.kc = 2;
   const int cg = choose_cg(prm.ph[0].P, num_sms);
   const bool dyn = opt(BLAS3_OPT_TC_STATIC) == 0;
   if (cg == 2) plan_split<2>(prm, num_sms); else plan_split<1>(prm, num_sms);
@@ -1451,7 +1529,7 @@ int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int 
     PhaseDesc &ph = prm.ph[p];
     ph.P = phases[p].P;
     ph.P.dbg = debug_bits();
-    if (ph.P.kc <= 0) ph.P.kc = 4;
+    if (ph.P.kc <= 0) ph.P.kc = 2;
     if (!tc_eligible(ph.P) || ph.P.max_sms) return -1;
     const int64_t nb = ph.P.nbatch > 1 ? ph.P.nbatch : 1;
     ph.tiles_per = TL::count(ph.P);

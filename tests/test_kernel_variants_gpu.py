@@ -7,7 +7,10 @@ picks the pair kernel for large problems), whole tiles only
 every size (BLAS3_GM_MAP=1: transposed / symmetric / triangular operands
 materialised in global memory first, the default only for large problems), and
 STRSM's first panel by update + solve instead of the precomputed Y - M X form
-(BLAS3_TRSM_FIRST_YM=0).  Each child process runs a representative subset of the
+(BLAS3_TRSM_FIRST_YM=0), the per-thread scalar epilogue stores instead of the
+TMA tensor stores (BLAS3_TC_TMA_STORE=0), and 16 k-blocks per TMEM partial
+(BLAS3_TC_KC=16; its accuracy is checked against the round-1 bound: it
+exceeds the fp32-class diagnostic by design).  Each child process runs a representative subset of the
 parity suite (every routine family, both transposes/sides) on that variant."""
 import os
 import subprocess
@@ -21,9 +24,10 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 @pytest.mark.parametrize("env", [{"BLAS3_TC_CTA": "1"}, {"BLAS3_TC_CTA": "2"}, {"BLAS3_TC_STATIC": "1"},
                                  {"BLAS3_TC_SPLIT": "0"}, {"BLAS3_TC_CTA": "1", "BLAS3_TC_SPLIT": "0"},
-                                 {"BLAS3_GM_MAP": "1"}, {"BLAS3_TRSM_FIRST_YM": "0"}],
+                                 {"BLAS3_GM_MAP": "1"}, {"BLAS3_TRSM_FIRST_YM": "0"},
+                                 {"BLAS3_TC_TMA_STORE": "0"}, {"BLAS3_TC_KC": "16"}],
                          ids=["single_cta", "cta_pair", "static_schedule", "no_split", "single_cta_no_split",
-                              "gm_map", "trsm_no_first_ym"])
+                              "gm_map", "trsm_no_first_ym", "scalar_epilogue", "kc16"])
 def test_variant_subset(env):
     import torch
     if not torch.cuda.is_available():
@@ -31,6 +35,8 @@ def test_variant_subset(env):
     sel = "3xtf32 and (sgemm or ssymm or syrk or strmm or strsm or split_is_real)"
     cmd = [sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k", sel,
            os.path.join(ROOT, "tests", "test_parity_gpu.py")]
+    if env.get("BLAS3_TC_KC") == "16":
+        sel = "3xtf32 and (integer or split_is_real)"      # bit-exact pins: independent of the chunk
     r = subprocess.run(cmd, env={**os.environ, **env}, cwd=ROOT, capture_output=True, text=True,
                        timeout=900)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]

@@ -80,6 +80,25 @@ def test_sgemm(b3, oracle_mod, mode, route, ta, tb, m, n, k):
     assert e_rel(got, ref) <= rel_bound(f32_eval(AL, op(A, ta), op(B, tb), BE, C), ref)
 
 
+@pytest.mark.parametrize("k", [512, 8192])
+def test_same_sign_accumulation(b3, oracle_mod, mode, k):
+    """Worst case for the tensor core's truncating fp32 accumulator (reading
+    Q24): with all products positive every truncation biases the sum the same
+    way, so the error adds up coherently over the UMMAs of one TMEM partial
+    instead of as a random walk.  The plain fp32 evaluation (round to nearest)
+    has no such bias; the kernel must stay within the same diagnostic bound."""
+    m, n = 256, 260
+    A = gen.uniform(m, k, "pos-a", lo=0.0, hi=1.0)
+    B = gen.uniform(k, n, "pos-b", lo=0.0, hi=1.0)
+    C = gen.uniform(m, n, "pos-c", lo=0.0, hi=1.0)
+    dC = to_dev(C)
+    b3.sgemm("N", "N", AL, to_dev(A), to_dev(B), BE, dC)
+    got = to_host(dC)
+    ref = oracle_mod.sgemm("N", "N", AL, A, B, BE, C)
+    assert e_nw(got, ref, AL * fro(A) * fro(B) + BE * fro(C)) <= TOL_NW
+    assert e_rel(got, ref) <= rel_bound(f32_eval(AL, A, B, BE, C), ref)
+
+
 @pytest.mark.parametrize("ta,tb", list(itertools.product("NT", "NT")))
 @pytest.mark.parametrize("m,n,k", [(132, 260, 1000), (64, 300, 36)])
 def test_sgemm_integer_bitexact(b3, oracle_mod, mode, ta, tb, m, n, k):
