@@ -146,21 +146,36 @@ def pinned(arr, torch):
 
 
 # ----------------------------------------------------------------------------- our arm
-def run_ours(args):
+def init_dist():
+    """One process per GPU (torchrun env).  NCCL communicators are created
+    eagerly (device_id) and exercised by a barrier, and each rank logs its
+    communicator to stderr so a launch's rank count is visible in the log."""
     import torch
     import torch.distributed as dist
-
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     local = local % max(1, torch.cuda.device_count())   # (a 1-GPU logic check may share a device)
     torch.cuda.set_device(local)
+    comm = {"backend": None, "world": world}
     if world > 1:
         backend = os.environ.get("BLAS3_BENCH_BACKEND", "nccl")   # gloo: 1-GPU logic check only
         if backend == "nccl":
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         else:
             dist.init_process_group(backend)
+        dist.barrier()
+        comm["backend"] = backend
+        if backend == "nccl":
+            v = torch.cuda.nccl.version()
+            comm["nccl_version"] = ".".join(map(str, v)) if isinstance(v, tuple) else str(v)
+        print(f"[bench] rank {rank}/{world} on cuda:{local}: {backend} process group up "
+              f"(communicator initialised, barrier passed)", file=sys.stderr, flush=True)
+    return torch, dist, world, rank, local, comm
+
+
+def run_ours(args):
+    torch, dist, world, rank, local, comm_info = init_dist()
 
     import paper_conf_ipps_cuiwxyf11_b200 as b3
     b3.set_math_mode(args.math)
@@ -195,59 +210,95 @@ def run_ours(args):
 
     if world > 1:
         from paper_conf_ipps_cuiwxyf11_b200 import dist as d3
-        # SYRK/SYR2K at N>1: k-split weak scaling -- rank r's own k-slab A_r (= its B
-        # slab) and B_r (= its C0 slab), partials summed by one NCCL all-reduce; beta*C
-        # is applied on rank 0 only and the other ranks start from zeros, so the sum is
-        # exact on both triangles.
-        dCs = torch.empty((n, n), device=dev)
-        Cs = colmaj(dCs)
+        # The exchange steps, all overlapped with compute:
+        #  * A: broadcast in 8 K-panels on a comm stream, consumed by the
+        #    panel GEMMs of the sgemm as they land (d3.sgemm);
+        #  * T: only its lower triangle, 4 trapezoid panels, on a second comm
+        #    stream from the start of the step (needed from strmm on);
+        #  * SYRK/SYR2K (no right-hand side to shard): k-split weak scaling --
+        #    rank r's own k-slab (its B slab; for SYR2K its B and C0 slabs),
+        #    the partial products summed by an NCCL all-reduce on a third
+        #    stream that overlaps the next routines.  beta*C is applied on
+        #    rank 0 only (the others start from zeros), so the sum is exact.
+        # While a collective is in flight the products leave RESERVE SMs to
+        # NCCL (BLAS3_OPT_MAX_SMS).
+        RESERVE = 16
+        nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+        dCs1 = torch.empty((n, n), device=dev); dCs2 = torch.empty((n, n), device=dev)
+        Cs1, Cs2 = colmaj(dCs1), colmaj(dCs2)
+        comm_T = torch.cuda.Stream(device=dev)
+        comm_R = torch.cuda.Stream(device=dev)
         beta_r = BETA if rank == 0 else 0.0
 
-    def syrk_k(Bk=None):
-        Bk = Bm if Bk is None else Bk
-        if rank == 0:
-            dCs.copy_(dC0)
-        else:
-            dCs.zero_()
-        b3.ssyrk("L", "N", ALPHA, Bk, beta_r, Cs)
-        d3.syrk_k_split(dCs)
+        def allreduce_async(buf):
+            e = torch.cuda.Event(); e.record(torch.cuda.current_stream())
+            with torch.cuda.stream(comm_R):
+                comm_R.wait_event(e)
+                d3.syrk_k_split(buf)
 
-    def syr2k_k(Bk=None, Ck=None):
-        Bk = Bm if Bk is None else Bk
-        Ck = C0 if Ck is None else Ck
-        if rank != 0:
-            dCs.zero_()
-        b3.ssyr2k("L", "N", ALPHA, Bk, Ck, 1.0 if rank == 0 else 0.0, Cs)
-        d3.syrk_k_split(dCs)
+        def syrk_k(Bk=None):
+            Bk = Bm if Bk is None else Bk
+            if rank == 0:
+                dCs1.copy_(dC0)
+            else:
+                dCs1.zero_()
+            b3.ssyrk("L", "N", ALPHA, Bk, beta_r, Cs1)
+            allreduce_async(dCs1)
 
-    def chain_syrk_k(Bk=None, Ck=None):
-        syrk_k(Bk)
-        syr2k_k(Bk, Ck)
+        def syr2k_k(Bk=None, Ck=None):
+            Bk = Bm if Bk is None else Bk
+            Ck = C0 if Ck is None else Ck
+            if rank == 0:
+                dCs2.copy_(dC0)
+            else:
+                dCs2.zero_()
+            b3.ssyr2k("L", "N", ALPHA, Bk, Ck, beta_r, Cs2)
+            allreduce_async(dCs2)
+
+        def bcast_T_async(Tv):
+            e = torch.cuda.Event(); e.record(torch.cuda.current_stream())
+            with torch.cuda.stream(comm_T):
+                comm_T.wait_event(e)
+                for p0, p1 in d3.k_panels(n, 4):
+                    d3.broadcast_trapezoid(Tv, p0, p1, True)
+                eT = torch.cuda.Event(); eT.record(comm_T)
+            return eT
 
     def chain(record):
-        def timed(name, fn):
+        def timed(name, fn, reserve=False):
+            def run():
+                if reserve and world > 1:
+                    with b3.options(max_sms=nsm - RESERVE):
+                        fn()
+                else:
+                    fn()
             if record:
                 e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
-                e0.record(stream); fn(); e1.record(stream)
+                e0.record(stream); run(); e1.record(stream)
                 ev[name].append((e0, e1))
             else:
-                fn()
-        timed("sgemm", lambda: b3.sgemm("N", "N", ALPHA, A, Bm, BETA, C))
-        timed("ssymm", lambda: b3.ssymm("L", "L", ALPHA, A, Bm, BETA, C))
+                run()
         if world == 1:
+            timed("sgemm", lambda: b3.sgemm("N", "N", ALPHA, A, Bm, BETA, C))
+            timed("ssymm", lambda: b3.ssymm("L", "L", ALPHA, A, Bm, BETA, C))
             timed("ssyrk", lambda: b3.ssyrk("L", "N", ALPHA, A, BETA, C))
             timed("ssyr2k", lambda: b3.ssyr2k("L", "N", ALPHA, A, Bm, BETA, C))
-        else:
-            timed("ssyrk", syrk_k)
-            timed("ssyr2k", syr2k_k)
-        timed("strmm", lambda: b3.strmm("L", "L", "N", "N", ALPHA, T, X))
+            timed("strmm", lambda: b3.strmm("L", "L", "N", "N", ALPHA, T, X))
+            timed("strsm", lambda: b3.strsm("L", "L", "N", "N", ALPHA, T, X))
+            return
+        eT = bcast_T_async(T)
+        timed("sgemm", lambda: d3.sgemm("N", "N", ALPHA, A, Bm, BETA, C, panels=8, reserve_sms=RESERVE))
+        timed("ssymm", lambda: b3.ssymm("L", "L", ALPHA, A, Bm, BETA, C), reserve=True)
+        timed("ssyrk", syrk_k, reserve=True)
+        timed("ssyr2k", syr2k_k, reserve=True)
+        stream.wait_event(eT)
+        timed("strmm", lambda: b3.strmm("L", "L", "N", "N", ALPHA, T, X), reserve=True)
         timed("strsm", lambda: b3.strsm("L", "L", "N", "N", ALPHA, T, X))
+        stream.wait_stream(comm_R)            # the reduced SYRK/SYR2K results are part of the step
 
     def step_device(record=False):
         # fresh working copies so every step computes on the same data
         dC.copy_(dC0); dX.copy_(dB)
-        if world > 1:
-            dist.broadcast(dA, 0); dist.broadcast(dT, 0)      # the one exchange step
         chain(record)
 
     # ---- e2e leg: host (pinned) inputs -> the chain -> host results, every step.
@@ -285,26 +336,32 @@ def run_ours(args):
             eT = torch.cuda.Event(); eT.record(h2d_stream)
         stream.wait_event(eA)
         if world > 1:
-            dist.broadcast(bset["A"], 0)
-        for (c0, c1), e in zip(bounds, evs):
-            stream.wait_event(e)
-            b3.sgemm("N", "N", ALPHA, A_, Bm_[:, c0:c1], BETA, C_[:, c0:c1])
+            for (c0, c1), e in zip(bounds, evs):
+                stream.wait_event(e)
+            d3.sgemm("N", "N", ALPHA, A_, Bm_, BETA, C_, panels=8, reserve_sms=RESERVE)
+        else:
+            for (c0, c1), e in zip(bounds, evs):
+                stream.wait_event(e)
+                b3.sgemm("N", "N", ALPHA, A_, Bm_[:, c0:c1], BETA, C_[:, c0:c1])
         b3.ssymm("L", "L", ALPHA, A_, Bm_, BETA, C_)
         if world == 1:
             b3.ssyrk("L", "N", ALPHA, A_, BETA, C_)
             b3.ssyr2k("L", "N", ALPHA, A_, Bm_, BETA, C_)
         else:
-            chain_syrk_k(Bm_, C_)
+            syrk_k(Bm_)
+            syr2k_k(Bm_, C_)
         eC = torch.cuda.Event(); eC.record(stream)
         with torch.cuda.stream(d2h_stream):
             d2h_stream.wait_event(eC)
             hC_out.copy_(bset["C"], non_blocking=True)
         stream.wait_event(eT)
         if world > 1:
-            dist.broadcast(bset["T"], 0)
+            stream.wait_event(bcast_T_async(T_))
         bset["X"].copy_(bset["B"])
         b3.strmm("L", "L", "N", "N", ALPHA, T_, X_)
         b3.strsm("L", "L", "N", "N", ALPHA, T_, X_)
+        if world > 1:
+            stream.wait_stream(comm_R)
         eX = torch.cuda.Event(); eX.record(stream)
         with torch.cuda.stream(d2h_stream):
             d2h_stream.wait_event(eX)
@@ -479,9 +536,12 @@ def run_ours(args):
                         "(K=8192), strmm LLNN, strsm LLNN; alpha=1.5 beta=0.5",
             "n": n, "k": n, "cols_per_rank": cols, "math": args.math,
             "l2": "no flush: every operand is 256 MiB > 126 MB L2",
-            "parallelism": (f"dp{world}: column slabs of B/C/X per rank ({cols} columns each), A and T "
-                            f"broadcast from rank 0 (NCCL); ssyrk/ssyr2k k-split, partials "
-                            f"all-reduced (NCCL)") if world > 1 else "1 GPU",
+            "parallelism": (f"dp{world}: column slabs of B/C/X per rank ({cols} columns each); A broadcast "
+                            f"from rank 0 in 8 K-panels overlapped with the sgemm panels, T's lower "
+                            f"triangle in 4 trapezoid panels overlapped with sgemm..ssyr2k (NCCL, "
+                            f"comm streams, 16 SMs reserved while in flight); ssyrk/ssyr2k k-split, "
+                            f"partials all-reduced (NCCL) overlapped with the next routines")
+            if world > 1 else "1 GPU",
         },
         "routines": per,
         "pct_of_peak": round(100.0 * value / world / 1e3 / pk, 1),
@@ -503,6 +563,7 @@ def run_ours(args):
         "e2e": {"value": round(e2e_value, 1), "unit": "GFLOPS",
                 "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world},
         "gpu_launches": int(launches),
+        "comm": comm_info,
         "alt_mode": alt,
         "context": context,
         "gpu_launches_per_step": round(launches / args.steps, 1),
@@ -510,6 +571,216 @@ def run_ours(args):
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         out["cpu_baseline"] = cpu_baseline(args.cpu_seconds)
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+# ----------------------------------------------------------------------------- configs[4]
+CFG5_N = 32768
+CFG5_ROUTINES = ["sgemm", "ssymm", "strsm"]
+
+
+def cfg5_inputs(torch, n, c0, c1, rank, dev):
+    """Seeded device-side inputs of BASELINE configs[4] (an N = 32768 host
+    generation would take minutes).  Every 256-column block of a global
+    matrix has its own Philox seed (hash of name and block index), so a
+    rank's slab holds the same numbers for any world size.  A: U(-1,1) n x n
+    (rank 0); T: lower triangular, off-diagonal U(-1,1), a_ii = 1 + max(row,
+    column) abs-sum (reading Q22), NaN in the blank triangle (never read);
+    B, C: U(-1,1) column slabs [c0, c1)."""
+    import hashlib
+
+    def block(name, j, rows, cols):
+        h = hashlib.sha256(repr((20111, "cfg5", name, n, j)).encode()).digest()
+        g = torch.Generator(device=dev)
+        g.manual_seed(int.from_bytes(h[:8], "little") & ((1 << 63) - 1))
+        return torch.rand((cols, rows), generator=g, device=dev).mul_(2.0).sub_(1.0)
+
+    def slab_of(name, a, b, out):              # out: (b - a, n) row-major storage of columns a..b
+        for j in range(a // 256, -(-b // 256)):
+            x0, x1 = max(a, j * 256), min(b, (j + 1) * 256)
+            out[x0 - a:x1 - a] = block(name, j, n, min(256, n - j * 256))[x0 - j * 256:x1 - j * 256]
+        return out
+
+    dA = torch.empty((n, n), device=dev)
+    dT = torch.empty((n, n), device=dev)
+    if rank == 0:
+        slab_of("A", 0, n, dA)
+        slab_of("T", 0, n, dT)                 # dT[j] = column j of T
+        tt = dT                                # rows of tt = columns of T; keep rows > col (strict lower)
+        idx = torch.arange(n, device=dev)
+        rowsum = torch.zeros(n, dtype=torch.float64, device=dev)
+        colsum = torch.zeros(n, dtype=torch.float64, device=dev)
+        for j0 in range(0, n, 1024):
+            blk = tt[j0:j0 + 1024]             # columns j0.. of T, each a row here
+            jj = idx[j0:j0 + 1024, None]
+            strict = idx[None, :] > jj         # T(i, j) with i > j
+            blk.masked_fill_(~strict, 0.0)
+            a64 = blk.abs().double()
+            colsum[j0:j0 + 1024] = a64.sum(1)
+            rowsum += a64.sum(0)
+            blk.masked_fill_(idx[None, :] < jj, float("nan"))
+        dom = (1.0 + torch.maximum(rowsum, colsum)).float()
+        tt.diagonal().copy_(dom)
+    cols = c1 - c0
+    dB = slab_of("B", c0, c1, torch.empty((cols, n), device=dev))
+    dC0 = slab_of("C", c0, c1, torch.empty((cols, n), device=dev))
+    return dA, dT, dB, dC0
+
+
+def run_cfg5(args):
+    """BASELINE configs[4]: N = 32768 SGEMM NN, SSYMM LL and STRSM LLNN with
+    the right-hand side in column slabs of N/P columns per rank (pre-resident)
+    and A (T) resident on rank 0 and broadcast INSIDE each routine's timed
+    region: A in 8 K-panels for SGEMM, only the stored lower triangle in
+    trapezoid panels for SSYMM (8) and STRSM (4), every broadcast pipelined
+    with the products that consume it (dist.py).  Strong scaling: the global
+    problem is fixed; value = its LAWN-41 flops / step time (max over ranks),
+    so T1/TP = value(P) / value(1)."""
+    torch, dist, world, rank, local, comm_info = init_dist()
+    import paper_conf_ipps_cuiwxyf11_b200 as b3
+    from paper_conf_ipps_cuiwxyf11_b200 import dist as d3
+    b3.set_math_mode(args.math)
+    n = CFG5_N if args.size == N else args.size
+    c0, c1 = d3.slab(n, world, rank)
+    cols = c1 - c0
+    dev = torch.device("cuda", local)
+    dA, dT, dB, dC0 = cfg5_inputs(torch, n, c0, c1, rank, dev)
+    dC = torch.empty_like(dC0); dX = torch.empty_like(dB)
+    A, T, Bm, C0, C, X = dA.t(), dT.t(), dB.t(), dC0.t(), dC.t(), dX.t()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    stream = torch.cuda.current_stream()
+    ev = {r: [] for r in CFG5_ROUTINES}
+    calls = {
+        "sgemm": lambda: d3.sgemm("N", "N", ALPHA, A, Bm, BETA, C, panels=8),
+        "ssymm": lambda: d3.ssymm("L", "L", ALPHA, A, Bm, BETA, C, panels=8),
+        "strsm": lambda: d3.strsm("L", "L", "N", "N", ALPHA, T, X, panels=4),
+    }
+
+    def step(record=False):
+        dC.copy_(dC0); dX.copy_(dB)
+        for r in CFG5_ROUTINES:
+            if record:
+                e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+                e0.record(stream); calls[r](); e1.record(stream)
+                ev[r].append((e0, e1))
+            else:
+                calls[r]()
+
+    def timed_loop(steps, record):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(steps):
+            step(record)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1)
+        if world > 1:
+            t = torch.tensor([ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+        return ms
+
+    for _ in range(args.warmup):
+        step()
+    launches0 = b3.launch_count()
+    with ClockSampler(local) as clk:
+        time.sleep(0.6)
+        ms = timed_loop(args.steps, True)
+    launches = b3.launch_count() - launches0
+
+    # e2e: the same step through the public API with host buffers: A and T
+    # uploaded on rank 0, the B/C slabs on every rank, C/X slabs downloaded
+    e2e = None
+    if not args.no_e2e:
+        try:
+            hA = torch.empty_like(dA, device="cpu").pin_memory() if rank == 0 else None
+            hT = torch.empty_like(dT, device="cpu").pin_memory() if rank == 0 else None
+            hB = torch.empty_like(dB, device="cpu").pin_memory()
+            hC = torch.empty_like(dC0, device="cpu").pin_memory()
+            hCo = torch.empty_like(dC0, device="cpu").pin_memory()
+            hXo = torch.empty_like(dB, device="cpu").pin_memory()
+            if rank == 0:
+                hA.copy_(dA); hT.copy_(dT)
+            hB.copy_(dB); hC.copy_(dC0)
+            e2e_steps = max(1, min(args.steps, 3))
+
+            def e2e_step():
+                if rank == 0:
+                    dA.copy_(hA, non_blocking=True); dT.copy_(hT, non_blocking=True)
+                dB.copy_(hB, non_blocking=True); dC0.copy_(hC, non_blocking=True)
+                step()
+                hCo.copy_(dC, non_blocking=True); hXo.copy_(dX, non_blocking=True)
+            e2e_step()
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            t0 = torch.cuda.Event(enable_timing=True); t1 = torch.cuda.Event(enable_timing=True)
+            t0.record(stream)
+            for _ in range(e2e_steps):
+                e2e_step()
+            t1.record(stream)
+            torch.cuda.synchronize()
+            ms_e = t0.elapsed_time(t1)
+            if world > 1:
+                t = torch.tensor([ms_e], device=dev)
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                ms_e = float(t.item())
+            tot = 5.0 * n ** 3
+            e2e = {"value": round(tot / (ms_e / e2e_steps * 1e-3) / 1e9, 1), "unit": "GFLOPS",
+                   "h2d_bytes_per_step": int(2 * n * n * 4 + 2 * n * n * 4), "d2h_bytes_per_step": int(2 * n * n * 4),
+                   "steps": e2e_steps}
+        except RuntimeError as exc:            # pinned host memory of the N = 32768 operands
+            e2e = {"value": None, "unit": "GFLOPS", "h2d_bytes_per_step": None, "d2h_bytes_per_step": None,
+                   "unavailable": f"host buffers: {str(exc).splitlines()[0][:120]}"}
+
+    per = {}
+    fl = {"sgemm": 2.0 * n ** 3, "ssymm": 2.0 * n ** 3, "strsm": 1.0 * n ** 3}
+    for r in CFG5_ROUTINES:
+        avg = float(np.mean([a.elapsed_time(b) for a, b in ev[r]]))
+        if world > 1:
+            t = torch.tensor([avg], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            avg = float(t.item())
+        per[r] = {"ms": round(avg, 3), "gflops": round(fl[r] / (avg * 1e-3) / 1e9, 1)}
+    step_ms = ms / args.steps
+    value = sum(fl.values()) / (step_ms * 1e-3) / 1e9
+    peaks, peak_src = load_peaks()
+    pk = fp32_3xtf32_peak(peaks, sustained=True)
+    out = {
+        "metric": "GFLOPS per routine (SGEMM/SSYMM/SSYRK/SSYR2K/STRMM/STRSM) at N=8192, "
+                  "1/2/4/8 B200, % of peak",
+        "value": round(value, 1), "unit": "GFLOPS", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(step_ms, 3), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic (seeded device-side U(-1,1) per 256-column block; diagonally dominant T)",
+        "config": {"workload": f"configs[4]: N={n} sgemm NN, ssymm LL, strsm LLNN, right-hand side in "
+                               f"column slabs of N/P columns, A/T broadcast from rank 0 inside the timed region",
+                   "n": n, "cols_per_rank": cols, "math": args.math,
+                   "l2": "no flush: every operand is >= 512 MiB > 126 MB L2",
+                   "parallelism": (f"dp{world}: column slabs; A broadcast in 8 K-panels (sgemm), lower "
+                                   f"triangle in trapezoid panels (ssymm 8, strsm 4), pipelined with the "
+                                   f"consuming products, 16 SMs reserved while in flight")
+                   if world > 1 else "1 GPU (T1 of the strong-scaling curve)"},
+        "routines": per,
+        "pct_of_peak": round(100.0 * value / world / 1e3 / pk, 1),
+        "roofline": {"bound": "tensor", "kernel": "tc_structured_gemm (whole step)",
+                     "achieved": round(value / world / 1e3, 2), "peak": round(pk, 1), "unit": "TFLOP/s",
+                     "frac": round(value / world / 1e3 / pk, 3),
+                     "peak_source": f"{peak_src} bf16 sustained x tf32/bf16 {TF32_OVER_BF16:.3f} / 3",
+                     "traffic": None},
+        "e2e": e2e,
+        "gpu_launches": int(launches),
+        "comm": comm_info,
+        "clocks": clk.summary(),
+    }
     if rank == 0:
         print(json.dumps(out), flush=True)
     if world > 1:
@@ -610,6 +881,20 @@ def run_reference(args):
     print(json.dumps(out), flush=True)
 
 
+def spawn_command(gpus, argv, port=None):
+    """argv for `python -m torch.distributed.run` with one process per GPU on
+    127.0.0.1 (used when bench.py --gpus N > 1 is started without torchrun)."""
+    if port is None:
+        import socket
+        s = socket.socket()
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+        s.close()
+    script = os.path.abspath(argv[0])
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={gpus}",
+            "--master-addr", "127.0.0.1", "--master-port", str(port), script, *argv[1:]]
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -624,11 +909,22 @@ def main():
     ap.add_argument("--no-context", action="store_true", help="skip the cuBLAS context timing")
     ap.add_argument("--no-alt-mode", action="store_true",
                     help="skip the extra device-only pass in the opt-in TF32+BF16X mode")
+    ap.add_argument("--workload", default="chain", choices=["chain", "cfg5"],
+                    help="chain: the six-routine N=8192 step (default, weak scaling at N>1); "
+                         "cfg5: BASELINE configs[4], N=32768 column slabs (strong scaling)")
     args = ap.parse_args()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # not under torchrun: re-launch this command with one process per GPU
+        os.execv(sys.executable, spawn_command(args.gpus, sys.argv))
+    if "WORLD_SIZE" in os.environ and int(os.environ["WORLD_SIZE"]) != args.gpus:
+        print(f"warning: --gpus {args.gpus} but WORLD_SIZE={os.environ['WORLD_SIZE']}; "
+              f"using WORLD_SIZE", file=sys.stderr)
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)
     if args.impl == "reference":
         run_reference(args)
+    elif args.workload == "cfg5":
+        run_cfg5(args)
     else:
         run_ours(args)
 

@@ -220,6 +220,10 @@ int blas3_get_math_mode(void);
  *                          tensor stores (32-row x 8-column boxes, 128-B rows),
  *                          when C is 16-B aligned with ldc % 4 == 0; 0 per-thread
  *                          coalesced 4-B stores
+ *   BLAS3_OPT_MAX_SMS      [BLAS3_MAX_SMS]  launch at most this many SMs' worth of CTAs
+ *                          (0 = all, default): leaves SMs to concurrent kernels,
+ *                          e.g. NCCL broadcasts overlapped with the products
+ *                          (paper_conf_ipps_cuiwxyf11_b200.dist)
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */
@@ -231,7 +235,7 @@ enum {
     BLAS3_OPT_TRSM_RESERVE = 12, BLAS3_OPT_TRSM_GEO_LEAF = 13, BLAS3_OPT_TRSM_FUSED = 14,
     BLAS3_OPT_TRSM_FIRST_YM = 15, BLAS3_OPT_TRSM_FIRST_FUSED = 16, BLAS3_OPT_TRSM_FIRST_SPLIT = 17,
     BLAS3_OPT_TRSM_FIRST_ALL = 18, BLAS3_OPT_TC_RASTER = 19, BLAS3_OPT_TC_KC = 20,
-    BLAS3_OPT_TC_TMA_STORE = 21, BLAS3_OPT_COUNT = 22
+    BLAS3_OPT_TC_TMA_STORE = 21, BLAS3_OPT_MAX_SMS = 22, BLAS3_OPT_COUNT = 23
 };
 int blas3_set_option(int key, int64_t value);
 int64_t blas3_get_option(int key);

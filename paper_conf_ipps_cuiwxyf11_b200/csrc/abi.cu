@@ -49,6 +49,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TC_RASTER", 0, 0, 64, false},
     {"BLAS3_TC_KC", 2, 1, 64, true},
     {"BLAS3_TC_TMA_STORE", 1, 0, 1, false},
+    {"BLAS3_MAX_SMS", 0, 0, 4096, false},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;
@@ -138,6 +139,8 @@ static int device_check(int &sms) {
     }
   }
   sms = di.sms;
+  const int64_t cap = opt(BLAS3_OPT_MAX_SMS);          // SMs left to concurrent kernels
+  if (cap >= 2 && cap < sms) sms = (int)cap;
   return di.ok ? 0 : BLAS3_ERR_ARCH;
 }
 

@@ -20,10 +20,24 @@ Three layers:
                  rank's slab; local work is ALWAYS the CUDA library
                  (paper_conf_ipps_cuiwxyf11_b200), never a CPU path.
 
-SGEMM with transa='N' overlaps the broadcast with compute: A is sent in
-column panels on a side stream and the compute stream consumes panel p
-(K-range p of the product) as soon as it has landed; beta applies to the
-first panel only.
+Pipelined broadcast: A travels in column panels on a side
+(comm) stream while the compute stream consumes each panel as soon as it has
+landed, so the exposed broadcast is about one panel.  For a structured A only
+the stored triangle travels, one TRAPEZOID per column panel (columns [p0, p1),
+rows [p0, n) of a lower / [0, p1) of an upper triangle), packed into a
+contiguous staging buffer for NCCL: half the NVLink bytes.  The consumers:
+  * SGEMM NN   -- panel p is the K-range p: C += alpha A[:, p] B[p, :];
+  * SSYMM L    -- panel p contributes its diagonal block by SSYMM and its
+                  off-diagonal rectangle R twice, C_below += R B_p (NN) and
+                  C_p += R^T B_below (TN): sym(A) = sum of those (planner
+                  `symm_plan`);
+  * STRSM L, N -- the right-looking blocked solve in processing order: X_p by
+                  the library's STRSM on the diagonal block, then one SGEMM
+                  update of the rows after it (planner `trsm_plan`).
+While panels are still in flight the local kernels leave `reserve_sms` SMs
+free (BLAS3_OPT_MAX_SMS), so NCCL's kernels are never starved by the
+persistent GEMM grid.  Every plan is a pure list of operations, unit-tested
+on CPU by executing it with numpy against the unpartitioned product.
 """
 from __future__ import annotations
 
@@ -61,6 +75,54 @@ def k_panels(k: int, panels: int, align: int = 32) -> List[Tuple[int, int]]:
     """K-range panels for the pipelined broadcast (multiples of the k-block)."""
     panels = max(1, min(panels, -(-k // align)))
     return [p for p in (slab(k, panels, i, align) for i in range(panels)) if p[1] > p[0]]
+
+
+def trapezoid_rows(n: int, p0: int, p1: int, lower: bool) -> Tuple[int, int]:
+    """Rows of the stored triangle in columns [p0, p1) (diagonal block included)."""
+    return (p0, n) if lower else (0, p1)
+
+
+def symm_plan(n: int, panels: int, lower: bool, align: int = 32):
+    """SSYMM side='L' as column panels of the stored triangle, in broadcast
+    order.  Ops (alpha everywhere; `first` = apply beta, else 1.0):
+      ("symm", p0, p1, first)               C[p0:p1] (+)= sym(A_pp) B[p0:p1]
+      ("gemm", "N", r0, r1, p0, p1, first)  C[r0:r1] (+)= A[r0:r1, p0:p1] B[p0:p1]
+      ("gemm", "T", p0, p1, r0, r1, first)  C[p0:p1] (+)= A[r0:r1, p0:p1]^T B[r0:r1]
+    where [r0, r1) is the panel's off-diagonal rectangle ([p1, n) lower,
+    [0, p0) upper).  Every row of C receives beta from exactly its first op."""
+    ops, pan = [], k_panels(n, panels, align)
+    for i, (p0, p1) in enumerate(pan):
+        r0, r1 = (p1, n) if lower else (0, p0)
+        if lower:
+            ops.append(("symm", p0, p1, i == 0))
+            if r1 > r0:
+                ops.append(("gemm", "N", r0, r1, p0, p1, i == 0))
+                ops.append(("gemm", "T", p0, p1, r0, r1, False))
+        else:
+            ops.append(("symm", p0, p1, True))           # panel i is the first to touch its rows
+            if r1 > r0:
+                ops.append(("gemm", "N", r0, r1, p0, p1, False))
+                ops.append(("gemm", "T", p0, p1, r0, r1, False))
+    return pan, ops
+
+
+def trsm_plan(n: int, panels: int, lower: bool, align: int = 32):
+    """STRSM side='L', transa='N' as the right-looking blocked solve over
+    column panels of the stored triangle, in processing (= broadcast) order:
+    forward for lower, backward for upper.  Ops:
+      ("trsm", p0, p1, first)               X_p = inv(A_pp) (alpha if first else 1) B_p
+      ("upd", r0, r1, p0, p1, first)        B[r0:r1] = (alpha if first else 1) B[r0:r1] - A[r0:r1, p0:p1] X_p
+    alpha is folded into the first operation that touches each row."""
+    pan = k_panels(n, panels, align)
+    if not lower:
+        pan = pan[::-1]
+    ops = []
+    for i, (p0, p1) in enumerate(pan):
+        ops.append(("trsm", p0, p1, i == 0))
+        r0, r1 = (p1, n) if lower else (0, p0)
+        if r1 > r0:
+            ops.append(("upd", r0, r1, p0, p1, i == 0))
+    return pan, ops
 
 
 # =============================================================== comms
@@ -107,6 +169,25 @@ def _bcast(view, root, group):
         view.t().copy_(buf)
 
 
+def broadcast_trapezoid(A, p0: int, p1: int, lower: bool, root: int = 0, group=None):
+    """Broadcast the stored-triangle part of columns [p0, p1) of the n x n
+    column-major A (rows [p0, n) lower / [0, p1) upper) from `root`.  The
+    trapezoid is packed into a contiguous buffer (NCCL / gloo need one),
+    sent, and unpacked on the receivers only."""
+    world, rank = world_rank(group)
+    if world <= 1:
+        return
+    r0, r1 = trapezoid_rows(A.shape[0], p0, p1, lower)
+    view = A[r0:r1, p0:p1]
+    if view.t().is_contiguous():
+        _dist().broadcast(view.t(), root, group=group)
+        return
+    buf = view.t().contiguous() if rank == root else view.new_empty((p1 - p0, r1 - r0))
+    _dist().broadcast(buf, root, group=group)
+    if rank != root:
+        view.t().copy_(buf)
+
+
 def syrk_k_split(C_partial, group=None):
     """Sum the per-rank partial products of a k-distributed SYRK/SYR2K."""
     dist = _dist()
@@ -122,13 +203,12 @@ def _b3():
 
 
 def sgemm(transa, transb, alpha, A, B_slab, beta, C_slab, root=0, group=None, panels=8,
-          pipeline=None):
+          pipeline=None, reserve_sms=16):
     """C_slab <- alpha*op(A)*op(B)_slab + beta*C_slab on this rank's columns.
 
     A is replicated from `root` (NCCL broadcast).  For transa='N' the
     broadcast is pipelined in K panels on a side stream, overlapped with the
     panel GEMMs on the compute stream (`pipeline` defaults to world > 1)."""
-    import torch
     b3 = _b3()
     world, _ = world_rank(group)
     if pipeline is None:
@@ -137,27 +217,52 @@ def sgemm(transa, transb, alpha, A, B_slab, beta, C_slab, root=0, group=None, pa
         broadcast_panels(A, root, group, 1)
         b3.sgemm(transa, transb, alpha, A, B_slab, beta, C_slab)
         return
-    compute = torch.cuda.current_stream()
-    comm = torch.cuda.Stream()
-    comm.wait_stream(compute)
-    k = A.shape[1]
-    first = True
-    for c0, c1 in k_panels(k, panels):
-        with torch.cuda.stream(comm):
-            if world > 1:
-                _bcast(A[:, c0:c1], root, group)
-            ev = torch.cuda.Event()
-            ev.record(comm)
-        compute.wait_event(ev)
-        b3.sgemm("N", "N", alpha, A[:, c0:c1], B_slab[c0:c1], beta if first else 1.0, C_slab)
-        first = False
+    pan = k_panels(A.shape[1], panels)
+
+    def consume(i, c0, c1):
+        b3.sgemm("N", "N", alpha, A[:, c0:c1], B_slab[c0:c1], beta if i == 0 else 1.0, C_slab)
+
+    _Pipeline(b3, reserve_sms).run(pan, lambda c0, c1: _bcast(A[:, c0:c1], root, group) if world > 1 else None,
+                                   consume)
 
 
-def ssymm(side, uplo, alpha, A, B_slab, beta, C_slab, root=0, group=None):
+def ssymm(side, uplo, alpha, A, B_slab, beta, C_slab, root=0, group=None, panels=8,
+          pipeline=None, reserve_sms=16):
     """side='L': C_slab <- alpha*A*B_slab + beta*C_slab (column slabs);
-    side='R': row slabs (C_slab, B_slab are row blocks of C, B)."""
-    broadcast_panels(A, root, group, 1)
-    _b3().ssymm(side, uplo, alpha, A, B_slab, beta, C_slab)
+    side='R': row slabs (C_slab, B_slab are row blocks of C, B).
+    For side='L' (world > 1 by default) only the uplo triangle of A travels,
+    in trapezoid panels consumed as they land (`symm_plan`)."""
+    b3 = _b3()
+    world, _ = world_rank(group)
+    lower = uplo.upper() == "L"
+    if pipeline is None:
+        pipeline = world > 1
+    n = A.shape[0]
+    if not pipeline or side.upper() != "L" or panels <= 1:
+        for p0, p1 in k_panels(n, 1, 1):
+            broadcast_trapezoid(A, p0, p1, lower, root, group)
+        b3.ssymm(side, uplo, alpha, A, B_slab, beta, C_slab)
+        return
+    pan, ops = symm_plan(n, panels, lower)
+    by_panel = {}
+    for op in ops:
+        key = (op[1], op[2]) if op[0] == "symm" else ((op[4], op[5]) if op[1] == "N" else (op[2], op[3]))
+        by_panel.setdefault(key, []).append(op)
+
+    def consume(i, p0, p1):
+        for op in by_panel[(p0, p1)]:
+            be = beta if op[-1] else 1.0
+            if op[0] == "symm":
+                b3.ssymm("L", uplo, alpha, A[p0:p1, p0:p1], B_slab[p0:p1], be, C_slab[p0:p1])
+            elif op[1] == "N":
+                _, _, r0, r1, q0, q1, _ = op
+                b3.sgemm("N", "N", alpha, A[r0:r1, q0:q1], B_slab[q0:q1], be, C_slab[r0:r1])
+            else:
+                _, _, q0, q1, r0, r1, _ = op
+                b3.sgemm("T", "N", alpha, A[r0:r1, q0:q1], B_slab[r0:r1], be, C_slab[q0:q1])
+
+    _Pipeline(b3, reserve_sms).run(
+        pan, lambda p0, p1: broadcast_trapezoid(A, p0, p1, lower, root, group), consume)
 
 
 def strmm(side, uplo, transa, diag, alpha, A, B_slab, root=0, group=None):
@@ -165,9 +270,40 @@ def strmm(side, uplo, transa, diag, alpha, A, B_slab, root=0, group=None):
     _b3().strmm(side, uplo, transa, diag, alpha, A, B_slab)
 
 
-def strsm(side, uplo, transa, diag, alpha, A, B_slab, root=0, group=None):
-    broadcast_panels(A, root, group, 1)
-    _b3().strsm(side, uplo, transa, diag, alpha, A, B_slab)
+def strsm(side, uplo, transa, diag, alpha, A, B_slab, root=0, group=None, panels=4,
+          pipeline=None, reserve_sms=16):
+    """Solve op(A) X = alpha B_slab on this rank's columns (side='L'; rows
+    for side='R').  For side='L', transa='N' (world > 1 by default) only the
+    stored triangle travels, in trapezoid panels, and the solve is the
+    right-looking blocked sweep over those panels (`trsm_plan`): each
+    panel's diagonal solve by the library's STRSM and its update of the
+    remaining rows by SGEMM start as soon as the panel has landed."""
+    b3 = _b3()
+    world, _ = world_rank(group)
+    lower = uplo.upper() == "L"
+    if pipeline is None:
+        pipeline = world > 1
+    n = A.shape[0]
+    if not pipeline or side.upper() != "L" or transa.upper() != "N" or panels <= 1:
+        broadcast_trapezoid(A, 0, n, lower, root, group)
+        b3.strsm(side, uplo, transa, diag, alpha, A, B_slab)
+        return
+    pan, ops = trsm_plan(n, panels, lower)
+    by_panel = {}
+    for op in ops:
+        by_panel.setdefault((op[1], op[2]) if op[0] == "trsm" else (op[3], op[4]), []).append(op)
+
+    def consume(i, p0, p1):
+        for op in by_panel[(p0, p1)]:
+            a1 = alpha if op[-1] else 1.0
+            if op[0] == "trsm":
+                b3.strsm("L", uplo, "N", diag, a1, A[p0:p1, p0:p1], B_slab[p0:p1])
+            else:
+                _, r0, r1, q0, q1, _ = op
+                b3.sgemm("N", "N", -1.0, A[r0:r1, q0:q1], B_slab[q0:q1], a1, B_slab[r0:r1])
+
+    _Pipeline(b3, reserve_sms).run(
+        pan, lambda p0, p1: broadcast_trapezoid(A, p0, p1, lower, root, group), consume)
 
 
 def _tri_slab_products(two, uplo, trans, alpha, A, B, beta, C, slabs):

@@ -185,4 +185,5 @@ def test_options_roundtrip_and_validation(lib):
     for bad in (0, 3, 128):                       # power of two in [1, 64]
         assert lib.blas3_set_option(lib.OPTIONS["tc_kc"], bad) == 1
     assert lib.get_option("tc_tma_store") == 1
-    assert len(lib.OPTIONS) == 22
+    assert lib.get_option("max_sms") == 0
+    assert len(lib.OPTIONS) == 23

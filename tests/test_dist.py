@@ -49,6 +49,74 @@ def test_k_panels():
     assert p[0][0] == 0 and p[-1][1] == 100 and all(b - a > 0 for a, b in p)
 
 
+# ------------------------------------------------------------------ panel plans (pure)
+def _sym(A, lower):
+    T = np.tril(A) if lower else np.triu(A)
+    return T + (np.tril(T, -1).T if lower else np.triu(T, 1).T)
+
+
+def _run_symm_plan(A, B, C, alpha, beta, lower, panels):
+    """Execute symm_plan's op list with numpy (fp64), reading ONLY the stored
+    triangle's trapezoids of A, as the executor does with the library."""
+    n = A.shape[0]
+    pan, ops = d3.symm_plan(n, panels, lower)
+    stored = np.tril(A) if lower else np.triu(A)           # what the broadcast delivers
+    out = C.copy()
+    for op in ops:
+        be = beta if op[-1] else 1.0
+        if op[0] == "symm":
+            _, p0, p1, _ = op
+            out[p0:p1] = alpha * _sym(stored[p0:p1, p0:p1], lower) @ B[p0:p1] + be * out[p0:p1]
+        elif op[1] == "N":
+            _, _, r0, r1, q0, q1, _ = op
+            out[r0:r1] = alpha * stored[r0:r1, q0:q1] @ B[q0:q1] + be * out[r0:r1]
+        else:
+            _, _, q0, q1, r0, r1, _ = op
+            out[q0:q1] = alpha * stored[r0:r1, q0:q1].T @ B[r0:r1] + be * out[q0:q1]
+    return pan, out
+
+
+@pytest.mark.parametrize("n,panels", [(256, 4), (1000, 8), (96, 1), (130, 3)])
+@pytest.mark.parametrize("lower", [True, False])
+def test_symm_plan_reproduces_symm(n, panels, lower):
+    g = np.random.default_rng(7)
+    A, B, C = g.uniform(-1, 1, (n, n)), g.uniform(-1, 1, (n, 40)), g.uniform(-1, 1, (n, 40))
+    pan, out = _run_symm_plan(A, B, C, 1.5, 0.5, lower, panels)
+    ref = 1.5 * _sym(A, lower) @ B + 0.5 * C
+    assert np.allclose(out, ref, rtol=1e-12, atol=1e-12)
+    # panels tile the order exactly once, in broadcast order
+    assert [c for a, b in pan for c in range(a, b)] == list(range(n))
+
+
+@pytest.mark.parametrize("n,panels", [(256, 4), (1000, 8), (96, 1), (130, 3)])
+@pytest.mark.parametrize("lower", [True, False])
+def test_trsm_plan_reproduces_solve(n, panels, lower):
+    g = np.random.default_rng(11)
+    A = g.uniform(-1, 1, (n, n)) / n + np.eye(n) * 2.0
+    stored = np.tril(A) if lower else np.triu(A)
+    B = g.uniform(-1, 1, (n, 30))
+    pan, ops = d3.trsm_plan(n, panels, lower)
+    X = B.copy()
+    for op in ops:
+        a1 = 1.5 if op[-1] else 1.0
+        if op[0] == "trsm":
+            _, p0, p1, _ = op
+            X[p0:p1] = np.linalg.solve(stored[p0:p1, p0:p1], a1 * X[p0:p1])
+        else:
+            _, r0, r1, q0, q1, _ = op
+            X[r0:r1] = a1 * X[r0:r1] - stored[r0:r1, q0:q1] @ X[q0:q1]
+    assert np.allclose(X, np.linalg.solve(stored, 1.5 * B), rtol=1e-10, atol=1e-12)
+    # processing order: forward for lower, backward for upper
+    starts = [a for a, _ in pan]
+    assert starts == sorted(starts, reverse=not lower)
+    # every panel only needs its own trapezoid (rows of the stored triangle)
+    for op in ops:
+        if op[0] == "upd":
+            _, r0, r1, q0, q1, _ = op
+            t0, t1 = d3.trapezoid_rows(n, q0, q1, lower)
+            assert t0 <= r0 and r1 <= t1
+
+
 # ------------------------------------------------------------------ gloo, world 2
 def _free_port():
     s = socket.socket()
@@ -99,7 +167,26 @@ def _worker(rank, world, port, q):
         d3.syrk_k_split(Cp)
         ok_red = np.allclose(Cp.numpy(), A_np.astype(np.float64) @ A_np.T.astype(np.float64),
                              rtol=1e-12, atol=1e-12)
-        q.put((rank, ok_bcast, ok_pad, ok_slab, ok_red))
+        # trapezoid (triangle-only) broadcast: the receiver gets the stored
+        # triangle; of the other triangle only the panels' diagonal blocks travel
+        nt = 128
+        T_np = gen.uniform(nt, nt, "dist-T")
+        ok_tri = True
+        for lower in (True, False):
+            Tt = _colmajor(T_np) if rank == 0 else _colmajor(np.full((nt, nt), -7.0, np.float32))
+            sent = np.zeros((nt, nt), bool)
+            for p0, p1 in d3.k_panels(nt, 4):
+                d3.broadcast_trapezoid(Tt, p0, p1, lower, root=0)
+                r0, r1 = d3.trapezoid_rows(nt, p0, p1, lower)
+                sent[r0:r1, p0:p1] = True
+            got = Tt.numpy()
+            keep = np.tril(np.ones((nt, nt), bool)) if lower else np.triu(np.ones((nt, nt), bool))
+            ok_tri &= bool(keep[~sent].sum() == 0)               # the whole stored triangle travels
+            ok_tri &= np.array_equal(got[sent], T_np[sent])
+            if rank == 1:
+                ok_tri &= bool((got[~sent] == -7.0).all())
+            ok_tri &= sent.sum() < 0.7 * nt * nt                 # about half the matrix
+        q.put((rank, ok_bcast, ok_pad, ok_slab, ok_red, ok_tri))
     finally:
         dist.destroy_process_group()
 

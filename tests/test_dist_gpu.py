@@ -94,3 +94,55 @@ def test_pipelined_sgemm_panels(mods, oracle_mod):
     d3.sgemm("N", "N", 1.5, to_dev(A), to_dev(B), 0.5, dC, panels=8, pipeline=True)
     ref = oracle_mod.sgemm("N", "N", 1.5, A, B, 0.5, C)
     assert e_nw(to_host(dC), ref, 1.5 * fro(A) * fro(B) + 0.5 * fro(C)) <= TOL_NW
+
+
+@pytest.mark.parametrize("uplo", ["L", "U"])
+def test_pipelined_ssymm_trapezoid_panels(mods, oracle_mod, uplo):
+    """SSYMM as consumed from trapezoid panels (dist.symm_plan: diagonal block
+    by SSYMM, the off-diagonal rectangle by an NN and a TN SGEMM) with the
+    SM reservation of the overlapped broadcast: the north-star tolerance and
+    the fp32-class diagnostic against the fp64 oracle."""
+    from check import e_rel, rel_bound, sym_f32, f32_eval
+    b3, d3 = mods
+    n, cols = 1000, 520
+    A = gen.symmetric_stored(n, uplo, "pt-S")
+    B, C = gen.uniform(n, cols, "pt-B"), gen.uniform(n, cols, "pt-C")
+    dC = to_dev(C)
+    d3.ssymm("L", uplo, 1.5, to_dev(A), to_dev(B), 0.5, dC, panels=4, pipeline=True)
+    got = to_host(dC)
+    ref = oracle_mod.ssymm("L", uplo, 1.5, A, B, 0.5, C)
+    S = sym_f32(A, uplo)
+    assert e_nw(got, ref, 1.5 * fro(S) * fro(B) + 0.5 * fro(C)) <= TOL_NW
+    assert e_rel(got, ref) <= rel_bound(f32_eval(1.5, S, B, 0.5, C), ref)
+
+
+@pytest.mark.parametrize("uplo", ["L", "U"])
+def test_pipelined_strsm_trapezoid_panels(mods, oracle_mod, uplo):
+    """STRSM as the right-looking sweep over trapezoid panels (dist.trsm_plan)."""
+    from check import f64, e_rel
+    b3, d3 = mods
+    n, cols = 1100, 300
+    A = gen.triangular_dd(n, uplo, "N", "pt-T")
+    B = gen.uniform(n, cols, "pt-X")
+    dX = to_dev(B)
+    d3.strsm("L", uplo, "N", "N", 1.5, to_dev(A), dX, panels=4, pipeline=True)
+    X = f64(to_host(dX))
+    T = np.nan_to_num(f64(A))
+    T = np.tril(T) if uplo == "L" else np.triu(T)
+    assert fro(T @ X - 1.5 * f64(B)) / (fro(T) * fro(X)) <= 1e-5 * np.sqrt(n)
+    assert e_rel(X, oracle_mod.strsm("L", uplo, "N", "N", 1.5, A, B)) <= 1e-5
+
+
+def test_max_sms_option_same_result(mods):
+    """BLAS3_OPT_MAX_SMS (SMs left to NCCL) changes only the grid size (tile
+    shape and k-splitting pinned, so every tile's arithmetic is the same)."""
+    b3, d3 = mods
+    m, n, k = 1536, 1024, 1024
+    A, B, C = gen.uniform(m, k, "ms-A"), gen.uniform(k, n, "ms-B"), gen.uniform(m, n, "ms-C")
+    outs = []
+    for cap in (0, 132, 20):
+        dC = to_dev(C)
+        with b3.options(max_sms=cap, tc_cta=2, tc_split=0):
+            b3.sgemm("N", "N", 1.5, to_dev(A), to_dev(B), 0.5, dC)
+        outs.append(bits(to_host(dC)))
+    assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[0], outs[2])
