@@ -215,15 +215,20 @@ int blas3_get_math_mode(void);
  *                          8-deep k-step); measured e_rel on U(-1,1) SGEMM
  *                          16 -> 3.9e-6, 4 -> 1.1e-6, 2 -> 6.8e-7, and 2.6e-6 at
  *                          4 on an all-positive (SYRK diagonal) sum
- *   BLAS3_OPT_TC_TMA_STORE [BLAS3_TC_TMA_STORE] tcgen05 epilogue: 1 (default) the
- *                          output tile leaves through shared memory as TMA
- *                          tensor stores (32-row x 8-column boxes, 128-B rows),
+ *   BLAS3_OPT_TC_VEC_STORE [BLAS3_TC_VEC_STORE] tcgen05 epilogue: 1 (default) C is
+ *                          read and written with 16-B vector accesses (each
+ *                          warp's rows transposed through a 1 KiB shared box:
+ *                          a thread holds 4 consecutive rows of one column),
  *                          when C is 16-B aligned with ldc % 4 == 0; 0 per-thread
- *                          coalesced 4-B stores
+ *                          coalesced 4-B accesses
  *   BLAS3_OPT_MAX_SMS      [BLAS3_MAX_SMS]  launch at most this many SMs' worth of CTAs
  *                          (0 = all, default): leaves SMs to concurrent kernels,
  *                          e.g. NCCL broadcasts overlapped with the products
  *                          (paper_conf_ipps_cuiwxyf11_b200.dist)
+ *   BLAS3_OPT_TC_C_PREFETCH [BLAS3_TC_C_PREFETCH] tcgen05 epilogue, beta != 0: 1
+ *                          (default) each CTA's C tile is prefetched into L2
+ *                          (one TMA prefetch) a few TMEM chunks before it is
+ *                          read, so the store phase does not wait on HBM; 0 off
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */
@@ -235,7 +240,8 @@ enum {
     BLAS3_OPT_TRSM_RESERVE = 12, BLAS3_OPT_TRSM_GEO_LEAF = 13, BLAS3_OPT_TRSM_FUSED = 14,
     BLAS3_OPT_TRSM_FIRST_YM = 15, BLAS3_OPT_TRSM_FIRST_FUSED = 16, BLAS3_OPT_TRSM_FIRST_SPLIT = 17,
     BLAS3_OPT_TRSM_FIRST_ALL = 18, BLAS3_OPT_TC_RASTER = 19, BLAS3_OPT_TC_KC = 20,
-    BLAS3_OPT_TC_TMA_STORE = 21, BLAS3_OPT_MAX_SMS = 22, BLAS3_OPT_COUNT = 23
+    BLAS3_OPT_TC_VEC_STORE = 21, BLAS3_OPT_MAX_SMS = 22, BLAS3_OPT_TC_C_PREFETCH = 23,
+    BLAS3_OPT_COUNT = 24
 };
 int blas3_set_option(int key, int64_t value);
 int64_t blas3_get_option(int key);

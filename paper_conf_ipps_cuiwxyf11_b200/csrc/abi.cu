@@ -48,8 +48,9 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TRSM_FIRST_ALL", 0, 0, 1, false},
     {"BLAS3_TC_RASTER", 0, 0, 64, false},
     {"BLAS3_TC_KC", 2, 1, 64, true},
-    {"BLAS3_TC_TMA_STORE", 1, 0, 1, false},
+    {"BLAS3_TC_VEC_STORE", 1, 0, 1, false},
     {"BLAS3_MAX_SMS", 0, 0, 4096, false},
+    {"BLAS3_TC_C_PREFETCH", 1, 0, 1, false},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;
@@ -195,7 +196,8 @@ static Problem problem(int64_t M, int64_t N, float alpha, float beta, const floa
   P.nbatch = 1; P.per = 1;
   P.raster_gm = (int32_t)opt(BLAS3_OPT_TC_RASTER);
   P.kc = (int32_t)opt(BLAS3_OPT_TC_KC);
-  P.c_map = -1;
+  P.c_vec = 0;
+  P.c_pf_map = -1;
   return P;
 }
 

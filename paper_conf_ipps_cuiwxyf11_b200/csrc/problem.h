@@ -87,9 +87,11 @@ struct Problem {
   int32_t raster_gm;
   // tcgen05 path: k-blocks per TMEM partial (power of 2; BLAS3_OPT_TC_KC)
   int32_t kc;
-  // tcgen05 path: tensor-map slot of Cout for the bulk (TMA) epilogue
-  // stores, or -1 (scalar coalesced stores); set at launch
-  int32_t c_map;
+  // tcgen05 path, set at launch: 1 = the epilogue may use 16-B vector
+  // accesses of C (Cout, and Cin when beta != 0, 16-B aligned, ld % 4 == 0);
+  // tensor-map slot of Cin for the L2 prefetch of C tiles, or -1
+  int32_t c_vec;
+  int32_t c_pf_map;
 };
 
 HD int64_t batch_off(const BatchStride &s, int64_t b, int64_t per) {

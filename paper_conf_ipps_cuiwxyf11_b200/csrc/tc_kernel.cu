@@ -79,7 +79,9 @@ constexpr int TR_THREADS = NUM_TR_WARPS * 32;
 constexpr int EPI_THREADS = NUM_EPI_WARPS * 32;
 constexpr int TMEM_COLS = 512;             // 2 accumulators x BN columns
 constexpr int MAX_MAPS = 10;                 // 2 segments x 2 operands x 2 views + C
-// epilogue staging: per epilogue warp two 32-row x 8-column fp32 boxes (TMA store)
+// epilogue: per epilogue warp one 32-row x 8-column fp32 shared box, the
+// transpose between the TMEM layout (thread = row) and 16-B vector accesses
+// of column-major C (thread = 4 consecutive rows of one column)
 constexpr int EPI_GW = 8, EPI_BOX = 32 * EPI_GW;
 constexpr int LAYOUT_K = 0, LAYOUT_MN = 1;
 
@@ -126,7 +128,7 @@ struct Geo {
     uint32_t split_last;     // epilogue: this CTA's slice of a split tile is the last one
   };
   struct alignas(1024) EpiStage {
-    float box[NUM_EPI_WARPS][2][EPI_BOX];   // D staging for the TMA tensor stores
+    float box[NUM_EPI_WARPS][EPI_BOX];      // epilogue transpose boxes
   };
   static constexpr size_t SMEM =
       sizeof(RawBuf) * RS + sizeof(LoBuf) * LS + sizeof(EpiStage) + sizeof(Barriers) + 1024;
@@ -736,6 +738,10 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));
           atomicMin(prm.ph_trace + 2 * w.ph, t_);
         }
+        // C (beta != 0) into L2 while the tile's last k-blocks are loaded: the
+        // epilogue's loads then hit L2, which keeps its store phase (during
+        // which the next tile's TMEM partials wait to be drained) short
+        int64_t pf_left = (P.c_pf_map >= 0 && w.slice < 0) ? imax(0, (w.g1 - w.g0) - 6) : -1;
         int64_t gi = 0;
         for (int s = 0; s < P.nseg; ++s) {
           const Segment &sg = P.seg[s];
@@ -744,6 +750,10 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           clip_kblocks(w, gi, kb0, kb1);
           const StageBand bd = make_band<CG>(P, sg, m0, n0);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
+            if (pf_left-- == 0) {
+              ptx::tma_prefetch_l2_4d(&prm.maps[P.c_pf_map], (int32_t)ma, (int32_t)n0, bj, bg);
+              ptx::tma_prefetch_l2_4d(&prm.maps[P.c_pf_map], (int32_t)ma, (int32_t)(n0 + BN / 2), bj, bg);
+            }
             const int rs = it % RS;
             const uint32_t ph = (it / RS) & 1;
             const int64_t k0 = kb * BK;
@@ -963,8 +973,8 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
     const int q = warp & 3;                     // TMEM lane quarter of this warp
     const int half = (warp - WARP_EPI0) >> 2;   // which 128 of the 256 columns
     constexpr int NG = BN / 2 / EC;             // column groups per thread (8)
-    uint32_t cc = 0, qi = 0, ebox = 0;
-    float *box0 = epi_stage + (warp - WARP_EPI0) * 2 * EPI_BOX;
+    uint32_t cc = 0, qi = 0;
+    const uint32_t box_s = ptx::smem_u32(epi_stage + (warp - WARP_EPI0) * EPI_BOX);
     for (;;) {
       const Work w = next_work(qi, 5, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
       if (w.tb < 0) break;
@@ -1058,55 +1068,43 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
       constexpr int SG = 8;
       if (none) {
         // nothing of this warp's 32 x 128 block is referenced (ragged edge)
-      } else if (full && P.c_map >= 0) {
-        // ---- bulk stores (NS "coalesced 128-bit epilogue stores"; DESIGN A6):
-        // the warp's whole 32 x 128 block is valid (ragged-edge and
-        // uplo-cut warps take the predicated path below).  Per group of 8
-        // columns the warp forms D = alpha*S + beta*C for its 32 rows in a
-        // 1 KiB shared box (column-major: the thread's row is the lane, so the
-        // 8 shared stores are conflict-free) and ONE lane writes the box with
-        // a TMA tensor store (128-B rows).  Two boxes per warp alternate:
-        // forming the next group overlaps the previous store's read of shared
-        // memory.  C (beta != 0) is read one group ahead, coalesced.
-        const int32_t rw0 = (int32_t)(m0 + HA * rank + q * 32), cb = (int32_t)cbase;
-        const int32_t bj = (int32_t)(w.b % per), bg = (int32_t)(w.b / per);
-        const uint32_t box_s = ptx::smem_u32(box0) + lane * 4;
+      } else if (full && P.c_vec) {
+        // ---- 16-B vector accesses of C (NS "coalesced 128-bit epilogue
+        // stores"; DESIGN A6), for warps whose whole 32 x 128 block is valid
+        // (ragged-edge and uplo-cut warps take the predicated paths below).
+        // Per group of 8 columns: alpha*S goes to the warp's shared box
+        // column-major (thread = row: conflict-free), is read back as float4s
+        // of 4 consecutive rows of one column (lane -> column lane/8 and
+        // lane/8 + 4, rows 4*(lane%8)..+3), combined with beta*C read the
+        // same way, and stored with st.global.v4: each warp instruction moves
+        // 4 columns x 128 B.  C is read one group ahead.
+        const int vr = (lane & 7) * 4, vc = lane >> 3;
+        const float *cq = P.Cin + coff + (m0 + HA * rank + q * 32 + vr) + (cbase + vc) * ldi;
+        float *oq = P.Cout + coff + (m0 + HA * rank + q * 32 + vr) + (cbase + vc) * ldo;
+        const uint32_t rd = box_s + (uint32_t)(vc * 32 + vr) * 4;       // float4 of column vc
         constexpr int NGW = BN / 2 / EPI_GW;
-        const bool l0 = lane == 0;
-        const CUtensorMap *cmap = &prm.maps[P.c_map];
-        // one group: box <- S[g*8 .. g*8+7] (alpha/beta already applied), TMA store
-        auto put = [&](int g) {
-          const uint32_t box = box_s + (ebox & 1) * (EPI_BOX * 4);
-          ptx::bulk_wait_group_read1_if(l0);         // the store that used this box has read it
+        const bool ld_on = be != 0.f;
+        float4 c0v = make_float4(0.f, 0.f, 0.f, 0.f), c1v = c0v;
+        if (ld_on) { c0v = ptx::ld_cs_v4(cq); c1v = ptx::ld_cs_v4(cq + 4 * ldi); }
+#pragma unroll
+        for (int g = 0; g < NGW; ++g) {
+#pragma unroll
+          for (int j = 0; j < EPI_GW; ++j) ptx::st_shared_f32(box_s + (j * 32 + lane) * 4, al * S[g * EPI_GW + j]);
           __syncwarp();
-#pragma unroll
-          for (int j = 0; j < EPI_GW; ++j) ptx::st_shared_f32(box + j * 128, S[g * EPI_GW + j]);
-          ptx::fence_proxy_async_smem();
-          __syncwarp();
-          ptx::tma_store_4d_commit_if(l0, cmap, box - lane * 4, rw0, cb + g * EPI_GW, bj, bg);
-          ++ebox;
-        };
-        if (be != 0.f) {
-          float cv[EPI_GW];
-#pragma unroll
-          for (int j = 0; j < EPI_GW; ++j) { cv[j] = ptx::ld_cs(cp); cp += ldi; }
-#pragma unroll
-          for (int g = 0; g < NGW; ++g) {
-#pragma unroll
-            for (int j = 0; j < EPI_GW; ++j) S[g * EPI_GW + j] = fmaf(be, cv[j], al * S[g * EPI_GW + j]);
+          float4 d0 = ptx::ld_shared_v4(rd), d1 = ptx::ld_shared_v4(rd + 4 * 128);
+          __syncwarp();                                   // box free for the next group
+          if (ld_on) {
+            d0.x = fmaf(be, c0v.x, d0.x); d0.y = fmaf(be, c0v.y, d0.y);
+            d0.z = fmaf(be, c0v.z, d0.z); d0.w = fmaf(be, c0v.w, d0.w);
+            d1.x = fmaf(be, c1v.x, d1.x); d1.y = fmaf(be, c1v.y, d1.y);
+            d1.z = fmaf(be, c1v.z, d1.z); d1.w = fmaf(be, c1v.w, d1.w);
             if (g + 1 < NGW) {
-#pragma unroll
-              for (int j = 0; j < EPI_GW; ++j) { cv[j] = ptx::ld_cs(cp); cp += ldi; }
+              cq += EPI_GW * ldi;
+              c0v = ptx::ld_cs_v4(cq); c1v = ptx::ld_cs_v4(cq + 4 * ldi);
             }
-            if (st_on) put(g);
           }
-        } else {
-#pragma unroll
-          for (int g = 0; g < NGW; ++g) {
-#pragma unroll
-            for (int j = 0; j < EPI_GW; ++j) S[g * EPI_GW + j] *= al;
-            if (st_on) put(g);
-          }
+          if (st_on) { ptx::st_cs_v4(oq, d0); ptx::st_cs_v4(oq + 4 * ldo, d1); }
+          oq += EPI_GW * ldo;
         }
       } else if (full && be == 0.f) {
         if (st_on) {
@@ -1151,10 +1149,6 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
         }
       }
       if (FUSED) {                                 // this CTA's half of the tile is stored
-        if (P.c_map >= 0 && lane == 0) {           // bulk stores complete, ordered before the signal
-          ptx::bulk_wait_group<0>();
-          ptx::fence_proxy_async_global();
-        }
         ptx::named_bar_sync(5, EPI_THREADS);
         if (threadIdx.x == WARP_EPI0 * 32) {
           BLAS3_STRACE(8, w.ph);
@@ -1169,7 +1163,6 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
       }
       if (threadIdx.x == WARP_EPI0 * 32) BLAS3_TRACE(8);
     }
-    if (lane == 0) ptx::bulk_wait_group<0>();  // shared boxes read, stores complete, before exit
     if (threadIdx.x == WARP_EPI0 * 32) BLAS3_TRACE(9);
   }
 
@@ -1284,18 +1277,25 @@ static int launch_cg(PRM &prm, cudaStream_t stream, int num_sms, bool allow_pdl 
       if (!op_maps(prm, slot, sg.b, P.N, sg.K, G::HB, per, groups, P.bs_b)) return -4;
     }
   }
-  // Cout as a TMA store target (bulk epilogue): 16-B aligned, ld % 4 == 0
+  // epilogue access of C: 16-B vectors when aligned; Cin (beta != 0) as an
+  // L2-prefetch tensor map (128-row x 128-column boxes, one per CTA half)
   for (int p = 0; p < prm.nphase; ++p) {
     Problem &P = prm.ph[p].P;
-    P.c_map = -1;
     const int64_t nb = P.nbatch > 1 ? P.nbatch : 1;
-    const bool ok = opt(BLAS3_OPT_TC_TMA_STORE) != 0 && reinterpret_cast<uintptr_t>(P.Cout) % 16 == 0 &&
-                    P.ldcout % 4 == 0 && (nb == 1 || (P.bs_c.inner % 4 == 0 && P.bs_c.outer % 4 == 0));
-    if (!ok || slot >= (int)(sizeof(prm.maps) / sizeof(prm.maps[0]))) continue;
+    auto vec_ok = [&](const float *ptr, int64_t ld, const BatchStride &bs) {
+      return reinterpret_cast<uintptr_t>(ptr) % 16 == 0 && ld % 4 == 0 &&
+             (nb == 1 || (bs.inner % 4 == 0 && bs.outer % 4 == 0));
+    };
+    const bool rd = P.beta != 0.f;
+    P.c_vec = opt(BLAS3_OPT_TC_VEC_STORE) != 0 && vec_ok(P.Cout, P.ldcout, P.bs_c) &&
+              (!rd || vec_ok(P.Cin, P.ldcin, P.bs_c)) ? 1 : 0;
+    P.c_pf_map = -1;
+    if (!rd || !opt(BLAS3_OPT_TC_C_PREFETCH) || !vec_ok(P.Cin, P.ldcin, P.bs_c) ||
+        slot >= (int)(sizeof(prm.maps) / sizeof(prm.maps[0]))) continue;
     const int64_t per = nb > 1 ? P.per : 1, groups = cdiv(nb, per);
-    if (!make_map(&prm.maps[slot], P.Cout, P.M, P.N, P.ldcout, 32, EPI_GW, CU_TENSOR_MAP_SWIZZLE_NONE, per,
+    if (!make_map(&prm.maps[slot], P.Cin, P.M, P.N, P.ldcin, HA, BN / 2, CU_TENSOR_MAP_SWIZZLE_NONE, per,
                   groups, P.bs_c)) return -4;
-    P.c_map = slot++;
+    P.c_pf_map = slot++;
   }
   // the TF32+BF16X instantiation in that mode (every phase of a fused launch
   // carries the same mode)

@@ -184,6 +184,6 @@ def test_options_roundtrip_and_validation(lib):
     assert lib.get_option("tc_kc") == 2
     for bad in (0, 3, 128):                       # power of two in [1, 64]
         assert lib.blas3_set_option(lib.OPTIONS["tc_kc"], bad) == 1
-    assert lib.get_option("tc_tma_store") == 1
+    assert lib.get_option("tc_vec_store") == 1 and lib.get_option("tc_c_prefetch") == 1
     assert lib.get_option("max_sms") == 0
-    assert len(lib.OPTIONS) == 23
+    assert len(lib.OPTIONS) == 24
