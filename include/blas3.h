@@ -208,13 +208,15 @@ int blas3_get_math_mode(void);
  *   BLAS3_OPT_TC_KC        [BLAS3_TC_KC]    tcgen05 path: k-blocks (32 deep) summed in
  *                          one TMEM partial before it is folded into the
  *                          round-to-nearest register sum (Q24): power
- *                          of 2 in [1, 64], default 2 (K = 64).  The tensor
- *                          core's accumulator truncates on every UMMA add, so
- *                          the output-relative error grows with this value:
- *                          ~4e-8 per add, coherent on same-sign data (3 adds per
- *                          8-deep k-step); measured e_rel on U(-1,1) SGEMM
- *                          16 -> 3.9e-6, 4 -> 1.1e-6, 2 -> 6.8e-7, and 2.6e-6 at
- *                          4 on an all-positive (SYRK diagonal) sum
+ *                          of 2 in [1, 64], default 4 (K = 128).  The tensor
+ *                          core's accumulator truncates on every UMMA add (~4e-8
+ *                          relative per add, coherent on same-sign data), so the
+ *                          error grows with the full-size adds per partial: the
+ *                          pair kernel issues a k-block pair's cross terms before
+ *                          its hi*hi terms (8 full-size adds per pair, 32 per
+ *                          partial at 4), the single-CTA kernel uses kc/2 blocks
+ *                          (24 adds).  Each drain costs TMEM bandwidth: SGEMM
+ *                          N=8192 at 16 / 4 / 2: 100 / ~95 / ~91 %
  *   BLAS3_OPT_TC_VEC_STORE [BLAS3_TC_VEC_STORE] tcgen05 epilogue: 1 (default) C is
  *                          read and written with 16-B vector accesses (each
  *                          warp's rows transposed through a 1 KiB shared box:

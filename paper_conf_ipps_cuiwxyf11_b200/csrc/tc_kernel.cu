@@ -67,7 +67,7 @@ constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;       // 640
 constexpr int EPI_REGS = 144, OTHER_REGS = 64;   // 36864 + 24576 = 61440
 // Chunked accumulation: the tensor core's fp32 accumulator truncates on every
 // UMMA add (Q24), so a TMEM partial only ever sums Problem::kc
-// k-blocks (BLAS3_OPT_TC_KC, default 2: K = 64) before the epilogue folds it
+// k-blocks (BLAS3_OPT_TC_KC, default 4: K = 128) before the epilogue folds it
 // into a register running sum with round-to-nearest adds; the two TMEM
 // buffers ping-pong per chunk.
 constexpr int EC = 16;                            // epilogue column group
@@ -123,6 +123,7 @@ struct Geo {
     uint64_t wk_full[TQ];    // local producer -> local roles: decoded work item published
     Work wk[TQ];
     uint64_t tfull[2];       // MMA -> epilogue: TMEM partial ready (multicast to the pair)
+    uint64_t mirror;         // transform: the mirrored view of a symmetric diagonal block landed
     uint64_t tempty[2];      // epilogue -> MMA: partial drained (one arrival per CTA, leader)
     uint32_t tmem_base;
     uint32_t split_last;     // epilogue: this CTA's slice of a split tile is the last one
@@ -362,20 +363,21 @@ __device__ __forceinline__ void load_operand(const PRM &prm, const OpDesc &o, in
 }
 
 // ---------------------------------------------------------------- transform
-// Symmetric block crossing the diagonal (staged from the rk view): elements
-// whose stored position is the mirrored one (the "shadow area")
-// are SELECTED from the stored triangle, S(r,k) := S(k,r), read straight from
-// global memory (rare blocks; keeps the raw ring free of a second view).
-__device__ __forceinline__ void sym_merge(const OpDesc &o, uint8_t *raw, int64_t r0, int64_t k0,
-                                          int rows, int64_t R, int64_t K, int t) {
-  // k fastest across a warp: the stored elements S(k, r) of one r are
-  // contiguous in memory, so each warp load is one coalesced 128-B access
+// Symmetric block crossing the diagonal (staged from the rk view, MN-major):
+// the elements whose stored position is the mirrored one (the "shadow area",
+// P:144-148) are SELECTED from the block's kr view, S(r,k) := S(k,r), which
+// the transform has TMA-loaded (K-major) into the stage's lo slot (`kr`):
+// both orientations come from the stored triangle by TMA, no per-element
+// global loads (selection, never src + src^T - diag, reading Q7).  Elements
+// outside the matrix are zero in both views (TMA zero fill).
+__device__ __forceinline__ void sym_merge(const OpDesc &o, uint8_t *raw, const uint8_t *kr, int64_t r0,
+                                          int64_t k0, int rows, int t) {
+  const int64_t d = r0 - k0;                       // gr - gk = d + r - k
   for (int e = t; e < rows * BK; e += TR_THREADS) {
-    int k = e % BK, r = e / BK;
-    int64_t gr = r0 + r, gk = k0 + k;
-    bool mirrored = o.lower ? (gr < gk) : (gr > gk);
-    if (mirrored && gr < R && gk < K)
-      *reinterpret_cast<float *>(raw + off_mn(r, k)) = __ldg(o.ptr + gk + gr * o.ld);
+    const int r = e / BK, k = e % BK;
+    const bool mirrored = o.lower ? (d + r - k < 0) : (d + r - k > 0);
+    if (mirrored)
+      *reinterpret_cast<float *>(raw + off_mn(r, k)) = *reinterpret_cast<const float *>(kr + off_k(r, k));
   }
 }
 
@@ -584,6 +586,16 @@ __device__ __forceinline__ void signal_done(const PRM &prm, const Work &w) {
   }
 }
 
+// k-blocks per TMEM partial: Problem::kc, except for the single-CTA kernel's
+// block-by-block 3xTF32 issue (12 full-size truncating adds per k-block, vs
+// 8 per k-block PAIR in the pair kernel), which halves it -- every variant
+// keeps at most 8 * kc full-size adds per partial (Q24)
+template <int CG, bool BX>
+__device__ __forceinline__ int32_t chunk_len(const Problem &P) {
+  if (CG == 1 && !BX && P.passes == 3) return P.kc > 1 ? P.kc / 2 : 1;
+  return P.kc;
+}
+
 template <int CG>
 __device__ __forceinline__ void arrive_leader(uint64_t *bar, uint32_t rank, uint32_t id,
                                               uint32_t nthreads, bool first) {
@@ -608,6 +620,13 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
   using LoBuf = typename G::LoBuf;
   using Barriers = typename G::Barriers;
   constexpr int RS = G::RS, LS = G::LS, TM = G::TM, HB = G::HB;
+  // k-block pairs (cross terms before hi*hi, see the MMA issuer) hold two raw
+  // stages until the pair's hi*hi terms: only the pair kernel's 4-deep raw
+  // ring has room to keep the producer running ahead meanwhile.  The
+  // single-CTA kernel (2 raw stages) issues block by block with chunks of
+  // kc / 2 k-blocks -- the same number of full-size truncating adds per TMEM
+  // partial (Q24).
+  constexpr bool PAIRED = CG == 2;
   extern __shared__ uint8_t smem_raw[];
   // 1024-B aligned base by pointer arithmetic on the __shared__ array (not via
   // an integer round trip), so the compiler keeps the shared address space and
@@ -641,6 +660,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
       ptx::mbar_init(&bars->tfull[a], 1);
       ptx::mbar_init(&bars->tempty[a], CG);
     }
+    ptx::mbar_init(&bars->mirror, 1);
     ptx::fence_mbar_init();
   }
   if (warp == WARP_MMA) ptx::tmem_alloc<CG>(&bars->tmem_base, TMEM_COLS);
@@ -786,8 +806,12 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
         const int64_t m0 = w.m0, n0 = w.n0;
         const int64_t nkb = w.g1 - w.g0;
         int64_t done = 0;
-        const int64_t kc = P.kc;
+        int32_t chunk_left = 0;                     // k-blocks left in the open TMEM chunk
         uint32_t accumulate = 0, buf = 0;
+        // the first block of a k-block pair whose hi*hi terms are still to issue
+        bool pend_valid = false;
+        uint32_t pend_hiA = 0, pend_hiB = 0, pend_idesc = 0;
+        int pend_layA = 0, pend_layB = 0, pend_rs = 0;
         auto open_chunk = [&]() {
           buf = cc & 1;
           const uint32_t aph = (cc >> 1) & 1;
@@ -818,7 +842,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           clip_kblocks(w, gi, kb0, kb1);
           const StageBand bd = make_band<CG>(P, sg, m0, n0);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
-            if (done % kc == 0) open_chunk();
+            if (chunk_left == 0) { open_chunk(); chunk_left = chunk_len<CG, BX>(P); }
             const uint32_t d_tmem = tmem + buf * BN;
             const int rs = it % RS, ls = it % LS;
             const uint32_t lph = (it / LS) & 1;
@@ -831,11 +855,52 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
               const uint32_t hiA = ptx::smem_u32(raw[rs].A), hiB = ptx::smem_u32(raw[rs].B);
               const uint32_t loA = ptx::smem_u32(lo[ls].A), loB = ptx::smem_u32(lo[ls].B);
               const uint32_t idesc = ptx::idesc_tf32(TM, BN, si.layA == LAYOUT_MN, si.layB == LAYOUT_MN);
+              const bool one = (P.dbg & 2) || P.passes == 1;
+              auto mma = [&](uint64_t a, uint64_t b, uint32_t id, uint32_t acc) {
+                if constexpr (CG == 1) ptx::mma_tf32_ss(d_tmem, a, b, id, acc);
+                else ptx::mma_tf32_ss_pair(d_tmem, a, b, id, acc);
+              };
+              auto commit = [&](uint64_t *bar) {
+                if constexpr (CG == 1) ptx::mma_commit(bar);
+                else ptx::mma_commit_pair(bar, 0x3);
+              };
+              if (!BX && !one && PAIRED && !(P.dbg & 8)) {
+                // 3xTF32, k-block pairs (Q24): both cross terms of
+                // the pair first, while the fresh TMEM partial is still ~2^-11
+                // of its final size (their truncation is negligible), then the
+                // two blocks' hi*hi terms: 8 full-size truncating adds per
+                // pair instead of 24.  The lo slot is released after the cross
+                // terms, the raw slot after the hi*hi terms.
+#pragma unroll
+                for (int k8 = 0; k8 < BK / 8; ++k8) {
+                  mma(op_desc(loA, si.layA, k8), op_desc(hiB, si.layB, k8), idesc, accumulate);
+                  mma(op_desc(hiA, si.layA, k8), op_desc(loB, si.layB, k8), idesc, 1);
+                  accumulate = 1;
+                }
+                commit(&bars->lo_empty[ls]);
+                const bool last = chunk_left == 1 || done + 1 == nkb;
+                if (pend_valid || last) {
+                  if (pend_valid) {
+#pragma unroll
+                    for (int k8 = 0; k8 < BK / 8; ++k8)
+                      mma(op_desc(pend_hiA, pend_layA, k8), op_desc(pend_hiB, pend_layB, k8), pend_idesc, 1);
+                    commit(&bars->empty[pend_rs]);
+                    pend_valid = false;
+                  }
+#pragma unroll
+                  for (int k8 = 0; k8 < BK / 8; ++k8)
+                    mma(op_desc(hiA, si.layA, k8), op_desc(hiB, si.layB, k8), idesc, 1);
+                  commit(&bars->empty[rs]);
+                } else {                                   // first block of a pair: hi*hi later
+                  pend_valid = true;
+                  pend_hiA = hiA; pend_hiB = hiB; pend_idesc = idesc;
+                  pend_layA = si.layA; pend_layB = si.layB; pend_rs = rs;
+                }
+              } else {
 #pragma unroll
               for (int k8 = 0; k8 < BK / 8; ++k8) {
                 const uint64_t ah = op_desc(hiA, si.layA, k8), al = op_desc(loA, si.layA, k8);
                 const uint64_t bh = op_desc(hiB, si.layB, k8), bl = op_desc(loB, si.layB, k8);
-                const bool one = (P.dbg & 2) || P.passes == 1;
                 if (P.dbg & 8) continue;                       // diag: no MMAs
                 if constexpr (BX) {
                   // packed cross terms (one bf16 UMMA, K = 16, K-major) + hi*hi (tf32)
@@ -852,31 +917,21 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
                   accumulate = 1;
                   continue;
                 }
-                if constexpr (CG == 1) {
-                  if (!one) ptx::mma_tf32_ss(d_tmem, al, bh, idesc, accumulate);
-                  if (!one) ptx::mma_tf32_ss(d_tmem, ah, bl, idesc, 1);
-                  ptx::mma_tf32_ss(d_tmem, ah, bh, idesc, one ? accumulate : 1);
-                } else {
-                  if (!one) ptx::mma_tf32_ss_pair(d_tmem, al, bh, idesc, accumulate);
-                  if (!one) ptx::mma_tf32_ss_pair(d_tmem, ah, bl, idesc, 1);
-                  ptx::mma_tf32_ss_pair(d_tmem, ah, bh, idesc, one ? accumulate : 1);
-                }
+                if (!one) mma(al, bh, idesc, accumulate);
+                if (!one) mma(ah, bl, idesc, 1);
+                mma(ah, bh, idesc, one ? accumulate : 1);
                 accumulate = 1;
               }
               BLAS3_TRACE(6);
-              if constexpr (CG == 1) {
-                ptx::mma_commit(&bars->empty[rs]);
-                ptx::mma_commit(&bars->lo_empty[ls]);
-              } else {
-                ptx::mma_commit_pair(&bars->empty[rs], 0x3);
-                ptx::mma_commit_pair(&bars->lo_empty[ls], 0x3);
+              commit(&bars->empty[rs]);
+              commit(&bars->lo_empty[ls]);
               }
             }
             accumulate = 1;
             __syncwarp();
             ++done;
             if (lane == 0 && done == nkb) BLAS3_STRACE(5, w.ph);
-            if (done % kc == 0 || done == nkb) close_chunk(true);
+            if (--chunk_left == 0 || done == nkb) close_chunk(true);
           }
         }
       }
@@ -886,7 +941,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
     // ============================ transform warps (own halves; arrive at the leader)
     BLAS3_DEC_REGS();
     const int tt = threadIdx.x - WARP_TR0 * 32;
-    uint32_t it = 0, qi = 0;
+    uint32_t it = 0, qi = 0, mirror_ph = 0;
     for (;;) {
       const Work w = next_work(qi, 4, TR_THREADS, tt == 0);
       if (w.tb < 0) break;
@@ -905,6 +960,20 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           const uint32_t ph = (it / RS) & 1, lph = (it / LS) & 1;
           const int64_t k0 = kb * BK;
           const StageInfo si = stage_at<CG>(bd, P, sg, m0, n0, kb);
+          // symmetric diagonal block: its mirrored (kr) view goes to this
+          // stage's lo slot first (free once the MMA released it), loaded by
+          // TMA beside the raw (rk) view, and is merged from shared memory
+          const bool symA = si.clsA == BLK_SYM_DIAG, symB = si.clsB == BLK_SYM_DIAG;
+          if (symA || symB) {
+            ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
+            if (tt == 0) {
+              const int64_t per = P.per > 0 ? P.per : 1;
+              const int32_t bj = (int32_t)(w.b % per), bg = (int32_t)(w.b / per);
+              ptx::mbar_arrive_expect_tx(&bars->mirror, (symA ? HA * BK * 4 : 0) + (symB ? HB * BK * 4 : 0));
+              if (symA) load_operand(prm, sg.a, LAYOUT_K, lo[ls].A, ma, k0, HA, &bars->mirror, bj, bg);
+              if (symB) load_operand(prm, sg.b, LAYOUT_K, lo[ls].B, nb, k0, HB, &bars->mirror, bj, bg);
+            }
+          }
           ptx::mbar_wait(&bars->full[rs], ph);
           if (tt == 0) BLAS3_TRACE(4);
           if (tt == 0 && kb == kb0) BLAS3_STRACE(2, w.ph);
@@ -914,14 +983,19 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           // in the nonzero region needs none, an entirely blank half is a
           // vectorised zero-fill, only halves touching the diagonal go per element
           const int64_t k1 = imin(sg.K, k0 + BK);
-          if (si.clsA == BLK_SYM_DIAG) { sym_merge(sg.a, rb.A, ma, k0, HA, P.M, sg.K, tt); fix = true; }
-          else if (si.clsA == BLK_TRI_DIAG) {
+          if (symA || symB) {
+            ptx::mbar_wait(&bars->mirror, mirror_ph);
+            mirror_ph ^= 1;
+            if (symA) sym_merge(sg.a, rb.A, lo[ls].A, ma, k0, HA, tt);
+            if (symB) sym_merge(sg.b, rb.B, lo[ls].B, nb, k0, HB, tt);
+            ptx::named_bar_sync(1, TR_THREADS);       // merged; the lo slot is free again for the split
+          }
+          if (si.clsA == BLK_TRI_DIAG) {
             const int own = block_class(sg.a, ma, imin(P.M, ma + HA), k0, k1);
             if (own == BLK_ZERO) { zero_fill(rb.A, G::A_BYTES, tt); fix = true; }
             else if (own == BLK_TRI_DIAG && !(P.dbg & 32)) { tri_fix(sg.a, si.layA, rb.A, ma, k0, HA, P.M, sg.K, tt); fix = true; }
           }
-          if (si.clsB == BLK_SYM_DIAG) { sym_merge(sg.b, rb.B, nb, k0, HB, P.N, sg.K, tt); fix = true; }
-          else if (si.clsB == BLK_TRI_DIAG) {
+          if (si.clsB == BLK_TRI_DIAG) {
             const int own = block_class(sg.b, nb, imin(P.N, nb + HB), k0, k1);
             if (own == BLK_ZERO) { zero_fill(rb.B, G::B_BYTES, tt); fix = true; }
             else if (own == BLK_TRI_DIAG && !(P.dbg & 32)) { tri_fix(sg.b, si.layB, rb.B, nb, k0, HB, P.N, sg.K, tt); fix = true; }
@@ -983,7 +1057,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
       const int64_t coff = (P.nbatch > 1) ? batch_off(P.bs_c, w.b, per) : 0;
       const int64_t m0 = w.m0, n0 = w.n0;
       const int64_t nkb = w.g1 - w.g0;
-      const int64_t nchunks = nkb > 0 ? cdiv(nkb, P.kc) : 1;
+      const int64_t nchunks = nkb > 0 ? cdiv(nkb, chunk_len<CG, BX>(P)) : 1;
       float S[NG * EC];
 #pragma unroll
       for (int i = 0; i < NG * EC; ++i) S[i] = 0.f;
@@ -1473,7 +1547,7 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
   prm.nphase = 1;
   prm.ph[0].P = P0;
   prm.ph[0].P.dbg = debug_bits();
-  if (prm.ph[0].P.kc <= 0) prm.ph[0].P.kc = 2;
+  if (prm.ph[0].P.kc <= 0) prm.ph[0].P.kc = 4;
   const int cg = choose_cg(prm.ph[0].P, num_sms);
   const bool dyn = opt(BLAS3_OPT_TC_STATIC) == 0;
   if (cg == 2) plan_split<2>(prm, num_sms); else plan_split<1>(prm, num_sms);
@@ -1529,7 +1603,7 @@ int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int 
     PhaseDesc &ph = prm.ph[p];
     ph.P = phases[p].P;
     ph.P.dbg = debug_bits();
-    if (ph.P.kc <= 0) ph.P.kc = 2;
+    if (ph.P.kc <= 0) ph.P.kc = 4;
     if (!tc_eligible(ph.P) || ph.P.max_sms) return -1;
     const int64_t nb = ph.P.nbatch > 1 ? ph.P.nbatch : 1;
     ph.tiles_per = TL::count(ph.P);

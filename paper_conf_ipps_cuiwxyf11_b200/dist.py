@@ -202,6 +202,40 @@ def _b3():
     return b3
 
 
+class _Pipeline:
+    """Comm-stream broadcast of A's panels, each consumed on the compute
+    stream once it has landed; local kernels leave `reserve_sms` SMs to NCCL
+    while panels are in flight."""
+
+    def __init__(self, b3, reserve_sms):
+        import torch
+        self.torch = torch
+        self.b3 = b3
+        self.compute = torch.cuda.current_stream()
+        self.comm = torch.cuda.Stream()
+        self.comm.wait_stream(self.compute)
+        self.reserve = max(0, int(reserve_sms))
+
+    def run(self, panels, send, consume):
+        torch = self.torch
+        evs = []
+        for p0, p1 in panels:                      # enqueue every broadcast up front
+            with torch.cuda.stream(self.comm):
+                send(p0, p1)
+                ev = torch.cuda.Event()
+                ev.record(self.comm)
+            evs.append(ev)
+        nsm = torch.cuda.get_device_properties(self.compute.device).multi_processor_count
+        for i, ((p0, p1), ev) in enumerate(zip(panels, evs)):
+            self.compute.wait_event(ev)
+            last = i == len(panels) - 1
+            if self.reserve and not last:
+                with self.b3.options(max_sms=max(2, nsm - self.reserve)):
+                    consume(i, p0, p1)
+            else:
+                consume(i, p0, p1)
+
+
 def sgemm(transa, transb, alpha, A, B_slab, beta, C_slab, root=0, group=None, panels=8,
           pipeline=None, reserve_sms=16):
     """C_slab <- alpha*op(A)*op(B)_slab + beta*C_slab on this rank's columns.

@@ -21,12 +21,17 @@ what = sys.argv[1:] or ["acc", "speed"]
 
 if "acc" in what:
     m = n = 1024
-    for k in [512, 2048, 8192, 16384]:
-        A = gen.uniform(m, k, "kc-a", k); B = gen.uniform(k, n, "kc-b", k)
+    for k, lo in [(512, -1.0), (2048, -1.0), (8192, -1.0), (16384, -1.0), (512, 0.0), (8192, 0.0)]:
+        A = gen.uniform(m, k, "kc-a", k, lo=lo); B = gen.uniform(k, n, "kc-b", k, lo=lo)
         ref = A.astype(np.float64) @ B.astype(np.float64)
         rel = lambda got: float(np.linalg.norm(np.asarray(got, np.float64) - ref) / np.linalg.norm(ref))  # noqa
-        row = [f"k={k:6d}", f"np_fp32={rel(A @ B):.2e}"]
+        row = [f"k={k:6d}{' U(0,1)' if lo == 0.0 else ' U(-1,1)'}", f"np_fp32={rel(A @ B):.2e}"]
         dA, dB = b3.from_fortran(A), b3.from_fortran(B)
+        for cta in (2, 1):                                # pair (paired issue) vs single-CTA kernel
+            with b3.options(tc_cta=cta, tc_split=0):
+                dC = b3.colmajor(m, n, fill=0.0)
+                b3.sgemm("N", "N", 1.0, dA, dB, 0.0, dC)
+                row.append(f"3x_default_cta{cta}={rel(dC.cpu().numpy()):.2e}")
         b3.set_math_mode("simt")
         dC = b3.colmajor(m, n, fill=0.0)
         b3.sgemm("N", "N", 1.0, dA, dB, 0.0, dC)
