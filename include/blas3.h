@@ -207,16 +207,16 @@ int blas3_get_math_mode(void);
  *                          the built-in default (8)
  *   BLAS3_OPT_TC_KC        [BLAS3_TC_KC]    tcgen05 path: k-blocks (32 deep) summed in
  *                          one TMEM partial before it is folded into the
- *                          round-to-nearest register sum (Q24): power
- *                          of 2 in [1, 64], default 4 (K = 128).  The tensor
- *                          core's accumulator truncates on every UMMA add (~4e-8
- *                          relative per add, coherent on same-sign data), so the
- *                          error grows with the full-size adds per partial: the
- *                          pair kernel issues a k-block pair's cross terms before
- *                          its hi*hi terms (8 full-size adds per pair, 32 per
- *                          partial at 4), the single-CTA kernel uses kc/2 blocks
- *                          (24 adds).  Each drain costs TMEM bandwidth: SGEMM
- *                          N=8192 at 16 / 4 / 2: 100 / ~95 / ~91 %
+ *                          round-to-nearest register sum (Q24): 1..64,
+ *                          default 3 (K = 96).  The tensor core's accumulator
+ *                          truncates on every UMMA add (~4e-8 relative per add,
+ *                          coherent on same-sign data); each k-block issues its
+ *                          8 cross-term UMMAs before its 4 hi*hi ones, so a
+ *                          partial of c blocks takes 12c - 8 full-size adds.
+ *                          Measured (SGEMM, K = 8192): e_rel 7.9e-7 on U(-1,1),
+ *                          1.66e-6 on U(0,1) at 3; 3.8e-6 / 9.9e-6 at 16.  Each
+ *                          drain stalls the tensor pipe briefly: SGEMM N = 8192
+ *                          at 2 / 3 / 4 / 16 = 89 / 98 / 98 / 100 %
  *   BLAS3_OPT_TC_VEC_STORE [BLAS3_TC_VEC_STORE] tcgen05 epilogue: 1 (default) C is
  *                          read and written with 16-B vector accesses (each
  *                          warp's rows transposed through a 1 KiB shared box:

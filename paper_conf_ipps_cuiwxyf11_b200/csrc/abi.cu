@@ -47,7 +47,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TRSM_FIRST_SPLIT", 0, 0, 8192, true},
     {"BLAS3_TRSM_FIRST_ALL", 0, 0, 1, false},
     {"BLAS3_TC_RASTER", 0, 0, 64, false},
-    {"BLAS3_TC_KC", 4, 1, 64, true},
+    {"BLAS3_TC_KC", 3, 1, 64, false},
     {"BLAS3_TC_VEC_STORE", 1, 0, 1, false},
     {"BLAS3_MAX_SMS", 0, 0, 4096, false},
     {"BLAS3_TC_C_PREFETCH", 1, 0, 1, false},

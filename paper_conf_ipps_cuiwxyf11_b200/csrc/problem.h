@@ -75,7 +75,8 @@ struct Problem {
   // set, never used by tests or the bench): bit0 skip the split pass,
   // bit1 issue only hi*hi (1xTF32), bit2 skip the epilogue stores,
   // bit3 issue no MMAs (commits only), bit4 issue no TMA loads,
-  // bit5 skip the triangular zero-select/unit-diagonal fix-up
+  // bit5 skip the triangular zero-select/unit-diagonal fix-up,
+  // bit6 skip the TMEM loads of the epilogue's chunk drains
   int32_t dbg;
   // launch at most this many SMs' worth of CTAs (0: all).  The STRSM driver
   // leaves SMs free for its latency-bound side-stream kernels this way.

@@ -586,16 +586,6 @@ __device__ __forceinline__ void signal_done(const PRM &prm, const Work &w) {
   }
 }
 
-// k-blocks per TMEM partial: Problem::kc, except for the single-CTA kernel's
-// block-by-block 3xTF32 issue (12 full-size truncating adds per k-block, vs
-// 8 per k-block PAIR in the pair kernel), which halves it -- every variant
-// keeps at most 8 * kc full-size adds per partial (Q24)
-template <int CG, bool BX>
-__device__ __forceinline__ int32_t chunk_len(const Problem &P) {
-  if (CG == 1 && !BX && P.passes == 3) return P.kc > 1 ? P.kc / 2 : 1;
-  return P.kc;
-}
-
 template <int CG>
 __device__ __forceinline__ void arrive_leader(uint64_t *bar, uint32_t rank, uint32_t id,
                                               uint32_t nthreads, bool first) {
@@ -620,13 +610,6 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
   using LoBuf = typename G::LoBuf;
   using Barriers = typename G::Barriers;
   constexpr int RS = G::RS, LS = G::LS, TM = G::TM, HB = G::HB;
-  // k-block pairs (cross terms before hi*hi, see the MMA issuer) hold two raw
-  // stages until the pair's hi*hi terms: only the pair kernel's 4-deep raw
-  // ring has room to keep the producer running ahead meanwhile.  The
-  // single-CTA kernel (2 raw stages) issues block by block with chunks of
-  // kc / 2 k-blocks -- the same number of full-size truncating adds per TMEM
-  // partial (Q24).
-  constexpr bool PAIRED = CG == 2;
   extern __shared__ uint8_t smem_raw[];
   // 1024-B aligned base by pointer arithmetic on the __shared__ array (not via
   // an integer round trip), so the compiler keeps the shared address space and
@@ -808,10 +791,6 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
         int64_t done = 0;
         int32_t chunk_left = 0;                     // k-blocks left in the open TMEM chunk
         uint32_t accumulate = 0, buf = 0;
-        // the first block of a k-block pair whose hi*hi terms are still to issue
-        bool pend_valid = false;
-        uint32_t pend_hiA = 0, pend_hiB = 0, pend_idesc = 0;
-        int pend_layA = 0, pend_layB = 0, pend_rs = 0;
         auto open_chunk = [&]() {
           buf = cc & 1;
           const uint32_t aph = (cc >> 1) & 1;
@@ -842,7 +821,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           clip_kblocks(w, gi, kb0, kb1);
           const StageBand bd = make_band<CG>(P, sg, m0, n0);
           for (int64_t kb = kb0; kb < kb1; ++kb, ++it) {
-            if (chunk_left == 0) { open_chunk(); chunk_left = chunk_len<CG, BX>(P); }
+            if (chunk_left == 0) { open_chunk(); chunk_left = P.kc; }
             const uint32_t d_tmem = tmem + buf * BN;
             const int rs = it % RS, ls = it % LS;
             const uint32_t lph = (it / LS) & 1;
@@ -864,38 +843,25 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
                 if constexpr (CG == 1) ptx::mma_commit(bar);
                 else ptx::mma_commit_pair(bar, 0x3);
               };
-              if (!BX && !one && PAIRED && !(P.dbg & 8)) {
-                // 3xTF32, k-block pairs (Q24): both cross terms of
-                // the pair first, while the fresh TMEM partial is still ~2^-11
-                // of its final size (their truncation is negligible), then the
-                // two blocks' hi*hi terms: 8 full-size truncating adds per
-                // pair instead of 24.  The lo slot is released after the cross
-                // terms, the raw slot after the hi*hi terms.
+              if (!BX && !one && !(P.dbg & 8)) {
+                // 3xTF32: the block's 8 cross-term UMMAs first, then its 4
+                // hi*hi UMMAs.  In the first block of a TMEM partial the
+                // cross terms land in a fresh accumulator still ~2^-11 of its
+                // final size, where the accumulator's truncation costs nothing
+                // (Q24): a partial of c k-blocks takes 12c - 8
+                // full-size truncating adds instead of 12c.
 #pragma unroll
                 for (int k8 = 0; k8 < BK / 8; ++k8) {
                   mma(op_desc(loA, si.layA, k8), op_desc(hiB, si.layB, k8), idesc, accumulate);
                   mma(op_desc(hiA, si.layA, k8), op_desc(loB, si.layB, k8), idesc, 1);
                   accumulate = 1;
                 }
+#pragma unroll
+                for (int k8 = 0; k8 < BK / 8; ++k8)
+                  mma(op_desc(hiA, si.layA, k8), op_desc(hiB, si.layB, k8), idesc, 1);
+                BLAS3_TRACE(6);
+                commit(&bars->empty[rs]);
                 commit(&bars->lo_empty[ls]);
-                const bool last = chunk_left == 1 || done + 1 == nkb;
-                if (pend_valid || last) {
-                  if (pend_valid) {
-#pragma unroll
-                    for (int k8 = 0; k8 < BK / 8; ++k8)
-                      mma(op_desc(pend_hiA, pend_layA, k8), op_desc(pend_hiB, pend_layB, k8), pend_idesc, 1);
-                    commit(&bars->empty[pend_rs]);
-                    pend_valid = false;
-                  }
-#pragma unroll
-                  for (int k8 = 0; k8 < BK / 8; ++k8)
-                    mma(op_desc(hiA, si.layA, k8), op_desc(hiB, si.layB, k8), idesc, 1);
-                  commit(&bars->empty[rs]);
-                } else {                                   // first block of a pair: hi*hi later
-                  pend_valid = true;
-                  pend_hiA = hiA; pend_hiB = hiB; pend_idesc = idesc;
-                  pend_layA = si.layA; pend_layB = si.layB; pend_rs = rs;
-                }
               } else {
 #pragma unroll
               for (int k8 = 0; k8 < BK / 8; ++k8) {
@@ -1057,7 +1023,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
       const int64_t coff = (P.nbatch > 1) ? batch_off(P.bs_c, w.b, per) : 0;
       const int64_t m0 = w.m0, n0 = w.n0;
       const int64_t nkb = w.g1 - w.g0;
-      const int64_t nchunks = nkb > 0 ? cdiv(nkb, chunk_len<CG, BX>(P)) : 1;
+      const int64_t nchunks = nkb > 0 ? cdiv(nkb, P.kc) : 1;
       float S[NG * EC];
 #pragma unroll
       for (int i = 0; i < NG * EC; ++i) S[i] = 0.f;
@@ -1067,15 +1033,21 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
         ptx::tc_fence_after();
         if (threadIdx.x == WARP_EPI0 * 32) BLAS3_TRACE(7);
         if (threadIdx.x == WARP_EPI0 * 32 && c == nchunks - 1) BLAS3_STRACE(6, w.ph);
-        if (nkb > 0) {
+        if (nkb > 0 && !(P.dbg & 64)) {        // (diag knob 64: no drain loads, results wrong)
+          // two 16-column loads in flight per wait: half the TMEM round trips
+          // of the drain, which bounds how short a chunk can be without
+          // stalling the MMA issuer on the accumulator hand-back
+          const uint32_t ta = tmem + buf * BN + half * (BN / 2) + ((uint32_t)(q * 32) << 16);
 #pragma unroll
-          for (int g = 0; g < NG; ++g) {
-            uint32_t v[EC];
-            ptx::tmem_ld_32x32b_x16(tmem + buf * BN + half * (BN / 2) + g * EC +
-                                        ((uint32_t)(q * 32) << 16), v);
+          for (int g = 0; g < NG; g += 2) {
+            uint32_t v[EC], u[EC];
+            ptx::tmem_ld_32x32b_x16(ta + g * EC, v);
+            ptx::tmem_ld_32x32b_x16(ta + (g + 1) * EC, u);
             ptx::tmem_ld_wait();
 #pragma unroll
             for (int j = 0; j < EC; ++j) S[g * EC + j] += __uint_as_float(v[j]);
+#pragma unroll
+            for (int j = 0; j < EC; ++j) S[(g + 1) * EC + j] += __uint_as_float(u[j]);
           }
         }
         ptx::tc_fence_before();
@@ -1547,7 +1519,7 @@ int launch_tc(const Problem &P0, cudaStream_t stream, int num_sms) {
   prm.nphase = 1;
   prm.ph[0].P = P0;
   prm.ph[0].P.dbg = debug_bits();
-  if (prm.ph[0].P.kc <= 0) prm.ph[0].P.kc = 4;
+  if (prm.ph[0].P.kc <= 0) prm.ph[0].P.kc = 3;
   const int cg = choose_cg(prm.ph[0].P, num_sms);
   const bool dyn = opt(BLAS3_OPT_TC_STATIC) == 0;
   if (cg == 2) plan_split<2>(prm, num_sms); else plan_split<1>(prm, num_sms);
@@ -1603,7 +1575,7 @@ int launch_tc_fused(const FusedPhase *phases, int nph, cudaStream_t stream, int 
     PhaseDesc &ph = prm.ph[p];
     ph.P = phases[p].P;
     ph.P.dbg = debug_bits();
-    if (ph.P.kc <= 0) ph.P.kc = 4;
+    if (ph.P.kc <= 0) ph.P.kc = 3;
     if (!tc_eligible(ph.P) || ph.P.max_sms) return -1;
     const int64_t nb = ph.P.nbatch > 1 ? ph.P.nbatch : 1;
     ph.tiles_per = TL::count(ph.P);

@@ -181,8 +181,8 @@ def test_options_roundtrip_and_validation(lib):
     assert lib.blas3_set_option(lib.OPTIONS["tc_cta"], 3) == 1
     assert lib.blas3_set_option(99, 0) == 1
     assert lib.blas3_get_option(99) == -(2 ** 63)
-    assert lib.get_option("tc_kc") == 4
-    for bad in (0, 3, 128):                       # power of two in [1, 64]
+    assert lib.get_option("tc_kc") == 3
+    for bad in (0, -1, 65, 128):                  # in [1, 64]
         assert lib.blas3_set_option(lib.OPTIONS["tc_kc"], bad) == 1
     assert lib.get_option("tc_vec_store") == 1 and lib.get_option("tc_c_prefetch") == 1
     assert lib.get_option("max_sms") == 0

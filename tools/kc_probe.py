@@ -16,7 +16,7 @@ sys.path.insert(0, ".")
 import blas3_inputs as gen  # noqa: E402
 import paper_conf_ipps_cuiwxyf11_b200 as b3  # noqa: E402
 
-KCS = [1, 2, 4, 8, 16]
+KCS = [1, 2, 3, 4, 8, 16]
 what = sys.argv[1:] or ["acc", "speed"]
 
 if "acc" in what:

@@ -59,7 +59,10 @@ keys = ["gpu__time_duration.sum", "sm__cycles_elapsed.avg.per_second",
         "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
         "launch__registers_per_thread", "launch__shared_mem_per_block_dynamic",
         "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio",
-        "smsp__sass_inst_executed_op_utcmma.sum"]
+        "smsp__sass_inst_executed_op_utcmma.sum",
+        "smsp__sass_inst_executed_op_global_st.sum", "smsp__sass_inst_executed_op_global_ld.sum",
+        "smsp__sass_inst_executed_op_shared_st.sum", "smsp__sass_inst_executed_op_shared_ld.sum",
+        "smsp__inst_executed_op_ldgsts.sum", "lts__t_sectors_srcunit_tex_op_write.sum"]
 vals = {}
 for k in keys:
     v, u = get(k)
@@ -89,9 +92,12 @@ with open(f"profiles/{tag}_sgemm_ncu.md", "w") as f:
     f.write(f"\nDRAM traffic per launch: {traffic/1e6:.1f} MB vs algorithmic minimum "
             f"{alg_bytes/1e6:.1f} MB (A, B, C read once + C written once) -> "
             f"{traffic/alg_bytes:.2f}x\n")
+stamp = os.path.join("paper_conf_ipps_cuiwxyf11_b200", "libblas3.so.sha256")
+lib_sha = open(stamp).read().strip() if os.path.exists(stamp) else None
 json.dump({"tag": tag, "kernel": "tc_structured_gemm (sgemm NN N=8192)",
            "dram_bytes_per_launch": traffic, "dram_read": rd, "dram_write": wr,
-           "algorithmic_bytes": alg_bytes, "source": f"profiles/{tag}_sgemm_ncu.md"},
+           "algorithmic_bytes": alg_bytes, "source": f"profiles/{tag}_sgemm_ncu.md",
+           "lib_sha256": lib_sha},
           open("profiles/ncu_sgemm_traffic.json", "w"), indent=1)
 print(open(f"profiles/{tag}_launches.md").read())
 print(open(f"profiles/{tag}_sgemm_ncu.md").read())
