@@ -523,7 +523,7 @@ def run_ours(args):
             if tj.get("lib_sha256") and tj.get("lib_sha256") == cur:
                 traffic, traffic_src = tj.get("dram_bytes_per_launch"), tj.get("source")
             else:
-                traffic_src = f"stale: {tp} is a capture of another build"
+                traffic_src = "stale: profiles/ncu_sgemm_traffic.json is a capture of another build"
         except (ValueError, OSError):
             traffic = None
     h2d = (2 * n * n * 4 if rank == 0 else 0) + 2 * n * cols * 4

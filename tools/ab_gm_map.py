@@ -1,7 +1,7 @@
 """GM_map (pre-materialised operand) versus in-kernel staging, interleaved A/B
 per variant at N = 4096 and 8192 (tune.search).  Writes profiles/<tag>_gm_map.md.
 
-python tools/ab_gm_map.py [tag]
+python tools/ab_gm_map.py [tag] [routines,comma,separated] [sizes,comma,separated]
 """
 import itertools, json, os, sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -11,8 +11,10 @@ import paper_conf_ipps_cuiwxyf11_b200 as b3
 from paper_conf_ipps_cuiwxyf11_b200 import tune
 
 tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
+only = set(sys.argv[2].split(",")) if len(sys.argv) > 2 else None
+sizes = [int(x) for x in sys.argv[3].split(",")] if len(sys.argv) > 3 else [4096, 8192]
 rows = []
-for n in (4096, 8192):
+for n in sizes:
     A = b3.colmajor(n, n); A.uniform_(-1, 1)
     B = b3.colmajor(n, n); B.uniform_(-1, 1)
     C = b3.colmajor(n, n); C.uniform_(-1, 1)
@@ -28,6 +30,8 @@ for n in (4096, 8192):
         cases.append(("strsm", sd + ul + ta + "N", 1.0 * n ** 3,
                       lambda sd=sd, ul=ul, ta=ta: b3.strsm(sd, ul, ta, "N", 1.0, T, X)))
     for routine, var, fl, fn in cases:
+        if only and routine not in only:
+            continue
         best, table = tune.search(fn, [{"gm_map": 0}, {"gm_map": 1}], reps=3, rounds=4)
         t0, t1 = table[0][1], table[1][1]
         r = {"routine": routine, "variant": var, "n": n, "staged_tflops": round(fl / t0 / 1e9, 1),
