@@ -158,7 +158,9 @@ int blas3_get_math_mode(void);
  *                          memory first.  -1 auto (default: per-routine size
  *                          thresholds below), 0 never, 1 always
  *   BLAS3_OPT_GM_MIN_GEMM  SGEMM transa!='N': auto threshold on n (default 1<<30 = off)
- *   BLAS3_OPT_GM_MIN_SYMM  SSYMM: auto threshold on the non-symmetric extent (2048)
+ *   BLAS3_OPT_GM_MIN_SYMM  SSYMM: auto threshold on the non-symmetric extent (1<<30 = off:
+ *                          sym(A) is merged while staging, the paper's rule 3, P:144-158;
+ *                          within 1-5% of GM_map at N >= 4096, faster for side=L at 2048)
  *   BLAS3_OPT_GM_MIN_TRMM  STRMM: auto threshold on the right-hand-side extent (1<<30)
  *   BLAS3_OPT_GM_MIN_TRSM  STRSM transa!='N': auto threshold on the RHS extent (1<<30)
  *                          (auto also requires the structured order >= 2048)
@@ -169,9 +171,9 @@ int blas3_get_math_mode(void);
  *   BLAS3_OPT_PDL          [BLAS3_PDL]      1 programmatic dependent launch (default), 0 off
  *   BLAS3_OPT_TRSM_NB      [BLAS3_TRSM_NB]  STRSM panel width: power of 2 in [128, 8192] (2048)
  *   BLAS3_OPT_TRSM_SLABS   [BLAS3_TRSM_SLABS] right-hand-side slabs on own streams, 1..4 (2)
- *   BLAS3_OPT_TRSM_SLAB_MIN [BLAS3_TRSM_SLAB_MIN] minimum slab width, >= 256 (4096:
- *                          one slab below 8192 right-hand sides -- measured 12%
- *                          faster at 4096 -- two from 8192)
+ *   BLAS3_OPT_TRSM_SLAB_MIN [BLAS3_TRSM_SLAB_MIN] minimum slab width, >= 256 (16384:
+ *                          one slab up to 32767 right-hand sides -- measured 5.6%
+ *                          faster than two at 8192, profiles/r02_trsm_options.md)
  *   BLAS3_OPT_TRSM_RESERVE [BLAS3_TRSM_RESERVE] SMs the first panel's sweep leaves to
  *                          the panel-inverse doubling chain, 0..74 (48)
  *   BLAS3_OPT_TRSM_GEO_LEAF [BLAS3_TRSM_GEO_LEAF] the first panel is halved down to

@@ -29,7 +29,7 @@ struct OptSpec { const char *env; int64_t def, lo, hi; bool pow2; };
 static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_GM_MAP", -1, -1, 1, false},
     {"BLAS3_GM_MIN_GEMM", int64_t(1) << 30, 0, int64_t(1) << 40, false},
-    {"BLAS3_GM_MIN_SYMM", 2048, 0, int64_t(1) << 40, false},
+    {"BLAS3_GM_MIN_SYMM", int64_t(1) << 30, 0, int64_t(1) << 40, false},
     {"BLAS3_GM_MIN_TRMM", int64_t(1) << 30, 0, int64_t(1) << 40, false},
     {"BLAS3_GM_MIN_TRSM", int64_t(1) << 30, 0, int64_t(1) << 40, false},
     {"BLAS3_TC_CTA", 0, 0, 2, false},
@@ -38,7 +38,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_PDL", 1, 0, 1, false},
     {"BLAS3_TRSM_NB", 2048, 128, 8192, true},
     {"BLAS3_TRSM_SLABS", 2, 1, 4, false},
-    {"BLAS3_TRSM_SLAB_MIN", 4096, 256, int64_t(1) << 40, false},
+    {"BLAS3_TRSM_SLAB_MIN", 16384, 256, int64_t(1) << 40, false},
     {"BLAS3_TRSM_RESERVE", 48, 0, 74, false},
     {"BLAS3_TRSM_GEO_LEAF", 256, 128, 8192, true},
     {"BLAS3_TRSM_FUSED", 0, 0, 1, false},
