@@ -1091,15 +1091,6 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
     if (rc < 0) return rc;
     all_done = rc == 0;
   }
-  // the other panels' levels (needed one panel sweep later) on a second side
-  // stream, from the start
-  if (npanel > 1 && !all_done) {
-    const int64_t prest = forward ? 1 : 0, o = prest * NBO;
-    if (cudaStreamWaitEvent(ts->side2, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
-    if ((rc = trsm_panel_doubling(A + o * (1 + lda), lda, imin(nt, (prest + npanel - 1) * NBO) - o, lower,
-                                  D.p + prest * NBO * NBO, Tw.p, ts->side2, sms, ts->ev_lvl2)))
-      return rc;
-  }
   // the first processed panel: ONE fused persistent launch (its doubling
   // levels, the precomputed Y and M of every geometric pair, and the chain
   // leaf -> X_1 -> X_2 -> ... with per-slab tile-counter dependencies) on the
@@ -1148,6 +1139,18 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
     const int64_t o = pfirst * NBO;
     if ((rc = trsm_panel_doubling(A + o * (1 + lda), lda, imin(NBO, nt - o), lower,
                                   D.p + pfirst * NBO * NBO, Tw.p + t_rest, ts->side, sms, ts->ev_lvl)))
+      return rc;
+  }
+  // the other panels' levels (needed one panel sweep later) on a second side
+  // stream.  Enqueued AFTER the first panel's launches: the host takes a few
+  // microseconds per launch, and the first panel is the critical path (the
+  // fused chain started ~125 us late at N = 8192 when these ~8 launches were
+  // enqueued before it; profiles/r02_strsm_timeline.md)
+  if (npanel > 1 && !all_done) {
+    const int64_t prest = forward ? 1 : 0, o = prest * NBO;
+    if (cudaStreamWaitEvent(ts->side2, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+    if ((rc = trsm_panel_doubling(A + o * (1 + lda), lda, imin(nt, (prest + npanel - 1) * NBO) - o, lower,
+                                  D.p + prest * NBO * NBO, Tw.p, ts->side2, sms, ts->ev_lvl2)))
       return rc;
   }
   if (cudaEventRecord(ts->ev_fork2, s) != cudaSuccess) return BLAS3_ERR_CUDA;

@@ -38,6 +38,9 @@ ts, k = 16384, 512
 As, Bs, Cs = mk(ts, k), mk(ts, k), mk(ts, ts)
 A2, B2, C2 = mk(2048, 2048), mk(2048, 2048), mk(2048, 2048)
 A1, B1, C1 = mk(1024, 1024), mk(1024, 1024), mk(1024, 1024)
+T4, X4, B4 = mk(4096, 4096), mk(4096, 4096), mk(4096, 4096)
+T4.mul_(1.0 / 4096)
+T4.diagonal().fill_(1.0)
 cases = {
     "sgemm": (lambda: b3.sgemm("N", "N", 1.5, A, B, 0.5, C), 2.0 * n ** 3, 5, None),
     "ssymm": (lambda: b3.ssymm("L", "L", 1.5, A, B, 0.5, C), 2.0 * n ** 3, 5, None),
@@ -49,6 +52,7 @@ cases = {
     "ts_syr2k": (lambda: b3.ssyr2k("L", "N", 1.5, As, Bs, 0.5, Cs), 2.0 * k * ts * ts + ts, 10, None),
     "sgemm2048": (lambda: b3.sgemm("N", "N", 1.5, A2, B2, 0.5, C2), 2.0 * 2048 ** 3, 40, None),
     "sgemm1024": (lambda: b3.sgemm("N", "N", 1.5, A1, B1, 0.5, C1), 2.0 * 1024 ** 3, 100, None),
+    "strsm4096": (lambda: b3.strsm("L", "L", "N", "N", 1.0, T4, X4), 1.0 * 4096 ** 3, 10, lambda: X4.copy_(B4)),
 }
 sel = [c for c in args.cases.split(",") if c in cases]
 
