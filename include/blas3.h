@@ -175,7 +175,8 @@ int blas3_get_math_mode(void);
  *                          one slab up to 32767 right-hand sides -- measured 5.6%
  *                          faster than two at 8192, profiles/r02_trsm_options.md)
  *   BLAS3_OPT_TRSM_RESERVE [BLAS3_TRSM_RESERVE] SMs the first panel's sweep leaves to
- *                          the panel-inverse doubling chain, 0..74 (48)
+ *                          the panel-inverse doubling chain, 0..74, or -1 (default,
+ *                          auto: 48 from order 8192, 16 below)
  *   BLAS3_OPT_TRSM_GEO_LEAF [BLAS3_TRSM_GEO_LEAF] the first panel is halved down to
  *                          this width: power of 2 in [128, 8192] (256)
  *   BLAS3_OPT_TRSM_FUSED   [BLAS3_TRSM_FUSED] 1: the whole STRSM (panel-inverse

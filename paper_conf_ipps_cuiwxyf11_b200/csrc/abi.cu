@@ -39,7 +39,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TRSM_NB", 2048, 128, 8192, true},
     {"BLAS3_TRSM_SLABS", 2, 1, 4, false},
     {"BLAS3_TRSM_SLAB_MIN", 16384, 256, int64_t(1) << 40, false},
-    {"BLAS3_TRSM_RESERVE", 48, 0, 74, false},
+    {"BLAS3_TRSM_RESERVE", -1, -1, 74, false},
     {"BLAS3_TRSM_GEO_LEAF", 256, 128, 8192, true},
     {"BLAS3_TRSM_FUSED", 0, 0, 1, false},
     {"BLAS3_TRSM_FIRST_YM", 1, 0, 1, false},
@@ -642,7 +642,12 @@ static int64_t trsm_slabs(int64_t other) {
 }
 static inline int64_t align_down(int64_t v, int64_t a) { return v / a * a; }
 // SMs the first panel's sweep kernels leave free for its doubling chain
-static int64_t trsm_reserve() { return opt(BLAS3_OPT_TRSM_RESERVE); }
+// (-1 = auto: 48 from order 8192 on, where the other panels' doubling has the
+// most work beside the chain; 16 below -- measured, profiles/r02_trsm_options.md)
+static int64_t trsm_reserve(int64_t nt) {
+  const int64_t v = opt(BLAS3_OPT_TRSM_RESERVE);
+  return v >= 0 ? v : (nt >= 8192 ? 48 : 16);
+}
 // width below which the first panel's geometric halving stops (power of 2)
 static int64_t trsm_geo_leaf() { return opt(BLAS3_OPT_TRSM_GEO_LEAF); }
 
@@ -968,7 +973,7 @@ static int strsm_first_fused(const TrsmGeom &g, const std::vector<GeoPair> &gp, 
   // the chain is latency-bound: leave SMs to the other panels' doubling,
   // which runs concurrently on a side stream
   const int rc = launch_tc_fused(ph.data(), (int)ph.size(), s,
-                                 all ? sms : (int)imax(sms / 2, sms - trsm_reserve()));
+                                 all ? sms : (int)imax(sms / 2, sms - trsm_reserve(nt)));
   return rc == 0 ? 0 : (rc == -4 ? BLAS3_ERR_TMA : BLAS3_ERR_CUDA);
 }
 
@@ -1232,7 +1237,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
     // leaf: rows (L) / columns (R) [e0, e0 + cnt) of X, aligned block width wblk
     // kernels of the first panel leave SMs to the latency-bound doubling
     // chain of that panel (high-priority side stream)
-    const int32_t first_sms = (int32_t)imax(sms / 2, sms - trsm_reserve());
+    const int32_t first_sms = (int32_t)imax(sms / 2, sms - trsm_reserve(nt));
     int64_t app_lo = 0, app_hi = 0;                   // split sweep: updates already applied
     auto leaf = [&](int64_t e0, int64_t cnt, int64_t wblk, bool scaled, bool in_w, bool restrict_sms = true) -> int {
       int rc2;

@@ -720,6 +720,11 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
         Work w;
         if (tb >= 0) w = work_of<CG>(prm, tb);
         else w.tb = -1;
+        // fused launches: the producing tiles are complete (gpu-scope acquire)
+        // BEFORE the item is published, so every local role that takes it
+        // through wk_full (release / acquire at CTA scope) also observes the
+        // producing CTAs' stores -- the epilogue needs no acquire of its own
+        if (tb >= 0) wait_deps<CG>(prm, w);
         bars->wk[slot] = w;
         ptx::mbar_arrive(&bars->wk_full[slot]);       // release: local roles see wk[slot]
         ++qi;
@@ -734,7 +739,6 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
         const int32_t bj = (int32_t)(w.b % per), bg = (int32_t)(w.b / per);
         const int64_t m0 = w.m0, n0 = w.n0;
         const int64_t ma = m0 + HA * rank, nb = n0 + HB * rank;
-        wait_deps<CG>(prm, w);                        // fused launches: producing tiles done
         BLAS3_STRACE(0, w.ph);
         if (FUSED && prm.ph_trace != nullptr) {
           unsigned long long t_;
@@ -1085,11 +1089,10 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
         }
       }
       if (FUSED) {
-        // C may have been written by earlier phases on other SMs: one acquire
-        // (which also invalidates this SM's L1) before any thread loads it
-        if (threadIdx.x == WARP_EPI0 * 32) BLAS3_STRACE(11, w.ph);
-        if (threadIdx.x == WARP_EPI0 * 32) wait_deps<CG>(prm, w, false);
-        ptx::named_bar_sync(5, EPI_THREADS);
+        // C may have been written by earlier phases on other SMs: this CTA's
+        // producer acquired the dependency counters before publishing the
+        // item, and the epilogue took the item through wk_full (CTA-scope
+        // release / acquire), so those stores are visible here
         if (threadIdx.x == WARP_EPI0 * 32) BLAS3_STRACE(7, w.ph);
       }
       // ---- store phase: D = alpha*S + beta*C for row r, columns cbase + [0,128).
