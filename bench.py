@@ -179,7 +179,7 @@ def run_ours(args):
 
     import paper_conf_ipps_cuiwxyf11_b200 as b3
     b3.set_math_mode(args.math)
-    n = args.size
+    n = N if args.size is None else args.size
     cols = n                                   # per-rank slab width (weak scaling)
     A_h, T_h, B_h, C_h = make_inputs(n, cols, rank)
     dev = torch.device("cuda", local)
@@ -661,7 +661,7 @@ def run_cfg5(args):
     import paper_conf_ipps_cuiwxyf11_b200 as b3
     from paper_conf_ipps_cuiwxyf11_b200 import dist as d3
     b3.set_math_mode(args.math)
-    n = CFG5_N if args.size == N else args.size
+    n = CFG5_N if args.size is None else args.size
     c0, c1 = d3.slab(n, world, rank)
     cols = c1 - c0
     dev = torch.device("cuda", local)
@@ -920,7 +920,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--math", default="3xtf32", choices=["3xtf32", "simt", "tf32_bf16x"])
-    ap.add_argument("--size", type=int, default=N, help="matrix order (default 8192)")
+    ap.add_argument("--size", type=int, default=None,
+                    help="matrix order (default 8192; 32768 for --workload cfg5)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the e2e leg (profiling runs)")
