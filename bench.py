@@ -214,7 +214,7 @@ def run_ours(args):
         #  * A: broadcast in 8 K-panels on a comm stream, consumed by the
         #    panel GEMMs of the sgemm as they land (d3.sgemm);
         #  * T: only its lower triangle, 4 trapezoid panels, on a second comm
-        #    stream from the start of the step (needed from strmm on);
+        #    stream, enqueued right after A's panels (needed from strmm on);
         #  * SYRK/SYR2K (no right-hand side to shard): k-split weak scaling --
         #    rank r's own k-slab (its B slab; for SYR2K its B and C0 slabs),
         #    the partial products summed by an NCCL all-reduce on a third
@@ -286,8 +286,10 @@ def run_ours(args):
             timed("strmm", lambda: b3.strmm("L", "L", "N", "N", ALPHA, T, X))
             timed("strsm", lambda: b3.strsm("L", "L", "N", "N", ALPHA, T, X))
             return
-        eT = bcast_T_async(T)
+        # (collectives of one process group share one NCCL stream in enqueue
+        # order: A's panels go first, T's triangle queues behind them)
         timed("sgemm", lambda: d3.sgemm("N", "N", ALPHA, A, Bm, BETA, C, panels=8, reserve_sms=RESERVE))
+        eT = bcast_T_async(T)
         timed("ssymm", lambda: b3.ssymm("L", "L", ALPHA, A, Bm, BETA, C), reserve=True)
         timed("ssyrk", syrk_k, reserve=True)
         timed("ssyr2k", syr2k_k, reserve=True)
