@@ -45,6 +45,16 @@ for mode in ("3xtf32", "simt", "tf32_bf16x"):
             b3.strsm("R", "U", "T", "N", 1.5, Tn, rnd(300, 900))
     calls += 12
 b3.set_math_mode("3xtf32")
+with b3.options(gm_map=1):                                       # GM_map SSYMM beside the staged default
+    b3.ssymm("L", "U", 1.5, rnd(300, 300), rnd(300, 260), 0.5, rnd(300, 260))
+# a captured graph (graph-private scheduler state / split workspace), replayed twice
+cs = torch.cuda.Stream()
+Cg = rnd(1024, 768)
+Ag, Bg = rnd(1024, 2048), rnd(2048, 768)
+g = torch.cuda.CUDAGraph()
+with torch.cuda.graph(g, stream=cs):
+    b3.sgemm("N", "N", 1.0, Ag, Bg, 0.5, Cg)
+g.replay(); g.replay()
 C2 = rnd(1024, 768)
 b3.sgemm("N", "N", 1.0, rnd(1024, 2048), rnd(2048, 768), 0.0, C2)   # few tiles: split-k tail
 torch.cuda.synchronize()
