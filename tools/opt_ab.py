@@ -58,15 +58,18 @@ sel = [c for c in args.cases.split(",") if c in cases]
 
 
 def timed(fn, reps, pre):
-    tot = 0.0
+    """reps calls back to back between two events (pre() once before: the
+    in-place routines' operand drifts slowly, ||T|| ~ 1)."""
+    if pre:
+        pre()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(True); e1 = torch.cuda.Event(True)
+    e0.record()
     for _ in range(reps):
-        if pre:
-            pre()
-        e0 = torch.cuda.Event(True); e1 = torch.cuda.Event(True)
-        e0.record(); fn(); e1.record()
-        torch.cuda.synchronize()
-        tot += e0.elapsed_time(e1)
-    return tot / reps
+        fn()
+    e1.record()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / reps
 
 
 res = {(c, v): [] for c in sel for v in args.values}

@@ -1,6 +1,8 @@
 """Size-stability sweep (the paper's Fig. 13 range): every routine family at
-N = 512..8192, CUDA events, interleaved rounds, medians; % of this library's SGEMM
-NN at the same N.  python tools/size_sweep.py [sizes] [rounds]"""
+N = 512..8192.  Each measurement is `reps` calls back to back between two CUDA
+events (the GPU never waits for the host, as in any stream of calls), rounds
+interleaved, medians; % of this library's SGEMM NN at the same N.
+python tools/size_sweep.py [sizes] [rounds]"""
 import sys
 
 import numpy as np
@@ -34,14 +36,16 @@ for n in sizes:
     res = {i: [] for i in range(len(cases))}
     for rnd in range(rounds):
         for i, (_, _, fl, fn, pre) in enumerate(cases):
-            tot = 0.0
+            if pre:
+                pre()
+            fn()
+            torch.cuda.synchronize()
+            e0 = torch.cuda.Event(True); e1 = torch.cuda.Event(True)
+            e0.record()
             for _ in range(reps):
-                if pre:
-                    pre()
-                e0 = torch.cuda.Event(True); e1 = torch.cuda.Event(True)
-                e0.record(); fn(); e1.record(); torch.cuda.synchronize()
-                tot += e0.elapsed_time(e1)
-            res[i].append(tot / reps)
+                fn()
+            e1.record(); torch.cuda.synchronize()
+            res[i].append(e0.elapsed_time(e1) / reps)
     sg = None
     for i, (r, v, fl, _, _) in enumerate(cases):
         ms = float(np.median(res[i]))
