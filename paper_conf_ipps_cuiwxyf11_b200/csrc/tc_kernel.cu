@@ -1301,14 +1301,17 @@ bool tc_eligible(const Problem &P) {
 
 // CTA-group choice.  The pair kernel (CG=2: 256x256 tiles, tcgen05
 // cta_group::2, each CTA staging half of B) needs half the per-SM operand
-// traffic and a 4-deep raw ring; it is used whenever it still gives every CTA
-// pair at least one tile, else the single-CTA kernel (more, smaller tiles,
-// dynamic scheduling).  BLAS3_TC_CTA=1|2 forces one (tests).
+// traffic and has a 4-deep raw ring: it is faster per SM even when its tiles
+// do not fill the machine (measured: SGEMM 2048^3 82.8 vs 106 us, 1024^3 46.0
+// vs 48.6 us, profiles/r02_sizes.md).  The single-CTA kernel (128x256 tiles)
+// is kept for problems of fewer than 256 rows, where a 256-row pair tile
+// would compute mostly padding (the TRSM doubling's 128-blocks, skinny
+// updates).  BLAS3_TC_CTA=1|2 forces one (tests).
 static int choose_cg(const Problem &P, int num_sms) {
   const int forced = (int)opt(BLAS3_OPT_TC_CTA);
   if (forced) return forced;
   const int64_t nb = P.nbatch > 1 ? P.nbatch : 1;
-  return Tiles<Geo<2>::TM, BN>::count(P) * nb >= num_sms / 2 ? 2 : 1;
+  return (P.M >= 256 || Tiles<Geo<2>::TM, BN>::count(P) * nb >= num_sms / 2) ? 2 : 1;
 }
 
 template <int CG, class PRM>
