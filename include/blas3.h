@@ -234,6 +234,11 @@ int blas3_get_math_mode(void);
  *                          (default) each CTA's C tile is prefetched into L2
  *                          (one TMA prefetch) a few TMEM chunks before it is
  *                          read, so the store phase does not wait on HBM; 0 off
+ *   BLAS3_OPT_TC_C_ASYNC   [BLAS3_TC_C_ASYNC] tcgen05 epilogue, beta != 0 with 16-B vector
+ *                          access: 1 C goes to shared memory by cp.async two 8-column
+ *                          groups ahead of its use; 0 (default) one group ahead in
+ *                          registers (measured within noise of each other: SGEMM
+ *                          +2%, tall-skinny SSYRK -2%)
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */
@@ -246,7 +251,7 @@ enum {
     BLAS3_OPT_TRSM_FIRST_YM = 15, BLAS3_OPT_TRSM_FIRST_FUSED = 16, BLAS3_OPT_TRSM_FIRST_SPLIT = 17,
     BLAS3_OPT_TRSM_FIRST_ALL = 18, BLAS3_OPT_TC_RASTER = 19, BLAS3_OPT_TC_KC = 20,
     BLAS3_OPT_TC_VEC_STORE = 21, BLAS3_OPT_MAX_SMS = 22, BLAS3_OPT_TC_C_PREFETCH = 23,
-    BLAS3_OPT_COUNT = 24
+    BLAS3_OPT_TC_C_ASYNC = 24, BLAS3_OPT_COUNT = 25
 };
 int blas3_set_option(int key, int64_t value);
 int64_t blas3_get_option(int key);

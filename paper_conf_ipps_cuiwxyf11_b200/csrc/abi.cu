@@ -51,6 +51,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TC_VEC_STORE", 1, 0, 1, false},
     {"BLAS3_MAX_SMS", 0, 0, 4096, false},
     {"BLAS3_TC_C_PREFETCH", 1, 0, 1, false},
+    {"BLAS3_TC_C_ASYNC", 0, 0, 1, false},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;

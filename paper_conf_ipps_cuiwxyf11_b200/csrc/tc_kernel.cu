@@ -129,7 +129,7 @@ struct Geo {
     uint32_t split_last;     // epilogue: this CTA's slice of a split tile is the last one
   };
   struct alignas(1024) EpiStage {
-    float box[NUM_EPI_WARPS][EPI_BOX];      // epilogue transpose boxes
+    float box[NUM_EPI_WARPS][3][EPI_BOX];   // epilogue: transpose box + 2 C boxes per warp
   };
   static constexpr size_t SMEM =
       sizeof(RawBuf) * RS + sizeof(LoBuf) * LS + sizeof(EpiStage) + sizeof(Barriers) + 1024;
@@ -1018,7 +1018,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
     const int half = (warp - WARP_EPI0) >> 2;   // which 128 of the 256 columns
     constexpr int NG = BN / 2 / EC;             // column groups per thread (8)
     uint32_t cc = 0, qi = 0;
-    const uint32_t box_s = ptx::smem_u32(epi_stage + (warp - WARP_EPI0) * EPI_BOX);
+    const uint32_t box_s = ptx::smem_u32(epi_stage + (warp - WARP_EPI0) * 3 * EPI_BOX);
     for (;;) {
       const Work w = next_work(qi, 5, EPI_THREADS, threadIdx.x == WARP_EPI0 * 32);
       if (w.tb < 0) break;
@@ -1117,6 +1117,47 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
       constexpr int SG = 8;
       if (none) {
         // nothing of this warp's 32 x 128 block is referenced (ragged edge)
+      } else if (full && P.c_vec == 2 && be != 0.f) {
+        // ---- as below, but C arrives by cp.async in the warp's two C boxes,
+        // two groups ahead and without registers: the store phase (during
+        // which the next tile's TMEM partials wait to be drained) is bound by
+        // the L2 latency of C, and the running sum leaves no registers for a
+        // deeper register prefetch.  Each lane copies, and later reads back,
+        // exactly the float4s it combines (no cross-lane sync on the C boxes).
+        const int vr = (lane & 7) * 4, vc = lane >> 3;
+        const float *cq = P.Cin + coff + (m0 + HA * rank + q * 32 + vr) + (cbase + vc) * ldi;
+        float *oq = P.Cout + coff + (m0 + HA * rank + q * 32 + vr) + (cbase + vc) * ldo;
+        const uint32_t own = (uint32_t)(vc * 32 + vr) * 4;
+        const uint32_t rd = box_s + own;                                  // transpose box
+        const uint32_t cb = box_s + EPI_BOX * 4 + own;                    // C box 0 (box 1: + 1 KiB)
+        constexpr int NGW = BN / 2 / EPI_GW;
+        auto fetch = [&](int g) {
+          const float *src = cq + (int64_t)g * EPI_GW * ldi;
+          const uint32_t dst = cb + (uint32_t)(g & 1) * (EPI_BOX * 4);
+          ptx::cp_async16(dst, src);
+          ptx::cp_async16(dst + 4 * 128, src + 4 * ldi);
+        };
+        fetch(0); ptx::cp_async_commit();
+        fetch(1); ptx::cp_async_commit();
+#pragma unroll
+        for (int g = 0; g < NGW; ++g) {
+#pragma unroll
+          for (int j = 0; j < EPI_GW; ++j) ptx::st_shared_f32(box_s + (j * 32 + lane) * 4, al * S[g * EPI_GW + j]);
+          __syncwarp();
+          float4 d0 = ptx::ld_shared_v4(rd), d1 = ptx::ld_shared_v4(rd + 4 * 128);
+          __syncwarp();                                   // transpose box free for the next group
+          ptx::cp_async_wait<1>();                        // group g landed (g + 1 may be in flight)
+          const uint32_t cg = cb + (uint32_t)(g & 1) * (EPI_BOX * 4);
+          const float4 c0v = ptx::ld_shared_v4(cg), c1v = ptx::ld_shared_v4(cg + 4 * 128);
+          if (g + 2 < NGW) fetch(g + 2);                  // into the box just read
+          ptx::cp_async_commit();                         // (empty groups keep the count uniform)
+          d0.x = fmaf(be, c0v.x, d0.x); d0.y = fmaf(be, c0v.y, d0.y);
+          d0.z = fmaf(be, c0v.z, d0.z); d0.w = fmaf(be, c0v.w, d0.w);
+          d1.x = fmaf(be, c1v.x, d1.x); d1.y = fmaf(be, c1v.y, d1.y);
+          d1.z = fmaf(be, c1v.z, d1.z); d1.w = fmaf(be, c1v.w, d1.w);
+          if (st_on) { ptx::st_cs_v4(oq, d0); ptx::st_cs_v4(oq + 4 * ldo, d1); }
+          oq += EPI_GW * ldo;
+        }
       } else if (full && P.c_vec) {
         // ---- 16-B vector accesses of C (NS "coalesced 128-bit epilogue
         // stores"; DESIGN A6), for warps whose whole 32 x 128 block is valid
@@ -1341,6 +1382,7 @@ static int launch_cg(PRM &prm, cudaStream_t stream, int num_sms, bool allow_pdl 
     const bool rd = P.beta != 0.f;
     P.c_vec = opt(BLAS3_OPT_TC_VEC_STORE) != 0 && vec_ok(P.Cout, P.ldcout, P.bs_c) &&
               (!rd || vec_ok(P.Cin, P.ldcin, P.bs_c)) ? 1 : 0;
+    if (P.c_vec && rd && opt(BLAS3_OPT_TC_C_ASYNC)) P.c_vec = 2;     // C by cp.async into shared boxes
     P.c_pf_map = -1;
     if (!rd || !opt(BLAS3_OPT_TC_C_PREFETCH) || !vec_ok(P.Cin, P.ldcin, P.bs_c) ||
         slot >= (int)(sizeof(prm.maps) / sizeof(prm.maps[0]))) continue;

@@ -186,4 +186,5 @@ def test_options_roundtrip_and_validation(lib):
         assert lib.blas3_set_option(lib.OPTIONS["tc_kc"], bad) == 1
     assert lib.get_option("tc_vec_store") == 1 and lib.get_option("tc_c_prefetch") == 1
     assert lib.get_option("max_sms") == 0
-    assert len(lib.OPTIONS) == 24
+    assert lib.get_option("tc_c_async") == 0
+    assert len(lib.OPTIONS) == 25
