@@ -77,13 +77,16 @@ def fp32_3xtf32_peak(peaks, sustained=True):
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    """nvidia-smi clocks + throttle reasons sampled during the timed region
+    (every `interval_ms`; each row keeps the host time it arrived at, so a
+    window of the run can be summarised on its own)."""
     Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
-    def __init__(self, index):
+    def __init__(self, index, interval_ms=200):
         self.index = index
+        self.interval_ms = interval_ms
         self.rows = []
         self.proc = None
 
@@ -91,7 +94,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                 "--format=csv,noheader,nounits", "-lms", "200"],
+                 "--format=csv,noheader,nounits", "-lms", str(self.interval_ms)],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -101,7 +104,7 @@ class ClockSampler:
 
     def _read(self):
         for line in self.proc.stdout:
-            self.rows.append([x.strip() for x in line.split(",")])
+            self.rows.append([x.strip() for x in line.split(",")] + [time.time()])
 
     def __exit__(self, *a):
         if self.proc:
@@ -111,20 +114,25 @@ class ClockSampler:
             except subprocess.TimeoutExpired:
                 self.proc.kill()
 
-    def summary(self):
-        if not self.rows:
+    def summary(self, t0=None, t1=None):
+        rows = [r for r in self.rows if (t0 is None or r[-1] >= t0) and (t1 is None or r[-1] <= t1)]
+        if not rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
-        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
-        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        pw = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = set()
-        for r in self.rows:
+        for r in rows:
             for nm, v in zip(names, r[4:8]):
                 if v.lower().startswith("active"):
                     reasons.add(nm)
-        return {"sm_mhz": float(np.median(sm)) if sm else None,
-                "sm_max_mhz": max(mx) if mx else None,
-                "samples": len(self.rows), "reasons": sorted(reasons)}
+        out = {"sm_mhz": float(np.median(sm)) if sm else None,
+               "sm_max_mhz": max(mx) if mx else None,
+               "samples": len(rows), "reasons": sorted(reasons)}
+        if pw:
+            out["power_w"] = float(np.median(pw))
+        return out
 
 
 # ----------------------------------------------------------------------------- inputs
@@ -430,6 +438,8 @@ def run_ours(args):
         e2e_loop(max(1, min(2, args.warmup)))          # warm-up (both buffer sets)
         ms_e2e = e2e_loop(args.steps)
 
+    ev_ms = {r: float(np.mean([a.elapsed_time(b) for a, b in ev[r]])) for r in ROUTINES}
+
     # the opt-in TF32+BF16X mode on the same data, device timing only, reported
     # beside (never instead of) the default 3xTF32 headline
     alt = None
@@ -456,6 +466,38 @@ def run_ours(args):
             b3.set_math_mode(args.math)
             for r in ROUTINES:
                 ev[r][:] = per_default[r]
+
+    # per routine, in isolation: each routine back to back for ~0.5 s with the
+    # clocks sampled every 50 ms (the chain's own clock record covers the whole
+    # step); STRMM / STRSM restore X every call (the copy is inside the time)
+    isolated = None
+    if world == 1 and not args.no_routine_clocks:
+        isolated = {}
+        single = {
+            "sgemm": lambda: b3.sgemm("N", "N", ALPHA, A, Bm, BETA, C),
+            "ssymm": lambda: b3.ssymm("L", "L", ALPHA, A, Bm, BETA, C),
+            "ssyrk": lambda: b3.ssyrk("L", "N", ALPHA, A, BETA, C),
+            "ssyr2k": lambda: b3.ssyr2k("L", "N", ALPHA, A, Bm, BETA, C),
+            "strmm": lambda: (dX.copy_(dB), b3.strmm("L", "L", "N", "N", ALPHA, T, X)),
+            "strsm": lambda: (dX.copy_(dB), b3.strsm("L", "L", "N", "N", ALPHA, T, X)),
+        }
+        with ClockSampler(local, interval_ms=50) as clk_r:
+            time.sleep(0.4)
+            for r in ROUTINES:
+                fn = single[r]
+                fn(); torch.cuda.synchronize()
+                reps = max(3, int(500.0 / max(0.1, ev_ms[r])))
+                c0 = torch.cuda.Event(enable_timing=True); c1 = torch.cuda.Event(enable_timing=True)
+                t0 = time.time()
+                c0.record(stream)
+                for _ in range(reps):
+                    fn()
+                c1.record(stream)
+                torch.cuda.synchronize()
+                t1 = time.time()
+                ms_r = c0.elapsed_time(c1) / reps
+                isolated[r] = {"ms": round(ms_r, 4), "gflops": round(fl[r] / (ms_r * 1e-3) / 1e9, 1),
+                               "reps": reps, "clocks": clk_r.summary(t0, t1)}
 
     # context (north star: "reports the box's cuBLAS SGEMM as context"): torch's
     # cuBLAS fp32 SGEMM (TF32 off) and its 1-pass TF32 mode on the same A, B
@@ -587,6 +629,7 @@ def run_ours(args):
         "alt_mode": alt,
         "context": context,
         "gpu_launches_per_step": round(launches / args.steps, 1),
+        "isolated": isolated,
         "clocks": clk.summary(),
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -930,6 +973,8 @@ def main():
     ap.add_argument("--no-context", action="store_true", help="skip the cuBLAS context timing")
     ap.add_argument("--no-alt-mode", action="store_true",
                     help="skip the extra device-only pass in the opt-in TF32+BF16X mode")
+    ap.add_argument("--no-routine-clocks", action="store_true",
+                    help="skip the per-routine isolated loops (~0.5 s each, clocks sampled every 50 ms)")
     ap.add_argument("--workload", default="chain", choices=["chain", "cfg5"],
                     help="chain: the six-routine N=8192 step (default, weak scaling at N>1); "
                          "cfg5: BASELINE configs[4], N=32768 column slabs (strong scaling)")
