@@ -427,9 +427,11 @@ def run_ours(args):
         step_device()
     torch.cuda.synchronize()
     launches0 = b3.launch_count()
-    with ClockSampler(local) as clk:
+    with ClockSampler(local, interval_ms=50) as clk:
         time.sleep(0.6)                       # nvidia-smi start-up, before the timed region
+        t_clk0 = time.time()
         ms = timed_loop(lambda rec: step_device(rec), args.steps, record=True)
+        t_clk1 = time.time()
     launches = b3.launch_count() - launches0
 
     # e2e: same metric through the public API with host buffers
@@ -630,7 +632,7 @@ def run_ours(args):
         "context": context,
         "gpu_launches_per_step": round(launches / args.steps, 1),
         "isolated": isolated,
-        "clocks": clk.summary(),
+        "clocks": clk.summary(t_clk0, t_clk1 + 0.05),
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         out["cpu_baseline"] = cpu_baseline(args.cpu_seconds)
@@ -754,9 +756,11 @@ def run_cfg5(args):
     for _ in range(args.warmup):
         step()
     launches0 = b3.launch_count()
-    with ClockSampler(local) as clk:
+    with ClockSampler(local, interval_ms=50) as clk:
         time.sleep(0.6)
+        t_clk0 = time.time()
         ms = timed_loop(args.steps, True)
+        t_clk1 = time.time()
     launches = b3.launch_count() - launches0
 
     # e2e: the same step through the public API with host buffers: A and T
@@ -842,7 +846,7 @@ def run_cfg5(args):
         "e2e": e2e,
         "gpu_launches": int(launches),
         "comm": comm_info,
-        "clocks": clk.summary(),
+        "clocks": clk.summary(t_clk0, t_clk1 + 0.05),
     }
     if rank == 0:
         print(json.dumps(out), flush=True)
