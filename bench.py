@@ -116,6 +116,8 @@ class ClockSampler:
 
     def summary(self, t0=None, t1=None):
         rows = [r for r in self.rows if (t0 is None or r[-1] >= t0) and (t1 is None or r[-1] <= t1)]
+        if not rows and (t0 is not None or t1 is not None):
+            rows = self.rows                    # window shorter than one sample: every sample
         if not rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
         sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
