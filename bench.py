@@ -233,6 +233,11 @@ def run_ours(args):
         # While a collective is in flight the products leave RESERVE SMs to
         # NCCL (BLAS3_OPT_MAX_SMS).
         RESERVE = 16
+        # device-side panel consumption (one streamed GEMM polling per-panel
+        # flags) needs its own GPU per rank: ranks sharing one device (the gloo
+        # logic check) would let one rank's persistent grid take the SMs the
+        # other rank's flag writes need
+        DEVICE_SIDE = comm_info.get("backend") == "nccl"
         nsm = torch.cuda.get_device_properties(dev).multi_processor_count
         dCs1 = torch.empty((n, n), device=dev); dCs2 = torch.empty((n, n), device=dev)
         Cs1, Cs2 = colmaj(dCs1), colmaj(dCs2)
@@ -298,7 +303,8 @@ def run_ours(args):
             return
         # (collectives of one process group share one NCCL stream in enqueue
         # order: A's panels go first, T's triangle queues behind them)
-        timed("sgemm", lambda: d3.sgemm("N", "N", ALPHA, A, Bm, BETA, C, panels=8, reserve_sms=RESERVE))
+        timed("sgemm", lambda: d3.sgemm("N", "N", ALPHA, A, Bm, BETA, C, panels=8, reserve_sms=RESERVE,
+                                        device_side=DEVICE_SIDE))
         eT = bcast_T_async(T)
         timed("ssymm", lambda: b3.ssymm("L", "L", ALPHA, A, Bm, BETA, C), reserve=True)
         timed("ssyrk", syrk_k, reserve=True)
@@ -350,7 +356,7 @@ def run_ours(args):
         if world > 1:
             for (c0, c1), e in zip(bounds, evs):
                 stream.wait_event(e)
-            d3.sgemm("N", "N", ALPHA, A_, Bm_, BETA, C_, panels=8, reserve_sms=RESERVE)
+            d3.sgemm("N", "N", ALPHA, A_, Bm_, BETA, C_, panels=8, reserve_sms=RESERVE, device_side=DEVICE_SIDE)
         else:
             for (c0, c1), e in zip(bounds, evs):
                 stream.wait_event(e)
@@ -599,7 +605,8 @@ def run_ours(args):
             "n": n, "k": n, "cols_per_rank": cols, "math": args.math,
             "l2": "no flush: every operand is 256 MiB > 126 MB L2",
             "parallelism": (f"dp{world}: column slabs of B/C/X per rank ({cols} columns each); A broadcast "
-                            f"from rank 0 in 8 K-panels overlapped with the sgemm panels, T's lower "
+                            f"from rank 0 in 8 K-panels consumed as they land by one streamed sgemm "
+                            f"(device-side panel flags; per-panel GEMMs under gloo), T's lower "
                             f"triangle in 4 trapezoid panels overlapped with sgemm..ssyr2k (NCCL, "
                             f"comm streams, 16 SMs reserved while in flight); ssyrk/ssyr2k k-split, "
                             f"partials all-reduced (NCCL) overlapped with the next routines")
@@ -723,7 +730,8 @@ def run_cfg5(args):
     stream = torch.cuda.current_stream()
     ev = {r: [] for r in CFG5_ROUTINES}
     calls = {
-        "sgemm": lambda: d3.sgemm("N", "N", ALPHA, A, Bm, BETA, C, panels=8),
+        "sgemm": lambda: d3.sgemm("N", "N", ALPHA, A, Bm, BETA, C, panels=8,
+                                  device_side=comm_info.get("backend") == "nccl"),
         "ssymm": lambda: d3.ssymm("L", "L", ALPHA, A, Bm, BETA, C, panels=8),
         "strsm": lambda: d3.strsm("L", "L", "N", "N", ALPHA, T, X, panels=4),
     }

@@ -38,7 +38,9 @@
  *             < 0 : runtime failure: BLAS3_ERR_CUDA (a CUDA launch/runtime
  *                   error), BLAS3_ERR_ARCH (current device is not sm_100),
  *                   BLAS3_ERR_ALLOC (scratch allocation failed),
- *                   BLAS3_ERR_TMA (tensor-map encoding failed).
+ *                   BLAS3_ERR_TMA (tensor-map encoding failed),
+ *                   BLAS3_ERR_UNSUPPORTED (a configuration the entry point
+ *                   does not cover, e.g. a streamed operand in SIMT mode).
  *             The ABI never aborts and never throws.
  *  Special    beta == 0: C is not read (NaN/Inf in C do not propagate).
  *  values     alpha == 0: A and B are not read (C <- beta*C; B <- 0 for
@@ -76,7 +78,8 @@ enum {
     BLAS3_ERR_CUDA = -1,
     BLAS3_ERR_ARCH = -2,
     BLAS3_ERR_ALLOC = -3,
-    BLAS3_ERR_TMA = -4
+    BLAS3_ERR_TMA = -4,
+    BLAS3_ERR_UNSUPPORTED = -5
 };
 
 enum { BLAS3_MATH_3XTF32 = 0, BLAS3_MATH_SIMT_FP32 = 1, BLAS3_MATH_1XTF32 = 2, BLAS3_MATH_TF32_BF16X = 3 };
@@ -90,6 +93,33 @@ enum { BLAS3_MATH_3XTF32 = 0, BLAS3_MATH_SIMT_FP32 = 1, BLAS3_MATH_1XTF32 = 2, B
 int blas3_sgemm(char transa, char transb, int64_t m, int64_t n, int64_t k,
                 float alpha, const float *A, int64_t lda, const float *B, int64_t ldb,
                 float beta, float *C, int64_t ldc, blas3_stream_t stream);
+
+/* SGEMM with A STREAMED in column panels (transa = 'N'; multi-GPU row F1,
+ * the device-side consumption of a panel-pipelined broadcast, P:382 future
+ * work).  Same arithmetic and result as blas3_sgemm -- bit for bit, one
+ * kernel, k-blocks in the same order -- but the kernel may start before all
+ * of A has arrived: A's columns come in panels of `panel_k` columns (a
+ * multiple of 32), and panel p (columns [p*panel_k, (p+1)*panel_k)) is read
+ * only once panel_ready[p] >= ready_value.  Another stream or device agent
+ * (e.g. an NCCL broadcast of the panel followed by blas3_signal on that
+ * stream) writes the flags; the kernel polls them with gpu-scope acquires and
+ * orders its TMA reads after them.  The flags are caller-owned device memory
+ * (ceil(k / panel_k) uint32), never reset by the library: give every call a
+ * larger ready_value.  A panel that never arrives traps the kernel after 4 s
+ * (a broken pipeline fails loudly instead of hanging).
+ * XERBLA: as blas3_sgemm, plus 1 transa != 'N', 14 panel_ready NULL, 15 panel_k
+ * not a positive multiple of 32.  BLAS3_ERR_UNSUPPORTED in SIMT mode or when A
+ * / B are not TMA-addressable (16-B aligned, ld % 4 == 0). */
+int blas3_sgemm_streamed(char transa, char transb, int64_t m, int64_t n, int64_t k,
+                         float alpha, const float *A, int64_t lda, const float *B, int64_t ldb,
+                         float beta, float *C, int64_t ldc, const uint32_t *panel_ready,
+                         int64_t panel_k, uint32_t ready_value, blas3_stream_t stream);
+
+/* Stream-ordered release write: *flag = value once every earlier operation on
+ * `stream` has completed (a one-thread kernel: fence, then st.release.gpu).
+ * The producer side of blas3_sgemm_streamed's panel flags.  Returns 0 or
+ * BLAS3_ERR_CUDA. */
+int blas3_signal(uint32_t *flag, uint32_t value, blas3_stream_t stream);
 
 /* SSYMM: side=L: C <- alpha*A*B + beta*C (A m x m);
  *        side=R: C <- alpha*B*A + beta*C (A n x n).

@@ -39,6 +39,9 @@ _SIGS = {
     "blas3_ssyr2k": [_c, _c, _i64, _i64, _f, _p, _i64, _p, _i64, _f, _p, _i64, _p],
     "blas3_strmm": [_c, _c, _c, _c, _i64, _i64, _f, _p, _i64, _p, _i64, _p],
     "blas3_strsm": [_c, _c, _c, _c, _i64, _i64, _f, _p, _i64, _p, _i64, _p],
+    "blas3_sgemm_streamed": [_c, _c, _i64, _i64, _i64, _f, _p, _i64, _p, _i64, _f, _p, _i64, _p, _i64,
+                             ctypes.c_uint32, _p],
+    "blas3_signal": [_p, ctypes.c_uint32, _p],
     "blas3_set_math_mode": [_i],
     "blas3_get_math_mode": [],
     "blas3_set_workspace": [_p, ctypes.c_size_t],
@@ -142,6 +145,32 @@ def sgemm(transa, transb, alpha, A, B, beta, C):
     _need("B", B, *((n, k) if _t(transb) else (k, n)))
     _chk("blas3_sgemm", blas3_sgemm(_ch(transa), _ch(transb), m, n, k, alpha, pa, lda, pb, ldb,  # noqa: F821
                                     beta, pc, ldc, _stream()))
+
+
+def sgemm_streamed(transa, transb, alpha, A, B, beta, C, ready, panel_k, value):
+    """C <- alpha*A*op(B) + beta*C with A arriving in column panels of panel_k
+    columns: panel p is read once ready[p] >= value (ready: a 1-D int32 CUDA
+    tensor of uint32 flags, written by another stream, e.g. via signal())."""
+    import torch
+    pc, m, n, ldc = _mat(C, "C")
+    pa, ar, ac, lda = _mat(A, "A")
+    pb, br, bc, ldb = _mat(B, "B")
+    k = ac
+    _need("A", A, m, k)
+    _need("B", B, *((n, k) if _t(transb) else (k, n)))
+    if not isinstance(ready, torch.Tensor) or not ready.is_cuda or ready.dtype != torch.int32:
+        raise TypeError("ready must be an int32 CUDA tensor")
+    if ready.numel() < -(-k // int(panel_k)):
+        raise ValueError("ready holds fewer flags than A has panels")
+    _chk("blas3_sgemm_streamed", blas3_sgemm_streamed(  # noqa: F821
+        _ch(transa), _ch(transb), m, n, k, alpha, pa, lda, pb, ldb, beta, pc, ldc, ready.data_ptr(),
+        int(panel_k), int(value) & 0xFFFFFFFF, _stream()))
+
+
+def signal(ready, index, value):
+    """Stream-ordered release write ready[index] = value on the current stream."""
+    _chk("blas3_signal", blas3_signal(ready.data_ptr() + 4 * int(index), int(value) & 0xFFFFFFFF,  # noqa: F821
+                                      _stream()))
 
 
 def ssymm(side, uplo, alpha, A, B, beta, C):
@@ -265,6 +294,6 @@ def launch_count(path=None):
     return int(blas3_launch_count_by_path(path))  # noqa: F821
 
 
-__all__ = ["sgemm", "ssymm", "ssyrk", "ssyr2k", "strmm", "strsm", "set_math_mode",
+__all__ = ["sgemm", "sgemm_streamed", "signal", "ssymm", "ssyrk", "ssyr2k", "strmm", "strsm", "set_math_mode",
            "get_math_mode", "launch_count", "colmajor", "from_fortran", "Blas3Error",
            "MATH_3XTF32", "MATH_SIMT_FP32", *EXPORTED]

@@ -199,6 +199,7 @@ static Problem problem(int64_t M, int64_t N, float alpha, float beta, const floa
   P.kc = (int32_t)opt(BLAS3_OPT_TC_KC);
   P.c_vec = 0;
   P.c_pf_map = -1;
+  P.a_ready = nullptr;
   return P;
 }
 
@@ -284,6 +285,7 @@ const char *blas3_error_string(int code) {
     case BLAS3_ERR_ARCH: return "current device is not sm_100 (B200)";
     case BLAS3_ERR_ALLOC: return "scratch allocation failed";
     case BLAS3_ERR_TMA: return "TMA tensor-map encoding failed";
+    case BLAS3_ERR_UNSUPPORTED: return "configuration not supported by this entry point";
     default: return code > 0 ? "invalid argument (value = 1-based XERBLA position)" : "unknown error";
   }
 }
@@ -325,6 +327,49 @@ int blas3_sgemm(char transa, char transb, int64_t m, int64_t n, int64_t k, float
     P.seg[0].a = dense(Wm.p, ldw, false);
   }
   return finish(run_problem(P, s, sms));
+}
+
+// ------------------------------------------------------------------- SGEMM, A streamed in panels
+int blas3_sgemm_streamed(char transa, char transb, int64_t m, int64_t n, int64_t k, float alpha,
+                         const float *A, int64_t lda, const float *B, int64_t ldb, float beta, float *C,
+                         int64_t ldc, const uint32_t *panel_ready, int64_t panel_k, uint32_t ready_value,
+                         blas3_stream_t stream) {
+  CallOpts call_opts;
+  const bool tb = up(transb) != 'N';
+  if (up(transa) != 'N') return 1;             // A's panels are K-ranges of its columns
+  if (!is_trans(transb)) return 2;
+  if (m < 0) return 3;
+  if (n < 0) return 4;
+  if (k < 0) return 5;
+  if (lda < mx1(m)) return 8;
+  if (ldb < mx1(tb ? n : k)) return 10;
+  if (ldc < mx1(m)) return 13;
+  if (!panel_ready) return 14;
+  if (panel_k <= 0 || panel_k % 32) return 15;
+  if (m == 0 || n == 0 || ((alpha == 0.f || k == 0) && beta == 1.f)) return 0;
+  if (!C) return 12;
+  const bool reads_ab = alpha != 0.f && k > 0;
+  if (reads_ab && !A) return 7;
+  if (reads_ab && !B) return 9;
+  int sms, rc = device_check(sms);
+  if (rc) return rc;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!reads_ab) return finish(launch_scale(C, ldc, m, n, beta, 0, s) ? BLAS3_ERR_CUDA : 0);
+  Problem P = problem(m, n, alpha, beta, C, ldc, C, ldc);
+  P.seg[0].a = dense(A, lda, false);
+  P.seg[0].b = dense(B, ldb, !tb);
+  P.seg[0].K = k;
+  P.a_ready = panel_ready;
+  P.a_panel_kb = (int32_t)(panel_k / 32);
+  P.a_ready_val = ready_value;
+  // the panel wait lives in the tcgen05 producer (no host synchronisation anywhere)
+  if (!tensor_mode() || !tc_eligible(P)) return BLAS3_ERR_UNSUPPORTED;
+  return finish(run_problem(P, s, sms));
+}
+
+int blas3_signal(uint32_t *flag, uint32_t value, blas3_stream_t stream) {
+  if (!flag) return 1;
+  return finish(launch_signal(flag, value, (cudaStream_t)stream) ? BLAS3_ERR_CUDA : 0);
 }
 
 // ------------------------------------------------------------------- SSYMM

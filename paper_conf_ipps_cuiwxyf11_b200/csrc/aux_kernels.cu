@@ -378,6 +378,17 @@ trsm_diag_inv_kernel(const float *A, int64_t lda, int64_t n, int stored_lower, i
   }
 }
 
+// blas3_signal: a stream-ordered release write of a flag
+__global__ void signal_kernel(uint32_t *flag, uint32_t value) {
+  __threadfence();
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(flag), "r"(value) : "memory");
+}
+int launch_signal(uint32_t *flag, uint32_t value, cudaStream_t s) {
+  signal_kernel<<<1, 1, 0, s>>>(flag, value);
+  note_launch();
+  return cudaGetLastError() == cudaSuccess ? 0 : -1;
+}
+
 int launch_trsm_diag_inv(const float *A, int64_t lda, int64_t n, int stored_lower, int unit,
                          float *Dinv, int64_t ldD, cudaStream_t s) {
   if (ldD % DNB) return -1;

@@ -38,6 +38,9 @@ enum MatMode : int { MAT_TRANS = 0, MAT_SYM = 1, MAT_TRI = 2 };
 int launch_materialize(float *dst, int64_t ldd, const float *src, int64_t lds, int64_t rows,
                        int64_t cols, int mode, int lower, int trans, int unit, cudaStream_t s);
 
+// stream-ordered release write *flag = value (blas3_signal)
+int launch_signal(uint32_t *flag, uint32_t value, cudaStream_t s);
+
 // TRSM diagonal blocks: for every 128 x 128 diagonal block b of L, where L
 // is the stored triangle of A brought to lower form (L(i,j) = A(i,j) if A is
 // stored lower, A(j,i) if stored upper; unit -> L(i,i) = 1), writes inv(L_bb)

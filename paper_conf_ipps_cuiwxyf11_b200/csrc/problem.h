@@ -93,6 +93,11 @@ struct Problem {
   // tensor-map slot of Cin for the L2 prefetch of C tiles, or -1
   int32_t c_vec;
   int32_t c_pf_map;
+  // streamed A (blas3_sgemm_streamed, segment 0): k-block kb of A may be
+  // loaded once a_ready[kb / a_panel_kb] >= a_ready_val (null: A resident)
+  const uint32_t *a_ready;
+  int32_t a_panel_kb;
+  uint32_t a_ready_val;
 };
 
 HD int64_t batch_off(const BatchStride &s, int64_t b, int64_t per) {

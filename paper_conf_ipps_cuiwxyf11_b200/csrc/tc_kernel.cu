@@ -688,6 +688,7 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
     if (lane == 0) {
       for (int i = 0; i < NMAPS; ++i) ptx::tma_prefetch(&prm.maps[i]);
       uint32_t it = 0;
+      int64_t a_ready_upto = 0;              // streamed A: panels [0, this) seen ready
       for (uint32_t qi = 0;;) {
         int64_t tb;
         const int slot = qi % TQ;
@@ -765,6 +766,12 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
             const uint32_t ph = (it / RS) & 1;
             const int64_t k0 = kb * BK;
             const StageInfo si = stage_at<CG>(bd, P, sg, m0, n0, kb);
+            if (P.a_ready != nullptr && s == 0 && kb / P.a_panel_kb >= a_ready_upto) {
+              // streamed A: its panel has landed (acquire), then the TMA reads it
+              spin_until(P.a_ready + kb / P.a_panel_kb, P.a_ready_val);
+              asm volatile("fence.proxy.async.global;" ::: "memory");
+              a_ready_upto = kb / P.a_panel_kb + 1;
+            }
             ptx::mbar_wait(&bars->empty[rs], ph ^ 1);
             if (P.dbg & 16) { ptx::mbar_arrive(&bars->full[rs]); continue; }   // diag: no loads
             ptx::mbar_arrive_expect_tx(&bars->full[rs], (HA + HB) * BK * 4);

@@ -26,7 +26,10 @@ landed, so the exposed broadcast is about one panel.  For a structured A only
 the stored triangle travels, one TRAPEZOID per column panel (columns [p0, p1),
 rows [p0, n) of a lower / [0, p1) of an upper triangle), packed into a
 contiguous staging buffer for NCCL: half the NVLink bytes.  The consumers:
-  * SGEMM NN   -- panel p is the K-range p: C += alpha A[:, p] B[p, :];
+  * SGEMM NN   -- panel p is the K-range p.  Default: ONE streamed GEMM whose
+                  producer waits per k-block for its panel's flag (device-side
+                  consumption, blas3_sgemm_streamed); alternative: one GEMM per
+                  landed panel, C += alpha A[:, p] B[p, :];
   * SSYMM L    -- panel p contributes its diagonal block by SSYMM and its
                   off-diagonal rectangle R twice, C_below += R B_p (NN) and
                   C_p += R^T B_below (TN): sym(A) = sum of those (planner
@@ -75,6 +78,15 @@ def k_panels(k: int, panels: int, align: int = 32) -> List[Tuple[int, int]]:
     """K-range panels for the pipelined broadcast (multiples of the k-block)."""
     panels = max(1, min(panels, -(-k // align)))
     return [p for p in (slab(k, panels, i, align) for i in range(panels)) if p[1] > p[0]]
+
+
+def uniform_panels(k: int, panels: int, align: int = 32) -> List[Tuple[int, int]]:
+    """K-range panels of ONE width (a multiple of `align`; the last one
+    ragged), as the streamed GEMM expects: panel p = k-block // width."""
+    if k <= 0:
+        return []
+    w = -(-(-(-k // max(1, panels))) // align) * align
+    return [(c0, min(k, c0 + w)) for c0 in range(0, k, w)]
 
 
 def trapezoid_rows(n: int, p0: int, p1: int, lower: bool) -> Tuple[int, int]:
@@ -236,13 +248,37 @@ class _Pipeline:
                 consume(i, p0, p1)
 
 
+_FLAGS = {}
+
+
+def _panel_flags(device, n):
+    """Per-device uint32 panel flags and a monotonically growing call value
+    (the library never resets them: every call waits for a larger value)."""
+    import torch
+    key = str(device)
+    if key not in _FLAGS or _FLAGS[key][0].numel() < n:
+        _FLAGS[key] = [torch.zeros(max(64, n), dtype=torch.int32, device=device), 0]
+    _FLAGS[key][1] += 1
+    return _FLAGS[key][0], _FLAGS[key][1]
+
+
 def sgemm(transa, transb, alpha, A, B_slab, beta, C_slab, root=0, group=None, panels=8,
-          pipeline=None, reserve_sms=16):
+          pipeline=None, reserve_sms=16, device_side=True):
     """C_slab <- alpha*op(A)*op(B)_slab + beta*C_slab on this rank's columns.
 
     A is replicated from `root` (NCCL broadcast).  For transa='N' the
-    broadcast is pipelined in K panels on a side stream, overlapped with the
-    panel GEMMs on the compute stream (`pipeline` defaults to world > 1)."""
+    broadcast is pipelined in K panels on a comm stream (`pipeline` defaults
+    to world > 1):
+      * device_side=True (default, row F1): ONE streamed GEMM
+        (blas3_sgemm_streamed) starts at once; its producer waits, per
+        k-block, for the flag of the panel holding it, which the comm stream
+        sets (blas3_signal) after each panel's broadcast.  Same result as a
+        plain SGEMM bit for bit, C read and written once.  The GEMM leaves
+        `reserve_sms` SMs to NCCL for its whole run (the broadcast cannot
+        progress without SMs: the persistent grid would otherwise wait on it
+        forever -- the 4 s trap of the panel wait);
+      * device_side=False: one GEMM per panel as it lands (host-sequenced),
+        beta on the first panel, SMs reserved while panels are in flight."""
     b3 = _b3()
     world, _ = world_rank(group)
     if pipeline is None:
@@ -252,6 +288,23 @@ def sgemm(transa, transb, alpha, A, B_slab, beta, C_slab, root=0, group=None, pa
         b3.sgemm(transa, transb, alpha, A, B_slab, beta, C_slab)
         return
     pan = k_panels(A.shape[1], panels)
+    if device_side and b3.get_math_mode() != b3.MATH_SIMT_FP32:
+        import torch
+        pan = uniform_panels(A.shape[1], panels)        # the kernel maps k-block -> panel by division
+        flags, value = _panel_flags(A.device, len(pan))
+        compute = torch.cuda.current_stream()
+        comm = torch.cuda.Stream()
+        comm.wait_stream(compute)                  # A's buffer / flags free on both streams
+        with torch.cuda.stream(comm):
+            for i, (c0, c1) in enumerate(pan):
+                if world > 1:
+                    _bcast(A[:, c0:c1], root, group)
+                b3.signal(flags, i, value)
+        nsm = torch.cuda.get_device_properties(compute.device).multi_processor_count
+        with b3.options(max_sms=max(2, nsm - max(0, int(reserve_sms)))):
+            b3.sgemm_streamed("N", "N", alpha, A, B_slab, beta, C_slab, flags, pan[0][1] - pan[0][0], value)
+        compute.wait_stream(comm)                  # the comm stream's work is part of the call
+        return
 
     def consume(i, c0, c1):
         b3.sgemm("N", "N", alpha, A[:, c0:c1], B_slab[c0:c1], beta if i == 0 else 1.0, C_slab)

@@ -82,6 +82,28 @@ def test_sgemm_xerbla(lib):
     assert call(ta=b"c") == 12                   # 'C' == 'T', lowercase accepted; then NULL C
 
 
+def test_sgemm_streamed_xerbla(lib):
+    f = lib.blas3_sgemm_streamed
+    flag = (ctypes.c_uint32 * 4)()
+    fp = ctypes.addressof(flag)
+    ok = dict(ta=b"N", tb=b"N", m=4, n=4, k=64, lda=4, ldb=64, ldc=4, fl=fp, pk=32)
+
+    def call(**kw):
+        a = {**ok, **kw}
+        return f(a["ta"], a["tb"], a["m"], a["n"], a["k"], 1.0, NULL, a["lda"], NULL, a["ldb"], 0.0,
+                 NULL, a["ldc"], a["fl"], a["pk"], 1, NULL)
+    assert call(ta=b"T") == 1                    # A's panels are K-ranges of its columns: 'N' only
+    assert call(ta=b"X") == 1
+    assert call(tb=b"Q") == 2
+    assert call(m=-1) == 3 and call(n=-1) == 4 and call(k=-1) == 5
+    assert call(lda=3) == 8 and call(ldb=63) == 10 and call(ldc=3) == 13
+    assert call(fl=NULL) == 14
+    assert call(pk=0) == 15 and call(pk=48) == 15 and call(pk=-32) == 15
+    assert call(m=0) == 0                        # quick return before any device work
+    assert lib.blas3_signal(NULL, 1, NULL) == 1
+    assert lib.blas3_error_string(-5).decode().startswith("configuration not supported")
+
+
 def test_ssymm_xerbla(lib):
     f = lib.blas3_ssymm
     call = lambda side=b"L", uplo=b"L", m=4, n=3, lda=4, ldb=4, ldc=4: f(  # noqa: E731

@@ -43,6 +43,17 @@ def test_balanced_triangle_slabs(n, world, lower):
     assert max(areas) / min(areas) < (1.001 if n % (8 * world) == 0 else 1.05)   # balanced
 
 
+@pytest.mark.parametrize("k,panels", [(8192, 8), (1000, 8), (100, 8), (32, 8), (4097, 3)])
+def test_uniform_panels(k, panels):
+    """The streamed GEMM maps k-block -> panel by division: one width, a
+    multiple of 32, the last panel ragged, every column once."""
+    pan = d3.uniform_panels(k, panels)
+    w = pan[0][1] - pan[0][0]
+    assert w % 32 == 0 and all(b - a == w for a, b in pan[:-1]) and 0 < pan[-1][1] - pan[-1][0] <= w
+    assert [c for a, b in pan for c in range(a, b)] == list(range(k))
+    assert len(pan) <= panels
+
+
 def test_k_panels():
     assert d3.k_panels(8192, 8) == [(i * 1024, (i + 1) * 1024) for i in range(8)]
     p = d3.k_panels(100, 8)
