@@ -96,8 +96,8 @@ int blas3_sgemm(char transa, char transb, int64_t m, int64_t n, int64_t k,
 
 /* SGEMM with A STREAMED in column panels (transa = 'N'; multi-GPU row F1,
  * the device-side consumption of a panel-pipelined broadcast, P:382 future
- * work).  Same arithmetic and result as blas3_sgemm -- bit for bit, one
- * kernel, k-blocks in the same order -- but the kernel may start before all
+ * work).  Same arithmetic and result as blas3_sgemm (bit for bit at the same
+ * SM count: one kernel, k-blocks in the same order) -- but it may start before all
  * of A has arrived: A's columns come in panels of `panel_k` columns (a
  * multiple of 32), and panel p (columns [p*panel_k, (p+1)*panel_k)) is read
  * only once panel_ready[p] >= ready_value.  Another stream or device agent

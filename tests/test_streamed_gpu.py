@@ -4,7 +4,8 @@ writes A's column panels into the operand buffer (after a delay, so the GEMM
 really starts before its data) and releases each panel's flag with
 blas3_signal; the GEMM is launched at once on the compute stream.  The result
 must equal a plain SGEMM bit for bit (same kernel, same k order), whatever
-order the panels arrive in.  Runs in a subprocess: a broken flag protocol
+order the panels arrive in (at the same SM count: the split-tail plan depends
+on it).  Runs in a subprocess: a broken flag protocol
 traps the kernel (4 s) and would poison the CUDA context of the test run."""
 import os
 import subprocess
@@ -31,7 +32,8 @@ for (m, n, k, panels, tb, order) in [(1000, 1200, 2048, 8, "N", "fwd"), (512, 76
     C = gen.uniform(m, n, "st-c")
     dA_src, dB = dev(A), dev(B)
     want = dev(C)
-    b3.sgemm("N", tb, 1.5, dA_src, dB, 0.5, want)
+    with b3.options(max_sms=132):                         # the same launch shape (split tail) as below
+        b3.sgemm("N", tb, 1.5, dA_src, dB, 0.5, want)
     pan = d3.uniform_panels(k, panels)
     flags = torch.zeros(len(pan), dtype=torch.int32, device="cuda")
     for value in (1, 2):                                  # two calls on the same flags
@@ -55,7 +57,9 @@ for (m, n, k, panels, tb, order) in [(1000, 1200, 2048, 8, "N", "fwd"), (512, 76
         ok &= same
 # the dist executor's device-side path at world size 1 (flags only, no broadcast)
 A = gen.uniform(1024, 2048, "sd-a"); B = gen.uniform(2048, 512, "sd-b"); C = gen.uniform(1024, 512, "sd-c")
-want = dev(C); b3.sgemm("N", "N", 1.5, dev(A), dev(B), 0.5, want)
+want = dev(C)
+with b3.options(max_sms=torch.cuda.get_device_properties(0).multi_processor_count - 16):
+    b3.sgemm("N", "N", 1.5, dev(A), dev(B), 0.5, want)
 got = dev(C); d3.sgemm("N", "N", 1.5, dev(A), dev(B), 0.5, got, panels=8, pipeline=True, device_side=True)
 torch.cuda.synchronize()
 same = np.array_equal(bits(got), bits(want))
