@@ -269,6 +269,14 @@ int blas3_get_math_mode(void);
  *                          groups ahead of its use; 0 (default) one group ahead in
  *                          registers (measured within noise of each other: SGEMM
  *                          +2%, tall-skinny SSYRK -2%)
+ *   BLAS3_OPT_TRSM_PANEL   [BLAS3_TRSM_PANEL] 1 (default): STRSM's first processed
+ *                          panel by the diagonal-panel solver -- one CTA pair per
+ *                          128 right-hand sides forward-substitutes the whole
+ *                          panel (256-row blocks, precomputed couplings
+ *                          -inv(op(A)_ss) op(A)_sf), no grid-wide dependency
+ *                          steps; 0: the fused doubling + geometric chain.  Used
+ *                          when the panel's order is a multiple of 256 and B is
+ *                          16-B aligned with ldb % 4 == 0
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */
@@ -281,7 +289,7 @@ enum {
     BLAS3_OPT_TRSM_FIRST_YM = 15, BLAS3_OPT_TRSM_FIRST_FUSED = 16, BLAS3_OPT_TRSM_FIRST_SPLIT = 17,
     BLAS3_OPT_TRSM_FIRST_ALL = 18, BLAS3_OPT_TC_RASTER = 19, BLAS3_OPT_TC_KC = 20,
     BLAS3_OPT_TC_VEC_STORE = 21, BLAS3_OPT_MAX_SMS = 22, BLAS3_OPT_TC_C_PREFETCH = 23,
-    BLAS3_OPT_TC_C_ASYNC = 24, BLAS3_OPT_COUNT = 25
+    BLAS3_OPT_TC_C_ASYNC = 24, BLAS3_OPT_TRSM_PANEL = 25, BLAS3_OPT_COUNT = 26
 };
 int blas3_set_option(int key, int64_t value);
 int64_t blas3_get_option(int key);

@@ -52,6 +52,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_MAX_SMS", 0, 0, 4096, false},
     {"BLAS3_TC_C_PREFETCH", 1, 0, 1, false},
     {"BLAS3_TC_C_ASYNC", 0, 0, 1, false},
+    {"BLAS3_TRSM_PANEL", 1, 0, 1, false},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;
@@ -1023,6 +1024,54 @@ static int strsm_first_fused(const TrsmGeom &g, const std::vector<GeoPair> &gp, 
   return rc == 0 ? 0 : (rc == -4 ? BLAS3_ERR_TMA : BLAS3_ERR_CUDA);
 }
 
+// The first processed panel by the diagonal-panel solver (BLAS3_OPT_TRSM_PANEL,
+// panel_kernel.cu): level 0 of the panel's doubling (its 256-block inverses),
+// the couplings M = -inv(op(A)_ss) op(A)_sf of every 256-block s (one batched
+// GEMM over the whole panel row -- the kernel reads only the solved part) and
+// alpha * inv(op(A)_ss) on M's diagonal, then ONE launch in which every CTA
+// pair forward-substitutes its 128 right-hand sides through the panel.
+// Returns 1 if not applicable (nothing enqueued), 0, or < 0 on an error.
+static int strsm_first_panel(const TrsmGeom &g, int64_t pfirst, float *Mw, void *pws, cudaStream_t s, int sms) {
+  const int64_t NBO = g.NBO, p0 = pfirst * NBO, R = imin(NBO, g.nt - p0), ldm = R;
+  if (R % 256 || R > 8192 || (reinterpret_cast<uintptr_t>(g.B) % 16) || g.ldb % 4) return 1;
+  const int64_t nb = R / 256;
+  float *Dp = g.D + pfirst * NBO * NBO;
+  const float *Ap = g.A + p0 * (1 + g.lda);
+  Problem P;
+  if (g.left) {        // M(s, c) = -sum_k inv(op(A)_ss)(r, k) op(A)(s_lo + k, p0 + c), batch over s
+    P = problem(256, R, -1.f, 0.f, nullptr, 0, Mw, ldm);
+    P.seg[0].a = tri_zeroed(Dp, NBO, true, !g.lower_op);
+    P.seg[0].b = dense(Ap, g.lda, !g.ta);
+    P.rev_m = tri_kle(P.seg[0].a);
+    P.bs_a = {0, 256 * (1 + NBO)};
+    P.bs_b = {0, g.ta ? 256 * g.lda : 256};
+    P.bs_c = {0, 256};
+  } else {             // M(f, s) = -sum_k op(A)(p0 + f, s_lo + k) inv(op(A)_ss)(k, c)
+    P = problem(R, 256, -1.f, 0.f, nullptr, 0, Mw, ldm);
+    P.seg[0].a = dense(Ap, g.lda, g.ta);
+    P.seg[0].b = tri_zeroed(Dp, NBO, true, g.lower_op);
+    P.rev_n = tri_kle(P.seg[0].b);
+    P.bs_a = {0, g.ta ? 256 : 256 * g.lda};
+    P.bs_b = {0, 256 * (1 + NBO)};
+    P.bs_c = {0, 256 * ldm};
+  }
+  P.seg[0].K = 256;
+  P.nbatch = nb;
+  P.per = nb;
+  if (nb > 1 && !tc_eligible(P)) return 1;
+  int rc;
+  std::vector<LevelProblem> lv;
+  trsm_doubling_problems(Ap, g.lda, R, g.lower, Dp, g.Tw, lv);
+  for (const LevelProblem &q : lv)
+    if (q.lvl == 0 && (rc = run_problem(q.P, s, sms))) return rc;
+  if (nb > 1 && (rc = run_problem(P, s, sms))) return rc;
+  if (launch_trsm_panel_diag(Dp, NBO, Mw, ldm, R, g.lower_op, g.alpha, s)) return BLAS3_ERR_CUDA;
+  float *X = g.left ? g.B + p0 : g.B + p0 * g.ldb;
+  rc = launch_trsm_panel(Mw, ldm, X, g.ldb, !g.left, R, g.other, g.forward, (int)opt(BLAS3_OPT_TC_KC), pws, s,
+                         sms);
+  return rc == 0 ? 0 : (rc == -4 ? BLAS3_ERR_TMA : BLAS3_ERR_CUDA);
+}
+
 int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t n, float alpha,
                 const float *A, int64_t lda, float *B, int64_t ldb, blas3_stream_t stream) {
   CallOpts call_opts;
@@ -1090,9 +1139,18 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   const int64_t pfirst = forward ? 0 : npanel - 1;
   int nlvl = 0;
   for (int64_t sz = 128; sz < NBO; sz *= 2) ++nlvl;
+  // BLAS3_OPT_TRSM_PANEL: the first panel by the diagonal-panel solver (its
+  // M workspace after W); the geometric chain's Y/M are then not needed
+  const int64_t r_first = imin(NBO, nt - pfirst * NBO);
+  const bool use_panel = opt(BLAS3_OPT_TRSM_PANEL) != 0 && tensor_mode() && r_first % 256 == 0;
+  Scratch Mw;
+  const size_t m_bytes = (size_t)r_first * r_first * sizeof(float);
+  if (use_panel &&
+      (rc = get_scratch(Mw, m_bytes + trsm_panel_ws_bytes(other, sms), s, aop_bytes + d_bytes + t_bytes + w_bytes)))
+    return rc;
   std::vector<GeoPair> gp;
   Scratch YM;
-  const bool use_ym = opt(BLAS3_OPT_TRSM_FIRST_YM) != 0 || opt(BLAS3_OPT_TRSM_FIRST_FUSED) != 0;
+  const bool use_ym = !use_panel && (opt(BLAS3_OPT_TRSM_FIRST_YM) != 0 || opt(BLAS3_OPT_TRSM_FIRST_FUSED) != 0);
   if (use_ym) {
     std::function<void(int64_t, int64_t)> pairs = [&](int64_t lo, int64_t w) {
       const int64_t e1 = imin(nt, lo + w);
@@ -1133,9 +1191,16 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // BLAS3_OPT_TRSM_FIRST_ALL: every panel's doubling inside the first panel's
   // fused launch (levels the chain needs first, the rest claimed after the
   // chain), on the whole grid -- no side stream competes for SMs
-  bool all_done = false;
-  if (opt(BLAS3_OPT_TRSM_FIRST_ALL) && opt(BLAS3_OPT_TRSM_FIRST_FUSED) && opt(BLAS3_OPT_TRSM_FIRST_SPLIT) == 0 &&
-      tensor_mode() && !gp.empty()) {
+  bool all_done = false, panel_done = false;
+  if (use_panel) {
+    const TrsmGeom g{left, lower, ta, unit, lower_op, forward, m, n, nt, NBO, npanel, other, alpha,
+                     A, lda, B, ldb, D.p, Tw.p + t_rest, W.p};
+    rc = strsm_first_panel(g, pfirst, Mw.p, reinterpret_cast<uint8_t *>(Mw.p) + m_bytes, s, sms);
+    if (rc < 0) return rc;
+    panel_done = rc == 0;
+  }
+  if (!panel_done && opt(BLAS3_OPT_TRSM_FIRST_ALL) && opt(BLAS3_OPT_TRSM_FIRST_FUSED) &&
+      opt(BLAS3_OPT_TRSM_FIRST_SPLIT) == 0 && tensor_mode() && !gp.empty()) {
     const TrsmGeom g{left, lower, ta, unit, lower_op, forward, m, n, nt, NBO, npanel, other, alpha,
                      A, lda, B, ldb, D.p, Tw.p, W.p};
     rc = strsm_first_fused(g, gp, pfirst, s, sms, -1, -1, true);
@@ -1158,8 +1223,8 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // stream, concurrently with the chain (they do not depend on X).
   std::vector<GeoPair> outer;                         // popped pairs, inner -> outer
   const int64_t fsplit = opt(BLAS3_OPT_TRSM_FIRST_SPLIT);
-  first_done = all_done;
-  if (!all_done && opt(BLAS3_OPT_TRSM_FIRST_FUSED) && tensor_mode() && !gp.empty()) {
+  first_done = all_done || panel_done;
+  if (!first_done && opt(BLAS3_OPT_TRSM_FIRST_FUSED) && tensor_mode() && !gp.empty()) {
     if (fsplit > 0)
       while (gp.size() >= 2 && gp.back().h >= fsplit && outer.size() < (size_t)MAX_LEVELS) { outer.insert(outer.begin(), gp.back()); gp.pop_back(); }
     const int64_t c_lo = outer.empty() ? -1 : outer[0].f_lo, c_hi = outer.empty() ? -1 : outer[0].f_hi;

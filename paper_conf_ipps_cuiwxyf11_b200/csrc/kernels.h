@@ -1,6 +1,7 @@
 // kernels.h -- internal launcher interface between the routine drivers
 // (abi.cu) and the device kernels.  Not part of the public C ABI.
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include "problem.h"
@@ -40,6 +41,29 @@ int launch_materialize(float *dst, int64_t ldd, const float *src, int64_t lds, i
 
 // stream-ordered release write *flag = value (blas3_signal)
 int launch_signal(uint32_t *flag, uint32_t value, cudaStream_t s);
+
+// 2-D fp32 TMA map (dim0 contiguous, extent d0; dim1 stride ld floats), box
+// box0 x box1, MN-major (mn32) or K-major staging swizzle.
+bool tma_map_f32(CUtensorMap *m, const float *ptr, int64_t d0, int64_t d1, int64_t ld, uint32_t box0,
+                 uint32_t box1, bool mn32);
+
+// STRSM diagonal-panel solve (panel_kernel.cu).  The R x R panel (R a
+// multiple of 256, at most 8192) in 256-row blocks, processing order forward
+// (block i at rows 256 i) or backward; M (R x R, column-major, ldm) holds
+// alpha * inv(op(A)_bb) on its diagonal blocks and the precomputed couplings
+// -inv(op(A)_ss) op(A)_sf (left: M(s,f)) / -op(A)_fs inv(op(A)_ss) (right:
+// M(f,s)) of every block s to the blocks f solved before it.  X is the panel
+// of B, solved in place: left X(k,n) = X[k + n ldx] (nrhs columns), right
+// X[n + k ldx] (nrhs rows).  One team of two CTA pairs per 256 right-hand
+// sides; ws: trsm_panel_ws_bytes(nrhs, num_sms) bytes of device workspace
+// (16-B aligned; the partials of the teams and their counters).
+size_t trsm_panel_ws_bytes(int64_t nrhs, int num_sms);
+int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool right, int64_t R,
+                      int64_t nrhs, bool forward, int kc, void *ws, cudaStream_t s, int num_sms);
+// M's diagonal blocks from the lower-form inverses of the panel-inverse
+// workspace (Dp: the panel's ldD x ldD inverse, its 256-blocks complete).
+int launch_trsm_panel_diag(const float *Dp, int64_t ldD, float *M, int64_t ldm, int64_t R, bool lower_op,
+                           float alpha, cudaStream_t s);
 
 // TRSM diagonal blocks: for every 128 x 128 diagonal block b of L, where L
 // is the stored triangle of A brought to lower form (L(i,j) = A(i,j) if A is

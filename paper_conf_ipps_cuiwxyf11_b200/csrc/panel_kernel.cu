@@ -1,0 +1,477 @@
+// panel_kernel.cu -- STRSM diagonal-panel solve (rows A7/A8 of the hot-path
+// table): every right-hand-side slab of 256 columns (rows for side=R) is
+// forward-substituted through the whole R x R diagonal panel by ONE team of
+// two CTA pairs, so the panel's dependency chain (Fig. 14
+// / Adaptor_Solver: X_i needs X_k, k < i) never becomes a grid-wide step.
+//
+// With the panel split into 256-row blocks (processing order i = 0..nblk-1;
+// block i at rows blk_row(i): 256 i forward, 256 (nblk-1-i) backward) and
+//     M(i, i) = alpha * inv(op(A)_ii)                     (diagonal blocks)
+//     M(i, j) = -inv(op(A)_ii) op(A)_ij, j solved before  (left; side=R transposed)
+// precomputed from A alone, block i of the solution is ONE sum of i + 1
+// "groups" of K = 256:
+//     X_i = M(i, i) B_i  +  sum_{j<i} M(i, j) X_j        (group 0, groups j + 1)
+// The team splits the groups of every block between its two pairs (host-side
+// greedy balance, hmask): member 0 always takes the newest group (j = i - 1,
+// the only one that waits for the block just solved), sums its partial with
+// the helper's (member 1, fp32 partial through L2) and stores X_i in place
+// over B_i; the helper's groups are older, so its partial runs ahead.  A pair
+// computes 256 x 256 tiles, the tcgen05 shape at which the 3xTF32 UMMAs run
+// at full rate (a 128-wide N takes as long per instruction as 256).
+//
+// Kernel structure (640 threads per CTA, the tc_kernel.cu roles):
+//   warp 0      TMA producer: M rows (its 128) x 32 k, X/B rows k x its 128 RHS
+//   warp 1      MMA issuer (leader CTA): 3xTF32 tcgen05.mma cta_group::2,
+//               M = N = 256, TMEM partials restarted every kc k-blocks
+//   warps 4-11  transform: lo = x - trunc_tf32(x) (hi is the raw TMA tile)
+//   warps 12-19 epilogue: partials -> register sum (+ the helper's partial) ->
+//               X_i stored -> release counter (member 0) / partial -> L2 (member 1)
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <atomic>
+#include <cstring>
+#include <mutex>
+#include <stdlib.h>
+
+#include "../../include/blas3.h"
+#include "kernels.h"
+#include "tc_ptx.h"
+
+namespace blas3 {
+namespace {
+
+constexpr int BK = 32;                     // k-block (elements)
+constexpr int HA = 128;                    // M rows staged per CTA (block = 256 per pair)
+constexpr int BLK = 256;                   // rows of X per block (UMMA M of the pair)
+constexpr int KB_BLK = BLK / BK;           // k-blocks per group (8)
+constexpr int PN = 256;                    // right-hand sides per team (UMMA N)
+constexpr int HB = PN / 2;                 // right-hand sides staged per CTA
+constexpr int RS = 4, LS = 2;              // raw / lo stages
+constexpr int NACC = 2;                    // TMEM partials (2 x 256 columns)
+constexpr int MAX_BLK = 32;                // blocks per panel (R <= 8192)
+constexpr int WARP_TMA = 0, WARP_MMA = 1, WARP_TR0 = 4, NUM_TR_WARPS = 8;
+constexpr int WARP_EPI0 = WARP_TR0 + NUM_TR_WARPS, NUM_EPI_WARPS = 8;
+constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;       // 640
+constexpr int TR_THREADS = NUM_TR_WARPS * 32, EPI_THREADS = NUM_EPI_WARPS * 32;
+constexpr int EPI_REGS = 144, OTHER_REGS = 64;
+constexpr int NCOL = PN / 2;               // columns per epilogue thread (two warps per lane quarter)
+constexpr int LAYOUT_K = 0, LAYOUT_MN = 1;
+constexpr size_t PART_FLOATS = (size_t)HA * PN;   // one CTA's partial (128 rows x 256)
+
+struct alignas(1024) Stage {
+  uint8_t A[HA * BK * 4];                  // 16 KiB
+  uint8_t B[HB * BK * 4];                  // 16 KiB
+};
+struct Bars {
+  uint64_t full[RS], empty[RS], ready[LS], lo_empty[LS];
+  uint64_t tfull[NACC], tempty[NACC];
+  uint32_t tmem_base;
+};
+constexpr size_t SMEM = sizeof(Stage) * (RS + LS) + sizeof(Bars) + 1024;
+
+struct PanelParams {
+  CUtensorMap mapA;                        // M: rk (left) / kr (right) view
+  CUtensorMap mapB;                        // X over B: kr (left) / rk (right) view
+  float *X;                                // panel origin: left X(k,n) = X[k + n ldx], right X[n + k ldx]
+  float *ws;                               // helper partials: [team][slot 2][rank 2][col 256][row 128]
+  uint32_t *ctr;                           // [team][2]: X blocks stored, partials written (x2 CTAs)
+  int64_t ldx, R, nrhs;
+  int32_t nblk, layA, layB, right, forward, kc, nslab, nteams;
+  int32_t dbg;                             // BLAS3_DEBUG_PANEL knock-outs (timing experiments only)
+  uint32_t hmask[MAX_BLK];                 // groups of block i summed by the helper (member 1)
+};
+
+// first row of processing block i
+__device__ __forceinline__ int64_t blk_row(const PanelParams &p, int i) {
+  return (int64_t)(p.forward ? i : p.nblk - 1 - i) * BLK;
+}
+// groups of block i summed by member h (bit g: group g; g = 0 the block's own
+// right-hand side, g >= 1 the solved block g - 1)
+__device__ __forceinline__ uint32_t groups_of(const PanelParams &p, int i, int h) {
+  const uint32_t all = i >= 31 ? 0xFFFFFFFFu : ((2u << i) - 1u);
+  return h ? p.hmask[i] : (all & ~p.hmask[i]);
+}
+
+__device__ __forceinline__ uint64_t op_desc(uint32_t base, int lay, int k8) {
+  if (lay == LAYOUT_MN) return ptx::smem_desc(base + k8 * 1024, BK * 128, 512, 1);
+  return ptx::smem_desc(base + k8 * 32, 16, 1024, 2);
+}
+__device__ __forceinline__ void load_op(const CUtensorMap *m, int lay, uint8_t *dst, int64_t r0,
+                                        int64_t k0, int rows, uint64_t *bar) {
+  if (lay == LAYOUT_MN) {
+    for (int c = 0; c < rows / 32; ++c)
+      ptx::tma_load_4d(m, bar, dst + c * (BK * 128), (int32_t)(r0 + 32 * c), (int32_t)k0, 0, 0);
+  } else {
+    ptx::tma_load_4d(m, bar, dst, (int32_t)k0, (int32_t)r0, 0, 0);
+  }
+}
+__device__ __forceinline__ void split_pass(const uint8_t *raw, uint8_t *lo, uint32_t bytes, int t) {
+  const float4 *r4 = reinterpret_cast<const float4 *>(raw);
+  float4 *l4 = reinterpret_cast<float4 *>(lo);
+#pragma unroll 4
+  for (uint32_t c = t; c < bytes / 16; c += TR_THREADS) {
+    const float4 v = r4[c];
+    float4 l;
+    l.x = v.x - __uint_as_float(__float_as_uint(v.x) & 0xFFFFE000u);
+    l.y = v.y - __uint_as_float(__float_as_uint(v.y) & 0xFFFFE000u);
+    l.z = v.z - __uint_as_float(__float_as_uint(v.z) & 0xFFFFE000u);
+    l.w = v.w - __uint_as_float(__float_as_uint(v.w) & 0xFFFFE000u);
+    l4[c] = l;
+  }
+}
+__device__ __forceinline__ void arrive_leader(uint64_t *bar, uint32_t rank, uint32_t id, uint32_t n,
+                                              bool first) {
+  ptx::named_bar_sync(id, n);
+  if (first) {
+    if (rank == 0) ptx::mbar_arrive(bar);
+    else ptx::mbar_arrive_cluster(bar, 0);
+  }
+}
+// Team hand-offs go through global counters (the two pairs of a team are
+// different clusters): release = __threadfence + atomicAdd after a CTA's
+// stores; acquire = ld.acquire.gpu poll, plus a proxy fence before TMA reads.
+__device__ __forceinline__ void wait_count(const uint32_t *ctr, uint32_t target) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+  if (v >= target) return;
+  unsigned long long t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  for (;;) {
+    __nanosleep(64);
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+    if (v >= target) return;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t - t0 > 4000000000ull) __trap();      // a team partner that never runs fails loudly
+  }
+}
+
+__global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_constant__ PanelParams prm) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t *smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
+  Stage *raw = reinterpret_cast<Stage *>(smem);
+  Stage *lo = raw + RS;
+  Bars *bars = reinterpret_cast<Bars *>(smem + sizeof(Stage) * (RS + LS));
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const uint32_t rank = ptx::cluster_ctarank();
+  const int pair = blockIdx.x / 2;
+  const int team = pair / 2, h = pair % 2;           // team member: 0 stores X, 1 helps
+  const int nblk = prm.nblk;
+  uint32_t *ctr_x = prm.ctr + 2 * team, *ctr_p = ctr_x + 1;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < RS; ++s) { ptx::mbar_init(&bars->full[s], 1); ptx::mbar_init(&bars->empty[s], 1); }
+    for (int s = 0; s < LS; ++s) { ptx::mbar_init(&bars->ready[s], 2); ptx::mbar_init(&bars->lo_empty[s], 1); }
+    for (int a = 0; a < NACC; ++a) { ptx::mbar_init(&bars->tfull[a], 1); ptx::mbar_init(&bars->tempty[a], 2); }
+    ptx::fence_mbar_init();
+  }
+  if (warp == WARP_MMA) ptx::tmem_alloc<2>(&bars->tmem_base, NACC * PN);
+  ptx::tc_fence_before();
+  ptx::cluster_sync();
+  ptx::tc_fence_after();
+  const uint32_t tmem = bars->tmem_base;
+  ptx::griddep_wait();
+
+#define BLAS3_DEC_REGS() asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(OTHER_REGS))
+#define BLAS3_INC_REGS() asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(EPI_REGS))
+  if (warp < WARP_TR0) {
+    BLAS3_DEC_REGS();
+    if (warp == WARP_TMA && lane == 0) {
+      // ============================ producer (each CTA stages its own halves)
+      ptx::tma_prefetch(&prm.mapA);
+      ptx::tma_prefetch(&prm.mapB);
+      uint32_t it = 0, gblk = 0, x_seen = 0;
+      for (int slab = team; slab < prm.nslab; slab += prm.nteams) {
+        const int64_t n0 = (int64_t)slab * PN + HB * rank;
+        const uint32_t gbase = gblk;
+        for (int i = 0; i < nblk; ++i, ++gblk) {
+          const int64_t r0 = blk_row(prm, i) + HA * rank;
+          for (uint32_t m = groups_of(prm, i, h); m; m &= m - 1) {
+            const int g = __ffs(m) - 1;
+            if (g > 0 && !(prm.dbg & 1)) {            // X of solved block g - 1 stored (both CTAs of member 0)
+              const uint32_t need = 2 * (gbase + g);
+              if (need > x_seen) {
+                wait_count(ctr_x, need);
+                asm volatile("fence.proxy.async.global;" ::: "memory");
+                x_seen = need;
+              }
+            }
+            const int64_t kg = blk_row(prm, g == 0 ? i : g - 1);
+            for (int w = 0; w < KB_BLK; ++w, ++it) {
+              const int rs = it % RS;
+              ptx::mbar_wait(&bars->empty[rs], ((it / RS) & 1) ^ 1);
+              ptx::mbar_arrive_expect_tx(&bars->full[rs], (HA + HB) * BK * 4);
+              load_op(&prm.mapA, prm.layA, raw[rs].A, r0, kg + w * BK, HA, &bars->full[rs]);
+              load_op(&prm.mapB, prm.layB, raw[rs].B, n0, kg + w * BK, HB, &bars->full[rs]);
+            }
+          }
+        }
+      }
+      for (int i = 0; i < RS; ++i, ++it) ptx::mbar_wait(&bars->empty[it % RS], ((it / RS) & 1) ^ 1);
+    } else if (warp == WARP_MMA && rank == 0) {
+      // ============================ MMA issuer (leader CTA)
+      const uint32_t idesc = ptx::idesc_tf32(BLK, PN, prm.layA == LAYOUT_MN, prm.layB == LAYOUT_MN);
+      uint32_t it = 0, cc = 0;
+      for (int slab = team; slab < prm.nslab; slab += prm.nteams) {
+        for (int i = 0; i < nblk; ++i) {
+          const int nkb = KB_BLK * __popc(groups_of(prm, i, h));
+          int left = 0;
+          uint32_t acc = 0, buf = 0;
+          for (int t = 0; t < nkb; ++t, ++it) {
+            if (left == 0) {
+              buf = cc % NACC;
+              ptx::mbar_wait_cluster(&bars->tempty[buf], ((cc / NACC) & 1) ^ 1);
+              ptx::tc_fence_after();
+              acc = 0;
+              left = prm.kc;
+            }
+            const int rs = it % RS, ls = it % LS;
+            ptx::mbar_wait_cluster(&bars->ready[ls], (it / LS) & 1);
+            ptx::tc_fence_after();
+            if (lane == 0) {
+              const uint32_t d = tmem + buf * PN;
+              const uint32_t hiA = ptx::smem_u32(raw[rs].A), hiB = ptx::smem_u32(raw[rs].B);
+              const uint32_t loA = ptx::smem_u32(lo[ls].A), loB = ptx::smem_u32(lo[ls].B);
+              if (!(prm.dbg & 8)) {
+                // cross terms first (small, into a fresh partial), then hi*hi (Q24)
+#pragma unroll
+                for (int k8 = 0; k8 < BK / 8; ++k8) {
+                  ptx::mma_tf32_ss_pair(d, op_desc(loA, prm.layA, k8), op_desc(hiB, prm.layB, k8), idesc, acc);
+                  ptx::mma_tf32_ss_pair(d, op_desc(hiA, prm.layA, k8), op_desc(loB, prm.layB, k8), idesc, 1);
+                  acc = 1;
+                }
+#pragma unroll
+                for (int k8 = 0; k8 < BK / 8; ++k8)
+                  ptx::mma_tf32_ss_pair(d, op_desc(hiA, prm.layA, k8), op_desc(hiB, prm.layB, k8), idesc, 1);
+              }
+              ptx::mma_commit_pair(&bars->empty[rs], 0x3);
+              ptx::mma_commit_pair(&bars->lo_empty[ls], 0x3);
+            }
+            acc = 1;
+            __syncwarp();
+            if (--left == 0 || t == nkb - 1) {
+              if (lane == 0) ptx::mma_commit_pair(&bars->tfull[buf], 0x3);
+              __syncwarp();
+              ++cc;
+              left = 0;
+            }
+          }
+        }
+      }
+    }
+  } else if (warp < WARP_EPI0) {
+    // ============================ transform (own halves)
+    BLAS3_DEC_REGS();
+    const int tt = threadIdx.x - WARP_TR0 * 32;
+    uint32_t it = 0;
+    for (int slab = team; slab < prm.nslab; slab += prm.nteams) {
+      for (int i = 0; i < nblk; ++i) {
+        const int nkb = KB_BLK * __popc(groups_of(prm, i, h));
+        for (int t = 0; t < nkb; ++t, ++it) {
+          const int rs = it % RS, ls = it % LS;
+          ptx::mbar_wait(&bars->full[rs], (it / RS) & 1);
+          ptx::mbar_wait(&bars->lo_empty[ls], ((it / LS) & 1) ^ 1);
+          if (!(prm.dbg & 2)) {
+            split_pass(raw[rs].A, lo[ls].A, HA * BK * 4, tt);
+            split_pass(raw[rs].B, lo[ls].B, HB * BK * 4, tt);
+          }
+          ptx::fence_proxy_async_smem();
+          arrive_leader(&bars->ready[ls], rank, 2, TR_THREADS, tt == 0);
+        }
+      }
+    }
+  } else {
+    // ============================ epilogue (own 128 rows; two warps per lane quarter)
+    BLAS3_INC_REGS();
+    const int q = warp & 3, half = (warp - WARP_EPI0) >> 2;
+    const bool lead = threadIdx.x == WARP_EPI0 * 32;
+    const int rloc = q * 32 + lane;                           // row within this CTA's 128
+    uint32_t cc = 0, gblk = 0;
+    for (int slab = team; slab < prm.nslab; slab += prm.nteams) {
+      const int64_t c0 = (int64_t)slab * PN + half * NCOL;     // first right-hand side of this thread
+      for (int i = 0; i < nblk; ++i, ++gblk) {
+        const int nkb = KB_BLK * __popc(groups_of(prm, i, h));
+        const int nch = nkb > 0 ? (nkb + prm.kc - 1) / prm.kc : 0;
+        float S[NCOL];
+#pragma unroll
+        for (int j = 0; j < NCOL; ++j) S[j] = 0.f;
+        for (int c = 0; c < nch; ++c, ++cc) {
+          const uint32_t buf = cc % NACC;
+          ptx::mbar_wait(&bars->tfull[buf], (cc / NACC) & 1);
+          ptx::tc_fence_after();
+          const uint32_t ta = tmem + buf * PN + half * NCOL + ((uint32_t)(q * 32) << 16);
+#pragma unroll
+          for (int g = 0; g < NCOL / 16; g += 2) {
+            uint32_t v[16], u[16];
+            ptx::tmem_ld_32x32b_x16(ta + g * 16, v);
+            ptx::tmem_ld_32x32b_x16(ta + (g + 1) * 16, u);
+            ptx::tmem_ld_wait();
+#pragma unroll
+            for (int j = 0; j < 16; ++j) S[g * 16 + j] += __uint_as_float(v[j]);
+#pragma unroll
+            for (int j = 0; j < 16; ++j) S[(g + 1) * 16 + j] += __uint_as_float(u[j]);
+          }
+          ptx::tc_fence_before();
+          arrive_leader(&bars->tempty[buf], rank, 3, EPI_THREADS, lead);
+        }
+        // this CTA's partial slot: [col][row] so a warp's accesses per column are one 128-B line
+        float *part = prm.ws + ((((size_t)team * 2 + (gblk & 1)) * 2 + rank) * PART_FLOATS) +
+                      (size_t)(half * NCOL) * HA + rloc;
+        if (h == 1) {
+          // helper: the slot was last read for block gblk - 2 (X of it stored)
+          if (lead && gblk >= 2) wait_count(ctr_x, 2 * (gblk - 1));
+          ptx::named_bar_sync(5, EPI_THREADS);
+#pragma unroll
+          for (int j = 0; j < NCOL; ++j) __stcg(part + (size_t)j * HA, S[j]);
+          ptx::named_bar_sync(5, EPI_THREADS);
+          if (lead) { __threadfence(); atomicAdd(ctr_p, 1u); }
+          continue;
+        }
+        // member 0: + the helper's partial, then X_i
+        if (lead) wait_count(ctr_p, 2 * (gblk + 1));
+        ptx::named_bar_sync(5, EPI_THREADS);
+#pragma unroll
+        for (int j = 0; j < NCOL; ++j) S[j] += __ldcg(part + (size_t)j * HA);
+        // X_i rows [blk_row + 128 rank, +128) x right-hand sides [c0, c0 + 128)
+        const int64_t row = blk_row(prm, i) + HA * rank + rloc;
+        const int64_t nval = prm.nrhs - c0;                  // valid columns (warp-uniform)
+        if (!prm.right) {
+          float *p = prm.X + row + c0 * prm.ldx;
+#pragma unroll
+          for (int j = 0; j < NCOL; ++j) {
+            if (j < nval) *p = S[j];
+            p += prm.ldx;
+          }
+        } else {
+          float *p = prm.X + c0 + row * prm.ldx;
+          const bool vec = nval >= NCOL && (prm.ldx % 4) == 0 && (reinterpret_cast<uintptr_t>(p) % 16) == 0;
+          if (vec) {
+#pragma unroll
+            for (int j = 0; j < NCOL; j += 4)
+              *reinterpret_cast<float4 *>(p + j) = make_float4(S[j], S[j + 1], S[j + 2], S[j + 3]);
+          } else {
+#pragma unroll
+            for (int j = 0; j < NCOL; ++j)
+              if (j < nval) p[j] = S[j];
+          }
+        }
+        ptx::named_bar_sync(5, EPI_THREADS);
+        if (lead) { __threadfence(); atomicAdd(ctr_x, 1u); }
+      }
+    }
+  }
+
+  ptx::tc_fence_before();
+  ptx::cluster_sync();
+  if (warp == WARP_MMA) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc<2>(tmem, NACC * PN);
+  }
+#undef BLAS3_DEC_REGS
+#undef BLAS3_INC_REGS
+}
+
+// M's diagonal blocks: alpha * inv(op(A)_bb), natural column-major, zeros in
+// the blank triangle, from the lower-form inverses in the panel-inverse
+// workspace (inv(L_bb); op(A)_bb = L_bb if lower_op, else L_bb^T).
+__global__ void panel_diag_kernel(const float *Dp, int64_t ldD, float *M, int64_t ldm, int lower_op,
+                                  float alpha) {
+  const int64_t o = (int64_t)blockIdx.y * BLK;
+  const int c = blockIdx.x, r = threadIdx.x;
+  float v = 0.f;
+  if (lower_op) { if (r >= c) v = Dp[(o + r) + (o + c) * ldD]; }
+  else          { if (c >= r) v = Dp[(o + c) + (o + r) * ldD]; }
+  M[(o + r) + (o + c) * ldm] = alpha * v;
+}
+
+}  // namespace
+
+int launch_trsm_panel_diag(const float *Dp, int64_t ldD, float *M, int64_t ldm, int64_t R, bool lower_op,
+                           float alpha, cudaStream_t s) {
+  if (R % BLK) return -1;
+  panel_diag_kernel<<<dim3(BLK, (unsigned)(R / BLK)), BLK, 0, s>>>(Dp, ldD, M, ldm, lower_op ? 1 : 0, alpha);
+  note_launch();
+  return cudaGetLastError() == cudaSuccess ? 0 : -1;
+}
+
+// teams: one per 256 right-hand sides, at most num_sms / 4 (two CTA pairs each)
+static int64_t panel_teams(int64_t nrhs, int num_sms) {
+  return imin((nrhs + PN - 1) / PN, (int64_t)(num_sms / 4));
+}
+size_t trsm_panel_ws_bytes(int64_t nrhs, int num_sms) {
+  const int64_t t = panel_teams(nrhs, num_sms);
+  return (size_t)t * 4 * PART_FLOATS * sizeof(float) + (size_t)t * 2 * sizeof(uint32_t);
+}
+
+int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool right, int64_t R,
+                      int64_t nrhs, bool forward, int kc, void *ws, cudaStream_t s, int num_sms) {
+  if (R <= 0 || R % BLK || R / BLK > MAX_BLK || nrhs <= 0 || kc < 1 || !ws) return -1;
+  const int64_t nteams = panel_teams(nrhs, num_sms);
+  if (nteams < 1) return -1;
+  static PanelParams prm;
+  static std::mutex mu;
+  std::lock_guard<std::mutex> lk(mu);
+  memset(&prm, 0, sizeof(prm));
+  // M: left rk (Xa(r,k) = M[r + k ldm]) / right kr (Xa(r,k) = M[k + r ldm]);
+  // X: left kr (Xb(n,k) = X[k + n ldx]) / right rk (Xb(n,k) = X[n + k ldx])
+  prm.layA = right ? LAYOUT_K : LAYOUT_MN;
+  prm.layB = right ? LAYOUT_MN : LAYOUT_K;
+  bool ok = right ? tma_map_f32(&prm.mapA, M, R, R, ldm, BK, HA, false)
+                  : tma_map_f32(&prm.mapA, M, R, R, ldm, 32, BK, true);
+  ok = ok && (right ? tma_map_f32(&prm.mapB, X, nrhs, R, ldx, 32, BK, true)
+                    : tma_map_f32(&prm.mapB, X, R, nrhs, ldx, BK, HB, false));
+  if (!ok) return -4;
+  prm.X = X;
+  prm.ws = static_cast<float *>(ws);
+  prm.ctr = reinterpret_cast<uint32_t *>(static_cast<uint8_t *>(ws) + (size_t)nteams * 4 * PART_FLOATS * sizeof(float));
+  prm.ldx = ldx;
+  prm.R = R;
+  prm.nrhs = nrhs;
+  prm.nblk = (int32_t)(R / BLK);
+  prm.right = right ? 1 : 0;
+  prm.forward = forward ? 1 : 0;
+  prm.kc = kc;
+  prm.nslab = (int32_t)((nrhs + PN - 1) / PN);
+  prm.nteams = (int32_t)nteams;
+  // group split of every block: member 0 takes the newest group (it alone
+  // waits for the block just solved), the others go greedily to the member
+  // with less work so far (ties to the helper, whose partial runs ahead)
+  int64_t load[2] = {0, 0};
+  for (int i = 0; i < prm.nblk; ++i) {
+    ++load[0];
+    uint32_t hm = 0;
+    for (int g = 0; g < i; ++g) {
+      if (load[1] <= load[0]) { hm |= 1u << g; ++load[1]; }
+      else ++load[0];
+    }
+    prm.hmask[i] = i == 0 ? 0u : hm;
+  }
+  static const int dbg = [] { const char *e = getenv("BLAS3_DEBUG_PANEL"); return e ? atoi(e) : 0; }();
+  prm.dbg = dbg;
+  static std::atomic<bool> attr[64];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return -1;
+  if (!attr[dev].load(std::memory_order_acquire)) {
+    if (cudaFuncSetAttribute(trsm_panel_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM) !=
+        cudaSuccess)
+      return -1;
+    attr[dev].store(true, std::memory_order_release);
+  }
+  if (cudaMemsetAsync(prm.ctr, 0, (size_t)nteams * 2 * sizeof(uint32_t), s) != cudaSuccess) return -1;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(4 * nteams));
+  cfg.blockDim = dim3(NTHREADS);
+  cfg.dynamicSmemBytes = SMEM;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = 2;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  const cudaError_t e = cudaLaunchKernelEx(&cfg, trsm_panel_kernel, prm);
+  note_launch(0);
+  return (e == cudaSuccess && cudaGetLastError() == cudaSuccess) ? 0 : -1;
+}
+
+}  // namespace blas3

@@ -1312,6 +1312,14 @@ static bool make_map(CUtensorMap *m, const float *ptr, int64_t d0, int64_t d1, i
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// plain 2-D fp32 map (other kernels of the library): mn32 -> the MN-major
+// staging swizzle (SWIZZLE_128B_ATOM_32B), else the K-major one (SWIZZLE_128B)
+bool tma_map_f32(CUtensorMap *m, const float *ptr, int64_t d0, int64_t d1, int64_t ld, uint32_t box0,
+                 uint32_t box1, bool mn32) {
+  return make_map(m, ptr, d0, d1, ld, box0, box1,
+                  mn32 ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B, 1, 1, BatchStride{0, 0});
+}
+
 // maps for one operand with R rows, K columns, staged `rows` at a time
 template <class PRM>
 static bool op_maps(PRM &prm, int &slot, OpDesc &o, int64_t R, int64_t K, int rows,

@@ -209,4 +209,5 @@ def test_options_roundtrip_and_validation(lib):
     assert lib.get_option("tc_vec_store") == 1 and lib.get_option("tc_c_prefetch") == 1
     assert lib.get_option("max_sms") == 0
     assert lib.get_option("tc_c_async") == 0
-    assert len(lib.OPTIONS) == 25
+    assert lib.get_option("trsm_panel") == 1
+    assert len(lib.OPTIONS) == 26

@@ -54,6 +54,9 @@ T.diagonal().fill_(1.0)
 ts, k = 16384, 512
 As, Bs, Cs = mk(ts, k), mk(ts, k), mk(ts, ts)
 A2, B2, C2 = mk(2048, 2048), mk(2048, 2048), mk(2048, 2048)
+T4, X4, B4 = mk(4096, 4096), mk(4096, 4096), mk(4096, 4096)
+T4.mul_(1.0 / 4096)
+T4.diagonal().fill_(1.0)
 st = torch.cuda.current_stream().cuda_stream
 
 
@@ -66,6 +69,7 @@ def cases(lib):
     (pa, la), (pb, lb), (pc, lc), (px, lx), (pt, lt) = P(A), P(B), P(C), P(X), P(T)
     (pas, las), (pbs, lbs), (pcs, lcs) = P(As), P(Bs), P(Cs)
     (pa2, la2), (pb2, lb2), (pc2, lc2) = P(A2), P(B2), P(C2)
+    (pt4, lt4), (px4, lx4) = P(T4), P(X4)
     return {
         "sgemm": (lambda: call(lib, "blas3_sgemm", b"N", b"N", n, n, n, 1.5, pa, la, pb, lb, 0.5, pc, lc, st),
                   2.0 * n ** 3, 5, None),
@@ -79,6 +83,8 @@ def cases(lib):
                   1.0 * n ** 3, 5, lambda: X.copy_(B)),
         "strsm": (lambda: call(lib, "blas3_strsm", b"L", b"L", b"N", b"N", n, n, 1.0, pt, lt, px, lx, st),
                   1.0 * n ** 3, 5, lambda: X.copy_(B)),
+        "strsm4096": (lambda: call(lib, "blas3_strsm", b"L", b"L", b"N", b"N", 4096, 4096, 1.0, pt4, lt4, px4, lx4,
+                                   st), 1.0 * 4096 ** 3, 10, lambda: X4.copy_(B4)),
         "ts_syrk": (lambda: call(lib, "blas3_ssyrk", b"L", b"N", ts, k, 1.5, pas, las, 0.5, pcs, lcs, st),
                     1.0 * k * ts * (ts + 1), 10, None),
         "ts_syr2k": (lambda: call(lib, "blas3_ssyr2k", b"L", b"N", ts, k, 1.5, pas, las, pbs, lbs, 0.5, pcs, lcs,
