@@ -1062,9 +1062,39 @@ static int strsm_first_panel(const TrsmGeom &g, int64_t pfirst, float *Mw, void 
   int rc;
   std::vector<LevelProblem> lv;
   trsm_doubling_problems(Ap, g.lda, R, g.lower, Dp, g.Tw, lv);
-  for (const LevelProblem &q : lv)
-    if (q.lvl == 0 && (rc = run_problem(q.P, s, sms))) return rc;
-  if (nb > 1 && (rc = run_problem(P, s, sms))) return rc;
+  // level 0 (step 1, step 2) and the couplings as ONE fused launch (three
+  // dependent phases, no launch gaps); one launch each if not fusable
+  std::vector<FusedPhase> ph;
+  uint32_t prev = 0;
+  for (int step = 1; step <= 2; ++step) {
+    uint32_t cur = 0;
+    for (const LevelProblem &q : lv)
+      if (q.lvl == 0 && q.step == step) {
+        FusedPhase f;
+        f.P = q.P; f.dep_full = (int32_t)prev; f.dep_slab = 0; f.slab_m = 0;
+        cur |= 1u << ph.size();
+        ph.push_back(f);
+      }
+    prev = cur;
+  }
+  if (nb > 1) {
+    FusedPhase f;
+    f.P = P; f.dep_full = (int32_t)prev; f.dep_slab = 0; f.slab_m = 0;
+    ph.push_back(f);
+  }
+  bool fused = false;
+  if (tensor_mode() && math_mode() == BLAS3_MATH_3XTF32 && !ph.empty()) {
+    bool elig = true;
+    for (const FusedPhase &f : ph) elig = elig && tc_eligible(f.P);
+    if (elig) {
+      rc = launch_tc_fused(ph.data(), (int)ph.size(), s, sms);
+      if (rc == -4) return BLAS3_ERR_TMA;
+      fused = rc == 0;
+    }
+  }
+  if (!fused)
+    for (const FusedPhase &f : ph)
+      if ((rc = run_problem(f.P, s, sms))) return rc;
   if (launch_trsm_panel_diag(Dp, NBO, Mw, ldm, R, g.lower_op, g.alpha, s)) return BLAS3_ERR_CUDA;
   float *X = g.left ? g.B + p0 : g.B + p0 * g.ldb;
   rc = launch_trsm_panel(Mw, ldm, X, g.ldb, !g.left, R, g.other, g.forward, (int)opt(BLAS3_OPT_TC_KC), pws, s,
@@ -1142,7 +1172,11 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // BLAS3_OPT_TRSM_PANEL: the first panel by the diagonal-panel solver (its
   // M workspace after W); the geometric chain's Y/M are then not needed
   const int64_t r_first = imin(NBO, nt - pfirst * NBO);
-  const bool use_panel = opt(BLAS3_OPT_TRSM_PANEL) != 0 && tensor_mode() && r_first % 256 == 0;
+  // (only when its teams of two CTA pairs fill most of the machine: with fewer
+  // right-hand sides the panel-inverse chain is cheaper, STRSM N = 4096 608 vs
+  // 581 us, profiles/r02_strsm_panel.md)
+  const bool use_panel = opt(BLAS3_OPT_TRSM_PANEL) != 0 && tensor_mode() && r_first % 256 == 0 &&
+                         4 * cdiv(other, 256) >= (int64_t)sms * 4 / 5;
   Scratch Mw;
   const size_t m_bytes = (size_t)r_first * r_first * sizeof(float);
   if (use_panel &&

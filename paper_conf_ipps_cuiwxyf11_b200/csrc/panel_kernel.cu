@@ -11,11 +11,12 @@
 // precomputed from A alone, block i of the solution is ONE sum of i + 1
 // "groups" of K = 256:
 //     X_i = M(i, i) B_i  +  sum_{j<i} M(i, j) X_j        (group 0, groups j + 1)
-// The team splits the groups of every block between its two pairs (host-side
-// greedy balance, hmask): member 0 always takes the newest group (j = i - 1,
-// the only one that waits for the block just solved), sums its partial with
-// the helper's (member 1, fp32 partial through L2) and stores X_i in place
-// over B_i; the helper's groups are older, so its partial runs ahead.  A pair
+// The team (2-4 CTA pairs, as many as the machine holds) splits the groups of
+// every block between its members (host-side greedy balance, gmask): member 0
+// always takes the newest group (j = i - 1, the only one that waits for the
+// block just solved), sums its partial with the helpers' (members 1.., fp32
+// partials through L2) and stores X_i in place over B_i; the helpers' groups
+// are older, so their partials run ahead.  A pair
 // computes 256 x 256 tiles, the tcgen05 shape at which the 3xTF32 UMMAs run
 // at full rate (a 128-wide N takes as long per instruction as 256).
 //
@@ -32,6 +33,7 @@
 #include <cstring>
 #include <mutex>
 #include <stdlib.h>
+#include <cstdio>
 
 #include "../../include/blas3.h"
 #include "kernels.h"
@@ -49,6 +51,7 @@ constexpr int HB = PN / 2;                 // right-hand sides staged per CTA
 constexpr int RS = 4, LS = 2;              // raw / lo stages
 constexpr int NACC = 2;                    // TMEM partials (2 x 256 columns)
 constexpr int MAX_BLK = 32;                // blocks per panel (R <= 8192)
+constexpr int MAX_MEM = 4;                 // CTA pairs per team
 constexpr int WARP_TMA = 0, WARP_MMA = 1, WARP_TR0 = 4, NUM_TR_WARPS = 8;
 constexpr int WARP_EPI0 = WARP_TR0 + NUM_TR_WARPS, NUM_EPI_WARPS = 8;
 constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;       // 640
@@ -73,12 +76,14 @@ struct PanelParams {
   CUtensorMap mapA;                        // M: rk (left) / kr (right) view
   CUtensorMap mapB;                        // X over B: kr (left) / rk (right) view
   float *X;                                // panel origin: left X(k,n) = X[k + n ldx], right X[n + k ldx]
-  float *ws;                               // helper partials: [team][slot 2][rank 2][col 256][row 128]
-  uint32_t *ctr;                           // [team][2]: X blocks stored, partials written (x2 CTAs)
+  float *ws;                               // helper partials: [team][helper][slot 2][rank 2][col 256][row 128]
+  uint32_t *ctr;                           // [team][MAX_MEM]: X blocks stored, then each helper's
+                                           // partials written (x2 CTAs each)
   int64_t ldx, R, nrhs;
-  int32_t nblk, layA, layB, right, forward, kc, nslab, nteams;
+  int32_t nblk, layA, layB, right, forward, kc, nslab, nteams, nmem;
   int32_t dbg;                             // BLAS3_DEBUG_PANEL knock-outs (timing experiments only)
-  uint32_t hmask[MAX_BLK];                 // groups of block i summed by the helper (member 1)
+  unsigned long long *trace;               // BLAS3_TRACE_PANEL: per-block stage times of team 0 (diagnostics)
+  uint32_t gmask[MAX_BLK][MAX_MEM];        // groups of block i summed by member h
 };
 
 // first row of processing block i
@@ -87,10 +92,7 @@ __device__ __forceinline__ int64_t blk_row(const PanelParams &p, int i) {
 }
 // groups of block i summed by member h (bit g: group g; g = 0 the block's own
 // right-hand side, g >= 1 the solved block g - 1)
-__device__ __forceinline__ uint32_t groups_of(const PanelParams &p, int i, int h) {
-  const uint32_t all = i >= 31 ? 0xFFFFFFFFu : ((2u << i) - 1u);
-  return h ? p.hmask[i] : (all & ~p.hmask[i]);
-}
+__device__ __forceinline__ uint32_t groups_of(const PanelParams &p, int i, int h) { return p.gmask[i][h]; }
 
 __device__ __forceinline__ uint64_t op_desc(uint32_t base, int lay, int k8) {
   if (lay == LAYOUT_MN) return ptx::smem_desc(base + k8 * 1024, BK * 128, 512, 1);
@@ -145,6 +147,15 @@ __device__ __forceinline__ void wait_count(const uint32_t *ctr, uint32_t target)
   }
 }
 
+// diagnostics: %globaltimer of stage st of block i, team 0, CTA rank 0 of member h
+__device__ __forceinline__ void ptrace(const PanelParams &p, int h, int i, int st) {
+  if (p.trace != nullptr && blockIdx.x == 2 * h && h < 2 && i < MAX_BLK) {
+    unsigned long long v;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(v));
+    p.trace[(h * MAX_BLK + i) * 4 + st] = v;
+  }
+}
+
 __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_constant__ PanelParams prm) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
@@ -154,9 +165,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const uint32_t rank = ptx::cluster_ctarank();
   const int pair = blockIdx.x / 2;
-  const int team = pair / 2, h = pair % 2;           // team member: 0 stores X, 1 helps
+  const int team = pair / prm.nmem, h = pair % prm.nmem;   // team member: 0 stores X, others help
   const int nblk = prm.nblk;
-  uint32_t *ctr_x = prm.ctr + 2 * team, *ctr_p = ctr_x + 1;
+  uint32_t *ctr_x = prm.ctr + MAX_MEM * team;              // then ctr_x[m]: helper m's partials
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < RS; ++s) { ptx::mbar_init(&bars->full[s], 1); ptx::mbar_init(&bars->empty[s], 1); }
@@ -227,6 +238,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
             const int rs = it % RS, ls = it % LS;
             ptx::mbar_wait_cluster(&bars->ready[ls], (it / LS) & 1);
             ptx::tc_fence_after();
+            if (lane == 0 && t == 0) ptrace(prm, h, i, 0);
+            if (lane == 0 && t == nkb - KB_BLK) ptrace(prm, h, i, 1);
             if (lane == 0) {
               const uint32_t d = tmem + buf * PN;
               const uint32_t hiA = ptx::smem_u32(raw[rs].A), hiB = ptx::smem_u32(raw[rs].B);
@@ -291,10 +304,28 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
       for (int i = 0; i < nblk; ++i, ++gblk) {
         const int nkb = KB_BLK * __popc(groups_of(prm, i, h));
         const int nch = nkb > 0 ? (nkb + prm.kc - 1) / prm.kc : 0;
+        // this CTA's partial slot: [col][row] so a warp's accesses per column are one 128-B line
+        // helper m's slot for this block: [col][row] (a warp's accesses per column are one 128-B line)
+        auto slot = [&](int m) {
+          return prm.ws + (((((size_t)team * (MAX_MEM - 1) + (m - 1)) * 2 + (gblk & 1)) * 2 + rank) * PART_FLOATS) +
+                 (size_t)(half * NCOL) * HA + rloc;
+        };
         float S[NCOL];
 #pragma unroll
         for (int j = 0; j < NCOL; ++j) S[j] = 0.f;
+        // member 0 adds the helper's partial (which runs ahead) while its MMA
+        // works on the newest group: before waiting for that group's first chunk
+        const int cpart = h == 0 ? (nkb - KB_BLK) / prm.kc : -1;
         for (int c = 0; c < nch; ++c, ++cc) {
+          if (c == cpart) {
+            for (int m = 1; m < prm.nmem; ++m) {
+              if (lead) wait_count(ctr_x + m, 2 * (gblk + 1));
+              ptx::named_bar_sync(5, EPI_THREADS);
+              const float *part = slot(m);
+#pragma unroll
+              for (int j = 0; j < NCOL; ++j) S[j] += __ldcg(part + (size_t)j * HA);
+            }
+          }
           const uint32_t buf = cc % NACC;
           ptx::mbar_wait(&bars->tfull[buf], (cc / NACC) & 1);
           ptx::tc_fence_after();
@@ -313,24 +344,19 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
           ptx::tc_fence_before();
           arrive_leader(&bars->tempty[buf], rank, 3, EPI_THREADS, lead);
         }
-        // this CTA's partial slot: [col][row] so a warp's accesses per column are one 128-B line
-        float *part = prm.ws + ((((size_t)team * 2 + (gblk & 1)) * 2 + rank) * PART_FLOATS) +
-                      (size_t)(half * NCOL) * HA + rloc;
-        if (h == 1) {
+        if (lead) ptrace(prm, h, i, 2);
+        if (h > 0) {
           // helper: the slot was last read for block gblk - 2 (X of it stored)
           if (lead && gblk >= 2) wait_count(ctr_x, 2 * (gblk - 1));
           ptx::named_bar_sync(5, EPI_THREADS);
+          float *part = slot(h);
 #pragma unroll
           for (int j = 0; j < NCOL; ++j) __stcg(part + (size_t)j * HA, S[j]);
           ptx::named_bar_sync(5, EPI_THREADS);
-          if (lead) { __threadfence(); atomicAdd(ctr_p, 1u); }
+          if (lead) { __threadfence(); atomicAdd(ctr_x + h, 1u); ptrace(prm, h, i, 3); }
           continue;
         }
-        // member 0: + the helper's partial, then X_i
-        if (lead) wait_count(ctr_p, 2 * (gblk + 1));
-        ptx::named_bar_sync(5, EPI_THREADS);
-#pragma unroll
-        for (int j = 0; j < NCOL; ++j) S[j] += __ldcg(part + (size_t)j * HA);
+        // member 0: X_i
         // X_i rows [blk_row + 128 rank, +128) x right-hand sides [c0, c0 + 128)
         const int64_t row = blk_row(prm, i) + HA * rank + rloc;
         const int64_t nval = prm.nrhs - c0;                  // valid columns (warp-uniform)
@@ -355,7 +381,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
           }
         }
         ptx::named_bar_sync(5, EPI_THREADS);
-        if (lead) { __threadfence(); atomicAdd(ctr_x, 1u); }
+        if (lead) { __threadfence(); atomicAdd(ctr_x, 1u); ptrace(prm, h, i, 3); }
       }
     }
   }
@@ -393,19 +419,40 @@ int launch_trsm_panel_diag(const float *Dp, int64_t ldD, float *M, int64_t ldm, 
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
 
-// teams: one per 256 right-hand sides, at most num_sms / 4 (two CTA pairs each)
-static int64_t panel_teams(int64_t nrhs, int num_sms) {
-  return imin((nrhs + PN - 1) / PN, (int64_t)(num_sms / 4));
+// member 0's serial hand-off per block in tenths of a group (BLAS3_PANEL_HANDOFF, experiments)
+static int64_t prm_handoff() {
+  static const int64_t v = [] { const char *e = getenv("BLAS3_PANEL_HANDOFF"); return e ? atoll(e) : 6; }();
+  return v;
+}
+// members per team at most (BLAS3_PANEL_MEMBERS, 1..MAX_MEM; default 2: a
+// third and fourth pair did not shorten the solve -- member 0's per-block
+// chain of newest group, store and reload bounds it -- and take SMs from the
+// concurrent panel-inverse doubling, STRSM N = 4096 643 vs 623 us)
+static int panel_members() {
+  static const int v = [] { const char *e = getenv("BLAS3_PANEL_MEMBERS"); const int m = e ? atoi(e) : 2;
+                            return m < 1 ? 1 : (m > MAX_MEM ? MAX_MEM : m); }();
+  return v;
+}
+// teams: one per 256 right-hand sides (at most num_sms / 4); members: the
+// CTA pairs the machine holds per team, up to panel_members()
+static void panel_shape(int64_t nrhs, int num_sms, int64_t &teams, int &nmem) {
+  const int64_t nslab = (nrhs + PN - 1) / PN, pairs = num_sms / 2;
+  teams = imin(nslab, imax(1, pairs / 2));
+  nmem = (int)imax(1, imin(panel_members(), pairs / teams));
 }
 size_t trsm_panel_ws_bytes(int64_t nrhs, int num_sms) {
-  const int64_t t = panel_teams(nrhs, num_sms);
-  return (size_t)t * 4 * PART_FLOATS * sizeof(float) + (size_t)t * 2 * sizeof(uint32_t);
+  int64_t t;
+  int m;
+  panel_shape(nrhs, num_sms, t, m);
+  return (size_t)t * (MAX_MEM - 1) * 4 * PART_FLOATS * sizeof(float) + (size_t)t * MAX_MEM * sizeof(uint32_t);
 }
 
 int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool right, int64_t R,
                       int64_t nrhs, bool forward, int kc, void *ws, cudaStream_t s, int num_sms) {
   if (R <= 0 || R % BLK || R / BLK > MAX_BLK || nrhs <= 0 || kc < 1 || !ws) return -1;
-  const int64_t nteams = panel_teams(nrhs, num_sms);
+  int64_t nteams;
+  int nmem;
+  panel_shape(nrhs, num_sms, nteams, nmem);
   if (nteams < 1) return -1;
   static PanelParams prm;
   static std::mutex mu;
@@ -422,7 +469,8 @@ int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool r
   if (!ok) return -4;
   prm.X = X;
   prm.ws = static_cast<float *>(ws);
-  prm.ctr = reinterpret_cast<uint32_t *>(static_cast<uint8_t *>(ws) + (size_t)nteams * 4 * PART_FLOATS * sizeof(float));
+  prm.ctr = reinterpret_cast<uint32_t *>(static_cast<uint8_t *>(ws) +
+                                         (size_t)nteams * (MAX_MEM - 1) * 4 * PART_FLOATS * sizeof(float));
   prm.ldx = ldx;
   prm.R = R;
   prm.nrhs = nrhs;
@@ -432,21 +480,37 @@ int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool r
   prm.kc = kc;
   prm.nslab = (int32_t)((nrhs + PN - 1) / PN);
   prm.nteams = (int32_t)nteams;
+  prm.nmem = nmem;
   // group split of every block: member 0 takes the newest group (it alone
-  // waits for the block just solved), the others go greedily to the member
-  // with less work so far (ties to the helper, whose partial runs ahead)
-  int64_t load[2] = {0, 0};
+  // waits for the block just solved), every other group goes to the member
+  // with the least work so far (ties to a helper, whose partial runs ahead).
+  // Member 0 is also charged its serial per-block hand-off (store, release,
+  // reload of X_i: about 0.6 of a group's MMA time, measured)
+  const int64_t grp = 10, handoff = prm_handoff();
+  int64_t load[MAX_MEM] = {0, 0, 0, 0};
   for (int i = 0; i < prm.nblk; ++i) {
-    ++load[0];
-    uint32_t hm = 0;
+    uint32_t gm[MAX_MEM] = {0, 0, 0, 0};
+    gm[0] = 1u << i;
+    load[0] += grp + handoff;
     for (int g = 0; g < i; ++g) {
-      if (load[1] <= load[0]) { hm |= 1u << g; ++load[1]; }
-      else ++load[0];
+      int best = 0;
+      for (int m = nmem - 1; m >= 0; --m)
+        if (load[m] < load[best]) best = m;
+      if (nmem > 1 && best == 0 && load[nmem - 1] == load[0]) best = nmem - 1;
+      gm[best] |= 1u << g;
+      load[best] += grp;
     }
-    prm.hmask[i] = i == 0 ? 0u : hm;
+    for (int m = 0; m < MAX_MEM; ++m) prm.gmask[i][m] = gm[m];
   }
   static const int dbg = [] { const char *e = getenv("BLAS3_DEBUG_PANEL"); return e ? atoi(e) : 0; }();
   prm.dbg = dbg;
+  static const bool trace = getenv("BLAS3_TRACE_PANEL") != nullptr;
+  static unsigned long long *tbuf = nullptr;
+  if (trace) {
+    if (!tbuf && cudaMalloc(&tbuf, 2 * MAX_BLK * 4 * sizeof(unsigned long long)) != cudaSuccess) return -1;
+    cudaMemsetAsync(tbuf, 0, 2 * MAX_BLK * 4 * sizeof(unsigned long long), s);
+    prm.trace = tbuf;
+  }
   static std::atomic<bool> attr[64];
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return -1;
@@ -456,9 +520,9 @@ int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool r
       return -1;
     attr[dev].store(true, std::memory_order_release);
   }
-  if (cudaMemsetAsync(prm.ctr, 0, (size_t)nteams * 2 * sizeof(uint32_t), s) != cudaSuccess) return -1;
+  if (cudaMemsetAsync(prm.ctr, 0, (size_t)nteams * MAX_MEM * sizeof(uint32_t), s) != cudaSuccess) return -1;
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)(4 * nteams));
+  cfg.gridDim = dim3((unsigned)(2 * nmem * nteams));
   cfg.blockDim = dim3(NTHREADS);
   cfg.dynamicSmemBytes = SMEM;
   cfg.stream = s;
@@ -471,6 +535,21 @@ int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool r
   cfg.numAttrs = 1;
   const cudaError_t e = cudaLaunchKernelEx(&cfg, trsm_panel_kernel, prm);
   note_launch(0);
+  if (trace && e == cudaSuccess) {            // member, block: mma start / newest group / drained / released (us)
+    unsigned long long hb[2 * MAX_BLK * 4];
+    cudaStreamSynchronize(s);
+    cudaMemcpy(hb, tbuf, sizeof(hb), cudaMemcpyDeviceToHost);
+    unsigned long long t0 = ~0ull;
+    for (int k = 0; k < 2 * MAX_BLK * 4; ++k) if (hb[k] && hb[k] < t0) t0 = hb[k];
+    for (int hh = 0; hh < 2; ++hh)
+      for (int i = 0; i < prm.nblk && hh < nmem; ++i) {
+        const unsigned long long *r = hb + (hh * MAX_BLK + i) * 4;
+        auto us = [&](unsigned long long v) { return v ? (double)(v - t0) / 1e3 : -1.0; };
+        fprintf(stderr, "[panel] m%d blk %2d groups %2d: mma %7.2f newest %7.2f drained %7.2f released %7.2f\n", hh, i,
+                __builtin_popcount(prm.gmask[i][hh]), us(r[0]), us(r[1]),
+                us(r[2]), us(r[3]));
+      }
+  }
   return (e == cudaSuccess && cudaGetLastError() == cudaSuccess) ? 0 : -1;
 }
 
