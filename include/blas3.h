@@ -274,9 +274,11 @@ int blas3_get_math_mode(void);
  *                          128 right-hand sides forward-substitutes the whole
  *                          panel (256-row blocks, precomputed couplings
  *                          -inv(op(A)_ss) op(A)_sf), no grid-wide dependency
- *                          steps; 0: the fused doubling + geometric chain.  Used
- *                          when the panel's order is a multiple of 256 and B is
- *                          16-B aligned with ldb % 4 == 0
+ *                          steps; 0: the fused doubling + geometric chain; 2: the
+ *                          solver even when its teams (two CTA pairs per 256
+ *                          right-hand sides) do not fill most of the SMs (1 uses
+ *                          it only then).  Used when the panel's order is a
+ *                          multiple of 256 and B is 16-B aligned with ldb % 4 == 0
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */
@@ -309,9 +311,10 @@ int64_t blas3_launch_count(void);
 
 /* Same counter split by route: BLAS3_PATH_TCGEN05 (tcgen05 tensor-core
  * structured GEMM, any tensor math mode), BLAS3_PATH_SIMT (FP32 SIMT structured GEMM),
- * BLAS3_PATH_AUX (scale / copy / TRSM diagonal-inverse kernels).  Returns -1
+ * BLAS3_PATH_AUX (scale / copy / TRSM diagonal-inverse kernels),
+ * BLAS3_PATH_TRSM_PANEL (the STRSM diagonal-panel solver, tcgen05).  Returns -1
  * for an unknown path.  Lets tests assert which route a call took. */
-enum { BLAS3_PATH_TCGEN05 = 0, BLAS3_PATH_SIMT = 1, BLAS3_PATH_AUX = 2 };
+enum { BLAS3_PATH_TCGEN05 = 0, BLAS3_PATH_SIMT = 1, BLAS3_PATH_AUX = 2, BLAS3_PATH_TRSM_PANEL = 3 };
 int64_t blas3_launch_count_by_path(int path);
 
 /* Static string for a return code. */

@@ -244,7 +244,7 @@ def get_math_mode():
     return blas3_get_math_mode()  # noqa: F821
 
 
-PATH_TCGEN05, PATH_SIMT, PATH_AUX = 0, 1, 2
+PATH_TCGEN05, PATH_SIMT, PATH_AUX, PATH_TRSM_PANEL = 0, 1, 2, 3
 
 # tuning options (include/blas3.h BLAS3_OPT_*): name -> key
 OPTIONS = {"gm_map": 0, "gm_min_gemm": 1, "gm_min_symm": 2, "gm_min_trmm": 3, "gm_min_trsm": 4,
@@ -286,11 +286,11 @@ class options:
 
 
 def launch_count(path=None):
-    """Kernels launched since load (all, or one route: 'tc', 'simt', 'aux')."""
+    """Kernels launched since load (all, or one route: 'tc', 'simt', 'aux', 'panel')."""
     if path is None:
         return int(blas3_launch_count())  # noqa: F821
     if isinstance(path, str):
-        path = {"tc": PATH_TCGEN05, "simt": PATH_SIMT, "aux": PATH_AUX}[path]
+        path = {"tc": PATH_TCGEN05, "simt": PATH_SIMT, "aux": PATH_AUX, "panel": PATH_TRSM_PANEL}[path]
     return int(blas3_launch_count_by_path(path))  # noqa: F821
 
 

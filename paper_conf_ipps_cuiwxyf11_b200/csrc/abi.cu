@@ -18,10 +18,10 @@
 namespace blas3 {
 
 static std::atomic<int64_t> g_launches{0};
-static std::atomic<int64_t> g_path_launches[3];
+static std::atomic<int64_t> g_path_launches[4];
 void note_launch(int path) {
   g_launches.fetch_add(1, std::memory_order_relaxed);
-  if (path >= 0 && path < 3) g_path_launches[path].fetch_add(1, std::memory_order_relaxed);
+  if (path >= 0 && path < 4) g_path_launches[path].fetch_add(1, std::memory_order_relaxed);
 }
 
 // ---- tuning options (include/blas3.h): defaults, environment names, ranges
@@ -52,7 +52,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_MAX_SMS", 0, 0, 4096, false},
     {"BLAS3_TC_C_PREFETCH", 1, 0, 1, false},
     {"BLAS3_TC_C_ASYNC", 0, 0, 1, false},
-    {"BLAS3_TRSM_PANEL", 1, 0, 1, false},
+    {"BLAS3_TRSM_PANEL", 1, 0, 2, false},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;
@@ -250,7 +250,7 @@ extern "C" {
 int blas3_version(void) { return 100; }
 int64_t blas3_launch_count(void) { return g_launches.load(); }
 int64_t blas3_launch_count_by_path(int path) {
-  return (path >= 0 && path < 3) ? g_path_launches[path].load() : -1;
+  return (path >= 0 && path < 4) ? g_path_launches[path].load() : -1;
 }
 
 int blas3_set_option(int key, int64_t value) {
@@ -1176,7 +1176,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // right-hand sides the panel-inverse chain is cheaper, STRSM N = 4096 608 vs
   // 581 us, profiles/r02_strsm_panel.md)
   const bool use_panel = opt(BLAS3_OPT_TRSM_PANEL) != 0 && tensor_mode() && r_first % 256 == 0 &&
-                         4 * cdiv(other, 256) >= (int64_t)sms * 4 / 5;
+                         (opt(BLAS3_OPT_TRSM_PANEL) == 2 || 4 * cdiv(other, 256) >= (int64_t)sms * 4 / 5);
   Scratch Mw;
   const size_t m_bytes = (size_t)r_first * r_first * sizeof(float);
   if (use_panel &&

@@ -8,7 +8,7 @@
 
 namespace blas3 {
 
-void note_launch(int path = 2);      // host-side launch counter (blas3_launch_count[_by_path])
+void note_launch(int path = 2);      // host-side launch counter (blas3_launch_count[_by_path]; 0..3)
 int64_t opt(int key);                // tuning option (blas3_set_option / environment)
 
 // Structured GEMM kernels (all routines canonicalise to a Problem).

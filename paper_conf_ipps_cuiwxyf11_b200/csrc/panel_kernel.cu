@@ -534,7 +534,7 @@ int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool r
   cfg.attrs = at;
   cfg.numAttrs = 1;
   const cudaError_t e = cudaLaunchKernelEx(&cfg, trsm_panel_kernel, prm);
-  note_launch(0);
+  note_launch(3);
   if (trace && e == cudaSuccess) {            // member, block: mma start / newest group / drained / released (us)
     unsigned long long hb[2 * MAX_BLK * 4];
     cudaStreamSynchronize(s);
