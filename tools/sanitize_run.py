@@ -1,7 +1,8 @@
 """Small-N workload for compute-sanitizer (memcheck / synccheck / initcheck):
 every routine, several variants, both math modes, ragged sizes, and the STRSM
 multi-panel sweep (256-wide panels via BLAS3_TRSM_NB, set by the caller) on both
-the multi-launch and the fused path, plus a split-k tail.  Prints one line.
+the multi-launch and the fused path, the STRSM diagonal-panel solver, plus a
+split-k tail.  Prints one line.
 
 BLAS3_TRSM_NB=256 compute-sanitizer --tool memcheck python tools/sanitize_run.py
 """
@@ -45,6 +46,16 @@ for mode in ("3xtf32", "simt", "tf32_bf16x"):
             b3.strsm("R", "U", "T", "N", 1.5, Tn, rnd(300, 900))
     calls += 12
 b3.set_math_mode("3xtf32")
+# the STRSM diagonal-panel solver (forced): forward / backward, both sides, a
+# ragged right-hand side, and a shrunken grid whose teams loop over slabs
+for opts in ({"trsm_panel": 2}, {"trsm_panel": 2, "max_sms": 16}):
+    with b3.options(**opts):
+        Tp = rnd(768, 768)
+        Tp.diagonal().add_(768.0)
+        b3.strsm("L", "L", "N", "N", 1.5, Tp, rnd(768, 600))
+        b3.strsm("L", "U", "N", "U", 1.5, Tp, rnd(768, 260))
+        b3.strsm("R", "L", "T", "N", 1.5, Tp, rnd(300, 768))
+        calls += 3
 with b3.options(gm_map=1):                                       # GM_map SSYMM beside the staged default
     b3.ssymm("L", "U", 1.5, rnd(300, 300), rnd(300, 260), 0.5, rnd(300, 260))
 # a captured graph (graph-private scheduler state / split workspace), replayed twice
