@@ -211,9 +211,11 @@ int blas3_get_math_mode(void);
  *                          this width: power of 2 in [128, 8192] (256)
  *   BLAS3_OPT_TRSM_FUSED   [BLAS3_TRSM_FUSED] 1: the whole STRSM (panel-inverse
  *                          doubling + sweep) as one persistent dependency-driven
- *                          launch when it fits; 0 (default): one launch per step
- *                          on the caller's and the side streams (measured equal
- *                          or faster on B200 at N = 8192)
+ *                          launch when it fits; 2: when the diagonal-panel solver
+ *                          took the first panel, the sweep over the other panels
+ *                          (with their last doubling level) as one such launch;
+ *                          0 (default): one launch per step on the caller's and
+ *                          the side streams
  *   BLAS3_OPT_TRSM_FIRST_YM [BLAS3_TRSM_FIRST_YM] 1 (default): the first panel's
  *                          blocks are solved as X_s = Y_s - M X_f with Y, M
  *                          precomputed off the critical path; 0: update + solve

@@ -41,7 +41,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TRSM_SLAB_MIN", 16384, 256, int64_t(1) << 40, false},
     {"BLAS3_TRSM_RESERVE", -1, -1, 74, false},
     {"BLAS3_TRSM_GEO_LEAF", 256, 128, 8192, true},
-    {"BLAS3_TRSM_FUSED", 0, 0, 1, false},
+    {"BLAS3_TRSM_FUSED", 0, 0, 2, false},
     {"BLAS3_TRSM_FIRST_YM", 1, 0, 1, false},
     {"BLAS3_TRSM_FIRST_FUSED", 1, 0, 1, false},
     {"BLAS3_TRSM_FIRST_SPLIT", 0, 0, 8192, true},
@@ -627,16 +627,19 @@ static void trsm_doubling_problems(const float *A, int64_t lda, int64_t nt, bool
 }
 // Runs the doubling on stream s, recording ev_lvl[l] once the inverses of
 // every aligned 2^(l+8)-block are complete.
+// Levels [from, to) only (to < 0: all).
 static int trsm_panel_doubling(const float *A, int64_t lda, int64_t nt, bool lower, float *D,
-                               float *Tw, cudaStream_t s, int sms, cudaEvent_t *ev_lvl) {
+                               float *Tw, cudaStream_t s, int sms, cudaEvent_t *ev_lvl, int from = 0,
+                               int to = -1) {
   std::vector<LevelProblem> probs;
   trsm_doubling_problems(A, lda, nt, lower, D, Tw, probs);
   size_t i = 0;
   int rc;
   for (int64_t sz = 128, lvl = 0; sz < trsm_nbo(); sz *= 2, ++lvl) {
+    if (to >= 0 && lvl >= to) break;
     for (; i < probs.size() && probs[i].lvl == lvl; ++i)
-      if ((rc = run_problem(probs[i].P, s, sms))) return rc;
-    if (cudaEventRecord(ev_lvl[lvl], s) != cudaSuccess) return BLAS3_ERR_CUDA;
+      if (lvl >= from && (rc = run_problem(probs[i].P, s, sms))) return rc;
+    if (lvl >= from && cudaEventRecord(ev_lvl[lvl], s) != cudaSuccess) return BLAS3_ERR_CUDA;
   }
   return 0;
 }
@@ -722,11 +725,21 @@ struct TrsmGeom {
   float *B; int64_t ldb;
   float *D, *Tw, *W;
 };
-static int strsm_fused(const TrsmGeom &g, cudaStream_t s, int sms) {
+// first_solved (BLAS3_OPT_TRSM_FUSED = 2): the first processed panel is
+// already solved (the diagonal-panel solver, earlier on the stream) and the
+// other panels' doubling levels below lvl_from are complete (side stream,
+// waited on by the caller): the launch holds the remaining levels of the
+// other panels -- claimed first -- and the sweep after the first panel.
+static int strsm_fused(const TrsmGeom &g, cudaStream_t s, int sms, bool first_solved = false,
+                       int lvl_from = 0) {
   const int64_t NBO = g.NBO, nt = g.nt;
   const int64_t ldw = g.left ? NBO : g.m;              // W(r, c) = W[r + c * ldw]
   std::vector<LevelProblem> lv;
-  trsm_doubling_problems(g.A, g.lda, nt, g.lower, g.D, g.Tw, lv);
+  if (!first_solved) trsm_doubling_problems(g.A, g.lda, nt, g.lower, g.D, g.Tw, lv);
+  else if (g.npanel > 1) {                             // the other panels only
+    const int64_t o = g.forward ? NBO : 0, len = g.forward ? nt - NBO : (g.npanel - 1) * NBO;
+    trsm_doubling_problems(g.A + o * (1 + g.lda), g.lda, len, g.lower, g.D + (o / NBO) * NBO * NBO, g.Tw, lv);
+  }
   int nlvl = 0;
   for (int64_t sz = 128; sz < NBO; sz *= 2) ++nlvl;
 
@@ -869,7 +882,7 @@ static int strsm_fused(const TrsmGeom &g, cudaStream_t s, int sms) {
     if (q1 - q0 == 1) {
       const int64_t p = g.forward ? q0 : g.npanel - 1 - q0;
       const int64_t p0 = p * NBO, pr = imin(NBO, nt - p0);
-      if (q0 == 0) geo(p0, NBO, scaled);
+      if (q0 == 0) { if (!first_solved) geo(p0, NBO, scaled); }
       else leaf(p0, pr, NBO, scaled, in_w);
       return;
     }
@@ -889,13 +902,17 @@ static int strsm_fused(const TrsmGeom &g, cudaStream_t s, int sms) {
     }
     rec(mid, q1, true, true);
   };
+  if (first_solved) {                                  // the remaining levels first, then the sweep
+    emitted_lvl = lvl_from - 1;
+    levels_upto(nlvl - 1);
+  }
   rec(0, g.npanel, false, false);
   flush_pending();
   if (!ok || ph.empty()) return 1;
   for (const FusedPhase &f : ph)
     if (!tc_eligible(f.P)) return 1;
   // 128-block inverses (the fused phases read them), then the one launch
-  if (launch_trsm_diag_inv(g.A, g.lda, nt, g.lower, g.unit, g.D, NBO, s)) return BLAS3_ERR_CUDA;
+  if (!first_solved && launch_trsm_diag_inv(g.A, g.lda, nt, g.lower, g.unit, g.D, NBO, s)) return BLAS3_ERR_CUDA;
   const int rc = launch_tc_fused(ph.data(), (int)ph.size(), s, sms);
   return rc == 0 ? 0 : (rc == -4 ? BLAS3_ERR_TMA : BLAS3_ERR_CUDA);
 }
@@ -1148,7 +1165,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   if ((rc = get_scratch(Tw, t_bytes, s, aop_bytes + d_bytes))) return rc;
   if ((rc = get_scratch(W, w_bytes, s, aop_bytes + d_bytes + t_bytes))) return rc;
 
-  if (opt(BLAS3_OPT_TRSM_FUSED) && tensor_mode()) {
+  if (opt(BLAS3_OPT_TRSM_FUSED) == 1 && tensor_mode()) {
     const TrsmGeom g{left, lower, ta, unit, lower_op, forward, m, n, nt, NBO, npanel, other, alpha,
                      A, lda, B, ldb, D.p, Tw.p, W.p};
     rc = strsm_fused(g, s, sms);
@@ -1296,11 +1313,28 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // microseconds per launch, and the first panel is the critical path (the
   // fused chain started ~125 us late at N = 8192 when these ~8 launches were
   // enqueued before it; profiles/r02_strsm_timeline.md)
+  // BLAS3_OPT_TRSM_FUSED = 2 (after the panel solver): the sweep over the
+  // other panels as ONE fused launch, holding the last doubling level of
+  // those panels (the side stream builds the levels below it)
+  const bool fused_sweep = panel_done && opt(BLAS3_OPT_TRSM_FUSED) == 2 && npanel > 1 && nlvl >= 2 &&
+                           math_mode() == BLAS3_MATH_3XTF32;
+  const int64_t prest = forward ? 1 : 0, orest = prest * NBO;
+  const int64_t nrest = imin(nt, (prest + npanel - 1) * NBO) - orest;
   if (npanel > 1 && !all_done) {
-    const int64_t prest = forward ? 1 : 0, o = prest * NBO;
     if (cudaStreamWaitEvent(ts->side2, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
-    if ((rc = trsm_panel_doubling(A + o * (1 + lda), lda, imin(nt, (prest + npanel - 1) * NBO) - o, lower,
-                                  D.p + prest * NBO * NBO, Tw.p, ts->side2, sms, ts->ev_lvl2)))
+    if ((rc = trsm_panel_doubling(A + orest * (1 + lda), lda, nrest, lower, D.p + prest * NBO * NBO, Tw.p,
+                                  ts->side2, sms, ts->ev_lvl2, 0, fused_sweep ? nlvl - 1 : -1)))
+      return rc;
+  }
+  if (fused_sweep) {
+    if (cudaStreamWaitEvent(s, ts->ev_lvl2[nlvl - 2], 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+    const TrsmGeom g{left, lower, ta, unit, lower_op, forward, m, n, nt, NBO, npanel, other, alpha,
+                     A, lda, B, ldb, D.p, Tw.p, W.p};
+    rc = strsm_fused(g, s, sms, true, nlvl - 1);
+    if (rc <= 0) return finish(rc);
+    // not fusable: the last level on the side stream, then the multi-launch sweep
+    if ((rc = trsm_panel_doubling(A + orest * (1 + lda), lda, nrest, lower, D.p + prest * NBO * NBO, Tw.p,
+                                  ts->side2, sms, ts->ev_lvl2, nlvl - 1, -1)))
       return rc;
   }
   if (cudaEventRecord(ts->ev_fork2, s) != cudaSuccess) return BLAS3_ERR_CUDA;
