@@ -1077,41 +1077,10 @@ static int strsm_first_panel(const TrsmGeom &g, int64_t pfirst, float *Mw, void 
   P.per = nb;
   if (nb > 1 && !tc_eligible(P)) return 1;
   int rc;
-  std::vector<LevelProblem> lv;
-  trsm_doubling_problems(Ap, g.lda, R, g.lower, Dp, g.Tw, lv);
-  // level 0 (step 1, step 2) and the couplings as ONE fused launch (three
-  // dependent phases, no launch gaps); one launch each if not fusable
-  std::vector<FusedPhase> ph;
-  uint32_t prev = 0;
-  for (int step = 1; step <= 2; ++step) {
-    uint32_t cur = 0;
-    for (const LevelProblem &q : lv)
-      if (q.lvl == 0 && q.step == step) {
-        FusedPhase f;
-        f.P = q.P; f.dep_full = (int32_t)prev; f.dep_slab = 0; f.slab_m = 0;
-        cur |= 1u << ph.size();
-        ph.push_back(f);
-      }
-    prev = cur;
-  }
-  if (nb > 1) {
-    FusedPhase f;
-    f.P = P; f.dep_full = (int32_t)prev; f.dep_slab = 0; f.slab_m = 0;
-    ph.push_back(f);
-  }
-  bool fused = false;
-  if (tensor_mode() && math_mode() == BLAS3_MATH_3XTF32 && !ph.empty()) {
-    bool elig = true;
-    for (const FusedPhase &f : ph) elig = elig && tc_eligible(f.P);
-    if (elig) {
-      rc = launch_tc_fused(ph.data(), (int)ph.size(), s, sms);
-      if (rc == -4) return BLAS3_ERR_TMA;
-      fused = rc == 0;
-    }
-  }
-  if (!fused)
-    for (const FusedPhase &f : ph)
-      if ((rc = run_problem(f.P, s, sms))) return rc;
+  // level 0 of the panel's doubling (its 256-block inverses) on CUDA cores,
+  // one launch, then the couplings
+  if (launch_trsm_level0(Ap, g.lda, R, g.lower, Dp, NBO, s)) return BLAS3_ERR_CUDA;
+  if (nb > 1 && (rc = run_problem(P, s, sms))) return rc;
   if (launch_trsm_panel_diag(Dp, NBO, Mw, ldm, R, g.lower_op, g.alpha, s)) return BLAS3_ERR_CUDA;
   float *X = g.left ? g.B + p0 : g.B + p0 * g.ldb;
   rc = launch_trsm_panel(Mw, ldm, X, g.ldb, !g.left, R, g.other, g.forward, (int)opt(BLAS3_OPT_TC_KC), pws, s,
@@ -1322,8 +1291,14 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   const int64_t nrest = imin(nt, (prest + npanel - 1) * NBO) - orest;
   if (npanel > 1 && !all_done) {
     if (cudaStreamWaitEvent(ts->side2, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+    // (beside the panel solver, level 0 on CUDA cores in one launch, as for the first panel)
+    const int from = panel_done && nlvl >= 1 ? 1 : 0;
+    if (from == 1 && (launch_trsm_level0(A + orest * (1 + lda), lda, nrest, lower, D.p + prest * NBO * NBO, NBO,
+                                         ts->side2) ||
+                      cudaEventRecord(ts->ev_lvl2[0], ts->side2) != cudaSuccess))
+      return BLAS3_ERR_CUDA;
     if ((rc = trsm_panel_doubling(A + orest * (1 + lda), lda, nrest, lower, D.p + prest * NBO * NBO, Tw.p,
-                                  ts->side2, sms, ts->ev_lvl2, 0, fused_sweep ? nlvl - 1 : -1)))
+                                  ts->side2, sms, ts->ev_lvl2, from, fused_sweep ? nlvl - 1 : -1)))
       return rc;
   }
   if (fused_sweep) {

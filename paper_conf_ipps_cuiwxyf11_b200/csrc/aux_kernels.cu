@@ -378,6 +378,116 @@ trsm_diag_inv_kernel(const float *A, int64_t lda, int64_t n, int stored_lower, i
   }
 }
 
+// Level 0 of the panel-inverse doubling on CUDA cores (exact fp32 FMAs): for
+// every pair [[L11, 0], [L21, L22]] of 128-blocks of L (rows [256p, 256p + 256)),
+// the off-diagonal block of its inverse,
+//     X21 = -inv(L22) (L21 inv(L11)),
+// written into the panel-inverse workspace beside inv(L11) and inv(L22)
+// (trsm_diag_inv_kernel, which must have run).  Columns of X21 are
+// independent: grid (pairs, 128 / L0C), one CTA per L0C columns.  A ragged last
+// pair (L22 of nr2 < 128 rows) reads zeros beyond n and writes zero rows there.
+// It replaces two dependent tcgen05 launches of 128-blocks (the first level of
+// trsm_doubling_problems) with one launch (profiles/r02_strsm_panel.md).
+namespace {
+constexpr int L0C = 8;             // columns of X21 per CTA
+constexpr int L0R = DNB * L0C / DT; // rows of X21 per thread (4)
+constexpr int L0S = DNB + 4;       // smem row stride (16-B aligned rows)
+}
+__global__ void __launch_bounds__(DT)
+trsm_level0_kernel(const float *A, int64_t lda, int64_t n, int stored_lower, float *Dinv, int64_t ldD) {
+  extern __shared__ __align__(16) float sm[];
+  float *Lr = sm;                          // [128][L0S] row-major: L21, then inv(L22)
+  float *Xc = sm + DNB * L0S;              // [128][L0C + 1]: inv(L11)(:, cols), then T(:, cols)
+  const int tid = threadIdx.x;
+  const int64_t o = (int64_t)blockIdx.x * 2 * DNB;
+  const int cs = blockIdx.y * L0C;
+  const int nr2 = (int)imin(DNB, n - o - DNB);
+  const int64_t bpp = ldD / DNB, b1 = o / DNB;          // 128-blocks per panel; block of L11
+  float *D11 = Dinv + (b1 / bpp) * ldD * ldD + (b1 % bpp) * DNB * (1 + ldD);
+  const float *D22 = D11 + DNB * (1 + ldD);             // a pair never straddles a panel (ldD >= 256)
+  float *D21 = D11 + DNB;
+  // the loads are latency-bound: 16 independent ones in flight per thread
+  constexpr int LB = 16;
+  for (int e0 = tid; e0 < DNB * DNB; e0 += DT * LB) {   // L21(r, c) = L(o + 128 + r, o + c)
+    float v[LB];
+#pragma unroll
+    for (int u = 0; u < LB; ++u) {
+      const int e = e0 + u * DT, r = e % DNB, c = e / DNB;
+      v[u] = r < nr2 ? (stored_lower ? __ldg(A + (o + DNB + r) + (o + c) * lda)
+                                     : __ldg(A + (o + c) + (o + DNB + r) * lda)) : 0.f;
+    }
+#pragma unroll
+    for (int u = 0; u < LB; ++u) { const int e = e0 + u * DT; Lr[(e % DNB) * L0S + e / DNB] = v[u]; }
+  }
+  {
+    float v[DNB * L0C / DT];
+#pragma unroll
+    for (int u = 0; u < DNB * L0C / DT; ++u) {
+      const int e = tid + u * DT, k = e % DNB, c = e / DNB;
+      v[u] = __ldg(D11 + k + (int64_t)(cs + c) * ldD);
+    }
+#pragma unroll
+    for (int u = 0; u < DNB * L0C / DT; ++u) { const int e = tid + u * DT; Xc[(e % DNB) * (L0C + 1) + e / DNB] = v[u]; }
+  }
+  __syncthreads();
+  const int c = tid % L0C, rg = tid / L0C;              // thread: rows rg*L0R .. +L0R-1 of column c
+  // rows of (Lr x Xc)(:, c); Lr rows read as float4
+  auto rows_times = [&](float (&t)[L0R]) {
+#pragma unroll
+    for (int i = 0; i < L0R; ++i) t[i] = 0.f;
+    for (int k = 0; k < DNB; k += 4) {
+      const float x0 = Xc[k * (L0C + 1) + c], x1 = Xc[(k + 1) * (L0C + 1) + c];
+      const float x2 = Xc[(k + 2) * (L0C + 1) + c], x3 = Xc[(k + 3) * (L0C + 1) + c];
+#pragma unroll
+      for (int i = 0; i < L0R; ++i) {
+        const float4 l = *reinterpret_cast<const float4 *>(&Lr[(rg * L0R + i) * L0S + k]);
+        t[i] = fmaf(l.x, x0, t[i]);
+        t[i] = fmaf(l.y, x1, t[i]);
+        t[i] = fmaf(l.z, x2, t[i]);
+        t[i] = fmaf(l.w, x3, t[i]);
+      }
+    }
+  };
+  float t[L0R];
+  rows_times(t);                                        // T = L21 inv(L11)
+  __syncthreads();
+#pragma unroll
+  for (int i = 0; i < L0R; ++i) Xc[(rg * L0R + i) * (L0C + 1) + c] = t[i];
+  for (int e0 = tid; e0 < DNB * DNB; e0 += DT * LB) {
+    float v[LB];
+#pragma unroll
+    for (int u = 0; u < LB; ++u) { const int e = e0 + u * DT; v[u] = __ldg(D22 + e % DNB + (int64_t)(e / DNB) * ldD); }
+#pragma unroll
+    for (int u = 0; u < LB; ++u) { const int e = e0 + u * DT; Lr[(e % DNB) * L0S + e / DNB] = v[u]; }
+  }
+  __syncthreads();
+  rows_times(t);                                        // inv(L22) T
+#pragma unroll
+  for (int i = 0; i < L0R; ++i) {
+    const int r = rg * L0R + i;
+    D21[r + (int64_t)(cs + c) * ldD] = r < nr2 ? -t[i] : 0.f;
+  }
+}
+
+int launch_trsm_level0(const float *A, int64_t lda, int64_t n, int stored_lower, float *Dinv, int64_t ldD,
+                       cudaStream_t s) {
+  if (ldD % (2 * DNB)) return -1;
+  const int64_t pairs = n > DNB ? (n - DNB + 2 * DNB - 1) / (2 * DNB) : 0;   // pairs with an L21
+  if (pairs == 0) return 0;
+  const size_t smem = (DNB * L0S + DNB * (L0C + 1)) * sizeof(float);
+  static std::atomic<bool> attr[64];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return -1;
+  if (!attr[dev].load(std::memory_order_acquire)) {
+    if (cudaFuncSetAttribute(trsm_level0_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+        cudaSuccess) return -1;
+    attr[dev].store(true, std::memory_order_release);
+  }
+  trsm_level0_kernel<<<dim3((unsigned)pairs, DNB / L0C), DT, smem, s>>>(A, lda, n, stored_lower, Dinv, ldD);
+  note_launch();
+  return cudaGetLastError() == cudaSuccess ? 0 : -1;
+}
+
 // blas3_signal: a stream-ordered release write of a flag
 __global__ void signal_kernel(uint32_t *flag, uint32_t value) {
   __threadfence();

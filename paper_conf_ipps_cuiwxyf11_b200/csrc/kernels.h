@@ -74,4 +74,10 @@ int launch_trsm_panel_diag(const float *Dp, int64_t ldD, float *M, int64_t ldm, 
 int launch_trsm_diag_inv(const float *A, int64_t lda, int64_t n, int stored_lower, int unit,
                          float *Dinv, int64_t ldD, cudaStream_t s);
 
+// Level 0 of that doubling (128 -> 256) on CUDA cores, one launch: for every
+// 256-row pair of L, X21 = -inv(L22) L21 inv(L11) beside the 128-block inverses
+// (launch_trsm_diag_inv first).  ldD a multiple of 256.
+int launch_trsm_level0(const float *A, int64_t lda, int64_t n, int stored_lower, float *Dinv, int64_t ldD,
+                       cudaStream_t s);
+
 }  // namespace blas3
