@@ -24,7 +24,7 @@ with open(f"profiles/{tag}_launches.md", "w") as f:
     f.write(f"# {tag}: kernel launch list of one bench step (ncu gpu__time_duration, "
             f"--clock-control none; serialized, cold caches: compare shares, not absolutes)\n\n")
     f.write(f"command: `ncu --metrics gpu__time_duration.sum --clock-control none python bench.py "
-            f"--steps 1 --warmup 0 --no-cpu-baseline --no-e2e --no-alt-mode --no-context`\n\n")
+            f"--steps 1 --warmup 0 --no-cpu-baseline --no-e2e --no-alt-mode --no-context --no-routine-clocks`\n\n")
     f.write(f"total kernel time {tot:.3f} ms over {len(seq)} launches\n\n")
     f.write("| kernel | launches | total ms | share |\n|---|---|---|---|\n")
     for n, (c, t) in agg.items():
