@@ -140,3 +140,63 @@ def test_graph_replay_concurrent_with_eager_calls(b3):
         torch.cuda.synchronize()
         for o in outs + eager:
             assert bits_equal(to_host(o), want), f"replay {rep}"
+
+
+def test_strsm_panel_solver_graph_replay(b3):
+    """The STRSM diagonal-panel solver (forced) inside a captured graph: its
+    team counters are zeroed by a memset node and its partial workspace comes
+    from the call's stream-ordered scratch.  Replays on two input sets must
+    match the eager results bit for bit (first panel forward, and backward)."""
+    import torch
+    b3.set_math_mode("3xtf32")
+    n = 2304                                      # first panel 2048 (forward) / 256 (backward)
+
+    def solve(T, X):
+        with b3.options(trsm_panel=2):
+            b3.strsm("L", "L", "N", "N", AL, T, X)
+            b3.strsm("R", "U", "T", "N", AL, T, X)
+
+    inputs = [dict(T=gen.triangular_dd(n, "L", "N", f"gp-t{s}"), B=gen.uniform(n, 768, f"gp-b{s}"))
+              for s in range(2)]
+    before = b3.launch_count("panel")
+    eager = []
+    for inp in inputs:
+        T = to_dev(inp["T"])
+        X = to_dev(inp["B"])
+        Tr = to_dev(inp["T"][:768, :768].copy())
+        with b3.options(trsm_panel=2):
+            b3.strsm("L", "L", "N", "N", AL, T, X)
+        Y = b3.colmajor(768, 768)
+        Y.copy_(X[:768])
+        with b3.options(trsm_panel=2):
+            b3.strsm("R", "U", "T", "N", AL, Tr, Y)
+        torch.cuda.synchronize()
+        eager.append((to_host(X), to_host(Y)))
+    assert b3.launch_count("panel") - before == 4, "expected the panel solver in every call"
+    sT, sX = to_dev(inputs[0]["T"]), to_dev(inputs[0]["B"])
+    sTr = to_dev(inputs[0]["T"][:768, :768].copy())
+    sY = b3.colmajor(768, 768)
+    cs = torch.cuda.Stream()
+    cs.wait_stream(torch.cuda.current_stream())
+
+    def captured():
+        with b3.options(trsm_panel=2):
+            b3.strsm("L", "L", "N", "N", AL, sT, sX)
+            sY.copy_(sX[:768])
+            b3.strsm("R", "U", "T", "N", AL, sTr, sY)
+
+    with torch.cuda.stream(cs):
+        captured()                                # per-stream state allocated eagerly first
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=cs):
+        captured()
+    for rep in range(2):
+        for s, inp in enumerate(inputs):
+            sT.copy_(to_dev(inp["T"]))
+            sTr.copy_(to_dev(inp["T"][:768, :768].copy()))
+            sX.copy_(to_dev(inp["B"]))
+            g.replay()
+            torch.cuda.synchronize()
+            assert bits_equal(to_host(sX), eager[s][0]), f"left solve differs (set {s}, replay {rep})"
+            assert bits_equal(to_host(sY), eager[s][1]), f"right solve differs (set {s}, replay {rep})"
