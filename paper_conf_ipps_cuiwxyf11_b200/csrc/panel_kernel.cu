@@ -38,11 +38,12 @@
 #include "../../include/blas3.h"
 #include "kernels.h"
 #include "tc_ptx.h"
+#include "tc_stage.h"
 
 namespace blas3 {
 namespace {
 
-constexpr int BK = 32;                     // k-block (elements)
+constexpr int BK = stage::BK;              // k-block (elements)
 constexpr int HA = 128;                    // M rows staged per CTA (block = 256 per pair)
 constexpr int BLK = 256;                   // rows of X per block (UMMA M of the pair)
 constexpr int KB_BLK = BLK / BK;           // k-blocks per group (8)
@@ -58,7 +59,9 @@ constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;       // 640
 constexpr int TR_THREADS = NUM_TR_WARPS * 32, EPI_THREADS = NUM_EPI_WARPS * 32;
 constexpr int EPI_REGS = 144, OTHER_REGS = 64;
 constexpr int NCOL = PN / 2;               // columns per epilogue thread (two warps per lane quarter)
-constexpr int LAYOUT_K = 0, LAYOUT_MN = 1;
+using stage::LAYOUT_K;
+using stage::LAYOUT_MN;
+using stage::op_desc;
 constexpr size_t PART_FLOATS = (size_t)HA * PN;   // one CTA's partial (128 rows x 256)
 
 struct alignas(1024) Stage {
@@ -94,10 +97,6 @@ __device__ __forceinline__ int64_t blk_row(const PanelParams &p, int i) {
 // right-hand side, g >= 1 the solved block g - 1)
 __device__ __forceinline__ uint32_t groups_of(const PanelParams &p, int i, int h) { return p.gmask[i][h]; }
 
-__device__ __forceinline__ uint64_t op_desc(uint32_t base, int lay, int k8) {
-  if (lay == LAYOUT_MN) return ptx::smem_desc(base + k8 * 1024, BK * 128, 512, 1);
-  return ptx::smem_desc(base + k8 * 32, 16, 1024, 2);
-}
 __device__ __forceinline__ void load_op(const CUtensorMap *m, int lay, uint8_t *dst, int64_t r0,
                                         int64_t k0, int rows, uint64_t *bar) {
   if (lay == LAYOUT_MN) {
@@ -105,20 +104,6 @@ __device__ __forceinline__ void load_op(const CUtensorMap *m, int lay, uint8_t *
       ptx::tma_load_4d(m, bar, dst + c * (BK * 128), (int32_t)(r0 + 32 * c), (int32_t)k0, 0, 0);
   } else {
     ptx::tma_load_4d(m, bar, dst, (int32_t)k0, (int32_t)r0, 0, 0);
-  }
-}
-__device__ __forceinline__ void split_pass(const uint8_t *raw, uint8_t *lo, uint32_t bytes, int t) {
-  const float4 *r4 = reinterpret_cast<const float4 *>(raw);
-  float4 *l4 = reinterpret_cast<float4 *>(lo);
-#pragma unroll 4
-  for (uint32_t c = t; c < bytes / 16; c += TR_THREADS) {
-    const float4 v = r4[c];
-    float4 l;
-    l.x = v.x - __uint_as_float(__float_as_uint(v.x) & 0xFFFFE000u);
-    l.y = v.y - __uint_as_float(__float_as_uint(v.y) & 0xFFFFE000u);
-    l.z = v.z - __uint_as_float(__float_as_uint(v.z) & 0xFFFFE000u);
-    l.w = v.w - __uint_as_float(__float_as_uint(v.w) & 0xFFFFE000u);
-    l4[c] = l;
   }
 }
 __device__ __forceinline__ void arrive_leader(uint64_t *bar, uint32_t rank, uint32_t id, uint32_t n,
@@ -133,18 +118,7 @@ __device__ __forceinline__ void arrive_leader(uint64_t *bar, uint32_t rank, uint
 // different clusters): release = __threadfence + atomicAdd after a CTA's
 // stores; acquire = ld.acquire.gpu poll, plus a proxy fence before TMA reads.
 __device__ __forceinline__ void wait_count(const uint32_t *ctr, uint32_t target) {
-  uint32_t v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
-  if (v >= target) return;
-  unsigned long long t0, t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
-  for (;;) {
-    __nanosleep(64);
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
-    if (v >= target) return;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-    if (t - t0 > 4000000000ull) __trap();      // a team partner that never runs fails loudly
-  }
+  stage::spin_until(ctr, target, 64);
 }
 
 // diagnostics: %globaltimer of stage st of block i, team 0, CTA rank 0 of member h
@@ -284,8 +258,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
           ptx::mbar_wait(&bars->full[rs], (it / RS) & 1);
           ptx::mbar_wait(&bars->lo_empty[ls], ((it / LS) & 1) ^ 1);
           if (!(prm.dbg & 2)) {
-            split_pass(raw[rs].A, lo[ls].A, HA * BK * 4, tt);
-            split_pass(raw[rs].B, lo[ls].B, HB * BK * 4, tt);
+            stage::split_pass<TR_THREADS>(raw[rs].A, lo[ls].A, HA * BK * 4, tt);
+            stage::split_pass<TR_THREADS>(raw[rs].B, lo[ls].B, HB * BK * 4, tt);
           }
           ptx::fence_proxy_async_smem();
           arrive_leader(&bars->ready[ls], rank, 2, TR_THREADS, tt == 0);

@@ -44,6 +44,7 @@
 #include "../../include/blas3.h"
 #include "kernels.h"
 #include "tc_ptx.h"
+#include "tc_stage.h"
 #include <cuda_bf16.h>
 
 namespace blas3 {
@@ -54,7 +55,7 @@ namespace {
 // tile, each CTA staging its 128 rows of A and 128 of the 256 B rows: per SM
 // the tensor core reads half as many B bytes per flop, and shared-memory
 // bandwidth is what bounds this kernel (profiles/r01_sgemm_ncu.md).
-constexpr int BK = 32;
+constexpr int BK = stage::BK;
 constexpr int HA = 128;                    // A rows staged per CTA
 constexpr int BN = 256;                    // tile columns (UMMA N)
 // Roles are aligned to warpgroups so setmaxnreg can move registers to the
@@ -83,7 +84,10 @@ constexpr int MAX_MAPS = 10;                 // 2 segments x 2 operands x 2 view
 // transpose between the TMEM layout (thread = row) and 16-B vector accesses
 // of column-major C (thread = 4 consecutive rows of one column)
 constexpr int EPI_GW = 8, EPI_BOX = 32 * EPI_GW;
-constexpr int LAYOUT_K = 0, LAYOUT_MN = 1;
+using stage::LAYOUT_K;
+using stage::LAYOUT_MN;
+using stage::op_desc;
+using stage::spin_until;
 
 // A work item: the tile (batch member b, tile t at m0, n0) and the range
 // [g0, g1) of its k-blocks, counted over the concatenated segments.
@@ -423,19 +427,6 @@ __device__ __forceinline__ void zero_fill(uint8_t *buf, uint32_t bytes, int t) {
   for (uint32_t c = t; c < bytes / 16; c += TR_THREADS) b4[c] = make_float4(0.f, 0.f, 0.f, 0.f);
 }
 
-// 3xTF32 split without rewriting hi: kind::tf32 UMMA reads the raw fp32
-// word and ignores its low 13 mantissa bits, i.e. it consumes
-// hi = trunc_tf32(x) directly from the TMA-staged tile (pinned by
-// tests/test_parity_gpu.py::test_split_is_real).  Only lo = x - hi (exact in
-// fp32: the 13 bits below hi) is produced; the tensor core reads its top 11
-// bits the same way, so hi + tf32(lo) represents x to within 2^-21 |x|, far
-// below the K-linear accumulation error of the fp32 TMEM accumulator
-// (Q17, Q24).  Two ops per element (LOP + FADD).
-__device__ __forceinline__ float split_lo(float x) {
-  const float hi = __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
-  return x - hi;
-}
-
 // BLAS3_MATH_TF32_BF16X: the two cross terms of the split packed into ONE bf16
 // operand pair per k8 step.  For a staged tile (raw, either layout) with
 // x = hi + lo (hi = trunc_tf32(x)), the K-major bf16 tile `dst` holds, per
@@ -505,27 +496,7 @@ __device__ __forceinline__ void pack_cross(const uint8_t *raw, int lay, uint8_t 
   }
 }
 
-__device__ __forceinline__ void split_pass(const uint8_t *raw, uint8_t *lo, uint32_t bytes, int t) {
-  const float4 *r4 = reinterpret_cast<const float4 *>(raw);
-  float4 *l4 = reinterpret_cast<float4 *>(lo);
-#pragma unroll 4
-  for (uint32_t c = t; c < bytes / 16; c += TR_THREADS) {
-    const float4 v = r4[c];
-    float4 l;
-    l.x = split_lo(v.x);
-    l.y = split_lo(v.y);
-    l.z = split_lo(v.z);
-    l.w = split_lo(v.w);
-    l4[c] = l;
-  }
-}
-
 // ---------------------------------------------------------------- MMA
-__device__ __forceinline__ uint64_t op_desc(uint32_t base, int lay, int k8) {
-  if (lay == LAYOUT_MN) return ptx::smem_desc(base + k8 * 1024, BK * 128, 512, 1);
-  return ptx::smem_desc(base + k8 * 32, 16, 1024, 2);
-}
-
 // A role's warps (nthreads, named barrier `id`) have finished with a stage:
 // sync them CTA-locally, then ONE thread arrives on the barrier owned by the
 // pair's leader (a cluster-scope release per thread would cost a GPU-scope
@@ -535,20 +506,6 @@ template <int CG>
 __device__ __forceinline__ int64_t slab_of(const PhaseDesc &ph, const Work &w) {
   const int64_t s = ph.slab_m ? w.m0 / Geo<CG>::TM : w.n0 / BN;
   return s < MAX_SLAB ? s : MAX_SLAB - 1;
-}
-__device__ __forceinline__ void spin_until(const uint32_t *ctr, uint32_t target) {
-  uint32_t v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
-  if (v >= target) return;
-  unsigned long long t0, t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
-  for (;;) {
-    __nanosleep(128);
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
-    if (v >= target) return;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-    if (t - t0 > 4000000000ull) __trap();      // a broken dependency graph fails loudly, never hangs
-  }
 }
 // Wait (one thread) until the tile's dependencies are complete; the acquire
 // makes the producing CTAs' stores visible, and the proxy fence orders them
@@ -1004,8 +961,8 @@ tc_structured_gemm(const __grid_constant__ PRM prm) {
           } else {
             ptx::mbar_wait(&bars->lo_empty[ls], lph ^ 1);
             if (!(P.dbg & 1) && P.passes != 1) {
-              split_pass(rb.A, lo[ls].A, G::A_BYTES, tt);
-              split_pass(rb.B, lo[ls].B, G::B_BYTES, tt);
+              stage::split_pass<TR_THREADS>(rb.A, lo[ls].A, G::A_BYTES, tt);
+              stage::split_pass<TR_THREADS>(rb.B, lo[ls].B, G::B_BYTES, tt);
             }
           }
           ptx::fence_proxy_async_smem();
