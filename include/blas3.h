@@ -277,10 +277,9 @@ int blas3_get_math_mode(void);
  *                          panel (256-row blocks, precomputed couplings
  *                          -inv(op(A)_ss) op(A)_sf), no grid-wide dependency
  *                          steps; 0: the fused doubling + geometric chain; 2: the
- *                          solver even when its teams (two CTA pairs per 256
- *                          right-hand sides) do not fill most of the SMs (1 uses
- *                          it only then).  Used when the panel's order is a
- *                          multiple of 256 and B is 16-B aligned with ldb % 4 == 0
+ *                          same as 1 (kept for scripts).  Used when the panel's
+ *                          order is a multiple of 256 and B is 16-B aligned with
+ *                          ldb % 4 == 0
  * blas3_set_option returns 0, or 1 for an unknown key or an invalid value
  * (nothing changed).  blas3_get_option returns the current value, or
  * INT64_MIN for an unknown key. */

@@ -1158,11 +1158,9 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // BLAS3_OPT_TRSM_PANEL: the first panel by the diagonal-panel solver (its
   // M workspace after W); the geometric chain's Y/M are then not needed
   const int64_t r_first = imin(NBO, nt - pfirst * NBO);
-  // (only when its teams of two CTA pairs fill most of the machine: with fewer
-  // right-hand sides the panel-inverse chain is cheaper, STRSM N = 4096 608 vs
-  // 581 us, profiles/r02_strsm_panel.md)
-  const bool use_panel = opt(BLAS3_OPT_TRSM_PANEL) != 0 && tensor_mode() && r_first % 256 == 0 &&
-                         (opt(BLAS3_OPT_TRSM_PANEL) == 2 || 4 * cdiv(other, 256) >= (int64_t)sms * 4 / 5);
+  // (at every right-hand-side count: STRSM 2048 / 4096 / 8192 x 4096 RHS / 8192
+  // measured 2.6 / 7.5 / 3.3 / 3.4% faster than the fused chain, profiles/r02_strsm_panel.md)
+  const bool use_panel = opt(BLAS3_OPT_TRSM_PANEL) != 0 && tensor_mode() && r_first % 256 == 0;
   Scratch Mw;
   const size_t m_bytes = (size_t)r_first * r_first * sizeof(float);
   if (use_panel &&

@@ -41,6 +41,10 @@ A1, B1, C1 = mk(1024, 1024), mk(1024, 1024), mk(1024, 1024)
 T4, X4, B4 = mk(4096, 4096), mk(4096, 4096), mk(4096, 4096)
 T4.mul_(1.0 / 4096)
 T4.diagonal().fill_(1.0)
+T2, X2, Bx2 = mk(2048, 2048), mk(2048, 2048), mk(2048, 2048)
+T2.mul_(1.0 / 2048)
+T2.diagonal().fill_(1.0)
+X84, B84 = mk(8192, 4096), mk(8192, 4096)
 cases = {
     "sgemm": (lambda: b3.sgemm("N", "N", 1.5, A, B, 0.5, C), 2.0 * n ** 3, 5, None),
     "ssymm": (lambda: b3.ssymm("L", "L", 1.5, A, B, 0.5, C), 2.0 * n ** 3, 5, None),
@@ -53,6 +57,9 @@ cases = {
     "sgemm2048": (lambda: b3.sgemm("N", "N", 1.5, A2, B2, 0.5, C2), 2.0 * 2048 ** 3, 40, None),
     "sgemm1024": (lambda: b3.sgemm("N", "N", 1.5, A1, B1, 0.5, C1), 2.0 * 1024 ** 3, 100, None),
     "strsm4096": (lambda: b3.strsm("L", "L", "N", "N", 1.0, T4, X4), 1.0 * 4096 ** 3, 10, lambda: X4.copy_(B4)),
+    "strsm2048": (lambda: b3.strsm("L", "L", "N", "N", 1.0, T2, X2), 1.0 * 2048 ** 3, 20, lambda: X2.copy_(Bx2)),
+    "strsm8k4k": (lambda: b3.strsm("L", "L", "N", "N", 1.0, T, X84), 1.0 * 8192 ** 2 * 4096, 5,
+                  lambda: X84.copy_(B84)),
 }
 sel = [c for c in args.cases.split(",") if c in cases]
 
