@@ -395,7 +395,7 @@ int launch_trsm_panel_diag(const float *Dp, int64_t ldD, float *M, int64_t ldm, 
 
 // member 0's serial hand-off per block in tenths of a group (BLAS3_PANEL_HANDOFF, experiments)
 static int64_t prm_handoff() {
-  static const int64_t v = [] { const char *e = getenv("BLAS3_PANEL_HANDOFF"); return e ? atoll(e) : 6; }();
+  static const int64_t v = [] { const char *e = getenv("BLAS3_PANEL_HANDOFF"); return e ? atoll(e) : 3; }();
   return v;
 }
 // members per team at most (BLAS3_PANEL_MEMBERS, 1..MAX_MEM; default 2: a
@@ -459,7 +459,8 @@ int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool r
   // waits for the block just solved), every other group goes to the member
   // with the least work so far (ties to a helper, whose partial runs ahead).
   // Member 0 is also charged its serial per-block hand-off (store, release,
-  // reload of X_i: about 0.6 of a group's MMA time, measured)
+  // reload of X_i), 0.3 of a group: kernel 187 / 189 us at N = 4096 / 8192
+  // against 194 / 196 at 0.6 and 188 / 190 at 0 (profiles/r02_strsm_panel.md)
   const int64_t grp = 10, handoff = prm_handoff();
   int64_t load[MAX_MEM] = {0, 0, 0, 0};
   for (int i = 0; i < prm.nblk; ++i) {
