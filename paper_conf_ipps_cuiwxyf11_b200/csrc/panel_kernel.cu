@@ -398,21 +398,38 @@ static int64_t prm_handoff() {
   static const int64_t v = [] { const char *e = getenv("BLAS3_PANEL_HANDOFF"); return e ? atoll(e) : 3; }();
   return v;
 }
-// members per team at most (BLAS3_PANEL_MEMBERS, 1..MAX_MEM; default 2: a
-// third and fourth pair did not shorten the solve -- member 0's per-block
-// chain of newest group, store and reload bounds it -- and take SMs from the
-// concurrent panel-inverse doubling, STRSM N = 4096 643 vs 623 us)
+// members per team at most (BLAS3_PANEL_MEMBERS, 1..MAX_MEM; default 3, when
+// the machine holds them: N = 4096, 16 teams, kernel 167 us with three
+// members against 187 with two and 200 with four -- with four, member 0 only
+// keeps the newest group and its per-block chain, which now includes reading
+// three partials, bounds the solve; profiles/r02_strsm_panel.md)
 static int panel_members() {
-  static const int v = [] { const char *e = getenv("BLAS3_PANEL_MEMBERS"); const int m = e ? atoi(e) : 2;
+  static const int v = [] { const char *e = getenv("BLAS3_PANEL_MEMBERS"); const int m = e ? atoi(e) : 3;
                             return m < 1 ? 1 : (m > MAX_MEM ? MAX_MEM : m); }();
   return v;
 }
 // teams: one per 256 right-hand sides (at most num_sms / 4); members: the
 // CTA pairs the machine holds per team, up to panel_members()
+// The member count -- and with it each block's split into partial sums, i.e.
+// the rounding -- follows the DEVICE's SM count, not the launch limit
+// (BLAS3_OPT_MAX_SMS): a solve on fewer SMs runs fewer teams, each looping over
+// more slabs, and gives the same bits (tests/test_trsm_panel_gpu.py).
+static int device_sms() {
+  static std::atomic<int> cache[64];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 148;
+  int v = cache[dev].load(std::memory_order_relaxed);
+  if (v == 0) {
+    if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v < 2) v = 148;
+    cache[dev].store(v, std::memory_order_relaxed);
+  }
+  return v;
+}
 static void panel_shape(int64_t nrhs, int num_sms, int64_t &teams, int &nmem) {
-  const int64_t nslab = (nrhs + PN - 1) / PN, pairs = num_sms / 2;
-  teams = imin(nslab, imax(1, pairs / 2));
-  nmem = (int)imax(1, imin(panel_members(), pairs / teams));
+  const int64_t nslab = (nrhs + PN - 1) / PN, pairs = num_sms / 2, full = device_sms() / 2;
+  nmem = (int)imax(1, imin(panel_members(), full / imin(nslab, imax(1, full / 2))));
+  if (nmem > pairs) nmem = (int)imax(1, pairs);        // (a launch limit below one team)
+  teams = imin(nslab, imax(1, pairs / nmem));
 }
 size_t trsm_panel_ws_bytes(int64_t nrhs, int num_sms) {
   int64_t t;
