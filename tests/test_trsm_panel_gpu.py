@@ -118,3 +118,29 @@ def test_panel_solver_leaves_outside_untouched(b3):
     assert np.isnan(host[:rhs, order:]).all()   # padding rows of each column
     assert np.isnan(host[rhs:]).all()           # columns beyond n
     assert np.isfinite(host[:rhs, :order]).all()
+
+
+def test_panel_solver_concurrent_streams(b3):
+    """Two solves on two streams at once, each with more teams than fit beside
+    the other: the second grid's CTAs become resident as the first one's
+    retire, a team's pairs are consecutive in launch order, and both results
+    match the same solves run one after the other (bit for bit)."""
+    import torch
+    order, rhs = 2048, 8192
+    A = gen.triangular_dd(order, "L", "N", "pc")
+    Bs = [gen.uniform(order, rhs, f"pc-b{i}") for i in range(2)]
+    dA = to_dev(A)
+    seq = []
+    for B in Bs:
+        X, _ = solve(b3, "L", "L", "N", "N", A, B)
+        seq.append(X)
+    dX = [to_dev(B) for B in Bs]
+    streams = [torch.cuda.Stream() for _ in range(2)]
+    torch.cuda.synchronize()
+    with b3.options(trsm_panel=2):
+        for X, st in zip(dX, streams):
+            with torch.cuda.stream(st):
+                b3.strsm("L", "L", "N", "N", AL, dA, X)
+    torch.cuda.synchronize()
+    for X, ref in zip(dX, seq):
+        assert np.array_equal(to_host(X).view(np.uint32), ref.view(np.uint32))
