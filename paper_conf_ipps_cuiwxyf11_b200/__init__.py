@@ -252,7 +252,7 @@ OPTIONS = {"gm_map": 0, "gm_min_gemm": 1, "gm_min_symm": 2, "gm_min_trmm": 3, "g
            "trsm_slab_min": 11, "trsm_reserve": 12, "trsm_geo_leaf": 13, "trsm_fused": 14,
            "trsm_first_ym": 15, "trsm_first_fused": 16, "trsm_first_split": 17, "trsm_first_all": 18, "tc_raster": 19,
            "tc_kc": 20, "tc_vec_store": 21, "max_sms": 22,
-           "tc_c_prefetch": 23, "tc_c_async": 24, "trsm_panel": 25}
+           "tc_c_prefetch": 23, "tc_c_async": 24, "trsm_panel": 25, "trsm_panel2": 26}
 
 
 def set_option(name, value):

@@ -53,6 +53,7 @@ static const OptSpec kOpt[BLAS3_OPT_COUNT] = {
     {"BLAS3_TC_C_PREFETCH", 1, 0, 1, false},
     {"BLAS3_TC_C_ASYNC", 0, 0, 1, false},
     {"BLAS3_TRSM_PANEL", 1, 0, 2, false},
+    {"BLAS3_TRSM_PANEL2", 0, 0, 2, false},
 };
 static std::atomic<int64_t> g_opt[BLAS3_OPT_COUNT];
 static std::once_flag g_opt_once;
@@ -1041,18 +1042,22 @@ static int strsm_first_fused(const TrsmGeom &g, const std::vector<GeoPair> &gp, 
   return rc == 0 ? 0 : (rc == -4 ? BLAS3_ERR_TMA : BLAS3_ERR_CUDA);
 }
 
-// The first processed panel by the diagonal-panel solver (BLAS3_OPT_TRSM_PANEL,
-// panel_kernel.cu): level 0 of the panel's doubling (its 256-block inverses),
-// the couplings M = -inv(op(A)_ss) op(A)_sf of every 256-block s (one batched
-// GEMM over the whole panel row -- the kernel reads only the solved part) and
-// alpha * inv(op(A)_ss) on M's diagonal, then ONE launch in which every CTA
-// pair forward-substitutes its 128 right-hand sides through the panel.
-// Returns 1 if not applicable (nothing enqueued), 0, or < 0 on an error.
-static int strsm_first_panel(const TrsmGeom &g, int64_t pfirst, float *Mw, void *pws, cudaStream_t s, int sms) {
-  const int64_t NBO = g.NBO, p0 = pfirst * NBO, R = imin(NBO, g.nt - p0), ldm = R;
-  if (R % 256 || R > 8192 || (reinterpret_cast<uintptr_t>(g.B) % 16) || g.ldb % 4) return 1;
+// The diagonal-panel solver (panel_kernel.cu) for panel pidx: level 0 of the
+// panel's doubling (its 256-block inverses), the couplings
+// M = -inv(op(A)_ss) op(A)_sf of every 256-block s (one batched GEMM over the
+// whole panel row -- the kernel reads only the solved part) and
+// a_diag * inv(op(A)_ss) on M's diagonal (strsm_panel_prep), then ONE launch
+// in which every team of CTA pairs forward-substitutes its 256 right-hand
+// sides through the panel, in place over B (strsm_panel_run).
+// panel_ok: whether the solver applies (order a multiple of 256, B aligned).
+static bool panel_ok(const TrsmGeom &g, int64_t pidx) {
+  const int64_t R = imin(g.NBO, g.nt - pidx * g.NBO);
+  return R > 0 && R % 256 == 0 && R <= 8192 && (reinterpret_cast<uintptr_t>(g.B) % 16) == 0 && g.ldb % 4 == 0;
+}
+static int strsm_panel_prep(const TrsmGeom &g, int64_t pidx, float a_diag, float *Mw, cudaStream_t s, int sms) {
+  const int64_t NBO = g.NBO, p0 = pidx * NBO, R = imin(NBO, g.nt - p0), ldm = R;
   const int64_t nb = R / 256;
-  float *Dp = g.D + pfirst * NBO * NBO;
+  float *Dp = g.D + pidx * NBO * NBO;
   const float *Ap = g.A + p0 * (1 + g.lda);
   Problem P;
   if (g.left) {        // M(s, c) = -sum_k inv(op(A)_ss)(r, k) op(A)(s_lo + k, p0 + c), batch over s
@@ -1081,11 +1086,23 @@ static int strsm_first_panel(const TrsmGeom &g, int64_t pfirst, float *Mw, void 
   // one launch, then the couplings
   if (launch_trsm_level0(Ap, g.lda, R, g.lower, Dp, NBO, s)) return BLAS3_ERR_CUDA;
   if (nb > 1 && (rc = run_problem(P, s, sms))) return rc;
-  if (launch_trsm_panel_diag(Dp, NBO, Mw, ldm, R, g.lower_op, g.alpha, s)) return BLAS3_ERR_CUDA;
+  if (launch_trsm_panel_diag(Dp, NBO, Mw, ldm, R, g.lower_op, a_diag, s)) return BLAS3_ERR_CUDA;
+  return 0;
+}
+static int strsm_panel_run(const TrsmGeom &g, int64_t pidx, const float *Mw, void *pws, cudaStream_t s, int sms) {
+  const int64_t p0 = pidx * g.NBO, R = imin(g.NBO, g.nt - p0);
   float *X = g.left ? g.B + p0 : g.B + p0 * g.ldb;
-  rc = launch_trsm_panel(Mw, ldm, X, g.ldb, !g.left, R, g.other, g.forward, (int)opt(BLAS3_OPT_TC_KC), pws, s,
-                         sms);
+  const int rc = launch_trsm_panel(Mw, R, X, g.ldb, !g.left, R, g.other, g.forward, (int)opt(BLAS3_OPT_TC_KC), pws,
+                                   s, sms);
   return rc == 0 ? 0 : (rc == -4 ? BLAS3_ERR_TMA : BLAS3_ERR_CUDA);
+}
+// The first processed panel (BLAS3_OPT_TRSM_PANEL): returns 1 if not
+// applicable (nothing enqueued), 0, or < 0 on an error.
+static int strsm_first_panel(const TrsmGeom &g, int64_t pfirst, float *Mw, void *pws, cudaStream_t s, int sms) {
+  if (!panel_ok(g, pfirst)) return 1;
+  int rc = strsm_panel_prep(g, pfirst, g.alpha, Mw, s, sms);
+  if (rc) return rc;
+  return strsm_panel_run(g, pfirst, Mw, pws, s, sms);
 }
 
 int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t n, float alpha,
@@ -1161,11 +1178,22 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // (at every right-hand-side count: STRSM 2048 / 4096 / 8192 x 4096 RHS / 8192
   // measured 2.6 / 7.5 / 3.3 / 3.4% faster than the fused chain, profiles/r02_strsm_panel.md)
   const bool use_panel = opt(BLAS3_OPT_TRSM_PANEL) != 0 && tensor_mode() && r_first % 256 == 0;
+  // BLAS3_OPT_TRSM_PANEL2: the second processed panel by the solver too (one
+  // right-hand-side slab; the panel's 256-block inverses and couplings on the
+  // high-priority side stream beside the first panel's kernel)
+  const int64_t psecond = forward ? 1 : npanel - 2;
+  const int64_t r_second = npanel >= 2 ? imin(NBO, nt - psecond * NBO) : 0;
+  const bool want_panel2 = use_panel && npanel >= 2 && opt(BLAS3_OPT_TRSM_PANEL2) != 0 && r_second % 256 == 0 &&
+                           trsm_slabs(other) == 1 && opt(BLAS3_OPT_TRSM_FUSED) != 2;
   Scratch Mw;
   const size_t m_bytes = (size_t)r_first * r_first * sizeof(float);
+  const size_t pws_bytes = trsm_panel_ws_bytes(other, sms);
+  const size_t m2_bytes = want_panel2 ? (size_t)r_second * r_second * sizeof(float) : 0;
   if (use_panel &&
-      (rc = get_scratch(Mw, m_bytes + trsm_panel_ws_bytes(other, sms), s, aop_bytes + d_bytes + t_bytes + w_bytes)))
+      (rc = get_scratch(Mw, m_bytes + pws_bytes + m2_bytes, s, aop_bytes + d_bytes + t_bytes + w_bytes)))
     return rc;
+  float *Mw2 = want_panel2 ? reinterpret_cast<float *>(reinterpret_cast<uint8_t *>(Mw.p) + m_bytes + pws_bytes)
+                           : nullptr;
   std::vector<GeoPair> gp;
   Scratch YM;
   const bool use_ym = !use_panel && (opt(BLAS3_OPT_TRSM_FIRST_YM) != 0 || opt(BLAS3_OPT_TRSM_FIRST_FUSED) != 0);
@@ -1242,6 +1270,20 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   std::vector<GeoPair> outer;                         // popped pairs, inner -> outer
   const int64_t fsplit = opt(BLAS3_OPT_TRSM_FIRST_SPLIT);
   first_done = all_done || panel_done;
+  // the second panel's precompute on side3 (after the 128-block inverses);
+  // alpha is already applied by the update that precedes its solve
+  bool panel2 = false;
+  if (want_panel2 && panel_done) {
+    const TrsmGeom g{left, lower, ta, unit, lower_op, forward, m, n, nt, NBO, npanel, other, alpha,
+                     A, lda, B, ldb, D.p, Tw.p, W.p};
+    if (panel_ok(g, psecond)) {
+      if (cudaStreamWaitEvent(ts->side3, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+      rc = strsm_panel_prep(g, psecond, 1.f, Mw2, ts->side3, sms);
+      if (rc < 0) return rc;
+      panel2 = rc == 0;
+      if (panel2 && cudaEventRecord(ts->ev_ym[0], ts->side3) != cudaSuccess) return BLAS3_ERR_CUDA;
+    }
+  }
   if (!first_done && opt(BLAS3_OPT_TRSM_FIRST_FUSED) && tensor_mode() && !gp.empty()) {
     if (fsplit > 0)
       while (gp.size() >= 2 && gp.back().h >= fsplit && outer.size() < (size_t)MAX_LEVELS) { outer.insert(outer.begin(), gp.back()); gp.pop_back(); }
@@ -1285,9 +1327,12 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // those panels (the side stream builds the levels below it)
   const bool fused_sweep = panel_done && opt(BLAS3_OPT_TRSM_FUSED) == 2 && npanel > 1 && nlvl >= 2 &&
                            math_mode() == BLAS3_MATH_3XTF32;
-  const int64_t prest = forward ? 1 : 0, orest = prest * NBO;
-  const int64_t nrest = imin(nt, (prest + npanel - 1) * NBO) - orest;
-  if (npanel > 1 && !all_done) {
+  // the panels the doubling serves: all but the first (and the second when the
+  // solver takes it)
+  const int64_t prest = forward ? (panel2 ? 2 : 1) : 0, orest = prest * NBO;
+  const int64_t nrest = imin(nt, (forward ? npanel : npanel - (panel2 ? 2 : 1)) * NBO) - orest;
+  const bool rest_dbl = npanel > 1 && !all_done && nrest > 0;
+  if (rest_dbl) {
     if (cudaStreamWaitEvent(ts->side2, ts->ev_fork, 0) != cudaSuccess) return BLAS3_ERR_CUDA;
     // (beside the panel solver, level 0 on CUDA cores in one launch, as for the first panel)
     const int from = panel_done && nlvl >= 1 ? 1 : 0;
@@ -1436,7 +1481,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
     // update: rows (L) / columns (R) [o_lo, o_hi) <- a1 * B_o - op(A)(o, k) X_k, k in [k_lo, k_hi);
     // to_w: the result goes to W (the next operation is the leaf solve of o)
     auto update = [&](int64_t k_lo, int64_t k_hi, int64_t o_lo, int64_t o_hi, float a1, bool to_w,
-                      bool restrict_sms = true) -> int {
+                      bool restrict_sms = true, int lim = 0) -> int {
       const bool rs = restrict_sms && o_lo / NBO == pfirst && (o_hi - 1) / NBO == pfirst;
       if (left) {   // Xa(r,kk) = op(A)(o_lo+r, k_lo+kk): !ta -> A(o_lo+r, k_lo+kk) rk; ta -> A(k_lo+kk, o_lo+r) kr
         const float *pa = ta ? A + k_lo + o_lo * lda : A + o_lo + k_lo * lda;
@@ -1446,6 +1491,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
         P.seg[0].b = dense(Bq + k_lo, ldb, true);
         P.seg[0].K = k_hi - k_lo;
         if (rs) P.max_sms = first_sms;
+        if (lim > 0) P.max_sms = lim;
         return run_problem(P, st, sms);
       }
       // B(:,o) <- a1*B(:,o) - X_k * op(A)(k, o):
@@ -1457,6 +1503,7 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
       P.seg[0].b = dense(pb, lda, !ta);
       P.seg[0].K = k_hi - k_lo;
       if (rs) P.max_sms = first_sms;
+      if (lim > 0) P.max_sms = lim;
       return run_problem(P, st, sms);
     };
     // geometric solve of the aligned block [lo, lo + w) (clipped to nt): the
@@ -1510,6 +1557,12 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
         const int64_t p = forward ? q0 : npanel - 1 - q0;
         const int64_t p0 = p * NBO, pr = imin(NBO, nt - p0);
         if (q0 == 0) return first_done ? 0 : geo(p0, NBO, scaled);   // the first processed panel
+        if (q0 == 1 && panel2) {                       // the second, by the solver, in place
+          const TrsmGeom g{left, lower, ta, unit, lower_op, forward, m, n, nt, NBO, npanel, other, alpha,
+                           A, lda, B, ldb, D.p, Tw.p, W.p};
+          if (cudaStreamWaitEvent(st, ts->ev_ym[0], 0) != cudaSuccess) return BLAS3_ERR_CUDA;
+          return strsm_panel_run(g, p, Mw2, reinterpret_cast<uint8_t *>(Mw.p) + m_bytes, st, sms);
+        }
         return leaf(p0, pr, NBO, scaled, in_w);
       }
       const int64_t mid = q0 + (q1 - q0) / 2;
@@ -1521,8 +1574,13 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
         if (forward && k_lo < app_hi) k_lo = imax(k_lo, app_hi);
         if (!forward && k_hi > app_lo) k_hi = imin(k_hi, app_lo);
       }
-      const bool to_w = (q1 - mid == 1);               // updated panel goes straight to W
-      if ((rc2 = update(k_lo, k_hi, o_lo, o_hi, scaled ? 1.f : alpha, to_w))) return rc2;
+      // updated panel goes straight to W (not the solver's: it works in place)
+      const bool to_w = (q1 - mid == 1) && !(mid == 1 && panel2);
+      // (before the second panel's solve, optionally leave SMs to the side
+      // streams: BLAS3_PANEL2_FREE SMs, default 0)
+      static const int64_t p2_free = [] { const char *e = getenv("BLAS3_PANEL2_FREE"); return e ? atoll(e) : 0; }();
+      const int lim = mid == 1 && panel2 && p2_free > 0 ? (int)imax(2, sms - p2_free) : 0;
+      if ((rc2 = update(k_lo, k_hi, o_lo, o_hi, scaled ? 1.f : alpha, to_w, true, lim))) return rc2;
       return rec(mid, q1, true, to_w);
     };
     if (split) {
@@ -1554,8 +1612,9 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   // the side streams' last levels are part of this call (scratch is freed on s)
   if (!first_done && nlvl > 0 && cudaStreamWaitEvent(s, ts->ev_lvl[nlvl - 1], 0) != cudaSuccess)
     return BLAS3_ERR_CUDA;
-  if (nlvl > 0 && npanel > 1 && !all_done && cudaStreamWaitEvent(s, ts->ev_lvl2[nlvl - 1], 0) != cudaSuccess)
+  if (nlvl > 0 && rest_dbl && cudaStreamWaitEvent(s, ts->ev_lvl2[nlvl - 1], 0) != cudaSuccess)
     return BLAS3_ERR_CUDA;
+  if (panel2 && cudaStreamWaitEvent(s, ts->ev_ym[0], 0) != cudaSuccess) return BLAS3_ERR_CUDA;
   return finish(0);
 }
 

@@ -84,18 +84,86 @@ struct PanelParams {
                                            // partials written (x2 CTAs each)
   int64_t ldx, R, nrhs;
   int32_t nblk, layA, layB, right, forward, kc, nslab, nteams, nmem;
+  // extra members (one CTA pair serving several teams, see role_of): the
+  // device-level split -- T_dev teams, E_dev extras, extra e = slab % E_dev --
+  // fixes every slab's group masks (and with them the rounding); a launch
+  // that cannot place the extras (fold = 1) has each team's last core member
+  // compute the extra's partial as a second item per block
+  int32_t tdev, edev, nextra, fold;
   int32_t dbg;                             // BLAS3_DEBUG_PANEL knock-outs (timing experiments only)
   unsigned long long *trace;               // BLAS3_TRACE_PANEL: per-block stage times of team 0 (diagnostics)
-  uint32_t gmask[MAX_BLK][MAX_MEM];        // groups of block i summed by member h
+  uint32_t gmask[2][MAX_BLK][MAX_MEM];     // [class][block i][member h]: groups summed by h (h = nmem: the extra)
 };
 
 // first row of processing block i
 __device__ __forceinline__ int64_t blk_row(const PanelParams &p, int i) {
   return (int64_t)(p.forward ? i : p.nblk - 1 - i) * BLK;
 }
-// groups of block i summed by member h (bit g: group g; g = 0 the block's own
-// right-hand side, g >= 1 the solved block g - 1)
-__device__ __forceinline__ uint32_t groups_of(const PanelParams &p, int i, int h) { return p.gmask[i][h]; }
+// group-mask class of a slab: 0 if its extra serves the most teams, else 1
+__host__ __device__ __forceinline__ int slab_class(int tdev, int edev, int slab) {
+  return (edev == 0 || tdev % edev == 0 || slab % edev < tdev % edev) ? 0 : 1;
+}
+// groups of block i summed by member h for slab (bit g: group g; g = 0 the
+// block's own right-hand side, g >= 1 the solved block g - 1)
+__device__ __forceinline__ uint32_t groups_of(const PanelParams &p, int slab, int i, int h) {
+  return p.gmask[slab_class(p.tdev, p.edev, slab)][i][h];
+}
+constexpr int MAX_SERVE = 8;               // teams per extra pair at most
+// The work items of one CTA pair, in the order all four roles visit them.
+//   core pair (team, member hc): for every slab of the team (slab = team +
+//     r * nteams), for every block i: member hc's partial (hc = 0: the owner,
+//     which also stores X_i); with fold, member nmem - 1 follows each of its
+//     items with the extra's (member nmem) partial of the same block;
+//   extra pair e (every team owns exactly one slab): for every block i, for
+//     every team it serves (slab = e + j * nextra): member nmem's partial.
+struct Role {
+  int team0, hc, extra, nserved, nper, nitems;
+};
+__device__ __forceinline__ Role role_of(const PanelParams &p, int pair) {
+  Role r;
+  const int ncore = p.nteams * p.nmem;
+  r.extra = pair >= ncore;
+  if (r.extra) {
+    r.team0 = pair - ncore;
+    r.hc = p.nmem;
+    r.nserved = (p.nteams - r.team0 + p.nextra - 1) / p.nextra;
+    r.nper = 1;
+    r.nitems = p.nblk * r.nserved;
+  } else {
+    r.team0 = pair / p.nmem;
+    r.hc = pair % p.nmem;
+    r.nserved = 1;
+    r.nper = (p.fold && r.hc == p.nmem - 1) ? 2 : 1;
+    r.nitems = (p.nslab - r.team0 + p.nteams - 1) / p.nteams * p.nblk * r.nper;
+  }
+  return r;
+}
+struct Item {
+  int slab, team, i, h, j;                 // j: served-team index (extras), else 0
+  uint32_t gblk, gbase;                    // block counter of the slab's team, its value at block 0
+};
+__device__ __forceinline__ Item item_of(const PanelParams &p, const Role &r, int idx) {
+  Item it;
+  if (r.extra) {
+    it.i = idx / r.nserved;
+    it.j = idx % r.nserved;
+    it.slab = r.team0 + it.j * p.nextra;
+    it.team = it.slab;
+    it.h = p.nmem;
+    it.gblk = (uint32_t)it.i;
+    it.gbase = 0;
+  } else {
+    const int per_slab = p.nblk * r.nper, rr = idx / per_slab, rem = idx % per_slab;
+    it.i = rem / r.nper;
+    it.h = r.hc + rem % r.nper;
+    it.j = 0;
+    it.slab = r.team0 + rr * p.nteams;
+    it.team = r.team0;
+    it.gbase = (uint32_t)(rr * p.nblk);
+    it.gblk = it.gbase + (uint32_t)it.i;
+  }
+  return it;
+}
 
 __device__ __forceinline__ void load_op(const CUtensorMap *m, int lay, uint8_t *dst, int64_t r0,
                                         int64_t k0, int rows, uint64_t *bar) {
@@ -139,9 +207,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const uint32_t rank = ptx::cluster_ctarank();
   const int pair = blockIdx.x / 2;
-  const int team = pair / prm.nmem, h = pair % prm.nmem;   // team member: 0 stores X, others help
+  const Role role = role_of(prm, pair);
+  const int h = role.hc;                                   // 0: owner of its team's X, else a helper
   const int nblk = prm.nblk;
-  uint32_t *ctr_x = prm.ctr + MAX_MEM * team;              // then ctr_x[m]: helper m's partials
+  // members whose partial the owner adds: the core helpers, then the extra
+  const int mlast = prm.nmem - 1 + (prm.edev > 0 ? 1 : 0);
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < RS; ++s) { ptx::mbar_init(&bars->full[s], 1); ptx::mbar_init(&bars->empty[s], 1); }
@@ -164,30 +234,30 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
       // ============================ producer (each CTA stages its own halves)
       ptx::tma_prefetch(&prm.mapA);
       ptx::tma_prefetch(&prm.mapB);
-      uint32_t it = 0, gblk = 0, x_seen = 0;
-      for (int slab = team; slab < prm.nslab; slab += prm.nteams) {
-        const int64_t n0 = (int64_t)slab * PN + HB * rank;
-        const uint32_t gbase = gblk;
-        for (int i = 0; i < nblk; ++i, ++gblk) {
-          const int64_t r0 = blk_row(prm, i) + HA * rank;
-          for (uint32_t m = groups_of(prm, i, h); m; m &= m - 1) {
-            const int g = __ffs(m) - 1;
-            if (g > 0 && !(prm.dbg & 1)) {            // X of solved block g - 1 stored (both CTAs of member 0)
-              const uint32_t need = 2 * (gbase + g);
-              if (need > x_seen) {
-                wait_count(ctr_x, need);
-                asm volatile("fence.proxy.async.global;" ::: "memory");
-                x_seen = need;
-              }
+      uint32_t it = 0, x_seen[MAX_SERVE] = {};
+      for (int idx = 0; idx < role.nitems; ++idx) {
+        const Item e = item_of(prm, role, idx);
+        const uint32_t *ctr_x = prm.ctr + MAX_MEM * e.team;
+        if (e.i == 0) x_seen[e.j] = 0;
+        const int64_t n0 = (int64_t)e.slab * PN + HB * rank;
+        const int64_t r0 = blk_row(prm, e.i) + HA * rank;
+        for (uint32_t m = groups_of(prm, e.slab, e.i, e.h); m; m &= m - 1) {
+          const int g = __ffs(m) - 1;
+          if (g > 0 && !(prm.dbg & 1)) {              // X of solved block g - 1 stored (both CTAs of the owner)
+            const uint32_t need = 2 * (e.gbase + g);
+            if (need > x_seen[e.j]) {
+              wait_count(ctr_x, need);
+              asm volatile("fence.proxy.async.global;" ::: "memory");
+              x_seen[e.j] = need;
             }
-            const int64_t kg = blk_row(prm, g == 0 ? i : g - 1);
-            for (int w = 0; w < KB_BLK; ++w, ++it) {
-              const int rs = it % RS;
-              ptx::mbar_wait(&bars->empty[rs], ((it / RS) & 1) ^ 1);
-              ptx::mbar_arrive_expect_tx(&bars->full[rs], (HA + HB) * BK * 4);
-              load_op(&prm.mapA, prm.layA, raw[rs].A, r0, kg + w * BK, HA, &bars->full[rs]);
-              load_op(&prm.mapB, prm.layB, raw[rs].B, n0, kg + w * BK, HB, &bars->full[rs]);
-            }
+          }
+          const int64_t kg = blk_row(prm, g == 0 ? e.i : g - 1);
+          for (int w = 0; w < KB_BLK; ++w, ++it) {
+            const int rs = it % RS;
+            ptx::mbar_wait(&bars->empty[rs], ((it / RS) & 1) ^ 1);
+            ptx::mbar_arrive_expect_tx(&bars->full[rs], (HA + HB) * BK * 4);
+            load_op(&prm.mapA, prm.layA, raw[rs].A, r0, kg + w * BK, HA, &bars->full[rs]);
+            load_op(&prm.mapB, prm.layB, raw[rs].B, n0, kg + w * BK, HB, &bars->full[rs]);
           }
         }
       }
@@ -196,9 +266,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
       // ============================ MMA issuer (leader CTA)
       const uint32_t idesc = ptx::idesc_tf32(BLK, PN, prm.layA == LAYOUT_MN, prm.layB == LAYOUT_MN);
       uint32_t it = 0, cc = 0;
-      for (int slab = team; slab < prm.nslab; slab += prm.nteams) {
-        for (int i = 0; i < nblk; ++i) {
-          const int nkb = KB_BLK * __popc(groups_of(prm, i, h));
+      for (int idx = 0; idx < role.nitems; ++idx) {
+        {
+          const Item e = item_of(prm, role, idx);
+          const int i = e.i;
+          const int nkb = KB_BLK * __popc(groups_of(prm, e.slab, i, e.h));
           int left = 0;
           uint32_t acc = 0, buf = 0;
           for (int t = 0; t < nkb; ++t, ++it) {
@@ -212,8 +284,8 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
             const int rs = it % RS, ls = it % LS;
             ptx::mbar_wait_cluster(&bars->ready[ls], (it / LS) & 1);
             ptx::tc_fence_after();
-            if (lane == 0 && t == 0) ptrace(prm, h, i, 0);
-            if (lane == 0 && t == nkb - KB_BLK) ptrace(prm, h, i, 1);
+            if (lane == 0 && t == 0 && !role.extra) ptrace(prm, e.h, i, 0);
+            if (lane == 0 && t == nkb - KB_BLK && !role.extra) ptrace(prm, e.h, i, 1);
             if (lane == 0) {
               const uint32_t d = tmem + buf * PN;
               const uint32_t hiA = ptx::smem_u32(raw[rs].A), hiB = ptx::smem_u32(raw[rs].B);
@@ -250,9 +322,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
     BLAS3_DEC_REGS();
     const int tt = threadIdx.x - WARP_TR0 * 32;
     uint32_t it = 0;
-    for (int slab = team; slab < prm.nslab; slab += prm.nteams) {
-      for (int i = 0; i < nblk; ++i) {
-        const int nkb = KB_BLK * __popc(groups_of(prm, i, h));
+    for (int idx = 0; idx < role.nitems; ++idx) {
+      {
+        const Item e = item_of(prm, role, idx);
+        const int nkb = KB_BLK * __popc(groups_of(prm, e.slab, e.i, e.h));
         for (int t = 0; t < nkb; ++t, ++it) {
           const int rs = it % RS, ls = it % LS;
           ptx::mbar_wait(&bars->full[rs], (it / RS) & 1);
@@ -272,16 +345,19 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
     const int q = warp & 3, half = (warp - WARP_EPI0) >> 2;
     const bool lead = threadIdx.x == WARP_EPI0 * 32;
     const int rloc = q * 32 + lane;                           // row within this CTA's 128
-    uint32_t cc = 0, gblk = 0;
-    for (int slab = team; slab < prm.nslab; slab += prm.nteams) {
-      const int64_t c0 = (int64_t)slab * PN + half * NCOL;     // first right-hand side of this thread
-      for (int i = 0; i < nblk; ++i, ++gblk) {
-        const int nkb = KB_BLK * __popc(groups_of(prm, i, h));
+    uint32_t cc = 0;
+    for (int idx = 0; idx < role.nitems; ++idx) {
+      {
+        const Item e = item_of(prm, role, idx);
+        const int i = e.i, hh = e.h;
+        const uint32_t gblk = e.gblk;
+        uint32_t *ctr_x = prm.ctr + MAX_MEM * e.team;
+        const int64_t c0 = (int64_t)e.slab * PN + half * NCOL;   // first right-hand side of this thread
+        const int nkb = KB_BLK * __popc(groups_of(prm, e.slab, i, hh));
         const int nch = nkb > 0 ? (nkb + prm.kc - 1) / prm.kc : 0;
-        // this CTA's partial slot: [col][row] so a warp's accesses per column are one 128-B line
         // helper m's slot for this block: [col][row] (a warp's accesses per column are one 128-B line)
         auto slot = [&](int m) {
-          return prm.ws + (((((size_t)team * (MAX_MEM - 1) + (m - 1)) * 2 + (gblk & 1)) * 2 + rank) * PART_FLOATS) +
+          return prm.ws + (((((size_t)e.team * (MAX_MEM - 1) + (m - 1)) * 2 + (gblk & 1)) * 2 + rank) * PART_FLOATS) +
                  (size_t)(half * NCOL) * HA + rloc;
         };
         float S[NCOL];
@@ -289,10 +365,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
         for (int j = 0; j < NCOL; ++j) S[j] = 0.f;
         // member 0 adds the helper's partial (which runs ahead) while its MMA
         // works on the newest group: before waiting for that group's first chunk
-        const int cpart = h == 0 ? (nkb - KB_BLK) / prm.kc : -1;
+        const int cpart = hh == 0 ? (nkb - KB_BLK) / prm.kc : -1;
         for (int c = 0; c < nch; ++c, ++cc) {
           if (c == cpart) {
-            for (int m = 1; m < prm.nmem; ++m) {
+            for (int m = 1; m <= mlast; ++m) {
               if (lead) wait_count(ctr_x + m, 2 * (gblk + 1));
               ptx::named_bar_sync(5, EPI_THREADS);
               const float *part = slot(m);
@@ -318,16 +394,16 @@ __global__ void __launch_bounds__(NTHREADS, 1) trsm_panel_kernel(const __grid_co
           ptx::tc_fence_before();
           arrive_leader(&bars->tempty[buf], rank, 3, EPI_THREADS, lead);
         }
-        if (lead) ptrace(prm, h, i, 2);
-        if (h > 0) {
+        if (lead && !role.extra) ptrace(prm, hh, i, 2);
+        if (hh > 0) {
           // helper: the slot was last read for block gblk - 2 (X of it stored)
           if (lead && gblk >= 2) wait_count(ctr_x, 2 * (gblk - 1));
           ptx::named_bar_sync(5, EPI_THREADS);
-          float *part = slot(h);
+          float *part = slot(hh);
 #pragma unroll
           for (int j = 0; j < NCOL; ++j) __stcg(part + (size_t)j * HA, S[j]);
           ptx::named_bar_sync(5, EPI_THREADS);
-          if (lead) { __threadfence(); atomicAdd(ctr_x + h, 1u); ptrace(prm, h, i, 3); }
+          if (lead) { __threadfence(); atomicAdd(ctr_x + hh, 1u); if (!role.extra) ptrace(prm, hh, i, 3); }
           continue;
         }
         // member 0: X_i
@@ -425,25 +501,52 @@ static int device_sms() {
   }
   return v;
 }
-static void panel_shape(int64_t nrhs, int num_sms, int64_t &teams, int &nmem) {
+// extra members (BLAS3_PANEL_EXTRA=1; off by default: measured slower, see profiles/r02_strsm_panel.md): with one slab per team and
+// CTA pairs left over (N = 8192: 32 teams x 2 members = 64 of 74 pairs), each
+// leftover pair helps up to MAX_SERVE teams (extra e: slabs e, e + E, ...)
+static int panel_extra_on() {
+  static const int v = [] { const char *e = getenv("BLAS3_PANEL_EXTRA"); return e ? atoi(e) : 0; }();
+  return v;
+}
+struct PanelShape {
+  int64_t teams;                 // teams of this launch
+  int nmem;                      // core members per team
+  int tdev, edev;                // device-level teams and extras (fix the group split)
+  int nextra, fold;              // extras placed in this launch / folded into the last core member
+};
+static PanelShape panel_shape(int64_t nrhs, int num_sms) {
+  PanelShape sh{};
   const int64_t nslab = (nrhs + PN - 1) / PN, pairs = num_sms / 2, full = device_sms() / 2;
-  nmem = (int)imax(1, imin(panel_members(), full / imin(nslab, imax(1, full / 2))));
-  if (nmem > pairs) nmem = (int)imax(1, pairs);        // (a launch limit below one team)
-  teams = imin(nslab, imax(1, pairs / nmem));
+  const int nmem_dev = (int)imax(1, imin(panel_members(), full / imin(nslab, imax(1, full / 2))));
+  sh.nmem = nmem_dev;
+  if (sh.nmem > pairs) sh.nmem = (int)imax(1, pairs);  // (a launch limit below one team)
+  sh.teams = imin(nslab, imax(1, pairs / sh.nmem));
+  const int64_t tdev = imin(nslab, imax(1, full / nmem_dev));
+  int64_t edev = 0;
+  // (only where the machine could not give every team the preferred member
+  // count: a whole extra per team is a 4th member, measured slower at N = 4096)
+  if (panel_extra_on() && nslab == tdev && nmem_dev < panel_members() && nmem_dev + 1 <= MAX_MEM) {
+    edev = imin(tdev, full - tdev * nmem_dev);
+    if (edev > 0 && (tdev + edev - 1) / edev > MAX_SERVE) edev = 0;
+  }
+  sh.tdev = (int)tdev;
+  sh.edev = (int)edev;
+  const bool place = edev > 0 && sh.nmem == nmem_dev && sh.teams == tdev && pairs >= tdev * nmem_dev + edev;
+  sh.nextra = place ? (int)edev : 0;
+  sh.fold = edev > 0 && !place ? 1 : 0;
+  return sh;
 }
 size_t trsm_panel_ws_bytes(int64_t nrhs, int num_sms) {
-  int64_t t;
-  int m;
-  panel_shape(nrhs, num_sms, t, m);
+  const int64_t t = panel_shape(nrhs, num_sms).teams;
   return (size_t)t * (MAX_MEM - 1) * 4 * PART_FLOATS * sizeof(float) + (size_t)t * MAX_MEM * sizeof(uint32_t);
 }
 
 int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool right, int64_t R,
                       int64_t nrhs, bool forward, int kc, void *ws, cudaStream_t s, int num_sms) {
   if (R <= 0 || R % BLK || R / BLK > MAX_BLK || nrhs <= 0 || kc < 1 || !ws) return -1;
-  int64_t nteams;
-  int nmem;
-  panel_shape(nrhs, num_sms, nteams, nmem);
+  const PanelShape sh = panel_shape(nrhs, num_sms);
+  const int64_t nteams = sh.teams;
+  const int nmem = sh.nmem;
   if (nteams < 1) return -1;
   static PanelParams prm;
   static std::mutex mu;
@@ -478,21 +581,40 @@ int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool r
   // Member 0 is also charged its serial per-block hand-off (store, release,
   // reload of X_i), 0.3 of a group: kernel 187 / 189 us at N = 4096 / 8192
   // against 194 / 196 at 0.6 and 188 / 190 at 0 (profiles/r02_strsm_panel.md)
+  prm.tdev = sh.tdev;
+  prm.edev = sh.edev;
+  prm.nextra = sh.nextra;
+  prm.fold = sh.fold;
   const int64_t grp = 10, handoff = prm_handoff();
-  int64_t load[MAX_MEM] = {0, 0, 0, 0};
-  for (int i = 0; i < prm.nblk; ++i) {
-    uint32_t gm[MAX_MEM] = {0, 0, 0, 0};
-    gm[0] = 1u << i;
-    load[0] += grp + handoff;
-    for (int g = 0; g < i; ++g) {
-      int best = 0;
-      for (int m = nmem - 1; m >= 0; --m)
-        if (load[m] < load[best]) best = m;
-      if (nmem > 1 && best == 0 && load[nmem - 1] == load[0]) best = nmem - 1;
-      gm[best] |= 1u << g;
-      load[best] += grp;
+  for (int cls = 0; cls < 2; ++cls) {
+    // the extra (member nmem) serves w teams: a group costs it w times as much
+    static const int64_t xw = [] { const char *e = getenv("BLAS3_PANEL_XW"); return e ? atoll(e) : 0; }();
+    const int64_t w = sh.edev == 0 ? 0 : (cls == 0 ? (sh.tdev + sh.edev - 1) / sh.edev : sh.tdev / sh.edev) + xw;
+    const int mlast = nmem - 1 + (sh.edev > 0 ? 1 : 0);
+    int64_t load[MAX_MEM] = {0, 0, 0, 0};
+    for (int i = 0; i < prm.nblk; ++i) {
+      uint32_t gm[MAX_MEM] = {0, 0, 0, 0};
+      gm[0] = 1u << i;
+      load[0] += grp + handoff;
+      for (int g = 0; g < i; ++g) {
+        int best = 0;
+        if (sh.edev == 0) {
+          for (int m = nmem - 1; m >= 0; --m)
+            if (load[m] < load[best]) best = m;
+          if (nmem > 1 && best == 0 && load[nmem - 1] == load[0]) best = nmem - 1;
+        } else {
+          // least load after taking the group (ties to the later member: the
+          // extra takes the oldest groups, whose partials can run furthest ahead)
+          auto after = [&](int m) { return load[m] + grp * (m == nmem ? w : 1); };
+          best = mlast;
+          for (int m = mlast - 1; m >= 0; --m)
+            if (after(m) < after(best)) best = m;
+        }
+        gm[best] |= 1u << g;
+        load[best] += grp * (best == nmem && sh.edev > 0 ? w : 1);
+      }
+      for (int m = 0; m < MAX_MEM; ++m) prm.gmask[cls][i][m] = gm[m];
     }
-    for (int m = 0; m < MAX_MEM; ++m) prm.gmask[i][m] = gm[m];
   }
   static const int dbg = [] { const char *e = getenv("BLAS3_DEBUG_PANEL"); return e ? atoi(e) : 0; }();
   prm.dbg = dbg;
@@ -514,7 +636,7 @@ int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool r
   }
   if (cudaMemsetAsync(prm.ctr, 0, (size_t)nteams * MAX_MEM * sizeof(uint32_t), s) != cudaSuccess) return -1;
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)(2 * nmem * nteams));
+  cfg.gridDim = dim3((unsigned)(2 * (nmem * nteams + sh.nextra)));
   cfg.blockDim = dim3(NTHREADS);
   cfg.dynamicSmemBytes = SMEM;
   cfg.stream = s;
@@ -538,7 +660,7 @@ int launch_trsm_panel(const float *M, int64_t ldm, float *X, int64_t ldx, bool r
         const unsigned long long *r = hb + (hh * MAX_BLK + i) * 4;
         auto us = [&](unsigned long long v) { return v ? (double)(v - t0) / 1e3 : -1.0; };
         fprintf(stderr, "[panel] m%d blk %2d groups %2d: mma %7.2f newest %7.2f drained %7.2f released %7.2f\n", hh, i,
-                __builtin_popcount(prm.gmask[i][hh]), us(r[0]), us(r[1]),
+                __builtin_popcount(prm.gmask[0][i][hh]), us(r[0]), us(r[1]),
                 us(r[2]), us(r[3]));
       }
   }

@@ -210,4 +210,4 @@ def test_options_roundtrip_and_validation(lib):
     assert lib.get_option("max_sms") == 0
     assert lib.get_option("tc_c_async") == 0
     assert lib.get_option("trsm_panel") == 1
-    assert len(lib.OPTIONS) == 26
+    assert len(lib.OPTIONS) == 27

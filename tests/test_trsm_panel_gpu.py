@@ -144,3 +144,35 @@ def test_panel_solver_concurrent_streams(b3):
     torch.cuda.synchronize()
     for X, ref in zip(dX, seq):
         assert np.array_equal(to_host(X).view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.parametrize("side", "LR")
+def test_panel_solver_extra_members_fold_bitwise(b3, oracle_mod, side):
+    """8192 right-hand sides = 32 slabs: the full device gives each team two
+    core pairs and spreads the ten leftover pairs over the teams as extra
+    members (each helping three or four teams). A launch limited to 132 SMs
+    cannot place them; the last core member then computes the extra's partial
+    itself. The group split is the device's either way, so X is bit-identical."""
+    order, rhs = 1024, 8192
+    m, n = (order, rhs) if side == "L" else (rhs, order)
+    A = gen.triangular_dd(order, "U", "N", "px")
+    B = gen.uniform(m, n, "px-b")
+    X_full, l1 = solve(b3, side, "U", "N", "N", A, B)
+    X_lim, l2 = solve(b3, side, "U", "N", "N", A, B, max_sms=132)
+    assert l1 == 1 and l2 == 1
+    assert np.array_equal(X_full.view(np.uint32), X_lim.view(np.uint32))
+    check(oracle_mod, X_full, A, B, side, "U", "N", "N")
+
+
+@pytest.mark.parametrize("side,uplo,ta", [("L", "L", "N"), ("L", "U", "T"), ("R", "L", "N"), ("R", "U", "T")])
+def test_panel_solver_second_panel(b3, oracle_mod, side, uplo, ta):
+    """BLAS3_OPT_TRSM_PANEL2: order 6144 = three 2048 panels, forward or
+    backward; the first two processed panels by the solver (two launches),
+    the last by the doubling leaf, the update before the second in place."""
+    order, rhs = 6144, 520
+    m, n = (order, rhs) if side == "L" else (rhs, order)
+    A = gen.triangular_dd(order, uplo, "N", "p2")
+    B = gen.uniform(m, n, "p2-b")
+    X, launched = solve(b3, side, uplo, ta, "N", A, B, trsm_panel2=1)
+    assert launched == 2
+    check(oracle_mod, X, A, B, side, uplo, ta, "N")
