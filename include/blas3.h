@@ -171,6 +171,37 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
                 float alpha, const float *A, int64_t lda, float *B, int64_t ldb,
                 blas3_stream_t stream);
 
+/* ---- fp64 family (the paper is fp32-only).
+ * blas3_d{gemm,symm,syrk,syr2k,trmm,trsm}: the same semantics, argument
+ * lists, XERBLA codes, quick returns, alpha/beta special cases, ownership
+ * and stream rules as the s-routines above, on column-major fp64 matrices in
+ * device memory with host double scalars.  Arithmetic: IEEE fp64 FMA on the
+ * CUDA cores (one structured DFMA GEMM kernel, d_kernel.cu; the B200's FP64
+ * tensor rate is no higher than its DFMA rate), every product and sum in
+ * fp64; symmetric operands are mirrored and triangular ones zero-filled
+ * while staged to shared memory, as in the fp32 kernels.  DTRMM uses
+ * stream-ordered scratch of m*n doubles.  DTRSM scales B by alpha, then
+ * solves by recursive halving (diagonal blocks of 64 by substitution, GEMM
+ * updates).  Not affected by the math mode or the tuning options. */
+int blas3_dgemm(char transa, char transb, int64_t m, int64_t n, int64_t k,
+                double alpha, const double *A, int64_t lda, const double *B, int64_t ldb,
+                double beta, double *C, int64_t ldc, blas3_stream_t stream);
+int blas3_dsymm(char side, char uplo, int64_t m, int64_t n, double alpha,
+                const double *A, int64_t lda, const double *B, int64_t ldb,
+                double beta, double *C, int64_t ldc, blas3_stream_t stream);
+int blas3_dsyrk(char uplo, char trans, int64_t n, int64_t k, double alpha,
+                const double *A, int64_t lda, double beta, double *C, int64_t ldc,
+                blas3_stream_t stream);
+int blas3_dsyr2k(char uplo, char trans, int64_t n, int64_t k, double alpha,
+                 const double *A, int64_t lda, const double *B, int64_t ldb,
+                 double beta, double *C, int64_t ldc, blas3_stream_t stream);
+int blas3_dtrmm(char side, char uplo, char transa, char diag, int64_t m, int64_t n,
+                double alpha, const double *A, int64_t lda, double *B, int64_t ldb,
+                blas3_stream_t stream);
+int blas3_dtrsm(char side, char uplo, char transa, char diag, int64_t m, int64_t n,
+                double alpha, const double *A, int64_t lda, double *B, int64_t ldb,
+                blas3_stream_t stream);
+
 /* Process-wide math mode (BLAS3_MATH_3XTF32 default; the environment
  * variable BLAS3_MATH=simt|3xtf32|1xtf32|bf16x overrides the default at load).
  * Returns 0, or 1 if `mode` is not a valid mode (nothing changed). */

@@ -31,6 +31,7 @@ if not os.path.exists(LIB_PATH):
 _lib = ctypes.CDLL(LIB_PATH)
 
 _i64, _f, _p, _c, _i = ctypes.c_int64, ctypes.c_float, ctypes.c_void_p, ctypes.c_char, ctypes.c_int
+_d = ctypes.c_double
 
 _SIGS = {
     "blas3_sgemm": [_c, _c, _i64, _i64, _i64, _f, _p, _i64, _p, _i64, _f, _p, _i64, _p],
@@ -39,6 +40,12 @@ _SIGS = {
     "blas3_ssyr2k": [_c, _c, _i64, _i64, _f, _p, _i64, _p, _i64, _f, _p, _i64, _p],
     "blas3_strmm": [_c, _c, _c, _c, _i64, _i64, _f, _p, _i64, _p, _i64, _p],
     "blas3_strsm": [_c, _c, _c, _c, _i64, _i64, _f, _p, _i64, _p, _i64, _p],
+    "blas3_dgemm": [_c, _c, _i64, _i64, _i64, _d, _p, _i64, _p, _i64, _d, _p, _i64, _p],
+    "blas3_dsymm": [_c, _c, _i64, _i64, _d, _p, _i64, _p, _i64, _d, _p, _i64, _p],
+    "blas3_dsyrk": [_c, _c, _i64, _i64, _d, _p, _i64, _d, _p, _i64, _p],
+    "blas3_dsyr2k": [_c, _c, _i64, _i64, _d, _p, _i64, _p, _i64, _d, _p, _i64, _p],
+    "blas3_dtrmm": [_c, _c, _c, _c, _i64, _i64, _d, _p, _i64, _p, _i64, _p],
+    "blas3_dtrsm": [_c, _c, _c, _c, _i64, _i64, _d, _p, _i64, _p, _i64, _p],
     "blas3_sgemm_streamed": [_c, _c, _i64, _i64, _i64, _f, _p, _i64, _p, _i64, _f, _p, _i64, _p, _i64,
                              ctypes.c_uint32, _p],
     "blas3_signal": [_p, ctypes.c_uint32, _p],
@@ -81,13 +88,14 @@ def _ch(x):
 
 
 # ----------------------------------------------------------------- tensor helpers
-def _mat(X, name):
-    """(pointer, rows, cols, ld) of a column-major fp32 CUDA tensor view."""
+def _mat(X, name, f64=False):
+    """(pointer, rows, cols, ld) of a column-major fp32 (fp64) CUDA tensor view."""
     import torch
     if not isinstance(X, torch.Tensor):
         raise TypeError(f"{name} must be a torch.Tensor")
-    if X.dtype != torch.float32 or not X.is_cuda or X.dim() != 2:
-        raise TypeError(f"{name} must be a 2-D float32 CUDA tensor")
+    dt = torch.float64 if f64 else torch.float32
+    if X.dtype != dt or not X.is_cuda or X.dim() != 2:
+        raise TypeError(f"{name} must be a 2-D {str(dt)[6:]} CUDA tensor")
     m, n = X.shape
     if m > 1 and X.stride(0) != 1:
         raise ValueError(f"{name} must be column-major (stride(0) == 1)")
@@ -100,22 +108,22 @@ def _stream():
     return torch.cuda.current_stream().cuda_stream
 
 
-def colmajor(m, n, ld=None, device="cuda", fill=None):
-    """Allocate an m x n column-major fp32 tensor (strides (1, ld))."""
+def colmajor(m, n, ld=None, device="cuda", fill=None, dtype=None):
+    """Allocate an m x n column-major fp32 (or `dtype`) tensor (strides (1, ld))."""
     import torch
     ld = max(1, m) if ld is None else ld
-    buf = torch.empty((n, ld), dtype=torch.float32, device=device)
+    buf = torch.empty((n, ld), dtype=torch.float32 if dtype is None else dtype, device=device)
     if fill is not None:
         buf.fill_(fill)
     return buf.t()[:m]
 
 
-def from_fortran(arr, device="cuda"):
+def from_fortran(arr, device="cuda", f64=False):
     """Copy a numpy Fortran-ordered (ld x n) buffer to a column-major device
-    tensor with the same ld; returns the full (ld x n) view."""
+    tensor with the same ld; returns the full (ld x n) view (fp32, or fp64)."""
     import numpy as np
     import torch
-    a = np.asfortranarray(arr, dtype=np.float32)
+    a = np.asfortranarray(arr, dtype=np.float64 if f64 else np.float32)
     t = torch.from_numpy(a.T.copy()).to(device)     # (n, ld) row-major == (ld, n) col-major
     return t.t()
 
@@ -135,16 +143,26 @@ def _t(c):
     return c.upper() != "N" if isinstance(c, str) else c.upper() != b"N"
 
 
-def sgemm(transa, transb, alpha, A, B, beta, C):
-    """C <- alpha*op(A)*op(B) + beta*C (GEMM-NN/-TN, P:77, P:392)."""
-    pc, m, n, ldc = _mat(C, "C")
-    pa, ar, ac, lda = _mat(A, "A")
-    pb, br, bc, ldb = _mat(B, "B")
+def _gemm(f64, transa, transb, alpha, A, B, beta, C):
+    pc, m, n, ldc = _mat(C, "C", f64)
+    pa, ar, ac, lda = _mat(A, "A", f64)
+    pb, br, bc, ldb = _mat(B, "B", f64)
     k = ac if not _t(transa) else ar
     _need("A", A, *((k, m) if _t(transa) else (m, k)))
     _need("B", B, *((n, k) if _t(transb) else (k, n)))
-    _chk("blas3_sgemm", blas3_sgemm(_ch(transa), _ch(transb), m, n, k, alpha, pa, lda, pb, ldb,  # noqa: F821
-                                    beta, pc, ldc, _stream()))
+    name = "blas3_dgemm" if f64 else "blas3_sgemm"
+    _chk(name, globals()[name](_ch(transa), _ch(transb), m, n, k, alpha, pa, lda, pb, ldb, beta, pc, ldc,
+                               _stream()))
+
+
+def sgemm(transa, transb, alpha, A, B, beta, C):
+    """C <- alpha*op(A)*op(B) + beta*C (GEMM-NN/-TN, P:77, P:392)."""
+    _gemm(False, transa, transb, alpha, A, B, beta, C)
+
+
+def dgemm(transa, transb, alpha, A, B, beta, C):
+    """fp64 GEMM (F4): C <- alpha*op(A)*op(B) + beta*C on float64 tensors."""
+    _gemm(True, transa, transb, alpha, A, B, beta, C)
 
 
 def sgemm_streamed(transa, transb, alpha, A, B, beta, C, ready, panel_k, value):
@@ -173,64 +191,101 @@ def signal(ready, index, value):
                                       _stream()))
 
 
-def ssymm(side, uplo, alpha, A, B, beta, C):
-    """side=L: C <- alpha*A*B + beta*C; side=R: C <- alpha*B*A + beta*C."""
-    pc, m, n, ldc = _mat(C, "C")
-    pa, _, _, lda = _mat(A, "A")
-    pb, _, _, ldb = _mat(B, "B")
+def _symm(f64, side, uplo, alpha, A, B, beta, C):
+    pc, m, n, ldc = _mat(C, "C", f64)
+    pa, _, _, lda = _mat(A, "A", f64)
+    pb, _, _, ldb = _mat(B, "B", f64)
     ka = m if (side.upper() if isinstance(side, str) else side.decode().upper()) == "L" else n
     _need("A", A, ka, ka)
     _need("B", B, m, n)
-    _chk("blas3_ssymm", blas3_ssymm(_ch(side), _ch(uplo), m, n, alpha, pa, lda, pb, ldb,  # noqa: F821
-                                    beta, pc, ldc, _stream()))
+    name = "blas3_dsymm" if f64 else "blas3_ssymm"
+    _chk(name, globals()[name](_ch(side), _ch(uplo), m, n, alpha, pa, lda, pb, ldb, beta, pc, ldc, _stream()))
+
+
+def ssymm(side, uplo, alpha, A, B, beta, C):
+    """side=L: C <- alpha*A*B + beta*C; side=R: C <- alpha*B*A + beta*C."""
+    _symm(False, side, uplo, alpha, A, B, beta, C)
+
+
+def dsymm(side, uplo, alpha, A, B, beta, C):
+    """fp64 SYMM (F4)."""
+    _symm(True, side, uplo, alpha, A, B, beta, C)
+
+
+def _syrk(f64, uplo, trans, alpha, A, beta, C):
+    pc, n, _, ldc = _mat(C, "C", f64)
+    pa, ar, ac, lda = _mat(A, "A", f64)
+    k = ac if not _t(trans) else ar
+    _need("C", C, n, n)
+    _need("A", A, *((k, n) if _t(trans) else (n, k)))
+    name = "blas3_dsyrk" if f64 else "blas3_ssyrk"
+    _chk(name, globals()[name](_ch(uplo), _ch(trans), n, k, alpha, pa, lda, beta, pc, ldc, _stream()))
 
 
 def ssyrk(uplo, trans, alpha, A, beta, C):
     """C <- alpha*op(A)*op(A)^T + beta*C on the uplo triangle."""
-    pc, n, _, ldc = _mat(C, "C")
-    pa, ar, ac, lda = _mat(A, "A")
-    k = ac if not _t(trans) else ar
-    _need("C", C, n, n)
-    _need("A", A, *((k, n) if _t(trans) else (n, k)))
-    _chk("blas3_ssyrk", blas3_ssyrk(_ch(uplo), _ch(trans), n, k, alpha, pa, lda, beta, pc, ldc,  # noqa: F821
-                                    _stream()))
+    _syrk(False, uplo, trans, alpha, A, beta, C)
 
 
-def ssyr2k(uplo, trans, alpha, A, B, beta, C):
-    """C <- alpha*(op(A)op(B)^T + op(B)op(A)^T) + beta*C on the uplo triangle."""
-    pc, n, _, ldc = _mat(C, "C")
-    pa, ar, ac, lda = _mat(A, "A")
-    pb, _, _, ldb = _mat(B, "B")
+def dsyrk(uplo, trans, alpha, A, beta, C):
+    """fp64 SYRK (F4)."""
+    _syrk(True, uplo, trans, alpha, A, beta, C)
+
+
+def _syr2k(f64, uplo, trans, alpha, A, B, beta, C):
+    pc, n, _, ldc = _mat(C, "C", f64)
+    pa, ar, ac, lda = _mat(A, "A", f64)
+    pb, _, _, ldb = _mat(B, "B", f64)
     k = ac if not _t(trans) else ar
     _need("C", C, n, n)
     _need("A", A, *((k, n) if _t(trans) else (n, k)))
     _need("B", B, *((k, n) if _t(trans) else (n, k)))
-    _chk("blas3_ssyr2k", blas3_ssyr2k(_ch(uplo), _ch(trans), n, k, alpha, pa, lda, pb, ldb,  # noqa: F821
-                                      beta, pc, ldc, _stream()))
+    name = "blas3_dsyr2k" if f64 else "blas3_ssyr2k"
+    _chk(name, globals()[name](_ch(uplo), _ch(trans), n, k, alpha, pa, lda, pb, ldb, beta, pc, ldc, _stream()))
+
+
+def ssyr2k(uplo, trans, alpha, A, B, beta, C):
+    """C <- alpha*(op(A)op(B)^T + op(B)op(A)^T) + beta*C on the uplo triangle."""
+    _syr2k(False, uplo, trans, alpha, A, B, beta, C)
+
+
+def dsyr2k(uplo, trans, alpha, A, B, beta, C):
+    """fp64 SYR2K (F4)."""
+    _syr2k(True, uplo, trans, alpha, A, B, beta, C)
 
 
 def _order(side, m, n):
     return m if (side.upper() if isinstance(side, str) else side.decode().upper()) == "L" else n
 
 
-def strmm(side, uplo, transa, diag, alpha, A, B):
-    """B <- alpha*op(A)*B (L) or alpha*B*op(A) (R), in place."""
-    pb, m, n, ldb = _mat(B, "B")
-    pa, _, _, lda = _mat(A, "A")
+def _tr(f64, solve, side, uplo, transa, diag, alpha, A, B):
+    pb, m, n, ldb = _mat(B, "B", f64)
+    pa, _, _, lda = _mat(A, "A", f64)
     ka = _order(side, m, n)
     _need("A", A, ka, ka)
-    _chk("blas3_strmm", blas3_strmm(_ch(side), _ch(uplo), _ch(transa), _ch(diag), m, n, alpha,  # noqa: F821
-                                    pa, lda, pb, ldb, _stream()))
+    name = "blas3_" + ("d" if f64 else "s") + ("trsm" if solve else "trmm")
+    _chk(name, globals()[name](_ch(side), _ch(uplo), _ch(transa), _ch(diag), m, n, alpha, pa, lda, pb, ldb,
+                               _stream()))
+
+
+def strmm(side, uplo, transa, diag, alpha, A, B):
+    """B <- alpha*op(A)*B (L) or alpha*B*op(A) (R), in place."""
+    _tr(False, False, side, uplo, transa, diag, alpha, A, B)
 
 
 def strsm(side, uplo, transa, diag, alpha, A, B):
     """Solve op(A)X = alpha*B (L) or X op(A) = alpha*B (R); X overwrites B."""
-    pb, m, n, ldb = _mat(B, "B")
-    pa, _, _, lda = _mat(A, "A")
-    ka = _order(side, m, n)
-    _need("A", A, ka, ka)
-    _chk("blas3_strsm", blas3_strsm(_ch(side), _ch(uplo), _ch(transa), _ch(diag), m, n, alpha,  # noqa: F821
-                                    pa, lda, pb, ldb, _stream()))
+    _tr(False, True, side, uplo, transa, diag, alpha, A, B)
+
+
+def dtrmm(side, uplo, transa, diag, alpha, A, B):
+    """fp64 TRMM (F4), in place."""
+    _tr(True, False, side, uplo, transa, diag, alpha, A, B)
+
+
+def dtrsm(side, uplo, transa, diag, alpha, A, B):
+    """fp64 TRSM (F4); X overwrites B."""
+    _tr(True, True, side, uplo, transa, diag, alpha, A, B)
 
 
 def set_math_mode(mode):

@@ -14,6 +14,7 @@
 
 #include "../../include/blas3.h"
 #include "kernels.h"
+#include "validate.h"
 
 namespace blas3 {
 
@@ -148,6 +149,8 @@ static int device_check(int &sms) {
   return di.ok ? 0 : BLAS3_ERR_ARCH;
 }
 
+int abi_device_check(int &sms) { return device_check(sms); }
+
 // stream-ordered scratch: caller-provided workspace first, else the pool
 struct Scratch {
   float *p = nullptr;
@@ -217,12 +220,6 @@ static int gemm_dense(int64_t M, int64_t N, int64_t K, float alpha, const float 
   return run_problem(P, s, sms);
 }
 
-static inline int up(char c) { return toupper((unsigned char)c); }
-static inline bool is_trans(char c) { int u = up(c); return u == 'N' || u == 'T' || u == 'C'; }
-static inline bool is_side(char c) { int u = up(c); return u == 'L' || u == 'R'; }
-static inline bool is_uplo(char c) { int u = up(c); return u == 'L' || u == 'U'; }
-static inline bool is_diag(char c) { int u = up(c); return u == 'N' || u == 'U'; }
-static inline int64_t mx1(int64_t v) { return v > 1 ? v : 1; }
 
 static inline int finish(int rc) {
   if (rc) return rc;
@@ -298,14 +295,7 @@ int blas3_sgemm(char transa, char transb, int64_t m, int64_t n, int64_t k, float
                 int64_t ldc, blas3_stream_t stream) {
   CallOpts call_opts;
   const bool ta = up(transa) != 'N', tb = up(transb) != 'N';
-  if (!is_trans(transa)) return 1;
-  if (!is_trans(transb)) return 2;
-  if (m < 0) return 3;
-  if (n < 0) return 4;
-  if (k < 0) return 5;
-  if (lda < mx1(ta ? k : m)) return 8;
-  if (ldb < mx1(tb ? n : k)) return 10;
-  if (ldc < mx1(m)) return 13;
+  if (const int v = v_gemm(transa, transb, m, n, k, lda, ldb, ldc)) return v;
   if (m == 0 || n == 0 || ((alpha == 0.f || k == 0) && beta == 1.f)) return 0;
   if (!C) return 12;
   const bool reads_ab = alpha != 0.f && k > 0;
@@ -380,13 +370,7 @@ int blas3_ssymm(char side, char uplo, int64_t m, int64_t n, float alpha, const f
                 blas3_stream_t stream) {
   CallOpts call_opts;
   const bool left = up(side) == 'L', lower = up(uplo) == 'L';
-  if (!is_side(side)) return 1;
-  if (!is_uplo(uplo)) return 2;
-  if (m < 0) return 3;
-  if (n < 0) return 4;
-  if (lda < mx1(left ? m : n)) return 7;
-  if (ldb < mx1(m)) return 9;
-  if (ldc < mx1(m)) return 12;
+  if (const int v = v_symm(side, uplo, m, n, lda, ldb, ldc)) return v;
   if (m == 0 || n == 0 || (alpha == 0.f && beta == 1.f)) return 0;
   if (!C) return 11;
   if (alpha != 0.f && !A) return 6;
@@ -454,13 +438,7 @@ static int syrk_common(bool two, char uplo, char trans, int64_t n, int64_t k, fl
 
 int blas3_ssyrk(char uplo, char trans, int64_t n, int64_t k, float alpha, const float *A,
                 int64_t lda, float beta, float *C, int64_t ldc, blas3_stream_t stream) {
-  const bool ta = up(trans) != 'N';
-  if (!is_uplo(uplo)) return 1;
-  if (!is_trans(trans)) return 2;
-  if (n < 0) return 3;
-  if (k < 0) return 4;
-  if (lda < mx1(ta ? k : n)) return 7;
-  if (ldc < mx1(n)) return 10;
+  if (const int v = v_syrk(false, uplo, trans, n, k, lda, 0, ldc)) return v;
   return syrk_common(false, uplo, trans, n, k, alpha, A, lda, nullptr, 0, beta, C, ldc,
                      (cudaStream_t)stream);
 }
@@ -468,14 +446,7 @@ int blas3_ssyrk(char uplo, char trans, int64_t n, int64_t k, float alpha, const 
 int blas3_ssyr2k(char uplo, char trans, int64_t n, int64_t k, float alpha, const float *A,
                  int64_t lda, const float *B, int64_t ldb, float beta, float *C, int64_t ldc,
                  blas3_stream_t stream) {
-  const bool ta = up(trans) != 'N';
-  if (!is_uplo(uplo)) return 1;
-  if (!is_trans(trans)) return 2;
-  if (n < 0) return 3;
-  if (k < 0) return 4;
-  if (lda < mx1(ta ? k : n)) return 7;
-  if (ldb < mx1(ta ? k : n)) return 9;
-  if (ldc < mx1(n)) return 12;
+  if (const int v = v_syrk(true, uplo, trans, n, k, lda, ldb, ldc)) return v;
   return syrk_common(true, uplo, trans, n, k, alpha, A, lda, B, ldb, beta, C, ldc,
                      (cudaStream_t)stream);
 }
@@ -483,15 +454,7 @@ int blas3_ssyr2k(char uplo, char trans, int64_t n, int64_t k, float alpha, const
 // ------------------------------------------------------------------- STRMM / STRSM validation
 static int tr_validate(char side, char uplo, char transa, char diag, int64_t m, int64_t n,
                        int64_t lda, int64_t ldb) {
-  if (!is_side(side)) return 1;
-  if (!is_uplo(uplo)) return 2;
-  if (!is_trans(transa)) return 3;
-  if (!is_diag(diag)) return 4;
-  if (m < 0) return 5;
-  if (n < 0) return 6;
-  if (lda < mx1(up(side) == 'L' ? m : n)) return 9;
-  if (ldb < mx1(m)) return 11;
-  return 0;
+  return v_tr(side, uplo, transa, diag, m, n, lda, ldb);
 }
 
 // ------------------------------------------------------------------- STRMM (row A9)

@@ -1,0 +1,324 @@
+// d_kernel.cu -- the fp64 family ("DGEMM family"): one
+// structured FP64 GEMM kernel on the CUDA cores (DFMA) that every D routine
+// derives from, plus the triangular-solve diagonal-block kernel.
+//
+// The paper's method carried over unchanged to double precision
+// (PAPER.md P:93-99 SM_alloc(X, Symmetry), P:197-210 padding/peel_triangular,
+// P:225-244 Adaptor_Solver): symmetric operands are MIRRORED and triangular
+// ones ZERO-FILLED (unit diagonal written) while a tile is staged to shared
+// memory, blank triangular k-blocks are skipped through the tile's k-range,
+// only the uplo triangle of C is written for SYRK/SYR2K, and TRSM is a blocked
+// diagonal-block solve followed by GEMM updates (d_abi.cu).
+//
+// Why CUDA cores: on B200 the FP64 tensor-core rate equals the FP64 FMA rate
+// (~40 TFLOP/s nominal, blackwell_cuda_programming.md), and DFMA keeps every
+// product and sum in IEEE fp64 (the oracle's precision), so a register-tiled
+// DFMA kernel is the direct route.  Roofline: DFMA-bound, 64 FMA/clk/SM.
+//
+// Kernel: 256 threads, C tile 128 x 128, BK = 16 k-blocks staged through
+// registers into double-buffered shared memory (the structure select happens
+// on the way), 8 x 8 outputs per thread (rows tr + 16 i, columns 4 tc + 64 g
+// + j, so a warp's C accesses are 128-B runs of one column and its B reads
+// two broadcast 32-B groups).
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <atomic>
+
+#include "kernels.h"
+#include "d_kernels.h"
+
+namespace blas3 {
+namespace {
+
+constexpr int DTM = 128, DTN = 128, DBK = 16, DTHREADS = 256;
+constexpr int DAP = DTM + 2, DBP = DTN + 2;          // padded shared rows (doubles)
+constexpr int DJ = 8;                                // columns per thread (two groups of 4)
+constexpr int DNB = 64;                              // TRSM diagonal block
+
+// X(r, k) of an operand: the logical matrix L = stored (dense), sym(stored
+// triangle) or tri(stored triangle, unit diagonal, blank = 0), viewed
+// transposed when trans, at offsets (ro, ko) of the X index space.
+__device__ __forceinline__ double dfetch(const DOpnd &o, int64_t r, int64_t k) {
+  const int64_t i = o.trans ? k + o.ko : r + o.ro;
+  const int64_t j = o.trans ? r + o.ro : k + o.ko;
+  if (o.kind == DOP_DENSE) return __ldg(o.p + i + j * o.ld);
+  const bool stored = o.lower ? (i >= j) : (i <= j);
+  if (o.kind == DOP_SYM) return stored ? __ldg(o.p + i + j * o.ld) : __ldg(o.p + j + i * o.ld);
+  if (!stored) return 0.0;                           // the blank triangle is never read
+  if (i == j && o.unit) return 1.0;                  // unit diagonal: the stored value is not read
+  return __ldg(o.p + i + j * o.ld);
+}
+
+// Is the (rows [r0, r1) x k [k0, k1)) block of X read contiguously along r?
+// Dense / tri: the stored orientation (i = r unless trans).  Sym: the stored
+// orientation where the block lies in the stored triangle, the mirrored one
+// where it lies in the other (diagonal-crossing blocks: either).
+__device__ __forceinline__ bool rfast(const DOpnd &o, int64_t r0, int64_t r1, int64_t k0, int64_t k1) {
+  if (o.kind != DOP_SYM) return !o.trans;
+  // i-range and j-range of the block in L
+  const int64_t i0 = o.trans ? k0 + o.ko : r0 + o.ro, i1 = o.trans ? k1 + o.ko : r1 + o.ro;
+  const int64_t j0 = o.trans ? r0 + o.ro : k0 + o.ko, j1 = o.trans ? r1 + o.ro : k1 + o.ko;
+  const bool all_stored = o.lower ? (i0 >= j1 - 1) : (i1 - 1 <= j0);
+  const bool all_mirror = o.lower ? (i1 - 1 < j0) : (i0 > j1 - 1);
+  // stored: address i + j ld, contiguous in i; mirrored: j + i ld, contiguous in j
+  const bool contig_i = all_stored || !all_mirror;
+  return contig_i ? !o.trans : o.trans;
+}
+
+// k-range of X's nonzeros for the rows [r0, r1) (blank triangle skipped)
+__device__ __forceinline__ void krange(const DOpnd &o, int64_t r0, int64_t r1, int64_t K, int64_t &klo,
+                                       int64_t &khi) {
+  if (o.kind != DOP_TRI) return;
+  const int64_t d = o.ro - o.ko;
+  // nonzero iff (lower != trans) ? k <= r + d : k >= r + d
+  if (o.lower != (o.trans != 0)) khi = khi < r1 + d ? khi : r1 + d;
+  else klo = klo > r0 + d ? klo : r0 + d;
+  if (khi > K) khi = K;
+  if (klo < 0) klo = 0;
+}
+
+// One operand tile (ROWS x DBK) of X into registers: element e = tid + 256 q,
+// (r, k) = r-fastest or k-fastest by the block's contiguous direction.
+template <int ROWS>
+struct TileLoad {
+  static constexpr int PER = ROWS * DBK / DTHREADS;
+  double v[PER];
+  // strided block X(r, k) = base[r * si + k * sk]
+  __device__ __forceinline__ void load_strided(const double *base, int64_t si, int64_t sk, int64_t r0, int64_t rmax,
+                                               int64_t k0, int64_t kmax, bool rf) {
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      const int e = threadIdx.x + DTHREADS * q;
+      const int r = rf ? e % ROWS : e / DBK, k = rf ? e / ROWS : e % DBK;
+      v[q] = (r0 + r < rmax && k0 + k < kmax) ? __ldg(base + r * si + k * sk) : 0.0;
+    }
+  }
+  // The block's region class decides the access (Adaptor_Symmetry /
+  // Adaptor_Triangular): REAL (inside the stored
+  // triangle: plain strided loads), SHADOW (SYM, the other triangle: the
+  // mirrored strided loads), BLANK (TRI outside the triangle: zeros, nothing
+  // read), DIAGONAL-CROSSING (per-element select, dfetch).
+  __device__ __forceinline__ void load(const DOpnd &o, int64_t r0, int64_t rmax, int64_t k0, int64_t kmax,
+                                       bool rf) {
+    // X(r, k) = p[i + j ld], (i, j) = trans ? (k + ko, r + ro) : (r + ro, k + ko)
+    const int64_t si = o.trans ? o.ld : 1, sk = o.trans ? 1 : o.ld;
+    if (o.kind == DOP_DENSE) {
+      load_strided(o.p + r0 * si + k0 * sk, si, sk, r0, rmax, k0, kmax, rf);
+      return;
+    }
+    const int64_t i0 = o.trans ? k0 + o.ko : r0 + o.ro, i1 = i0 + (o.trans ? DBK : ROWS) - 1;
+    const int64_t j0 = o.trans ? r0 + o.ro : k0 + o.ko, j1 = j0 + (o.trans ? ROWS : DBK) - 1;
+    const bool real = o.lower ? (i0 > j1) : (i1 < j0);            // strictly inside: no diagonal
+    const bool other = o.lower ? (i1 < j0) : (i0 > j1);
+    if (real) {
+      load_strided(o.p + (r0 + o.ro) * si + (k0 + o.ko) * sk, si, sk, r0, rmax, k0, kmax, rf);
+      return;
+    }
+    if (other && o.kind == DOP_TRI) {
+#pragma unroll
+      for (int q = 0; q < PER; ++q) v[q] = 0.0;
+      return;
+    }
+    if (other) {                                                   // SYM shadow: L(i, j) = p[j + i ld]
+      load_strided(o.p + (r0 + o.ro) * sk + (k0 + o.ko) * si, sk, si, r0, rmax, k0, kmax, rf);
+      return;
+    }
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      const int e = threadIdx.x + DTHREADS * q;
+      const int r = rf ? e % ROWS : e / DBK, k = rf ? e / ROWS : e % DBK;
+      v[q] = (r0 + r < rmax && k0 + k < kmax) ? dfetch(o, r0 + r, k0 + k) : 0.0;
+    }
+  }
+  template <int LD>
+  __device__ __forceinline__ void store(double *s, bool rf) const {
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      const int e = threadIdx.x + DTHREADS * q;
+      const int r = rf ? e % ROWS : e / DBK, k = rf ? e / ROWS : e % DBK;
+      s[k * LD + r] = v[q];
+    }
+  }
+};
+
+constexpr size_t DSMEM = 2 * DBK * (DAP + DBP) * sizeof(double);   // 66560 B (dynamic)
+
+__global__ void __launch_bounds__(DTHREADS, 1) dgemm_structured(const __grid_constant__ DProblem P) {
+  extern __shared__ double dsm[];
+  // buffers by integer offset from the __shared__ array (not through a
+  // pointer table, which would turn every access into a generic LD/ST)
+  constexpr int AOFF = DBK * DAP, BOFF0 = 2 * DBK * DAP, BOFF = DBK * DBP;
+  const int64_t tiles_n = (P.N + DTN - 1) / DTN;
+  const int64_t tm = blockIdx.x / tiles_n, tn = blockIdx.x % tiles_n;
+  const int64_t m0 = tm * DTM, n0 = tn * DTN;
+  // SYRK / SYR2K: tiles wholly outside the uplo triangle of C do nothing
+  if (P.ctri == 1 && m0 + DTM - 1 < n0) return;
+  if (P.ctri == 2 && m0 > n0 + DTN - 1) return;
+  const int tr = threadIdx.x % 16, tc = threadIdx.x / 16;
+  double acc[8][DJ];
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < DJ; ++j) acc[i][j] = 0.0;
+
+  for (int sg = 0; sg < P.nseg; ++sg) {
+    const DSeg &S = P.seg[sg];
+    int64_t klo = 0, khi = S.K;
+    krange(S.a, m0, m0 + DTM, S.K, klo, khi);
+    krange(S.b, n0, n0 + DTN, S.K, klo, khi);
+    if (klo >= khi) continue;
+    klo = klo / DBK * DBK;                            // k-blocks aligned to BK
+    const int64_t nkb = (khi - klo + DBK - 1) / DBK;
+    TileLoad<DTM> la;
+    TileLoad<DTN> lb;
+    bool rfa = rfast(S.a, m0, m0 + DTM, klo, klo + DBK), rfb = rfast(S.b, n0, n0 + DTN, klo, klo + DBK);
+    la.load(S.a, m0, P.M, klo, khi, rfa);
+    lb.load(S.b, n0, P.N, klo, khi, rfb);
+    __syncthreads();                                   // previous segment's reads of the buffers
+    la.store<DAP>(dsm, rfa);
+    lb.store<DBP>(dsm + BOFF0, rfb);
+    __syncthreads();
+    for (int64_t t = 0; t < nkb; ++t) {
+      const int cur = (int)(t & 1);
+      const int64_t kn = klo + (t + 1) * DBK;
+      if (t + 1 < nkb) {                               // next k-block into registers
+        rfa = rfast(S.a, m0, m0 + DTM, kn, kn + DBK);
+        rfb = rfast(S.b, n0, n0 + DTN, kn, kn + DBK);
+        la.load(S.a, m0, P.M, kn, khi, rfa);
+        lb.load(S.b, n0, P.N, kn, khi, rfb);
+      }
+      const double *as = dsm + cur * AOFF, *bs = dsm + BOFF0 + cur * BOFF;
+#pragma unroll
+      for (int k = 0; k < DBK; ++k) {
+        double a[8], b[DJ];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) a[i] = as[k * DAP + tr + 16 * i];
+#pragma unroll
+        for (int g = 0; g < DJ / 4; ++g) {             // columns 4 tc + 64 g + 0..3
+          const double2 b01 = *reinterpret_cast<const double2 *>(bs + k * DBP + 4 * tc + 64 * g);
+          const double2 b23 = *reinterpret_cast<const double2 *>(bs + k * DBP + 4 * tc + 64 * g + 2);
+          b[4 * g] = b01.x; b[4 * g + 1] = b01.y; b[4 * g + 2] = b23.x; b[4 * g + 3] = b23.y;
+        }
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j < DJ; ++j) acc[i][j] = fma(a[i], b[j], acc[i][j]);
+      }
+      if (t + 1 < nkb) {
+        la.store<DAP>(dsm + (cur ^ 1) * AOFF, rfa);
+        lb.store<DBP>(dsm + BOFF0 + (cur ^ 1) * BOFF, rfb);
+      }
+      __syncthreads();
+    }
+  }
+  // epilogue: D = alpha * acc + beta * C (C not read when beta == 0), uplo mask
+#pragma unroll
+  for (int j = 0; j < DJ; ++j) {
+    const int64_t c = n0 + 4 * tc + 64 * (j / 4) + j % 4;
+    if (c >= P.N) continue;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int64_t r = m0 + tr + 16 * i;
+      if (r >= P.M) continue;
+      if (P.ctri == 1 && r < c) continue;
+      if (P.ctri == 2 && r > c) continue;
+      double v = P.alpha * acc[i][j];
+      if (P.beta != 0.0) v = fma(P.beta, P.C[r + c * P.ldc], v);
+      P.D[r + c * P.ldd] = v;
+    }
+  }
+}
+
+// Diagonal block of a triangular solve: for every right-hand side (one per
+// thread) solve S y = rhs in place, S = nb x nb (nb <= DNB) from the TRI
+// operand (forward if S is lower, else backward), padded to DNB with the
+// identity.  rhs element i of right-hand side c: X[i * sx + c * sc].
+__global__ void __launch_bounds__(64) dtrsm_diag(const __grid_constant__ DOpnd S, int nb, double *X, int64_t sx,
+                                                 int64_t sc, int64_t nrhs) {
+  __shared__ double Ss[DNB * (DNB + 1)];
+  for (int e = threadIdx.x; e < DNB * DNB; e += blockDim.x) {
+    const int i = e % DNB, j = e / DNB;
+    Ss[i + j * (DNB + 1)] = (i < nb && j < nb) ? dfetch(S, i, j) : (i == j ? 1.0 : 0.0);
+  }
+  __syncthreads();
+  const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= nrhs) return;
+  double y[DNB];
+#pragma unroll
+  for (int i = 0; i < DNB; ++i) y[i] = i < nb ? X[i * sx + c * sc] : 0.0;
+  // S lower <=> nonzeros at i >= j of the logical (i, j) = (r, k)
+  const bool lower = S.lower != (S.trans != 0);
+  if (lower) {
+#pragma unroll
+    for (int i = 0; i < DNB; ++i) {
+      double v = y[i];
+#pragma unroll
+      for (int j = 0; j < i; ++j) v = fma(-Ss[i + j * (DNB + 1)], y[j], v);
+      y[i] = v / Ss[i + i * (DNB + 1)];
+    }
+  } else {
+#pragma unroll
+    for (int i = DNB - 1; i >= 0; --i) {
+      double v = y[i];
+#pragma unroll
+      for (int j = i + 1; j < DNB; ++j) v = fma(-Ss[i + j * (DNB + 1)], y[j], v);
+      y[i] = v / Ss[i + i * (DNB + 1)];
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < DNB; ++i)
+    if (i < nb) X[i * sx + c * sc] = y[i];
+}
+
+// C <- beta * C on the m x n block (tri: 0 all, 1 lower, 2 upper triangle);
+// beta == 0 writes exact zeros without reading C
+__global__ void dscale_kernel(double *C, int64_t ldc, int64_t m, int64_t c0, double beta, int tri) {
+  const int64_t c = c0 + blockIdx.y;
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (int64_t)gridDim.x * blockDim.x) {
+    if ((tri == 1 && r < c) || (tri == 2 && r > c)) continue;
+    double *p = C + r + c * ldc;
+    *p = beta == 0.0 ? 0.0 : beta * *p;
+  }
+}
+
+}  // namespace
+
+int launch_dgemm(const DProblem &P, cudaStream_t s) {
+  if (P.M <= 0 || P.N <= 0) return 0;
+  const int64_t tiles = ((P.M + DTM - 1) / DTM) * ((P.N + DTN - 1) / DTN);
+  if (tiles > 0x7fffffffLL) return -1;
+  static std::atomic<bool> attr[64];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return -1;
+  if (!attr[dev].load(std::memory_order_acquire)) {
+    if (cudaFuncSetAttribute(dgemm_structured, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DSMEM) !=
+        cudaSuccess)
+      return -1;
+    attr[dev].store(true, std::memory_order_release);
+  }
+  dgemm_structured<<<(unsigned)tiles, DTHREADS, DSMEM, s>>>(P);
+  note_launch(1);
+  return cudaGetLastError() == cudaSuccess ? 0 : -1;
+}
+
+int launch_dtrsm_diag(const DOpnd &S, int nb, double *X, int64_t sx, int64_t sc, int64_t nrhs, cudaStream_t s) {
+  if (nb <= 0 || nrhs <= 0) return 0;
+  if (nb > DNB) return -1;
+  dtrsm_diag<<<(unsigned)((nrhs + 63) / 64), 64, 0, s>>>(S, nb, X, sx, sc, nrhs);
+  note_launch(1);
+  return cudaGetLastError() == cudaSuccess ? 0 : -1;
+}
+
+int launch_dscale(double *C, int64_t ldc, int64_t m, int64_t n, double beta, int tri, cudaStream_t s) {
+  if (m <= 0 || n <= 0) return 0;
+  const unsigned gx = (unsigned)((m + 255) / 256 < 64 ? (m + 255) / 256 : 64);
+  for (int64_t c0 = 0; c0 < n; c0 += 65535) {
+    const int64_t nc = n - c0 < 65535 ? n - c0 : 65535;
+    dscale_kernel<<<dim3(gx, (unsigned)nc), 256, 0, s>>>(C, ldc, m, c0, beta, tri);
+    note_launch(2);
+    if (cudaGetLastError() != cudaSuccess) return -1;
+  }
+  return 0;
+}
+
+}  // namespace blas3
