@@ -508,6 +508,9 @@ def run_ours(args):
                 ms_r = c0.elapsed_time(c1) / reps
                 isolated[r] = {"ms": round(ms_r, 4), "gflops": round(fl[r] / (ms_r * 1e-3) / 1e9, 1),
                                "reps": reps, "clocks": clk_r.summary(t0, t1)}
+        for r in ROUTINES:            # each routine in its own sustained loop (the chain's
+            isolated[r]["pct_of_sgemm"] = round(   # per-routine times carry the power state of the
+                100.0 * isolated[r]["gflops"] / isolated["sgemm"]["gflops"], 1)   # routine before)
 
     # context (north star: "reports the box's cuBLAS SGEMM as context"): torch's
     # cuBLAS fp32 SGEMM (TF32 off) and its 1-pass TF32 mode on the same A, B
@@ -541,6 +544,36 @@ def run_ours(args):
                                                              "Tesla C2050": 3.4},
                              "gtx285_cublas3.2_sgemm_gflops": 420, "gtx285_cublas3.2_ssymm_gflops": 155,
                              "gtx285_oa_ssymm_gflops": 403, "problem": "fp32, N=4096"}}
+
+    # fp64 family (blas3_d*): DGEMM NN and DTRSM LLNN at N = 4096 on
+    # the same device, against the DFMA peak (148 SM x 64 DFMA/clk x 2 x max
+    # clock; tools/probes/dmma_rate.cu measured 36.4 TF/s for DFMA and 37.1 for
+    # DMMA, so the CUDA cores are the FP64 roofline)
+    fp64 = None
+    if world == 1 and not args.no_fp64:
+        n64 = 4096
+        f64t = lambda: b3.colmajor(n64, n64, dtype=torch.float64).uniform_(-1, 1)  # noqa: E731
+        A64, B64, C64, X64 = f64t(), f64t(), f64t(), f64t()
+        T64 = f64t().mul_(1.0 / n64)
+        T64.diagonal().fill_(1.0)
+        pk64 = 148 * 64 * 2 * load_peaks()[0].get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+        fp64 = {"n": n64, "peak_tflops": round(pk64, 1),
+                "peak_source": "148 SM x 64 DFMA/clk x 2 x max SM clock (DFMA; DMMA measured no faster)"}
+        for name, fn, flops64 in (("dgemm", lambda: b3.dgemm("N", "N", ALPHA, A64, B64, BETA, C64), 2.0 * n64 ** 3),
+                                  ("dtrsm", lambda: b3.dtrsm("L", "L", "N", "N", ALPHA, T64, X64), 1.0 * n64 ** 3)):
+            X64.copy_(B64)
+            fn()
+            torch.cuda.synchronize()
+            c0 = torch.cuda.Event(enable_timing=True); c1 = torch.cuda.Event(enable_timing=True)
+            c0.record(stream)
+            for _ in range(3):
+                fn()
+            c1.record(stream)
+            torch.cuda.synchronize()
+            ms64 = c0.elapsed_time(c1) / 3
+            fp64[name] = {"ms": round(ms64, 3), "gflops": round(flops64 / (ms64 * 1e-3) / 1e9, 1),
+                          "frac": round(flops64 / (ms64 * 1e-3) / 1e12 / pk64, 3)}
+        del A64, B64, C64, X64, T64
 
     total_flops = sum(fl.values()) * world
     step_ms = ms / args.steps
@@ -638,6 +671,7 @@ def run_ours(args):
         "gpu_launches": int(launches),
         "comm": comm_info,
         "alt_mode": alt,
+        "fp64": fp64,
         "context": context,
         "gpu_launches_per_step": round(launches / args.steps, 1),
         "isolated": isolated,
@@ -985,6 +1019,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the e2e leg (profiling runs)")
     ap.add_argument("--no-context", action="store_true", help="skip the cuBLAS context timing")
+    ap.add_argument("--no-fp64", action="store_true", help="skip the fp64-family context timing")
     ap.add_argument("--no-alt-mode", action="store_true",
                     help="skip the extra device-only pass in the opt-in TF32+BF16X mode")
     ap.add_argument("--no-routine-clocks", action="store_true",
