@@ -68,7 +68,7 @@ constexpr int NTHREADS = (WARP_EPI0 + NUM_EPI_WARPS) * 32;       // 640
 constexpr int EPI_REGS = 144, OTHER_REGS = 64;   // 36864 + 24576 = 61440
 // Chunked accumulation: the tensor core's fp32 accumulator truncates on every
 // UMMA add (Q24), so a TMEM partial only ever sums Problem::kc
-// k-blocks (BLAS3_OPT_TC_KC, default 4: K = 128) before the epilogue folds it
+// k-blocks (BLAS3_OPT_TC_KC, default 3: K = 96) before the epilogue folds it
 // into a register running sum with round-to-nearest adds; the two TMEM
 // buffers ping-pong per chunk.
 constexpr int EC = 16;                            // epilogue column group
@@ -113,7 +113,7 @@ struct Geo {
     uint8_t B[B_BYTES];
   };
   struct alignas(1024) LoBuf {
-    uint8_t A[A_BYTES];      // lo = rna_tf32(x - hi), written by the transform
+    uint8_t A[A_BYTES];      // lo = x - hi (exact in fp32), written by the transform
     uint8_t B[B_BYTES];
   };
   struct Barriers {
