@@ -12,8 +12,10 @@
 //   DTRSM  op(tri(A)) X = alpha B  /  X op(tri(A)) = alpha B: B scaled by alpha,
 //          then recursive halving in dependency order (Fig. 7):
 //          solve the first half, ONE GEMM update of the second half by it,
-//          solve the second half; 64-wide diagonal blocks by substitution
-//          (dtrsm_diag: one thread per right-hand side, exact fp64).
+//          solve the second half; leaves of <= 512 rows in ONE launch each
+//          (dtrsm_panel: the panel's rows of 32 right-hand sides per CTA in
+//          shared memory, 64-blocks in dependency order with the inverses of
+//          all 64-blocks computed up front by substitution, dtri_inv64).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -64,7 +66,8 @@ struct DScratch {
   }
 };
 
-constexpr int64_t DNB = 64;
+constexpr int64_t DNB = 64;          // diagonal blocks (inverted by dtri_inv64)
+constexpr int64_t DPANEL = 512;      // recursion leaves (dtrsm_panel)
 
 }  // namespace
 }  // namespace blas3
@@ -207,13 +210,19 @@ int blas3_dtrsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
   const bool s_lower = lower != strans;
   const int64_t nt = left ? m : n, nrhs = left ? n : m;
   const int64_t sx = left ? 1 : ldb, sc = left ? ldb : 1;   // element i of right-hand side c
+  // the inverses of all 64-blocks of S in one launch, then the recursion
+  // down to panels of <= DPANEL rows, each solved by one launch
+  DScratch Dinv;
+  if ((rc = Dinv.get((size_t)((nt + DNB - 1) / DNB) * DNB * DNB * sizeof(double), s))) return rc;
+  if (launch_dtri_inv64(dtri(A, lda, lower, strans, unit), nt, Dinv.p, s)) return BLAS3_ERR_CUDA;
   // rows [lo, hi) of the system, in dependency order by recursive halving
   int err = 0;
   auto solve = [&](auto &&self, int64_t lo, int64_t hi) -> void {
     if (err) return;
     const int64_t w = hi - lo;
-    if (w <= DNB) {
-      if (launch_dtrsm_diag(dtri(A, lda, lower, strans, unit, lo, lo), (int)w, B + lo * sx, sx, sc, nrhs, s))
+    if (w <= DPANEL) {                                // lo is a multiple of 64
+      if (launch_dtrsm_panel(dtri(A, lda, lower, strans, unit, lo, lo), Dinv.p + (lo / DNB) * DNB * DNB, (int)w,
+                             B + lo * sx, sx, sc, nrhs, s))
         err = BLAS3_ERR_CUDA;
       return;
     }

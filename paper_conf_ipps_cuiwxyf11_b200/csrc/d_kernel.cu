@@ -229,25 +229,9 @@ __global__ void __launch_bounds__(DTHREADS, 1) dgemm_structured(const __grid_con
   }
 }
 
-// Diagonal block of a triangular solve: for every right-hand side (one per
-// thread) solve S y = rhs in place, S = nb x nb (nb <= DNB) from the TRI
-// operand (forward if S is lower, else backward), padded to DNB with the
-// identity.  rhs element i of right-hand side c: X[i * sx + c * sc].
-__global__ void __launch_bounds__(64) dtrsm_diag(const __grid_constant__ DOpnd S, int nb, double *X, int64_t sx,
-                                                 int64_t sc, int64_t nrhs) {
-  __shared__ double Ss[DNB * (DNB + 1)];
-  for (int e = threadIdx.x; e < DNB * DNB; e += blockDim.x) {
-    const int i = e % DNB, j = e / DNB;
-    Ss[i + j * (DNB + 1)] = (i < nb && j < nb) ? dfetch(S, i, j) : (i == j ? 1.0 : 0.0);
-  }
-  __syncthreads();
-  const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= nrhs) return;
-  double y[DNB];
-#pragma unroll
-  for (int i = 0; i < DNB; ++i) y[i] = i < nb ? X[i * sx + c * sc] : 0.0;
-  // S lower <=> nonzeros at i >= j of the logical (i, j) = (r, k)
-  const bool lower = S.lower != (S.trans != 0);
+// In-register substitution S y = y for one 64-block S (shared, ld DNB + 1),
+// forward (S lower) or backward, a division per row as in the oracle
+__device__ __forceinline__ void subst64(const double *Ss, double (&y)[DNB], bool lower) {
   if (lower) {
 #pragma unroll
     for (int i = 0; i < DNB; ++i) {
@@ -265,9 +249,104 @@ __global__ void __launch_bounds__(64) dtrsm_diag(const __grid_constant__ DOpnd S
       y[i] = v / Ss[i + i * (DNB + 1)];
     }
   }
+}
+// one 64-block of S into shared memory, padded with the identity beyond nb
+__device__ __forceinline__ void load_block64(const DOpnd &S, int64_t o, int nb, double *Ss) {
+  for (int e = threadIdx.x; e < DNB * DNB; e += blockDim.x) {
+    const int i = e % DNB, j = e / DNB;
+    Ss[i + j * (DNB + 1)] = (i < nb && j < nb) ? dfetch(S, o + i, o + j) : (i == j ? 1.0 : 0.0);
+  }
+}
+
+// inv(S_bb) of every 64-block b on the diagonal of the order-nt triangle S
+// (one CTA per block, thread c solves S_bb y = e_c): Dinv + 4096 b, 64 x 64
+// column-major, the identity where a ragged last block is padded
+__global__ void __launch_bounds__(64) dtri_inv64(const __grid_constant__ DOpnd S, int64_t nt, double *Dinv) {
+  __shared__ double Ss[DNB * (DNB + 1)];
+  const int64_t o = (int64_t)blockIdx.x * DNB;
+  const int nb = (int)(nt - o < DNB ? nt - o : DNB);
+  load_block64(S, o, nb, Ss);
+  __syncthreads();
+  const int c = threadIdx.x;
+  double y[DNB];
 #pragma unroll
-  for (int i = 0; i < DNB; ++i)
-    if (i < nb) X[i * sx + c * sc] = y[i];
+  for (int i = 0; i < DNB; ++i) y[i] = i == c ? 1.0 : 0.0;
+  subst64(Ss, y, S.lower != (S.trans != 0));
+  double *d = Dinv + (size_t)blockIdx.x * DNB * DNB + (size_t)c * DNB;
+#pragma unroll
+  for (int i = 0; i < DNB; ++i) d[i] = y[i];
+}
+
+// A diagonal panel of R <= DPR rows (64-blocks, processing order forward if S
+// is lower) for DRC right-hand sides per CTA, the panel's rows of those
+// right-hand sides resident in shared memory:
+//   y_i <- inv(S_ii) (y_i - sum_{j before i} S_ij y_j)
+// with the 64-block inverses from dtri_inv64 (Dp: this panel's first block).
+// One launch replaces the 64-row recursion's small launches at the bottom of
+// the DTRSM sweep.
+constexpr int DPR = 512, DRC = 32, DPT = 256;
+constexpr size_t DPANEL_SMEM = (size_t)(DPR * DRC + DNB * (DNB + 1)) * sizeof(double);   // 164 KB
+__global__ void __launch_bounds__(DPT, 1) dtrsm_panel(const __grid_constant__ DOpnd S, const double *Dp, int R,
+                                                      double *X, int64_t sx, int64_t sc, int64_t nrhs) {
+  extern __shared__ double dps[];
+  double *Y = dps;                                    // Y[i * DRC + c]
+  double *Ss = dps + DPR * DRC;                       // one 64-block, ld DNB + 1
+  const int64_t c0 = (int64_t)blockIdx.x * DRC;
+  const int ncol = (int)(nrhs - c0 < DRC ? nrhs - c0 : DRC);
+  const int nb = (R + DNB - 1) / DNB;
+  const bool lower = S.lower != (S.trans != 0);
+  // load the panel's rows of this CTA's right-hand sides (i fastest when the
+  // rows are contiguous, sx == 1)
+  for (int e = threadIdx.x; e < nb * DNB * DRC; e += DPT) {
+    const int i = sx == 1 ? e % (nb * DNB) : e / DRC, c = sx == 1 ? e / (nb * DNB) : e % DRC;
+    Y[i * DRC + c] = (i < R && c < ncol) ? X[i * sx + (c0 + c) * sc] : 0.0;
+  }
+  // this thread's outputs: rows r = tid % 64, columns cq = tid / 64 + 4 q (q < 8)
+  const int r = threadIdx.x % DNB, cb = threadIdx.x / DNB;
+  for (int st = 0; st < nb; ++st) {
+    const int bi = lower ? st : nb - 1 - st;
+    double acc[DRC / 4];
+#pragma unroll
+    for (int q = 0; q < DRC / 4; ++q) acc[q] = 0.0;
+    for (int tt = 0; tt < st; ++tt) {                 // the blocks solved before bi
+      const int bj = lower ? tt : nb - 1 - tt;
+      __syncthreads();
+      for (int e = threadIdx.x; e < DNB * DNB; e += DPT) {
+        const int i = e % DNB, j = e / DNB;
+        const int64_t gi = (int64_t)bi * DNB + i, gj = (int64_t)bj * DNB + j;
+        Ss[i + j * (DNB + 1)] = (gi < R && gj < R) ? dfetch(S, gi, gj) : 0.0;
+      }
+      __syncthreads();
+#pragma unroll 8
+      for (int k = 0; k < DNB; ++k) {
+        const double sv = Ss[r + k * (DNB + 1)];
+#pragma unroll
+        for (int q = 0; q < DRC / 4; ++q) acc[q] = fma(sv, Y[(bj * DNB + k) * DRC + cb + 4 * q], acc[q]);
+      }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < DRC / 4; ++q) Y[(bi * DNB + r) * DRC + cb + 4 * q] -= acc[q];
+    for (int e = threadIdx.x; e < DNB * DNB; e += DPT)          // inv(S_ii)
+      Ss[e % DNB + (e / DNB) * (DNB + 1)] = Dp[(size_t)bi * DNB * DNB + e];
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < DRC / 4; ++q) acc[q] = 0.0;
+#pragma unroll 8
+    for (int k = 0; k < DNB; ++k) {
+      const double sv = Ss[r + k * (DNB + 1)];
+#pragma unroll
+      for (int q = 0; q < DRC / 4; ++q) acc[q] = fma(sv, Y[(bi * DNB + k) * DRC + cb + 4 * q], acc[q]);
+    }
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < DRC / 4; ++q) Y[(bi * DNB + r) * DRC + cb + 4 * q] = acc[q];
+  }
+  __syncthreads();
+  for (int e = threadIdx.x; e < nb * DNB * DRC; e += DPT) {
+    const int i = sx == 1 ? e % (nb * DNB) : e / DRC, c = sx == 1 ? e / (nb * DNB) : e % DRC;
+    if (i < R && c < ncol) X[i * sx + (c0 + c) * sc] = Y[i * DRC + c];
+  }
 }
 
 // C <- beta * C on the m x n block (tri: 0 all, 1 lower, 2 upper triangle);
@@ -301,10 +380,27 @@ int launch_dgemm(const DProblem &P, cudaStream_t s) {
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
 
-int launch_dtrsm_diag(const DOpnd &S, int nb, double *X, int64_t sx, int64_t sc, int64_t nrhs, cudaStream_t s) {
-  if (nb <= 0 || nrhs <= 0) return 0;
-  if (nb > DNB) return -1;
-  dtrsm_diag<<<(unsigned)((nrhs + 63) / 64), 64, 0, s>>>(S, nb, X, sx, sc, nrhs);
+int launch_dtri_inv64(const DOpnd &S, int64_t nt, double *Dinv, cudaStream_t s) {
+  if (nt <= 0) return 0;
+  dtri_inv64<<<(unsigned)((nt + DNB - 1) / DNB), DNB, 0, s>>>(S, nt, Dinv);
+  note_launch(1);
+  return cudaGetLastError() == cudaSuccess ? 0 : -1;
+}
+
+int launch_dtrsm_panel(const DOpnd &S, const double *Dp, int R, double *X, int64_t sx, int64_t sc, int64_t nrhs,
+                       cudaStream_t s) {
+  if (R <= 0 || nrhs <= 0) return 0;
+  if (R > DPR) return -1;
+  static std::atomic<bool> attr[64];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return -1;
+  if (!attr[dev].load(std::memory_order_acquire)) {
+    if (cudaFuncSetAttribute(dtrsm_panel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DPANEL_SMEM) !=
+        cudaSuccess)
+      return -1;
+    attr[dev].store(true, std::memory_order_release);
+  }
+  dtrsm_panel<<<(unsigned)((nrhs + DRC - 1) / DRC), DPT, DPANEL_SMEM, s>>>(S, Dp, R, X, sx, sc, nrhs);
   note_launch(1);
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }

@@ -29,9 +29,14 @@ struct DProblem {
 };
 
 int launch_dgemm(const DProblem &P, cudaStream_t s);
-// one diagonal block of a triangular solve, in place: S (nb x nb <= 64, a TRI
-// operand) y = rhs for nrhs right-hand sides, element i of rhs c at X[i*sx + c*sc]
-int launch_dtrsm_diag(const DOpnd &S, int nb, double *X, int64_t sx, int64_t sc, int64_t nrhs, cudaStream_t s);
+// inv(S_bb) of every 64-block on the diagonal of the order-nt TRI operand S
+// (offsets 0): Dinv + 4096 b, 64 x 64 column-major (identity-padded)
+int launch_dtri_inv64(const DOpnd &S, int64_t nt, double *Dinv, cudaStream_t s);
+// a diagonal panel of R <= 512 rows in one launch (64-blocks in dependency
+// order, their inverses at Dp), in place: rhs element i of right-hand side c
+// at X[i*sx + c*sc]; S's offsets point at the panel's corner
+int launch_dtrsm_panel(const DOpnd &S, const double *Dp, int R, double *X, int64_t sx, int64_t sc, int64_t nrhs,
+                       cudaStream_t s);
 // C <- beta * C (tri 0 all / 1 lower / 2 upper), beta == 0 -> exact zeros
 int launch_dscale(double *C, int64_t ldc, int64_t m, int64_t n, double beta, int tri, cudaStream_t s);
 

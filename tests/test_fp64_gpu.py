@@ -10,7 +10,7 @@ orders of magnitude below what a dropped term, a wrong mirror or a wrong
 triangle would give. Integer-valued inputs have an exact, unique fp64
 result: it must be reproduced bit for bit. The unreferenced triangle of A
 and, for SYRK/SYR2K, of C hold NaN sentinels (never read, never written).
-Sizes span several 128 x 64 tiles with ragged tails.
+Sizes span several 128 x 128 tiles with ragged tails.
 """
 import itertools
 
@@ -129,11 +129,12 @@ def test_dtrmm(b3, oracle_mod, side, uplo, ta, diag):
 
 
 @pytest.mark.parametrize("side,uplo,ta,diag", V16)
-@pytest.mark.parametrize("order,rhs", [(200, 131), (64, 65), (331, 40)])
+@pytest.mark.parametrize("order,rhs", [(200, 131), (64, 65), (331, 40), (1100, 37)])
 def test_dtrsm(b3, oracle_mod, side, uplo, ta, diag, order, rhs):
     """Diagonally dominant A (cond ~ 1): forward error vs the oracle and the
-    residual, both at fp64 level. order 331 = five 64-blocks + a ragged one;
-    200 forces a ragged first half in the recursive split."""
+    residual, both at fp64 level. Orders up to 512 are one panel launch
+    (331 = five 64-blocks + a ragged one); 1100 recurses (576 + 524 -> panels
+    of 512, 64 and a ragged 524 split again), with the GEMM updates between."""
     m, n = (order, rhs) if side == "L" else (rhs, order)
     A = gen.triangular_dd(order, uplo, diag, "dr-a")
     B = gen.uniform(m, n, "dr-b")
