@@ -211,3 +211,44 @@ def test_options_roundtrip_and_validation(lib):
     assert lib.get_option("tc_c_async") == 0
     assert lib.get_option("trsm_panel") == 1
     assert len(lib.OPTIONS) == 27
+
+
+def test_fp64_family_xerbla_and_quick_returns(lib):
+    """The fp64 entry points share the s-routines' validators (csrc/validate.h):
+    same XERBLA positions, same quick returns, all before any CUDA call."""
+    g = lib.blas3_dgemm
+    assert g(b"X", b"N", 4, 4, 4, 1.0, NULL, 4, NULL, 4, 0.0, NULL, 4, NULL) == 1
+    assert g(b"N", b"N", 4, 4, 4, 1.0, NULL, 3, NULL, 4, 0.0, NULL, 4, NULL) == 8
+    assert g(b"N", b"T", 4, 6, 4, 1.0, NULL, 4, NULL, 5, 0.0, NULL, 4, NULL) == 10
+    assert g(b"N", b"N", 4, 4, 4, 1.0, NULL, 4, NULL, 4, 0.0, NULL, 3, NULL) == 13
+    assert g(b"N", b"N", 0, 4, 4, 1.0, NULL, 4, NULL, 4, 0.0, NULL, 4, NULL) == 0
+    assert g(b"N", b"N", 4, 4, 4, 0.0, NULL, 4, NULL, 4, 1.0, NULL, 4, NULL) == 0
+    assert g(b"N", b"N", 4, 4, 4, 1.0, NULL, 4, NULL, 4, 0.0, NULL, 4, NULL) == 12   # NULL C
+    s = lib.blas3_dsymm
+    assert s(b"R", b"L", 4, 3, 1.0, NULL, 2, NULL, 4, 0.0, NULL, 4, NULL) == 7
+    assert s(b"L", b"X", 4, 3, 1.0, NULL, 4, NULL, 4, 0.0, NULL, 4, NULL) == 2
+    k = lib.blas3_dsyrk
+    assert k(b"L", b"T", 5, 3, 1.0, NULL, 2, 0.0, NULL, 5, NULL) == 7
+    assert k(b"L", b"N", 5, 3, 1.0, NULL, 5, 0.0, NULL, 4, NULL) == 10
+    k2 = lib.blas3_dsyr2k
+    assert k2(b"U", b"N", 5, 3, 1.0, NULL, 5, NULL, 4, 0.0, NULL, 5, NULL) == 9
+    assert k2(b"U", b"N", 5, 3, 1.0, NULL, 5, NULL, 5, 0.0, NULL, 4, NULL) == 12
+    for f in (lib.blas3_dtrmm, lib.blas3_dtrsm):
+        assert f(b"L", b"L", b"N", b"X", 4, 4, 1.0, NULL, 4, NULL, 4, NULL) == 4
+        assert f(b"R", b"L", b"N", b"N", 4, 6, 1.0, NULL, 5, NULL, 4, NULL) == 9
+        assert f(b"L", b"L", b"N", b"N", 4, 6, 1.0, NULL, 4, NULL, 3, NULL) == 11
+        assert f(b"L", b"L", b"N", b"N", 0, 6, 1.0, NULL, 1, NULL, 1, NULL) == 0
+        assert f(b"L", b"L", b"N", b"N", 4, 6, 1.0, NULL, 4, NULL, 4, NULL) == 10     # NULL B
+
+
+def test_fp64_wrappers_check_dtype_and_shape():
+    """The tensor wrappers refuse fp32 tensors for d-routines (and the reverse)
+    before any library call: marshalling only, no silent conversion."""
+    torch = pytest.importorskip("torch")
+    import paper_conf_ipps_cuiwxyf11_b200 as b
+    a32 = torch.zeros((4, 4), dtype=torch.float32)
+    a64 = torch.zeros((4, 4), dtype=torch.float64)
+    with pytest.raises(TypeError):
+        b.dgemm("N", "N", 1.0, a32, a32, 0.0, a32)
+    with pytest.raises(TypeError):
+        b.sgemm("N", "N", 1.0, a64, a64, 0.0, a64)
