@@ -34,16 +34,21 @@ def _headers():
     return hs
 
 
+REPO = os.path.dirname(HERE)
+
+
 def _digest(paths, extra):
     """Content hash of the inputs of one build step (sources, every header,
     compiler and flags): rebuilds follow content, never file times, so a
-    stale object or library shipped with a snapshot is never reused."""
+    stale object or library shipped with a snapshot is never reused.  Paths
+    enter relative to the repository, so the same sources give the same
+    digest wherever the checkout lives (the GPU box's copy included)."""
     h = hashlib.sha256()
     for p in paths:
-        h.update(p.encode())
+        h.update(os.path.relpath(p, REPO).encode())
         with open(p, "rb") as f:
             h.update(f.read())
-    h.update(repr(extra).encode())
+    h.update(repr(extra).replace(REPO, "<repo>").encode())
     return h.hexdigest()
 
 
