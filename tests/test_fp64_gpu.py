@@ -223,3 +223,49 @@ def test_large_dgemm_and_dtrsm_sampled(b3, oracle_mod):
     X = f64(to_host(dB))[:, sel]
     ref = oracle_mod.strsm("L", "U", "N", "N", AL, T, B, sel=sel)
     assert fro(X - ref) / fro(ref) <= 64 * n * U53
+
+
+@pytest.mark.parametrize("routine", ["dgemm", "dsyrk", "dtrmm", "dtrsm"])
+def test_padded_ld_untouched(b3, oracle_mod, routine):
+    """Outputs inside larger NaN-filled allocations with odd leading dimensions
+    (ld = rows + 5): only the m x n block changes, the padding rows and the
+    columns beyond n keep their NaN sentinels, and the block is correct
+    (a bounds check in place of a memory checker)."""
+    import torch
+    m, n, k = 150, 97, 70
+    ld = m + 5
+    full = torch.full((n + 2, ld), float("nan"), dtype=torch.float64, device="cuda")
+    view = full[:n].t()[:m]                          # m x n, column-major, ld = m + 5
+    if routine == "dtrsm" or routine == "dtrmm":
+        T = gen.triangular_dd(m, "L", "N", "pad-t")
+        B = gen.uniform(m, n, "pad-b")
+        view.copy_(torch.from_numpy(f64(B)))
+        getattr(b3, routine)("L", "L", "N", "N", AL, dev(b3, T), view)
+        ref = getattr(oracle_mod, "s" + routine[1:])("L", "L", "N", "N", AL, T, B)
+        tolr = 64 * m * U53
+    elif routine == "dgemm":
+        A = gen.uniform(m, k, "pad-a"); B = gen.uniform(k, n, "pad-b2"); C = gen.uniform(m, n, "pad-c")
+        view.copy_(torch.from_numpy(f64(C)))
+        b3.dgemm("N", "N", AL, dev(b3, A), dev(b3, B), BE, view)
+        ref = oracle_mod.sgemm("N", "N", AL, A, B, BE, C)
+        tolr = tol(k) * 10
+    else:                                            # dsyrk on an n x n block
+        n = m
+        full = torch.full((n + 2, ld), float("nan"), dtype=torch.float64, device="cuda")
+        view = full[:n].t()[:m]
+        A = gen.uniform(m, k, "pad-k"); C = gen.nan_outside(gen.uniform(m, m, "pad-kc"), "U")
+        view.copy_(torch.from_numpy(f64(C)))
+        b3.dsyrk("U", "N", AL, dev(b3, A), BE, view)
+        ref = oracle_mod.ssyrk("U", "N", AL, A, BE, C)
+        up = np.triu(np.ones((m, m), bool))
+        got = view.cpu().numpy()
+        assert fro(np.where(up, got, 0) - np.where(up, ref, 0)) / fro(np.where(up, ref, 0)) <= tol(k) * 10
+        host = full.cpu().numpy()
+        assert np.isnan(host[:n, m:]).all() and np.isnan(host[n:]).all()
+        assert np.isnan(got[~up]).all()
+        return
+    got = view.cpu().numpy()
+    assert fro(got - ref) / fro(ref) <= tolr
+    host = full.cpu().numpy()
+    assert np.isnan(host[:n, m:]).all(), "padding rows written"
+    assert np.isnan(host[n:]).all(), "columns beyond n written"
