@@ -23,6 +23,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <atomic>
+#include <stdlib.h>
 
 #include "kernels.h"
 #include "d_kernels.h"
@@ -31,7 +32,7 @@ namespace blas3 {
 namespace {
 
 constexpr int DTM = 128, DTN = 128, DBK = 16, DTHREADS = 256;
-constexpr int DAP = DTM + 2, DBP = DTN + 2;          // padded shared rows (doubles)
+constexpr int DAP = DTM + 8, DBP = DTN + 8;          // padded shared rows: 1088 B = 64 B mod 128 (DMMA fragment loads conflict-free)
 constexpr int DJ = 8;                                // columns per thread (two groups of 4)
 constexpr int DNB = 64;                              // TRSM diagonal block
 
@@ -141,8 +142,18 @@ struct TileLoad {
   }
 };
 
-constexpr size_t DSMEM = 2 * DBK * (DAP + DBP) * sizeof(double);   // 66560 B (dynamic)
+constexpr size_t DSMEM = 2 * DBK * (DAP + DBP) * sizeof(double);   // 69632 B (dynamic)
 
+// one DMMA (m8n8k4, f64): d += a (8x4 row-major fragment) * b (4x8 col-major)
+__device__ __forceinline__ void dmma(double &d0, double &d1, double a, double b) {
+  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
+               : "+d"(d0), "+d"(d1) : "d"(a), "d"(b));
+}
+
+// MMA = false: DFMA, 8 x 8 outputs per thread.  MMA = true: DMMA m8n8k4 on
+// register fragments, each warp a 64 x 32 block (8 x 4 fragments), the same
+// staging and epilogue semantics.
+template <bool MMA>
 __global__ void __launch_bounds__(DTHREADS, 1) dgemm_structured(const __grid_constant__ DProblem P) {
   extern __shared__ double dsm[];
   // buffers by integer offset from the __shared__ array (not through a
@@ -188,6 +199,22 @@ __global__ void __launch_bounds__(DTHREADS, 1) dgemm_structured(const __grid_con
         lb.load(S.b, n0, P.N, kn, khi, rfb);
       }
       const double *as = dsm + cur * AOFF, *bs = dsm + BOFF0 + cur * BOFF;
+      if constexpr (MMA) {
+        const int lane = threadIdx.x % 32, wid = threadIdx.x / 32;
+        const int am = 64 * (wid % 2) + lane / 4, bn = 32 * (wid / 2) + lane / 4, kq = lane % 4;
+#pragma unroll
+        for (int kk = 0; kk < DBK / 4; ++kk) {
+          double a[8], b[4];
+#pragma unroll
+          for (int i = 0; i < 8; ++i) a[i] = as[(kk * 4 + kq) * DAP + am + 8 * i];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) b[j] = bs[(kk * 4 + kq) * DBP + bn + 8 * j];
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+#pragma unroll
+            for (int j = 0; j < 4; ++j) dmma(acc[i][2 * j], acc[i][2 * j + 1], a[i], b[j]);
+        }
+      } else {
 #pragma unroll
       for (int k = 0; k < DBK; ++k) {
         double a[8], b[DJ];
@@ -204,6 +231,7 @@ __global__ void __launch_bounds__(DTHREADS, 1) dgemm_structured(const __grid_con
 #pragma unroll
           for (int j = 0; j < DJ; ++j) acc[i][j] = fma(a[i], b[j], acc[i][j]);
       }
+      }
       if (t + 1 < nkb) {
         la.store<DAP>(dsm + (cur ^ 1) * AOFF, rfa);
         lb.store<DBP>(dsm + BOFF0 + (cur ^ 1) * BOFF, rfb);
@@ -214,11 +242,14 @@ __global__ void __launch_bounds__(DTHREADS, 1) dgemm_structured(const __grid_con
   // epilogue: D = alpha * acc + beta * C (C not read when beta == 0), uplo mask
 #pragma unroll
   for (int j = 0; j < DJ; ++j) {
-    const int64_t c = n0 + 4 * tc + 64 * (j / 4) + j % 4;
+    // DMMA: acc[i][2 jf + e] is C row 64 (w % 2) + 8 i + lane / 4, column
+    // 32 (w / 2) + 8 jf + 2 (lane % 4) + e
+    const int64_t c = MMA ? n0 + 32 * ((threadIdx.x / 32) / 2) + 8 * (j / 2) + 2 * ((threadIdx.x % 32) % 4) + j % 2
+                          : n0 + 4 * tc + 64 * (j / 4) + j % 4;
     if (c >= P.N) continue;
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
-      const int64_t r = m0 + tr + 16 * i;
+      const int64_t r = MMA ? m0 + 64 * ((threadIdx.x / 32) % 2) + 8 * i + (threadIdx.x % 32) / 4 : m0 + tr + 16 * i;
       if (r >= P.M) continue;
       if (P.ctri == 1 && r < c) continue;
       if (P.ctri == 2 && r > c) continue;
@@ -366,16 +397,18 @@ int launch_dgemm(const DProblem &P, cudaStream_t s) {
   if (P.M <= 0 || P.N <= 0) return 0;
   const int64_t tiles = ((P.M + DTM - 1) / DTM) * ((P.N + DTN - 1) / DTN);
   if (tiles > 0x7fffffffLL) return -1;
-  static std::atomic<bool> attr[64];
+  // BLAS3_D_MMA: 1 (default) DMMA fragments, 0 DFMA (A/B)
+  static const bool use_mma = [] { const char *e = getenv("BLAS3_D_MMA"); return e ? atoi(e) != 0 : true; }();
+  void (*kfn)(const DProblem) = use_mma ? dgemm_structured<true> : dgemm_structured<false>;
+  static std::atomic<bool> attr[64][2];
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return -1;
-  if (!attr[dev].load(std::memory_order_acquire)) {
-    if (cudaFuncSetAttribute(dgemm_structured, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DSMEM) !=
-        cudaSuccess)
+  if (!attr[dev][use_mma].load(std::memory_order_acquire)) {
+    if (cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DSMEM) != cudaSuccess)
       return -1;
-    attr[dev].store(true, std::memory_order_release);
+    attr[dev][use_mma].store(true, std::memory_order_release);
   }
-  dgemm_structured<<<(unsigned)tiles, DTHREADS, DSMEM, s>>>(P);
+  kfn<<<(unsigned)tiles, DTHREADS, DSMEM, s>>>(P);
   note_launch(1);
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
