@@ -175,10 +175,10 @@ int blas3_strsm(char side, char uplo, char transa, char diag, int64_t m, int64_t
  * blas3_d{gemm,symm,syrk,syr2k,trmm,trsm}: the same semantics, argument
  * lists, XERBLA codes, quick returns, alpha/beta special cases, ownership
  * and stream rules as the s-routines above, on column-major fp64 matrices in
- * device memory with host double scalars.  Arithmetic: IEEE fp64 FMA on the
- * CUDA cores (one structured DFMA GEMM kernel, d_kernel.cu; the B200's FP64
- * tensor rate is no higher than its DFMA rate), every product and sum in
- * fp64; symmetric operands are mirrored and triangular ones zero-filled
+ * device memory with host double scalars.  Arithmetic: fp64 products and sums
+ * throughout (one structured fp64 GEMM kernel, d_kernel.cu, on DMMA m8n8k4
+ * fragments; B200's DMMA and DFMA share one 37 TF/s roofline, DMMA needs 8x
+ * fewer instructions); symmetric operands are mirrored and triangular ones zero-filled
  * while staged to shared memory, as in the fp32 kernels.  DTRMM uses
  * stream-ordered scratch of m*n doubles.  DTRSM scales B by alpha, then
  * solves by recursive halving (diagonal blocks of 64 by substitution, GEMM

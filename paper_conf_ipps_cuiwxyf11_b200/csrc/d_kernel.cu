@@ -1,6 +1,6 @@
 // d_kernel.cu -- the fp64 family ("DGEMM family"): one
-// structured FP64 GEMM kernel on the CUDA cores (DFMA) that every D routine
-// derives from, plus the triangular-solve diagonal-block kernel.
+// structured fp64 GEMM kernel that every D routine derives from, plus the
+// triangular-solve kernels (64-block inverses, panel leaves).
 //
 // The paper's method carried over unchanged to double precision
 // (PAPER.md P:93-99 SM_alloc(X, Symmetry), P:197-210 padding/peel_triangular,
@@ -10,16 +10,16 @@
 // only the uplo triangle of C is written for SYRK/SYR2K, and TRSM is a blocked
 // diagonal-block solve followed by GEMM updates (d_abi.cu).
 //
-// Why CUDA cores: on B200 the FP64 tensor-core rate equals the FP64 FMA rate
-// (~40 TFLOP/s nominal, blackwell_cuda_programming.md), and DFMA keeps every
-// product and sum in IEEE fp64 (the oracle's precision), so a register-tiled
-// DFMA kernel is the direct route.  Roofline: DFMA-bound, 64 FMA/clk/SM.
+// Which unit: on B200 the FP64 tensor path (DMMA, mma.sync m8n8k4 f64) and the
+// FMA pipe (DFMA) top out at the same ~37 TF/s (tools/probes/dmma_rate.cu:
+// 37.1 vs 36.4).  DMMA does 256 FMAs per instruction against DFMA's 32, so the
+// default instantiation issues DMMA from register fragments; DFMA stays as
+// the BLAS3_D_MMA=0 alternative.  Products and sums are fp64 either way.
 //
 // Kernel: 256 threads, C tile 128 x 128, BK = 16 k-blocks staged through
 // registers into double-buffered shared memory (the structure select happens
-// on the way), 8 x 8 outputs per thread (rows tr + 16 i, columns 4 tc + 64 g
-// + j, so a warp's C accesses are 128-B runs of one column and its B reads
-// two broadcast 32-B groups).
+// on the way); DMMA: each warp a 64 x 32 block of 8 x 4 fragments; DFMA: 8 x 8
+// outputs per thread (rows tr + 16 i, columns 4 tc + 64 g + j).
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <atomic>
