@@ -13,3 +13,4 @@ timeout 600 ncu --set full --clock-control none --import-source on -k regex:tc_s
 python tools/ncu_summary.py r02 gpurun_out/final/launches.csv gpurun_out/final/sgemm.ncu-rep > gpurun_out/final/summary.log 2>&1
 cp profiles/r02_launches.md profiles/r02_sgemm_ncu.md profiles/ncu_sgemm_traffic.json gpurun_out/final/
 timeout 900 python bench.py > gpurun_out/final/bench.json 2> gpurun_out/final/bench.err
+timeout 900 python bench.py --workload cfg5 --steps 2 --warmup 3 --no-cpu-baseline > gpurun_out/final/cfg5.json 2> gpurun_out/final/cfg5.err
