@@ -383,8 +383,13 @@ int blas3_ssymm(char side, char uplo, int64_t m, int64_t n, float alpha, const f
   const int64_t ka = left ? m : n;
   // (SIMT mode: always from order 512 -- the materialisation is ~0.5% of the
   // FFMA GEMM, and the shadow area would otherwise be read uncoalesced)
-  if (tensor_mode() ? use_gm_map(ka, left ? n : m, BLAS3_OPT_GM_MIN_SYMM)
-                    : (opt(BLAS3_OPT_GM_MAP) != 0 && (opt(BLAS3_OPT_GM_MAP) == 1 || ka >= 512))) {
+  // (tcgen05, auto: GM_map below order 4096, where it measured faster at every
+  // size -- 512 / 1024 / 1536 / 2048 / 3072: 86-88 / 88 / 89-91 / 91-92 / 95% of
+  // SGEMM against 74 / 79 / 84-86 / 90 / 93-94% staged, profiles/r02_gm_map.md --
+  // and from 4096 the merge while staging, the paper's rule 3, within 1-5%)
+  const int64_t gm = opt(BLAS3_OPT_GM_MAP);
+  if (tensor_mode() ? (gm < 0 ? ka < 4096 || use_gm_map(ka, left ? n : m, BLAS3_OPT_GM_MIN_SYMM) : gm == 1)
+                    : (gm != 0 && (gm == 1 || ka >= 512))) {
     // GM_map: sym(A) materialised as a full ka x ka matrix, then a plain GEMM
     Scratch Wm;
     const int64_t ldw = ld4(ka);

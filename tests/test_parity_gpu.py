@@ -182,12 +182,16 @@ def test_determinism(b3):
 # ------------------------------------------------------------------------------------ SSYMM
 @pytest.mark.parametrize("side,uplo", list(itertools.product("LR", "LU")))
 @pytest.mark.parametrize("m,n", [(1, 1), (44, 68), (200, 132), (256, 300), (516, 260)])
-def test_ssymm(b3, oracle_mod, mode, route, side, uplo, m, n):
+@pytest.mark.parametrize("gm_map", [-1, 0])
+def test_ssymm(b3, oracle_mod, mode, route, side, uplo, m, n, gm_map):
+    """gm_map=-1: the default policy (below order 4096: sym(A) materialised,
+    then the GEMM); gm_map=0: mirrored while staging, the route from 4096."""
     ka = m if side == "L" else n
     A = gen.symmetric_stored(ka, uplo, "ps", side)        # other triangle = NaN sentinel
     B, C = gen.uniform(m, n, "ps-b"), gen.uniform(m, n, "ps-c")
     dC = to_dev(C)
-    b3.ssymm(side, uplo, AL, to_dev(A), to_dev(B), BE, dC)
+    with b3.options(gm_map=gm_map):
+        b3.ssymm(side, uplo, AL, to_dev(A), to_dev(B), BE, dC)
     got = to_host(dC)
     route(ka, m)
     ref = oracle_mod.ssymm(side, uplo, AL, A, B, BE, C)
@@ -198,13 +202,15 @@ def test_ssymm(b3, oracle_mod, mode, route, side, uplo, m, n):
 
 
 @pytest.mark.parametrize("side,uplo", list(itertools.product("LR", "LU")))
-def test_ssymm_integer_bitexact_and_equals_gemm(b3, oracle_mod, mode, side, uplo):
+@pytest.mark.parametrize("gm_map", [-1, 0])
+def test_ssymm_integer_bitexact_and_equals_gemm(b3, oracle_mod, mode, side, uplo, gm_map):
     m, n = 300, 172
     ka = m if side == "L" else n
     A = gen.symmetric_stored(ka, uplo, "is", integer=True)
     B, C = gen.integers(m, n, "is-b"), gen.integers(m, n, "is-c")
     dC = to_dev(C)
-    b3.ssymm(side, uplo, AL, to_dev(A), to_dev(B), BE, dC)
+    with b3.options(gm_map=gm_map):
+        b3.ssymm(side, uplo, AL, to_dev(A), to_dev(B), BE, dC)
     got = to_host(dC)
     assert bits_equal(got, oracle_mod.ssymm(side, uplo, AL, A, B, BE, C).astype(np.float32))
     # SYMM == GEMM on the explicitly symmetrised A (north-star identity)
