@@ -316,62 +316,113 @@ __global__ void __launch_bounds__(64) dtri_inv64(const __grid_constant__ DOpnd S
 // One launch replaces the 64-row recursion's small launches at the bottom of
 // the DTRSM sweep.
 constexpr int DPR = 512, DRC = 32, DPT = 256;
-constexpr size_t DPANEL_SMEM = (size_t)(DPR * DRC + DNB * (DNB + 1)) * sizeof(double);   // 164 KB
+constexpr int DSL = DNB + 1;                          // shared 64-block leading dimension
+constexpr size_t DPANEL_SMEM = (size_t)(DPR * DRC + 2 * DNB * DSL) * sizeof(double);   // 193 KB
+constexpr int DPE = DNB * DNB / DPT;                  // block elements per thread (16)
+
+// The work list of one panel, in order: for every processing step st, the
+// coupling blocks (bi, bj) of the st blocks solved before it, then the
+// inverse of block bi (bj = -1): st + 1 items, st(st+1)/2 items before it.
+__device__ __forceinline__ void panel_item(int it, int nb, bool lower, int &bi, int &bj) {
+  int st = 0;
+  while ((st + 1) * (st + 2) / 2 <= it) ++st;
+  const int tt = it - st * (st + 1) / 2;              // 0..st; tt == st: the inverse
+  bi = lower ? st : nb - 1 - st;
+  bj = tt == st ? -1 : (lower ? tt : nb - 1 - tt);
+}
+
 __global__ void __launch_bounds__(DPT, 1) dtrsm_panel(const __grid_constant__ DOpnd S, const double *Dp, int R,
                                                       double *X, int64_t sx, int64_t sc, int64_t nrhs) {
   extern __shared__ double dps[];
   double *Y = dps;                                    // Y[i * DRC + c]
-  double *Ss = dps + DPR * DRC;                       // one 64-block, ld DNB + 1
+  double *Sb = dps + DPR * DRC;                       // two 64-blocks, ld DSL
   const int64_t c0 = (int64_t)blockIdx.x * DRC;
   const int ncol = (int)(nrhs - c0 < DRC ? nrhs - c0 : DRC);
   const int nb = (R + DNB - 1) / DNB;
   const bool lower = S.lower != (S.trans != 0);
-  // load the panel's rows of this CTA's right-hand sides (i fastest when the
-  // rows are contiguous, sx == 1)
+  // the panel's rows of this CTA's right-hand sides (i fastest when the rows
+  // are contiguous, sx == 1)
   for (int e = threadIdx.x; e < nb * DNB * DRC; e += DPT) {
     const int i = sx == 1 ? e % (nb * DNB) : e / DRC, c = sx == 1 ? e / (nb * DNB) : e % DRC;
     Y[i * DRC + c] = (i < R && c < ncol) ? X[i * sx + (c0 + c) * sc] : 0.0;
   }
-  // this thread's outputs: rows r = tid % 64, columns cq = tid / 64 + 4 q (q < 8)
-  const int r = threadIdx.x % DNB, cb = threadIdx.x / DNB;
-  for (int st = 0; st < nb; ++st) {
-    const int bi = lower ? st : nb - 1 - st;
-    double acc[DRC / 4];
+  // A coupling block (bi, bj) lies strictly inside the triangle (bj is solved
+  // before bi), so it is read as stored: S(r, k) = L(i, j) = p[i + j ld] with
+  // (i, j) = trans ? (k + ko, r + ro) : (r + ro, k + ko), without the TRI
+  // select; the element order follows the contiguous direction.
+  const bool tr = S.trans != 0;
+  auto fetch_block = [&](int bi, int bj, double (&v)[DPE]) {
+    if (bj < 0) {                                     // inv(S_ii): contiguous 64 x 64
+      const double *d = Dp + (size_t)bi * DNB * DNB;
 #pragma unroll
-    for (int q = 0; q < DRC / 4; ++q) acc[q] = 0.0;
-    for (int tt = 0; tt < st; ++tt) {                 // the blocks solved before bi
-      const int bj = lower ? tt : nb - 1 - tt;
-      __syncthreads();
-      for (int e = threadIdx.x; e < DNB * DNB; e += DPT) {
-        const int i = e % DNB, j = e / DNB;
-        const int64_t gi = (int64_t)bi * DNB + i, gj = (int64_t)bj * DNB + j;
-        Ss[i + j * (DNB + 1)] = (gi < R && gj < R) ? dfetch(S, gi, gj) : 0.0;
-      }
-      __syncthreads();
+      for (int q = 0; q < DPE; ++q) v[q] = __ldg(d + threadIdx.x + DPT * q);
+      return;
+    }
+#pragma unroll
+    for (int q = 0; q < DPE; ++q) {
+      const int e = threadIdx.x + DPT * q;
+      const int rr = tr ? e / DNB : e % DNB, kk = tr ? e % DNB : e / DNB;
+      const int64_t gi = (int64_t)bi * DNB + rr, gj = (int64_t)bj * DNB + kk;
+      const int64_t li = tr ? gj + S.ko : gi + S.ro, lj = tr ? gi + S.ro : gj + S.ko;
+      v[q] = (gi < R && gj < R) ? __ldg(S.p + li + lj * S.ld) : 0.0;
+    }
+  };
+  auto store_block = [&](int bj, const double (&v)[DPE], double *dst) {
+#pragma unroll
+    for (int q = 0; q < DPE; ++q) {
+      const int e = threadIdx.x + DPT * q;
+      const int rr = (bj >= 0 && tr) ? e / DNB : e % DNB, kk = (bj >= 0 && tr) ? e % DNB : e / DNB;
+      dst[rr + kk * DSL] = v[q];
+    }
+  };
+  // this thread's outputs: row r = tid % 64 of the block, columns cb + 4 q
+  // (a warp reads 32 consecutive S rows -- conflict-free -- and broadcast Y;
+  // a 4 x 2 register block with 16-B loads measured slower: 245 vs 183 us)
+  const int r = threadIdx.x % DNB, cb = threadIdx.x / DNB;
+  const int nitems = nb * (nb + 1) / 2;
+  double pre[DPE];
+  int bi, bj;
+  panel_item(0, nb, lower, bi, bj);
+  fetch_block(bi, bj, pre);
+  double acc[DRC / 4];
+#pragma unroll
+  for (int q = 0; q < DRC / 4; ++q) acc[q] = 0.0;
+  for (int it = 0; it < nitems; ++it) {
+    const int cur = it & 1;
+    double *Ss = Sb + cur * DNB * DSL;
+    store_block(bj, pre, Ss);                         // (its buffer was last read two items ago)
+    const int ci = bi, cj = bj;
+    if (it + 1 < nitems) {                            // the next block into registers
+      panel_item(it + 1, nb, lower, bi, bj);
+      fetch_block(bi, bj, pre);
+    }
+    __syncthreads();
+    if (cj >= 0) {                                    // acc += S(ci, cj) y_cj
 #pragma unroll 8
       for (int k = 0; k < DNB; ++k) {
-        const double sv = Ss[r + k * (DNB + 1)];
+        const double sv = Ss[r + k * DSL];
 #pragma unroll
-        for (int q = 0; q < DRC / 4; ++q) acc[q] = fma(sv, Y[(bj * DNB + k) * DRC + cb + 4 * q], acc[q]);
+        for (int q = 0; q < DRC / 4; ++q) acc[q] = fma(sv, Y[(cj * DNB + k) * DRC + cb + 4 * q], acc[q]);
+      }
+    } else {                                          // y_ci <- inv(S_ii) (y_ci - acc)
+#pragma unroll
+      for (int q = 0; q < DRC / 4; ++q) Y[(ci * DNB + r) * DRC + cb + 4 * q] -= acc[q];
+      __syncthreads();
+#pragma unroll
+      for (int q = 0; q < DRC / 4; ++q) acc[q] = 0.0;
+#pragma unroll 8
+      for (int k = 0; k < DNB; ++k) {
+        const double sv = Ss[r + k * DSL];
+#pragma unroll
+        for (int q = 0; q < DRC / 4; ++q) acc[q] = fma(sv, Y[(ci * DNB + k) * DRC + cb + 4 * q], acc[q]);
+      }
+      __syncthreads();
+#pragma unroll
+      for (int q = 0; q < DRC / 4; ++q) {
+        Y[(ci * DNB + r) * DRC + cb + 4 * q] = acc[q];
+        acc[q] = 0.0;
       }
     }
-    __syncthreads();
-#pragma unroll
-    for (int q = 0; q < DRC / 4; ++q) Y[(bi * DNB + r) * DRC + cb + 4 * q] -= acc[q];
-    for (int e = threadIdx.x; e < DNB * DNB; e += DPT)          // inv(S_ii)
-      Ss[e % DNB + (e / DNB) * (DNB + 1)] = Dp[(size_t)bi * DNB * DNB + e];
-    __syncthreads();
-#pragma unroll
-    for (int q = 0; q < DRC / 4; ++q) acc[q] = 0.0;
-#pragma unroll 8
-    for (int k = 0; k < DNB; ++k) {
-      const double sv = Ss[r + k * (DNB + 1)];
-#pragma unroll
-      for (int q = 0; q < DRC / 4; ++q) acc[q] = fma(sv, Y[(bi * DNB + k) * DRC + cb + 4 * q], acc[q]);
-    }
-    __syncthreads();
-#pragma unroll
-    for (int q = 0; q < DRC / 4; ++q) Y[(bi * DNB + r) * DRC + cb + 4 * q] = acc[q];
   }
   __syncthreads();
   for (int e = threadIdx.x; e < nb * DNB * DRC; e += DPT) {
