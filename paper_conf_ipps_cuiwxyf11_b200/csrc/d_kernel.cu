@@ -32,7 +32,15 @@ namespace blas3 {
 namespace {
 
 constexpr int DTM = 128, DTN = 128, DBK = 16, DTHREADS = 256;
-constexpr int DAP = DTM + 8, DBP = DTN + 8;          // padded shared rows: 1088 B = 64 B mod 128 (DMMA fragment loads conflict-free)
+// shared-row padding: 132 doubles = 32 B mod 128 keeps the DMMA fragment
+// loads (4 k-rows x 64 B) at 2 wavefronts and the k-fastest staging stores at
+// 4-way; measured against 2 and 8 (tools/lib_ab_fp64.py: DGEMM TN 24.0 vs
+// 23.4 / 21.5 TF/s, DSYMM 21.7 vs 21.3 / 20.2)
+#ifndef BLAS3_DPAD
+#define BLAS3_DPAD 4
+#endif
+constexpr int DPAD = BLAS3_DPAD;
+constexpr int DAP = DTM + DPAD, DBP = DTN + DPAD;
 constexpr int DJ = 8;                                // columns per thread (two groups of 4)
 constexpr int DNB = 64;                              // TRSM diagonal block
 
