@@ -16,10 +16,10 @@
 // default instantiation issues DMMA from register fragments; DFMA stays as
 // the BLAS3_D_MMA=0 alternative.  Products and sums are fp64 either way.
 //
-// Kernel: 256 threads, C tile 128 x 128, BK = 16 k-blocks staged through
-// registers into double-buffered shared memory (the structure select happens
-// on the way); DMMA: each warp a 64 x 32 block of 8 x 4 fragments; DFMA: 8 x 8
-// outputs per thread (rows tr + 16 i, columns 4 tc + 64 g + j).
+// Kernel: C tile 128 x 128, BK = 16 k-blocks staged through registers into
+// double-buffered shared memory (the structure select happens on the way);
+// DMMA: 512 threads, each warp a 32 x 32 block of 4 x 4 fragments; DFMA: 256
+// threads, 8 x 8 outputs per thread (rows tr + 16 i, columns 4 tc + 64 g + j).
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <atomic>
@@ -31,7 +31,7 @@
 namespace blas3 {
 namespace {
 
-constexpr int DTM = 128, DTN = 128, DBK = 16, DTHREADS = 256;
+constexpr int DTM = 128, DTN = 128, DBK = 16;
 // shared-row padding: 132 doubles = 32 B mod 128 keeps the DMMA fragment
 // loads (4 k-rows x 64 B) at 2 wavefronts and the k-fastest staging stores at
 // 4-way; measured against 2 and 8 (tools/lib_ab_fp64.py: DGEMM TN 24.0 vs
@@ -88,16 +88,16 @@ __device__ __forceinline__ void krange(const DOpnd &o, int64_t r0, int64_t r1, i
 
 // One operand tile (ROWS x DBK) of X into registers: element e = tid + 256 q,
 // (r, k) = r-fastest or k-fastest by the block's contiguous direction.
-template <int ROWS>
+template <int ROWS, int NT>
 struct TileLoad {
-  static constexpr int PER = ROWS * DBK / DTHREADS;
+  static constexpr int PER = ROWS * DBK / NT;
   double v[PER];
   // strided block X(r, k) = base[r * si + k * sk]
   __device__ __forceinline__ void load_strided(const double *base, int64_t si, int64_t sk, int64_t r0, int64_t rmax,
                                                int64_t k0, int64_t kmax, bool rf) {
 #pragma unroll
     for (int q = 0; q < PER; ++q) {
-      const int e = threadIdx.x + DTHREADS * q;
+      const int e = threadIdx.x + NT * q;
       const int r = rf ? e % ROWS : e / DBK, k = rf ? e / ROWS : e % DBK;
       v[q] = (r0 + r < rmax && k0 + k < kmax) ? __ldg(base + r * si + k * sk) : 0.0;
     }
@@ -134,7 +134,7 @@ struct TileLoad {
     }
 #pragma unroll
     for (int q = 0; q < PER; ++q) {
-      const int e = threadIdx.x + DTHREADS * q;
+      const int e = threadIdx.x + NT * q;
       const int r = rf ? e % ROWS : e / DBK, k = rf ? e / ROWS : e % DBK;
       v[q] = (r0 + r < rmax && k0 + k < kmax) ? dfetch(o, r0 + r, k0 + k) : 0.0;
     }
@@ -143,7 +143,7 @@ struct TileLoad {
   __device__ __forceinline__ void store(double *s, bool rf) const {
 #pragma unroll
     for (int q = 0; q < PER; ++q) {
-      const int e = threadIdx.x + DTHREADS * q;
+      const int e = threadIdx.x + NT * q;
       const int r = rf ? e % ROWS : e / DBK, k = rf ? e / ROWS : e % DBK;
       s[k * LD + r] = v[q];
     }
@@ -161,8 +161,12 @@ __device__ __forceinline__ void dmma(double &d0, double &d1, double a, double b)
 // MMA = false: DFMA, 8 x 8 outputs per thread.  MMA = true: DMMA m8n8k4 on
 // register fragments, each warp a 64 x 32 block (8 x 4 fragments), the same
 // staging and epilogue semantics.
+// threads per CTA: DMMA 512 (16 warps, each a 32 x 32 block of 4 x 4
+// fragments: <= 128 registers), DFMA 256 (8 x 8 outputs per thread)
+template <bool MMA> __host__ __device__ constexpr int dthreads() { return MMA ? 512 : 256; }
 template <bool MMA>
-__global__ void __launch_bounds__(DTHREADS, 1) dgemm_structured(const __grid_constant__ DProblem P) {
+__global__ void __launch_bounds__(dthreads<MMA>(), 1) dgemm_structured(const __grid_constant__ DProblem P) {
+  constexpr int NT = dthreads<MMA>();
   extern __shared__ double dsm[];
   // buffers by integer offset from the __shared__ array (not through a
   // pointer table, which would turn every access into a generic LD/ST)
@@ -188,8 +192,8 @@ __global__ void __launch_bounds__(DTHREADS, 1) dgemm_structured(const __grid_con
     if (klo >= khi) continue;
     klo = klo / DBK * DBK;                            // k-blocks aligned to BK
     const int64_t nkb = (khi - klo + DBK - 1) / DBK;
-    TileLoad<DTM> la;
-    TileLoad<DTN> lb;
+    TileLoad<DTM, NT> la;
+    TileLoad<DTN, NT> lb;
     bool rfa = rfast(S.a, m0, m0 + DTM, klo, klo + DBK), rfb = rfast(S.b, n0, n0 + DTN, klo, klo + DBK);
     la.load(S.a, m0, P.M, klo, khi, rfa);
     lb.load(S.b, n0, P.N, klo, khi, rfb);
@@ -209,16 +213,16 @@ __global__ void __launch_bounds__(DTHREADS, 1) dgemm_structured(const __grid_con
       const double *as = dsm + cur * AOFF, *bs = dsm + BOFF0 + cur * BOFF;
       if constexpr (MMA) {
         const int lane = threadIdx.x % 32, wid = threadIdx.x / 32;
-        const int am = 64 * (wid % 2) + lane / 4, bn = 32 * (wid / 2) + lane / 4, kq = lane % 4;
+        const int am = 32 * (wid % 4) + lane / 4, bn = 32 * (wid / 4) + lane / 4, kq = lane % 4;
 #pragma unroll
         for (int kk = 0; kk < DBK / 4; ++kk) {
-          double a[8], b[4];
+          double a[4], b[4];
 #pragma unroll
-          for (int i = 0; i < 8; ++i) a[i] = as[(kk * 4 + kq) * DAP + am + 8 * i];
+          for (int i = 0; i < 4; ++i) a[i] = as[(kk * 4 + kq) * DAP + am + 8 * i];
 #pragma unroll
           for (int j = 0; j < 4; ++j) b[j] = bs[(kk * 4 + kq) * DBP + bn + 8 * j];
 #pragma unroll
-          for (int i = 0; i < 8; ++i)
+          for (int i = 0; i < 4; ++i)
 #pragma unroll
             for (int j = 0; j < 4; ++j) dmma(acc[i][2 * j], acc[i][2 * j + 1], a[i], b[j]);
         }
@@ -250,14 +254,14 @@ __global__ void __launch_bounds__(DTHREADS, 1) dgemm_structured(const __grid_con
   // epilogue: D = alpha * acc + beta * C (C not read when beta == 0), uplo mask
 #pragma unroll
   for (int j = 0; j < DJ; ++j) {
-    // DMMA: acc[i][2 jf + e] is C row 64 (w % 2) + 8 i + lane / 4, column
-    // 32 (w / 2) + 8 jf + 2 (lane % 4) + e
-    const int64_t c = MMA ? n0 + 32 * ((threadIdx.x / 32) / 2) + 8 * (j / 2) + 2 * ((threadIdx.x % 32) % 4) + j % 2
+    // DMMA: acc[i][2 jf + e] is C row 32 (w % 4) + 8 i + lane / 4, column
+    // 32 (w / 4) + 8 jf + 2 (lane % 4) + e  (i < 4)
+    const int64_t c = MMA ? n0 + 32 * ((threadIdx.x / 32) / 4) + 8 * (j / 2) + 2 * ((threadIdx.x % 32) % 4) + j % 2
                           : n0 + 4 * tc + 64 * (j / 4) + j % 4;
     if (c >= P.N) continue;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) {
-      const int64_t r = MMA ? m0 + 64 * ((threadIdx.x / 32) % 2) + 8 * i + (threadIdx.x % 32) / 4 : m0 + tr + 16 * i;
+    for (int i = 0; i < (MMA ? 4 : 8); ++i) {
+      const int64_t r = MMA ? m0 + 32 * ((threadIdx.x / 32) % 4) + 8 * i + (threadIdx.x % 32) / 4 : m0 + tr + 16 * i;
       if (r >= P.M) continue;
       if (P.ctri == 1 && r < c) continue;
       if (P.ctri == 2 && r > c) continue;
@@ -467,7 +471,7 @@ int launch_dgemm(const DProblem &P, cudaStream_t s) {
       return -1;
     attr[dev][use_mma].store(true, std::memory_order_release);
   }
-  kfn<<<(unsigned)tiles, DTHREADS, DSMEM, s>>>(P);
+  kfn<<<(unsigned)tiles, use_mma ? dthreads<true>() : dthreads<false>(), DSMEM, s>>>(P);
   note_launch(1);
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
