@@ -269,3 +269,57 @@ def test_padded_ld_untouched(b3, oracle_mod, routine):
     host = full.cpu().numpy()
     assert np.isnan(host[:n, m:]).all(), "padding rows written"
     assert np.isnan(host[n:]).all(), "columns beyond n written"
+
+
+@pytest.mark.parametrize("routine", ["dsymm", "dsyrk", "dsyr2k", "dtrmm", "dtrsm_R"])
+def test_large_structured_sampled(b3, oracle_mod, routine):
+    """N = 4096 (32 x 32 tiles of 128, the fp64 bench size) on sampled oracle
+    columns (rows for side = R): the structured routines at scale, where every
+    region class (real / shadow / blank / diagonal-crossing) occurs many times."""
+    import torch
+    n = 4096
+    sel = gen.sample_indices(n, 12, "dL-s", routine)
+    B = gen.uniform(n, n, "dL-b")
+    C = gen.uniform(n, n, "dL-c")
+    if routine == "dsymm":
+        S = gen.symmetric_stored(n, "U", "dL-a")
+        dC = dev(b3, C)
+        b3.dsymm("L", "U", AL, dev(b3, S), dev(b3, B), BE, dC)
+        torch.cuda.synchronize()
+        got = to_host(dC)[:, sel]
+        ref = oracle_mod.ssymm("L", "U", AL, S, B, BE, C, sel=sel)
+        scale = AL * fro(sym_full(S, "U", n)) * fro(B[:, sel]) + BE * fro(C[:, sel])
+        assert enw(got, ref, scale) <= tol(n)
+    elif routine in ("dsyrk", "dsyr2k"):
+        k = 512
+        A = gen.uniform(n, k, "dL-ka"); A2 = gen.uniform(n, k, "dL-kb")
+        Cl = gen.nan_outside(C, "L")
+        dC = dev(b3, Cl)
+        if routine == "dsyrk":
+            b3.dsyrk("L", "N", AL, dev(b3, A), BE, dC)
+            ref = oracle_mod.ssyrk("L", "N", AL, A, BE, Cl, sel=sel)
+        else:
+            b3.dsyr2k("L", "N", AL, dev(b3, A), dev(b3, A2), BE, dC)
+            ref = oracle_mod.ssyr2k("L", "N", AL, A, A2, BE, Cl, sel=sel)
+        torch.cuda.synchronize()
+        got = to_host(dC)[:, sel]
+        low = np.array([[i >= j for j in sel] for i in range(n)])
+        assert np.isnan(got[~low]).all()
+        d = np.where(low, np.nan_to_num(f64(got)) - np.nan_to_num(f64(ref)), 0.0)
+        assert fro(d) / fro(np.where(low, np.nan_to_num(f64(ref)), 0.0)) <= tol(2 * k) * 10
+    elif routine == "dtrmm":
+        T = gen.nan_outside(gen.uniform(n, n, "dL-t"), "L", keep_diag=False)
+        dB = dev(b3, B)
+        b3.dtrmm("L", "L", "T", "U", AL, dev(b3, T), dB)
+        torch.cuda.synchronize()
+        got = to_host(dB)[:, sel]
+        ref = oracle_mod.strmm("L", "L", "T", "U", AL, T, B, sel=sel)
+        assert enw(got, ref, AL * fro(tri_full(T, "L", "U", n)) * fro(B[:, sel])) <= tol(n)
+    else:                                            # DTRSM side = R, sampled rows
+        T = gen.triangular_dd(n, "U", "N", "dL-tr")
+        dB = dev(b3, B)
+        b3.dtrsm("R", "U", "T", "N", AL, dev(b3, T), dB)
+        torch.cuda.synchronize()
+        X = f64(to_host(dB))[sel, :]
+        ref = oracle_mod.strsm("R", "U", "T", "N", AL, T, B, sel=sel)
+        assert fro(X - ref) / fro(ref) <= 64 * n * U53
